@@ -1,0 +1,181 @@
+/*
+ * cusfft.h — C ABI of the B200-native sparse FFT engine (sFFT hot path as
+ * parallelised by cusFFT, Wang/Chandrasekaran/Chapman, IPDPS'16).
+ *
+ * Citations are to the paper text, /root/reference/PAPER.md, as L<line>.
+ * The paper has no API; the shapes follow its problem statement (L13, L77:
+ * x in C^n, k large Fourier coefficients) and its algorithms:
+ *
+ *   Step 1  random spectral permutation         Def. 1 (L81), Alg. 1
+ *   Step 2  flat-window filter + fold into B    L85, Alg. 1, Fig. 3, Alg. 2
+ *   Step 3  batched B-point FFT                  L87, L232
+ *   Step 4  cutoff (top-num buckets)             L89, Alg. 3
+ *   Step 5  reverse hash + vote                  L91-L93, Alg. 4
+ *   Step 6  median estimation                    L95, Alg. 5
+ *
+ * Conventions:
+ *   - Signals are interleaved complex fp64 ("complex double", L196): element t
+ *     is {re, im} at byte offset 16 t.  Device pointers must be 16-B aligned and
+ *     live on the plan's device.
+ *   - Forward DFT x^_f = sum_t x_t e^{-2 pi i f t/n}.  The engine returns
+ *     x^_f / n, so a planted x_t = sum_f X_f e^{+2 pi i f t/n} is returned as X.
+ *   - Every call is stream-ordered on the plan's stream (cusfft_set_stream) and
+ *     asynchronous unless stated; no call except cusfft_status /
+ *     cusfft_get_debug / cusfft_execute_host synchronises the host.
+ *   - A plan is not thread-safe; distinct plans are independent.
+ *   - Errors: every function returns 0 (CUSFFT_SUCCESS) or a negative
+ *     cusfft_status_t.  On error nothing is launched and outputs are untouched.
+ *     There is no CPU fallback: without a CUDA device cusfft_plan fails with
+ *     CUSFFT_CUDA.
+ */
+#ifndef CUSFFT_H_
+#define CUSFFT_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define CUSFFT_ABI_VERSION 1
+
+typedef struct cusfft_plan_s* cusfft_plan_t; /* opaque; owns all device workspace */
+
+typedef enum {
+  CUSFFT_SUCCESS = 0,
+  CUSFFT_INVALID_N = -1,      /* n not a power of two, n < 16 or n > 2^31            */
+  CUSFFT_INVALID_B = -2,      /* B not a power of two, B < 2, or B >= n               */
+  CUSFFT_INVALID_K = -3,      /* k < 1, k > 8192, num_select < k or num_select > B    */
+  CUSFFT_INVALID_LOOPS = -4,  /* L < 1, L > 64, T > L_loc, L_loc > L, or world !| L   */
+  CUSFFT_INVALID_PARAM = -5,  /* filter/tolerance/lobefrac/box/taps out of range      */
+  CUSFFT_NULL_PTR = -6,       /* a required pointer argument is NULL                  */
+  CUSFFT_ALLOC = -7,          /* device allocation failed                             */
+  CUSFFT_CUDA = -8,           /* a CUDA runtime call failed (cusfft_last_cuda_error)  */
+  CUSFFT_HIT_OVERFLOW = -9,   /* more than max_hits frequencies reached T votes       */
+  CUSFFT_INVALID_PLAN = -10,  /* NULL or destroyed plan                               */
+  CUSFFT_INTERNAL = -11       /* a device-side consistency check failed               */
+} cusfft_status_t;
+
+typedef enum {
+  CUSFFT_FILTER_DOLPH_CHEBYSHEV = 0, /* L25, L85 */
+  CUSFFT_FILTER_GAUSSIAN = 1         /* L25, L85 */
+} cusfft_filter_t;
+
+/* Plan parameters.  Fill with cusfft_params_default, then override. */
+typedef struct {
+  int32_t filter;          /* cusfft_filter_t; default DOLPH_CHEBYSHEV (L85)                     */
+  double tolerance;        /* delta: filter side-lobe / leakage level; default 1e-8              */
+  double lobefrac;         /* lambda: main-lobe half width in cycles/sample; default 0.5/B       */
+  int64_t box_width;       /* b: width of the frequency box, odd, default n/B - 1                */
+  int32_t loc_loops;       /* L_loc <= L: loops that vote (L93); default min(L, 8)                */
+  int32_t vote_threshold;  /* T: hit iff votes >= T; default floor(L_loc/2)+1 ("s_i > L/2", L93)  */
+  int32_t num_select;      /* buckets kept per location loop (L89); default k                     */
+  int32_t tau_mode;        /* 1: random tau (Def. 1); 0: tau = 0 (Alg. 2 L216 literal)       */
+  uint64_t seed;           /* drives (a_r, sigma_r, tau_r) through SplitMix64      */
+  int64_t max_hits;        /* hit-buffer capacity; default from the expected false-hit count      */
+  int32_t device;          /* CUDA device ordinal; default: the current device                   */
+  int32_t debug;           /* 1: keep per-loop estimates for cusfft_get_debug; default 0          */
+  const double* taps;      /* optional HOST array of num_taps real taps g_i (Alg. 1 filter[]);
+                              NULL: build the filter from filter/tolerance/lobefrac/box_width.
+                              Copied at plan time; the caller keeps ownership.                    */
+  int64_t num_taps;        /* length of taps when taps != NULL (odd not required)                */
+} cusfft_params;
+
+/* Fill *p with the defaults for (n, k, B).  Returns CUSFFT_NULL_PTR / INVALID_*. */
+int cusfft_params_default(cusfft_params* p, int64_t n, int64_t k, int64_t B);
+
+/* B = floor_pow2(bcst * sqrt(n k / log2 n)) (L85, L196, L228); 0 on bad input. */
+int64_t cusfft_default_B(int64_t n, int64_t k, double bcst);
+
+/* Create a plan for length-n signals, k outputs, B buckets and L loops.
+ * p may be NULL (defaults).  Draws (a_r, sigma_r, tau_r), builds the filter
+ * taps, the filter response G^(q) for |q| <= n/(2B) and the B-point twiddles
+ * on the device, allocates all workspace.  Synchronous.  *out is written only
+ * on success. */
+int cusfft_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L,
+                const cusfft_params* p);
+
+/* Loop-sharded plan for rank `rank` of `world` processes (one GPU each).
+ * world must divide L.  Loop r is owned by rank r mod world.  Outputs are
+ * identical on every rank and identical to a world = 1 plan with the same
+ * parameters.  The exchange between cusfft_execute_local and
+ * cusfft_execute_finish is an all-gather of the buffer returned by
+ * cusfft_exchange_buffer, done by the caller (e.g. torch.distributed / NCCL). */
+int cusfft_plan_dist(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L,
+                     const cusfft_params* p, int32_t rank, int32_t world);
+
+/* Release every device allocation of the plan.  Synchronises the plan's stream.
+ * Destroying NULL returns CUSFFT_INVALID_PLAN. */
+int cusfft_destroy(cusfft_plan_t plan);
+
+/* Set the CUDA stream (a cudaStream_t; NULL = legacy default stream). */
+int cusfft_set_stream(cusfft_plan_t plan, void* cuda_stream);
+
+/* The whole transform on one GPU (world = 1 plans only):
+ *   d_x    : device, read-only, complex fp64 [n]
+ *   d_locs : device, int64 [k]      output: recovered frequencies, ascending; -1 pads
+ *   d_vals : device, complex fp64 [k] output: x^_f / n at d_locs; 0 pads
+ * Runs Steps 1-6 (fold, B-point FFT, cutoff, vote, estimate, output).
+ * Asynchronous; hit-buffer overflow is reported by cusfft_status. */
+int cusfft_execute(cusfft_plan_t plan, const void* d_x, int64_t* d_locs, void* d_vals);
+
+/* Same transform from HOST buffers: copies h_x [n] to a plan-owned device
+ * buffer, executes, copies k locations / values back and synchronises the
+ * stream.  Pinned host memory gives asynchronous copies.  Returns the
+ * cusfft_status result of the transform. */
+int cusfft_execute_host(cusfft_plan_t plan, const void* h_x, int64_t* h_locs, void* h_vals);
+
+/* Loop-sharded execution (any world): Steps 1-4 for this rank's loops, written
+ * into this rank's slice of the exchange buffer. */
+int cusfft_execute_local(cusfft_plan_t plan, const void* d_x);
+/* Steps 5-6 plus output selection, after the exchange buffer holds every
+ * rank's slice.  Outputs as in cusfft_execute. */
+int cusfft_execute_finish(cusfft_plan_t plan, int64_t* d_locs, void* d_vals);
+/* The exchange buffer: *d_buf points at world * (*bytes_per_rank) bytes of
+ * device memory, rank r's slice at offset r * (*bytes_per_rank). */
+int cusfft_exchange_buffer(cusfft_plan_t plan, void** d_buf, int64_t* bytes_per_rank);
+
+/* Plan facts (host arrays, caller-owned):
+ *   info[0..9] = n, k, B, L, w (taps), n/B, num_select, loc_loops, vote_threshold, max_hits
+ *   a, sigma, tau : int64 [L], in loop order r = 0..L-1 (NULL to skip).  sigma is
+ *   the gather stride (Alg. 1's ai), a = sigma^-1 mod n, tau the offset. */
+int cusfft_get_info(cusfft_plan_t plan, int64_t* info, int64_t* a, int64_t* sigma, int64_t* tau);
+
+typedef enum {
+  CUSFFT_DEBUG_U = 0,        /* complex fp64 [L_local][B]: fold output, this rank's loops  */
+  CUSFFT_DEBUG_UHAT = 1,     /* complex fp64 [L][B]: B-point FFTs, loop order                */
+  CUSFFT_DEBUG_WINNERS = 2,  /* int32 [L_loc][num_select]: kept buckets, ascending            */
+  CUSFFT_DEBUG_HITS = 3,     /* int32 [H]: frequencies with >= T votes (unordered)           */
+  CUSFFT_DEBUG_HIT_VALS = 4, /* complex fp64 [H]: median estimates aligned with HITS          */
+  CUSFFT_DEBUG_PER_LOOP = 5, /* complex fp64 [H][L]: per-loop estimates (params.debug = 1)    */
+  CUSFFT_DEBUG_TAPS = 6,     /* fp64 [w]: filter taps g_i                                    */
+  CUSFFT_DEBUG_GHAT = 7,     /* complex fp64 [n/B + 1]: G^(q), q = -n/(2B) .. n/(2B)          */
+  CUSFFT_DEBUG_NUM_HITS = 8  /* int64 [1]: H (may exceed max_hits on overflow)               */
+} cusfft_debug_t;
+
+/* Copy a debug artefact of the last execution to host memory.  cap is the
+ * destination size in bytes; returns the number of bytes the artefact needs
+ * (>= 0; nothing copied if cap is smaller) or a negative status.  Synchronises. */
+int64_t cusfft_get_debug(cusfft_plan_t plan, int32_t what, void* host_dst, int64_t cap);
+
+/* Synchronise the plan's stream and report device-side status of the last
+ * execution: CUSFFT_SUCCESS, CUSFFT_HIT_OVERFLOW or CUSFFT_INTERNAL. */
+int cusfft_status(cusfft_plan_t plan);
+
+/* Per-stage device times (ms) of the last execution when timing is enabled:
+ * ms[0..5] = fold, B-point FFT, cutoff, vote, estimate, output.  Enabling
+ * records CUDA events between the kernels on the plan's stream.  get syncs. */
+int cusfft_set_timing(cusfft_plan_t plan, int32_t enable);
+int cusfft_get_stage_times(cusfft_plan_t plan, float* ms, int32_t cap);
+
+/* Number of kernel launches one cusfft_execute issues for this plan. */
+int32_t cusfft_launches_per_execute(cusfft_plan_t plan);
+
+const char* cusfft_strerror(int code);
+int32_t cusfft_last_cuda_error(void);
+int32_t cusfft_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CUSFFT_H_ */

@@ -1,0 +1,298 @@
+"""ctypes binding of ``libcusfft.so`` (the C ABI in ``include/cusfft.h``).
+
+Argument marshalling only: every step of the transform runs in the CUDA
+kernels of ``csrc/``.  There is no CPU fallback — if the shared library is
+missing or no CUDA device is present, plan creation raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libcusfft.so")
+
+SUCCESS = 0
+INVALID_N, INVALID_B, INVALID_K, INVALID_LOOPS, INVALID_PARAM = -1, -2, -3, -4, -5
+NULL_PTR, ALLOC, CUDA, HIT_OVERFLOW, INVALID_PLAN, INTERNAL = -6, -7, -8, -9, -10, -11
+
+FILTER_DOLPH_CHEBYSHEV = 0
+FILTER_GAUSSIAN = 1
+
+DEBUG_U, DEBUG_UHAT, DEBUG_WINNERS, DEBUG_HITS, DEBUG_HIT_VALS = 0, 1, 2, 3, 4
+DEBUG_PER_LOOP, DEBUG_TAPS, DEBUG_GHAT, DEBUG_NUM_HITS = 5, 6, 7, 8
+
+# Every symbol include/cusfft.h declares (checked by tests/test_abi.py).
+EXPORTED = (
+    "cusfft_params_default", "cusfft_default_B", "cusfft_plan", "cusfft_plan_dist",
+    "cusfft_destroy", "cusfft_set_stream", "cusfft_execute", "cusfft_execute_host",
+    "cusfft_execute_local", "cusfft_execute_finish", "cusfft_exchange_buffer",
+    "cusfft_get_info", "cusfft_get_debug", "cusfft_status", "cusfft_set_timing",
+    "cusfft_get_stage_times", "cusfft_launches_per_execute", "cusfft_strerror",
+    "cusfft_last_cuda_error", "cusfft_abi_version",
+)
+
+
+class CusfftParams(ctypes.Structure):
+    _fields_ = [
+        ("filter", ctypes.c_int32),
+        ("tolerance", ctypes.c_double),
+        ("lobefrac", ctypes.c_double),
+        ("box_width", ctypes.c_int64),
+        ("loc_loops", ctypes.c_int32),
+        ("vote_threshold", ctypes.c_int32),
+        ("num_select", ctypes.c_int32),
+        ("tau_mode", ctypes.c_int32),
+        ("seed", ctypes.c_uint64),
+        ("max_hits", ctypes.c_int64),
+        ("device", ctypes.c_int32),
+        ("debug", ctypes.c_int32),
+        ("taps", ctypes.POINTER(ctypes.c_double)),
+        ("num_taps", ctypes.c_int64),
+    ]
+
+
+_lib = None
+
+
+def load_library():
+    """Load libcusfft.so (built in-tree by ``__graft_entry__.build()``)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise RuntimeError(
+            f"CUDA extension {LIB_PATH} is missing; build it with "
+            "`python -c 'import __graft_entry__ as g; g.build()'` (no CPU fallback exists)")
+    lib = ctypes.CDLL(LIB_PATH)
+    P = ctypes.c_void_p
+    i64, i32 = ctypes.c_int64, ctypes.c_int32
+    pp = ctypes.POINTER(CusfftParams)
+    sig = {
+        "cusfft_params_default": (ctypes.c_int, [pp, i64, i64, i64]),
+        "cusfft_default_B": (i64, [i64, i64, ctypes.c_double]),
+        "cusfft_plan": (ctypes.c_int, [ctypes.POINTER(P), i64, i64, i64, i32, pp]),
+        "cusfft_plan_dist": (ctypes.c_int, [ctypes.POINTER(P), i64, i64, i64, i32, pp, i32, i32]),
+        "cusfft_destroy": (ctypes.c_int, [P]),
+        "cusfft_set_stream": (ctypes.c_int, [P, P]),
+        "cusfft_execute": (ctypes.c_int, [P, P, P, P]),
+        "cusfft_execute_host": (ctypes.c_int, [P, P, P, P]),
+        "cusfft_execute_local": (ctypes.c_int, [P, P]),
+        "cusfft_execute_finish": (ctypes.c_int, [P, P, P]),
+        "cusfft_exchange_buffer": (ctypes.c_int, [P, ctypes.POINTER(P), ctypes.POINTER(i64)]),
+        "cusfft_get_info": (ctypes.c_int, [P, P, P, P, P]),
+        "cusfft_get_debug": (i64, [P, i32, P, i64]),
+        "cusfft_status": (ctypes.c_int, [P]),
+        "cusfft_set_timing": (ctypes.c_int, [P, i32]),
+        "cusfft_get_stage_times": (ctypes.c_int, [P, P, i32]),
+        "cusfft_launches_per_execute": (i32, [P]),
+        "cusfft_strerror": (ctypes.c_char_p, [ctypes.c_int]),
+        "cusfft_last_cuda_error": (i32, []),
+        "cusfft_abi_version": (i32, []),
+    }
+    for name, (res, args) in sig.items():
+        fn = getattr(lib, name)
+        fn.restype = res
+        fn.argtypes = args
+    _lib = lib
+    return lib
+
+
+class CusfftError(RuntimeError):
+    def __init__(self, code: int, what: str = ""):
+        lib = load_library()
+        msg = lib.cusfft_strerror(code).decode()
+        if code == CUDA:
+            msg += f" (cudaError {lib.cusfft_last_cuda_error()})"
+        super().__init__(f"{what}: {msg} [{code}]" if what else f"{msg} [{code}]")
+        self.code = code
+
+
+def check(code: int, what: str = ""):
+    if code != SUCCESS:
+        raise CusfftError(code, what)
+    return code
+
+
+def default_B(n: int, k: int, bcst: float = 1.0) -> int:
+    return int(load_library().cusfft_default_B(n, k, bcst))
+
+
+def default_params(n: int, k: int, B: int) -> CusfftParams:
+    p = CusfftParams()
+    check(load_library().cusfft_params_default(ctypes.byref(p), n, k, B), "cusfft_params_default")
+    return p
+
+
+def _ptr(t) -> int:
+    """Raw data pointer of a torch tensor or numpy array."""
+    if hasattr(t, "data_ptr"):
+        return t.data_ptr()
+    return t.ctypes.data
+
+
+class Plan:
+    """A cusfft plan: ``Plan(n, k, B=None, L=16, **params)``.
+
+    ``params`` are the fields of ``cusfft_params`` (filter, tolerance,
+    lobefrac, box_width, loc_loops, vote_threshold, num_select, tau_mode,
+    seed, max_hits, device, debug) plus ``taps`` (a float64 array of user
+    taps).  ``rank`` / ``world`` make a loop-sharded plan (cusfft_plan_dist).
+    """
+
+    def __init__(self, n: int, k: int, B: int | None = None, L: int = 16, rank: int = 0,
+                 world: int = 1, **params):
+        self._lib = load_library()
+        self._h = ctypes.c_void_p()
+        if B is None:
+            B = default_B(n, k)
+        self.n, self.k, self.B, self.L = int(n), int(k), int(B), int(L)
+        self.rank, self.world = int(rank), int(world)
+        prm = default_params(self.n, self.k, self.B)
+        taps = params.pop("taps", None)
+        for key, val in params.items():
+            if not hasattr(prm, key):
+                raise TypeError(f"unknown cusfft parameter {key!r}")
+            setattr(prm, key, val)
+        if taps is not None:
+            self._taps = np.ascontiguousarray(taps, dtype=np.float64)
+            prm.taps = self._taps.ctypes.data_as(ctypes.POINTER(ctypes.c_double))
+            prm.num_taps = self._taps.shape[0]
+        self.params = prm
+        if self.world == 1:
+            rc = self._lib.cusfft_plan(ctypes.byref(self._h), self.n, self.k, self.B, self.L, ctypes.byref(prm))
+        else:
+            rc = self._lib.cusfft_plan_dist(ctypes.byref(self._h), self.n, self.k, self.B, self.L,
+                                            ctypes.byref(prm), self.rank, self.world)
+        check(rc, "cusfft_plan")
+        info = self.info()
+        self.w, self.nb, self.num, self.loc_loops, self.T, self.max_hits = (
+            int(info["w"]), int(info["nb"]), int(info["num"]), int(info["loc_loops"]),
+            int(info["T"]), int(info["max_hits"]))
+
+    # -- lifetime
+    def close(self):
+        if getattr(self, "_h", None) is not None and self._h.value:
+            self._lib.cusfft_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+    # -- execution
+    def set_stream(self, stream_handle: int):
+        check(self._lib.cusfft_set_stream(self._h, ctypes.c_void_p(stream_handle)), "cusfft_set_stream")
+
+    def _use_current_stream(self):
+        import torch
+        self.set_stream(torch.cuda.current_stream().cuda_stream)
+
+    def execute(self, x, locs=None, vals=None):
+        """x: complex128 CUDA tensor [n].  Returns (locs int64[k], vals complex128[k])."""
+        import torch
+        if x.dtype != torch.complex128 or not x.is_cuda or x.numel() != self.n or not x.is_contiguous():
+            raise ValueError("x must be a contiguous complex128 CUDA tensor of length n")
+        if locs is None:
+            locs = torch.empty(self.k, dtype=torch.int64, device=x.device)
+        if vals is None:
+            vals = torch.empty(self.k, dtype=torch.complex128, device=x.device)
+        self._use_current_stream()
+        check(self._lib.cusfft_execute(self._h, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(locs.data_ptr()),
+                                       ctypes.c_void_p(vals.data_ptr())), "cusfft_execute")
+        return locs, vals
+
+    def execute_raw(self, x_ptr: int, locs_ptr: int, vals_ptr: int):
+        """Enqueue on the plan's current stream with raw device pointers."""
+        return check(self._lib.cusfft_execute(self._h, ctypes.c_void_p(x_ptr), ctypes.c_void_p(locs_ptr),
+                                              ctypes.c_void_p(vals_ptr)), "cusfft_execute")
+
+    def execute_host(self, x, locs=None, vals=None):
+        """x: host complex128 [n] (numpy or pinned torch).  Synchronous; returns host arrays."""
+        if locs is None:
+            locs = np.empty(self.k, dtype=np.int64)
+        if vals is None:
+            vals = np.empty(self.k, dtype=np.complex128)
+        if isinstance(x, np.ndarray):
+            x = np.ascontiguousarray(x, dtype=np.complex128)
+        check(self._lib.cusfft_execute_host(self._h, ctypes.c_void_p(_ptr(x)), ctypes.c_void_p(_ptr(locs)),
+                                            ctypes.c_void_p(_ptr(vals))), "cusfft_execute_host")
+        return locs, vals
+
+    def execute_local(self, x):
+        self._use_current_stream()
+        check(self._lib.cusfft_execute_local(self._h, ctypes.c_void_p(x.data_ptr())), "cusfft_execute_local")
+
+    def execute_finish(self, locs, vals):
+        self._use_current_stream()
+        check(self._lib.cusfft_execute_finish(self._h, ctypes.c_void_p(locs.data_ptr()),
+                                              ctypes.c_void_p(vals.data_ptr())), "cusfft_execute_finish")
+        return locs, vals
+
+    def exchange_buffer(self):
+        """(device pointer, bytes per rank) of the all-gather buffer."""
+        ptr = ctypes.c_void_p()
+        per = ctypes.c_int64()
+        check(self._lib.cusfft_exchange_buffer(self._h, ctypes.byref(ptr), ctypes.byref(per)),
+              "cusfft_exchange_buffer")
+        return int(ptr.value), int(per.value)
+
+    def status(self) -> int:
+        return int(self._lib.cusfft_status(self._h))
+
+    # -- introspection
+    def info(self):
+        info = np.zeros(10, dtype=np.int64)
+        a = np.zeros(self.L, dtype=np.int64)
+        s = np.zeros(self.L, dtype=np.int64)
+        t = np.zeros(self.L, dtype=np.int64)
+        check(self._lib.cusfft_get_info(self._h, ctypes.c_void_p(info.ctypes.data), ctypes.c_void_p(a.ctypes.data),
+                                        ctypes.c_void_p(s.ctypes.data), ctypes.c_void_p(t.ctypes.data)),
+              "cusfft_get_info")
+        keys = ("n", "k", "B", "L", "w", "nb", "num", "loc_loops", "T", "max_hits")
+        d = dict(zip(keys, info.tolist()))
+        d.update(a=a, sigma=s, tau=t)
+        return d
+
+    def debug(self, what: int):
+        dtype = {DEBUG_U: np.complex128, DEBUG_UHAT: np.complex128, DEBUG_WINNERS: np.int32,
+                 DEBUG_HITS: np.int32, DEBUG_HIT_VALS: np.complex128, DEBUG_PER_LOOP: np.complex128,
+                 DEBUG_TAPS: np.float64, DEBUG_GHAT: np.complex128, DEBUG_NUM_HITS: np.int64}[what]
+        need = int(self._lib.cusfft_get_debug(self._h, what, None, 0))
+        if need < 0:
+            check(need, "cusfft_get_debug")
+        buf = np.zeros(need // np.dtype(dtype).itemsize, dtype=dtype)
+        if need:
+            got = int(self._lib.cusfft_get_debug(self._h, what, ctypes.c_void_p(buf.ctypes.data), need))
+            if got < 0:
+                check(got, "cusfft_get_debug")
+        if what in (DEBUG_U,):
+            buf = buf.reshape(-1, self.B)
+        elif what == DEBUG_UHAT:
+            buf = buf.reshape(self.L, self.B)
+        elif what == DEBUG_WINNERS:
+            buf = buf.reshape(self.loc_loops, self.num)
+        elif what == DEBUG_PER_LOOP and buf.size:
+            buf = buf.reshape(-1, self.L)
+        return buf
+
+    def set_timing(self, enable: bool = True):
+        check(self._lib.cusfft_set_timing(self._h, 1 if enable else 0), "cusfft_set_timing")
+
+    def stage_times(self):
+        ms = (ctypes.c_float * 6)()
+        check(self._lib.cusfft_get_stage_times(self._h, ms, 6), "cusfft_get_stage_times")
+        return dict(zip(("fold", "fft", "cutoff", "vote", "estimate", "output"), list(ms)))
+
+    def launches_per_execute(self) -> int:
+        return int(self._lib.cusfft_launches_per_execute(self._h))

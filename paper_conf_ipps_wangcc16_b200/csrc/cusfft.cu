@@ -1,0 +1,779 @@
+// cusfft.cu — plan construction, launch sequence and the C ABI declared in
+// include/cusfft.h.  Host code runs only at plan time and to enqueue work;
+// every step of the transform runs in the kernels of exec_kernels.cuh.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdint>
+#include <cstring>
+#include <new>
+#include <vector>
+
+#include "../../include/cusfft.h"
+#include "exec_kernels.cuh"
+#include "plan_kernels.cuh"
+
+using namespace cusfft;
+
+namespace {
+
+constexpr uint32_t kMagic = 0x5FF7B200u;
+thread_local int g_last_cuda_error = 0;
+
+#define CK(expr)                                  \
+  do {                                            \
+    cudaError_t e_ = (expr);                      \
+    if (e_ != cudaSuccess) {                      \
+      g_last_cuda_error = (int)e_;                \
+      return e_ == cudaErrorMemoryAllocation ? CUSFFT_ALLOC : CUSFFT_CUDA; \
+    }                                             \
+  } while (0)
+
+#define CKL()                                     \
+  do {                                            \
+    cudaError_t e_ = cudaGetLastError();          \
+    if (e_ != cudaSuccess) {                      \
+      g_last_cuda_error = (int)e_;                \
+      return CUSFFT_CUDA;                         \
+    }                                             \
+  } while (0)
+
+bool is_pow2(int64_t v) { return v > 0 && (v & (v - 1)) == 0; }
+int ilog2(int64_t v) {
+  int l = 0;
+  while ((int64_t(1) << l) < v) ++l;
+  return l;
+}
+
+// SplitMix64 (Steele, Lea, Flood 2014): the seeded generator of the draws
+// (DESIGN.md §3 [Z-PRNG]).  The paper only says "a <- random() mod n" (L146).
+struct SplitMix64 {
+  uint64_t s;
+  uint64_t next() {
+    s += 0x9E3779B97F4A7C15ull;
+    uint64_t z = s;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+  }
+};
+
+int64_t gcd64(int64_t a, int64_t b) {
+  while (b) {
+    int64_t t = a % b;
+    a = b;
+    b = t;
+  }
+  return a;
+}
+
+// a^-1 mod n by the extended Euclidean algorithm (Alg. 1 line 8, L153).
+int64_t inverse_mod(int64_t a, int64_t n) {
+  int64_t r0 = n, r1 = a % n, t0 = 0, t1 = 1;
+  while (r1) {
+    int64_t q = r0 / r1, tmp;
+    tmp = r0 - q * r1; r0 = r1; r1 = tmp;
+    tmp = t0 - q * t1; t0 = t1; t1 = tmp;
+  }
+  return ((t0 % n) + n) % n;
+}
+
+double binom_tail(int L, double p, int T) {  // P[Binomial(L, p) >= T]
+  double s = 0.0;
+  for (int v = T; v <= L; ++v) {
+    double c = 1.0;
+    for (int i = 0; i < v; ++i) c = c * (L - i) / (i + 1);
+    s += c * std::pow(p, v) * std::pow(1.0 - p, L - v);
+  }
+  return s;
+}
+
+}  // namespace
+
+struct cusfft_plan_s {
+  uint32_t magic = kMagic;
+  int64_t n = 0, k = 0, B = 0, nb = 0;
+  int L = 0, Lg = 0, rank = 0, world = 1;
+  cusfft_params prm{};
+  int log2nb = 0, w = 0, R = 0, num = 0, Lloc = 0, T = 0, max_hits = 0;
+  int B1 = 1, B2 = 1, logB1 = 0, logB2 = 0;
+  int kp2 = 1;
+  bool keys_in_smem = true;
+  int select_smem = 0, vote_smem = 0, output_smem = 0;
+  int vote_P = 1, vote_grid = 1, est_grid = 1;
+  std::vector<SlotParam> slots_h;       // slot order
+  std::vector<int64_t> a_r, sigma_r, tau_r;  // loop order
+  std::vector<int> loc_slots_h, sel_slots_h;
+  RecLayout lay{};
+  // device memory
+  double* d_taps = nullptr;
+  double2* d_ghat = nullptr;
+  double2* d_tw = nullptr;
+  SlotParam* d_slots = nullptr;
+  int* d_loc_slots = nullptr;
+  uint32_t* d_loc_sigma = nullptr;
+  uint32_t* d_loc_a = nullptr;
+  int* d_sel_slots = nullptr;
+  double2* d_u = nullptr;
+  double2* d_v = nullptr;
+  uint8_t* d_records = nullptr;
+  uint64_t* d_gkeys = nullptr;
+  int* d_hits = nullptr;
+  double2* d_hit_vals = nullptr;
+  uint64_t* d_hit_keys = nullptr;
+  double2* d_per_loop = nullptr;
+  int* d_flags = nullptr;  // [0] hit_count (unsigned), [1] overflow, [2] select mismatch, [3] output mismatch
+  double2* d_xbuf = nullptr;
+  int64_t* d_locs_buf = nullptr;
+  double2* d_vals_buf = nullptr;
+  cudaStream_t stream = nullptr;
+  int device = 0;
+  bool timing = false;
+  cudaEvent_t ev[7] = {};
+  bool ev_made = false;
+};
+
+namespace {
+
+bool valid_plan(cusfft_plan_t p) { return p && p->magic == kMagic; }
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+void free_plan(cusfft_plan_t p) {
+  void* ptrs[] = {p->d_taps, p->d_ghat, p->d_tw, p->d_slots, p->d_loc_slots, p->d_loc_sigma, p->d_loc_a,
+                  p->d_sel_slots, p->d_u, p->d_v, p->d_records, p->d_gkeys, p->d_hits, p->d_hit_vals,
+                  p->d_hit_keys, p->d_per_loop, p->d_flags, p->d_xbuf, p->d_locs_buf, p->d_vals_buf};
+  for (void* q : ptrs)
+    if (q) cudaFree(q);
+  if (p->ev_made)
+    for (auto& e : p->ev) cudaEventDestroy(e);
+  p->magic = 0;
+  delete p;
+}
+
+int validate(int64_t n, int64_t k, int64_t B, int32_t L, const cusfft_params& q, int rank, int world) {
+  if (!is_pow2(n) || n < 16 || n > (int64_t(1) << 31)) return CUSFFT_INVALID_N;
+  if (!is_pow2(B) || B < 2 || B >= n) return CUSFFT_INVALID_B;
+  if (L < 1 || L > kMaxLoops) return CUSFFT_INVALID_LOOPS;
+  if (world < 1 || rank < 0 || rank >= world || L % world) return CUSFFT_INVALID_LOOPS;
+  if (q.loc_loops < 1 || q.loc_loops > L || q.vote_threshold < 1 || q.vote_threshold > q.loc_loops)
+    return CUSFFT_INVALID_LOOPS;
+  if (k < 1 || k > 8192 || q.num_select < k || q.num_select > B) return CUSFFT_INVALID_K;
+  if (q.taps) {
+    if (q.num_taps < 1 || q.num_taps > (int64_t(1) << 30)) return CUSFFT_INVALID_PARAM;
+  } else {
+    if (q.filter != CUSFFT_FILTER_DOLPH_CHEBYSHEV && q.filter != CUSFFT_FILTER_GAUSSIAN) return CUSFFT_INVALID_PARAM;
+    if (!(q.tolerance > 0.0 && q.tolerance < 1.0)) return CUSFFT_INVALID_PARAM;
+    if (!(q.lobefrac > 0.0 && q.lobefrac < 0.5)) return CUSFFT_INVALID_PARAM;
+    if (q.box_width < 1 || q.box_width > n || (q.box_width % 2) == 0) return CUSFFT_INVALID_PARAM;
+  }
+  if (q.max_hits < 1 || q.max_hits > (int64_t(1) << 30)) return CUSFFT_INVALID_PARAM;
+  if (q.tau_mode != 0 && q.tau_mode != 1) return CUSFFT_INVALID_PARAM;
+  return CUSFFT_SUCCESS;
+}
+
+int64_t filter_len(const cusfft_params& q) {
+  const double pi = 3.14159265358979323846;
+  int64_t w;
+  if (q.taps) return q.num_taps;
+  if (q.filter == CUSFFT_FILTER_DOLPH_CHEBYSHEV)
+    w = (int64_t)std::floor(std::acosh(1.0 / q.tolerance) / (pi * q.lobefrac));
+  else
+    w = (int64_t)std::floor(2.0 * std::log(1.0 / q.tolerance) / (pi * q.lobefrac));
+  if (w % 2 == 0) --w;
+  return w;
+}
+
+template <class T>
+int dalloc(T** ptr, size_t count) {
+  if (count == 0) count = 1;
+  CK(cudaMalloc((void**)ptr, count * sizeof(T)));
+  return CUSFFT_SUCCESS;
+}
+
+#define TRY(expr)              \
+  do {                         \
+    int rc_ = (expr);          \
+    if (rc_ != CUSFFT_SUCCESS) \
+      return rc_;              \
+  } while (0)
+
+int build_filter(cusfft_plan_t P) {
+  const cusfft_params& q = P->prm;
+  const int w = P->w;
+  const int padded = P->R * (int)P->B;
+  const int c = (w - 1) / 2;
+  cudaStream_t st = P->stream;
+  if (q.taps) {
+    CK(cudaMemsetAsync(P->d_taps, 0, (size_t)padded * sizeof(double), st));
+    CK(cudaMemcpyAsync(P->d_taps, q.taps, (size_t)w * sizeof(double), cudaMemcpyHostToDevice, st));
+  } else {
+    double* win = nullptr;
+    double* pj = nullptr;
+    TRY(dalloc(&win, (size_t)c + 1));
+    if (q.filter == CUSFFT_FILTER_DOLPH_CHEBYSHEV) {
+      TRY(dalloc(&pj, (size_t)c + 1));
+      const double x0 = std::cosh(std::acosh(1.0 / q.tolerance) / (double)(w - 1));
+      k_cheb_samples<<<(c + 256) / 256, 256, 0, st>>>(pj, w, x0);
+      CKL();
+      k_dc_window<<<c + 1, 256, 0, st>>>(pj, win, w);
+      CKL();
+    } else {
+      const double s = (double)c / std::sqrt(2.0 * std::log(1.0 / q.tolerance));
+      k_gauss_window<<<(c + 256) / 256, 256, 0, st>>>(win, w, s);
+      CKL();
+    }
+    k_taps<<<(padded + 255) / 256, 256, 0, st>>>(win, P->d_taps, w, padded, P->n, q.box_width);
+    CKL();
+    k_normalize<<<1, 1024, 0, st>>>(P->d_taps, w);
+    CKL();
+    CK(cudaStreamSynchronize(st));
+    cudaFree(win);
+    if (pj) cudaFree(pj);
+  }
+  k_ghat<<<(int)P->nb + 1, 256, 0, st>>>(P->d_taps, P->d_ghat, w, P->n, (int)P->nb);
+  CKL();
+  k_twiddles<<<(int)((P->B + 255) / 256), 256, 0, st>>>(P->d_tw, (int)P->B);
+  CKL();
+  return CUSFFT_SUCCESS;
+}
+
+int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, const cusfft_params* pin, int rank,
+              int world) {
+  if (!out) return CUSFFT_NULL_PTR;
+  cusfft_params q;
+  if (pin) {
+    q = *pin;
+  } else {
+    int rc = cusfft_params_default(&q, n, k, B);
+    if (rc) return rc;
+  }
+  if (!pin || q.loc_loops == 0) q.loc_loops = std::min<int32_t>(L, 8);
+  if (!pin || q.vote_threshold == 0) q.vote_threshold = q.loc_loops / 2 + 1;
+  if (q.num_select == 0) q.num_select = (int32_t)k;
+  if (q.max_hits == 0) {
+    const double pr = (double)q.num_select / (double)B;
+    double e = (double)n * binom_tail(q.loc_loops, pr, q.vote_threshold) + (double)k;
+    int64_t mh = std::max<int64_t>(16384, (int64_t)(4.0 * e));
+    q.max_hits = std::min<int64_t>(mh, std::min<int64_t>(n, int64_t(1) << 30));
+  }
+  {
+    int rc = validate(n, k, B, L, q, rank, world);
+    if (rc) return rc;
+  }
+  int ndev = 0;
+  CK(cudaGetDeviceCount(&ndev));
+  if (ndev < 1) {
+    g_last_cuda_error = (int)cudaErrorNoDevice;
+    return CUSFFT_CUDA;
+  }
+  int dev = q.device;
+  if (dev < 0) CK(cudaGetDevice(&dev));
+  if (dev >= ndev) return CUSFFT_INVALID_PARAM;
+  DeviceGuard guard(dev);
+
+  cusfft_plan_t P = new (std::nothrow) cusfft_plan_s();
+  if (!P) return CUSFFT_ALLOC;
+  P->n = n; P->k = k; P->B = B; P->L = L; P->prm = q; P->rank = rank; P->world = world;
+  P->device = dev;
+  P->nb = n / B;
+  P->log2nb = ilog2(P->nb);
+  P->Lg = L / world;
+  P->num = q.num_select;
+  P->Lloc = q.loc_loops;
+  P->T = q.vote_threshold;
+  P->max_hits = (int)q.max_hits;
+  const int64_t w64 = filter_len(q);
+  if (w64 < 1 || w64 > (int64_t(1) << 30)) {
+    free_plan(P);
+    return CUSFFT_INVALID_PARAM;
+  }
+  P->w = (int)w64;
+  P->R = (int)((w64 + B - 1) / B);
+  P->stream = nullptr;
+
+  // ---- draws (loop order), Alg. 1, Def. 1
+  SplitMix64 rng{q.seed};
+  P->a_r.resize(L); P->sigma_r.resize(L); P->tau_r.resize(L);
+  for (int r = 0; r < L; ++r) {
+    int64_t a = (int64_t)(rng.next() % (uint64_t)n);
+    while (gcd64(a, n) != 1) a = (int64_t)(rng.next() % (uint64_t)n);
+    P->a_r[r] = a;
+    P->sigma_r[r] = inverse_mod(a, n);
+    P->tau_r[r] = q.tau_mode ? (int64_t)(rng.next() % (uint64_t)n) : 0;
+  }
+  // ---- slots: rank g owns loops r = i*world + g at slots g*Lg + i
+  P->slots_h.resize(L);
+  for (int s = 0; s < L; ++s) {
+    const int g = s / P->Lg, i = s % P->Lg, r = i * world + g;
+    P->slots_h[s] = SlotParam{(uint32_t)P->sigma_r[r], (uint32_t)P->tau_r[r], (uint32_t)P->a_r[r], (uint32_t)r};
+  }
+  std::vector<uint32_t> loc_sig, loc_a;
+  for (int s = 0; s < L; ++s) {
+    if ((int)P->slots_h[s].loop < P->Lloc) {
+      P->loc_slots_h.push_back(s);
+      loc_sig.push_back(P->slots_h[s].sigma);
+      loc_a.push_back(P->slots_h[s].a);
+      if (s / P->Lg == rank) P->sel_slots_h.push_back(s);
+    }
+  }
+
+  // ---- layout
+  auto align256 = [](int64_t v) { return (v + 255) & ~int64_t(255); };
+  P->lay.off_bitmap = align256(B * 16);
+  P->lay.off_J = align256(P->lay.off_bitmap + ((B + 31) / 32) * 4);
+  P->lay.rec_bytes = align256(P->lay.off_J + (int64_t)P->num * 4);
+  if (B <= 2048) {
+    P->B1 = 1; P->B2 = (int)B;
+  } else {
+    const int lb = ilog2(B);
+    P->B1 = 1 << ((lb + 1) / 2);
+    P->B2 = (int)(B / P->B1);
+  }
+  P->logB1 = ilog2(P->B1);
+  P->logB2 = ilog2(P->B2);
+  P->keys_in_smem = B <= 16384;
+  P->select_smem = 4096 * 4 + 64 * 4 + (P->keys_in_smem ? (int)B * 8 : 0);
+  P->vote_smem = P->Lloc * (int)(B / 32) * 4;
+  P->kp2 = 1;
+  while (P->kp2 < k) P->kp2 <<= 1;
+  P->output_smem = 4096 * 4 + 64 * 4 + 2 * P->kp2 * 4;
+  P->vote_P = (int)std::min<int64_t>(P->nb, 16);
+  {
+    const int64_t items = (int64_t)(P->Lloc - P->T + 1) * P->num * (P->nb / P->vote_P);
+    int sms = 148;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    P->vote_grid = (int)std::max<int64_t>(1, std::min<int64_t>((items + 255) / 256, (int64_t)sms * 8));
+    P->est_grid = std::max(1, std::min((P->max_hits + 127) / 128, sms * 4));
+  }
+  if (P->vote_smem > 200 * 1024) {
+    free_plan(P);
+    return CUSFFT_INVALID_B;
+  }
+
+  int rc = CUSFFT_SUCCESS;
+  auto fail = [&](int code) {
+    free_plan(P);
+    return code;
+  };
+  if ((rc = dalloc(&P->d_taps, (size_t)P->R * B))) return fail(rc);
+  if ((rc = dalloc(&P->d_ghat, (size_t)P->nb + 1))) return fail(rc);
+  if ((rc = dalloc(&P->d_tw, (size_t)B))) return fail(rc);
+  if ((rc = dalloc(&P->d_slots, (size_t)L))) return fail(rc);
+  if ((rc = dalloc(&P->d_loc_slots, (size_t)P->Lloc))) return fail(rc);
+  if ((rc = dalloc(&P->d_loc_sigma, (size_t)P->Lloc))) return fail(rc);
+  if ((rc = dalloc(&P->d_loc_a, (size_t)P->Lloc))) return fail(rc);
+  if ((rc = dalloc(&P->d_sel_slots, std::max<size_t>(1, P->sel_slots_h.size())))) return fail(rc);
+  if ((rc = dalloc(&P->d_u, (size_t)P->Lg * B))) return fail(rc);
+  if (P->B1 > 1 && (rc = dalloc(&P->d_v, (size_t)P->Lg * B))) return fail(rc);
+  if ((rc = dalloc(&P->d_records, (size_t)L * P->lay.rec_bytes))) return fail(rc);
+  if (!P->keys_in_smem && (rc = dalloc(&P->d_gkeys, std::max<size_t>(1, P->sel_slots_h.size()) * B)))
+    return fail(rc);
+  if ((rc = dalloc(&P->d_hits, (size_t)P->max_hits))) return fail(rc);
+  if ((rc = dalloc(&P->d_hit_vals, (size_t)P->max_hits))) return fail(rc);
+  if ((rc = dalloc(&P->d_hit_keys, (size_t)P->max_hits))) return fail(rc);
+  if (q.debug && (rc = dalloc(&P->d_per_loop, (size_t)P->max_hits * L))) return fail(rc);
+  if ((rc = dalloc(&P->d_flags, 8))) return fail(rc);
+  auto upload = [&](void* dst, const void* src, size_t bytes) -> int {
+    CK(cudaMemcpy(dst, src, bytes, cudaMemcpyHostToDevice));
+    return CUSFFT_SUCCESS;
+  };
+  if ((rc = upload(P->d_slots, P->slots_h.data(), L * sizeof(SlotParam)))) return fail(rc);
+  if ((rc = upload(P->d_loc_slots, P->loc_slots_h.data(), P->Lloc * sizeof(int)))) return fail(rc);
+  if ((rc = upload(P->d_loc_sigma, loc_sig.data(), P->Lloc * sizeof(uint32_t)))) return fail(rc);
+  if ((rc = upload(P->d_loc_a, loc_a.data(), P->Lloc * sizeof(uint32_t)))) return fail(rc);
+  if (!P->sel_slots_h.empty() &&
+      (rc = upload(P->d_sel_slots, P->sel_slots_h.data(), P->sel_slots_h.size() * sizeof(int))))
+    return fail(rc);
+  if (cudaMemset(P->d_records, 0, (size_t)L * P->lay.rec_bytes) != cudaSuccess ||
+      cudaMemset(P->d_flags, 0, 8 * sizeof(int)) != cudaSuccess) {
+    g_last_cuda_error = (int)cudaGetLastError();
+    return fail(CUSFFT_CUDA);
+  }
+  if (cudaFuncSetAttribute(k_select, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
+      cudaFuncSetAttribute(k_vote, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
+      cudaFuncSetAttribute(k_output, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess) {
+    g_last_cuda_error = (int)cudaGetLastError();
+    return fail(CUSFFT_CUDA);
+  }
+  if ((rc = build_filter(P))) return fail(rc);
+  if (cudaStreamSynchronize(P->stream) != cudaSuccess) {
+    g_last_cuda_error = (int)cudaGetLastError();
+    return fail(CUSFFT_CUDA);
+  }
+  *out = P;
+  return CUSFFT_SUCCESS;
+}
+
+inline void mark(cusfft_plan_t P, int i) {
+  if (P->timing) cudaEventRecord(P->ev[i], P->stream);
+}
+
+int launch_local(cusfft_plan_t P, const double2* x) {
+  const int B = (int)P->B;
+  cudaStream_t st = P->stream;
+  CK(cudaMemsetAsync(P->d_flags, 0, 8 * sizeof(int), st));
+  mark(P, 0);
+  {
+    dim3 grid((B + 255) / 256, P->Lg);
+    k_fold<16><<<grid, 256, 0, st>>>(x, P->d_taps, P->d_slots + (size_t)P->rank * P->Lg, P->d_u, B, P->w, P->R,
+                                     (uint32_t)(P->n - 1));
+    CKL();
+  }
+  mark(P, 1);
+  uint8_t* myrec = P->d_records + (int64_t)P->rank * P->Lg * P->lay.rec_bytes;
+  const int64_t rec_e = P->lay.rec_bytes / 16;
+  if (P->B1 > 1) {
+    // pass 1: m = B1 over columns c (stride B2), twiddle e^{-2 pi i c k1 / B}
+    const int m = P->B1;
+    const int nseq = std::max(1, kFftSmemElems / m);
+    const int total = P->Lg * P->B2;
+    k_fft_pass<<<(total + nseq - 1) / nseq, 256, 0, st>>>(P->d_u, P->d_v, P->d_tw, B, P->logB1, nseq, P->B2, total,
+                                                         B, 1, P->B2, B, 1, P->B2, 1);
+    CKL();
+    const int m2 = P->B2;
+    const int nseq2 = std::max(1, kFftSmemElems / m2);
+    const int total2 = P->Lg * P->B1;
+    k_fft_pass<<<(total2 + nseq2 - 1) / nseq2, 256, 0, st>>>(
+        P->d_v, reinterpret_cast<double2*>(myrec), P->d_tw, B, P->logB2, nseq2, P->B1, total2, B, P->B2, 1, rec_e,
+        1, P->B1, 0);
+    CKL();
+  } else {
+    const int m = P->B2;
+    const int nseq = std::max(1, kFftSmemElems / m);
+    const int total = P->Lg;
+    k_fft_pass<<<(total + nseq - 1) / nseq, 256, 0, st>>>(P->d_u, reinterpret_cast<double2*>(myrec), P->d_tw, B,
+                                                         P->logB2, nseq, 1, total, B, 0, 1, rec_e, 0, 1, 0);
+    CKL();
+  }
+  mark(P, 2);
+  if (!P->sel_slots_h.empty()) {
+    k_select<<<(int)P->sel_slots_h.size(), 1024, P->select_smem, st>>>(
+        P->d_records, P->lay, P->d_sel_slots, B, P->num, P->d_gkeys, P->keys_in_smem ? 1 : 0, P->d_flags + 1);
+    CKL();
+  }
+  mark(P, 3);
+  return CUSFFT_SUCCESS;
+}
+
+int launch_finish(cusfft_plan_t P, int64_t* locs, double2* vals) {
+  cudaStream_t st = P->stream;
+  VoteArgs va;
+  va.records = P->d_records;
+  va.lay = P->lay;
+  va.loc_slots = P->d_loc_slots;
+  va.loc_sigma = P->d_loc_sigma;
+  va.loc_a = P->d_loc_a;
+  va.Lloc = P->Lloc;
+  va.T = P->T;
+  va.num = P->num;
+  va.B = (int)P->B;
+  va.nb = (int)P->nb;
+  va.log2nb = P->log2nb;
+  va.P = P->vote_P;
+  va.nmask = (uint32_t)(P->n - 1);
+  va.hits = P->d_hits;
+  va.hit_count = reinterpret_cast<unsigned*>(P->d_flags);
+  va.max_hits = P->max_hits;
+  k_vote<<<P->vote_grid, 256, P->vote_smem, st>>>(va);
+  CKL();
+  mark(P, 4);
+  EstArgs ea;
+  ea.records = P->d_records;
+  ea.lay = P->lay;
+  ea.slots = P->d_slots;
+  ea.L = P->L;
+  ea.ghat = P->d_ghat;
+  ea.hits = P->d_hits;
+  ea.hit_count = reinterpret_cast<const unsigned*>(P->d_flags);
+  ea.max_hits = P->max_hits;
+  ea.nmask = (uint32_t)(P->n - 1);
+  ea.log2nb = P->log2nb;
+  ea.nb = (int)P->nb;
+  ea.B = (int)P->B;
+  ea.n = (double)P->n;
+  ea.hit_vals = P->d_hit_vals;
+  ea.hit_keys = P->d_hit_keys;
+  ea.per_loop = P->d_per_loop;
+  k_estimate<<<P->est_grid, 128, 0, st>>>(ea);
+  CKL();
+  mark(P, 5);
+  k_output<<<1, 1024, P->output_smem, st>>>(P->d_hits, reinterpret_cast<const unsigned*>(P->d_flags), P->max_hits,
+                                            P->d_hit_vals, P->d_hit_keys, (int)P->k, P->kp2, locs, vals,
+                                            P->d_flags + 1);
+  CKL();
+  mark(P, 6);
+  return CUSFFT_SUCCESS;
+}
+
+}  // namespace
+
+// ===========================================================================
+// C ABI
+// ===========================================================================
+extern "C" {
+
+int32_t cusfft_abi_version(void) { return CUSFFT_ABI_VERSION; }
+int32_t cusfft_last_cuda_error(void) { return g_last_cuda_error; }
+
+const char* cusfft_strerror(int code) {
+  switch (code) {
+    case CUSFFT_SUCCESS: return "success";
+    case CUSFFT_INVALID_N: return "n must be a power of two in [16, 2^31]";
+    case CUSFFT_INVALID_B: return "B must be a power of two with 2 <= B < n";
+    case CUSFFT_INVALID_K: return "need 1 <= k <= 8192 and k <= num_select <= B";
+    case CUSFFT_INVALID_LOOPS: return "need 1 <= T <= L_loc <= L <= 64 and world | L";
+    case CUSFFT_INVALID_PARAM: return "invalid filter or plan parameter";
+    case CUSFFT_NULL_PTR: return "null pointer argument";
+    case CUSFFT_ALLOC: return "device allocation failed";
+    case CUSFFT_CUDA: return "CUDA runtime error (see cusfft_last_cuda_error)";
+    case CUSFFT_HIT_OVERFLOW: return "more than max_hits frequencies reached the vote threshold";
+    case CUSFFT_INVALID_PLAN: return "invalid or destroyed plan";
+    case CUSFFT_INTERNAL: return "device-side consistency check failed";
+    default: return "unknown cusfft status";
+  }
+}
+
+int64_t cusfft_default_B(int64_t n, int64_t k, double bcst) {
+  if (n < 2 || k < 1 || !(bcst > 0)) return 0;
+  const double v = bcst * std::sqrt((double)n * (double)k / std::log2((double)n));
+  int64_t b = 1;
+  while ((double)(2 * b) <= v) b *= 2;
+  return b;
+}
+
+int cusfft_params_default(cusfft_params* p, int64_t n, int64_t k, int64_t B) {
+  if (!p) return CUSFFT_NULL_PTR;
+  if (!is_pow2(n) || n < 16 || n > (int64_t(1) << 31)) return CUSFFT_INVALID_N;
+  if (!is_pow2(B) || B < 2 || B >= n) return CUSFFT_INVALID_B;
+  if (k < 1) return CUSFFT_INVALID_K;
+  std::memset(p, 0, sizeof(*p));
+  p->filter = CUSFFT_FILTER_DOLPH_CHEBYSHEV;
+  p->tolerance = 1e-8;
+  p->lobefrac = 0.5 / (double)B;
+  p->box_width = n / B - 1;
+  p->loc_loops = 0;       // -> min(L, 8) at plan time
+  p->vote_threshold = 0;  // -> floor(L_loc/2) + 1
+  p->num_select = (int32_t)std::min<int64_t>(k, B);
+  p->tau_mode = 1;
+  p->seed = 1;
+  p->max_hits = 0;  // -> from the expected false-hit count
+  p->device = -1;
+  p->debug = 0;
+  p->taps = nullptr;
+  p->num_taps = 0;
+  return CUSFFT_SUCCESS;
+}
+
+int cusfft_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, const cusfft_params* p) {
+  return make_plan(out, n, k, B, L, p, 0, 1);
+}
+
+int cusfft_plan_dist(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, const cusfft_params* p,
+                     int32_t rank, int32_t world) {
+  return make_plan(out, n, k, B, L, p, rank, world);
+}
+
+int cusfft_destroy(cusfft_plan_t plan) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  DeviceGuard g(plan->device);
+  cudaStreamSynchronize(plan->stream);
+  free_plan(plan);
+  return CUSFFT_SUCCESS;
+}
+
+int cusfft_set_stream(cusfft_plan_t plan, void* s) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  plan->stream = reinterpret_cast<cudaStream_t>(s);
+  return CUSFFT_SUCCESS;
+}
+
+int cusfft_execute_local(cusfft_plan_t plan, const void* d_x) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  if (!d_x) return CUSFFT_NULL_PTR;
+  DeviceGuard g(plan->device);
+  return launch_local(plan, reinterpret_cast<const double2*>(d_x));
+}
+
+int cusfft_execute_finish(cusfft_plan_t plan, int64_t* d_locs, void* d_vals) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  if (!d_locs || !d_vals) return CUSFFT_NULL_PTR;
+  DeviceGuard g(plan->device);
+  return launch_finish(plan, d_locs, reinterpret_cast<double2*>(d_vals));
+}
+
+int cusfft_execute(cusfft_plan_t plan, const void* d_x, int64_t* d_locs, void* d_vals) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  if (!d_x || !d_locs || !d_vals) return CUSFFT_NULL_PTR;
+  if (plan->world != 1) return CUSFFT_INVALID_LOOPS;
+  DeviceGuard g(plan->device);
+  int rc = launch_local(plan, reinterpret_cast<const double2*>(d_x));
+  if (rc) return rc;
+  return launch_finish(plan, d_locs, reinterpret_cast<double2*>(d_vals));
+}
+
+int cusfft_status(cusfft_plan_t plan) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  DeviceGuard g(plan->device);
+  int flags[8];
+  CK(cudaStreamSynchronize(plan->stream));
+  CK(cudaMemcpy(flags, plan->d_flags, sizeof(flags), cudaMemcpyDeviceToHost));
+  if (flags[1]) return CUSFFT_HIT_OVERFLOW;
+  if (flags[2] || flags[3]) return CUSFFT_INTERNAL;
+  return CUSFFT_SUCCESS;
+}
+
+int cusfft_execute_host(cusfft_plan_t plan, const void* h_x, int64_t* h_locs, void* h_vals) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  if (!h_x || !h_locs || !h_vals) return CUSFFT_NULL_PTR;
+  if (plan->world != 1) return CUSFFT_INVALID_LOOPS;
+  DeviceGuard g(plan->device);
+  int rc;
+  if (!plan->d_xbuf) {
+    if ((rc = dalloc(&plan->d_xbuf, (size_t)plan->n))) return rc;
+    if ((rc = dalloc(&plan->d_locs_buf, (size_t)plan->k))) return rc;
+    if ((rc = dalloc(&plan->d_vals_buf, (size_t)plan->k))) return rc;
+  }
+  cudaStream_t st = plan->stream;
+  CK(cudaMemcpyAsync(plan->d_xbuf, h_x, (size_t)plan->n * 16, cudaMemcpyHostToDevice, st));
+  if ((rc = launch_local(plan, plan->d_xbuf))) return rc;
+  if ((rc = launch_finish(plan, plan->d_locs_buf, plan->d_vals_buf))) return rc;
+  CK(cudaMemcpyAsync(h_locs, plan->d_locs_buf, (size_t)plan->k * 8, cudaMemcpyDeviceToHost, st));
+  CK(cudaMemcpyAsync(h_vals, plan->d_vals_buf, (size_t)plan->k * 16, cudaMemcpyDeviceToHost, st));
+  return cusfft_status(plan);
+}
+
+int cusfft_exchange_buffer(cusfft_plan_t plan, void** d_buf, int64_t* bytes_per_rank) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  if (!d_buf || !bytes_per_rank) return CUSFFT_NULL_PTR;
+  *d_buf = plan->d_records;
+  *bytes_per_rank = (int64_t)plan->Lg * plan->lay.rec_bytes;
+  return CUSFFT_SUCCESS;
+}
+
+int cusfft_get_info(cusfft_plan_t plan, int64_t* info, int64_t* a, int64_t* sigma, int64_t* tau) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  if (info) {
+    int64_t v[10] = {plan->n, plan->k, plan->B, plan->L, plan->w, plan->nb,
+                     plan->num, plan->Lloc, plan->T, plan->max_hits};
+    std::memcpy(info, v, sizeof(v));
+  }
+  for (int r = 0; r < plan->L; ++r) {
+    if (a) a[r] = plan->a_r[r];
+    if (sigma) sigma[r] = plan->sigma_r[r];
+    if (tau) tau[r] = plan->tau_r[r];
+  }
+  return CUSFFT_SUCCESS;
+}
+
+int64_t cusfft_get_debug(cusfft_plan_t plan, int32_t what, void* dst, int64_t cap) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  DeviceGuard g(plan->device);
+  CK(cudaStreamSynchronize(plan->stream));
+  unsigned hc = 0;
+  CK(cudaMemcpy(&hc, plan->d_flags, sizeof(unsigned), cudaMemcpyDeviceToHost));
+  const int64_t H = std::min<int64_t>(hc, plan->max_hits);
+  const int64_t B = plan->B, L = plan->L;
+  auto slot_of = [&](int r) { return (r % plan->world) * plan->Lg + r / plan->world; };
+  int64_t need = 0;
+  switch (what) {
+    case CUSFFT_DEBUG_U: need = (int64_t)plan->Lg * B * 16; break;
+    case CUSFFT_DEBUG_UHAT: need = L * B * 16; break;
+    case CUSFFT_DEBUG_WINNERS: need = (int64_t)plan->Lloc * plan->num * 4; break;
+    case CUSFFT_DEBUG_HITS: need = H * 4; break;
+    case CUSFFT_DEBUG_HIT_VALS: need = H * 16; break;
+    case CUSFFT_DEBUG_PER_LOOP: need = plan->d_per_loop ? H * L * 16 : 0; break;
+    case CUSFFT_DEBUG_TAPS: need = (int64_t)plan->w * 8; break;
+    case CUSFFT_DEBUG_GHAT: need = (plan->nb + 1) * 16; break;
+    case CUSFFT_DEBUG_NUM_HITS: need = 8; break;
+    default: return CUSFFT_INVALID_PARAM;
+  }
+  if (!dst || cap < need || need == 0) return need;
+  uint8_t* out = reinterpret_cast<uint8_t*>(dst);
+  switch (what) {
+    case CUSFFT_DEBUG_U:
+      CK(cudaMemcpy(out, plan->d_u, need, cudaMemcpyDeviceToHost));
+      break;
+    case CUSFFT_DEBUG_UHAT:
+      for (int r = 0; r < L; ++r)
+        CK(cudaMemcpy(out + (int64_t)r * B * 16, plan->d_records + (int64_t)slot_of(r) * plan->lay.rec_bytes, B * 16,
+                      cudaMemcpyDeviceToHost));
+      break;
+    case CUSFFT_DEBUG_WINNERS:
+      for (int r = 0; r < plan->Lloc; ++r)
+        CK(cudaMemcpy(out + (int64_t)r * plan->num * 4,
+                      plan->d_records + (int64_t)slot_of(r) * plan->lay.rec_bytes + plan->lay.off_J,
+                      (int64_t)plan->num * 4, cudaMemcpyDeviceToHost));
+      break;
+    case CUSFFT_DEBUG_HITS:
+      CK(cudaMemcpy(out, plan->d_hits, need, cudaMemcpyDeviceToHost));
+      break;
+    case CUSFFT_DEBUG_HIT_VALS:
+      CK(cudaMemcpy(out, plan->d_hit_vals, need, cudaMemcpyDeviceToHost));
+      break;
+    case CUSFFT_DEBUG_PER_LOOP: {
+      std::vector<double2> tmp((size_t)(H * L));
+      CK(cudaMemcpy(tmp.data(), plan->d_per_loop, need, cudaMemcpyDeviceToHost));
+      double2* o = reinterpret_cast<double2*>(out);
+      for (int64_t h = 0; h < H; ++h)
+        for (int r = 0; r < L; ++r) o[h * L + r] = tmp[(size_t)(h * L + slot_of(r))];
+      break;
+    }
+    case CUSFFT_DEBUG_TAPS:
+      CK(cudaMemcpy(out, plan->d_taps, need, cudaMemcpyDeviceToHost));
+      break;
+    case CUSFFT_DEBUG_GHAT:
+      CK(cudaMemcpy(out, plan->d_ghat, need, cudaMemcpyDeviceToHost));
+      break;
+    case CUSFFT_DEBUG_NUM_HITS: {
+      int64_t v = hc;
+      std::memcpy(out, &v, 8);
+      break;
+    }
+  }
+  return need;
+}
+
+int cusfft_set_timing(cusfft_plan_t plan, int32_t enable) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  DeviceGuard g(plan->device);
+  if (enable && !plan->ev_made) {
+    for (auto& e : plan->ev) CK(cudaEventCreate(&e));
+    plan->ev_made = true;
+  }
+  plan->timing = enable != 0;
+  return CUSFFT_SUCCESS;
+}
+
+int cusfft_get_stage_times(cusfft_plan_t plan, float* ms, int32_t cap) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  if (!ms) return CUSFFT_NULL_PTR;
+  if (!plan->ev_made) return CUSFFT_INVALID_PARAM;
+  DeviceGuard g(plan->device);
+  CK(cudaStreamSynchronize(plan->stream));
+  for (int i = 0; i < 6 && i < cap; ++i) {
+    float t = 0.f;
+    if (cudaEventElapsedTime(&t, plan->ev[i], plan->ev[i + 1]) != cudaSuccess) t = -1.f;
+    ms[i] = t;
+  }
+  return CUSFFT_SUCCESS;
+}
+
+int32_t cusfft_launches_per_execute(cusfft_plan_t plan) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  int n = 1 /*fold*/ + (plan->B1 > 1 ? 2 : 1) /*fft*/ + (plan->sel_slots_h.empty() ? 0 : 1) + 3 /*vote,est,out*/;
+  return n;
+}
+
+}  // extern "C"
