@@ -6,6 +6,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <vector>
@@ -99,9 +100,9 @@ struct cusfft_plan_s {
   int log2nb = 0, w = 0, R = 0, num = 0, Lloc = 0, T = 0, max_hits = 0;
   int B1 = 1, B2 = 1, logB1 = 0, logB2 = 0;
   int kp2 = 1;
-  bool keys_in_smem = true;
   int select_smem = 0, vote_smem = 0, output_smem = 0;
   int vote_P = 1, vote_grid = 1, est_grid = 1;
+  int fft_smem1 = 0, fft_smem2 = 0;
   std::vector<SlotParam> slots_h;       // slot order
   std::vector<int64_t> a_r, sigma_r, tau_r;  // loop order
   std::vector<int> loc_slots_h, sel_slots_h;
@@ -118,7 +119,9 @@ struct cusfft_plan_s {
   double2* d_u = nullptr;
   double2* d_v = nullptr;
   uint8_t* d_records = nullptr;
-  uint64_t* d_gkeys = nullptr;
+  uint64_t* d_keys = nullptr;     // [n_sel][B] cutoff keys of this rank's location loops
+  uint32_t* d_hist = nullptr;     // [n_sel][4096] top-digit histograms (self-resetting)
+  int* d_key_index = nullptr;     // [Lg] local slot -> selection index or -1
   int* d_hits = nullptr;
   double2* d_hit_vals = nullptr;
   uint64_t* d_hit_keys = nullptr;
@@ -132,6 +135,15 @@ struct cusfft_plan_s {
   bool timing = false;
   cudaEvent_t ev[7] = {};
   bool ev_made = false;
+  // CUDA graphs of the launch sequences, keyed by the caller's pointers
+  bool use_graph = true;
+  cudaStream_t cap_stream = nullptr;
+  struct GraphEntry {
+    const void* a = nullptr;
+    const void* b = nullptr;
+    const void* c = nullptr;
+    cudaGraphExec_t exec = nullptr;
+  } g_full, g_local, g_finish;
 };
 
 namespace {
@@ -152,12 +164,15 @@ struct DeviceGuard {
 
 void free_plan(cusfft_plan_t p) {
   void* ptrs[] = {p->d_taps, p->d_ghat, p->d_tw, p->d_slots, p->d_loc_slots, p->d_loc_sigma, p->d_loc_a,
-                  p->d_sel_slots, p->d_u, p->d_v, p->d_records, p->d_gkeys, p->d_hits, p->d_hit_vals,
+                  p->d_sel_slots, p->d_u, p->d_v, p->d_records, p->d_keys, p->d_hist, p->d_key_index, p->d_hits, p->d_hit_vals,
                   p->d_hit_keys, p->d_per_loop, p->d_flags, p->d_xbuf, p->d_locs_buf, p->d_vals_buf};
   for (void* q : ptrs)
     if (q) cudaFree(q);
   if (p->ev_made)
     for (auto& e : p->ev) cudaEventDestroy(e);
+  for (auto* g : {&p->g_full, &p->g_local, &p->g_finish})
+    if (g->exec) cudaGraphExecDestroy(g->exec);
+  if (p->cap_stream) cudaStreamDestroy(p->cap_stream);
   p->magic = 0;
   delete p;
 }
@@ -249,6 +264,52 @@ int build_filter(cusfft_plan_t P) {
   return CUSFFT_SUCCESS;
 }
 
+template <int M>
+constexpr int fft_E() { return M < 1024 ? 1024 : M; }
+
+template <int M>
+cudaError_t launch_fft_t(const FftPassArgs& a, int smem, cudaStream_t st) {
+  constexpr int E = fft_E<M>();
+  constexpr int NSEQ = E / M;
+  const int grid = (a.total_seq + NSEQ - 1) / NSEQ;
+  k_fft<M, E, 128><<<grid, 128, smem, st>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_fft(int M, const FftPassArgs& a, int smem, cudaStream_t st) {
+  switch (M) {
+    case 2: return launch_fft_t<2>(a, smem, st);
+    case 4: return launch_fft_t<4>(a, smem, st);
+    case 8: return launch_fft_t<8>(a, smem, st);
+    case 16: return launch_fft_t<16>(a, smem, st);
+    case 32: return launch_fft_t<32>(a, smem, st);
+    case 64: return launch_fft_t<64>(a, smem, st);
+    case 128: return launch_fft_t<128>(a, smem, st);
+    case 256: return launch_fft_t<256>(a, smem, st);
+    case 512: return launch_fft_t<512>(a, smem, st);
+    case 1024: return launch_fft_t<1024>(a, smem, st);
+    case 2048: return launch_fft_t<2048>(a, smem, st);
+    case 4096: return launch_fft_t<4096>(a, smem, st);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+template <int M>
+cudaError_t set_fft_attr_t() {
+  return cudaFuncSetAttribute(k_fft<M, fft_E<M>(), 128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              fft_smem_bytes(fft_E<M>()));
+}
+
+cudaError_t set_fft_attrs() {
+  cudaError_t e = cudaSuccess;
+  cudaError_t r[] = {set_fft_attr_t<2>(), set_fft_attr_t<4>(), set_fft_attr_t<8>(), set_fft_attr_t<16>(),
+                     set_fft_attr_t<32>(), set_fft_attr_t<64>(), set_fft_attr_t<128>(), set_fft_attr_t<256>(),
+                     set_fft_attr_t<512>(), set_fft_attr_t<1024>(), set_fft_attr_t<2048>(), set_fft_attr_t<4096>()};
+  for (cudaError_t x : r)
+    if (x != cudaSuccess) e = x;
+  return e;
+}
+
 int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, const cusfft_params* pin, int rank,
               int world) {
   if (!out) return CUSFFT_NULL_PTR;
@@ -302,6 +363,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   P->w = (int)w64;
   P->R = (int)((w64 + B - 1) / B);
   P->stream = nullptr;
+  if (const char* e = std::getenv("CUSFFT_NO_GRAPH")) P->use_graph = !(e[0] == '1');
 
   // ---- draws (loop order), Alg. 1, Def. 1
   SplitMix64 rng{q.seed};
@@ -343,19 +405,20 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   }
   P->logB1 = ilog2(P->B1);
   P->logB2 = ilog2(P->B2);
-  P->keys_in_smem = B <= 16384;
-  P->select_smem = 4096 * 4 + 64 * 4 + (P->keys_in_smem ? (int)B * 8 : 0);
-  P->vote_smem = P->Lloc * (int)(B / 32) * 4;
+  P->select_smem = 4096 * 4 + 64 * 4 + kSelCap * 12;
+  P->vote_smem = P->Lloc * (int)((B + 31) / 32) * 4;
   P->kp2 = 1;
   while (P->kp2 < k) P->kp2 <<= 1;
-  P->output_smem = 4096 * 4 + 64 * 4 + 2 * P->kp2 * 4;
+  P->output_smem = 4096 * 4 + 64 * 4 + kOutCap * 12 + std::max(P->kp2, 1024) * 8;
+  P->fft_smem1 = fft_smem_bytes(std::max(1024, P->B1));
+  P->fft_smem2 = fft_smem_bytes(std::max(1024, P->B2));
   P->vote_P = (int)std::min<int64_t>(P->nb, 16);
   {
     const int64_t items = (int64_t)(P->Lloc - P->T + 1) * P->num * (P->nb / P->vote_P);
     int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    P->vote_grid = (int)std::max<int64_t>(1, std::min<int64_t>((items + 255) / 256, (int64_t)sms * 8));
-    P->est_grid = std::max(1, std::min((P->max_hits + 127) / 128, sms * 4));
+    P->vote_grid = (int)std::max<int64_t>(1, std::min<int64_t>((items + 255) / 256, (int64_t)sms * 4));
+    P->est_grid = std::max(1, std::min((P->max_hits + 7) / 8, sms * 4));
   }
   if (P->vote_smem > 200 * 1024) {
     free_plan(P);
@@ -378,8 +441,19 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   if ((rc = dalloc(&P->d_u, (size_t)P->Lg * B))) return fail(rc);
   if (P->B1 > 1 && (rc = dalloc(&P->d_v, (size_t)P->Lg * B))) return fail(rc);
   if ((rc = dalloc(&P->d_records, (size_t)L * P->lay.rec_bytes))) return fail(rc);
-  if (!P->keys_in_smem && (rc = dalloc(&P->d_gkeys, std::max<size_t>(1, P->sel_slots_h.size()) * B)))
-    return fail(rc);
+  {
+    const size_t nsel = std::max<size_t>(1, P->sel_slots_h.size());
+    if ((rc = dalloc(&P->d_keys, nsel * B))) return fail(rc);
+    if ((rc = dalloc(&P->d_hist, nsel * 4096))) return fail(rc);
+    if ((rc = dalloc(&P->d_key_index, (size_t)P->Lg))) return fail(rc);
+    std::vector<int> kidx(P->Lg, -1);
+    for (size_t i = 0; i < P->sel_slots_h.size(); ++i) kidx[P->sel_slots_h[i] - rank * P->Lg] = (int)i;
+    if (cudaMemcpy(P->d_key_index, kidx.data(), P->Lg * sizeof(int), cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemset(P->d_hist, 0, nsel * 4096 * sizeof(uint32_t)) != cudaSuccess) {
+      g_last_cuda_error = (int)cudaGetLastError();
+      return fail(CUSFFT_CUDA);
+    }
+  }
   if ((rc = dalloc(&P->d_hits, (size_t)P->max_hits))) return fail(rc);
   if ((rc = dalloc(&P->d_hit_vals, (size_t)P->max_hits))) return fail(rc);
   if ((rc = dalloc(&P->d_hit_keys, (size_t)P->max_hits))) return fail(rc);
@@ -401,7 +475,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     g_last_cuda_error = (int)cudaGetLastError();
     return fail(CUSFFT_CUDA);
   }
-  if (cudaFuncSetAttribute(k_select, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
+  if (set_fft_attrs() != cudaSuccess ||
+      cudaFuncSetAttribute(k_select, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_vote, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_output, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess) {
     g_last_cuda_error = (int)cudaGetLastError();
@@ -434,33 +509,25 @@ int launch_local(cusfft_plan_t P, const double2* x) {
   mark(P, 1);
   uint8_t* myrec = P->d_records + (int64_t)P->rank * P->Lg * P->lay.rec_bytes;
   const int64_t rec_e = P->lay.rec_bytes / 16;
+  const bool keys = !P->sel_slots_h.empty();
   if (P->B1 > 1) {
-    // pass 1: m = B1 over columns c (stride B2), twiddle e^{-2 pi i c k1 / B}
-    const int m = P->B1;
-    const int nseq = std::max(1, kFftSmemElems / m);
-    const int total = P->Lg * P->B2;
-    k_fft_pass<<<(total + nseq - 1) / nseq, 256, 0, st>>>(P->d_u, P->d_v, P->d_tw, B, P->logB1, nseq, P->B2, total,
-                                                         B, 1, P->B2, B, 1, P->B2, 1);
-    CKL();
-    const int m2 = P->B2;
-    const int nseq2 = std::max(1, kFftSmemElems / m2);
-    const int total2 = P->Lg * P->B1;
-    k_fft_pass<<<(total2 + nseq2 - 1) / nseq2, 256, 0, st>>>(
-        P->d_v, reinterpret_cast<double2*>(myrec), P->d_tw, B, P->logB2, nseq2, P->B1, total2, B, P->B2, 1, rec_e,
-        1, P->B1, 0);
-    CKL();
+    // pass 1: B1-point FFTs over columns c (stride B2), twiddle e^{-2 pi i c k1 / B}
+    FftPassArgs a1{P->d_u, P->d_v, P->d_tw, B, P->logB2, P->Lg * P->B2, B, B, 1, P->B2, 1, P->B2, 1,
+                   nullptr, nullptr, nullptr};
+    CK(launch_fft(P->B1, a1, P->fft_smem1, st));
+    // pass 2: B2-point FFTs of contiguous rows k1, out to u^[k1 + B1 k2] (+ cutoff keys)
+    FftPassArgs a2{P->d_v, reinterpret_cast<double2*>(myrec), P->d_tw, B, P->logB1, P->Lg * P->B1, B, rec_e,
+                   P->B2, 1, 1, P->B1, 0, keys ? P->d_key_index : nullptr, P->d_keys, P->d_hist};
+    CK(launch_fft(P->B2, a2, P->fft_smem2, st));
   } else {
-    const int m = P->B2;
-    const int nseq = std::max(1, kFftSmemElems / m);
-    const int total = P->Lg;
-    k_fft_pass<<<(total + nseq - 1) / nseq, 256, 0, st>>>(P->d_u, reinterpret_cast<double2*>(myrec), P->d_tw, B,
-                                                         P->logB2, nseq, 1, total, B, 0, 1, rec_e, 0, 1, 0);
-    CKL();
+    FftPassArgs a{P->d_u, reinterpret_cast<double2*>(myrec), P->d_tw, B, 0, P->Lg, B, rec_e, 0, 1, 0, 1, 0,
+                  keys ? P->d_key_index : nullptr, P->d_keys, P->d_hist};
+    CK(launch_fft(P->B2, a, P->fft_smem2, st));
   }
   mark(P, 2);
-  if (!P->sel_slots_h.empty()) {
-    k_select<<<(int)P->sel_slots_h.size(), 1024, P->select_smem, st>>>(
-        P->d_records, P->lay, P->d_sel_slots, B, P->num, P->d_gkeys, P->keys_in_smem ? 1 : 0, P->d_flags + 1);
+  if (keys) {
+    k_select<<<(int)P->sel_slots_h.size(), 1024, P->select_smem, st>>>(P->d_records, P->lay, P->d_sel_slots, B,
+                                                                       P->num, P->d_keys, P->d_hist, P->d_flags + 1);
     CKL();
   }
   mark(P, 3);
@@ -482,6 +549,7 @@ int launch_finish(cusfft_plan_t P, int64_t* locs, double2* vals) {
   va.nb = (int)P->nb;
   va.log2nb = P->log2nb;
   va.P = P->vote_P;
+  va.log2P = ilog2(P->vote_P);
   va.nmask = (uint32_t)(P->n - 1);
   va.hits = P->d_hits;
   va.hit_count = reinterpret_cast<unsigned*>(P->d_flags);
@@ -506,7 +574,7 @@ int launch_finish(cusfft_plan_t P, int64_t* locs, double2* vals) {
   ea.hit_vals = P->d_hit_vals;
   ea.hit_keys = P->d_hit_keys;
   ea.per_loop = P->d_per_loop;
-  k_estimate<<<P->est_grid, 128, 0, st>>>(ea);
+  k_estimate<<<P->est_grid, 256, 0, st>>>(ea);
   CKL();
   mark(P, 5);
   k_output<<<1, 1024, P->output_smem, st>>>(P->d_hits, reinterpret_cast<const unsigned*>(P->d_flags), P->max_hits,
@@ -514,6 +582,43 @@ int launch_finish(cusfft_plan_t P, int64_t* locs, double2* vals) {
                                             P->d_flags + 1);
   CKL();
   mark(P, 6);
+  return CUSFFT_SUCCESS;
+}
+
+
+// Run `body` (which enqueues on P->stream) either directly or through a cached
+// CUDA graph captured on a plan-owned stream and launched on the caller's
+// stream.  Timing mode always launches directly (events between kernels).
+template <class F>
+int run_graphed(cusfft_plan_t P, cusfft_plan_s::GraphEntry& g, const void* a, const void* b, const void* c,
+                F&& body) {
+  if (!P->use_graph || P->timing) return body();
+  if (!(g.exec && g.a == a && g.b == b && g.c == c)) {
+    if (g.exec) {
+      cudaGraphExecDestroy(g.exec);
+      g.exec = nullptr;
+    }
+    if (!P->cap_stream) CK(cudaStreamCreateWithFlags(&P->cap_stream, cudaStreamNonBlocking));
+    CK(cudaStreamBeginCapture(P->cap_stream, cudaStreamCaptureModeThreadLocal));
+    cudaStream_t user = P->stream;
+    P->stream = P->cap_stream;
+    const int rc = body();
+    cudaGraph_t graph = nullptr;
+    const cudaError_t ce = cudaStreamEndCapture(P->cap_stream, &graph);
+    P->stream = user;
+    if (rc != CUSFFT_SUCCESS) {
+      if (graph) cudaGraphDestroy(graph);
+      return rc;
+    }
+    CK(ce);
+    const cudaError_t ie = cudaGraphInstantiate(&g.exec, graph, 0);
+    cudaGraphDestroy(graph);
+    CK(ie);
+    g.a = a;
+    g.b = b;
+    g.c = c;
+  }
+  CK(cudaGraphLaunch(g.exec, P->stream));
   return CUSFFT_SUCCESS;
 }
 
@@ -603,14 +708,16 @@ int cusfft_execute_local(cusfft_plan_t plan, const void* d_x) {
   if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
   if (!d_x) return CUSFFT_NULL_PTR;
   DeviceGuard g(plan->device);
-  return launch_local(plan, reinterpret_cast<const double2*>(d_x));
+  return run_graphed(plan, plan->g_local, d_x, nullptr, nullptr,
+                     [&] { return launch_local(plan, reinterpret_cast<const double2*>(d_x)); });
 }
 
 int cusfft_execute_finish(cusfft_plan_t plan, int64_t* d_locs, void* d_vals) {
   if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
   if (!d_locs || !d_vals) return CUSFFT_NULL_PTR;
   DeviceGuard g(plan->device);
-  return launch_finish(plan, d_locs, reinterpret_cast<double2*>(d_vals));
+  return run_graphed(plan, plan->g_finish, d_locs, d_vals, nullptr,
+                     [&] { return launch_finish(plan, d_locs, reinterpret_cast<double2*>(d_vals)); });
 }
 
 int cusfft_execute(cusfft_plan_t plan, const void* d_x, int64_t* d_locs, void* d_vals) {
@@ -618,9 +725,11 @@ int cusfft_execute(cusfft_plan_t plan, const void* d_x, int64_t* d_locs, void* d
   if (!d_x || !d_locs || !d_vals) return CUSFFT_NULL_PTR;
   if (plan->world != 1) return CUSFFT_INVALID_LOOPS;
   DeviceGuard g(plan->device);
-  int rc = launch_local(plan, reinterpret_cast<const double2*>(d_x));
-  if (rc) return rc;
-  return launch_finish(plan, d_locs, reinterpret_cast<double2*>(d_vals));
+  return run_graphed(plan, plan->g_full, d_x, d_locs, d_vals, [&] {
+    int rc = launch_local(plan, reinterpret_cast<const double2*>(d_x));
+    if (rc) return rc;
+    return launch_finish(plan, d_locs, reinterpret_cast<double2*>(d_vals));
+  });
 }
 
 int cusfft_status(cusfft_plan_t plan) {
@@ -647,8 +756,12 @@ int cusfft_execute_host(cusfft_plan_t plan, const void* h_x, int64_t* h_locs, vo
   }
   cudaStream_t st = plan->stream;
   CK(cudaMemcpyAsync(plan->d_xbuf, h_x, (size_t)plan->n * 16, cudaMemcpyHostToDevice, st));
-  if ((rc = launch_local(plan, plan->d_xbuf))) return rc;
-  if ((rc = launch_finish(plan, plan->d_locs_buf, plan->d_vals_buf))) return rc;
+  rc = run_graphed(plan, plan->g_full, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf, [&] {
+    int r = launch_local(plan, plan->d_xbuf);
+    if (r) return r;
+    return launch_finish(plan, plan->d_locs_buf, plan->d_vals_buf);
+  });
+  if (rc) return rc;
   CK(cudaMemcpyAsync(h_locs, plan->d_locs_buf, (size_t)plan->k * 8, cudaMemcpyDeviceToHost, st));
   CK(cudaMemcpyAsync(h_vals, plan->d_vals_buf, (size_t)plan->k * 16, cudaMemcpyDeviceToHost, st));
   return cusfft_status(plan);

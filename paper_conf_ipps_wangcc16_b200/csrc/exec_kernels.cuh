@@ -1,12 +1,13 @@
 // exec_kernels.cuh — the timed hot path:
 //   k_fold      Steps 1+2  permutation + filter + fold into B buckets
-//   k_fft_pass  Step 3     batched B-point FFT (one or two smem passes)
+//   k_fft       Step 3     batched B-point FFT (fft.cuh; one or two passes)
 //   k_select    Step 4     exact top-num cutoff per location loop
 //   k_vote      Step 5     reverse hash + vote
 //   k_estimate  Step 6     per-loop estimates and their median
 //   k_output    output     top-k hits by |val|^2, sorted by location
 #pragma once
 #include "common.cuh"
+#include "fft.cuh"
 
 namespace cusfft {
 
@@ -59,94 +60,13 @@ __global__ void __launch_bounds__(256) k_fold(const double2* __restrict__ x, con
 }
 
 // ---------------------------------------------------------------------------
-// Step 3 (L87, batched over loops as in L232): one pass of a four-step FFT.
-// A CTA transforms NSEQ sequences of length m = 2^logm held in shared memory
-// (radix-2 DIT after a bit-reversed load).  Sequence q = (slot l, column col):
-//   element e at in [l*in_ls + col*in_cs + e*in_es],
-//   result  e at out[l*out_ls + col*out_cs + e*out_es],
-// optionally multiplied by tw[(col * e) mod B] = e^{-2 pi i col e / B}.
-// Pass 1 (B = B1 B2, m = B1): in_cs = 1, in_es = B2, twiddle on.
-// Pass 2 (m = B2): in_cs = B2, in_es = 1, out_cs = 1, out_es = B1.
-// A single pass (B1 = 1) is a plain B-point FFT per slot.
-// ---------------------------------------------------------------------------
-constexpr int kFftSmemElems = 2048;
-
-__global__ void __launch_bounds__(256) k_fft_pass(const double2* __restrict__ in, double2* __restrict__ out,
-                                                  const double2* __restrict__ tw, int B, int logm, int nseq_cta,
-                                                  int seq_per_slot, int total_seq, int64_t in_ls, int in_cs,
-                                                  int in_es, int64_t out_ls, int out_cs, int out_es, int twiddle) {
-  __shared__ double2 S[kFftSmemElems];
-  const int m = 1 << logm;
-  const int q0 = blockIdx.x * nseq_cta;
-  const int nelem = nseq_cta * m;
-  // load (coalesced along whichever stride is 1), bit-reversed into smem
-  const bool col_fast_in = (in_cs == 1);
-  for (int t = threadIdx.x; t < nelem; t += blockDim.x) {
-    int sq, e;
-    if (col_fast_in) {
-      sq = t % nseq_cta;
-      e = t / nseq_cta;
-    } else {
-      sq = t / m;
-      e = t % m;
-    }
-    const int q = q0 + sq;
-    if (q < total_seq) {
-      const int l = q / seq_per_slot, col = q % seq_per_slot;
-      const int rev = logm ? (int)(__brev((unsigned)e) >> (32 - logm)) : 0;
-      S[sq * m + rev] = in[(int64_t)l * in_ls + (int64_t)col * in_cs + (int64_t)e * in_es];
-    }
-  }
-  __syncthreads();
-  const int twstride0 = B >> 1;  // tw index step for len = 2
-  for (int s = 1; s <= logm; ++s) {
-    const int half = 1 << (s - 1);
-    const int tstride = twstride0 >> (s - 1);  // B / len
-    for (int bf = threadIdx.x; bf < (nelem >> 1); bf += blockDim.x) {
-      const int sq = bf >> (logm - 1);
-      const int k = bf & ((m >> 1) - 1);
-      const int pos = k & (half - 1);
-      const int i0 = ((k >> (s - 1)) << s) + pos;
-      const int i1 = i0 + half;
-      const double2 wv = tw[pos * tstride];
-      const double2 a = S[sq * m + i0];
-      const double2 b = S[sq * m + i1];
-      const double2 bw = make_double2(b.x * wv.x - b.y * wv.y, b.x * wv.y + b.y * wv.x);
-      S[sq * m + i0] = make_double2(a.x + bw.x, a.y + bw.y);
-      S[sq * m + i1] = make_double2(a.x - bw.x, a.y - bw.y);
-    }
-    __syncthreads();
-  }
-  const bool col_fast_out = (out_cs == 1);
-  for (int t = threadIdx.x; t < nelem; t += blockDim.x) {
-    int sq, e;
-    if (col_fast_out) {
-      sq = t % nseq_cta;
-      e = t / nseq_cta;
-    } else {
-      sq = t / m;
-      e = t % m;
-    }
-    const int q = q0 + sq;
-    if (q < total_seq) {
-      const int l = q / seq_per_slot, col = q % seq_per_slot;
-      double2 v = S[sq * m + e];
-      if (twiddle) {
-        const double2 wv = tw[((int64_t)col * e) & (B - 1)];
-        v = make_double2(v.x * wv.x - v.y * wv.y, v.x * wv.y + v.y * wv.x);
-      }
-      out[(int64_t)l * out_ls + (int64_t)col * out_cs + (int64_t)e * out_es] = v;
-    }
-  }
-}
-
-// ---------------------------------------------------------------------------
 // Record layout of one slot in the exchange buffer:
 //   [u^ : B x double2][bitmap : B/32 x u32][J : num x int32], 256-B aligned.
 // ---------------------------------------------------------------------------
 struct RecLayout {
   int64_t rec_bytes, off_bitmap, off_J;
 };
+
 
 struct KeysSrc {
   const uint64_t* keys;
@@ -156,56 +76,135 @@ struct KeysSrc {
   }
 };
 
-// Step 4 (L89, Alg. 3): J_r = the num buckets of largest
-// |u^|^2 = re*re + im*im (ties to the smaller bucket), as a bitmap and as an
-// ascending list.  One CTA of 1024 threads per location slot of this rank.
-// Dynamic smem: 4096 u32 histogram + 64 ints + (keys_in_smem ? B u64 : 0).
+struct PairSrc {  // (key, index) pairs; the index is the tie-break
+  const uint64_t* keys;
+  const int* idx;
+  __device__ __forceinline__ void get(int i, uint64_t& hi, uint32_t& lo) const {
+    hi = keys[i];
+    lo = ~(uint32_t)idx[i];
+  }
+};
+
+// ---------------------------------------------------------------------------
+// Step 4 (L89, Alg. 3; the linear-time selection of §V.B,
+// made exact): J_r = the num buckets of largest |u^|^2 = re*re + im*im, ties
+// to the smaller bucket, as a bitmap and an ascending list.  One CTA of 1024
+// threads per location slot of this rank.
+//  1. the FFT epilogue already counted keys per top-12-bit digit: a block scan
+//     of that histogram gives the boundary digit d0 and the count above it;
+//  2. one pass over the B keys: digit > d0 -> selected, digit == d0 -> smem
+//     candidate list;
+//  3. exact 96-bit radix select (key, ~bucket) among the candidates.
+// Falls back to a full radix select over all keys when the boundary bin holds
+// more than kSelCap candidates.  Resets the histogram for the next execution.
+// Dynamic smem: 4096 u32 hist + 64 int + kSelCap x (u64 + int).
+// ---------------------------------------------------------------------------
+constexpr int kSelCap = 4096;
+
 __global__ void __launch_bounds__(1024) k_select(uint8_t* __restrict__ records, RecLayout lay,
                                                  const int* __restrict__ sel_slots, int B, int num,
-                                                 uint64_t* __restrict__ gkeys, int keys_in_smem,
+                                                 const uint64_t* __restrict__ gkeys, uint32_t* __restrict__ ghist,
                                                  int* __restrict__ status) {
   extern __shared__ __align__(16) uint8_t smem[];
   uint32_t* hist = reinterpret_cast<uint32_t*>(smem);
   int* sm = reinterpret_cast<int*>(smem + 4096 * 4);
-  uint64_t* skeys = reinterpret_cast<uint64_t*>(smem + 4096 * 4 + 64 * 4);
-  const int slot = sel_slots[blockIdx.x];
-  uint8_t* rec = records + (int64_t)slot * lay.rec_bytes;
-  const double2* uhat = reinterpret_cast<const double2*>(rec);
+  uint64_t* ckey = reinterpret_cast<uint64_t*>(smem + 4096 * 4 + 64 * 4);
+  int* cidx = reinterpret_cast<int*>(ckey + kSelCap);
+  const int tid = threadIdx.x;
+  const int sel = blockIdx.x;
+  uint8_t* rec = records + (int64_t)sel_slots[sel] * lay.rec_bytes;
   uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + lay.off_bitmap);
   int* J = reinterpret_cast<int*>(rec + lay.off_J);
-  uint64_t* keys = keys_in_smem ? skeys : gkeys + (int64_t)blockIdx.x * B;
-  for (int i = threadIdx.x; i < B; i += blockDim.x) {
-    const double2 v = uhat[i];
-    const double m2 = __dadd_rn(__dmul_rn(v.x, v.x), __dmul_rn(v.y, v.y));
-    keys[i] = (uint64_t)__double_as_longlong(m2);
+  const uint64_t* keys = gkeys + (int64_t)sel * B;
+  uint32_t* gh = ghist + (int64_t)sel * 4096;
+  const int words = (B + 31) >> 5;
+
+  // 1. boundary digit from the histogram (thread t owns bins 4095-4t .. 4092-4t)
+  const int base = 4095 - 4 * tid;
+  const int c0 = gh[base], c1 = gh[base - 1], c2 = gh[base - 2], c3 = gh[base - 3];
+  const int mine = c0 + c1 + c2 + c3;
+  int total;
+  const int ex = block_excl_scan<1024>(mine, &total, sm);
+  if (ex < num && num <= ex + mine) {
+    int cum = ex, d, cnt;
+    if (cum + c0 >= num) {
+      d = base; cnt = c0;
+    } else if ((cum += c0) + c1 >= num) {
+      d = base - 1; cnt = c1;
+    } else if ((cum += c1) + c2 >= num) {
+      d = base - 2; cnt = c2;
+    } else {
+      cum += c2; d = base - 3; cnt = c3;
+    }
+    sm[32] = d; sm[33] = cum; sm[34] = cnt;
+  }
+  gh[base] = 0; gh[base - 1] = 0; gh[base - 2] = 0; gh[base - 3] = 0;  // self-reset
+  for (int w = tid; w < words; w += 1024) bitmap[w] = 0;
+  if (tid == 0) sm[40] = 0;
+  __syncthreads();
+  const uint32_t d0 = (uint32_t)sm[32];
+  const int above = sm[33], cnt0 = sm[34];
+  const int k2 = num - above;  // 1 <= k2 <= cnt0
+  const bool whole_bin = (k2 == cnt0);
+  // 2. one pass over the keys, 16 loads in flight per thread
+  for (int i0 = 0; i0 < B; i0 += 16 * 1024) {
+    uint64_t kb[16];
+#pragma unroll
+    for (int u = 0; u < 16; ++u) {
+      const int i = i0 + u * 1024 + tid;
+      kb[u] = i < B ? __ldg(keys + i) : 0ull;
+    }
+#pragma unroll
+    for (int u = 0; u < 16; ++u) {
+      const int i = i0 + u * 1024 + tid;
+      if (i >= B) continue;
+      const uint32_t d = (uint32_t)(kb[u] >> 51) & 0xFFFu;
+      if (d > d0 || (d == d0 && whole_bin)) {
+        atomicOr(&bitmap[i >> 5], 1u << (i & 31));
+      } else if (d == d0) {
+        const int pos = atomicAdd(&sm[40], 1);
+        if (pos < kSelCap) {
+          ckey[pos] = kb[u];
+          cidx[pos] = i;
+        }
+      }
+    }
   }
   __syncthreads();
-  const Prefix96 p = block_radix_select(KeysSrc{keys}, B, num, hist, sm);
-  // bitmap words: thread t owns words [t*wpt, (t+1)*wpt)
-  const int words = (B + 31) >> 5;
+  if (!whole_bin) {
+    const int nc = sm[40];
+    if (nc <= kSelCap) {
+      const Prefix96 p = block_radix_select(PairSrc{ckey, cidx}, nc, k2, hist, sm);
+      for (int c = tid; c < nc; c += 1024)
+        if (ge96(p, ckey[c], ~(uint32_t)cidx[c])) atomicOr(&bitmap[cidx[c] >> 5], 1u << (cidx[c] & 31));
+    } else {  // crowded boundary bin: exact select over all keys
+      const Prefix96 p = block_radix_select(KeysSrc{keys}, B, num, hist, sm);
+      for (int w = tid; w < words; w += 1024) {
+        uint32_t bits = 0;
+        for (int b = 0; b < 32; ++b) {
+          const int i = w * 32 + b;
+          if (i < B && ge96(p, keys[i], ~(uint32_t)i)) bits |= 1u << b;
+        }
+        bitmap[w] = bits;
+      }
+    }
+  }
+  __syncthreads();
+  // 3. ascending winner list from the bitmap
   const int wpt = (words + 1023) >> 10;
   int cnt = 0;
-  for (int wi = threadIdx.x * wpt; wi < min(words, (threadIdx.x + 1) * wpt); ++wi) {
-    uint32_t bits = 0;
-    for (int b = 0; b < 32; ++b) {
-      const int i = wi * 32 + b;
-      if (i < B && ge96(p, keys[i], ~(uint32_t)i)) bits |= 1u << b;
-    }
-    bitmap[wi] = bits;
-    cnt += __popc(bits);
-  }
-  int total;
+  for (int w = tid * wpt; w < min(words, (tid + 1) * wpt); ++w) cnt += __popc(bitmap[w]);
   int pos = block_excl_scan<1024>(cnt, &total, sm);
-  for (int wi = threadIdx.x * wpt; wi < min(words, (threadIdx.x + 1) * wpt); ++wi) {
-    uint32_t bits = bitmap[wi];
+  for (int w = tid * wpt; w < min(words, (tid + 1) * wpt); ++w) {
+    uint32_t bits = bitmap[w];
     while (bits) {
       const int b = __ffs(bits) - 1;
       bits &= bits - 1;
-      if (pos < num) J[pos] = wi * 32 + b;
+      if (pos < num) J[pos] = w * 32 + b;
       ++pos;
     }
   }
-  if (threadIdx.x == 0 && total != num) atomicOr(status + 1, 1);
+  if (tid == 0 && total != num) atomicOr(status + 1, 1);
 }
 
 // ---------------------------------------------------------------------------
@@ -213,10 +212,11 @@ __global__ void __launch_bounds__(1024) k_select(uint8_t* __restrict__ records, 
 // is Alg. 4's range [ceil((J-1/2) nb), ceil((J+1/2) nb)).  A frequency with
 // >= T of L_loc votes is selected in at least one of the first L_loc - T + 1
 // location loops, so candidates f = a_{q0} p are enumerated only from those
-// loops' preimage ranges; f is counted at the first such loop it is selected
-// in (q < q0 bits must be clear) and then probed against the later loops'
-// bitmaps, stopping once more than L_loc - T loops have missed.
-// Dynamic smem: L_loc * B/32 u32 bitmaps.
+// loops' preimage ranges, and f is counted at the first loop q0 that selects
+// it: it needs T-1 votes among the loops after q0 (probed first: a random
+// candidate is rejected after L_loc - T - q0 + 1 misses) and no vote before
+// q0 (probed last, for the rare survivors).
+// Dynamic smem: L_loc * ceil(B/32) u32 bitmaps.
 // ---------------------------------------------------------------------------
 struct VoteArgs {
   const uint8_t* records;
@@ -224,7 +224,7 @@ struct VoteArgs {
   const int* loc_slots;  // [L_loc] slot of each location loop, in vote order
   const uint32_t* loc_sigma;
   const uint32_t* loc_a;
-  int Lloc, T, num, B, nb, log2nb, P;
+  int Lloc, T, num, B, nb, log2nb, P, log2P;
   uint32_t nmask;
   int* hits;
   unsigned* hit_count;
@@ -235,71 +235,90 @@ __global__ void __launch_bounds__(256) k_vote(VoteArgs A) {
   extern __shared__ __align__(16) uint8_t smem[];
   uint32_t* bm = reinterpret_cast<uint32_t*>(smem);
   __shared__ uint32_t ssig[64];
-  const int words = A.B >> 5;
-  for (int q = 0; q < A.Lloc; ++q) {
-    const uint32_t* src = reinterpret_cast<const uint32_t*>(A.records + (int64_t)A.loc_slots[q] * A.lay.rec_bytes +
-                                                             A.lay.off_bitmap);
-    for (int i = threadIdx.x; i < words; i += blockDim.x) bm[q * words + i] = src[i];
+  const int words = (A.B + 31) >> 5;
+  if ((words & 3) == 0) {  // 16-B vector loads, 8 in flight per thread
+    const int v4 = words >> 2, tot = A.Lloc * v4;
+    uint4* bm4 = reinterpret_cast<uint4*>(bm);
+    for (int i0 = 0; i0 < tot; i0 += 8 * (int)blockDim.x) {
+      uint4 tmp[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const int i = i0 + u * blockDim.x + threadIdx.x;
+        if (i < tot) {
+          const int q = i / v4, w = i - q * v4;
+          tmp[u] = __ldg(reinterpret_cast<const uint4*>(A.records + (int64_t)A.loc_slots[q] * A.lay.rec_bytes +
+                                                        A.lay.off_bitmap) + w);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const int i = i0 + u * blockDim.x + threadIdx.x;
+        if (i < tot) bm4[i] = tmp[u];
+      }
+    }
+  } else {
+    for (int q = 0; q < A.Lloc; ++q) {
+      const uint32_t* src = reinterpret_cast<const uint32_t*>(A.records + (int64_t)A.loc_slots[q] * A.lay.rec_bytes +
+                                                               A.lay.off_bitmap);
+      for (int i = threadIdx.x; i < words; i += blockDim.x) bm[q * words + i] = src[i];
+    }
   }
   if (threadIdx.x < A.Lloc) ssig[threadIdx.x] = A.loc_sigma[threadIdx.x];
   __syncthreads();
   const int lane = threadIdx.x & 31;
-  const int cpj = A.nb / A.P;  // chunks per bucket
-  const int64_t per_q = (int64_t)A.num * cpj;
-  const int64_t items = (int64_t)(A.Lloc - A.T + 1) * per_q;
+  const int log_cpj = A.log2nb - A.log2P;  // chunks per bucket = nb / P
+  const int per_q = A.num << log_cpj;
+  const int items = (A.Lloc - A.T + 1) * per_q;
   const uint32_t half = (uint32_t)(A.nb >> 1);
-  // uniform trip count per warp so that ballots see every lane
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  const int64_t start = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  const int64_t warp_start = start - lane;
-  for (int64_t it0 = warp_start; it0 < items; it0 += stride) {
-    const int64_t it = it0 + lane;
+  const int stride = gridDim.x * blockDim.x;
+  const int warp_start = blockIdx.x * blockDim.x + threadIdx.x - lane;
+  for (int it0 = warp_start; it0 < items; it0 += stride) {
+    const int it = it0 + lane;
     const bool valid_item = it < items;
     int q0 = 0;
     uint32_t a = 0, p = 0;
     if (valid_item) {
-      q0 = (int)(it / per_q);
-      const int64_t rem = it - (int64_t)q0 * per_q;
-      const int jidx = (int)(rem / cpj);
-      const int chunk = (int)(rem - (int64_t)jidx * cpj);
+      q0 = it / per_q;
+      const int rem = it - q0 * per_q;
+      const int jidx = rem >> log_cpj;
+      const int chunk = rem & ((1 << log_cpj) - 1);
       const int* Jl = reinterpret_cast<const int*>(A.records + (int64_t)A.loc_slots[q0] * A.lay.rec_bytes +
                                                    A.lay.off_J);
       const uint32_t Jv = (uint32_t)Jl[jidx];
       p = (Jv * (uint32_t)A.nb - half + (uint32_t)(chunk * A.P)) & A.nmask;
       a = A.loc_a[q0];
     }
-    for (int t = 0; t < A.P; ++t) {
+    const int allowed = A.Lloc - A.T - q0;
+    uint32_t f = (a * p) & A.nmask;
+    for (int t = 0; t < A.P; ++t, f = (f + a) & A.nmask) {
       bool hit = false;
-      uint32_t f = 0;
       if (valid_item) {
-        f = (a * ((p + (uint32_t)t) & A.nmask)) & A.nmask;
-        bool fresh = true;
-        for (int q = 0; q < q0; ++q) {
+        int miss = 0;
+        bool ok = true;
+        for (int q = q0 + 1; q < A.Lloc; ++q) {
           const uint32_t b = ((ssig[q] * f + half) & A.nmask) >> A.log2nb;
-          if ((bm[q * words + (b >> 5)] >> (b & 31)) & 1u) {
-            fresh = false;
+          if (!((bm[q * words + (b >> 5)] >> (b & 31)) & 1u) && ++miss > allowed) {
+            ok = false;
             break;
           }
         }
-        if (fresh) {
-          const int allowed = A.Lloc - A.T - q0;
-          int votes = 1, miss = 0;
-          for (int q = q0 + 1; q < A.Lloc; ++q) {
+        if (ok) {
+          for (int q = 0; q < q0; ++q) {
             const uint32_t b = ((ssig[q] * f + half) & A.nmask) >> A.log2nb;
             if ((bm[q * words + (b >> 5)] >> (b & 31)) & 1u) {
-              ++votes;
-            } else if (++miss > allowed) {
+              ok = false;
               break;
             }
           }
-          hit = votes >= A.T;
         }
+        hit = ok;
       }
       const unsigned ball = __ballot_sync(kFull, hit);
       if (ball) {
         unsigned base = 0;
-        if (lane == __ffs(ball) - 1) base = atomicAdd(A.hit_count, (unsigned)__popc(ball));
-        base = __shfl_sync(kFull, base, __ffs(ball) - 1);
+        const int leader = __ffs(ball) - 1;
+        if (lane == leader) base = atomicAdd(A.hit_count, (unsigned)__popc(ball));
+        base = __shfl_sync(kFull, base, leader);
         if (hit) {
           const unsigned slot = base + __popc(ball & ((1u << lane) - 1));
           if ((int)slot < A.max_hits) A.hits[slot] = (int)f;
@@ -310,10 +329,11 @@ __global__ void __launch_bounds__(256) k_vote(VoteArgs A) {
 }
 
 // ---------------------------------------------------------------------------
-// Step 6 (L95, Alg. 5).  For hit f and every loop (slot) l:
-//   p = sigma_l f mod n, h = p / nb, d = p mod nb; if d > nb/2: h = h+1 mod B, d -= nb;
-//   v_l = u^_l[h] * e^{-2 pi i tau_l f / n} / G^(-d)
-// then val = median(Re v) + i median(Im v), rank (L-1)/2 ascending.
+// Step 6 (L95, Alg. 5), one warp per hit, one lane per loop (slot).
+// For hit f and loop l:  p = sigma_l f mod n, h = p / nb, d = p mod nb;
+//   if d > nb/2: h = h+1 mod B, d -= nb;
+//   v_l = u^_l[h] * e^{-2 pi i tau_l f / n} / G^(-d);
+// val = (element of rank (L-1)/2 of Re v) + i (same of Im v), ties by loop.
 // ---------------------------------------------------------------------------
 struct EstArgs {
   const uint8_t* records;
@@ -334,56 +354,83 @@ struct EstArgs {
 
 constexpr int kMaxLoops = 64;
 
-__device__ __forceinline__ double rank_select(const double* v, int L, int med) {
-  for (int i = 0; i < L; ++i) {
-    int r = 0;
-    for (int j = 0; j < L; ++j) r += (v[j] < v[i]) || (v[j] == v[i] && j < i);
-    if (r == med) return v[i];
+__device__ __forceinline__ double2 loop_estimate(const EstArgs& A, int l, uint32_t f) {
+  const SlotParam sp = A.slots[l];
+  const uint32_t p = (sp.sigma * f) & A.nmask;
+  int hb = (int)(p >> A.log2nb);
+  int d = (int)(p & (uint32_t)(A.nb - 1));
+  if (d > (A.nb >> 1)) {
+    hb = (hb + 1) & (A.B - 1);
+    d -= A.nb;
   }
-  return v[0];
+  const double2 g = __ldg(A.ghat + (A.nb >> 1) - d);  // G^(-d)
+  const double2 b = reinterpret_cast<const double2*>(A.records + (int64_t)l * A.lay.rec_bytes)[hb];
+  const uint32_t tph = (sp.tau * f) & A.nmask;
+  double sn, cs;
+  sincospi(2.0 * (double)tph / A.n, &sn, &cs);
+  const double zr = b.x * cs + b.y * sn;  // b * e^{-i phi}
+  const double zi = b.y * cs - b.x * sn;
+  const double den = g.x * g.x + g.y * g.y;
+  return make_double2((zr * g.x + zi * g.y) / den, (zi * g.x - zr * g.y) / den);
 }
 
-__global__ void __launch_bounds__(128) k_estimate(EstArgs A) {
+// Element of rank `med` among the L values held as (lane: a0 = slot lane,
+// a1 = slot lane + 32); ties ordered by slot.  Returns it on every lane.
+__device__ __forceinline__ double warp_rank_select(double a0, double a1, int L, int med) {
+  const int lane = threadIdx.x & 31;
+  int r0 = 0, r1 = 0;
+  const int L0 = min(L, 32);
+  for (int j = 0; j < L0; ++j) {
+    const double v = __shfl_sync(kFull, a0, j);
+    r0 += (v < a0) || (v == a0 && j < lane);
+    r1 += (v < a1) || (v == a1);  // slot j < 32 <= slot of a1
+  }
+  for (int j = 32; j < L; ++j) {
+    const double v = __shfl_sync(kFull, a1, j - 32);
+    r0 += (v < a0);
+    r1 += (v < a1) || (v == a1 && j < lane + 32);
+  }
+  const bool h0 = lane < L0 && r0 == med;
+  const bool h1 = lane + 32 < L && r1 == med;
+  const unsigned b = __ballot_sync(kFull, h0 || h1);
+  const int src = __ffs(b) - 1;
+  const double mine = h0 ? a0 : a1;
+  return __shfl_sync(kFull, mine, src);
+}
+
+__global__ void __launch_bounds__(256) k_estimate(EstArgs A) {
   const int H = min((int)*A.hit_count, A.max_hits);
-  double re[kMaxLoops], im[kMaxLoops];
-  for (int h = blockIdx.x * blockDim.x + threadIdx.x; h < H; h += gridDim.x * blockDim.x) {
+  const int lane = threadIdx.x & 31;
+  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int nwarps = (gridDim.x * blockDim.x) >> 5;
+  const int med = (A.L - 1) >> 1;
+  for (int h = warp; h < H; h += nwarps) {
     const uint32_t f = (uint32_t)A.hits[h];
-    for (int l = 0; l < A.L; ++l) {
-      const SlotParam sp = A.slots[l];
-      const uint32_t p = (sp.sigma * f) & A.nmask;
-      int hb = (int)(p >> A.log2nb);
-      int d = (int)(p & (uint32_t)(A.nb - 1));
-      if (d > (A.nb >> 1)) {
-        hb = (hb + 1) & (A.B - 1);
-        d -= A.nb;
-      }
-      const double2 g = A.ghat[(A.nb >> 1) - d];  // G^(-d)
-      const double2 b = reinterpret_cast<const double2*>(A.records + (int64_t)l * A.lay.rec_bytes)[hb];
-      const uint32_t tph = (sp.tau * f) & A.nmask;
-      double sn, cs;
-      sincospi(2.0 * (double)tph / A.n, &sn, &cs);
-      // b * e^{-i phi} with e^{-i phi} = cs - i sn
-      const double zr = b.x * cs + b.y * sn;
-      const double zi = b.y * cs - b.x * sn;
-      // (zr + i zi) / (g.x + i g.y)
-      const double den = g.x * g.x + g.y * g.y;
-      re[l] = (zr * g.x + zi * g.y) / den;
-      im[l] = (zi * g.x - zr * g.y) / den;
-      if (A.per_loop) A.per_loop[(int64_t)h * A.L + l] = make_double2(re[l], im[l]);
+    double2 v0 = make_double2(0.0, 0.0), v1 = make_double2(0.0, 0.0);
+    if (lane < A.L) v0 = loop_estimate(A, lane, f);
+    if (lane + 32 < A.L) v1 = loop_estimate(A, lane + 32, f);
+    if (A.per_loop) {
+      if (lane < A.L) A.per_loop[(int64_t)h * A.L + lane] = v0;
+      if (lane + 32 < A.L) A.per_loop[(int64_t)h * A.L + lane + 32] = v1;
     }
-    const int med = (A.L - 1) >> 1;
-    const double vr = rank_select(re, A.L, med);
-    const double vi = rank_select(im, A.L, med);
-    A.hit_vals[h] = make_double2(vr, vi);
-    A.hit_keys[h] = (uint64_t)__double_as_longlong(__dadd_rn(__dmul_rn(vr, vr), __dmul_rn(vi, vi)));
+    const double vr = warp_rank_select(v0.x, v1.x, A.L, med);
+    const double vi = warp_rank_select(v0.y, v1.y, A.L, med);
+    if (lane == 0) {
+      A.hit_vals[h] = make_double2(vr, vi);
+      A.hit_keys[h] = (uint64_t)__double_as_longlong(__dadd_rn(__dmul_rn(vr, vr), __dmul_rn(vi, vi)));
+    }
   }
 }
 
 // ---------------------------------------------------------------------------
 // Output: the k hits of largest |val|^2 (ties to the smaller f), written in
-// ascending f; pads loc = -1, val = 0.  One CTA of 1024 threads.
-// Dynamic smem: 4096 u32 hist + 64 ints + 2 * kp2 ints (sort buffer).
+// ascending f; pads loc = -1, val = 0.  One CTA of 1024 threads.  Hits are
+// staged in smem when H <= kOutCap; the sort is a bitonic network (warp
+// shuffles below stride 32) over 64-bit (f << 32 | hit index) keys.
+// Dynamic smem: 4096 u32 hist + 64 ints + kOutCap x (u64 + int) + kp2 x u64.
 // ---------------------------------------------------------------------------
+constexpr int kOutCap = 8192;
+
 struct HitSrc {
   const uint64_t* keys;
   const int* hits;
@@ -401,53 +448,80 @@ __global__ void __launch_bounds__(1024) k_output(const int* __restrict__ hits, c
   extern __shared__ __align__(16) uint8_t smem[];
   uint32_t* hist = reinterpret_cast<uint32_t*>(smem);
   int* sm = reinterpret_cast<int*>(smem + 4096 * 4);
-  int* sf = reinterpret_cast<int*>(smem + 4096 * 4 + 64 * 4);
-  int* si = sf + kp2;
-  const int H = min((int)*hit_count, max_hits);
-  if (threadIdx.x == 0 && (int)*hit_count > max_hits) atomicOr(status, 1);
+  uint64_t* skey = reinterpret_cast<uint64_t*>(smem + 4096 * 4 + 64 * 4);
+  int* shit = reinterpret_cast<int*>(skey + kOutCap);
+  uint64_t* sort = reinterpret_cast<uint64_t*>(shit + kOutCap);
+  const int tid = threadIdx.x;
+  const unsigned hc = *hit_count;
+  const int H = min((int)hc, max_hits);
+  if (tid == 0 && (int)hc > max_hits) atomicOr(status, 1);
   const int K = min(k, H);
+  const bool staged = H <= kOutCap;
+  if (staged) {
+    for (int i = tid; i < H; i += 1024) {
+      skey[i] = hit_keys[i];
+      shit[i] = hits[i];
+    }
+  }
+  if (tid == 0) sm[40] = 0;
+  for (int i = tid; i < kp2; i += 1024) sort[i] = ~0ull;
+  __syncthreads();
+  const uint64_t* kk = staged ? skey : hit_keys;
+  const int* hh = staged ? shit : hits;
   Prefix96 p{0, 0, 0, 0};  // matches everything
-  if (H > K) p = block_radix_select(HitSrc{hit_keys, hits}, H, K, hist, sm);
-  if (threadIdx.x == 0) sm[40] = 0;
-  for (int i = threadIdx.x; i < kp2; i += blockDim.x) {
-    sf[i] = 0x7FFFFFFF;
-    si[i] = -1;
-  }
-  __syncthreads();
-  for (int i = threadIdx.x; i < H; i += blockDim.x) {
-    if (ge96(p, hit_keys[i], ~(uint32_t)hits[i])) {
+  if (H > K) p = block_radix_select(HitSrc{kk, hh}, H, K, hist, sm);
+  for (int i = tid; i < H; i += 1024) {
+    const int f = hh[i];
+    if (ge96(p, kk[i], ~(uint32_t)f)) {
       const int pos = atomicAdd(&sm[40], 1);
-      if (pos < kp2) {
-        sf[pos] = hits[i];
-        si[pos] = i;
-      }
+      if (pos < kp2) sort[pos] = ((uint64_t)(uint32_t)f << 32) | (uint32_t)i;
     }
   }
   __syncthreads();
-  if (threadIdx.x == 0 && sm[40] != K) atomicOr(status + 2, 1);
-  // bitonic sort of (sf, si) by sf ascending
-  for (int size = 2; size <= kp2; size <<= 1) {
-    for (int stride = size >> 1; stride > 0; stride >>= 1) {
-      for (int t = threadIdx.x; t < (kp2 >> 1); t += blockDim.x) {
-        const int i = 2 * t - (t & (stride - 1));
-        const int jn = i + stride;
-        const bool up = (i & size) == 0;
-        const int a = sf[i], b = sf[jn];
-        if ((a > b) == up) {
-          sf[i] = b;
-          sf[jn] = a;
-          const int ti = si[i];
-          si[i] = si[jn];
-          si[jn] = ti;
+  if (tid == 0 && sm[40] != K) atomicOr(status + 2, 1);
+  if (kp2 <= 1024) {
+    uint64_t v = tid < kp2 ? sort[tid] : ~0ull;
+    for (int size = 2; size <= kp2; size <<= 1) {
+      for (int stride = size >> 1; stride > 0; stride >>= 1) {
+        uint64_t o;
+        if (stride >= 32) {
+          __syncthreads();
+          sort[tid] = v;
+          __syncthreads();
+          o = sort[tid ^ stride];
+        } else {
+          o = __shfl_xor_sync(kFull, v, stride);
         }
+        const bool up = (tid & size) == 0;
+        const bool lower = (tid & stride) == 0;
+        v = (lower == up) ? min(v, o) : max(v, o);
       }
-      __syncthreads();
+    }
+    __syncthreads();
+    if (tid < kp2) sort[tid] = v;
+    __syncthreads();
+  } else {
+    for (int size = 2; size <= kp2; size <<= 1) {
+      for (int stride = size >> 1; stride > 0; stride >>= 1) {
+        for (int t = tid; t < (kp2 >> 1); t += 1024) {
+          const int i = 2 * t - (t & (stride - 1));
+          const int jn = i + stride;
+          const bool up = (i & size) == 0;
+          const uint64_t a = sort[i], b = sort[jn];
+          if ((a > b) == up) {
+            sort[i] = b;
+            sort[jn] = a;
+          }
+        }
+        __syncthreads();
+      }
     }
   }
-  for (int j = threadIdx.x; j < k; j += blockDim.x) {
+  for (int j = tid; j < k; j += 1024) {
     if (j < K) {
-      locs[j] = sf[j];
-      vals[j] = hit_vals[si[j]];
+      const uint64_t v = sort[j];
+      locs[j] = (int64_t)(v >> 32);
+      vals[j] = hit_vals[(uint32_t)v];
     } else {
       locs[j] = -1;
       vals[j] = make_double2(0.0, 0.0);
