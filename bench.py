@@ -6,7 +6,7 @@
 
 One step = one whole transform (fold, B-point FFT, cutoff, vote, estimate,
 output; for N > 1 plus the all-gather) of a planted k-sparse fp64 signal that
-is already resident in HBM.  L2 is flushed (256 MiB memset) between timed
+is already resident in HBM.  L2 is flushed (256 MiB write + 256 MiB read) between timed
 steps, outside the per-step CUDA events.  Prints ONE JSON line on rank 0.
 See DESIGN.md §8 for every field.
 """
@@ -221,7 +221,19 @@ def run_gpu(args):
     got = {int(f): complex(v) for f, v in zip(l_np, v_np) if f >= 0}
     l1 = sum(abs(got.get(f, 0) - truth.get(f, 0)) for f in set(truth) | set(got)) / k
 
-    flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=dev)
+    flush_w = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=dev)
+    flush_r = torch.ones(64 * 1024 * 1024, dtype=torch.int32, device=dev)
+
+    class _Flush:
+        """L2 flush between timed steps: write 256 MiB (evicts everything), then
+        read another 256 MiB so the write-backs happen here, not in the step."""
+
+        @staticmethod
+        def zero_():
+            flush_w.zero_()
+            flush_r.sum()
+
+    flush = _Flush()
     stream = torch.cuda.current_stream()
 
     def barrier():
@@ -265,17 +277,48 @@ def run_gpu(args):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
 
-    # ---- per-stage times (fold = dominant kernel) on the plan's stream
-    plan.set_timing(True)
-    stage = {key: [] for key in ("fold", "fft", "cutoff", "vote", "estimate", "output")}
-    for _ in range(max(5, args.steps)):
-        flush.zero_()
-        step()
-        st = plan.stage_times()
-        for key in stage:
-            stage[key].append(st[key])
-    plan.set_timing(False)
-    stage_ms = {key: (sum(v) / len(v)) for key, v in stage.items()}
+    # ---- per-stage times inside the CUDA graph: T_s = time of the graph that
+    # runs stages 1..s (cusfft_set_stage_limit), stage s = T_s - T_{s-1}.
+    # T_1 is the fold kernel alone (+ an 8-int memset node): the roofline's
+    # kernel time, measured with CUDA events on the plan's (current) stream.
+    def timed_mean(reps):
+        ts = []
+        for _ in range(reps):
+            flush.zero_()
+            a = torch.cuda.Event(enable_timing=True)
+            b = torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            step()
+            b.record(stream)
+            torch.cuda.synchronize()
+            ts.append(a.elapsed_time(b))
+        return sum(ts) / len(ts)
+
+    names = ("fold", "fft", "cutoff", "vote", "estimate", "output")
+    stage_ms = {}
+    if world == 1:
+        prev = 0.0
+        reps = max(10, args.steps)
+        for si, nm in enumerate(names, start=1):
+            plan.set_stage_limit(si)
+            step()
+            tsi = timed_mean(reps)
+            stage_ms[nm] = tsi - prev
+            prev = tsi
+        plan.set_stage_limit(6)
+        fold_ms = stage_ms["fold"]
+    else:
+        plan.set_timing(True)
+        acc = {nm: [] for nm in names}
+        for _ in range(max(5, args.steps)):
+            flush.zero_()
+            step()
+            st = plan.stage_times()
+            for nm in names:
+                acc[nm].append(st[nm])
+        plan.set_timing(False)
+        stage_ms = {nm: sum(v) / len(v) for nm, v in acc.items()}
+        fold_ms = stage_ms["fold"]
 
     # ---- dense cuFFT of the same n (context), complex128, L2 flushed
     dense = []
@@ -318,7 +361,6 @@ def run_gpu(args):
 
     peak, peak_src = hbm_peak()
     sector, useful = fold_bytes(plan.L // world if world > 1 else L, plan.w, B)
-    fold_ms = stage_ms["fold"]
     achieved = sector / (fold_ms * 1e-3) / 1e9
     traffic = None
     tf = os.path.join(ROOT, "profiles", f"fold_traffic_{args.config}.json")
@@ -335,7 +377,7 @@ def run_gpu(args):
         "config": {"workload": f"{args.config}: {desc}, L={L}, B={B}, w={plan.w} taps (Dolph-Chebyshev, delta=1e-8)",
                    "n": n, "k": k, "B": B, "L": L, "taps": plan.w, "loc_loops": plan.loc_loops,
                    "vote_threshold": plan.T, "parallelism": f"loop-sharded x{world}" if world > 1 else "single GPU",
-                   "l2": "flushed (256 MiB memset) between timed steps, outside the step events",
+                   "l2": "flushed between timed steps (256 MiB write + 256 MiB read), outside the step events",
                    "signal_seed": args.signal_seed, "plan_seed": args.plan_seed},
         "gpu_launches": launches * args.steps,
         "timed_region_ms_incl_flush": region_ms,

@@ -168,6 +168,11 @@ int cusfft_status(cusfft_plan_t plan);
 int cusfft_set_timing(cusfft_plan_t plan, int32_t enable);
 int cusfft_get_stage_times(cusfft_plan_t plan, float* ms, int32_t cap);
 
+/* Profiling: run only the first `stages` stages (1 = fold ... 6 = output,
+ * the default) so per-stage times can be taken inside the CUDA graph by
+ * differences of whole-execution times.  Outputs are undefined when < 6. */
+int cusfft_set_stage_limit(cusfft_plan_t plan, int32_t stages);
+
 /* Number of kernel launches one cusfft_execute issues for this plan. */
 int32_t cusfft_launches_per_execute(cusfft_plan_t plan);
 

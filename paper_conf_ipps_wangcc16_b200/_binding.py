@@ -12,7 +12,8 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libcusfft.so")
+# CUSFFT_LIB selects an alternative in-tree build (e.g. the -DCUSFFT_TRACE one).
+LIB_PATH = os.path.join(_HERE, os.environ.get("CUSFFT_LIB", "libcusfft.so"))
 
 SUCCESS = 0
 INVALID_N, INVALID_B, INVALID_K, INVALID_LOOPS, INVALID_PARAM = -1, -2, -3, -4, -5
@@ -30,7 +31,7 @@ EXPORTED = (
     "cusfft_destroy", "cusfft_set_stream", "cusfft_execute", "cusfft_execute_host",
     "cusfft_execute_local", "cusfft_execute_finish", "cusfft_exchange_buffer",
     "cusfft_get_info", "cusfft_get_debug", "cusfft_status", "cusfft_set_timing",
-    "cusfft_get_stage_times", "cusfft_launches_per_execute", "cusfft_strerror",
+    "cusfft_get_stage_times", "cusfft_set_stage_limit", "cusfft_launches_per_execute", "cusfft_strerror",
     "cusfft_last_cuda_error", "cusfft_abi_version",
 )
 
@@ -87,6 +88,7 @@ def load_library():
         "cusfft_status": (ctypes.c_int, [P]),
         "cusfft_set_timing": (ctypes.c_int, [P, i32]),
         "cusfft_get_stage_times": (ctypes.c_int, [P, P, i32]),
+        "cusfft_set_stage_limit": (ctypes.c_int, [P, i32]),
         "cusfft_launches_per_execute": (i32, [P]),
         "cusfft_strerror": (ctypes.c_char_p, [ctypes.c_int]),
         "cusfft_last_cuda_error": (i32, []),
@@ -293,6 +295,9 @@ class Plan:
         ms = (ctypes.c_float * 6)()
         check(self._lib.cusfft_get_stage_times(self._h, ms, 6), "cusfft_get_stage_times")
         return dict(zip(("fold", "fft", "cutoff", "vote", "estimate", "output"), list(ms)))
+
+    def set_stage_limit(self, stages: int):
+        check(self._lib.cusfft_set_stage_limit(self._h, stages), "cusfft_set_stage_limit")
 
     def launches_per_execute(self) -> int:
         return int(self._lib.cusfft_launches_per_execute(self._h))

@@ -9,6 +9,24 @@ namespace cusfft {
 
 constexpr unsigned kFull = 0xFFFFFFFFu;
 
+// Opt-in phase tracing (build with -DCUSFFT_TRACE): TRACE(slot) stores the
+// %globaltimer (ns) of thread 0 of the calling CTA into g_trace[slot].
+#ifdef CUSFFT_TRACE
+__device__ unsigned long long g_trace[256];
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define TRACE(slot) \
+  do { if (threadIdx.x == 0) g_trace[(slot)] = gtimer(); } while (0)
+#define TRACE_END(slot) \
+  do { if (threadIdx.x == 0) atomicMax(&g_trace[(slot)], gtimer()); } while (0)
+#else
+#define TRACE(slot) do { } while (0)
+#define TRACE_END(slot) do { } while (0)
+#endif
+
 // Per-slot loop parameters (slot order; see DESIGN.md §6 "slots").
 //   sigma: gather stride (Alg. 1's ai), a = sigma^-1 mod n,
 //   tau: offset (Def. 1), loop: the loop index r this slot holds.
@@ -82,64 +100,86 @@ __device__ __forceinline__ bool ge96(const Prefix96& p, uint64_t hi, uint32_t lo
   return (lo & p.mlo) >= p.plo;
 }
 
-// Block-wide radix select (blockDim.x == 1024): find a prefix such that the
+// Digit shift of radix pass `pass` (12-bit digits MSB-first; bit 95, the sign
+// of a non-negative fp64 key, is skipped; the last pass overlaps one bit).
+__device__ __forceinline__ int pass_shift(int pass) { return pass < 7 ? 83 - 12 * pass : 0; }
+
+// Block-wide scan of a 4096-bin histogram from the top digit down
+// (blockDim.x == NT): returns {digit, count above it, count in it} of the
+// bin holding the krem-th largest item.  Requires 1 <= krem <= total.
+struct BinPick {
+  int d, above, cnt;
+};
+
+template <int NT = 1024>
+__device__ __forceinline__ BinPick pick_bin(const uint32_t* hist, int krem, int* sm) {
+  constexpr int PER = 4096 / NT;  // bins per thread, descending
+  const int tid = threadIdx.x;
+  const int base = 4095 - PER * tid;
+  int c[PER];
+  int mine = 0;
+#pragma unroll
+  for (int j = 0; j < PER; ++j) {
+    c[j] = hist[base - j];
+    mine += c[j];
+  }
+  int total;
+  const int ex = block_excl_scan<NT>(mine, &total, sm);
+  if (ex < krem && krem <= ex + mine) {
+    int cum = ex;
+#pragma unroll
+    for (int j = 0; j < PER; ++j) {
+      if (cum + c[j] >= krem) {
+        sm[32] = base - j; sm[33] = cum; sm[34] = c[j];
+        break;
+      }
+      cum += c[j];
+    }
+  }
+  __syncthreads();
+  BinPick r{sm[32], sm[33], sm[34]};
+  __syncthreads();
+  return r;
+}
+
+// Block-wide radix select (blockDim.x == NT): find a prefix such that the
 // items with ge96(prefix, item) are exactly the K largest composites among N.
-// src.get(i, hi, lo) must be callable for 0 <= i < N.  Requires 1 <= K <= N.
-// hist: 4096 u32 in shared memory; sm: >= 40 ints in shared memory.
-// Digits: 12 bits MSB-first; bit 95 (the sign of a non-negative fp64 key) is
-// skipped; early exit once the boundary digit's whole bin is selected.
-template <class Src>
-__device__ Prefix96 block_radix_select(const Src& src, int N, int K, uint32_t* hist, int* sm) {
-  constexpr int NT = 1024;
+// src.get(i, hi, lo) must be callable for 0 <= i < N.  Starts at radix pass
+// `start` with the digits of earlier passes already fixed in `p` and `krem`
+// items still to choose among those matching p (start = 0: p empty, krem = K).
+// If `prebuilt`, hist already holds the counts of pass `start` (over the items
+// matching p).  hist: 4096 u32 in shared memory; sm: >= 40 ints.
+// Early exit once the boundary digit's whole bin is selected.
+template <class Src, int NT = 1024>
+__device__ Prefix96 block_radix_select(const Src& src, int N, int krem, uint32_t* hist, int* sm, int start = 0,
+                                       Prefix96 p = Prefix96{0, 0, 0, 0}, bool prebuilt = false) {
   const int tid = threadIdx.x, lane = tid & 31;
-  Prefix96 p{0, 0, 0, 0};
-  int krem = K;
-  for (int pass = 0; pass < 8; ++pass) {
-    const int shift = pass < 7 ? 83 - 12 * pass : 0;
-    for (int i = tid; i < 4096; i += NT) hist[i] = 0;
-    __syncthreads();
-    for (int i0 = 0; i0 < N; i0 += NT) {
-      const int i = i0 + tid;
-      bool valid = i < N;
-      uint32_t d = 0xFFFFFFFFu;
-      if (valid) {
-        uint64_t hi;
-        uint32_t lo;
-        src.get(i, hi, lo);
-        valid = match96(p, hi, lo);
-        if (valid) d = digit96(hi, lo, shift);
+  for (int pass = start; pass < 8; ++pass) {
+    const int shift = pass_shift(pass);
+    if (!(prebuilt && pass == start)) {
+      for (int i = tid; i < 4096; i += NT) hist[i] = 0;
+      __syncthreads();
+      for (int i0 = 0; i0 < N; i0 += NT) {
+        const int i = i0 + tid;
+        bool valid = i < N;
+        uint32_t d = 0xFFFFFFFFu;
+        if (valid) {
+          uint64_t hi;
+          uint32_t lo;
+          src.get(i, hi, lo);
+          valid = match96(p, hi, lo);
+          if (valid) d = digit96(hi, lo, shift);
+        }
+        const unsigned grp = __match_any_sync(kFull, d);
+        if (valid && lane == __ffs(grp) - 1) atomicAdd(&hist[d], (uint32_t)__popc(grp));
       }
-      const unsigned grp = __match_any_sync(kFull, d);
-      if (valid && lane == __ffs(grp) - 1) atomicAdd(&hist[d], (uint32_t)__popc(grp));
+      __syncthreads();
     }
-    __syncthreads();
-    // thread t owns bins 4095-4t .. 4092-4t (descending digit order)
-    const int base = 4095 - 4 * tid;
-    const int c0 = hist[base], c1 = hist[base - 1], c2 = hist[base - 2], c3 = hist[base - 3];
-    const int mine = c0 + c1 + c2 + c3;
-    int total;
-    const int ex = block_excl_scan<NT>(mine, &total, sm);
-    if (ex < krem && krem <= ex + mine) {
-      int cum = ex, d, cnt;
-      if (cum + c0 >= krem) {
-        d = base; cnt = c0;
-      } else if ((cum += c0) + c1 >= krem) {
-        d = base - 1; cnt = c1;
-      } else if ((cum += c1) + c2 >= krem) {
-        d = base - 2; cnt = c2;
-      } else {
-        cum += c2; d = base - 3; cnt = c3;
-      }
-      sm[32] = d; sm[33] = cum; sm[34] = cnt;
-    }
-    __syncthreads();
-    const uint32_t d = (uint32_t)sm[32];
-    const int above = sm[33], cnt = sm[34];
-    __syncthreads();
-    or96(p.phi, p.plo, d, shift);
+    const BinPick b = pick_bin<NT>(hist, krem, sm);
+    or96(p.phi, p.plo, (uint32_t)b.d, shift);
     or96(p.mhi, p.mlo, 0xFFFu, shift);
-    krem -= above;
-    if (cnt == krem) break;  // every item in the boundary bin is selected
+    krem -= b.above;
+    if (b.cnt == krem) break;  // every item in the boundary bin is selected
   }
   return p;
 }

@@ -9,6 +9,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <new>
+#include <utility>
 #include <vector>
 
 #include "../../include/cusfft.h"
@@ -20,6 +21,7 @@ using namespace cusfft;
 namespace {
 
 constexpr uint32_t kMagic = 0x5FF7B200u;
+constexpr int kFoldPad = 120 * 1024;  // dynamic smem that caps a fold launch at 1 CTA per SM
 thread_local int g_last_cuda_error = 0;
 
 #define CK(expr)                                  \
@@ -101,7 +103,7 @@ struct cusfft_plan_s {
   int B1 = 1, B2 = 1, logB1 = 0, logB2 = 0;
   int kp2 = 1;
   int select_smem = 0, vote_smem = 0, output_smem = 0;
-  int vote_P = 1, vote_grid = 1, est_grid = 1;
+  int vote_grid = 1, est_grid = 1;
   int fft_smem1 = 0, fft_smem2 = 0;
   std::vector<SlotParam> slots_h;       // slot order
   std::vector<int64_t> a_r, sigma_r, tau_r;  // loop order
@@ -109,6 +111,8 @@ struct cusfft_plan_s {
   RecLayout lay{};
   // device memory
   double* d_taps = nullptr;
+  double* d_taps_perm = nullptr;  // fused fold+pass-1 layout (two-pass B, B1 <= 256)
+  bool fused1 = false;
   double2* d_ghat = nullptr;
   double2* d_tw = nullptr;
   SlotParam* d_slots = nullptr;
@@ -122,10 +126,19 @@ struct cusfft_plan_s {
   uint64_t* d_keys = nullptr;     // [n_sel][B] cutoff keys of this rank's location loops
   uint32_t* d_hist = nullptr;     // [n_sel][4096] top-digit histograms (self-resetting)
   int* d_key_index = nullptr;     // [Lg] local slot -> selection index or -1
+  uint32_t* d_ohist = nullptr;    // [4096] top-digit histogram of the output keys (self-resetting)
+  uint32_t* d_hist1 = nullptr;    // [n_sel][4096] level-1 cutoff histograms (self-resetting)
+  uint64_t* d_ckey = nullptr;     // [n_sel][kSelCap] cutoff boundary candidates
+  int* d_cidx = nullptr;
+  int* d_ccount = nullptr;        // [n_sel] candidate counters (self-resetting)
+  int* d_done = nullptr;          // [n_sel] finished-CTA counters (self-resetting)
+  int sel_S = 1;                  // CTAs per location loop in k_select
   int* d_hits = nullptr;
   double2* d_hit_vals = nullptr;
   uint64_t* d_hit_keys = nullptr;
   double2* d_per_loop = nullptr;
+  int* d_zero = nullptr;   // per-execution block, zeroed by the first fold kernel of each execution:
+  int nzero = 0;           //   flags[8] | hist0[n_sel][4096] | hist1[n_sel][4096] | ohist[4096] | ccount | done
   int* d_flags = nullptr;  // [0] hit_count (unsigned), [1] overflow, [2] select mismatch, [3] output mismatch
   double2* d_xbuf = nullptr;
   int64_t* d_locs_buf = nullptr;
@@ -137,13 +150,20 @@ struct cusfft_plan_s {
   bool ev_made = false;
   // CUDA graphs of the launch sequences, keyed by the caller's pointers
   bool use_graph = true;
-  cudaStream_t cap_stream = nullptr;
+  bool branched = false;          // two-branch graph (location chain || estimation folds); opt-in
+  int nloc_local = 0;             // local slots [0, nloc_local) are location loops
+  cudaStream_t cap_stream = nullptr, cap_stream2 = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  int stage_limit = 6;
+  int cur_prio = 0, prio_hi = 0, prio_lo = 0;  // launch priorities (branched graph)
+  int fold_smem_pad = 0;  // unused dynamic smem that caps the estimation fold at 1 CTA / SM
   struct GraphEntry {
+    int lim = -1;
     const void* a = nullptr;
     const void* b = nullptr;
     const void* c = nullptr;
     cudaGraphExec_t exec = nullptr;
-  } g_full, g_local, g_finish;
+  } g_full, g_local, g_finish, g_full_t, g_local_t, g_finish_t;  // *_t: with timing event nodes
 };
 
 namespace {
@@ -163,16 +183,19 @@ struct DeviceGuard {
 };
 
 void free_plan(cusfft_plan_t p) {
-  void* ptrs[] = {p->d_taps, p->d_ghat, p->d_tw, p->d_slots, p->d_loc_slots, p->d_loc_sigma, p->d_loc_a,
-                  p->d_sel_slots, p->d_u, p->d_v, p->d_records, p->d_keys, p->d_hist, p->d_key_index, p->d_hits, p->d_hit_vals,
-                  p->d_hit_keys, p->d_per_loop, p->d_flags, p->d_xbuf, p->d_locs_buf, p->d_vals_buf};
+  void* ptrs[] = {p->d_taps, p->d_taps_perm, p->d_ghat, p->d_tw, p->d_slots, p->d_loc_slots, p->d_loc_sigma, p->d_loc_a,
+                  p->d_sel_slots, p->d_u, p->d_v, p->d_records, p->d_keys, p->d_zero, p->d_key_index, p->d_ckey, p->d_cidx, p->d_hits, p->d_hit_vals,
+                  p->d_hit_keys, p->d_per_loop, p->d_xbuf, p->d_locs_buf, p->d_vals_buf};
   for (void* q : ptrs)
     if (q) cudaFree(q);
   if (p->ev_made)
     for (auto& e : p->ev) cudaEventDestroy(e);
-  for (auto* g : {&p->g_full, &p->g_local, &p->g_finish})
+  for (auto* g : {&p->g_full, &p->g_local, &p->g_finish, &p->g_full_t, &p->g_local_t, &p->g_finish_t})
     if (g->exec) cudaGraphExecDestroy(g->exec);
   if (p->cap_stream) cudaStreamDestroy(p->cap_stream);
+  if (p->cap_stream2) cudaStreamDestroy(p->cap_stream2);
+  if (p->ev_fork) cudaEventDestroy(p->ev_fork);
+  if (p->ev_join) cudaEventDestroy(p->ev_join);
   p->magic = 0;
   delete p;
 }
@@ -264,32 +287,49 @@ int build_filter(cusfft_plan_t P) {
   return CUSFFT_SUCCESS;
 }
 
+// Kernel launch carrying an explicit scheduling priority: stream priorities are
+// not captured into graph kernel nodes, the launch attribute is.
+template <typename... KArgs, typename... Args>
+cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, int prio,
+                     Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributePriority;
+  attr[0].val.priority = prio;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
+
 template <int M>
 constexpr int fft_E() { return M < 1024 ? 1024 : M; }
 
 template <int M>
-cudaError_t launch_fft_t(const FftPassArgs& a, int smem, cudaStream_t st) {
+cudaError_t launch_fft_t(const FftPassArgs& a, int smem, cudaStream_t st, int prio) {
   constexpr int E = fft_E<M>();
   constexpr int NSEQ = E / M;
   const int grid = (a.total_seq + NSEQ - 1) / NSEQ;
-  k_fft<M, E, 128><<<grid, 128, smem, st>>>(a);
-  return cudaGetLastError();
+  return launch_k(k_fft<M, E, 128>, dim3(grid), dim3(128), smem, st, prio, a);
 }
 
-cudaError_t launch_fft(int M, const FftPassArgs& a, int smem, cudaStream_t st) {
+cudaError_t launch_fft(int M, const FftPassArgs& a, int smem, cudaStream_t st, int prio = 0) {
   switch (M) {
-    case 2: return launch_fft_t<2>(a, smem, st);
-    case 4: return launch_fft_t<4>(a, smem, st);
-    case 8: return launch_fft_t<8>(a, smem, st);
-    case 16: return launch_fft_t<16>(a, smem, st);
-    case 32: return launch_fft_t<32>(a, smem, st);
-    case 64: return launch_fft_t<64>(a, smem, st);
-    case 128: return launch_fft_t<128>(a, smem, st);
-    case 256: return launch_fft_t<256>(a, smem, st);
-    case 512: return launch_fft_t<512>(a, smem, st);
-    case 1024: return launch_fft_t<1024>(a, smem, st);
-    case 2048: return launch_fft_t<2048>(a, smem, st);
-    case 4096: return launch_fft_t<4096>(a, smem, st);
+    case 2: return launch_fft_t<2>(a, smem, st, prio);
+    case 4: return launch_fft_t<4>(a, smem, st, prio);
+    case 8: return launch_fft_t<8>(a, smem, st, prio);
+    case 16: return launch_fft_t<16>(a, smem, st, prio);
+    case 32: return launch_fft_t<32>(a, smem, st, prio);
+    case 64: return launch_fft_t<64>(a, smem, st, prio);
+    case 128: return launch_fft_t<128>(a, smem, st, prio);
+    case 256: return launch_fft_t<256>(a, smem, st, prio);
+    case 512: return launch_fft_t<512>(a, smem, st, prio);
+    case 1024: return launch_fft_t<1024>(a, smem, st, prio);
+    case 2048: return launch_fft_t<2048>(a, smem, st, prio);
+    case 4096: return launch_fft_t<4096>(a, smem, st, prio);
     default: return cudaErrorInvalidValue;
   }
 }
@@ -298,6 +338,31 @@ template <int M>
 cudaError_t set_fft_attr_t() {
   return cudaFuncSetAttribute(k_fft<M, fft_E<M>(), 128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                               fft_smem_bytes(fft_E<M>()));
+}
+
+// Every hot-path kernel runs with the maximum shared-memory carveout, so that
+// kernels of the two graph branches can be resident on one SM at the same time
+// (an SM changes its L1/smem split only when idle).
+template <typename K>
+cudaError_t carveout_max(K kern) {
+  return cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared);
+}
+
+template <int M>
+cudaError_t carve_fft_t() {
+  return carveout_max(k_fft<M, fft_E<M>(), 128>);
+}
+
+cudaError_t set_carveouts() {
+  cudaError_t r[] = {carve_fft_t<2>(), carve_fft_t<4>(), carve_fft_t<8>(), carve_fft_t<16>(), carve_fft_t<32>(),
+                     carve_fft_t<64>(), carve_fft_t<128>(), carve_fft_t<256>(), carve_fft_t<512>(),
+                     carve_fft_t<1024>(), carve_fft_t<2048>(), carve_fft_t<4096>(), carveout_max(k_fold<16>),
+                     carveout_max(k_fold_fft1<64, 8>), carveout_max(k_fold_fft1<128, 8>),
+                     carveout_max(k_fold_fft1<256, 8>), carveout_max(k_select), carveout_max(k_vote),
+                     carveout_max(k_estimate), carveout_max(k_output)};
+  for (cudaError_t x : r)
+    if (x != cudaSuccess) return x;
+  return cudaSuccess;
 }
 
 cudaError_t set_fft_attrs() {
@@ -364,6 +429,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   P->R = (int)((w64 + B - 1) / B);
   P->stream = nullptr;
   if (const char* e = std::getenv("CUSFFT_NO_GRAPH")) P->use_graph = !(e[0] == '1');
+  if (const char* e = std::getenv("CUSFFT_BRANCH")) P->branched = (e[0] == '1');
 
   // ---- draws (loop order), Alg. 1, Def. 1
   SplitMix64 rng{q.seed};
@@ -381,6 +447,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     const int g = s / P->Lg, i = s % P->Lg, r = i * world + g;
     P->slots_h[s] = SlotParam{(uint32_t)P->sigma_r[r], (uint32_t)P->tau_r[r], (uint32_t)P->a_r[r], (uint32_t)r};
   }
+  for (int i = 0; i < P->Lg; ++i)
+    if (i * world + rank < P->Lloc) P->nloc_local = i + 1;  // location loops are a prefix of the local slots
   std::vector<uint32_t> loc_sig, loc_a;
   for (int s = 0; s < L; ++s) {
     if ((int)P->slots_h[s].loop < P->Lloc) {
@@ -406,18 +474,18 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   P->logB1 = ilog2(P->B1);
   P->logB2 = ilog2(P->B2);
   P->select_smem = 4096 * 4 + 64 * 4 + kSelCap * 12;
+  P->sel_S = (int)std::max<int64_t>(1, std::min<int64_t>(16, B / 2048));
   P->vote_smem = P->Lloc * (int)((B + 31) / 32) * 4;
   P->kp2 = 1;
   while (P->kp2 < k) P->kp2 <<= 1;
-  P->output_smem = 4096 * 4 + 64 * 4 + kOutCap * 12 + std::max(P->kp2, 1024) * 8;
+  P->output_smem = 4096 * 4 + 64 * 4 + kOutCap * 12 + 2 * P->kp2 * 8 + 2 * 1024 * 4;
   P->fft_smem1 = fft_smem_bytes(std::max(1024, P->B1));
   P->fft_smem2 = fft_smem_bytes(std::max(1024, P->B2));
-  P->vote_P = (int)std::min<int64_t>(P->nb, 16);
   {
-    const int64_t items = (int64_t)(P->Lloc - P->T + 1) * P->num * (P->nb / P->vote_P);
+    const int64_t units = (int64_t)(P->Lloc - P->T + 1) * P->num;  // one warp per (q0, J) range
     int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    P->vote_grid = (int)std::max<int64_t>(1, std::min<int64_t>((items + 255) / 256, (int64_t)sms * 4));
+    P->vote_grid = (int)std::max<int64_t>(1, std::min<int64_t>((units + 7) / 8, (int64_t)sms * 4));
     P->est_grid = std::max(1, std::min((P->max_hits + 7) / 8, sms * 4));
   }
   if (P->vote_smem > 200 * 1024) {
@@ -444,12 +512,24 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   {
     const size_t nsel = std::max<size_t>(1, P->sel_slots_h.size());
     if ((rc = dalloc(&P->d_keys, nsel * B))) return fail(rc);
-    if ((rc = dalloc(&P->d_hist, nsel * 4096))) return fail(rc);
+    // per-execution counters and histograms: one block, zeroed by the first fold kernel
+    P->nzero = 8 + (int)(2 * nsel * 4096 + 4096 + 2 * nsel);
+    if ((rc = dalloc(&P->d_zero, (size_t)P->nzero))) return fail(rc);
+    P->d_flags = P->d_zero;
+    P->d_hist = reinterpret_cast<uint32_t*>(P->d_zero + 8);
+    P->d_hist1 = P->d_hist + nsel * 4096;
+    P->d_ohist = P->d_hist1 + nsel * 4096;
+    P->d_ccount = reinterpret_cast<int*>(P->d_ohist + 4096);
+    P->d_done = P->d_ccount + nsel;
     if ((rc = dalloc(&P->d_key_index, (size_t)P->Lg))) return fail(rc);
+
+    if ((rc = dalloc(&P->d_ckey, nsel * kSelCap))) return fail(rc);
+    if ((rc = dalloc(&P->d_cidx, nsel * kSelCap))) return fail(rc);
+
     std::vector<int> kidx(P->Lg, -1);
     for (size_t i = 0; i < P->sel_slots_h.size(); ++i) kidx[P->sel_slots_h[i] - rank * P->Lg] = (int)i;
     if (cudaMemcpy(P->d_key_index, kidx.data(), P->Lg * sizeof(int), cudaMemcpyHostToDevice) != cudaSuccess ||
-        cudaMemset(P->d_hist, 0, nsel * 4096 * sizeof(uint32_t)) != cudaSuccess) {
+        cudaMemset(P->d_zero, 0, (size_t)P->nzero * sizeof(int)) != cudaSuccess) {
       g_last_cuda_error = (int)cudaGetLastError();
       return fail(CUSFFT_CUDA);
     }
@@ -458,7 +538,6 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   if ((rc = dalloc(&P->d_hit_vals, (size_t)P->max_hits))) return fail(rc);
   if ((rc = dalloc(&P->d_hit_keys, (size_t)P->max_hits))) return fail(rc);
   if (q.debug && (rc = dalloc(&P->d_per_loop, (size_t)P->max_hits * L))) return fail(rc);
-  if ((rc = dalloc(&P->d_flags, 8))) return fail(rc);
   auto upload = [&](void* dst, const void* src, size_t bytes) -> int {
     CK(cudaMemcpy(dst, src, bytes, cudaMemcpyHostToDevice));
     return CUSFFT_SUCCESS;
@@ -471,11 +550,15 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       (rc = upload(P->d_sel_slots, P->sel_slots_h.data(), P->sel_slots_h.size() * sizeof(int))))
     return fail(rc);
   if (cudaMemset(P->d_records, 0, (size_t)L * P->lay.rec_bytes) != cudaSuccess ||
-      cudaMemset(P->d_flags, 0, 8 * sizeof(int)) != cudaSuccess) {
+      false) {
     g_last_cuda_error = (int)cudaGetLastError();
     return fail(CUSFFT_CUDA);
   }
   if (set_fft_attrs() != cudaSuccess ||
+      cudaFuncSetAttribute(k_fold<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024) != cudaSuccess ||
+      cudaFuncSetAttribute(k_fold_fft1<64, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024) != cudaSuccess ||
+      cudaFuncSetAttribute(k_fold_fft1<128, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024) != cudaSuccess ||
+      cudaFuncSetAttribute(k_fold_fft1<256, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_select, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_vote, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_output, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess) {
@@ -483,6 +566,24 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     return fail(CUSFFT_CUDA);
   }
   if ((rc = build_filter(P))) return fail(rc);
+  P->fused1 = P->B1 > 1 && P->B1 <= 256;
+  if (P->fused1) {  // taps_perm[rr B + cta 256 + t] = g[j(cta, t) + rr B], j = c + B2 j1
+    const int64_t padded = (int64_t)P->R * B;
+    std::vector<double> g((size_t)padded), gp((size_t)padded);
+    if (cudaMemcpy(g.data(), P->d_taps, padded * sizeof(double), cudaMemcpyDeviceToHost) != cudaSuccess) {
+      g_last_cuda_error = (int)cudaGetLastError();
+      return fail(CUSFFT_CUDA);
+    }
+    const int C = 256 / P->B1;
+    for (int64_t rr = 0; rr < P->R; ++rr)
+      for (int64_t cta = 0; cta < B / 256; ++cta)
+        for (int t = 0; t < 256; ++t) {
+          const int64_t cc = cta * C + t / P->B1, j1 = t % P->B1;
+          gp[(size_t)(rr * B + cta * 256 + t)] = g[(size_t)(rr * B + cc + (int64_t)P->B2 * j1)];
+        }
+    if ((rc = dalloc(&P->d_taps_perm, (size_t)padded))) return fail(rc);
+    if ((rc = upload(P->d_taps_perm, gp.data(), padded * sizeof(double)))) return fail(rc);
+  }
   if (cudaStreamSynchronize(P->stream) != cudaSuccess) {
     g_last_cuda_error = (int)cudaGetLastError();
     return fail(CUSFFT_CUDA);
@@ -491,51 +592,97 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   return CUSFFT_SUCCESS;
 }
 
+template <int B1T>
+cudaError_t launch_fold_fft1_t(cusfft_plan_t P, const double2* x, const SlotParam* sp, double2* u, double2* v,
+                               int nslots, ZeroArgs z, cudaStream_t st) {
+  dim3 grid((unsigned)(P->B / 256), (unsigned)nslots);
+  return launch_k(k_fold_fft1<B1T, 8>, grid, dim3(256), P->fold_smem_pad, st, P->cur_prio, x, (const double*)P->d_taps_perm, sp, u, v,
+                  (const double2*)P->d_tw, (int)P->B, P->B2, P->w, P->R, (uint32_t)(P->n - 1), z);
+}
+
+cudaError_t launch_fold_fft1(cusfft_plan_t P, const double2* x, const SlotParam* sp, double2* u, double2* v,
+                             int nslots, ZeroArgs z, cudaStream_t st) {
+  switch (P->B1) {
+    case 64: return launch_fold_fft1_t<64>(P, x, sp, u, v, nslots, z, st);
+    case 128: return launch_fold_fft1_t<128>(P, x, sp, u, v, nslots, z, st);
+    case 256: return launch_fold_fft1_t<256>(P, x, sp, u, v, nslots, z, st);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
 inline void mark(cusfft_plan_t P, int i) {
   if (P->timing) cudaEventRecord(P->ev[i], P->stream);
 }
 
-int launch_local(cusfft_plan_t P, const double2* x) {
+// Steps 1+2 (and the fused FFT pass 1) for this rank's local slots [s0, s1).
+// zero_block: this launch also zeroes the per-execution block (first fold only).
+int launch_fold(cusfft_plan_t P, const double2* x, int s0, int s1, cudaStream_t st, bool zero_block) {
+  if (s1 <= s0) return CUSFFT_SUCCESS;
   const int B = (int)P->B;
-  cudaStream_t st = P->stream;
-  CK(cudaMemsetAsync(P->d_flags, 0, 8 * sizeof(int), st));
-  mark(P, 0);
-  {
-    dim3 grid((B + 255) / 256, P->Lg);
-    k_fold<16><<<grid, 256, 0, st>>>(x, P->d_taps, P->d_slots + (size_t)P->rank * P->Lg, P->d_u, B, P->w, P->R,
-                                     (uint32_t)(P->n - 1));
-    CKL();
-  }
-  mark(P, 1);
-  uint8_t* myrec = P->d_records + (int64_t)P->rank * P->Lg * P->lay.rec_bytes;
-  const int64_t rec_e = P->lay.rec_bytes / 16;
-  const bool keys = !P->sel_slots_h.empty();
-  if (P->B1 > 1) {
-    // pass 1: B1-point FFTs over columns c (stride B2), twiddle e^{-2 pi i c k1 / B}
-    FftPassArgs a1{P->d_u, P->d_v, P->d_tw, B, P->logB2, P->Lg * P->B2, B, B, 1, P->B2, 1, P->B2, 1,
-                   nullptr, nullptr, nullptr};
-    CK(launch_fft(P->B1, a1, P->fft_smem1, st));
-    // pass 2: B2-point FFTs of contiguous rows k1, out to u^[k1 + B1 k2] (+ cutoff keys)
-    FftPassArgs a2{P->d_v, reinterpret_cast<double2*>(myrec), P->d_tw, B, P->logB1, P->Lg * P->B1, B, rec_e,
-                   P->B2, 1, 1, P->B1, 0, keys ? P->d_key_index : nullptr, P->d_keys, P->d_hist};
-    CK(launch_fft(P->B2, a2, P->fft_smem2, st));
+  const SlotParam* sp = P->d_slots + (size_t)P->rank * P->Lg + s0;
+  ZeroArgs z{zero_block ? P->d_zero : nullptr, zero_block ? P->nzero : 0};
+  if (P->fused1) {
+    CK(launch_fold_fft1(P, x, sp, P->d_u + (size_t)s0 * B, P->d_v + (size_t)s0 * B, s1 - s0, z, st));
   } else {
-    FftPassArgs a{P->d_u, reinterpret_cast<double2*>(myrec), P->d_tw, B, 0, P->Lg, B, rec_e, 0, 1, 0, 1, 0,
-                  keys ? P->d_key_index : nullptr, P->d_keys, P->d_hist};
-    CK(launch_fft(P->B2, a, P->fft_smem2, st));
+    dim3 grid((B + 255) / 256, s1 - s0);
+    CK(launch_k(k_fold<16>, grid, dim3(256), P->fold_smem_pad, st, P->cur_prio, x, (const double*)P->d_taps, sp,
+                P->d_u + (size_t)s0 * B, B, P->w, P->R, (uint32_t)(P->n - 1), z));
   }
+  return CUSFFT_SUCCESS;
+}
+
+// Step 3 (remaining FFT passes, cutoff keys) for local slots [s0, s1).
+int launch_bfft(cusfft_plan_t P, int s0, int s1, cudaStream_t st) {
+  if (s1 <= s0) return CUSFFT_SUCCESS;
+  const int B = (int)P->B;
+  const int ns = s1 - s0;
+  double2* rec = reinterpret_cast<double2*>(P->d_records + ((int64_t)P->rank * P->Lg + s0) * P->lay.rec_bytes);
+  const int64_t rec_e = P->lay.rec_bytes / 16;
+  const int* kidx = P->sel_slots_h.empty() ? nullptr : P->d_key_index + s0;
+  if (P->B1 > 1) {
+    if (!P->fused1) {  // pass 1: B1-point FFTs over columns c (stride B2), twiddle e^{-2 pi i c k1 / B}
+      FftPassArgs a1{P->d_u + (size_t)s0 * B, P->d_v + (size_t)s0 * B, P->d_tw, B, P->logB2, ns * P->B2, B, B, 1,
+                     P->B2, 1, P->B2, 1, nullptr, nullptr, nullptr};
+      CK(launch_fft(P->B1, a1, P->fft_smem1, st, P->cur_prio));
+    }
+    // pass 2: B2-point FFTs of contiguous rows k1, out to u^[k1 + B1 k2] (+ cutoff keys)
+    FftPassArgs a2{P->d_v + (size_t)s0 * B, rec, P->d_tw, B, P->logB1, ns * P->B1, B, rec_e, P->B2, 1, 1, P->B1, 0,
+                   kidx, P->d_keys, P->d_hist};
+    CK(launch_fft(P->B2, a2, P->fft_smem2, st, P->cur_prio));
+  } else {
+    FftPassArgs a{P->d_u + (size_t)s0 * B, rec, P->d_tw, B, 0, ns, B, rec_e, 0, 1, 0, 1, 0, kidx, P->d_keys,
+                  P->d_hist};
+    CK(launch_fft(P->B2, a, P->fft_smem2, st, P->cur_prio));
+  }
+  return CUSFFT_SUCCESS;
+}
+
+// Step 4 for this rank's location slots.
+int launch_select(cusfft_plan_t P, cudaStream_t st) {
+  if (P->sel_slots_h.empty()) return CUSFFT_SUCCESS;
+  SelArgs sa{P->d_records, P->lay, P->d_sel_slots, (int)P->B, P->num, P->sel_S, P->d_keys, P->d_hist, P->d_hist1,
+             P->d_ckey, P->d_cidx, P->d_ccount, P->d_done, P->d_flags + 1};
+  CK(launch_k(k_select, dim3((int)P->sel_slots_h.size() * P->sel_S), dim3(kSelNT), P->select_smem, st, P->cur_prio,
+              sa));
+  return CUSFFT_SUCCESS;
+}
+
+int launch_local(cusfft_plan_t P, const double2* x) {
+  cudaStream_t st = P->stream;
+  int rc;
+  mark(P, 0);
+  if ((rc = launch_fold(P, x, 0, P->Lg, st, true))) return rc;
+  mark(P, 1);
+  if (P->stage_limit < 2) return CUSFFT_SUCCESS;
+  if ((rc = launch_bfft(P, 0, P->Lg, st))) return rc;
   mark(P, 2);
-  if (keys) {
-    k_select<<<(int)P->sel_slots_h.size(), 1024, P->select_smem, st>>>(P->d_records, P->lay, P->d_sel_slots, B,
-                                                                       P->num, P->d_keys, P->d_hist, P->d_flags + 1);
-    CKL();
-  }
+  if (P->stage_limit < 3) return CUSFFT_SUCCESS;
+  if ((rc = launch_select(P, st))) return rc;
   mark(P, 3);
   return CUSFFT_SUCCESS;
 }
 
-int launch_finish(cusfft_plan_t P, int64_t* locs, double2* vals) {
-  cudaStream_t st = P->stream;
+int launch_vote(cusfft_plan_t P, cudaStream_t st) {
   VoteArgs va;
   va.records = P->d_records;
   va.lay = P->lay;
@@ -548,15 +695,17 @@ int launch_finish(cusfft_plan_t P, int64_t* locs, double2* vals) {
   va.B = (int)P->B;
   va.nb = (int)P->nb;
   va.log2nb = P->log2nb;
-  va.P = P->vote_P;
-  va.log2P = ilog2(P->vote_P);
+  va.log2n = ilog2(P->n);
+  va.log2B = ilog2(P->B);
   va.nmask = (uint32_t)(P->n - 1);
   va.hits = P->d_hits;
   va.hit_count = reinterpret_cast<unsigned*>(P->d_flags);
   va.max_hits = P->max_hits;
-  k_vote<<<P->vote_grid, 256, P->vote_smem, st>>>(va);
-  CKL();
-  mark(P, 4);
+  CK(launch_k(k_vote, dim3(P->vote_grid), dim3(256), P->vote_smem, st, P->cur_prio, va));
+  return CUSFFT_SUCCESS;
+}
+
+int launch_estimate(cusfft_plan_t P, cudaStream_t st) {
   EstArgs ea;
   ea.records = P->d_records;
   ea.lay = P->lay;
@@ -574,31 +723,94 @@ int launch_finish(cusfft_plan_t P, int64_t* locs, double2* vals) {
   ea.hit_vals = P->d_hit_vals;
   ea.hit_keys = P->d_hit_keys;
   ea.per_loop = P->d_per_loop;
+  ea.out_hist = P->d_ohist;
   k_estimate<<<P->est_grid, 256, 0, st>>>(ea);
   CKL();
-  mark(P, 5);
+  return CUSFFT_SUCCESS;
+}
+
+int launch_output(cusfft_plan_t P, int64_t* locs, double2* vals, cudaStream_t st) {
   k_output<<<1, 1024, P->output_smem, st>>>(P->d_hits, reinterpret_cast<const unsigned*>(P->d_flags), P->max_hits,
-                                            P->d_hit_vals, P->d_hit_keys, (int)P->k, P->kp2, locs, vals,
-                                            P->d_flags + 1);
+                                            P->d_hit_vals, P->d_hit_keys, P->d_ohist, (int)P->k, P->kp2,
+                                            ilog2(P->n), locs, vals, P->d_flags + 1);
   CKL();
+  return CUSFFT_SUCCESS;
+}
+
+int launch_finish(cusfft_plan_t P, int64_t* locs, double2* vals) {
+  cudaStream_t st = P->stream;
+  int rc;
+  if (P->stage_limit < 4) return CUSFFT_SUCCESS;
+  if ((rc = launch_vote(P, st))) return rc;
+  mark(P, 4);
+  if (P->stage_limit < 5) return CUSFFT_SUCCESS;
+  if ((rc = launch_estimate(P, st))) return rc;
+  mark(P, 5);
+  if (P->stage_limit < 6) return CUSFFT_SUCCESS;
+  if ((rc = launch_output(P, locs, vals, st))) return rc;
   mark(P, 6);
   return CUSFFT_SUCCESS;
 }
 
+// The whole transform as two concurrent branches (graph capture only): the
+// location chain (fold, FFT, cutoff, vote of loops r < L_loc) on the plan's
+// high-priority capture stream, and the fold + FFT of the estimation-only
+// loops on a second stream; they join before the estimation.
+int launch_branched(cusfft_plan_t P, const double2* x, int64_t* locs, double2* vals) {
+  cudaStream_t a = P->stream, b = P->cap_stream2;
+  int rc;
+  // the location fold runs alone (all of DRAM); the estimation fold then
+  // overlaps the location chain's FFT, cutoff and vote
+  P->cur_prio = P->prio_hi;
+  if ((rc = launch_fold(P, x, 0, P->nloc_local, a, true))) return rc;
+  CK(cudaEventRecord(P->ev_fork, a));
+  CK(cudaStreamWaitEvent(b, P->ev_fork, 0));
+  P->cur_prio = P->prio_lo;
+  if ((rc = launch_fold(P, x, P->nloc_local, P->Lg, b, false))) return rc;
+  if ((rc = launch_bfft(P, P->nloc_local, P->Lg, b))) return rc;
+  CK(cudaEventRecord(P->ev_join, b));
+  P->cur_prio = P->prio_hi;
+  if ((rc = launch_bfft(P, 0, P->nloc_local, a))) return rc;
+  if ((rc = launch_select(P, a))) return rc;
+  if ((rc = launch_vote(P, a))) return rc;
+  P->cur_prio = 0;
+  CK(cudaStreamWaitEvent(a, P->ev_join, 0));
+  if ((rc = launch_estimate(P, a))) return rc;
+  return launch_output(P, locs, vals, a);
+}
+
+// Branched execution only inside graph capture, for full-stage runs with both
+// location and estimation-only slots on this rank.
+inline bool use_branches(cusfft_plan_t P) {
+  return P->branched && P->use_graph && !P->timing && P->stage_limit == 6 && P->nloc_local > 0 &&
+         P->nloc_local < P->Lg;
+}
 
 // Run `body` (which enqueues on P->stream) either directly or through a cached
 // CUDA graph captured on a plan-owned stream and launched on the caller's
-// stream.  Timing mode always launches directly (events between kernels).
+// stream.  In timing mode the graph also holds the stage event-record nodes.
 template <class F>
-int run_graphed(cusfft_plan_t P, cusfft_plan_s::GraphEntry& g, const void* a, const void* b, const void* c,
-                F&& body) {
+int run_graphed(cusfft_plan_t P, cusfft_plan_s::GraphEntry& g_plain, cusfft_plan_s::GraphEntry& g_timed, const void* a,
+                const void* b, const void* c, F&& body) {
+  // Timing mode launches directly: events recorded inside a graph cannot be timed.
   if (!P->use_graph || P->timing) return body();
-  if (!(g.exec && g.a == a && g.b == b && g.c == c)) {
+  (void)g_timed;
+  cusfft_plan_s::GraphEntry& g = g_plain;
+  if (!(g.exec && g.a == a && g.b == b && g.c == c && g.lim == P->stage_limit)) {
     if (g.exec) {
       cudaGraphExecDestroy(g.exec);
       g.exec = nullptr;
     }
-    if (!P->cap_stream) CK(cudaStreamCreateWithFlags(&P->cap_stream, cudaStreamNonBlocking));
+    if (!P->cap_stream) {
+      int lo = 0, hi = 0;
+      CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+      P->prio_lo = lo;
+      P->prio_hi = hi;
+      CK(cudaStreamCreateWithPriority(&P->cap_stream, cudaStreamNonBlocking, hi));   // location chain
+      CK(cudaStreamCreateWithPriority(&P->cap_stream2, cudaStreamNonBlocking, lo));  // estimation folds
+      CK(cudaEventCreateWithFlags(&P->ev_fork, cudaEventDisableTiming));
+      CK(cudaEventCreateWithFlags(&P->ev_join, cudaEventDisableTiming));
+    }
     CK(cudaStreamBeginCapture(P->cap_stream, cudaStreamCaptureModeThreadLocal));
     cudaStream_t user = P->stream;
     P->stream = P->cap_stream;
@@ -617,6 +829,7 @@ int run_graphed(cusfft_plan_t P, cusfft_plan_s::GraphEntry& g, const void* a, co
     g.a = a;
     g.b = b;
     g.c = c;
+    g.lim = P->stage_limit;
   }
   CK(cudaGraphLaunch(g.exec, P->stream));
   return CUSFFT_SUCCESS;
@@ -708,7 +921,7 @@ int cusfft_execute_local(cusfft_plan_t plan, const void* d_x) {
   if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
   if (!d_x) return CUSFFT_NULL_PTR;
   DeviceGuard g(plan->device);
-  return run_graphed(plan, plan->g_local, d_x, nullptr, nullptr,
+  return run_graphed(plan, plan->g_local, plan->g_local_t, d_x, nullptr, nullptr,
                      [&] { return launch_local(plan, reinterpret_cast<const double2*>(d_x)); });
 }
 
@@ -716,7 +929,7 @@ int cusfft_execute_finish(cusfft_plan_t plan, int64_t* d_locs, void* d_vals) {
   if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
   if (!d_locs || !d_vals) return CUSFFT_NULL_PTR;
   DeviceGuard g(plan->device);
-  return run_graphed(plan, plan->g_finish, d_locs, d_vals, nullptr,
+  return run_graphed(plan, plan->g_finish, plan->g_finish_t, d_locs, d_vals, nullptr,
                      [&] { return launch_finish(plan, d_locs, reinterpret_cast<double2*>(d_vals)); });
 }
 
@@ -725,10 +938,13 @@ int cusfft_execute(cusfft_plan_t plan, const void* d_x, int64_t* d_locs, void* d
   if (!d_x || !d_locs || !d_vals) return CUSFFT_NULL_PTR;
   if (plan->world != 1) return CUSFFT_INVALID_LOOPS;
   DeviceGuard g(plan->device);
-  return run_graphed(plan, plan->g_full, d_x, d_locs, d_vals, [&] {
-    int rc = launch_local(plan, reinterpret_cast<const double2*>(d_x));
+  return run_graphed(plan, plan->g_full, plan->g_full_t, d_x, d_locs, d_vals, [&] {
+    const double2* x = reinterpret_cast<const double2*>(d_x);
+    double2* v = reinterpret_cast<double2*>(d_vals);
+    if (use_branches(plan)) return launch_branched(plan, x, d_locs, v);
+    int rc = launch_local(plan, x);
     if (rc) return rc;
-    return launch_finish(plan, d_locs, reinterpret_cast<double2*>(d_vals));
+    return launch_finish(plan, d_locs, v);
   });
 }
 
@@ -756,7 +972,8 @@ int cusfft_execute_host(cusfft_plan_t plan, const void* h_x, int64_t* h_locs, vo
   }
   cudaStream_t st = plan->stream;
   CK(cudaMemcpyAsync(plan->d_xbuf, h_x, (size_t)plan->n * 16, cudaMemcpyHostToDevice, st));
-  rc = run_graphed(plan, plan->g_full, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf, [&] {
+  rc = run_graphed(plan, plan->g_full, plan->g_full_t, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf, [&] {
+    if (use_branches(plan)) return launch_branched(plan, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf);
     int r = launch_local(plan, plan->d_xbuf);
     if (r) return r;
     return launch_finish(plan, plan->d_locs_buf, plan->d_vals_buf);
@@ -877,15 +1094,36 @@ int cusfft_get_stage_times(cusfft_plan_t plan, float* ms, int32_t cap) {
   CK(cudaStreamSynchronize(plan->stream));
   for (int i = 0; i < 6 && i < cap; ++i) {
     float t = 0.f;
-    if (cudaEventElapsedTime(&t, plan->ev[i], plan->ev[i + 1]) != cudaSuccess) t = -1.f;
+    if (cudaEventElapsedTime(&t, plan->ev[i], plan->ev[i + 1]) != cudaSuccess) {
+      t = -1.f;
+      cudaGetLastError();  // do not leave a stale error for later launch checks
+    }
     ms[i] = t;
   }
   return CUSFFT_SUCCESS;
 }
 
+int cusfft_set_stage_limit(cusfft_plan_t plan, int32_t stages) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  if (stages < 1 || stages > 6) return CUSFFT_INVALID_PARAM;
+  plan->stage_limit = stages;
+  return CUSFFT_SUCCESS;
+}
+
+#ifdef CUSFFT_TRACE
+// Trace builds only (not part of include/cusfft.h): copy g_trace to host.
+int cusfft_debug_trace(unsigned long long* host, int32_t n) {
+  if (!host) return CUSFFT_NULL_PTR;
+  CK(cudaDeviceSynchronize());
+  CK(cudaMemcpyFromSymbol(host, g_trace, sizeof(unsigned long long) * (n < 256 ? n : 256)));
+  return CUSFFT_SUCCESS;
+}
+#endif
+
 int32_t cusfft_launches_per_execute(cusfft_plan_t plan) {
   if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
-  int n = 1 /*fold*/ + (plan->B1 > 1 ? 2 : 1) /*fft*/ + (plan->sel_slots_h.empty() ? 0 : 1) + 3 /*vote,est,out*/;
+  int n = 1 /*fold*/ + (plan->B1 > 1 && !plan->fused1 ? 2 : 1) /*fft*/ + (plan->sel_slots_h.empty() ? 0 : 1) +
+          3 /*vote,est,out*/;
   return n;
 }
 

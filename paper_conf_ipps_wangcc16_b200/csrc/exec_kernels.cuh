@@ -20,6 +20,22 @@ namespace cusfft {
 // All RC gathers of a chunk are issued before the first add (memory-level
 // parallelism); gathers use the non-coherent path without L1 allocation.
 // ---------------------------------------------------------------------------
+// Per-execution block zeroed by the CTAs of the first fold launch (the fold is
+// memory-latency bound, so the stores are free): flags, histograms, counters.
+struct ZeroArgs {
+  int* p;
+  int n;
+};
+
+__device__ __forceinline__ void zero_part(const ZeroArgs& z) {
+  if (!z.p) return;
+  const int nblk = gridDim.x * gridDim.y;
+  const int blk = blockIdx.y * gridDim.x + blockIdx.x;
+  const int chunk = (z.n + nblk - 1) / nblk;
+  const int b = blk * chunk, e = min(z.n, b + chunk);
+  for (int i = b + threadIdx.x; i < e; i += blockDim.x) z.p[i] = 0;
+}
+
 __device__ __forceinline__ double2 ld_gather(const double2* p) {
   double2 v;
   asm volatile("ld.global.nc.L1::no_allocate.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
@@ -29,9 +45,11 @@ __device__ __forceinline__ double2 ld_gather(const double2* p) {
 template <int RC>
 __global__ void __launch_bounds__(256) k_fold(const double2* __restrict__ x, const double* __restrict__ taps,
                                               const SlotParam* __restrict__ slots, double2* __restrict__ u,
-                                              int B, int w, int R, uint32_t nmask) {
+                                              int B, int w, int R, uint32_t nmask, ZeroArgs zero) {
   const int j = blockIdx.x * blockDim.x + threadIdx.x;
   const int s = blockIdx.y;
+  if (blockIdx.x == 0 && blockIdx.y == 0) TRACE(0);
+  zero_part(zero);
   if (j >= B) return;
   const uint32_t sigma = slots[s].sigma, tau = slots[s].tau;
   double ar = 0.0, ai = 0.0;
@@ -57,6 +75,68 @@ __global__ void __launch_bounds__(256) k_fold(const double2* __restrict__ x, con
     }
   }
   u[(size_t)s * B + j] = make_double2(ar, ai);
+  TRACE_END(1);
+}
+
+// ---------------------------------------------------------------------------
+// Steps 1+2 fused with the first pass of Step 3 (four-step B = B1 x B2, B1 <=
+// 256): a CTA of 256 threads folds the buckets of C = 256 / B1 whole columns
+// c (j = c + B2 j1, j1 < B1) exactly as k_fold does (same per-bucket order),
+// writes u (kept for parity checks), then runs the C B1-point FFTs in shared
+// memory and writes v[c + B2 k1] = FFT(...)[k1] * e^{-2 pi i c k1 / B}, which
+// is what the stand-alone pass 1 produces.  Taps are read from a plan-time
+// permutation taps_perm[rr B + cta 256 + t] = g[j(t) + rr B] so that the tap
+// loads of a CTA stay contiguous.  RC gathers per thread in flight; two CTAs
+// per SM so one CTA's FFT epilogue overlaps the other's gathers.
+// ---------------------------------------------------------------------------
+template <int B1T, int RC>
+__global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict__ x,
+                                                      const double* __restrict__ taps_perm,
+                                                      const SlotParam* __restrict__ slots, double2* __restrict__ u,
+                                                      double2* __restrict__ v, const double2* __restrict__ tw, int B,
+                                                      int B2, int w, int R, uint32_t nmask, ZeroArgs zero) {
+  constexpr int C = 256 / B1T;
+  __shared__ double2 S[256 + 256 / 8];
+  __shared__ double2 twl[B1T];
+  const int t = threadIdx.x;
+  const int s = blockIdx.y;
+  if (blockIdx.x == 0 && blockIdx.y == 0) TRACE(0);
+  const int cl = t / B1T, j1 = t % B1T;
+  const int c = blockIdx.x * C + cl;
+  const int j = c + B2 * j1;
+  zero_part(zero);
+  for (int i = t; i < B1T; i += 256) twl[i] = __ldg(tw + (int64_t)i * B2);  // omega_B1^i
+  const double2 wout = __ldg(tw + (((int64_t)c * j1) & (B - 1)));          // omega_B^(c k1), k1 = j1
+  const uint32_t sigma = slots[s].sigma, tau = slots[s].tau;
+  const double* tp = taps_perm + (int64_t)blockIdx.x * 256 + t;
+  double ar = 0.0, ai = 0.0;
+  for (int r0 = 0; r0 < R; r0 += RC) {
+    double2 xv[RC];
+    double g[RC];
+#pragma unroll
+    for (int cc = 0; cc < RC; ++cc) {
+      const int i = j + (r0 + cc) * B;
+      if (r0 + cc < R && i < w) {
+        const uint32_t idx = (sigma * (uint32_t)i + tau) & nmask;  // mod n, n | 2^32
+        xv[cc] = ld_gather(x + idx);
+        g[cc] = __ldg(tp + (int64_t)(r0 + cc) * B);
+      }
+    }
+#pragma unroll
+    for (int cc = 0; cc < RC; ++cc) {
+      const int i = j + (r0 + cc) * B;
+      if (r0 + cc < R && i < w) {
+        ar = __dadd_rn(ar, __dmul_rn(g[cc], xv[cc].x));
+        ai = __dadd_rn(ai, __dmul_rn(g[cc], xv[cc].y));
+      }
+    }
+  }
+  u[(size_t)s * B + j] = make_double2(ar, ai);
+  S[fft_pad(cl * B1T + j1)] = make_double2(ar, ai);
+  __syncthreads();
+  fft_smem<B1T, 256, 256, true>(S, twl, B1T);
+  v[(size_t)s * B + c + (size_t)B2 * j1] = cmul(S[fft_pad(cl * B1T + j1)], wout);
+  TRACE_END(1);
 }
 
 // ---------------------------------------------------------------------------
@@ -85,126 +165,307 @@ struct PairSrc {  // (key, index) pairs; the index is the tie-break
   }
 };
 
-// ---------------------------------------------------------------------------
-// Step 4 (L89, Alg. 3 L238-L250; the linear-time selection of §V.B L353-L390,
-// made exact): J_r = the num buckets of largest |u^|^2 = re*re + im*im, ties
-// to the smaller bucket, as a bitmap and an ascending list.  One CTA of 1024
-// threads per location slot of this rank.
-//  1. the FFT epilogue already counted keys per top-12-bit digit: a block scan
-//     of that histogram gives the boundary digit d0 and the count above it;
-//  2. one pass over the B keys: digit > d0 -> selected, digit == d0 -> smem
-//     candidate list;
-//  3. exact 96-bit radix select (key, ~bucket) among the candidates.
-// Falls back to a full radix select over all keys when the boundary bin holds
-// more than kSelCap candidates.  Resets the histogram for the next execution.
-// Dynamic smem: 4096 u32 hist + 64 int + kSelCap x (u64 + int).
-// ---------------------------------------------------------------------------
-constexpr int kSelCap = 4096;
-
-__global__ void __launch_bounds__(1024) k_select(uint8_t* __restrict__ records, RecLayout lay,
-                                                 const int* __restrict__ sel_slots, int B, int num,
-                                                 const uint64_t* __restrict__ gkeys, uint32_t* __restrict__ ghist,
-                                                 int* __restrict__ status) {
-  extern __shared__ __align__(16) uint8_t smem[];
-  uint32_t* hist = reinterpret_cast<uint32_t*>(smem);
-  int* sm = reinterpret_cast<int*>(smem + 4096 * 4);
-  uint64_t* ckey = reinterpret_cast<uint64_t*>(smem + 4096 * 4 + 64 * 4);
-  int* cidx = reinterpret_cast<int*>(ckey + kSelCap);
+// Two-level top-K selection shared by the cutoff and the output selection
+// (blockDim.x == 1024).  Level 0: the producer kernel counted the items per
+// top digit (pass 0) into `ghist` (global, reset here).  One pass over the N
+// items (key(i), tie(i)) then accepts every item above the boundary digit
+// (on_sel(i)), keeps the boundary bin's items as smem candidates and counts
+// their pass-1 digits; a radix select among the candidates (usually one
+// histogram scan) finishes the job.  Falls back to a full radix select when the
+// boundary bin holds more than `cap` items.  hist: 4096 u32 smem; sm >= 64 ints.
+template <class KeyAt, class OnSel>
+__device__ void select_topk(int N, int K, uint32_t* ghist, KeyAt key_at, OnSel on_sel, uint64_t* ckey, int* cidx,
+                            int cap, uint32_t* hist, int* sm) {
   const int tid = threadIdx.x;
-  const int sel = blockIdx.x;
-  uint8_t* rec = records + (int64_t)sel_slots[sel] * lay.rec_bytes;
-  uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + lay.off_bitmap);
-  int* J = reinterpret_cast<int*>(rec + lay.off_J);
-  const uint64_t* keys = gkeys + (int64_t)sel * B;
-  uint32_t* gh = ghist + (int64_t)sel * 4096;
-  const int words = (B + 31) >> 5;
-
-  // 1. boundary digit from the histogram (thread t owns bins 4095-4t .. 4092-4t)
-  const int base = 4095 - 4 * tid;
-  const int c0 = gh[base], c1 = gh[base - 1], c2 = gh[base - 2], c3 = gh[base - 3];
-  const int mine = c0 + c1 + c2 + c3;
-  int total;
-  const int ex = block_excl_scan<1024>(mine, &total, sm);
-  if (ex < num && num <= ex + mine) {
-    int cum = ex, d, cnt;
-    if (cum + c0 >= num) {
-      d = base; cnt = c0;
-    } else if ((cum += c0) + c1 >= num) {
-      d = base - 1; cnt = c1;
-    } else if ((cum += c1) + c2 >= num) {
-      d = base - 2; cnt = c2;
-    } else {
-      cum += c2; d = base - 3; cnt = c3;
-    }
-    sm[32] = d; sm[33] = cum; sm[34] = cnt;
-  }
-  gh[base] = 0; gh[base - 1] = 0; gh[base - 2] = 0; gh[base - 3] = 0;  // self-reset
-  for (int w = tid; w < words; w += 1024) bitmap[w] = 0;
+  const BinPick b0 = pick_bin(ghist, K, sm);
+  for (int i = tid; i < 4096; i += 1024) hist[i] = 0;
   if (tid == 0) sm[40] = 0;
   __syncthreads();
-  const uint32_t d0 = (uint32_t)sm[32];
-  const int above = sm[33], cnt0 = sm[34];
-  const int k2 = num - above;  // 1 <= k2 <= cnt0
-  const bool whole_bin = (k2 == cnt0);
-  // 2. one pass over the keys, 16 loads in flight per thread
-  for (int i0 = 0; i0 < B; i0 += 16 * 1024) {
-    uint64_t kb[16];
+  const uint32_t d0 = (uint32_t)b0.d;
+  const int k2 = K - b0.above;  // 1 <= k2 <= b0.cnt
+  const bool whole = (k2 == b0.cnt);
+  const int shift1 = pass_shift(1);
+  for (int i0 = 0; i0 < N; i0 += 8 * 1024) {
+    uint64_t kb[8];
+    uint32_t tb[8];
 #pragma unroll
-    for (int u = 0; u < 16; ++u) {
+    for (int u = 0; u < 8; ++u) {
       const int i = i0 + u * 1024 + tid;
-      kb[u] = i < B ? __ldg(keys + i) : 0ull;
+      if (i < N) key_at(i, kb[u], tb[u]);
     }
 #pragma unroll
-    for (int u = 0; u < 16; ++u) {
+    for (int u = 0; u < 8; ++u) {
       const int i = i0 + u * 1024 + tid;
-      if (i >= B) continue;
+      if (i >= N) continue;
       const uint32_t d = (uint32_t)(kb[u] >> 51) & 0xFFFu;
-      if (d > d0 || (d == d0 && whole_bin)) {
-        atomicOr(&bitmap[i >> 5], 1u << (i & 31));
+      if (d > d0 || (d == d0 && whole)) {
+        on_sel(i);
       } else if (d == d0) {
         const int pos = atomicAdd(&sm[40], 1);
-        if (pos < kSelCap) {
+        if (pos < cap) {
           ckey[pos] = kb[u];
           cidx[pos] = i;
         }
+        atomicAdd(&hist[digit96(kb[u], ~tb[u], shift1)], 1u);
       }
     }
   }
   __syncthreads();
-  if (!whole_bin) {
-    const int nc = sm[40];
-    if (nc <= kSelCap) {
-      const Prefix96 p = block_radix_select(PairSrc{ckey, cidx}, nc, k2, hist, sm);
-      for (int c = tid; c < nc; c += 1024)
-        if (ge96(p, ckey[c], ~(uint32_t)cidx[c])) atomicOr(&bitmap[cidx[c] >> 5], 1u << (cidx[c] & 31));
-    } else {  // crowded boundary bin: exact select over all keys
-      const Prefix96 p = block_radix_select(KeysSrc{keys}, B, num, hist, sm);
-      for (int w = tid; w < words; w += 1024) {
-        uint32_t bits = 0;
-        for (int b = 0; b < 32; ++b) {
-          const int i = w * 32 + b;
-          if (i < B && ge96(p, keys[i], ~(uint32_t)i)) bits |= 1u << b;
+  if (whole) return;
+  const int nc = sm[40];
+  Prefix96 p{0, 0, 0, 0};
+  or96(p.phi, p.plo, d0, pass_shift(0));
+  or96(p.mhi, p.mlo, 0xFFFu, pass_shift(0));
+  if (nc <= 1024 && nc <= cap) {  // few candidates: exact rank counting, one pass
+    uint64_t mk = 0;
+    uint32_t mt = 0;
+    if (tid < nc) {
+      mk = ckey[tid];
+      uint64_t kk;
+      key_at(cidx[tid], kk, mt);
+      cidx[cap - 1 - tid] = (int)mt;  // tie values, stored from the top of cidx
+    }
+    __syncthreads();
+    if (tid < nc) {
+      int rank = 0;  // preferred: larger key, or equal key and smaller tie value
+      for (int c = 0; c < nc; ++c) {
+        const uint64_t kc = ckey[c];
+        rank += (kc > mk) || (kc == mk && (uint32_t)cidx[cap - 1 - c] < mt);
+      }
+      if (rank < k2) on_sel(cidx[tid]);
+    }
+    __syncthreads();
+  } else if (nc <= cap) {
+    struct CandSrc {
+      const uint64_t* k;
+      const int* c;
+      KeyAt ka;
+      __device__ __forceinline__ void get(int j, uint64_t& hi, uint32_t& lo) const {
+        uint32_t t;
+        uint64_t kk;
+        ka(c[j], kk, t);
+        hi = k[j];
+        lo = ~t;
+      }
+    };
+    p = block_radix_select(CandSrc{ckey, cidx, key_at}, nc, k2, hist, sm, 1, p, true);
+    for (int c = tid; c < nc; c += 1024) {
+      uint64_t kk;
+      uint32_t t;
+      key_at(cidx[c], kk, t);
+      if (ge96(p, kk, ~t)) on_sel(cidx[c]);
+    }
+  } else {  // crowded boundary bin: radix over all items matching the level-0 digit
+    struct AllSrc {
+      KeyAt ka;
+      __device__ __forceinline__ void get(int j, uint64_t& hi, uint32_t& lo) const {
+        uint32_t t;
+        ka(j, hi, t);
+        lo = ~t;
+      }
+    };
+    p = block_radix_select(AllSrc{key_at}, N, k2, hist, sm, 1, p, true);
+    for (int i = tid; i < N; i += 1024) {
+      uint64_t kk;
+      uint32_t t;
+      key_at(i, kk, t);
+      if (((kk >> 51) & 0xFFFu) == d0 && ge96(p, kk, ~t)) on_sel(i);
+    }
+  }
+  __syncthreads();
+}
+
+// ---------------------------------------------------------------------------
+// Step 4 (L89, Alg. 3 L238-L250; the linear-time selection of §V.B L353-L390,
+// made exact): J_r = the num buckets of largest |u^|^2 = re*re + im*im, ties
+// to the smaller bucket, as a bitmap and an ascending list.
+// Grid: S CTAs of 256 threads per location slot of this rank.  Level 0 (the
+// top 12 key bits below the sign) was counted by the FFT epilogue; every CTA
+// reads it, finds the boundary digit d0, and scans B/S keys, one warp per 32
+// keys: a ballot of "digit > d0" is the bitmap word; boundary-bin keys go to a
+// per-loop global candidate list and their next 12 bits to a level-1
+// histogram.  The last CTA of the loop (threadfence + counter) resolves the
+// boundary bin exactly (radix select from pass 1), ORs those bits in, resets
+// the loop's counters and histograms, and writes the ascending winner list.
+// ---------------------------------------------------------------------------
+constexpr int kSelCap = 4096;
+constexpr int kSelNT = 256;
+
+struct SelArgs {
+  uint8_t* records;
+  RecLayout lay;
+  const int* sel_slots;
+  int B, num, S;
+  const uint64_t* keys;  // [n_sel][B]
+  uint32_t* hist0;       // [n_sel][4096] (FFT epilogue)
+  uint32_t* hist1;       // [n_sel][4096]
+  uint64_t* ckey;        // [n_sel][kSelCap]
+  int* cidx;             // [n_sel][kSelCap]
+  int* ccount;           // [n_sel]
+  int* done;             // [n_sel]
+  int* status;
+};
+
+struct GKeySrc {
+  const uint64_t* keys;
+  __device__ __forceinline__ void get(int i, uint64_t& hi, uint32_t& lo) const {
+    hi = __ldcg(keys + i);
+    lo = ~(uint32_t)i;
+  }
+};
+
+__global__ void __launch_bounds__(kSelNT) k_select(SelArgs A) {
+  extern __shared__ __align__(16) uint8_t smem[];
+  uint32_t* hist = reinterpret_cast<uint32_t*>(smem);
+  int* sm = reinterpret_cast<int*>(smem + 4096 * 4);
+  uint64_t* skey = reinterpret_cast<uint64_t*>(smem + 4096 * 4 + 64 * 4);
+  int* sidx = reinterpret_cast<int*>(skey + kSelCap);
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int sel = blockIdx.x / A.S, part = blockIdx.x - sel * A.S;
+  uint8_t* rec = A.records + (int64_t)A.sel_slots[sel] * A.lay.rec_bytes;
+  uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap);
+  const uint64_t* keys = A.keys + (int64_t)sel * A.B;
+  uint32_t* h0 = A.hist0 + (int64_t)sel * 4096;
+  uint32_t* h1 = A.hist1 + (int64_t)sel * 4096;
+  const int words = (A.B + 31) >> 5;
+  if (blockIdx.x == 0) TRACE(10);
+  const BinPick b0 = pick_bin<kSelNT>(h0, A.num, sm);
+  if (blockIdx.x == 0) TRACE(11);
+  const uint32_t d0 = (uint32_t)b0.d;
+  const int k2 = A.num - b0.above;
+  const bool whole = (k2 == b0.cnt);
+  // this CTA's words
+  const int wpc = (words + A.S - 1) / A.S;
+  const int w_begin = part * wpc, w_end = min(words, w_begin + wpc);
+  for (int w0 = w_begin + wid; w0 < w_end; w0 += 8 * (kSelNT / 32)) {
+    uint64_t kb[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {  // 8 words' keys in flight per warp
+      const int w = w0 + u * (kSelNT / 32), i = w * 32 + lane;
+      kb[u] = (w < w_end && i < A.B) ? __ldg(keys + i) : 0ull;
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int w = w0 + u * (kSelNT / 32), i = w * 32 + lane;
+      if (w >= w_end) break;
+      const uint32_t d = (uint32_t)(kb[u] >> 51) & 0xFFFu;
+      const bool take = i < A.B && (d > d0 || (d == d0 && whole));
+      const bool cand = i < A.B && d == d0 && !whole;
+      const uint32_t word = __ballot_sync(kFull, take);
+      if (lane == 0) bitmap[w] = word;
+      if (cand) {
+        const int pos = atomicAdd(A.ccount + sel, 1);
+        if (pos < kSelCap) {
+          A.ckey[(int64_t)sel * kSelCap + pos] = kb[u];
+          A.cidx[(int64_t)sel * kSelCap + pos] = i;
         }
-        bitmap[w] = bits;
+        atomicAdd(h1 + digit96(kb[u], ~(uint32_t)i, pass_shift(1)), 1u);
       }
     }
   }
+  if (blockIdx.x == 0) TRACE(12);
+  __threadfence();
   __syncthreads();
-  // 3. ascending winner list from the bitmap
-  const int wpt = (words + 1023) >> 10;
+  if (blockIdx.x == 0) TRACE(13);
+  if (tid == 0) sm[40] = atomicAdd(A.done + sel, 1);
+  __syncthreads();
+  if (blockIdx.x == 0) TRACE(14);
+  if (sm[40] != A.S - 1) return;  // not the last CTA of this loop
+  __threadfence();
+  if (sel == 0) TRACE(20);
+  // ---- finalize (last CTA of the loop)
+  if (!whole) {
+    const int nc = __ldcg(A.ccount + sel);
+    if (nc > kSelNT) {  // level-1 histogram for the radix paths, 16 loads in flight per thread
+      uint32_t hb[4096 / kSelNT];
+#pragma unroll
+      for (int u = 0; u < 4096 / kSelNT; ++u) hb[u] = __ldcg(h1 + tid + u * kSelNT);
+#pragma unroll
+      for (int u = 0; u < 4096 / kSelNT; ++u) hist[tid + u * kSelNT] = hb[u];
+    }
+    Prefix96 p{0, 0, 0, 0};
+    or96(p.phi, p.plo, d0, pass_shift(0));
+    or96(p.mhi, p.mlo, 0xFFFu, pass_shift(0));
+    if (nc <= kSelNT) {  // few candidates: exact rank counting, one pass
+      uint64_t mk = 0;
+      int mi = 0x7FFFFFFF;
+      if (tid < nc) {
+        mk = __ldcg(A.ckey + (int64_t)sel * kSelCap + tid);
+        mi = __ldcg(A.cidx + (int64_t)sel * kSelCap + tid);
+        skey[tid] = mk;
+        sidx[tid] = mi;
+      }
+      __syncthreads();
+      if (tid < nc) {
+        int rank = 0;  // candidates preferred to mine: larger key, or equal key and smaller bucket
+        for (int c = 0; c < nc; ++c) rank += (skey[c] > mk) || (skey[c] == mk && sidx[c] < mi);
+        if (rank < k2) atomicOr(&bitmap[mi >> 5], 1u << (mi & 31));
+      }
+    } else if (nc <= kSelCap) {
+      for (int c0 = 0; c0 < nc; c0 += 4 * kSelNT) {
+        uint64_t kb[4];
+        int ib[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int c = c0 + u * kSelNT + tid;
+          if (c < nc) {
+            kb[u] = __ldcg(A.ckey + (int64_t)sel * kSelCap + c);
+            ib[u] = __ldcg(A.cidx + (int64_t)sel * kSelCap + c);
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const int c = c0 + u * kSelNT + tid;
+          if (c < nc) {
+            skey[c] = kb[u];
+            sidx[c] = ib[u];
+          }
+        }
+      }
+      __syncthreads();
+      p = block_radix_select<PairSrc, kSelNT>(PairSrc{skey, sidx}, nc, k2, hist, sm, 1, p, true);
+      for (int c = tid; c < nc; c += kSelNT)
+        if (ge96(p, skey[c], ~(uint32_t)sidx[c])) atomicOr(&bitmap[sidx[c] >> 5], 1u << (sidx[c] & 31));
+    } else {  // crowded boundary bin: radix over every key matching d0
+      __syncthreads();
+      p = block_radix_select<GKeySrc, kSelNT>(GKeySrc{keys}, A.B, k2, hist, sm, 1, p, true);
+      for (int i = tid; i < A.B; i += kSelNT) {
+        const uint64_t kk = __ldcg(keys + i);
+        if (((kk >> 51) & 0xFFFu) == d0 && ge96(p, kk, ~(uint32_t)i)) atomicOr(&bitmap[i >> 5], 1u << (i & 31));
+      }
+    }
+  }
+  if (sel == 0) TRACE(21);
+  __syncthreads();
+  // ascending winner list
+  int* J = reinterpret_cast<int*>(rec + A.lay.off_J);
+  const int wpt = (words + kSelNT - 1) / kSelNT;
+  constexpr int kWB = 8;  // words held in registers per thread (B <= 65536)
+  uint32_t wb[kWB];
   int cnt = 0;
-  for (int w = tid * wpt; w < min(words, (tid + 1) * wpt); ++w) cnt += __popc(bitmap[w]);
-  int pos = block_excl_scan<1024>(cnt, &total, sm);
+#pragma unroll
+  for (int u = 0; u < kWB; ++u) {
+    const int w = tid * wpt + u;
+    wb[u] = (u < wpt && w < words) ? __ldcg(bitmap + w) : 0u;
+  }
+  for (int w = tid * wpt + kWB; w < min(words, (tid + 1) * wpt); ++w) cnt += __popc(__ldcg(bitmap + w));
+#pragma unroll
+  for (int u = 0; u < kWB; ++u) cnt += __popc(wb[u]);
+  int total;
+  int pos = block_excl_scan<kSelNT>(cnt, &total, sm);
   for (int w = tid * wpt; w < min(words, (tid + 1) * wpt); ++w) {
-    uint32_t bits = bitmap[w];
+    const int u = w - tid * wpt;
+    uint32_t bits = u < kWB ? wb[u] : __ldcg(bitmap + w);
     while (bits) {
       const int b = __ffs(bits) - 1;
       bits &= bits - 1;
-      if (pos < num) J[pos] = w * 32 + b;
+      if (pos < A.num) J[pos] = w * 32 + b;
       ++pos;
     }
   }
-  if (tid == 0 && total != num) atomicOr(status + 1, 1);
+  if (tid == 0 && total != A.num) atomicOr(A.status + 1, 1);
+  if (sel == 0) TRACE(22);
+  TRACE_END(15);
 }
 
 // ---------------------------------------------------------------------------
@@ -212,10 +473,11 @@ __global__ void __launch_bounds__(1024) k_select(uint8_t* __restrict__ records, 
 // is Alg. 4's range [ceil((J-1/2) nb), ceil((J+1/2) nb)).  A frequency with
 // >= T of L_loc votes is selected in at least one of the first L_loc - T + 1
 // location loops, so candidates f = a_{q0} p are enumerated only from those
-// loops' preimage ranges, and f is counted at the first loop q0 that selects
-// it: it needs T-1 votes among the loops after q0 (probed first: a random
-// candidate is rejected after L_loc - T - q0 + 1 misses) and no vote before
-// q0 (probed last, for the rare survivors).
+// loops' preimage ranges, one warp per (q0, J) range, and f is counted at the
+// first loop q0 that selects it: it needs T-1 votes among the later loops and
+// none before q0.  The first min(L_loc-T-q0+1, later) later loops are probed
+// branch-free (if all miss, f is rejected); the rare survivors probe the rest
+// and then check the earlier loops.
 // Dynamic smem: L_loc * ceil(B/32) u32 bitmaps.
 // ---------------------------------------------------------------------------
 struct VoteArgs {
@@ -224,17 +486,135 @@ struct VoteArgs {
   const int* loc_slots;  // [L_loc] slot of each location loop, in vote order
   const uint32_t* loc_sigma;
   const uint32_t* loc_a;
-  int Lloc, T, num, B, nb, log2nb, P, log2P;
+  int Lloc, T, num, B, nb, log2nb, log2n, log2B;
   uint32_t nmask;
   int* hits;
   unsigned* hit_count;
   int max_hits;
 };
 
+// Scaled arithmetic: with F = f << (32 - log2 n), sigma * F + (nb/2 << (32 - log2 n))
+// wraps at 2^32 exactly like (sigma f + nb/2) mod n scaled, so the bucket is
+// the top log2 B bits: one IMAD + one shift, no mask.
+__device__ __forceinline__ uint32_t probe_s(const uint32_t* row, uint32_t sig, uint32_t F, uint32_t half_s, int bsh) {
+  const uint32_t b = (sig * F + half_s) >> bsh;
+  return (row[b >> 5] >> (b & 31)) & 1u;
+}
+
+// Survivors of the mandatory probes finish here, one per lane (convergent):
+// the remaining later loops and the "no vote before q0" check.
+__device__ __forceinline__ bool vote_finish(const VoteArgs& A, const uint32_t* bm, const uint32_t* ssig, int words,
+                                            int q0, int m, uint32_t F, int got, uint32_t half_s, int bsh) {
+  int votes = got;
+  for (int q = q0 + 1 + m; q < A.Lloc; ++q) votes += probe_s(bm + q * words, ssig[q], F, half_s, bsh);
+  bool hit = votes >= A.T - 1;
+  for (int q = 0; q < q0; ++q) hit = hit && !probe_s(bm + q * words, ssig[q], F, half_s, bsh);
+  return hit;
+}
+
+__device__ __forceinline__ void vote_emit(const VoteArgs& A, bool hit, uint32_t f) {
+  const int lane = threadIdx.x & 31;
+  const unsigned ball = __ballot_sync(kFull, hit);
+  if (ball) {
+    unsigned base = 0;
+    const int leader = __ffs(ball) - 1;
+    if (lane == leader) base = atomicAdd(A.hit_count, (unsigned)__popc(ball));
+    base = __shfl_sync(kFull, base, leader);
+    if (hit) {
+      const unsigned slot = base + __popc(ball & ((1u << lane) - 1));
+      if ((int)slot < A.max_hits) A.hits[slot] = (int)f;
+    }
+  }
+}
+
+// One (q0, J) preimage range per warp, two candidates per lane per step.
+// M = mandatory probes (compile time; M == 0: runtime count mrt).  Survivors
+// of the mandatory probes are queued in shared memory (qF: scaled f, qG:
+// votes so far) and finished 32 at a time (convergent).
+template <int M>
+__device__ __forceinline__ void vote_unit(const VoteArgs& A, const uint32_t* __restrict__ bm, const uint32_t* ssig,
+                                          int words, int q0, uint32_t Jv, uint32_t a, int mrt, uint32_t* qF,
+                                          uint8_t* qG) {
+  constexpr int MM = M > 0 ? M : 1;
+  const int lane = threadIdx.x & 31;
+  const int sh = 32 - A.log2n, bsh = 32 - A.log2B;
+  const uint32_t half = (uint32_t)(A.nb >> 1);
+  const uint32_t half_s = half << sh;
+  const int m = M > 0 ? M : mrt;
+  const int allowed = A.Lloc - A.T - q0;
+  int base[MM];
+  uint32_t sg[MM];
+#pragma unroll
+  for (int qq = 0; qq < MM; ++qq) {
+    base[qq] = (q0 + 1 + qq) * words;
+    sg[qq] = ssig[q0 + 1 + qq];
+  }
+  const uint32_t p0 = Jv * (uint32_t)A.nb - half;
+  uint32_t F0 = a * ((p0 + (uint32_t)lane) << sh);
+  const uint32_t d32 = a * (32u << sh);
+  const uint32_t d64 = a * (64u << sh);
+  int qn = 0;  // queued survivors (warp-uniform)
+  for (int t0 = 0; t0 < A.nb; t0 += 64, F0 += d64) {
+    const uint32_t F1 = F0 + d32;
+    int g0 = 0, g1 = 0;
+    if (M > 0) {
+#pragma unroll
+      for (int qq = 0; qq < MM; ++qq) {
+        const uint32_t b0 = (sg[qq] * F0 + half_s) >> bsh;
+        const uint32_t b1 = (sg[qq] * F1 + half_s) >> bsh;
+        g0 += (bm[base[qq] + (b0 >> 5)] >> (b0 & 31)) & 1u;
+        g1 += (bm[base[qq] + (b1 >> 5)] >> (b1 & 31)) & 1u;
+      }
+    } else {
+      for (int qq = 0; qq < m; ++qq) {
+        g0 += probe_s(bm + (q0 + 1 + qq) * words, ssig[q0 + 1 + qq], F0, half_s, bsh);
+        g1 += probe_s(bm + (q0 + 1 + qq) * words, ssig[q0 + 1 + qq], F1, half_s, bsh);
+      }
+    }
+    const bool s0 = (t0 + lane < A.nb) && (m - g0) <= allowed;
+    const bool s1 = (t0 + 32 + lane < A.nb) && (m - g1) <= allowed;
+    const unsigned b0 = __ballot_sync(kFull, s0);
+    const unsigned b1 = __ballot_sync(kFull, s1);
+    const unsigned lt = (1u << lane) - 1;
+    if (s0) {
+      const int pos = qn + __popc(b0 & lt);
+      qF[pos] = F0;
+      qG[pos] = (uint8_t)g0;
+    }
+    const int qn1 = qn + __popc(b0);
+    if (s1) {
+      const int pos = qn1 + __popc(b1 & lt);
+      qF[pos] = F1;
+      qG[pos] = (uint8_t)g1;
+    }
+    qn = qn1 + __popc(b1);
+    __syncwarp();
+    while (qn >= 32) {  // finish 32 queued survivors, one per lane
+      const uint32_t Fq = qF[qn - 32 + lane];
+      const int gq = qG[qn - 32 + lane];
+      __syncwarp();
+      qn -= 32;
+      const bool hit = vote_finish(A, bm, ssig, words, q0, m, Fq, gq, half_s, bsh);
+      vote_emit(A, hit, Fq >> sh);
+    }
+  }
+  if (qn > 0) {
+    const bool has = lane < qn;
+    const uint32_t Fq = has ? qF[lane] : 0u;
+    const int gq = has ? qG[lane] : 0;
+    __syncwarp();
+    const bool hit = has && vote_finish(A, bm, ssig, words, q0, m, Fq, gq, half_s, bsh);
+    vote_emit(A, hit, Fq >> sh);
+  }
+}
+
 __global__ void __launch_bounds__(256) k_vote(VoteArgs A) {
   extern __shared__ __align__(16) uint8_t smem[];
+  if (blockIdx.x == 0) TRACE(30);
   uint32_t* bm = reinterpret_cast<uint32_t*>(smem);
   __shared__ uint32_t ssig[64];
+  __shared__ uint32_t queueF[8][96];
+  __shared__ uint8_t queueG[8][96];
   const int words = (A.B + 31) >> 5;
   if ((words & 3) == 0) {  // 16-B vector loads, 8 in flight per thread
     const int v4 = words >> 2, tot = A.Lloc * v4;
@@ -265,67 +645,31 @@ __global__ void __launch_bounds__(256) k_vote(VoteArgs A) {
   }
   if (threadIdx.x < A.Lloc) ssig[threadIdx.x] = A.loc_sigma[threadIdx.x];
   __syncthreads();
-  const int lane = threadIdx.x & 31;
-  const int log_cpj = A.log2nb - A.log2P;  // chunks per bucket = nb / P
-  const int per_q = A.num << log_cpj;
-  const int items = (A.Lloc - A.T + 1) * per_q;
-  const uint32_t half = (uint32_t)(A.nb >> 1);
-  const int stride = gridDim.x * blockDim.x;
-  const int warp_start = blockIdx.x * blockDim.x + threadIdx.x - lane;
-  for (int it0 = warp_start; it0 < items; it0 += stride) {
-    const int it = it0 + lane;
-    const bool valid_item = it < items;
-    int q0 = 0;
-    uint32_t a = 0, p = 0;
-    if (valid_item) {
-      q0 = it / per_q;
-      const int rem = it - q0 * per_q;
-      const int jidx = rem >> log_cpj;
-      const int chunk = rem & ((1 << log_cpj) - 1);
-      const int* Jl = reinterpret_cast<const int*>(A.records + (int64_t)A.loc_slots[q0] * A.lay.rec_bytes +
-                                                   A.lay.off_J);
-      const uint32_t Jv = (uint32_t)Jl[jidx];
-      p = (Jv * (uint32_t)A.nb - half + (uint32_t)(chunk * A.P)) & A.nmask;
-      a = A.loc_a[q0];
-    }
-    const int allowed = A.Lloc - A.T - q0;
-    uint32_t f = (a * p) & A.nmask;
-    for (int t = 0; t < A.P; ++t, f = (f + a) & A.nmask) {
-      bool hit = false;
-      if (valid_item) {
-        int miss = 0;
-        bool ok = true;
-        for (int q = q0 + 1; q < A.Lloc; ++q) {
-          const uint32_t b = ((ssig[q] * f + half) & A.nmask) >> A.log2nb;
-          if (!((bm[q * words + (b >> 5)] >> (b & 31)) & 1u) && ++miss > allowed) {
-            ok = false;
-            break;
-          }
-        }
-        if (ok) {
-          for (int q = 0; q < q0; ++q) {
-            const uint32_t b = ((ssig[q] * f + half) & A.nmask) >> A.log2nb;
-            if ((bm[q * words + (b >> 5)] >> (b & 31)) & 1u) {
-              ok = false;
-              break;
-            }
-          }
-        }
-        hit = ok;
-      }
-      const unsigned ball = __ballot_sync(kFull, hit);
-      if (ball) {
-        unsigned base = 0;
-        const int leader = __ffs(ball) - 1;
-        if (lane == leader) base = atomicAdd(A.hit_count, (unsigned)__popc(ball));
-        base = __shfl_sync(kFull, base, leader);
-        if (hit) {
-          const unsigned slot = base + __popc(ball & ((1u << lane) - 1));
-          if ((int)slot < A.max_hits) A.hits[slot] = (int)f;
-        }
-      }
+  if (blockIdx.x == 0) TRACE(31);
+  const int units = (A.Lloc - A.T + 1) * A.num;
+  uint32_t* qF = queueF[threadIdx.x >> 5];
+  uint8_t* qG = queueG[threadIdx.x >> 5];
+  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const int nwarps = (gridDim.x * blockDim.x) >> 5;
+  for (int unit = warp; unit < units; unit += nwarps) {
+    const int q0 = unit / A.num;
+    const int jidx = unit - q0 * A.num;
+    const int* Jl = reinterpret_cast<const int*>(A.records + (int64_t)A.loc_slots[q0] * A.lay.rec_bytes + A.lay.off_J);
+    const uint32_t Jv = (uint32_t)__ldg(Jl + jidx);
+    const uint32_t a = __ldg(A.loc_a + q0);
+    const int m = min(A.Lloc - A.T - q0 + 1, A.Lloc - 1 - q0);  // mandatory probes
+    switch (m) {
+      case 0: vote_unit<0>(A, bm, ssig, words, q0, Jv, a, 0, qF, qG); break;
+      case 1: vote_unit<1>(A, bm, ssig, words, q0, Jv, a, 1, qF, qG); break;
+      case 2: vote_unit<2>(A, bm, ssig, words, q0, Jv, a, 2, qF, qG); break;
+      case 3: vote_unit<3>(A, bm, ssig, words, q0, Jv, a, 3, qF, qG); break;
+      case 4: vote_unit<4>(A, bm, ssig, words, q0, Jv, a, 4, qF, qG); break;
+      case 5: vote_unit<5>(A, bm, ssig, words, q0, Jv, a, 5, qF, qG); break;
+      case 6: vote_unit<6>(A, bm, ssig, words, q0, Jv, a, 6, qF, qG); break;
+      default: vote_unit<0>(A, bm, ssig, words, q0, Jv, a, m, qF, qG); break;
     }
   }
+  TRACE_END(32);
 }
 
 // ---------------------------------------------------------------------------
@@ -334,6 +678,7 @@ __global__ void __launch_bounds__(256) k_vote(VoteArgs A) {
 //   if d > nb/2: h = h+1 mod B, d -= nb;
 //   v_l = u^_l[h] * e^{-2 pi i tau_l f / n} / G^(-d);
 // val = (element of rank (L-1)/2 of Re v) + i (same of Im v), ties by loop.
+// Also counts the top digits of the output keys |val|^2 for k_output.
 // ---------------------------------------------------------------------------
 struct EstArgs {
   const uint8_t* records;
@@ -350,12 +695,12 @@ struct EstArgs {
   double2* hit_vals;
   uint64_t* hit_keys;
   double2* per_loop;  // may be null
+  uint32_t* out_hist;  // [4096] level-0 histogram of hit_keys
 };
 
 constexpr int kMaxLoops = 64;
 
-__device__ __forceinline__ double2 loop_estimate(const EstArgs& A, int l, uint32_t f) {
-  const SlotParam sp = A.slots[l];
+__device__ __forceinline__ double2 loop_estimate(const EstArgs& A, const SlotParam& sp, int l, uint32_t f) {
   const uint32_t p = (sp.sigma * f) & A.nmask;
   int hb = (int)(p >> A.log2nb);
   int d = (int)(p & (uint32_t)(A.nb - 1));
@@ -364,7 +709,7 @@ __device__ __forceinline__ double2 loop_estimate(const EstArgs& A, int l, uint32
     d -= A.nb;
   }
   const double2 g = __ldg(A.ghat + (A.nb >> 1) - d);  // G^(-d)
-  const double2 b = reinterpret_cast<const double2*>(A.records + (int64_t)l * A.lay.rec_bytes)[hb];
+  const double2 b = __ldg(reinterpret_cast<const double2*>(A.records + (int64_t)l * A.lay.rec_bytes) + hb);
   const uint32_t tph = (sp.tau * f) & A.nmask;
   double sn, cs;
   sincospi(2.0 * (double)tph / A.n, &sn, &cs);
@@ -399,127 +744,157 @@ __device__ __forceinline__ double warp_rank_select(double a0, double a1, int L, 
 }
 
 __global__ void __launch_bounds__(256) k_estimate(EstArgs A) {
+  __shared__ uint32_t sdig[8];
+  if (blockIdx.x == 0) TRACE(40);
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  SlotParam sp0{0, 0, 0, 0}, sp1{0, 0, 0, 0};
+  if (lane < A.L) sp0 = A.slots[lane];
+  if (lane + 32 < A.L) sp1 = A.slots[lane + 32];
   const int H = min((int)*A.hit_count, A.max_hits);
-  const int lane = threadIdx.x & 31;
-  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int nwarps = (gridDim.x * blockDim.x) >> 5;
   const int med = (A.L - 1) >> 1;
-  for (int h = warp; h < H; h += nwarps) {
-    const uint32_t f = (uint32_t)A.hits[h];
-    double2 v0 = make_double2(0.0, 0.0), v1 = make_double2(0.0, 0.0);
-    if (lane < A.L) v0 = loop_estimate(A, lane, f);
-    if (lane + 32 < A.L) v1 = loop_estimate(A, lane + 32, f);
-    if (A.per_loop) {
-      if (lane < A.L) A.per_loop[(int64_t)h * A.L + lane] = v0;
-      if (lane + 32 < A.L) A.per_loop[(int64_t)h * A.L + lane + 32] = v1;
+  for (int h0 = blockIdx.x * 8; h0 < H; h0 += gridDim.x * 8) {  // CTA-uniform
+    const int h = h0 + wib;
+    uint32_t dig = 0xFFFFFFFFu;
+    if (h < H) {
+      const uint32_t f = (uint32_t)__ldg(A.hits + h);
+      double2 v0 = make_double2(0.0, 0.0), v1 = make_double2(0.0, 0.0);
+      if (lane < A.L) v0 = loop_estimate(A, sp0, lane, f);
+      if (lane + 32 < A.L) v1 = loop_estimate(A, sp1, lane + 32, f);
+      if (A.per_loop) {
+        if (lane < A.L) A.per_loop[(int64_t)h * A.L + lane] = v0;
+        if (lane + 32 < A.L) A.per_loop[(int64_t)h * A.L + lane + 32] = v1;
+      }
+      const double vr = warp_rank_select(v0.x, v1.x, A.L, med);
+      const double vi = warp_rank_select(v0.y, v1.y, A.L, med);
+      const uint64_t key = (uint64_t)__double_as_longlong(__dadd_rn(__dmul_rn(vr, vr), __dmul_rn(vi, vi)));
+      if (lane == 0) {
+        A.hit_vals[h] = make_double2(vr, vi);
+        A.hit_keys[h] = key;
+      }
+      dig = (uint32_t)(key >> 51) & 0xFFFu;
     }
-    const double vr = warp_rank_select(v0.x, v1.x, A.L, med);
-    const double vi = warp_rank_select(v0.y, v1.y, A.L, med);
-    if (lane == 0) {
-      A.hit_vals[h] = make_double2(vr, vi);
-      A.hit_keys[h] = (uint64_t)__double_as_longlong(__dadd_rn(__dmul_rn(vr, vr), __dmul_rn(vi, vi)));
+    if (lane == 0) sdig[wib] = dig;
+    __syncthreads();
+    if (threadIdx.x < 8) {  // one atomic per distinct digit of this CTA's 8 hits
+      const uint32_t d = sdig[threadIdx.x];
+      bool first = d != 0xFFFFFFFFu;
+      uint32_t c = 0;
+      for (int j = 0; j < 8; ++j) {
+        first = first && !(j < (int)threadIdx.x && sdig[j] == d);
+        c += sdig[j] == d;
+      }
+      if (first) atomicAdd(A.out_hist + d, c);
     }
+    __syncthreads();
   }
+  TRACE_END(41);
 }
 
 // ---------------------------------------------------------------------------
 // Output: the k hits of largest |val|^2 (ties to the smaller f), written in
-// ascending f; pads loc = -1, val = 0.  One CTA of 1024 threads.  Hits are
-// staged in smem when H <= kOutCap; the sort is a bitonic network (warp
-// shuffles below stride 32) over 64-bit (f << 32 | hit index) keys.
-// Dynamic smem: 4096 u32 hist + 64 ints + kOutCap x (u64 + int) + kp2 x u64.
+// ascending f; pads loc = -1, val = 0.  One CTA of 1024 threads: two-level
+// selection (level 0 counted by k_estimate), then a bucket sort by the top 10
+// bits of f with a per-bucket insertion sort (bitonic fallback for crowded
+// buckets).  Dynamic smem: 4096 u32 hist + 64 ints + kOutCap x (u64 + int)
+// + kp2 x u64 + 1024 x 2 ints.
 // ---------------------------------------------------------------------------
-constexpr int kOutCap = 8192;
-
-struct HitSrc {
-  const uint64_t* keys;
-  const int* hits;
-  __device__ __forceinline__ void get(int i, uint64_t& hi, uint32_t& lo) const {
-    hi = keys[i];
-    lo = ~(uint32_t)hits[i];
-  }
-};
+constexpr int kOutCap = 4096;
 
 __global__ void __launch_bounds__(1024) k_output(const int* __restrict__ hits, const unsigned* __restrict__ hit_count,
                                                  int max_hits, const double2* __restrict__ hit_vals,
-                                                 const uint64_t* __restrict__ hit_keys, int k, int kp2,
-                                                 int64_t* __restrict__ locs, double2* __restrict__ vals,
-                                                 int* __restrict__ status) {
+                                                 const uint64_t* __restrict__ hit_keys, uint32_t* __restrict__ ghist,
+                                                 int k, int kp2, int log2n, int64_t* __restrict__ locs,
+                                                 double2* __restrict__ vals, int* __restrict__ status) {
   extern __shared__ __align__(16) uint8_t smem[];
   uint32_t* hist = reinterpret_cast<uint32_t*>(smem);
   int* sm = reinterpret_cast<int*>(smem + 4096 * 4);
-  uint64_t* skey = reinterpret_cast<uint64_t*>(smem + 4096 * 4 + 64 * 4);
-  int* shit = reinterpret_cast<int*>(skey + kOutCap);
-  uint64_t* sort = reinterpret_cast<uint64_t*>(shit + kOutCap);
+  uint64_t* ckey = reinterpret_cast<uint64_t*>(smem + 4096 * 4 + 64 * 4);
+  int* cidx = reinterpret_cast<int*>(ckey + kOutCap);
+  uint64_t* sel = reinterpret_cast<uint64_t*>(cidx + kOutCap);  // (f << 32 | i), kp2 entries
+  uint64_t* srt = sel + kp2;                                     // bucket-sorted copy
+  int* bcnt = reinterpret_cast<int*>(srt + kp2);                 // 1024 bucket counters
+  int* bstart = bcnt + 1024;                                     // 1024 bucket starts
   const int tid = threadIdx.x;
+  TRACE(50);
   const unsigned hc = *hit_count;
   const int H = min((int)hc, max_hits);
   if (tid == 0 && (int)hc > max_hits) atomicOr(status, 1);
   const int K = min(k, H);
-  const bool staged = H <= kOutCap;
-  if (staged) {
-    for (int i = tid; i < H; i += 1024) {
-      skey[i] = hit_keys[i];
-      shit[i] = hits[i];
-    }
-  }
-  if (tid == 0) sm[40] = 0;
-  for (int i = tid; i < kp2; i += 1024) sort[i] = ~0ull;
+  if (tid == 0) sm[41] = 0;
+  bcnt[tid] = 0;
   __syncthreads();
-  const uint64_t* kk = staged ? skey : hit_keys;
-  const int* hh = staged ? shit : hits;
-  Prefix96 p{0, 0, 0, 0};  // matches everything
-  if (H > K) p = block_radix_select(HitSrc{kk, hh}, H, K, hist, sm);
-  for (int i = tid; i < H; i += 1024) {
-    const int f = hh[i];
-    if (ge96(p, kk[i], ~(uint32_t)f)) {
-      const int pos = atomicAdd(&sm[40], 1);
-      if (pos < kp2) sort[pos] = ((uint64_t)(uint32_t)f << 32) | (uint32_t)i;
-    }
-  }
-  __syncthreads();
-  if (tid == 0 && sm[40] != K) atomicOr(status + 2, 1);
-  if (kp2 <= 1024) {
-    uint64_t v = tid < kp2 ? sort[tid] : ~0ull;
-    for (int size = 2; size <= kp2; size <<= 1) {
-      for (int stride = size >> 1; stride > 0; stride >>= 1) {
-        uint64_t o;
-        if (stride >= 32) {
-          __syncthreads();
-          sort[tid] = v;
-          __syncthreads();
-          o = sort[tid ^ stride];
-        } else {
-          o = __shfl_xor_sync(kFull, v, stride);
-        }
-        const bool up = (tid & size) == 0;
-        const bool lower = (tid & stride) == 0;
-        v = (lower == up) ? min(v, o) : max(v, o);
-      }
-    }
-    __syncthreads();
-    if (tid < kp2) sort[tid] = v;
-    __syncthreads();
+  auto add = [&](int i) {
+    const int pos = atomicAdd(&sm[41], 1);
+    if (pos < kp2) sel[pos] = ((uint64_t)(uint32_t)__ldg(hits + i) << 32) | (uint32_t)i;
+  };
+  if (H > K) {
+    select_topk(
+        H, K, ghist,
+        [&](int i, uint64_t& kk, uint32_t& t) {
+          kk = __ldg(hit_keys + i);
+          t = (uint32_t)__ldg(hits + i);
+        },
+        add, ckey, cidx, kOutCap, hist, sm);
   } else {
+    for (int i = tid; i < H; i += 1024) add(i);
+    __syncthreads();
+  }
+  TRACE(51);
+  const int ns = min(sm[41], kp2);
+  if (tid == 0 && sm[41] != K) atomicOr(status + 2, 1);
+  // bucket sort by the top 10 bits of f
+  const int sh = max(0, log2n - 10);
+  for (int i = tid; i < ns; i += 1024) atomicAdd(&bcnt[(int)(sel[i] >> 32) >> sh], 1);
+  __syncthreads();
+  const int c = bcnt[tid];
+  int total;
+  const int st = block_excl_scan<1024>(c, &total, sm);
+  bstart[tid] = st;
+  if (tid == 0) sm[42] = 0;
+  __syncthreads();
+  atomicMax(&sm[42], c);
+  bcnt[tid] = 0;
+  __syncthreads();
+  for (int i = tid; i < ns; i += 1024) {
+    const int bkt = (int)(sel[i] >> 32) >> sh;
+    srt[bstart[bkt] + atomicAdd(&bcnt[bkt], 1)] = sel[i];
+  }
+  __syncthreads();
+  if (sm[42] <= 32) {
+    const int b0 = bstart[tid];
+    for (int i = 1; i < c; ++i) {  // insertion sort of this thread's bucket
+      const uint64_t v = srt[b0 + i];
+      int j = i - 1;
+      while (j >= 0 && srt[b0 + j] > v) {
+        srt[b0 + j + 1] = srt[b0 + j];
+        --j;
+      }
+      srt[b0 + j + 1] = v;
+    }
+  } else {  // crowded bucket: bitonic over all selected entries
+    for (int i = ns + tid; i < kp2; i += 1024) srt[i] = ~0ull;
+    __syncthreads();
     for (int size = 2; size <= kp2; size <<= 1) {
       for (int stride = size >> 1; stride > 0; stride >>= 1) {
         for (int t = tid; t < (kp2 >> 1); t += 1024) {
           const int i = 2 * t - (t & (stride - 1));
           const int jn = i + stride;
           const bool up = (i & size) == 0;
-          const uint64_t a = sort[i], b = sort[jn];
+          const uint64_t a = srt[i], b = srt[jn];
           if ((a > b) == up) {
-            sort[i] = b;
-            sort[jn] = a;
+            srt[i] = b;
+            srt[jn] = a;
           }
         }
         __syncthreads();
       }
     }
   }
+  __syncthreads();
+  TRACE(52);
   for (int j = tid; j < k; j += 1024) {
-    if (j < K) {
-      const uint64_t v = sort[j];
+    if (j < ns) {
+      const uint64_t v = srt[j];
       locs[j] = (int64_t)(v >> 32);
       vals[j] = hit_vals[(uint32_t)v];
     } else {
@@ -527,6 +902,7 @@ __global__ void __launch_bounds__(1024) k_output(const int* __restrict__ hits, c
       vals[j] = make_double2(0.0, 0.0);
     }
   }
+  TRACE(53);
 }
 
 }  // namespace cusfft

@@ -71,7 +71,7 @@ __device__ __forceinline__ void dft<8>(double2* v) {
 
 // One Stockham stage of radix R over E elements (E/M sequences of length M) in
 // S, jobs strided over NT threads.  Ns = product of the radices done so far.
-template <int R, int M, int E, int NT>
+template <int R, int M, int E, int NT, bool TWS = false>
 __device__ __forceinline__ void stockham_stage(double2* S, int Ns, const double2* __restrict__ tw, int B) {
   constexpr int JOBS = E / R;
   constexpr int PER = (JOBS + NT - 1) / NT;
@@ -91,7 +91,7 @@ __device__ __forceinline__ void stockham_stage(double2* S, int Ns, const double2
       const int kk = j & (Ns - 1);
       if (Ns > 1) {
 #pragma unroll
-        for (int r = 1; r < R; ++r) v[p][r] = cmul(v[p][r], __ldg(tw + kk * r * twstep));
+        for (int r = 1; r < R; ++r) v[p][r] = cmul(v[p][r], TWS ? tw[kk * r * twstep] : __ldg(tw + kk * r * twstep));
       }
       dft<R>(v[p]);
       dst[p] = base + (j - kk) * R + kk;
@@ -108,23 +108,24 @@ __device__ __forceinline__ void stockham_stage(double2* S, int Ns, const double2
   __syncthreads();
 }
 
-template <int M, int E, int NT>
+// tw: table of e^{-2 pi i t / B}; TWS: tw lives in shared memory.
+template <int M, int E, int NT, bool TWS = false>
 __device__ __forceinline__ void fft_smem(double2* S, const double2* __restrict__ tw, int B) {
   constexpr int LOGM = (M >= 4096) ? 12 : (M >= 2048) ? 11 : (M >= 1024) ? 10 : (M >= 512) ? 9 : (M >= 256) ? 8
                        : (M >= 128) ? 7 : (M >= 64) ? 6 : (M >= 32) ? 5 : (M >= 16) ? 4 : (M >= 8) ? 3 : (M >= 4) ? 2 : 1;
   constexpr int REM = LOGM % 3;
   int Ns = 1;
   if constexpr (REM == 1) {
-    stockham_stage<2, M, E, NT>(S, Ns, tw, B);
+    stockham_stage<2, M, E, NT, TWS>(S, Ns, tw, B);
     Ns *= 2;
   } else if constexpr (REM == 2) {
-    stockham_stage<4, M, E, NT>(S, Ns, tw, B);
+    stockham_stage<4, M, E, NT, TWS>(S, Ns, tw, B);
     Ns *= 4;
   }
   if constexpr (LOGM >= 3) {
 #pragma unroll 1
     for (int s = 0; s < LOGM / 3; ++s) {
-      stockham_stage<8, M, E, NT>(S, Ns, tw, B);
+      stockham_stage<8, M, E, NT, TWS>(S, Ns, tw, B);
       Ns *= 8;
     }
   }
@@ -147,7 +148,7 @@ struct FftPassArgs {
 };
 
 // E = elements per CTA, NT = threads per CTA.  Dynamic smem: fft_smem_bytes(E).
-__host__ __device__ constexpr int fft_smem_bytes(int E) { return (E + E / 8) * 16 + 4096 * 4; }
+__host__ __device__ constexpr int fft_smem_bytes(int E) { return (E + E / 8) * 16 + 4096 * 4 + E * 16; }
 
 template <int M, int E, int NT>
 __global__ void __launch_bounds__(NT) k_fft(FftPassArgs A) {
@@ -155,7 +156,10 @@ __global__ void __launch_bounds__(NT) k_fft(FftPassArgs A) {
   extern __shared__ __align__(16) uint8_t fsm[];
   double2* S = reinterpret_cast<double2*>(fsm);
   uint32_t* shist = reinterpret_cast<uint32_t*>(fsm + (E + E / 8) * sizeof(double2));
+  double2* twl = reinterpret_cast<double2*>(fsm + (E + E / 8) * sizeof(double2) + 4096 * 4);  // omega_M^t, t < M
   const int q0 = blockIdx.x * NSEQ;
+  for (int t = threadIdx.x; t < M; t += NT) twl[t] = __ldg(A.tw + (int64_t)t * (A.B / M));
+  if (blockIdx.x == 0) TRACE(A.twiddle ? 2 : 4);
   const bool col_fast_in = (A.in_cs == 1);
   const int spm = (1 << A.log_seq_per_slot) - 1;
   {  // all E/NT loads of a thread in flight before the first smem store
@@ -186,7 +190,7 @@ __global__ void __launch_bounds__(NT) k_fft(FftPassArgs A) {
       if (dst[u] >= 0) S[dst[u]] = buf[u];
   }
   __syncthreads();
-  fft_smem<M, E, NT>(S, A.tw, A.B);
+  fft_smem<M, E, NT, true>(S, twl, M);
   // keys: a CTA's sequences all belong to one slot when NSEQ <= seq_per_slot
   const bool one_slot = NSEQ <= (1 << A.log_seq_per_slot);
   int kidx = -1;
@@ -233,6 +237,7 @@ __global__ void __launch_bounds__(NT) k_fft(FftPassArgs A) {
     for (int i = threadIdx.x; i < 4096; i += NT)
       if (shist[i]) atomicAdd(&A.hist[(int64_t)kidx * 4096 + i], shist[i]);
   }
+  if (A.twiddle) TRACE_END(3); else TRACE_END(5);
 }
 
 }  // namespace cusfft
