@@ -21,7 +21,6 @@ using namespace cusfft;
 namespace {
 
 constexpr uint32_t kMagic = 0x5FF7B200u;
-constexpr int kFoldPad = 120 * 1024;  // dynamic smem that caps a fold launch at 1 CTA per SM
 thread_local int g_last_cuda_error = 0;
 
 #define CK(expr)                                  \
@@ -156,7 +155,6 @@ struct cusfft_plan_s {
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
   int stage_limit = 6;
   int cur_prio = 0, prio_hi = 0, prio_lo = 0;  // launch priorities (branched graph)
-  int fold_smem_pad = 0;  // unused dynamic smem that caps the estimation fold at 1 CTA / SM
   struct GraphEntry {
     int lim = -1;
     const void* a = nullptr;
@@ -338,31 +336,6 @@ template <int M>
 cudaError_t set_fft_attr_t() {
   return cudaFuncSetAttribute(k_fft<M, fft_E<M>(), 128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                               fft_smem_bytes(fft_E<M>()));
-}
-
-// Every hot-path kernel runs with the maximum shared-memory carveout, so that
-// kernels of the two graph branches can be resident on one SM at the same time
-// (an SM changes its L1/smem split only when idle).
-template <typename K>
-cudaError_t carveout_max(K kern) {
-  return cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared);
-}
-
-template <int M>
-cudaError_t carve_fft_t() {
-  return carveout_max(k_fft<M, fft_E<M>(), 128>);
-}
-
-cudaError_t set_carveouts() {
-  cudaError_t r[] = {carve_fft_t<2>(), carve_fft_t<4>(), carve_fft_t<8>(), carve_fft_t<16>(), carve_fft_t<32>(),
-                     carve_fft_t<64>(), carve_fft_t<128>(), carve_fft_t<256>(), carve_fft_t<512>(),
-                     carve_fft_t<1024>(), carve_fft_t<2048>(), carve_fft_t<4096>(), carveout_max(k_fold<16>),
-                     carveout_max(k_fold_fft1<64, 8>), carveout_max(k_fold_fft1<128, 8>),
-                     carveout_max(k_fold_fft1<256, 8>), carveout_max(k_select), carveout_max(k_vote),
-                     carveout_max(k_estimate), carveout_max(k_output)};
-  for (cudaError_t x : r)
-    if (x != cudaSuccess) return x;
-  return cudaSuccess;
 }
 
 cudaError_t set_fft_attrs() {
@@ -596,7 +569,7 @@ template <int B1T>
 cudaError_t launch_fold_fft1_t(cusfft_plan_t P, const double2* x, const SlotParam* sp, double2* u, double2* v,
                                int nslots, ZeroArgs z, cudaStream_t st) {
   dim3 grid((unsigned)(P->B / 256), (unsigned)nslots);
-  return launch_k(k_fold_fft1<B1T, 8>, grid, dim3(256), P->fold_smem_pad, st, P->cur_prio, x, (const double*)P->d_taps_perm, sp, u, v,
+  return launch_k(k_fold_fft1<B1T, 8>, grid, dim3(256), 0, st, P->cur_prio, x, (const double*)P->d_taps_perm, sp, u, v,
                   (const double2*)P->d_tw, (int)P->B, P->B2, P->w, P->R, (uint32_t)(P->n - 1), z);
 }
 
@@ -625,7 +598,7 @@ int launch_fold(cusfft_plan_t P, const double2* x, int s0, int s1, cudaStream_t 
     CK(launch_fold_fft1(P, x, sp, P->d_u + (size_t)s0 * B, P->d_v + (size_t)s0 * B, s1 - s0, z, st));
   } else {
     dim3 grid((B + 255) / 256, s1 - s0);
-    CK(launch_k(k_fold<16>, grid, dim3(256), P->fold_smem_pad, st, P->cur_prio, x, (const double*)P->d_taps, sp,
+    CK(launch_k(k_fold<16>, grid, dim3(256), 0, st, P->cur_prio, x, (const double*)P->d_taps, sp,
                 P->d_u + (size_t)s0 * B, B, P->w, P->R, (uint32_t)(P->n - 1), z));
   }
   return CUSFFT_SUCCESS;
