@@ -36,9 +36,13 @@ __device__ __forceinline__ void zero_part(const ZeroArgs& z) {
   for (int i = b + threadIdx.x; i < e; i += blockDim.x) z.p[i] = 0;
 }
 
+// Random 16-B gather: non-coherent path, no L1 allocation, and an L2 fetch of
+// 64 B instead of the default 128-B line (halves the DRAM bytes per random
+// sample; the time is bound by DRAM row activations either way, see
+// scripts/probes/gather_probe.cu and DESIGN.md §6).
 __device__ __forceinline__ double2 ld_gather(const double2* p) {
   double2 v;
-  asm volatile("ld.global.nc.L1::no_allocate.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
+  asm volatile("ld.global.nc.L1::no_allocate.L2::64B.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
   return v;
 }
 

@@ -1,0 +1,152 @@
+"""Loop-sharded multi-GPU execution (paper_conf_ipps_wangcc16_b200.dist).
+
+CPU (gloo, world_size 2): the exchange logic of LoopShardedSfft — loop
+ownership, rank-major slot layout, one all-gather, rank-identical outputs —
+driven with a test engine whose per-loop arithmetic is the oracle's (tests may
+use the oracle; the product path never does).  GPU: two cusfft_plan_dist plans
+(rank 0 and 1 of 2) on one device with the all-gather emulated by copies must
+reproduce the single-GPU plan bit for bit.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+import oracle as O
+from paper_conf_ipps_wangcc16_b200.dist import LoopShardedSfft, loops_of_rank, slot_of_loop
+from paper_conf_ipps_wangcc16_b200.workload import planted_signal
+
+
+def test_slot_mapping_is_a_rank_major_permutation():
+    for L, world in [(16, 1), (16, 2), (16, 4), (16, 8), (12, 3)]:
+        slots = [slot_of_loop(r, L, world) for r in range(L)]
+        assert sorted(slots) == list(range(L))
+        for g in range(world):
+            mine = loops_of_rank(g, L, world)
+            assert sorted(slot_of_loop(r, L, world) for r in mine) == list(range(g * L // world, (g + 1) * L // world))
+            assert all(r % world == g for r in mine)
+    with pytest.raises(ValueError):
+        loops_of_rank(0, 10, 4)
+
+
+class OracleEngine:
+    """Test engine with the engine interface of dist.CudaEngine: per-loop
+    records (u^_r as fp64 pairs, then the cutoff list J_r for location loops)
+    in the rank-major exchange buffer; the oracle does the arithmetic."""
+
+    def __init__(self, x, p: O.SfftParams, rank: int, world: int):
+        self.x, self.p, self.rank, self.world = x, p, rank, world
+        self.a, self.sigma, self.tau = O.draw_permutations(p.seed, p.n, p.L, p.tau_mode)
+        self.g = O.filter_taps(p)
+        self.Lg = p.L // world
+        self.rec = p.B * 16 + p.num_select * 8
+        self.buf = torch.zeros(world * self.Lg * self.rec, dtype=torch.uint8)
+
+    def _slot_view(self, s):
+        return self.buf[s * self.rec:(s + 1) * self.rec]
+
+    def local(self, x):
+        for r in loops_of_rank(self.rank, self.p.L, self.world):
+            uh = O.bucket_fft(O.perm_filter(x, self.g, int(self.sigma[r]), int(self.tau[r]), self.p.B))
+            J = O.cutoff(uh, self.p.num_select) if r < self.p.loc_loops else np.zeros(self.p.num_select, np.int64)
+            rec = np.concatenate([uh.view(np.float64).view(np.uint8), J.astype(np.int64).view(np.uint8)])
+            self._slot_view(slot_of_loop(r, self.p.L, self.world)).copy_(torch.from_numpy(rec))
+
+    def exchange_tensor(self):
+        return self.buf
+
+    def finish(self):
+        p = self.p
+        uhat, J = [], []
+        for r in range(p.L):
+            rec = self._slot_view(slot_of_loop(r, p.L, self.world)).numpy()
+            uhat.append(rec[:p.B * 16].view(np.complex128).copy())
+            if r < p.loc_loops:
+                J.append(rec[p.B * 16:].view(np.int64).copy())
+        hits = np.sort(O.location_recovery(J, self.a[:p.loc_loops], p.n, p.B, p.vote_threshold))
+        G = O.filter_response(self.g, p.n, p.n // p.B)
+        vals, _ = O.estimate(hits, np.stack(uhat), self.sigma, self.tau, G, p.n, p.B)
+        return O.select_output(hits, vals, p.k)
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        n, k = 2 ** 12, 6
+        x, S, X = planted_signal(n, k, seed=4)
+        p = O.make_params(n, k, L=8, loc_loops=5, vote_threshold=3, seed=9)
+        eng = OracleEngine(x, p, rank, world)
+        locs, vals = LoopShardedSfft(eng).execute(x)
+        q.put((rank, locs.tolist(), vals.tolist()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_loop_sharded_exchange_gloo(world):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    out = [q.get(timeout=300) for _ in range(world)]
+    for pr in procs:
+        pr.join(timeout=60)
+        assert pr.exitcode == 0
+    n, k = 2 ** 12, 6
+    x, S, X = planted_signal(n, k, seed=4)
+    ref = O.sfft(x, O.make_params(n, k, L=8, loc_loops=5, vote_threshold=3, seed=9))
+    for rank, locs, vals in out:
+        assert locs == ref.locs.tolist(), rank
+        np.testing.assert_array_equal(np.array(vals), ref.vals)
+
+
+def test_loop_sharded_world1_no_collective():
+    n, k = 2 ** 12, 6
+    x, S, X = planted_signal(n, k, seed=5)
+    p = O.make_params(n, k, L=6, loc_loops=5, vote_threshold=3, seed=2)
+    locs, vals = LoopShardedSfft(OracleEngine(x, p, 0, 1)).execute(x)
+    ref = O.sfft(x, p)
+    assert np.array_equal(locs, ref.locs)
+    np.testing.assert_array_equal(vals, ref.vals)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("world", [2, 4])
+def test_dist_plans_emulated_allgather_match_single_gpu(world):
+    """cusfft_plan_dist ranks on one GPU; the all-gather is emulated by device
+    copies between the ranks' exchange buffers."""
+    from paper_conf_ipps_wangcc16_b200 import Plan
+    from paper_conf_ipps_wangcc16_b200.dist import CudaEngine
+    n, k, L = 2 ** 20, 100, 16
+    x, S, X = planted_signal(n, k, seed=8)
+    xd = torch.from_numpy(x).cuda()
+    ref_l, ref_v = Plan(n, k, L=L, seed=5).execute(xd)
+    engines = [CudaEngine(n, k, L=L, rank=r, world=world, seed=5) for r in range(world)]
+    for e in engines:
+        e.local(xd)
+    torch.cuda.synchronize()
+    per = engines[0].per_rank
+    for dst in engines:
+        for r, src in enumerate(engines):
+            if src is not dst:
+                dst.exchange_tensor()[r * per:(r + 1) * per].copy_(src.exchange_tensor()[r * per:(r + 1) * per])
+    torch.cuda.synchronize()
+    for e in engines:
+        locs, vals = e.finish()
+        torch.cuda.synchronize()
+        assert e.plan.status() == 0
+        assert torch.equal(locs, ref_l)
+        assert torch.equal(vals, ref_v)
