@@ -49,13 +49,15 @@ def hbm_peak():
         return FALLBACK_HBM, "fallback (B200_PROFILING.md)"
 
 
-def fold_bytes(L: int, w: int, B: int):
-    """Algorithmic bytes of one fold launch:
-    L*w random 16-B samples, each costing one 32-B DRAM sector, + the w fp64
-    taps read once + the L*B complex fp64 buckets written."""
-    sector = L * w * 32 + w * 8 + L * B * 16
-    useful = L * w * 16 + w * 8 + L * B * 16
-    return sector, useful
+def fold_bytes(L: int, w: int, B: int, sectors: int):
+    """Algorithmic bytes of the fold stage: the distinct
+    32-B DRAM sectors of x that the plan's L*w gather positions touch (exact,
+    counted at plan time; a random 16-B sample cannot cost less than its
+    sector, and a sector shared by several loops need be read once), the w fp64
+    taps, and the L*B complex fp64 buckets written (u, plus v when the first
+    FFT pass is fused, B > 2048).  `useful` counts 16 B per sample instead."""
+    out = L * B * 16 * (2 if 2048 < B <= 65536 else 1)
+    return sectors * 32 + w * 8 + out, L * w * 16 + w * 8 + out
 
 
 class ClockSampler:
@@ -360,7 +362,8 @@ def run_gpu(args):
                          "(plan-time filter construction excluded), numpy single thread"}
 
     peak, peak_src = hbm_peak()
-    sector, useful = fold_bytes(plan.L // world if world > 1 else L, plan.w, B)
+    info = plan.info()
+    sector, useful = fold_bytes(plan.L // world if world > 1 else L, plan.w, B, int(info["sectors"]))
     achieved = sector / (fold_ms * 1e-3) / 1e9
     traffic = None
     tf = os.path.join(ROOT, "profiles", f"fold_traffic_{args.config}.json")
@@ -382,7 +385,8 @@ def run_gpu(args):
         "gpu_launches": launches * args.steps,
         "timed_region_ms_incl_flush": region_ms,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                     "frac": achieved / peak, "traffic": traffic, "kernel": "k_fold",
+                     "frac": achieved / peak, "traffic": traffic,
+                     "kernel": "fold stage (k_stage + k_fold_fft1)" if info["staged"] else "k_fold_fft1",
                      "algorithmic_bytes_per_launch": sector, "useful_bytes_per_launch": useful,
                      "useful_gbs": useful / (fold_ms * 1e-3) / 1e9, "kernel_ms": fold_ms,
                      "peak_source": peak_src},

@@ -136,7 +136,9 @@ int cusfft_execute_finish(cusfft_plan_t plan, int64_t* d_locs, void* d_vals);
 int cusfft_exchange_buffer(cusfft_plan_t plan, void** d_buf, int64_t* bytes_per_rank);
 
 /* Plan facts (host arrays, caller-owned):
- *   info[0..9] = n, k, B, L, w (taps), n/B, num_select, loc_loops, vote_threshold, max_hits
+ *   info[0..11] = n, k, B, L, w (taps), n/B, num_select, loc_loops, vote_threshold, max_hits,
+ *                 distinct 32-B sectors of x this rank's gathers touch (the fold's DRAM floor),
+ *                 staged (1: address-sorted two-phase gather)
  *   a, sigma, tau : int64 [L], in loop order r = 0..L-1 (NULL to skip).  sigma is
  *   the gather stride (Alg. 1's ai), a = sigma^-1 mod n, tau the offset. */
 int cusfft_get_info(cusfft_plan_t plan, int64_t* info, int64_t* a, int64_t* sigma, int64_t* tau);

@@ -254,14 +254,14 @@ class Plan:
 
     # -- introspection
     def info(self):
-        info = np.zeros(10, dtype=np.int64)
+        info = np.zeros(12, dtype=np.int64)
         a = np.zeros(self.L, dtype=np.int64)
         s = np.zeros(self.L, dtype=np.int64)
         t = np.zeros(self.L, dtype=np.int64)
         check(self._lib.cusfft_get_info(self._h, ctypes.c_void_p(info.ctypes.data), ctypes.c_void_p(a.ctypes.data),
                                         ctypes.c_void_p(s.ctypes.data), ctypes.c_void_p(t.ctypes.data)),
               "cusfft_get_info")
-        keys = ("n", "k", "B", "L", "w", "nb", "num", "loc_loops", "T", "max_hits")
+        keys = ("n", "k", "B", "L", "w", "nb", "num", "loc_loops", "T", "max_hits", "sectors", "staged")
         d = dict(zip(keys, info.tolist()))
         d.update(a=a, sigma=s, tau=t)
         return d

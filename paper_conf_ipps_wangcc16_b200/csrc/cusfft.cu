@@ -112,6 +112,13 @@ struct cusfft_plan_s {
   double* d_taps = nullptr;
   double* d_taps_perm = nullptr;  // fused fold+pass-1 layout (two-pass B, B1 <= 256)
   bool fused1 = false;
+  // staged gather: address-sorted gather schedule of this rank
+  bool staged = false;
+  int64_t sectors = 0;            // distinct 32-B sectors of x gathered by this rank (the fold's DRAM floor)
+  int64_t stage_total = 0;        // Lg * w samples
+  uint32_t* d_spos = nullptr;     // [stage_total] sorted gather positions
+  uint32_t* d_inv = nullptr;      // [Lg][R][B] staging index in the fused kernel's thread order
+  double2* d_staging = nullptr;   // [stage_total]
   double2* d_ghat = nullptr;
   double2* d_tw = nullptr;
   SlotParam* d_slots = nullptr;
@@ -181,7 +188,7 @@ struct DeviceGuard {
 };
 
 void free_plan(cusfft_plan_t p) {
-  void* ptrs[] = {p->d_taps, p->d_taps_perm, p->d_ghat, p->d_tw, p->d_slots, p->d_loc_slots, p->d_loc_sigma, p->d_loc_a,
+  void* ptrs[] = {p->d_taps, p->d_taps_perm, p->d_spos, p->d_inv, p->d_staging, p->d_ghat, p->d_tw, p->d_slots, p->d_loc_slots, p->d_loc_sigma, p->d_loc_a,
                   p->d_sel_slots, p->d_u, p->d_v, p->d_records, p->d_keys, p->d_zero, p->d_key_index, p->d_ckey, p->d_cidx, p->d_hits, p->d_hit_vals,
                   p->d_hit_keys, p->d_per_loop, p->d_xbuf, p->d_locs_buf, p->d_vals_buf};
   for (void* q : ptrs)
@@ -528,10 +535,6 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     return fail(CUSFFT_CUDA);
   }
   if (set_fft_attrs() != cudaSuccess ||
-      cudaFuncSetAttribute(k_fold<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024) != cudaSuccess ||
-      cudaFuncSetAttribute(k_fold_fft1<64, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024) != cudaSuccess ||
-      cudaFuncSetAttribute(k_fold_fft1<128, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024) != cudaSuccess ||
-      cudaFuncSetAttribute(k_fold_fft1<256, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 160 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_select, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_vote, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_output, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess) {
@@ -557,6 +560,56 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     if ((rc = dalloc(&P->d_taps_perm, (size_t)padded))) return fail(rc);
     if ((rc = upload(P->d_taps_perm, gp.data(), padded * sizeof(double)))) return fail(rc);
   }
+  {  // distinct 32-B sectors (2 complex samples) of x this rank gathers
+    std::vector<uint64_t> bits((size_t)((n / 2 + 63) / 64), 0ull);
+    const uint32_t nm = (uint32_t)(n - 1);
+    for (int sl = 0; sl < P->Lg; ++sl) {
+      const SlotParam& sp = P->slots_h[(size_t)rank * P->Lg + sl];
+      for (int i = 0; i < P->w; ++i) {
+        const uint32_t sec = ((sp.sigma * (uint32_t)i + sp.tau) & nm) >> 1;
+        bits[sec >> 6] |= 1ull << (sec & 63);
+      }
+    }
+    int64_t cnt = 0;
+    for (uint64_t b : bits) cnt += __builtin_popcountll(b);
+    P->sectors = cnt;
+  }
+  {
+    const char* e = std::getenv("CUSFFT_NO_STAGE");
+    const int64_t total = (int64_t)P->Lg * P->w;
+    // staging must stay L2-resident between the two phases
+    P->staged = P->fused1 && total * 16 <= (int64_t)64 << 20 && total < (int64_t)1 << 31 && !(e && e[0] == '1');
+    if (P->staged) {
+      P->stage_total = total;
+      std::vector<uint64_t> ev((size_t)total);
+      const uint32_t nm = (uint32_t)(n - 1);
+      for (int sl = 0; sl < P->Lg; ++sl) {
+        const SlotParam& sp = P->slots_h[(size_t)rank * P->Lg + sl];
+        for (int i = 0; i < P->w; ++i) {
+          const uint32_t pos = (sp.sigma * (uint32_t)i + sp.tau) & nm;
+          const uint64_t id = (uint64_t)sl * P->w + i;
+          ev[(size_t)id] = ((uint64_t)pos << 32) | id;
+        }
+      }
+      std::sort(ev.begin(), ev.end());
+      std::vector<uint32_t> spos((size_t)total), inv((size_t)P->Lg * P->R * B, 0u);
+      const int C = 256 / P->B1;
+      for (int64_t q = 0; q < total; ++q) {
+        spos[(size_t)q] = (uint32_t)(ev[(size_t)q] >> 32);
+        const uint64_t id = ev[(size_t)q] & 0xFFFFFFFFull;
+        const int64_t sl = (int64_t)(id / P->w), i = (int64_t)(id % P->w);
+        const int64_t rr = i / B, j = i % B;
+        const int64_t c = j % P->B2, j1 = j / P->B2;
+        const int64_t cta = c / C, t = (c % C) * P->B1 + j1;
+        inv[(size_t)((sl * P->R + rr) * B + cta * 256 + t)] = (uint32_t)q;
+      }
+      if ((rc = dalloc(&P->d_spos, (size_t)total))) return fail(rc);
+      if ((rc = dalloc(&P->d_inv, inv.size()))) return fail(rc);
+      if ((rc = dalloc(&P->d_staging, (size_t)total))) return fail(rc);
+      if ((rc = upload(P->d_spos, spos.data(), spos.size() * sizeof(uint32_t)))) return fail(rc);
+      if ((rc = upload(P->d_inv, inv.data(), inv.size() * sizeof(uint32_t)))) return fail(rc);
+    }
+  }
   if (cudaStreamSynchronize(P->stream) != cudaSuccess) {
     g_last_cuda_error = (int)cudaGetLastError();
     return fail(CUSFFT_CUDA);
@@ -569,8 +622,13 @@ template <int B1T>
 cudaError_t launch_fold_fft1_t(cusfft_plan_t P, const double2* x, const SlotParam* sp, double2* u, double2* v,
                                int nslots, ZeroArgs z, cudaStream_t st) {
   dim3 grid((unsigned)(P->B / 256), (unsigned)nslots);
-  return launch_k(k_fold_fft1<B1T, 8>, grid, dim3(256), 0, st, P->cur_prio, x, (const double*)P->d_taps_perm, sp, u, v,
-                  (const double2*)P->d_tw, (int)P->B, P->B2, P->w, P->R, (uint32_t)(P->n - 1), z);
+  if (P->staged)  // x is the staging buffer; the whole rank's slots at once
+    return launch_k(k_fold_fft1<B1T, 8, true>, grid, dim3(256), 0, st, P->cur_prio, (const double2*)P->d_staging,
+                    (const uint32_t*)P->d_inv, (const double*)P->d_taps_perm, sp, u, v, (const double2*)P->d_tw,
+                    (int)P->B, P->B2, P->w, P->R, (uint32_t)(P->n - 1), z);
+  return launch_k(k_fold_fft1<B1T, 8, false>, grid, dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)nullptr,
+                  (const double*)P->d_taps_perm, sp, u, v, (const double2*)P->d_tw, (int)P->B, P->B2, P->w, P->R,
+                  (uint32_t)(P->n - 1), z);
 }
 
 cudaError_t launch_fold_fft1(cusfft_plan_t P, const double2* x, const SlotParam* sp, double2* u, double2* v,
@@ -594,6 +652,15 @@ int launch_fold(cusfft_plan_t P, const double2* x, int s0, int s1, cudaStream_t 
   const int B = (int)P->B;
   const SlotParam* sp = P->d_slots + (size_t)P->rank * P->Lg + s0;
   ZeroArgs z{zero_block ? P->d_zero : nullptr, zero_block ? P->nzero : 0};
+  if (P->staged) {  // phase 1: address-sorted gather of every local slot's samples (zeroes the block)
+    const int tot = (int)P->stage_total;
+    int sms = 148;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, P->device);
+    const int grid = std::max(1, std::min((tot + 8 * 256 - 1) / (8 * 256), sms * 8));
+    CK(launch_k(k_stage, dim3(grid), dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)P->d_spos, P->d_staging, tot,
+                z));
+    z = ZeroArgs{nullptr, 0};
+  }
   if (P->fused1) {
     CK(launch_fold_fft1(P, x, sp, P->d_u + (size_t)s0 * B, P->d_v + (size_t)s0 * B, s1 - s0, z, st));
   } else {
@@ -755,7 +822,7 @@ int launch_branched(cusfft_plan_t P, const double2* x, int64_t* locs, double2* v
 // Branched execution only inside graph capture, for full-stage runs with both
 // location and estimation-only slots on this rank.
 inline bool use_branches(cusfft_plan_t P) {
-  return P->branched && P->use_graph && !P->timing && P->stage_limit == 6 && P->nloc_local > 0 &&
+  return !P->staged && P->branched && P->use_graph && !P->timing && P->stage_limit == 6 && P->nloc_local > 0 &&
          P->nloc_local < P->Lg;
 }
 
@@ -968,8 +1035,8 @@ int cusfft_exchange_buffer(cusfft_plan_t plan, void** d_buf, int64_t* bytes_per_
 int cusfft_get_info(cusfft_plan_t plan, int64_t* info, int64_t* a, int64_t* sigma, int64_t* tau) {
   if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
   if (info) {
-    int64_t v[10] = {plan->n, plan->k, plan->B, plan->L, plan->w, plan->nb,
-                     plan->num, plan->Lloc, plan->T, plan->max_hits};
+    int64_t v[12] = {plan->n, plan->k, plan->B, plan->L, plan->w, plan->nb, plan->num, plan->Lloc, plan->T,
+                     plan->max_hits, plan->sectors, plan->staged ? 1 : 0};
     std::memcpy(info, v, sizeof(v));
   }
   for (int r = 0; r < plan->L; ++r) {
@@ -1095,7 +1162,7 @@ int cusfft_debug_trace(unsigned long long* host, int32_t n) {
 
 int32_t cusfft_launches_per_execute(cusfft_plan_t plan) {
   if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
-  int n = 1 /*fold*/ + (plan->B1 > 1 && !plan->fused1 ? 2 : 1) /*fft*/ + (plan->sel_slots_h.empty() ? 0 : 1) +
+  int n = 1 /*fold*/ + (plan->staged ? 1 : 0) + (plan->B1 > 1 && !plan->fused1 ? 2 : 1) /*fft*/ + (plan->sel_slots_h.empty() ? 0 : 1) +
           3 /*vote,est,out*/;
   return n;
 }

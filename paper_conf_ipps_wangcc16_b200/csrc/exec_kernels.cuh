@@ -83,6 +83,53 @@ __global__ void __launch_bounds__(256) k_fold(const double2* __restrict__ x, con
 }
 
 // ---------------------------------------------------------------------------
+// Staged gather, phase 1: the plan sorted every (slot, tap)
+// gather position of this rank; staging[q] = x[spos[q]] in that address order,
+// so DRAM rows are opened once for all loops' samples that share them (the
+// random-order gather is bound by row activations).  x is read evict-first
+// with 64-B L2 fetches; staging (L2-sized) is written evict-last for phase 2.
+// Also zeroes the per-execution block (first kernel of the execution).
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ uint64_t l2_policy_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t l2_policy_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+
+__global__ void __launch_bounds__(256) k_stage(const double2* __restrict__ x, const uint32_t* __restrict__ spos,
+                                               double2* __restrict__ staging, int total, ZeroArgs zero) {
+  if (blockIdx.x == 0) TRACE(0);
+  zero_part(zero);
+  const uint64_t pf = l2_policy_first(), pl = l2_policy_last();
+  const int T = gridDim.x * blockDim.x;
+  for (int q0 = blockIdx.x * blockDim.x + threadIdx.x; q0 < total; q0 += 8 * T) {
+    double2 v[8];
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      const int q = q0 + c * T;
+      if (q < total) {
+        const double2* p = x + __ldg(spos + q);
+        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.L2::64B.v2.f64 {%0, %1}, [%2], %3;"
+                     : "=d"(v[c].x), "=d"(v[c].y) : "l"(p), "l"(pf));
+      }
+    }
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      const int q = q0 + c * T;
+      if (q < total)
+        asm volatile("st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %3;" ::"l"(staging + q), "d"(v[c].x),
+                     "d"(v[c].y), "l"(pl));
+    }
+  }
+  TRACE_END(6);
+}
+
+// ---------------------------------------------------------------------------
 // Steps 1+2 fused with the first pass of Step 3 (four-step B = B1 x B2, B1 <=
 // 256): a CTA of 256 threads folds the buckets of C = 256 / B1 whole columns
 // c (j = c + B2 j1, j1 < B1) exactly as k_fold does (same per-bucket order),
@@ -93,8 +140,9 @@ __global__ void __launch_bounds__(256) k_fold(const double2* __restrict__ x, con
 // loads of a CTA stay contiguous.  RC gathers per thread in flight; two CTAs
 // per SM so one CTA's FFT epilogue overlaps the other's gathers.
 // ---------------------------------------------------------------------------
-template <int B1T, int RC>
+template <int B1T, int RC, bool STAGED>
 __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict__ x,
+                                                      const uint32_t* __restrict__ inv_perm,
                                                       const double* __restrict__ taps_perm,
                                                       const SlotParam* __restrict__ slots, double2* __restrict__ u,
                                                       double2* __restrict__ v, const double2* __restrict__ tw, int B,
@@ -113,6 +161,8 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict_
   const double2 wout = __ldg(tw + (((int64_t)c * j1) & (B - 1)));          // omega_B^(c k1), k1 = j1
   const uint32_t sigma = slots[s].sigma, tau = slots[s].tau;
   const double* tp = taps_perm + (int64_t)blockIdx.x * 256 + t;
+  // staged: x is the staging buffer, inv_perm[(s R + rr) B + cta 256 + t] its index
+  const uint32_t* ip = STAGED ? inv_perm + (int64_t)s * R * B + (int64_t)blockIdx.x * 256 + t : nullptr;
   double ar = 0.0, ai = 0.0;
   for (int r0 = 0; r0 < R; r0 += RC) {
     double2 xv[RC];
@@ -121,8 +171,12 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict_
     for (int cc = 0; cc < RC; ++cc) {
       const int i = j + (r0 + cc) * B;
       if (r0 + cc < R && i < w) {
-        const uint32_t idx = (sigma * (uint32_t)i + tau) & nmask;  // mod n, n | 2^32
-        xv[cc] = ld_gather(x + idx);
+        if (STAGED) {
+          xv[cc] = __ldcg(x + __ldg(ip + (int64_t)(r0 + cc) * B));
+        } else {
+          const uint32_t idx = (sigma * (uint32_t)i + tau) & nmask;  // mod n, n | 2^32
+          xv[cc] = ld_gather(x + idx);
+        }
         g[cc] = __ldg(tp + (int64_t)(r0 + cc) * B);
       }
     }
