@@ -27,6 +27,12 @@ __device__ __forceinline__ unsigned long long gtimer() {
 #define TRACE_END(slot) do { } while (0)
 #endif
 
+// Programmatic dependent launch: a kernel launched with programmatic stream
+// serialization may start while its predecessor drains; it must not touch
+// global memory the predecessor writes (or reads) before this wait.  No-op
+// for ordinary launches.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 // Per-slot loop parameters (slot order; see DESIGN.md §6 "slots").
 //   sigma: gather stride (Alg. 1's ai), a = sigma^-1 mod n,
 //   tau: offset (Def. 1), loop: the loop index r this slot holds.

@@ -115,10 +115,18 @@ struct cusfft_plan_s {
   // staged gather: address-sorted gather schedule of this rank
   bool staged = false;
   int64_t sectors = 0;            // distinct 32-B sectors of x gathered by this rank (the fold's DRAM floor)
-  int64_t stage_total = 0;        // Lg * w samples
-  uint32_t* d_spos = nullptr;     // [stage_total] sorted gather positions
-  uint32_t* d_inv = nullptr;      // [Lg][R][B] staging index in the fused kernel's thread order
-  double2* d_staging = nullptr;   // [stage_total]
+  // Slot groups, each with its own sorted schedule (default: one group of all
+  // local slots; CUSFFT_STAGE_GROUPS=2 splits location / estimation loops,
+  // which halves each staging buffer but costs phase-1 locality: slower on B200).
+  struct StageGroup {
+    int s0 = 0, s1 = 0;          // local slots [s0, s1)
+    int64_t total = 0;           // (s1 - s0) * w samples
+    uint32_t* spos = nullptr;    // [total] sorted gather positions
+    uint32_t* inv = nullptr;     // [s1 - s0][R][B] staging index in the fused kernel's thread order
+  };
+  std::vector<StageGroup> groups;
+  double2* d_staging = nullptr;   // [max group total]
+  cudaAccessPolicyWindow stage_window = {};  // persisting L2 window over d_staging
   double2* d_ghat = nullptr;
   double2* d_tw = nullptr;
   SlotParam* d_slots = nullptr;
@@ -188,7 +196,11 @@ struct DeviceGuard {
 };
 
 void free_plan(cusfft_plan_t p) {
-  void* ptrs[] = {p->d_taps, p->d_taps_perm, p->d_spos, p->d_inv, p->d_staging, p->d_ghat, p->d_tw, p->d_slots, p->d_loc_slots, p->d_loc_sigma, p->d_loc_a,
+  for (auto& g : p->groups) {
+    if (g.spos) cudaFree(g.spos);
+    if (g.inv) cudaFree(g.inv);
+  }
+  void* ptrs[] = {p->d_taps, p->d_taps_perm, p->d_staging, p->d_ghat, p->d_tw, p->d_slots, p->d_loc_slots, p->d_loc_sigma, p->d_loc_a,
                   p->d_sel_slots, p->d_u, p->d_v, p->d_records, p->d_keys, p->d_zero, p->d_key_index, p->d_ckey, p->d_cidx, p->d_hits, p->d_hit_vals,
                   p->d_hit_keys, p->d_per_loop, p->d_xbuf, p->d_locs_buf, p->d_vals_buf};
   for (void* q : ptrs)
@@ -294,6 +306,12 @@ int build_filter(cusfft_plan_t P) {
 
 // Kernel launch carrying an explicit scheduling priority: stream priorities are
 // not captured into graph kernel nodes, the launch attribute is.
+// g_pdl: programmatic dependent launch for this launch (every hot kernel
+// begins with pdl_wait(), so it may be launched while its predecessor drains).
+thread_local bool g_pdl = false;
+// g_apw: L2 access-policy window for this launch (persisting staging buffer).
+thread_local cudaAccessPolicyWindow g_apw = {};
+
 template <typename... KArgs, typename... Args>
 cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, int prio,
                      Args&&... args) {
@@ -302,11 +320,18 @@ cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem,
   cfg.blockDim = block;
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[3];
   attr[0].id = cudaLaunchAttributePriority;
   attr[0].val.priority = prio;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = g_pdl ? 1 : 0;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = 2;
+  if (g_apw.num_bytes) {
+    attr[2].id = cudaLaunchAttributeAccessPolicyWindow;
+    attr[2].val.accessPolicyWindow = g_apw;
+    cfg.numAttrs = 3;
+  }
   return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
 }
 
@@ -576,38 +601,65 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   }
   {
     const char* e = std::getenv("CUSFFT_NO_STAGE");
-    const int64_t total = (int64_t)P->Lg * P->w;
-    // staging must stay L2-resident between the two phases
-    P->staged = P->fused1 && total * 16 <= (int64_t)64 << 20 && total < (int64_t)1 << 31 && !(e && e[0] == '1');
+    const char* eg = std::getenv("CUSFFT_STAGE_GROUPS");
+    std::vector<std::pair<int, int>> ranges;
+    if (P->nloc_local > 0 && P->nloc_local < P->Lg && eg && eg[0] == '2')  // opt-in: two groups
+      ranges = {{0, P->nloc_local}, {P->nloc_local, P->Lg}};
+    else
+      ranges = {{0, P->Lg}};
+    int64_t maxtot = 0;
+    for (auto& r : ranges) maxtot = std::max<int64_t>(maxtot, (int64_t)(r.second - r.first) * P->w);
+    // the staging buffer must be (mostly) L2-resident between the two phases
+    P->staged = P->fused1 && maxtot * 16 <= (int64_t)64 << 20 && !(e && e[0] == '1');
     if (P->staged) {
-      P->stage_total = total;
-      std::vector<uint64_t> ev((size_t)total);
       const uint32_t nm = (uint32_t)(n - 1);
-      for (int sl = 0; sl < P->Lg; ++sl) {
-        const SlotParam& sp = P->slots_h[(size_t)rank * P->Lg + sl];
-        for (int i = 0; i < P->w; ++i) {
-          const uint32_t pos = (sp.sigma * (uint32_t)i + sp.tau) & nm;
-          const uint64_t id = (uint64_t)sl * P->w + i;
-          ev[(size_t)id] = ((uint64_t)pos << 32) | id;
-        }
-      }
-      std::sort(ev.begin(), ev.end());
-      std::vector<uint32_t> spos((size_t)total), inv((size_t)P->Lg * P->R * B, 0u);
       const int C = 256 / P->B1;
-      for (int64_t q = 0; q < total; ++q) {
-        spos[(size_t)q] = (uint32_t)(ev[(size_t)q] >> 32);
-        const uint64_t id = ev[(size_t)q] & 0xFFFFFFFFull;
-        const int64_t sl = (int64_t)(id / P->w), i = (int64_t)(id % P->w);
-        const int64_t rr = i / B, j = i % B;
-        const int64_t c = j % P->B2, j1 = j / P->B2;
-        const int64_t cta = c / C, t = (c % C) * P->B1 + j1;
-        inv[(size_t)((sl * P->R + rr) * B + cta * 256 + t)] = (uint32_t)q;
+      for (auto& r : ranges) {
+        cusfft_plan_s::StageGroup g;
+        g.s0 = r.first;
+        g.s1 = r.second;
+        g.total = (int64_t)(g.s1 - g.s0) * P->w;
+        std::vector<uint64_t> ev((size_t)g.total);
+        for (int sl = g.s0; sl < g.s1; ++sl) {
+          const SlotParam& sp = P->slots_h[(size_t)rank * P->Lg + sl];
+          for (int i = 0; i < P->w; ++i) {
+            const uint32_t pos = (sp.sigma * (uint32_t)i + sp.tau) & nm;
+            const uint64_t id = (uint64_t)(sl - g.s0) * P->w + i;
+            ev[(size_t)id] = ((uint64_t)pos << 32) | id;
+          }
+        }
+        std::sort(ev.begin(), ev.end());
+        std::vector<uint32_t> spos((size_t)g.total), inv((size_t)(g.s1 - g.s0) * P->R * B, 0u);
+        for (int64_t q = 0; q < g.total; ++q) {
+          spos[(size_t)q] = (uint32_t)(ev[(size_t)q] >> 32);
+          const uint64_t id = ev[(size_t)q] & 0xFFFFFFFFull;
+          const int64_t sl = (int64_t)(id / P->w), i = (int64_t)(id % P->w);
+          const int64_t rr = i / B, j = i % B;
+          const int64_t c = j % P->B2, j1 = j / P->B2;
+          const int64_t cta = c / C, t = (c % C) * P->B1 + j1;
+          inv[(size_t)((sl * P->R + rr) * B + cta * 256 + t)] = (uint32_t)q;
+        }
+        P->groups.push_back(g);
+        auto& gg = P->groups.back();
+        if ((rc = dalloc(&gg.spos, (size_t)g.total))) return fail(rc);
+        if ((rc = dalloc(&gg.inv, inv.size()))) return fail(rc);
+        if ((rc = upload(gg.spos, spos.data(), spos.size() * sizeof(uint32_t)))) return fail(rc);
+        if ((rc = upload(gg.inv, inv.data(), inv.size() * sizeof(uint32_t)))) return fail(rc);
       }
-      if ((rc = dalloc(&P->d_spos, (size_t)total))) return fail(rc);
-      if ((rc = dalloc(&P->d_inv, inv.size()))) return fail(rc);
-      if ((rc = dalloc(&P->d_staging, (size_t)total))) return fail(rc);
-      if ((rc = upload(P->d_spos, spos.data(), spos.size() * sizeof(uint32_t)))) return fail(rc);
-      if ((rc = upload(P->d_inv, inv.data(), inv.size() * sizeof(uint32_t)))) return fail(rc);
+      if ((rc = dalloc(&P->d_staging, (size_t)maxtot))) return fail(rc);
+      // Persisting-L2 set-aside for the staging buffer (a device-wide limit: raised, never lowered).
+      int maxp = 0;
+      cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev);
+      const size_t win = std::min<size_t>((size_t)maxtot * 16, (size_t)maxp);
+      size_t cur = 0;
+      cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+      if (win > cur) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, win);
+      cudaGetLastError();
+      P->stage_window.base_ptr = P->d_staging;
+      P->stage_window.num_bytes = win;
+      P->stage_window.hitRatio = 1.0f;
+      P->stage_window.hitProp = cudaAccessPropertyPersisting;
+      P->stage_window.missProp = cudaAccessPropertyStreaming;
     }
   }
   if (cudaStreamSynchronize(P->stream) != cudaSuccess) {
@@ -619,24 +671,24 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
 }
 
 template <int B1T>
-cudaError_t launch_fold_fft1_t(cusfft_plan_t P, const double2* x, const SlotParam* sp, double2* u, double2* v,
-                               int nslots, ZeroArgs z, cudaStream_t st) {
+cudaError_t launch_fold_fft1_t(cusfft_plan_t P, const double2* x, const uint32_t* inv, const SlotParam* sp, double2* u,
+                               double2* v, int nslots, ZeroArgs z, cudaStream_t st) {
   dim3 grid((unsigned)(P->B / 256), (unsigned)nslots);
-  if (P->staged)  // x is the staging buffer; the whole rank's slots at once
-    return launch_k(k_fold_fft1<B1T, 8, true>, grid, dim3(256), 0, st, P->cur_prio, (const double2*)P->d_staging,
-                    (const uint32_t*)P->d_inv, (const double*)P->d_taps_perm, sp, u, v, (const double2*)P->d_tw,
+  if (inv)  // staged: x is the staging buffer of the group, inv its index
+    return launch_k(k_fold_fft1<B1T, 4, true>, grid, dim3(256), 0, st, P->cur_prio, x, inv,
+                    (const double*)P->d_taps_perm, sp, u, v, (const double2*)P->d_tw,
                     (int)P->B, P->B2, P->w, P->R, (uint32_t)(P->n - 1), z);
   return launch_k(k_fold_fft1<B1T, 8, false>, grid, dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)nullptr,
                   (const double*)P->d_taps_perm, sp, u, v, (const double2*)P->d_tw, (int)P->B, P->B2, P->w, P->R,
                   (uint32_t)(P->n - 1), z);
 }
 
-cudaError_t launch_fold_fft1(cusfft_plan_t P, const double2* x, const SlotParam* sp, double2* u, double2* v,
-                             int nslots, ZeroArgs z, cudaStream_t st) {
+cudaError_t launch_fold_fft1(cusfft_plan_t P, const double2* x, const uint32_t* inv, const SlotParam* sp, double2* u,
+                             double2* v, int nslots, ZeroArgs z, cudaStream_t st) {
   switch (P->B1) {
-    case 64: return launch_fold_fft1_t<64>(P, x, sp, u, v, nslots, z, st);
-    case 128: return launch_fold_fft1_t<128>(P, x, sp, u, v, nslots, z, st);
-    case 256: return launch_fold_fft1_t<256>(P, x, sp, u, v, nslots, z, st);
+    case 64: return launch_fold_fft1_t<64>(P, x, inv, sp, u, v, nslots, z, st);
+    case 128: return launch_fold_fft1_t<128>(P, x, inv, sp, u, v, nslots, z, st);
+    case 256: return launch_fold_fft1_t<256>(P, x, inv, sp, u, v, nslots, z, st);
     default: return cudaErrorInvalidValue;
   }
 }
@@ -652,17 +704,26 @@ int launch_fold(cusfft_plan_t P, const double2* x, int s0, int s1, cudaStream_t 
   const int B = (int)P->B;
   const SlotParam* sp = P->d_slots + (size_t)P->rank * P->Lg + s0;
   ZeroArgs z{zero_block ? P->d_zero : nullptr, zero_block ? P->nzero : 0};
-  if (P->staged) {  // phase 1: address-sorted gather of every local slot's samples (zeroes the block)
-    const int tot = (int)P->stage_total;
+  if (P->staged) {  // per slot group: phase 1 (address-sorted gather into staging), phase 2 (fused fold)
     int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, P->device);
-    const int grid = std::max(1, std::min((tot + 8 * 256 - 1) / (8 * 256), sms * 8));
-    CK(launch_k(k_stage, dim3(grid), dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)P->d_spos, P->d_staging, tot,
-                z));
-    z = ZeroArgs{nullptr, 0};
-  }
-  if (P->fused1) {
-    CK(launch_fold_fft1(P, x, sp, P->d_u + (size_t)s0 * B, P->d_v + (size_t)s0 * B, s1 - s0, z, st));
+    for (const auto& g : P->groups) {
+      if (g.s1 <= s0 || g.s0 >= s1) continue;  // callers pass whole groups
+      const int tot = (int)g.total;
+      g_apw = P->stage_window;  // keep the staging buffer L2-resident for phase 2
+      const int grid = std::max(1, std::min((tot + 8 * 256 - 1) / (8 * 256), sms * 8));
+      cudaError_t e = launch_k(k_stage, dim3(grid), dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)g.spos,
+                               P->d_staging, tot, z);
+      z = ZeroArgs{nullptr, 0};
+      g_pdl = !P->timing;
+      if (e == cudaSuccess)
+        e = launch_fold_fft1(P, P->d_staging, g.inv, P->d_slots + (size_t)P->rank * P->Lg + g.s0,
+                             P->d_u + (size_t)g.s0 * B, P->d_v + (size_t)g.s0 * B, g.s1 - g.s0, z, st);
+      g_apw = cudaAccessPolicyWindow{};
+      CK(e);
+    }
+  } else if (P->fused1) {
+    CK(launch_fold_fft1(P, x, nullptr, sp, P->d_u + (size_t)s0 * B, P->d_v + (size_t)s0 * B, s1 - s0, z, st));
   } else {
     dim3 grid((B + 255) / 256, s1 - s0);
     CK(launch_k(k_fold<16>, grid, dim3(256), 0, st, P->cur_prio, x, (const double*)P->d_taps, sp,
@@ -711,7 +772,10 @@ int launch_local(cusfft_plan_t P, const double2* x) {
   cudaStream_t st = P->stream;
   int rc;
   mark(P, 0);
-  if ((rc = launch_fold(P, x, 0, P->Lg, st, true))) return rc;
+  g_pdl = false;  // the first kernel follows arbitrary caller work
+  rc = launch_fold(P, x, 0, P->Lg, st, true);
+  g_pdl = !P->timing;
+  if (rc) return rc;
   mark(P, 1);
   if (P->stage_limit < 2) return CUSFFT_SUCCESS;
   if ((rc = launch_bfft(P, 0, P->Lg, st))) return rc;
@@ -764,16 +828,15 @@ int launch_estimate(cusfft_plan_t P, cudaStream_t st) {
   ea.hit_keys = P->d_hit_keys;
   ea.per_loop = P->d_per_loop;
   ea.out_hist = P->d_ohist;
-  k_estimate<<<P->est_grid, 256, 0, st>>>(ea);
-  CKL();
+  CK(launch_k(k_estimate, dim3(P->est_grid), dim3(256), 0, st, P->cur_prio, ea));
   return CUSFFT_SUCCESS;
 }
 
 int launch_output(cusfft_plan_t P, int64_t* locs, double2* vals, cudaStream_t st) {
-  k_output<<<1, 1024, P->output_smem, st>>>(P->d_hits, reinterpret_cast<const unsigned*>(P->d_flags), P->max_hits,
-                                            P->d_hit_vals, P->d_hit_keys, P->d_ohist, (int)P->k, P->kp2,
-                                            ilog2(P->n), locs, vals, P->d_flags + 1);
-  CKL();
+  CK(launch_k(k_output, dim3(1), dim3(1024), P->output_smem, st, P->cur_prio, (const int*)P->d_hits,
+              reinterpret_cast<const unsigned*>(P->d_flags), P->max_hits, (const double2*)P->d_hit_vals,
+              (const uint64_t*)P->d_hit_keys, P->d_ohist, (int)P->k, P->kp2, ilog2(P->n), locs, vals,
+              P->d_flags + 1));
   return CUSFFT_SUCCESS;
 }
 
@@ -781,6 +844,7 @@ int launch_finish(cusfft_plan_t P, int64_t* locs, double2* vals) {
   cudaStream_t st = P->stream;
   int rc;
   if (P->stage_limit < 4) return CUSFFT_SUCCESS;
+  g_pdl = !P->timing;  // every kernel waits for its predecessor before touching memory
   if ((rc = launch_vote(P, st))) return rc;
   mark(P, 4);
   if (P->stage_limit < 5) return CUSFFT_SUCCESS;
@@ -1162,7 +1226,7 @@ int cusfft_debug_trace(unsigned long long* host, int32_t n) {
 
 int32_t cusfft_launches_per_execute(cusfft_plan_t plan) {
   if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
-  int n = 1 /*fold*/ + (plan->staged ? 1 : 0) + (plan->B1 > 1 && !plan->fused1 ? 2 : 1) /*fft*/ + (plan->sel_slots_h.empty() ? 0 : 1) +
+  int n = (plan->staged ? 2 * (int)plan->groups.size() : 1) /*stage + fold per group*/ + (plan->B1 > 1 && !plan->fused1 ? 2 : 1) /*fft*/ + (plan->sel_slots_h.empty() ? 0 : 1) +
           3 /*vote,est,out*/;
   return n;
 }

@@ -50,6 +50,7 @@ template <int RC>
 __global__ void __launch_bounds__(256) k_fold(const double2* __restrict__ x, const double* __restrict__ taps,
                                               const SlotParam* __restrict__ slots, double2* __restrict__ u,
                                               int B, int w, int R, uint32_t nmask, ZeroArgs zero) {
+  pdl_wait();
   const int j = blockIdx.x * blockDim.x + threadIdx.x;
   const int s = blockIdx.y;
   if (blockIdx.x == 0 && blockIdx.y == 0) TRACE(0);
@@ -103,6 +104,7 @@ __device__ __forceinline__ uint64_t l2_policy_last() {
 
 __global__ void __launch_bounds__(256) k_stage(const double2* __restrict__ x, const uint32_t* __restrict__ spos,
                                                double2* __restrict__ staging, int total, ZeroArgs zero) {
+  pdl_wait();
   if (blockIdx.x == 0) TRACE(0);
   zero_part(zero);
   const uint64_t pf = l2_policy_first(), pl = l2_policy_last();
@@ -141,12 +143,14 @@ __global__ void __launch_bounds__(256) k_stage(const double2* __restrict__ x, co
 // per SM so one CTA's FFT epilogue overlaps the other's gathers.
 // ---------------------------------------------------------------------------
 template <int B1T, int RC, bool STAGED>
-__global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict__ x,
-                                                      const uint32_t* __restrict__ inv_perm,
-                                                      const double* __restrict__ taps_perm,
-                                                      const SlotParam* __restrict__ slots, double2* __restrict__ u,
-                                                      double2* __restrict__ v, const double2* __restrict__ tw, int B,
-                                                      int B2, int w, int R, uint32_t nmask, ZeroArgs zero) {
+__global__ void __launch_bounds__(256, STAGED ? 3 : 2) k_fold_fft1(const double2* __restrict__ x,
+                                                                   const uint32_t* __restrict__ inv_perm,
+                                                                   const double* __restrict__ taps_perm,
+                                                                   const SlotParam* __restrict__ slots,
+                                                                   double2* __restrict__ u, double2* __restrict__ v,
+                                                                   const double2* __restrict__ tw, int B, int B2,
+                                                                   int w, int R, uint32_t nmask, ZeroArgs zero) {
+  pdl_wait();
   constexpr int C = 256 / B1T;
   __shared__ double2 S[256 + 256 / 8];
   __shared__ double2 twl[B1T];
@@ -159,33 +163,62 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict_
   zero_part(zero);
   for (int i = t; i < B1T; i += 256) twl[i] = __ldg(tw + (int64_t)i * B2);  // omega_B1^i
   const double2 wout = __ldg(tw + (((int64_t)c * j1) & (B - 1)));          // omega_B^(c k1), k1 = j1
-  const uint32_t sigma = slots[s].sigma, tau = slots[s].tau;
   const double* tp = taps_perm + (int64_t)blockIdx.x * 256 + t;
-  // staged: x is the staging buffer, inv_perm[(s R + rr) B + cta 256 + t] its index
-  const uint32_t* ip = STAGED ? inv_perm + (int64_t)s * R * B + (int64_t)blockIdx.x * 256 + t : nullptr;
   double ar = 0.0, ai = 0.0;
-  for (int r0 = 0; r0 < R; r0 += RC) {
-    double2 xv[RC];
-    double g[RC];
+  if constexpr (STAGED) {
+    // phase 2: every round's staging index first (one dependent step), then
+    // the L2-resident samples in chunks of RC, accumulated in round order.
+    constexpr int RMAX = 16;
+    const uint32_t* ip = inv_perm + (int64_t)s * R * B + (int64_t)blockIdx.x * 256 + t;
+    uint32_t q[RMAX];
 #pragma unroll
-    for (int cc = 0; cc < RC; ++cc) {
-      const int i = j + (r0 + cc) * B;
-      if (r0 + cc < R && i < w) {
-        if (STAGED) {
-          xv[cc] = __ldcg(x + __ldg(ip + (int64_t)(r0 + cc) * B));
-        } else {
-          const uint32_t idx = (sigma * (uint32_t)i + tau) & nmask;  // mod n, n | 2^32
-          xv[cc] = ld_gather(x + idx);
+    for (int rr = 0; rr < RMAX; ++rr) q[rr] = (rr < R && j + rr * B < w) ? __ldg(ip + (int64_t)rr * B) : 0xFFFFFFFFu;
+#pragma unroll
+    for (int r0 = 0; r0 < RMAX; r0 += RC) {
+      double2 xv[RC];
+#pragma unroll
+      for (int cc = 0; cc < RC; ++cc)
+        if (q[r0 + cc] != 0xFFFFFFFFu) xv[cc] = __ldcg(x + q[r0 + cc]);
+#pragma unroll
+      for (int cc = 0; cc < RC; ++cc) {
+        if (q[r0 + cc] != 0xFFFFFFFFu) {
+          const double g = __ldg(tp + (int64_t)(r0 + cc) * B);
+          ar = __dadd_rn(ar, __dmul_rn(g, xv[cc].x));
+          ai = __dadd_rn(ai, __dmul_rn(g, xv[cc].y));
         }
-        g[cc] = __ldg(tp + (int64_t)(r0 + cc) * B);
       }
     }
+    for (int rr = RMAX; rr < R; ++rr) {  // R > 16 (small tolerance / Gaussian filters)
+      const int i = j + rr * B;
+      if (i < w) {
+        const double2 xv = __ldcg(x + __ldg(inv_perm + (int64_t)s * R * B + (int64_t)rr * B +
+                                            (int64_t)blockIdx.x * 256 + t));
+        const double g = __ldg(tp + (int64_t)rr * B);
+        ar = __dadd_rn(ar, __dmul_rn(g, xv.x));
+        ai = __dadd_rn(ai, __dmul_rn(g, xv.y));
+      }
+    }
+  } else {
+    const uint32_t sigma = slots[s].sigma, tau = slots[s].tau;
+    for (int r0 = 0; r0 < R; r0 += RC) {
+      double2 xv[RC];
+      double g[RC];
 #pragma unroll
-    for (int cc = 0; cc < RC; ++cc) {
-      const int i = j + (r0 + cc) * B;
-      if (r0 + cc < R && i < w) {
-        ar = __dadd_rn(ar, __dmul_rn(g[cc], xv[cc].x));
-        ai = __dadd_rn(ai, __dmul_rn(g[cc], xv[cc].y));
+      for (int cc = 0; cc < RC; ++cc) {
+        const int i = j + (r0 + cc) * B;
+        if (r0 + cc < R && i < w) {
+          const uint32_t idx = (sigma * (uint32_t)i + tau) & nmask;  // mod n, n | 2^32
+          xv[cc] = ld_gather(x + idx);
+          g[cc] = __ldg(tp + (int64_t)(r0 + cc) * B);
+        }
+      }
+#pragma unroll
+      for (int cc = 0; cc < RC; ++cc) {
+        const int i = j + (r0 + cc) * B;
+        if (r0 + cc < R && i < w) {
+          ar = __dadd_rn(ar, __dmul_rn(g[cc], xv[cc].x));
+          ai = __dadd_rn(ai, __dmul_rn(g[cc], xv[cc].y));
+        }
       }
     }
   }
@@ -373,6 +406,7 @@ struct GKeySrc {
 };
 
 __global__ void __launch_bounds__(kSelNT) k_select(SelArgs A) {
+  pdl_wait();
   extern __shared__ __align__(16) uint8_t smem[];
   uint32_t* hist = reinterpret_cast<uint32_t*>(smem);
   int* sm = reinterpret_cast<int*>(smem + 4096 * 4);
@@ -667,6 +701,7 @@ __device__ __forceinline__ void vote_unit(const VoteArgs& A, const uint32_t* __r
 }
 
 __global__ void __launch_bounds__(256) k_vote(VoteArgs A) {
+  pdl_wait();
   extern __shared__ __align__(16) uint8_t smem[];
   if (blockIdx.x == 0) TRACE(30);
   uint32_t* bm = reinterpret_cast<uint32_t*>(smem);
@@ -802,6 +837,7 @@ __device__ __forceinline__ double warp_rank_select(double a0, double a1, int L, 
 }
 
 __global__ void __launch_bounds__(256) k_estimate(EstArgs A) {
+  pdl_wait();
   __shared__ uint32_t sdig[8];
   if (blockIdx.x == 0) TRACE(40);
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -863,6 +899,7 @@ __global__ void __launch_bounds__(1024) k_output(const int* __restrict__ hits, c
                                                  const uint64_t* __restrict__ hit_keys, uint32_t* __restrict__ ghist,
                                                  int k, int kp2, int log2n, int64_t* __restrict__ locs,
                                                  double2* __restrict__ vals, int* __restrict__ status) {
+  pdl_wait();
   extern __shared__ __align__(16) uint8_t smem[];
   uint32_t* hist = reinterpret_cast<uint32_t*>(smem);
   int* sm = reinterpret_cast<int*>(smem + 4096 * 4);

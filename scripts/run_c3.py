@@ -7,9 +7,10 @@ from paper_conf_ipps_wangcc16_b200.workload import planted_signal
 cfg = sys.argv[1] if len(sys.argv) > 1 else "C3"
 n, k = {"C1": (2**14, 8), "C2": (2**20, 100), "C3": (2**24, 1000), "C4": (2**27, 1000)}[cfg]
 reps = int(sys.argv[2]) if len(sys.argv) > 2 else 4
+LL = int(sys.argv[3]) if len(sys.argv) > 3 else 16
 x, S, X = planted_signal(n, k, 1)
 xd = torch.from_numpy(x).cuda()
-plan = Plan(n, k, L=16, seed=3)
+plan = Plan(n, k, L=LL, seed=3)
 for _ in range(reps):
     locs, vals = plan.execute(xd)
 torch.cuda.synchronize()
