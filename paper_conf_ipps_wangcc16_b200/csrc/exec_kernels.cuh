@@ -623,6 +623,12 @@ __device__ __forceinline__ void vote_emit(const VoteArgs& A, bool hit, uint32_t 
 // M = mandatory probes (compile time; M == 0: runtime count mrt).  Survivors
 // of the mandatory probes are queued in shared memory (qF: scaled f, qG:
 // votes so far) and finished 32 at a time (convergent).
+__device__ __forceinline__ uint32_t lds_u32(uint32_t saddr) {
+  uint32_t v;
+  asm("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(saddr));
+  return v;
+}
+
 template <int M>
 __device__ __forceinline__ void vote_unit(const VoteArgs& A, const uint32_t* __restrict__ bm, const uint32_t* ssig,
                                           int words, int q0, uint32_t Jv, uint32_t a, int mrt, uint32_t* qF,
@@ -634,13 +640,17 @@ __device__ __forceinline__ void vote_unit(const VoteArgs& A, const uint32_t* __r
   const uint32_t half_s = half << sh;
   const int m = M > 0 ? M : mrt;
   const int allowed = A.Lloc - A.T - q0;
-  int base[MM];
+  // 32-bit shared addresses of the probed bitmaps; sigma from global so that
+  // it stays in registers
+  const uint32_t bm_s = (uint32_t)__cvta_generic_to_shared(bm);
+  uint32_t base[MM];
   uint32_t sg[MM];
 #pragma unroll
   for (int qq = 0; qq < MM; ++qq) {
-    base[qq] = (q0 + 1 + qq) * words;
-    sg[qq] = ssig[q0 + 1 + qq];
+    base[qq] = bm_s + (uint32_t)((q0 + 1 + qq) * words) * 4u;
+    sg[qq] = __ldg(A.loc_sigma + q0 + 1 + qq);
   }
+  const int wsh = bsh + 5;
   const uint32_t p0 = Jv * (uint32_t)A.nb - half;
   uint32_t F0 = a * ((p0 + (uint32_t)lane) << sh);
   const uint32_t d32 = a * (32u << sh);
@@ -652,10 +662,11 @@ __device__ __forceinline__ void vote_unit(const VoteArgs& A, const uint32_t* __r
     if (M > 0) {
 #pragma unroll
       for (int qq = 0; qq < MM; ++qq) {
-        const uint32_t b0 = (sg[qq] * F0 + half_s) >> bsh;
-        const uint32_t b1 = (sg[qq] * F1 + half_s) >> bsh;
-        g0 += (bm[base[qq] + (b0 >> 5)] >> (b0 & 31)) & 1u;
-        g1 += (bm[base[qq] + (b1 >> 5)] >> (b1 & 31)) & 1u;
+        const uint32_t h0 = sg[qq] * F0 + half_s, h1 = sg[qq] * F1 + half_s;
+        const uint32_t w0 = lds_u32(base[qq] + ((h0 >> wsh) << 2));
+        const uint32_t w1 = lds_u32(base[qq] + ((h1 >> wsh) << 2));
+        g0 += __funnelshift_r(w0, w0, h0 >> bsh) & 1u;
+        g1 += __funnelshift_r(w1, w1, h1 >> bsh) & 1u;
       }
     } else {
       for (int qq = 0; qq < m; ++qq) {
@@ -667,27 +678,29 @@ __device__ __forceinline__ void vote_unit(const VoteArgs& A, const uint32_t* __r
     const bool s1 = (t0 + 32 + lane < A.nb) && (m - g1) <= allowed;
     const unsigned b0 = __ballot_sync(kFull, s0);
     const unsigned b1 = __ballot_sync(kFull, s1);
-    const unsigned lt = (1u << lane) - 1;
-    if (s0) {
-      const int pos = qn + __popc(b0 & lt);
-      qF[pos] = F0;
-      qG[pos] = (uint8_t)g0;
-    }
-    const int qn1 = qn + __popc(b0);
-    if (s1) {
-      const int pos = qn1 + __popc(b1 & lt);
-      qF[pos] = F1;
-      qG[pos] = (uint8_t)g1;
-    }
-    qn = qn1 + __popc(b1);
-    __syncwarp();
-    while (qn >= 32) {  // finish 32 queued survivors, one per lane
-      const uint32_t Fq = qF[qn - 32 + lane];
-      const int gq = qG[qn - 32 + lane];
+    if (b0 | b1) {
+      const unsigned lt = (1u << lane) - 1;
+      if (s0) {
+        const int pos = qn + __popc(b0 & lt);
+        qF[pos] = F0;
+        qG[pos] = (uint8_t)g0;
+      }
+      const int qn1 = qn + __popc(b0);
+      if (s1) {
+        const int pos = qn1 + __popc(b1 & lt);
+        qF[pos] = F1;
+        qG[pos] = (uint8_t)g1;
+      }
+      qn = qn1 + __popc(b1);
       __syncwarp();
-      qn -= 32;
-      const bool hit = vote_finish(A, bm, ssig, words, q0, m, Fq, gq, half_s, bsh);
-      vote_emit(A, hit, Fq >> sh);
+      while (qn >= 32) {  // finish 32 queued survivors, one per lane
+        const uint32_t Fq = qF[qn - 32 + lane];
+        const int gq = qG[qn - 32 + lane];
+        __syncwarp();
+        qn -= 32;
+        const bool hit = vote_finish(A, bm, ssig, words, q0, m, Fq, gq, half_s, bsh);
+        vote_emit(A, hit, Fq >> sh);
+      }
     }
   }
   if (qn > 0) {
