@@ -221,6 +221,7 @@ int validate(int64_t n, int64_t k, int64_t B, int32_t L, const cusfft_params& q,
   if (!is_pow2(n) || n < 16 || n > (int64_t(1) << 31)) return CUSFFT_INVALID_N;
   if (!is_pow2(B) || B < 2 || B >= n) return CUSFFT_INVALID_B;
   if (L < 1 || L > kMaxLoops) return CUSFFT_INVALID_LOOPS;
+  if (q.loc_loops > kMaxLoc) return CUSFFT_INVALID_LOOPS;
   if (world < 1 || rank < 0 || rank >= world || L % world) return CUSFFT_INVALID_LOOPS;
   if (q.loc_loops < 1 || q.loc_loops > L || q.vote_threshold < 1 || q.vote_threshold > q.loc_loops)
     return CUSFFT_INVALID_LOOPS;
@@ -761,8 +762,21 @@ int launch_bfft(cusfft_plan_t P, int s0, int s1, cudaStream_t st) {
 // Step 4 for this rank's location slots.
 int launch_select(cusfft_plan_t P, cudaStream_t st) {
   if (P->sel_slots_h.empty()) return CUSFFT_SUCCESS;
-  SelArgs sa{P->d_records, P->lay, P->d_sel_slots, (int)P->B, P->num, P->sel_S, P->d_keys, P->d_hist, P->d_hist1,
-             P->d_ckey, P->d_cidx, P->d_ccount, P->d_done, P->d_flags + 1};
+  SelArgs sa{};
+  for (size_t i = 0; i < P->sel_slots_h.size(); ++i)
+    sa.recs[i] = P->d_records + (int64_t)P->sel_slots_h[i] * P->lay.rec_bytes;
+  sa.lay = P->lay;
+  sa.B = (int)P->B;
+  sa.num = P->num;
+  sa.S = P->sel_S;
+  sa.keys = P->d_keys;
+  sa.hist0 = P->d_hist;
+  sa.hist1 = P->d_hist1;
+  sa.ckey = P->d_ckey;
+  sa.cidx = P->d_cidx;
+  sa.ccount = P->d_ccount;
+  sa.done = P->d_done;
+  sa.status = P->d_flags + 1;
   CK(launch_k(k_select, dim3((int)P->sel_slots_h.size() * P->sel_S), dim3(kSelNT), P->select_smem, st, P->cur_prio,
               sa));
   return CUSFFT_SUCCESS;
@@ -788,11 +802,14 @@ int launch_local(cusfft_plan_t P, const double2* x) {
 
 int launch_vote(cusfft_plan_t P, cudaStream_t st) {
   VoteArgs va;
-  va.records = P->d_records;
-  va.lay = P->lay;
-  va.loc_slots = P->d_loc_slots;
+  for (int q = 0; q < P->Lloc; ++q) {
+    const uint8_t* rec = P->d_records + (int64_t)P->loc_slots_h[q] * P->lay.rec_bytes;
+    va.bmp[q] = reinterpret_cast<const uint32_t*>(rec + P->lay.off_bitmap);
+    va.Jp[q] = reinterpret_cast<const int*>(rec + P->lay.off_J);
+    va.sig[q] = P->slots_h[P->loc_slots_h[q]].sigma;
+    va.aa[q] = P->slots_h[P->loc_slots_h[q]].a;
+  }
   va.loc_sigma = P->d_loc_sigma;
-  va.loc_a = P->d_loc_a;
   va.Lloc = P->Lloc;
   va.T = P->T;
   va.num = P->num;

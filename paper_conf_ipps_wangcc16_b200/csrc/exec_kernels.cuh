@@ -383,9 +383,8 @@ constexpr int kSelCap = 4096;
 constexpr int kSelNT = 256;
 
 struct SelArgs {
-  uint8_t* records;
+  uint8_t* recs[32];  // record of each location slot of this rank (by value)
   RecLayout lay;
-  const int* sel_slots;
   int B, num, S;
   const uint64_t* keys;  // [n_sel][B]
   uint32_t* hist0;       // [n_sel][4096] (FFT epilogue)
@@ -414,7 +413,7 @@ __global__ void __launch_bounds__(kSelNT) k_select(SelArgs A) {
   int* sidx = reinterpret_cast<int*>(skey + kSelCap);
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   const int sel = blockIdx.x / A.S, part = blockIdx.x - sel * A.S;
-  uint8_t* rec = A.records + (int64_t)A.sel_slots[sel] * A.lay.rec_bytes;
+  uint8_t* rec = A.recs[sel];
   uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap);
   const uint64_t* keys = A.keys + (int64_t)sel * A.B;
   uint32_t* h0 = A.hist0 + (int64_t)sel * 4096;
@@ -572,12 +571,15 @@ __global__ void __launch_bounds__(kSelNT) k_select(SelArgs A) {
 // and then check the earlier loops.
 // Dynamic smem: L_loc * ceil(B/32) u32 bitmaps.
 // ---------------------------------------------------------------------------
+constexpr int kMaxLoc = 32;  // location loops per plan (kernel-argument arrays)
+
 struct VoteArgs {
-  const uint8_t* records;
-  RecLayout lay;
-  const int* loc_slots;  // [L_loc] slot of each location loop, in vote order
-  const uint32_t* loc_sigma;
-  const uint32_t* loc_a;
+  // per location loop, in vote order, by value (no dependent loads):
+  const uint32_t* bmp[kMaxLoc];  // cutoff bitmap in the exchange buffer
+  const int* Jp[kMaxLoc];        // ascending winner list
+  uint32_t sig[kMaxLoc];         // sigma
+  uint32_t aa[kMaxLoc];          // a = sigma^-1
+  const uint32_t* loc_sigma;     // the same sigmas in global memory (register-resident loads)
   int Lloc, T, num, B, nb, log2nb, log2n, log2B;
   uint32_t nmask;
   int* hits;
@@ -722,34 +724,29 @@ __global__ void __launch_bounds__(256) k_vote(VoteArgs A) {
   __shared__ uint32_t queueF[8][96];
   __shared__ uint8_t queueG[8][96];
   const int words = (A.B + 31) >> 5;
-  if ((words & 3) == 0) {  // 16-B vector loads, 8 in flight per thread
-    const int v4 = words >> 2, tot = A.Lloc * v4;
-    uint4* bm4 = reinterpret_cast<uint4*>(bm);
-    for (int i0 = 0; i0 < tot; i0 += 8 * (int)blockDim.x) {
-      uint4 tmp[8];
+  if ((words & 3) == 0) {  // 16-B vector loads, all loops' words in flight before the first store
+    const int lv4 = A.log2B - 7;  // log2(words / 4)
+    const int tot = A.Lloc << lv4;
+    constexpr int PER = 8;
+    uint4* dst = reinterpret_cast<uint4*>(bm);
+    for (int i0 = 0; i0 < tot; i0 += PER * (int)blockDim.x) {
+      uint4 tmp[PER];
 #pragma unroll
-      for (int u = 0; u < 8; ++u) {
+      for (int u = 0; u < PER; ++u) {
         const int i = i0 + u * blockDim.x + threadIdx.x;
-        if (i < tot) {
-          const int q = i / v4, w = i - q * v4;
-          tmp[u] = __ldg(reinterpret_cast<const uint4*>(A.records + (int64_t)A.loc_slots[q] * A.lay.rec_bytes +
-                                                        A.lay.off_bitmap) + w);
-        }
+        if (i < tot) tmp[u] = __ldg(reinterpret_cast<const uint4*>(A.bmp[i >> lv4]) + (i & ((1 << lv4) - 1)));
       }
 #pragma unroll
-      for (int u = 0; u < 8; ++u) {
+      for (int u = 0; u < PER; ++u) {
         const int i = i0 + u * blockDim.x + threadIdx.x;
-        if (i < tot) bm4[i] = tmp[u];
+        if (i < tot) dst[i] = tmp[u];
       }
     }
   } else {
-    for (int q = 0; q < A.Lloc; ++q) {
-      const uint32_t* src = reinterpret_cast<const uint32_t*>(A.records + (int64_t)A.loc_slots[q] * A.lay.rec_bytes +
-                                                               A.lay.off_bitmap);
-      for (int i = threadIdx.x; i < words; i += blockDim.x) bm[q * words + i] = src[i];
-    }
+    for (int q = 0; q < A.Lloc; ++q)
+      for (int i = threadIdx.x; i < words; i += blockDim.x) bm[q * words + i] = A.bmp[q][i];
   }
-  if (threadIdx.x < A.Lloc) ssig[threadIdx.x] = A.loc_sigma[threadIdx.x];
+  if (threadIdx.x < A.Lloc) ssig[threadIdx.x] = A.sig[threadIdx.x];
   __syncthreads();
   if (blockIdx.x == 0) TRACE(31);
   const int units = (A.Lloc - A.T + 1) * A.num;
@@ -760,9 +757,8 @@ __global__ void __launch_bounds__(256) k_vote(VoteArgs A) {
   for (int unit = warp; unit < units; unit += nwarps) {
     const int q0 = unit / A.num;
     const int jidx = unit - q0 * A.num;
-    const int* Jl = reinterpret_cast<const int*>(A.records + (int64_t)A.loc_slots[q0] * A.lay.rec_bytes + A.lay.off_J);
-    const uint32_t Jv = (uint32_t)__ldg(Jl + jidx);
-    const uint32_t a = __ldg(A.loc_a + q0);
+    const uint32_t Jv = (uint32_t)__ldg(A.Jp[q0] + jidx);
+    const uint32_t a = A.aa[q0];
     const int m = min(A.Lloc - A.T - q0 + 1, A.Lloc - 1 - q0);  // mandatory probes
     switch (m) {
       case 0: vote_unit<0>(A, bm, ssig, words, q0, Jv, a, 0, qF, qG); break;
