@@ -61,6 +61,17 @@ typedef enum {
   CUSFFT_FILTER_GAUSSIAN = 1         /* L25, L85 */
 } cusfft_filter_t;
 
+/* Step 4 cutoff (L89).  EXACT: the num buckets of largest |u^|^2 (ties to the
+ * smaller bucket) by linear-time selection (default).  SORT: the same set by
+ * Alg. 3's sort-and-select (L238-L250), a full per-loop sort kept as an
+ * ablation (B <= 16384).  THRESHOLD: Alg. 6 (L361-L390), every bucket with
+ * |u^|^2 >= cutoff_threshold, a variable count ("slightly more than k", L390). */
+typedef enum {
+  CUSFFT_CUTOFF_EXACT = 0,
+  CUSFFT_CUTOFF_SORT = 1,
+  CUSFFT_CUTOFF_THRESHOLD = 2
+} cusfft_cutoff_t;
+
 /* Plan parameters.  Fill with cusfft_params_default, then override. */
 typedef struct {
   int32_t filter;          /* cusfft_filter_t; default DOLPH_CHEBYSHEV (L85)                     */
@@ -79,6 +90,8 @@ typedef struct {
                               NULL: build the filter from filter/tolerance/lobefrac/box_width.
                               Copied at plan time; the caller keeps ownership.                    */
   int64_t num_taps;        /* length of taps when taps != NULL (odd not required)                */
+  int32_t cutoff_mode;     /* cusfft_cutoff_t; default EXACT                                      */
+  double cutoff_threshold; /* THRESHOLD mode: absolute |u^|^2 threshold (> 0)                    */
 } cusfft_params;
 
 /* Fill *p with the defaults for (n, k, B).  Returns CUSFFT_NULL_PTR / INVALID_*. */
@@ -146,7 +159,8 @@ int cusfft_get_info(cusfft_plan_t plan, int64_t* info, int64_t* a, int64_t* sigm
 typedef enum {
   CUSFFT_DEBUG_U = 0,        /* complex fp64 [L_local][B]: fold output, this rank's loops  */
   CUSFFT_DEBUG_UHAT = 1,     /* complex fp64 [L][B]: B-point FFTs, loop order                */
-  CUSFFT_DEBUG_WINNERS = 2,  /* int32 [L_loc][num_select]: kept buckets, ascending            */
+  CUSFFT_DEBUG_WINNERS = 2,  /* int32 [L_loc][cap]: kept buckets, ascending, -1 padded; cap =
+                                num_select (B in THRESHOLD mode)                              */
   CUSFFT_DEBUG_HITS = 3,     /* int32 [H]: frequencies with >= T votes (unordered)           */
   CUSFFT_DEBUG_HIT_VALS = 4, /* complex fp64 [H]: median estimates aligned with HITS          */
   CUSFFT_DEBUG_PER_LOOP = 5, /* complex fp64 [H][L]: per-loop estimates (params.debug = 1)    */

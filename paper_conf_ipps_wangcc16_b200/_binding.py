@@ -22,6 +22,8 @@ NULL_PTR, ALLOC, CUDA, HIT_OVERFLOW, INVALID_PLAN, INTERNAL = -6, -7, -8, -9, -1
 FILTER_DOLPH_CHEBYSHEV = 0
 FILTER_GAUSSIAN = 1
 
+CUTOFF_EXACT, CUTOFF_SORT, CUTOFF_THRESHOLD = 0, 1, 2
+
 DEBUG_U, DEBUG_UHAT, DEBUG_WINNERS, DEBUG_HITS, DEBUG_HIT_VALS = 0, 1, 2, 3, 4
 DEBUG_PER_LOOP, DEBUG_TAPS, DEBUG_GHAT, DEBUG_NUM_HITS = 5, 6, 7, 8
 
@@ -52,6 +54,8 @@ class CusfftParams(ctypes.Structure):
         ("debug", ctypes.c_int32),
         ("taps", ctypes.POINTER(ctypes.c_double)),
         ("num_taps", ctypes.c_int64),
+        ("cutoff_mode", ctypes.c_int32),
+        ("cutoff_threshold", ctypes.c_double),
     ]
 
 
@@ -283,7 +287,7 @@ class Plan:
         elif what == DEBUG_UHAT:
             buf = buf.reshape(self.L, self.B)
         elif what == DEBUG_WINNERS:
-            buf = buf.reshape(self.loc_loops, self.num)
+            buf = buf.reshape(self.loc_loops, -1)
         elif what == DEBUG_PER_LOOP and buf.size:
             buf = buf.reshape(-1, self.L)
         return buf

@@ -99,6 +99,7 @@ struct cusfft_plan_s {
   int L = 0, Lg = 0, rank = 0, world = 1;
   cusfft_params prm{};
   int log2nb = 0, w = 0, R = 0, num = 0, Lloc = 0, T = 0, max_hits = 0;
+  int Jcap = 0;  // winner-list capacity per loop (num, or B in THRESHOLD mode)
   int B1 = 1, B2 = 1, logB1 = 0, logB2 = 0;
   int kp2 = 1;
   int select_smem = 0, vote_smem = 0, output_smem = 0;
@@ -235,6 +236,9 @@ int validate(int64_t n, int64_t k, int64_t B, int32_t L, const cusfft_params& q,
     if (q.box_width < 1 || q.box_width > n || (q.box_width % 2) == 0) return CUSFFT_INVALID_PARAM;
   }
   if (q.max_hits < 1 || q.max_hits > (int64_t(1) << 30)) return CUSFFT_INVALID_PARAM;
+  if (q.cutoff_mode < CUSFFT_CUTOFF_EXACT || q.cutoff_mode > CUSFFT_CUTOFF_THRESHOLD) return CUSFFT_INVALID_PARAM;
+  if (q.cutoff_mode == CUSFFT_CUTOFF_SORT && B > 16384) return CUSFFT_INVALID_PARAM;
+  if (q.cutoff_mode == CUSFFT_CUTOFF_THRESHOLD && !(q.cutoff_threshold > 0.0)) return CUSFFT_INVALID_PARAM;
   if (q.tau_mode != 0 && q.tau_mode != 1) return CUSFFT_INVALID_PARAM;
   return CUSFFT_SUCCESS;
 }
@@ -467,9 +471,11 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
 
   // ---- layout
   auto align256 = [](int64_t v) { return (v + 255) & ~int64_t(255); };
+  P->Jcap = q.cutoff_mode == CUSFFT_CUTOFF_THRESHOLD ? (int)B : P->num;
   P->lay.off_bitmap = align256(B * 16);
-  P->lay.off_J = align256(P->lay.off_bitmap + ((B + 31) / 32) * 4);
-  P->lay.rec_bytes = align256(P->lay.off_J + (int64_t)P->num * 4);
+  P->lay.off_cnt = align256(P->lay.off_bitmap + ((B + 31) / 32) * 4);
+  P->lay.off_J = P->lay.off_cnt + 16;
+  P->lay.rec_bytes = align256(P->lay.off_J + (int64_t)P->Jcap * 4);
   if (B <= 2048) {
     P->B1 = 1; P->B2 = (int)B;
   } else {
@@ -562,6 +568,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   }
   if (set_fft_attrs() != cudaSuccess ||
       cudaFuncSetAttribute(k_select, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
+      cudaFuncSetAttribute(k_select_sort, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_vote, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_output, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess) {
     g_last_cuda_error = (int)cudaGetLastError();
@@ -777,6 +784,18 @@ int launch_select(cusfft_plan_t P, cudaStream_t st) {
   sa.ccount = P->d_ccount;
   sa.done = P->d_done;
   sa.status = P->d_flags + 1;
+  sa.threshold_mode = P->prm.cutoff_mode == CUSFFT_CUTOFF_THRESHOLD ? 1 : 0;
+  {
+    const double th = P->prm.cutoff_threshold;
+    uint64_t bits;
+    std::memcpy(&bits, &th, 8);
+    sa.thr_key = bits;
+  }
+  if (P->prm.cutoff_mode == CUSFFT_CUTOFF_SORT) {
+    const int smem = (int)P->B * 12 + (int)((P->B + 31) / 32) * 4;
+    CK(launch_k(k_select_sort, dim3((int)P->sel_slots_h.size()), dim3(1024), smem, st, P->cur_prio, sa));
+    return CUSFFT_SUCCESS;
+  }
   CK(launch_k(k_select, dim3((int)P->sel_slots_h.size() * P->sel_S), dim3(kSelNT), P->select_smem, st, P->cur_prio,
               sa));
   return CUSFFT_SUCCESS;
@@ -806,6 +825,7 @@ int launch_vote(cusfft_plan_t P, cudaStream_t st) {
     const uint8_t* rec = P->d_records + (int64_t)P->loc_slots_h[q] * P->lay.rec_bytes;
     va.bmp[q] = reinterpret_cast<const uint32_t*>(rec + P->lay.off_bitmap);
     va.Jp[q] = reinterpret_cast<const int*>(rec + P->lay.off_J);
+    va.cntp[q] = reinterpret_cast<const int*>(rec + P->lay.off_cnt);
     va.sig[q] = P->slots_h[P->loc_slots_h[q]].sigma;
     va.aa[q] = P->slots_h[P->loc_slots_h[q]].a;
   }
@@ -1012,6 +1032,8 @@ int cusfft_params_default(cusfft_params* p, int64_t n, int64_t k, int64_t B) {
   p->debug = 0;
   p->taps = nullptr;
   p->num_taps = 0;
+  p->cutoff_mode = CUSFFT_CUTOFF_EXACT;
+  p->cutoff_threshold = 0.0;
   return CUSFFT_SUCCESS;
 }
 
@@ -1141,7 +1163,7 @@ int64_t cusfft_get_debug(cusfft_plan_t plan, int32_t what, void* dst, int64_t ca
   switch (what) {
     case CUSFFT_DEBUG_U: need = (int64_t)plan->Lg * B * 16; break;
     case CUSFFT_DEBUG_UHAT: need = L * B * 16; break;
-    case CUSFFT_DEBUG_WINNERS: need = (int64_t)plan->Lloc * plan->num * 4; break;
+    case CUSFFT_DEBUG_WINNERS: need = (int64_t)plan->Lloc * plan->Jcap * 4; break;
     case CUSFFT_DEBUG_HITS: need = H * 4; break;
     case CUSFFT_DEBUG_HIT_VALS: need = H * 16; break;
     case CUSFFT_DEBUG_PER_LOOP: need = plan->d_per_loop ? H * L * 16 : 0; break;
@@ -1162,10 +1184,15 @@ int64_t cusfft_get_debug(cusfft_plan_t plan, int32_t what, void* dst, int64_t ca
                       cudaMemcpyDeviceToHost));
       break;
     case CUSFFT_DEBUG_WINNERS:
-      for (int r = 0; r < plan->Lloc; ++r)
-        CK(cudaMemcpy(out + (int64_t)r * plan->num * 4,
-                      plan->d_records + (int64_t)slot_of(r) * plan->lay.rec_bytes + plan->lay.off_J,
-                      (int64_t)plan->num * 4, cudaMemcpyDeviceToHost));
+      for (int r = 0; r < plan->Lloc; ++r) {
+        const uint8_t* rec = plan->d_records + (int64_t)slot_of(r) * plan->lay.rec_bytes;
+        int cnt = 0;
+        CK(cudaMemcpy(&cnt, rec + plan->lay.off_cnt, 4, cudaMemcpyDeviceToHost));
+        cnt = std::max(0, std::min(cnt, plan->Jcap));
+        int32_t* o = reinterpret_cast<int32_t*>(out + (int64_t)r * plan->Jcap * 4);
+        CK(cudaMemcpy(o, rec + plan->lay.off_J, (int64_t)cnt * 4, cudaMemcpyDeviceToHost));
+        for (int j = cnt; j < plan->Jcap; ++j) o[j] = -1;
+      }
       break;
     case CUSFFT_DEBUG_HITS:
       CK(cudaMemcpy(out, plan->d_hits, need, cudaMemcpyDeviceToHost));

@@ -232,10 +232,11 @@ __global__ void __launch_bounds__(256, STAGED ? 3 : 2) k_fold_fft1(const double2
 
 // ---------------------------------------------------------------------------
 // Record layout of one slot in the exchange buffer:
-//   [u^ : B x double2][bitmap : B/32 x u32][J : num x int32], 256-B aligned.
+//   [u^ : B x double2][bitmap : B/32 x u32][count : int32][J : Jcap x int32],
+//   256-B aligned; Jcap = num (B in THRESHOLD mode).
 // ---------------------------------------------------------------------------
 struct RecLayout {
-  int64_t rec_bytes, off_bitmap, off_J;
+  int64_t rec_bytes, off_bitmap, off_cnt, off_J;
 };
 
 
@@ -386,6 +387,8 @@ struct SelArgs {
   uint8_t* recs[32];  // record of each location slot of this rank (by value)
   RecLayout lay;
   int B, num, S;
+  int threshold_mode;  // Alg. 6: keep every key >= thr_key, no selection
+  uint64_t thr_key;    // bits of the |u^|^2 threshold
   const uint64_t* keys;  // [n_sel][B]
   uint32_t* hist0;       // [n_sel][4096] (FFT epilogue)
   uint32_t* hist1;       // [n_sel][4096]
@@ -420,11 +423,12 @@ __global__ void __launch_bounds__(kSelNT) k_select(SelArgs A) {
   uint32_t* h1 = A.hist1 + (int64_t)sel * 4096;
   const int words = (A.B + 31) >> 5;
   if (blockIdx.x == 0) TRACE(10);
-  const BinPick b0 = pick_bin<kSelNT>(h0, A.num, sm);
+  BinPick b0{0, 0, 0};
+  if (!A.threshold_mode) b0 = pick_bin<kSelNT>(h0, A.num, sm);
   if (blockIdx.x == 0) TRACE(11);
   const uint32_t d0 = (uint32_t)b0.d;
   const int k2 = A.num - b0.above;
-  const bool whole = (k2 == b0.cnt);
+  const bool whole = A.threshold_mode || (k2 == b0.cnt);
   // this CTA's words
   const int wpc = (words + A.S - 1) / A.S;
   const int w_begin = part * wpc, w_end = min(words, w_begin + wpc);
@@ -440,8 +444,8 @@ __global__ void __launch_bounds__(kSelNT) k_select(SelArgs A) {
       const int w = w0 + u * (kSelNT / 32), i = w * 32 + lane;
       if (w >= w_end) break;
       const uint32_t d = (uint32_t)(kb[u] >> 51) & 0xFFFu;
-      const bool take = i < A.B && (d > d0 || (d == d0 && whole));
-      const bool cand = i < A.B && d == d0 && !whole;
+      const bool take = i < A.B && (A.threshold_mode ? kb[u] >= A.thr_key : (d > d0 || (d == d0 && whole)));
+      const bool cand = i < A.B && !A.threshold_mode && d == d0 && !whole;
       const uint32_t word = __ballot_sync(kFull, take);
       if (lane == 0) bitmap[w] = word;
       if (cand) {
@@ -550,13 +554,86 @@ __global__ void __launch_bounds__(kSelNT) k_select(SelArgs A) {
     while (bits) {
       const int b = __ffs(bits) - 1;
       bits &= bits - 1;
-      if (pos < A.num) J[pos] = w * 32 + b;
+      J[pos] = w * 32 + b;  // pos < total <= Jcap
       ++pos;
     }
   }
-  if (tid == 0 && total != A.num) atomicOr(A.status + 1, 1);
+  if (tid == 0) {
+    *reinterpret_cast<int*>(rec + A.lay.off_cnt) = total;
+    if (!A.threshold_mode && total != A.num) atomicOr(A.status + 1, 1);
+  }
   if (sel == 0) TRACE(22);
   TRACE_END(15);
+}
+
+// ---------------------------------------------------------------------------
+// Step 4, Alg. 3 (L238-L250) as an ablation: one CTA of 1024 threads per
+// location slot sorts all B (|u^|^2, bucket) pairs in shared memory (bitonic,
+// larger key first, ties to the smaller bucket) and keeps the first num.
+// Same winners as k_select; B <= 16384.  Dynamic smem: B x (u64 + int) + B/8.
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(1024) k_select_sort(SelArgs A) {
+  pdl_wait();
+  extern __shared__ __align__(16) uint8_t smem[];
+  const int B = A.B, tid = threadIdx.x;
+  uint64_t* sk = reinterpret_cast<uint64_t*>(smem);
+  int* si = reinterpret_cast<int*>(sk + B);
+  uint32_t* sbits = reinterpret_cast<uint32_t*>(si + B);
+  __shared__ int sm[40];
+  const int sel = blockIdx.x;
+  uint8_t* rec = A.recs[sel];
+  const uint64_t* keys = A.keys + (int64_t)sel * B;
+  const int words = (B + 31) >> 5;
+  for (int i = tid; i < B; i += 1024) {
+    sk[i] = __ldg(keys + i);
+    si[i] = i;
+  }
+  for (int w = tid; w < words; w += 1024) sbits[w] = 0;
+  __syncthreads();
+  // "a before b" iff key_a > key_b or (key_a == key_b and idx_a < idx_b)
+  for (int size = 2; size <= B; size <<= 1) {
+    for (int stride = size >> 1; stride > 0; stride >>= 1) {
+      for (int t = tid; t < (B >> 1); t += 1024) {
+        const int i = 2 * t - (t & (stride - 1));
+        const int jn = i + stride;
+        const bool up = (i & size) == 0;
+        const uint64_t ka = sk[i], kb = sk[jn];
+        const int ia = si[i], ib = si[jn];
+        const bool b_first = (kb > ka) || (kb == ka && ib < ia);
+        if (b_first == up) {
+          sk[i] = kb;
+          sk[jn] = ka;
+          si[i] = ib;
+          si[jn] = ia;
+        }
+      }
+      __syncthreads();
+    }
+  }
+  for (int r = tid; r < A.num; r += 1024) atomicOr(&sbits[si[r] >> 5], 1u << (si[r] & 31));
+  __syncthreads();
+  uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap);
+  int* J = reinterpret_cast<int*>(rec + A.lay.off_J);
+  const int wpt = (words + 1023) >> 10;
+  int cnt = 0;
+  for (int w = tid * wpt; w < min(words, (tid + 1) * wpt); ++w) {
+    bitmap[w] = sbits[w];
+    cnt += __popc(sbits[w]);
+  }
+  int total;
+  int pos = block_excl_scan<1024>(cnt, &total, sm);
+  for (int w = tid * wpt; w < min(words, (tid + 1) * wpt); ++w) {
+    uint32_t bits = sbits[w];
+    while (bits) {
+      const int b = __ffs(bits) - 1;
+      bits &= bits - 1;
+      J[pos++] = w * 32 + b;
+    }
+  }
+  if (tid == 0) {
+    *reinterpret_cast<int*>(rec + A.lay.off_cnt) = total;
+    if (total != A.num) atomicOr(A.status + 1, 1);
+  }
 }
 
 // ---------------------------------------------------------------------------
@@ -577,6 +654,7 @@ struct VoteArgs {
   // per location loop, in vote order, by value (no dependent loads):
   const uint32_t* bmp[kMaxLoc];  // cutoff bitmap in the exchange buffer
   const int* Jp[kMaxLoc];        // ascending winner list
+  const int* cntp[kMaxLoc];      // its length (num, or the Alg. 6 count)
   uint32_t sig[kMaxLoc];         // sigma
   uint32_t aa[kMaxLoc];          // a = sigma^-1
   const uint32_t* loc_sigma;     // the same sigmas in global memory (register-resident loads)
@@ -746,17 +824,27 @@ __global__ void __launch_bounds__(256) k_vote(VoteArgs A) {
     for (int q = 0; q < A.Lloc; ++q)
       for (int i = threadIdx.x; i < words; i += blockDim.x) bm[q * words + i] = A.bmp[q][i];
   }
+  __shared__ int scnt[kMaxLoc + 1];  // prefix sums of the enumerated loops' counts
   if (threadIdx.x < A.Lloc) ssig[threadIdx.x] = A.sig[threadIdx.x];
+  if (threadIdx.x == 0) {
+    int acc = 0;
+    scnt[0] = 0;
+    for (int q = 0; q <= A.Lloc - A.T; ++q) {
+      acc += __ldg(A.cntp[q]);
+      scnt[q + 1] = acc;
+    }
+  }
   __syncthreads();
   if (blockIdx.x == 0) TRACE(31);
-  const int units = (A.Lloc - A.T + 1) * A.num;
+  const int units = scnt[A.Lloc - A.T + 1];
   uint32_t* qF = queueF[threadIdx.x >> 5];
   uint8_t* qG = queueG[threadIdx.x >> 5];
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const int nwarps = (gridDim.x * blockDim.x) >> 5;
   for (int unit = warp; unit < units; unit += nwarps) {
-    const int q0 = unit / A.num;
-    const int jidx = unit - q0 * A.num;
+    int q0 = 0;
+    while (unit >= scnt[q0 + 1]) ++q0;
+    const int jidx = unit - scnt[q0];
     const uint32_t Jv = (uint32_t)__ldg(A.Jp[q0] + jidx);
     const uint32_t a = A.aa[q0];
     const int m = min(A.Lloc - A.T - q0 + 1, A.Lloc - 1 - q0);  // mandatory probes

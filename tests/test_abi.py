@@ -40,7 +40,7 @@ def test_library_is_sm100a():
 
 
 def test_params_struct_layout():
-    assert ctypes.sizeof(b.CusfftParams) == 88
+    assert ctypes.sizeof(b.CusfftParams) == 104
 
 
 def test_abi_version_and_strerror():
@@ -91,7 +91,8 @@ def test_null_pointers_and_invalid_plan():
     (dict(loc_loops=20), b.INVALID_LOOPS), (dict(vote_threshold=9), b.INVALID_LOOPS),
     (dict(num_select=4), b.INVALID_K), (dict(num_select=65), b.INVALID_K),
     (dict(tolerance=0.0), b.INVALID_PARAM), (dict(box_width=256), b.INVALID_PARAM),
-    (dict(tau_mode=2), b.INVALID_PARAM),
+    (dict(tau_mode=2), b.INVALID_PARAM), (dict(cutoff_mode=3), b.INVALID_PARAM),
+    (dict(cutoff_mode=2, cutoff_threshold=0.0), b.INVALID_PARAM),
 ])
 def test_plan_validation_before_device(kw, code):
     """Parameter validation happens before any CUDA call, so it is testable here."""

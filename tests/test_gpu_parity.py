@@ -25,7 +25,7 @@ REL = 1e-9
 
 def _oracle_params(n, k, B, L, **kw):
     okw = {key: kw[key] for key in ("loc_loops", "vote_threshold", "num_select", "filter", "tolerance",
-                                    "tau_mode", "seed") if key in kw}
+                                    "tau_mode", "seed", "cutoff_mode", "cutoff_threshold") if key in kw}
     return O.make_params(n, k, B=B, L=L, **okw)
 
 
@@ -65,9 +65,16 @@ def check_all(plan, ref, locs, vals, fold_bit_exact):
     assert (np.abs(uh - ref.uhat) / scale).max() <= 1e-12
     win = plan.debug(DEBUG_WINNERS)
     ties = 0
+    thr = plan.params.cutoff_threshold if plan.params.cutoff_mode == 2 else None
     for r in range(plan.loc_loops):
-        if not np.array_equal(win[r], ref.J[r]):
-            assert _near_tie(ref.uhat[r], plan.num), f"winners differ in loop {r}"
+        got = win[r][win[r] >= 0]
+        if not np.array_equal(got, ref.J[r]):
+            if thr is None:
+                assert _near_tie(ref.uhat[r], plan.num), f"winners differ in loop {r}"
+            else:  # Alg. 6: only buckets within rounding of the threshold may differ
+                diff = np.setxor1d(got, ref.J[r])
+                m2 = np.abs(ref.uhat[r][diff]) ** 2
+                assert np.all(np.abs(m2 - thr) <= 1e-12 * thr), f"winners differ in loop {r}"
             ties += 1
     if ties:
         pytest.skip(f"{ties} near-tied cutoff(s); downstream comparison not meaningful")
@@ -121,6 +128,16 @@ def test_parity_own_filter(n, k, B, L, extra):
     x, S, X = planted_signal(n, k, seed=3 + k)
     plan, ref, locs, vals = run_pair(x, n, k, B, L, shared_taps=False, seed=5, **extra)
     check_all(plan, ref, locs, vals, fold_bit_exact=False)
+
+
+@pytest.mark.parametrize("mode,extra", [(1, {}), (2, dict(cutoff_threshold=1e-3)), (2, dict(cutoff_threshold=0.05))])
+@pytest.mark.parametrize("n,k,B", [(2 ** 14, 8, None), (2 ** 16, 32, None), (2 ** 20, 100, None), (2 ** 18, 100, 4096)])
+def test_parity_cutoff_modes(mode, extra, n, k, B):
+    """Alg. 3 sort & select and Alg. 6 threshold cutoffs vs the oracle's."""
+    x, S, X = planted_signal(n, k, seed=17 + k)
+    plan, ref, locs, vals = run_pair(x, n, k, B, 16, shared_taps=True, seed=13, cutoff_mode=mode, **extra)
+    check_all(plan, ref, locs, vals, fold_bit_exact=True)
+    assert set(locs.tolist()) == set(S.tolist())
 
 
 @pytest.mark.parametrize("filt", [0, 1])
