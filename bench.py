@@ -360,6 +360,43 @@ def run_gpu(args):
                "d2h_bytes_per_step": k * (8 + 16),
                "note": "cusfft_execute_host: pinned H2D of x, transform, D2H of locs/vals, host wall clock"}
 
+    ablations = None
+    if world == 1 and args.ablations:
+        ablations = {}
+        variants = [("cutoff_sort_alg3", dict(cutoff_mode=1), {}),
+                    ("cutoff_threshold_alg6", dict(cutoff_mode=2, cutoff_threshold=1e-3), {}),
+                    ("direct_gather_no_stage", {}, {"CUSFFT_NO_STAGE": "1"})]
+        for name, kw, env in variants:
+            old = {e: os.environ.get(e) for e in env}
+            os.environ.update(env)
+            try:
+                p2 = Plan(n, k, B=B, L=L, seed=args.plan_seed, device=local_rank, tolerance=TOLERANCE[args.config], **kw)
+            finally:
+                for e, v in old.items():
+                    if v is None:
+                        os.environ.pop(e, None)
+                    else:
+                        os.environ[e] = v
+            l2_, v2_ = torch.empty_like(locs), torch.empty_like(vals)
+
+            def step2():
+                p2.execute(x, l2_, v2_)
+            for _ in range(3):
+                step2()
+            ts = []
+            for _ in range(max(10, args.steps)):
+                flush.zero_()
+                a = torch.cuda.Event(enable_timing=True)
+                b = torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                step2()
+                b.record(stream)
+                torch.cuda.synchronize()
+                ts.append(a.elapsed_time(b))
+            ok = set(l2_.cpu().tolist()) == set(S.tolist())
+            ablations[name] = {"ms": sum(ts) / len(ts), "exact_recovery": ok, "status": p2.status()}
+            p2.close()
+
     cpu = None
     if rank == 0 and not args.no_cpu_baseline:
         times, _ = oracle_time(n, k, L, B, x_np, args.plan_seed, budget_s=args.cpu_budget_s, min_runs=1,
@@ -400,6 +437,7 @@ def run_gpu(args):
                      "useful_gbs": useful / (fold_ms * 1e-3) / 1e9, "kernel_ms": fold_ms,
                      "peak_source": peak_src},
         "stage_ms": stage_ms,
+        "ablations": ablations,
         "dense_cufft_ms": dense_ms, "speedup_vs_dense_cufft": dense_ms / ms,
         "accuracy": {"exact_recovery": exact, "l1_per_coefficient": l1, "status": status},
         "clocks": clocks.summary(),
@@ -426,6 +464,8 @@ def main():
     ap.add_argument("--plan-seed", type=int, default=3)
     ap.add_argument("--cpu-budget-s", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--ablations", action="store_true",
+                    help="also time the cutoff variants (Alg. 3 sort, Alg. 6 threshold) and the direct gather")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

@@ -166,6 +166,7 @@ struct cusfft_plan_s {
   // CUDA graphs of the launch sequences, keyed by the caller's pointers
   bool use_graph = true;
   bool branched = false;          // two-branch graph (location chain || estimation folds); opt-in
+  bool skip_stage = false;        // measurement only (CUSFFT_SKIP_STAGE)
   int nloc_local = 0;             // local slots [0, nloc_local) are location loops
   cudaStream_t cap_stream = nullptr, cap_stream2 = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
@@ -440,6 +441,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   P->stream = nullptr;
   if (const char* e = std::getenv("CUSFFT_NO_GRAPH")) P->use_graph = !(e[0] == '1');
   if (const char* e = std::getenv("CUSFFT_BRANCH")) P->branched = (e[0] == '1');
+  // measurement only: skip the staged gather's phase 1 (valid only for a repeated x)
+  if (const char* e = std::getenv("CUSFFT_SKIP_STAGE")) P->skip_stage = (e[0] == '1');
 
   // ---- draws (loop order), Alg. 1, Def. 1
   SplitMix64 rng{q.seed};
@@ -683,7 +686,7 @@ cudaError_t launch_fold_fft1_t(cusfft_plan_t P, const double2* x, const uint32_t
                                double2* v, int nslots, ZeroArgs z, cudaStream_t st) {
   dim3 grid((unsigned)(P->B / 256), (unsigned)nslots);
   if (inv)  // staged: x is the staging buffer of the group, inv its index
-    return launch_k(k_fold_fft1<B1T, 4, true>, grid, dim3(256), 0, st, P->cur_prio, x, inv,
+    return launch_k(k_fold_fft1<B1T, 16, true>, grid, dim3(256), 0, st, P->cur_prio, x, inv,
                     (const double*)P->d_taps_perm, sp, u, v, (const double2*)P->d_tw,
                     (int)P->B, P->B2, P->w, P->R, (uint32_t)(P->n - 1), z);
   return launch_k(k_fold_fft1<B1T, 8, false>, grid, dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)nullptr,
@@ -720,9 +723,12 @@ int launch_fold(cusfft_plan_t P, const double2* x, int s0, int s1, cudaStream_t 
       const int tot = (int)g.total;
       g_apw = P->stage_window;  // keep the staging buffer L2-resident for phase 2
       const int grid = std::max(1, std::min((tot + 8 * 256 - 1) / (8 * 256), sms * 8));
-      cudaError_t e = launch_k(k_stage, dim3(grid), dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)g.spos,
-                               P->d_staging, tot, z);
-      z = ZeroArgs{nullptr, 0};
+      cudaError_t e = cudaSuccess;
+      if (!P->skip_stage) {
+        e = launch_k(k_stage, dim3(grid), dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)g.spos, P->d_staging, tot,
+                     z);
+        z = ZeroArgs{nullptr, 0};
+      }
       g_pdl = !P->timing;
       if (e == cudaSuccess)
         e = launch_fold_fft1(P, P->d_staging, g.inv, P->d_slots + (size_t)P->rank * P->Lg + g.s0,

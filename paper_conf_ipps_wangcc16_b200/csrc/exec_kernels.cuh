@@ -143,7 +143,7 @@ __global__ void __launch_bounds__(256) k_stage(const double2* __restrict__ x, co
 // per SM so one CTA's FFT epilogue overlaps the other's gathers.
 // ---------------------------------------------------------------------------
 template <int B1T, int RC, bool STAGED>
-__global__ void __launch_bounds__(256, STAGED ? 3 : 2) k_fold_fft1(const double2* __restrict__ x,
+__global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict__ x,
                                                                    const uint32_t* __restrict__ inv_perm,
                                                                    const double* __restrict__ taps_perm,
                                                                    const SlotParam* __restrict__ slots,
@@ -162,7 +162,6 @@ __global__ void __launch_bounds__(256, STAGED ? 3 : 2) k_fold_fft1(const double2
   const int j = c + B2 * j1;
   zero_part(zero);
   for (int i = t; i < B1T; i += 256) twl[i] = __ldg(tw + (int64_t)i * B2);  // omega_B1^i
-  const double2 wout = __ldg(tw + (((int64_t)c * j1) & (B - 1)));          // omega_B^(c k1), k1 = j1
   const double* tp = taps_perm + (int64_t)blockIdx.x * 256 + t;
   double ar = 0.0, ai = 0.0;
   if constexpr (STAGED) {
@@ -222,11 +221,18 @@ __global__ void __launch_bounds__(256, STAGED ? 3 : 2) k_fold_fft1(const double2
       }
     }
   }
-  u[(size_t)s * B + j] = make_double2(ar, ai);
   S[fft_pad(cl * B1T + j1)] = make_double2(ar, ai);
   __syncthreads();
+  // u and v hold the CTA's C columns at stride B2: write column-adjacent
+  // elements from neighbouring threads (full 32-B sectors when C >= 2)
+  const int wc = t % C, wj = t / C;  // writer's (column, row)
+  const size_t wpos = (size_t)s * B + (size_t)blockIdx.x * C + wc + (size_t)B2 * wj;
+  u[wpos] = S[fft_pad(wc * B1T + wj)];
+  __syncthreads();
   fft_smem<B1T, 256, 256, true>(S, twl, B1T);
-  v[(size_t)s * B + c + (size_t)B2 * j1] = cmul(S[fft_pad(cl * B1T + j1)], wout);
+  // v = FFT result times omega_B^(c k1); the writer's own twiddle
+  const double2 wv = __ldg(tw + (((int64_t)(blockIdx.x * C + wc) * wj) & (B - 1)));
+  v[wpos] = cmul(S[fft_pad(wc * B1T + wj)], wv);
   TRACE_END(1);
 }
 
@@ -668,19 +674,28 @@ struct VoteArgs {
 // Scaled arithmetic: with F = f << (32 - log2 n), sigma * F + (nb/2 << (32 - log2 n))
 // wraps at 2^32 exactly like (sigma f + nb/2) mod n scaled, so the bucket is
 // the top log2 B bits: one IMAD + one shift, no mask.
-__device__ __forceinline__ uint32_t probe_s(const uint32_t* row, uint32_t sig, uint32_t F, uint32_t half_s, int bsh) {
-  const uint32_t b = (sig * F + half_s) >> bsh;
-  return (row[b >> 5] >> (b & 31)) & 1u;
+__device__ __forceinline__ uint32_t lds_u32(uint32_t saddr) {
+  uint32_t v;
+  asm("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(saddr));
+  return v;
+}
+
+// probe with a 32-bit shared address of loop q's bitmap
+__device__ __forceinline__ uint32_t probe_sa(uint32_t row_s, uint32_t sig, uint32_t F, uint32_t half_s, int bsh) {
+  const uint32_t h = sig * F + half_s;
+  const uint32_t w = lds_u32(row_s + ((h >> (bsh + 5)) << 2));
+  return __funnelshift_r(w, w, h >> bsh) & 1u;
 }
 
 // Survivors of the mandatory probes finish here, one per lane (convergent):
 // the remaining later loops and the "no vote before q0" check.
-__device__ __forceinline__ bool vote_finish(const VoteArgs& A, const uint32_t* bm, const uint32_t* ssig, int words,
+__device__ __forceinline__ bool vote_finish(const VoteArgs& A, uint32_t bm_s, const uint32_t* ssig, int words,
                                             int q0, int m, uint32_t F, int got, uint32_t half_s, int bsh) {
   int votes = got;
-  for (int q = q0 + 1 + m; q < A.Lloc; ++q) votes += probe_s(bm + q * words, ssig[q], F, half_s, bsh);
+  for (int q = q0 + 1 + m; q < A.Lloc; ++q)
+    votes += probe_sa(bm_s + (uint32_t)(q * words) * 4u, ssig[q], F, half_s, bsh);
   bool hit = votes >= A.T - 1;
-  for (int q = 0; q < q0; ++q) hit = hit && !probe_s(bm + q * words, ssig[q], F, half_s, bsh);
+  for (int q = 0; q < q0; ++q) hit = hit && !probe_sa(bm_s + (uint32_t)(q * words) * 4u, ssig[q], F, half_s, bsh);
   return hit;
 }
 
@@ -703,12 +718,6 @@ __device__ __forceinline__ void vote_emit(const VoteArgs& A, bool hit, uint32_t 
 // M = mandatory probes (compile time; M == 0: runtime count mrt).  Survivors
 // of the mandatory probes are queued in shared memory (qF: scaled f, qG:
 // votes so far) and finished 32 at a time (convergent).
-__device__ __forceinline__ uint32_t lds_u32(uint32_t saddr) {
-  uint32_t v;
-  asm("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(saddr));
-  return v;
-}
-
 template <int M>
 __device__ __forceinline__ void vote_unit(const VoteArgs& A, const uint32_t* __restrict__ bm, const uint32_t* ssig,
                                           int words, int q0, uint32_t Jv, uint32_t a, int mrt, uint32_t* qF,
@@ -750,8 +759,9 @@ __device__ __forceinline__ void vote_unit(const VoteArgs& A, const uint32_t* __r
       }
     } else {
       for (int qq = 0; qq < m; ++qq) {
-        g0 += probe_s(bm + (q0 + 1 + qq) * words, ssig[q0 + 1 + qq], F0, half_s, bsh);
-        g1 += probe_s(bm + (q0 + 1 + qq) * words, ssig[q0 + 1 + qq], F1, half_s, bsh);
+        const uint32_t row = bm_s + (uint32_t)((q0 + 1 + qq) * words) * 4u;
+        g0 += probe_sa(row, ssig[q0 + 1 + qq], F0, half_s, bsh);
+        g1 += probe_sa(row, ssig[q0 + 1 + qq], F1, half_s, bsh);
       }
     }
     const bool s0 = (t0 + lane < A.nb) && (m - g0) <= allowed;
@@ -778,7 +788,7 @@ __device__ __forceinline__ void vote_unit(const VoteArgs& A, const uint32_t* __r
         const int gq = qG[qn - 32 + lane];
         __syncwarp();
         qn -= 32;
-        const bool hit = vote_finish(A, bm, ssig, words, q0, m, Fq, gq, half_s, bsh);
+        const bool hit = vote_finish(A, bm_s, ssig, words, q0, m, Fq, gq, half_s, bsh);
         vote_emit(A, hit, Fq >> sh);
       }
     }
@@ -788,7 +798,7 @@ __device__ __forceinline__ void vote_unit(const VoteArgs& A, const uint32_t* __r
     const uint32_t Fq = has ? qF[lane] : 0u;
     const int gq = has ? qG[lane] : 0;
     __syncwarp();
-    const bool hit = has && vote_finish(A, bm, ssig, words, q0, m, Fq, gq, half_s, bsh);
+    const bool hit = has && vote_finish(A, bm_s, ssig, words, q0, m, Fq, gq, half_s, bsh);
     vote_emit(A, hit, Fq >> sh);
   }
 }
@@ -849,13 +859,10 @@ __global__ void __launch_bounds__(256) k_vote(VoteArgs A) {
     const uint32_t a = A.aa[q0];
     const int m = min(A.Lloc - A.T - q0 + 1, A.Lloc - 1 - q0);  // mandatory probes
     switch (m) {
-      case 0: vote_unit<0>(A, bm, ssig, words, q0, Jv, a, 0, qF, qG); break;
       case 1: vote_unit<1>(A, bm, ssig, words, q0, Jv, a, 1, qF, qG); break;
       case 2: vote_unit<2>(A, bm, ssig, words, q0, Jv, a, 2, qF, qG); break;
       case 3: vote_unit<3>(A, bm, ssig, words, q0, Jv, a, 3, qF, qG); break;
       case 4: vote_unit<4>(A, bm, ssig, words, q0, Jv, a, 4, qF, qG); break;
-      case 5: vote_unit<5>(A, bm, ssig, words, q0, Jv, a, 5, qF, qG); break;
-      case 6: vote_unit<6>(A, bm, ssig, words, q0, Jv, a, 6, qF, qG); break;
       default: vote_unit<0>(A, bm, ssig, words, q0, Jv, a, m, qF, qG); break;
     }
   }

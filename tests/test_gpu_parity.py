@@ -259,3 +259,25 @@ def test_stage_timing_and_launch_count():
     t = plan.stage_times()
     assert all(v >= 0 for v in t.values()) and t["fold"] > 0
     assert plan.launches_per_execute() == 6
+
+
+def test_C4_full_size_parity():
+    """BASELINE.json configs[3] size: n = 2^27, k = 1000 (B = 65536, two-pass
+    FFT with B1 = B2 = 256, direct gather: the staging would not fit L2)."""
+    n, k = 2 ** 27, 1000
+    x, S, X = planted_signal(n, k, seed=2)
+    plan, ref, locs, vals = run_pair(x, n, k, None, 16, shared_taps=False, seed=4)
+    assert plan.info()["staged"] == 0
+    check_all(plan, ref, locs, vals, fold_bit_exact=False)
+    assert set(locs.tolist()) == set(S.tolist())
+    assert O.l1_error(locs, vals, S, X, k) <= 1e-6
+
+
+@pytest.mark.parametrize("snr_db", [40.0, 20.0, 10.0])
+def test_parity_snr_sweep(snr_db):
+    """configs[3]'s additive-noise sweep at n = 2^20 (k = 100): outputs match
+    the oracle whatever the noise does to recovery."""
+    n, k = 2 ** 20, 100
+    x, S, X = planted_signal(n, k, seed=11, snr_db=snr_db)
+    plan, ref, locs, vals = run_pair(x, n, k, None, 16, shared_taps=True, seed=6)
+    check_all(plan, ref, locs, vals, fold_bit_exact=True)
