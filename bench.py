@@ -192,7 +192,7 @@ def run_gpu(args):
         dist.init_process_group("nccl", device_id=dev)
 
     from paper_conf_ipps_wangcc16_b200 import Plan, default_B
-    from paper_conf_ipps_wangcc16_b200.dist import CudaEngine, LoopShardedSfft
+    from paper_conf_ipps_wangcc16_b200.dist import CudaEngine, LoopShardedSfft, signal_range
 
     n, k, L, desc = CONFIGS[args.config]
     B = default_B(n, k)
@@ -210,10 +210,14 @@ def run_gpu(args):
             return locs, vals
         launches = plan.launches_per_execute()
     else:
+        shard = 1 if args.shard == "signal" else 0
         eng = CudaEngine(n, k, B=B, L=L, rank=rank, world=world, device=local_rank, seed=args.plan_seed,
-                         tolerance=TOLERANCE[args.config])
+                         tolerance=TOLERANCE[args.config], shard_mode=shard)
         runner = LoopShardedSfft(eng)
         plan = eng.plan
+        if shard:  # this rank holds only its slice of x
+            lo, hi = signal_range(rank, n, world)
+            x = x[lo:hi].clone()
 
         def step():
             return runner.execute(x)
@@ -425,7 +429,7 @@ def run_gpu(args):
                                f"(Dolph-Chebyshev, delta={TOLERANCE[args.config]:g})",
                    "n": n, "k": k, "B": B, "L": L, "taps": plan.w, "tolerance": TOLERANCE[args.config],
                    "loc_loops": plan.loc_loops,
-                   "vote_threshold": plan.T, "parallelism": f"loop-sharded x{world}" if world > 1 else "single GPU",
+                   "vote_threshold": plan.T, "parallelism": f"{args.shard}-sharded x{world}" if world > 1 else "single GPU",
                    "l2": "flushed between timed steps (256 MiB write + 256 MiB read), outside the step events",
                    "signal_seed": args.signal_seed, "plan_seed": args.plan_seed},
         "gpu_launches": launches * args.steps,
@@ -462,6 +466,8 @@ def main():
     ap.add_argument("--config", default="C3", choices=sorted(CONFIGS))
     ap.add_argument("--signal-seed", type=int, default=1)
     ap.add_argument("--plan-seed", type=int, default=3)
+    ap.add_argument("--shard", default="loops", choices=["loops", "signal"],
+                    help="N>1: loop sharding (all-gather) or signal sharding (SURVEY N1, all-reduce)")
     ap.add_argument("--cpu-budget-s", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--ablations", action="store_true",

@@ -91,6 +91,7 @@ typedef struct {
                               Copied at plan time; the caller keeps ownership.                    */
   int64_t num_taps;        /* length of taps when taps != NULL (odd not required)                */
   int32_t cutoff_mode;     /* cusfft_cutoff_t; default EXACT                                      */
+  int32_t shard_mode;      /* cusfft_plan_dist only: 0 = loops (default), 1 = signal range       */
   double cutoff_threshold; /* THRESHOLD mode: absolute |u^|^2 threshold (> 0)                    */
 } cusfft_params;
 
@@ -108,12 +109,18 @@ int64_t cusfft_default_B(int64_t n, int64_t k, double bcst);
 int cusfft_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L,
                 const cusfft_params* p);
 
-/* Loop-sharded plan for rank `rank` of `world` processes (one GPU each).
- * world must divide L.  Loop r is owned by rank r mod world.  Outputs are
- * identical on every rank and identical to a world = 1 plan with the same
- * parameters.  The exchange between cusfft_execute_local and
- * cusfft_execute_finish is an all-gather of the buffer returned by
- * cusfft_exchange_buffer, done by the caller (e.g. torch.distributed / NCCL). */
+/* Multi-GPU plan for rank `rank` of `world` processes (one GPU each).
+ * shard_mode 0 (loops): world must divide L; loop r is owned by rank r mod
+ * world, every rank passes the whole signal; outputs are identical on every
+ * rank and bit-identical to a world = 1 plan.  The exchange between
+ * cusfft_execute_local and cusfft_execute_finish is an ALL-GATHER of the
+ * buffer returned by cusfft_exchange_buffer (rank-major slices).
+ * shard_mode 1 (signal): world must divide n; rank g passes only
+ * its slice x[g n/world, (g+1) n/world) to cusfft_execute_local and folds
+ * the samples it owns for all L loops; the exchange is a SUM ALL-REDUCE (fp64)
+ * of the whole buffer (the B-point FFT is linear, so partial bucket spectra
+ * add); every rank then runs Steps 4-6.  Equal to world = 1 within fp64
+ * rounding (the sum order differs).  See cusfft_exchange_kind. */
 int cusfft_plan_dist(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L,
                      const cusfft_params* p, int32_t rank, int32_t world);
 
@@ -145,8 +152,12 @@ int cusfft_execute_local(cusfft_plan_t plan, const void* d_x);
  * rank's slice.  Outputs as in cusfft_execute. */
 int cusfft_execute_finish(cusfft_plan_t plan, int64_t* d_locs, void* d_vals);
 /* The exchange buffer: *d_buf points at world * (*bytes_per_rank) bytes of
- * device memory, rank r's slice at offset r * (*bytes_per_rank). */
+ * device memory, rank r's slice at offset r * (*bytes_per_rank) (loop
+ * sharding); for signal sharding *bytes_per_rank is the whole buffer. */
 int cusfft_exchange_buffer(cusfft_plan_t plan, void** d_buf, int64_t* bytes_per_rank);
+/* 0: all-gather of the rank slices (loop sharding); 1: element-wise fp64 sum
+ * all-reduce of the whole buffer (signal sharding); negative: error. */
+int32_t cusfft_exchange_kind(cusfft_plan_t plan);
 
 /* Plan facts (host arrays, caller-owned):
  *   info[0..11] = n, k, B, L, w (taps), n/B, num_select, loc_loops, vote_threshold, max_hits,

@@ -31,7 +31,7 @@ DEBUG_PER_LOOP, DEBUG_TAPS, DEBUG_GHAT, DEBUG_NUM_HITS = 5, 6, 7, 8
 EXPORTED = (
     "cusfft_params_default", "cusfft_default_B", "cusfft_plan", "cusfft_plan_dist",
     "cusfft_destroy", "cusfft_set_stream", "cusfft_execute", "cusfft_execute_host",
-    "cusfft_execute_local", "cusfft_execute_finish", "cusfft_exchange_buffer",
+    "cusfft_execute_local", "cusfft_execute_finish", "cusfft_exchange_buffer", "cusfft_exchange_kind",
     "cusfft_get_info", "cusfft_get_debug", "cusfft_status", "cusfft_set_timing",
     "cusfft_get_stage_times", "cusfft_set_stage_limit", "cusfft_launches_per_execute", "cusfft_strerror",
     "cusfft_last_cuda_error", "cusfft_abi_version",
@@ -55,6 +55,7 @@ class CusfftParams(ctypes.Structure):
         ("taps", ctypes.POINTER(ctypes.c_double)),
         ("num_taps", ctypes.c_int64),
         ("cutoff_mode", ctypes.c_int32),
+        ("shard_mode", ctypes.c_int32),
         ("cutoff_threshold", ctypes.c_double),
     ]
 
@@ -87,6 +88,7 @@ def load_library():
         "cusfft_execute_local": (ctypes.c_int, [P, P]),
         "cusfft_execute_finish": (ctypes.c_int, [P, P, P]),
         "cusfft_exchange_buffer": (ctypes.c_int, [P, ctypes.POINTER(P), ctypes.POINTER(i64)]),
+        "cusfft_exchange_kind": (i32, [P]),
         "cusfft_get_info": (ctypes.c_int, [P, P, P, P, P]),
         "cusfft_get_debug": (i64, [P, i32, P, i64]),
         "cusfft_status": (ctypes.c_int, [P]),
@@ -236,6 +238,7 @@ class Plan:
         return locs, vals
 
     def execute_local(self, x):
+        """x: the whole signal (loop sharding) or this rank's slice (signal sharding)."""
         self._use_current_stream()
         check(self._lib.cusfft_execute_local(self._h, ctypes.c_void_p(x.data_ptr())), "cusfft_execute_local")
 
@@ -252,6 +255,13 @@ class Plan:
         check(self._lib.cusfft_exchange_buffer(self._h, ctypes.byref(ptr), ctypes.byref(per)),
               "cusfft_exchange_buffer")
         return int(ptr.value), int(per.value)
+
+    def exchange_kind(self) -> int:
+        """0: all-gather of rank slices (loop sharding); 1: fp64 sum all-reduce (signal sharding)."""
+        k = int(self._lib.cusfft_exchange_kind(self._h))
+        if k < 0:
+            check(k, "cusfft_exchange_kind")
+        return k
 
     def status(self) -> int:
         return int(self._lib.cusfft_status(self._h))

@@ -97,6 +97,12 @@ struct cusfft_plan_s {
   uint32_t magic = kMagic;
   int64_t n = 0, k = 0, B = 0, nb = 0;
   int L = 0, Lg = 0, rank = 0, world = 1;
+  // Loop layout: loop sharding uses (lrank, lworld) = (rank, world); a
+  // signal-sharded plan runs every loop, (lrank, lworld) = (0, 1),
+  // on its slice x[xlo, xlo + xspan) and sums partial spectra in the exchange.
+  bool xshard = false;
+  int lrank = 0, lworld = 1;
+  uint32_t xlo = 0, xspan = 0;
   cusfft_params prm{};
   int log2nb = 0, w = 0, R = 0, num = 0, Lloc = 0, T = 0, max_hits = 0;
   int Jcap = 0;  // winner-list capacity per loop (num, or B in THRESHOLD mode)
@@ -224,7 +230,13 @@ int validate(int64_t n, int64_t k, int64_t B, int32_t L, const cusfft_params& q,
   if (!is_pow2(B) || B < 2 || B >= n) return CUSFFT_INVALID_B;
   if (L < 1 || L > kMaxLoops) return CUSFFT_INVALID_LOOPS;
   if (q.loc_loops > kMaxLoc) return CUSFFT_INVALID_LOOPS;
-  if (world < 1 || rank < 0 || rank >= world || L % world) return CUSFFT_INVALID_LOOPS;
+  if (world < 1 || rank < 0 || rank >= world) return CUSFFT_INVALID_LOOPS;
+  if (q.shard_mode != 0 && q.shard_mode != 1) return CUSFFT_INVALID_PARAM;
+  if (q.shard_mode == 1 && world > 1) {
+    if (n % world) return CUSFFT_INVALID_PARAM;
+  } else if (L % world) {
+    return CUSFFT_INVALID_LOOPS;
+  }
   if (q.loc_loops < 1 || q.loc_loops > L || q.vote_threshold < 1 || q.vote_threshold > q.loc_loops)
     return CUSFFT_INVALID_LOOPS;
   if (k < 1 || k > 8192 || q.num_select < k || q.num_select > B) return CUSFFT_INVALID_K;
@@ -426,7 +438,12 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   P->device = dev;
   P->nb = n / B;
   P->log2nb = ilog2(P->nb);
-  P->Lg = L / world;
+  P->xshard = world > 1 && q.shard_mode == 1;
+  P->lrank = P->xshard ? 0 : rank;
+  P->lworld = P->xshard ? 1 : world;
+  P->xspan = (uint32_t)(P->xshard ? n / world : n);
+  P->xlo = P->xshard ? (uint32_t)rank * P->xspan : 0u;
+  P->Lg = L / P->lworld;
   P->num = q.num_select;
   P->Lloc = q.loc_loops;
   P->T = q.vote_threshold;
@@ -454,21 +471,22 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     P->sigma_r[r] = inverse_mod(a, n);
     P->tau_r[r] = q.tau_mode ? (int64_t)(rng.next() % (uint64_t)n) : 0;
   }
-  // ---- slots: rank g owns loops r = i*world + g at slots g*Lg + i
+  // ---- slots: rank g owns loops r = i*lworld + g at slots g*Lg + i
+  const int lworld = P->lworld, lrank = P->lrank;
   P->slots_h.resize(L);
   for (int s = 0; s < L; ++s) {
-    const int g = s / P->Lg, i = s % P->Lg, r = i * world + g;
+    const int g = s / P->Lg, i = s % P->Lg, r = i * lworld + g;
     P->slots_h[s] = SlotParam{(uint32_t)P->sigma_r[r], (uint32_t)P->tau_r[r], (uint32_t)P->a_r[r], (uint32_t)r};
   }
   for (int i = 0; i < P->Lg; ++i)
-    if (i * world + rank < P->Lloc) P->nloc_local = i + 1;  // location loops are a prefix of the local slots
+    if (i * lworld + lrank < P->Lloc) P->nloc_local = i + 1;  // location loops are a prefix of the local slots
   std::vector<uint32_t> loc_sig, loc_a;
   for (int s = 0; s < L; ++s) {
     if ((int)P->slots_h[s].loop < P->Lloc) {
       P->loc_slots_h.push_back(s);
       loc_sig.push_back(P->slots_h[s].sigma);
       loc_a.push_back(P->slots_h[s].a);
-      if (s / P->Lg == rank) P->sel_slots_h.push_back(s);
+      if (s / P->Lg == lrank) P->sel_slots_h.push_back(s);
     }
   }
 
@@ -542,7 +560,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     if ((rc = dalloc(&P->d_cidx, nsel * kSelCap))) return fail(rc);
 
     std::vector<int> kidx(P->Lg, -1);
-    for (size_t i = 0; i < P->sel_slots_h.size(); ++i) kidx[P->sel_slots_h[i] - rank * P->Lg] = (int)i;
+    for (size_t i = 0; i < P->sel_slots_h.size(); ++i) kidx[P->sel_slots_h[i] - lrank * P->Lg] = (int)i;
     if (cudaMemcpy(P->d_key_index, kidx.data(), P->Lg * sizeof(int), cudaMemcpyHostToDevice) != cudaSuccess ||
         cudaMemset(P->d_zero, 0, (size_t)P->nzero * sizeof(int)) != cudaSuccess) {
       g_last_cuda_error = (int)cudaGetLastError();
@@ -600,9 +618,11 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     std::vector<uint64_t> bits((size_t)((n / 2 + 63) / 64), 0ull);
     const uint32_t nm = (uint32_t)(n - 1);
     for (int sl = 0; sl < P->Lg; ++sl) {
-      const SlotParam& sp = P->slots_h[(size_t)rank * P->Lg + sl];
+      const SlotParam& sp = P->slots_h[(size_t)lrank * P->Lg + sl];
       for (int i = 0; i < P->w; ++i) {
-        const uint32_t sec = ((sp.sigma * (uint32_t)i + sp.tau) & nm) >> 1;
+        const uint32_t pos = (sp.sigma * (uint32_t)i + sp.tau) & nm;
+        if (pos - P->xlo >= P->xspan) continue;
+        const uint32_t sec = pos >> 1;
         bits[sec >> 6] |= 1ull << (sec & 63);
       }
     }
@@ -621,7 +641,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     int64_t maxtot = 0;
     for (auto& r : ranges) maxtot = std::max<int64_t>(maxtot, (int64_t)(r.second - r.first) * P->w);
     // the staging buffer must be (mostly) L2-resident between the two phases
-    P->staged = P->fused1 && maxtot * 16 <= (int64_t)64 << 20 && !(e && e[0] == '1');
+    // (the staging schedule gathers from the whole signal: not for signal-sharded plans)
+    P->staged = P->fused1 && !P->xshard && maxtot * 16 <= (int64_t)64 << 20 && !(e && e[0] == '1');
     if (P->staged) {
       const uint32_t nm = (uint32_t)(n - 1);
       const int C = 256 / P->B1;
@@ -632,7 +653,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
         g.total = (int64_t)(g.s1 - g.s0) * P->w;
         std::vector<uint64_t> ev((size_t)g.total);
         for (int sl = g.s0; sl < g.s1; ++sl) {
-          const SlotParam& sp = P->slots_h[(size_t)rank * P->Lg + sl];
+          const SlotParam& sp = P->slots_h[(size_t)lrank * P->Lg + sl];
           for (int i = 0; i < P->w; ++i) {
             const uint32_t pos = (sp.sigma * (uint32_t)i + sp.tau) & nm;
             const uint64_t id = (uint64_t)(sl - g.s0) * P->w + i;
@@ -688,10 +709,10 @@ cudaError_t launch_fold_fft1_t(cusfft_plan_t P, const double2* x, const uint32_t
   if (inv)  // staged: x is the staging buffer of the group, inv its index
     return launch_k(k_fold_fft1<B1T, 16, true>, grid, dim3(256), 0, st, P->cur_prio, x, inv,
                     (const double*)P->d_taps_perm, sp, u, v, (const double2*)P->d_tw,
-                    (int)P->B, P->B2, P->w, P->R, (uint32_t)(P->n - 1), z);
+                    (int)P->B, P->B2, P->w, P->R, (uint32_t)(P->n - 1), 0u, (uint32_t)P->n, z);
   return launch_k(k_fold_fft1<B1T, 8, false>, grid, dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)nullptr,
                   (const double*)P->d_taps_perm, sp, u, v, (const double2*)P->d_tw, (int)P->B, P->B2, P->w, P->R,
-                  (uint32_t)(P->n - 1), z);
+                  (uint32_t)(P->n - 1), P->xlo, P->xspan, z);
 }
 
 cudaError_t launch_fold_fft1(cusfft_plan_t P, const double2* x, const uint32_t* inv, const SlotParam* sp, double2* u,
@@ -713,7 +734,7 @@ inline void mark(cusfft_plan_t P, int i) {
 int launch_fold(cusfft_plan_t P, const double2* x, int s0, int s1, cudaStream_t st, bool zero_block) {
   if (s1 <= s0) return CUSFFT_SUCCESS;
   const int B = (int)P->B;
-  const SlotParam* sp = P->d_slots + (size_t)P->rank * P->Lg + s0;
+  const SlotParam* sp = P->d_slots + (size_t)P->lrank * P->Lg + s0;
   ZeroArgs z{zero_block ? P->d_zero : nullptr, zero_block ? P->nzero : 0};
   if (P->staged) {  // per slot group: phase 1 (address-sorted gather into staging), phase 2 (fused fold)
     int sms = 148;
@@ -731,7 +752,7 @@ int launch_fold(cusfft_plan_t P, const double2* x, int s0, int s1, cudaStream_t 
       }
       g_pdl = !P->timing;
       if (e == cudaSuccess)
-        e = launch_fold_fft1(P, P->d_staging, g.inv, P->d_slots + (size_t)P->rank * P->Lg + g.s0,
+        e = launch_fold_fft1(P, P->d_staging, g.inv, P->d_slots + (size_t)P->lrank * P->Lg + g.s0,
                              P->d_u + (size_t)g.s0 * B, P->d_v + (size_t)g.s0 * B, g.s1 - g.s0, z, st);
       g_apw = cudaAccessPolicyWindow{};
       CK(e);
@@ -741,7 +762,7 @@ int launch_fold(cusfft_plan_t P, const double2* x, int s0, int s1, cudaStream_t 
   } else {
     dim3 grid((B + 255) / 256, s1 - s0);
     CK(launch_k(k_fold<16>, grid, dim3(256), 0, st, P->cur_prio, x, (const double*)P->d_taps, sp,
-                P->d_u + (size_t)s0 * B, B, P->w, P->R, (uint32_t)(P->n - 1), z));
+                P->d_u + (size_t)s0 * B, B, P->w, P->R, (uint32_t)(P->n - 1), P->xlo, P->xspan, z));
   }
   return CUSFFT_SUCCESS;
 }
@@ -751,9 +772,10 @@ int launch_bfft(cusfft_plan_t P, int s0, int s1, cudaStream_t st) {
   if (s1 <= s0) return CUSFFT_SUCCESS;
   const int B = (int)P->B;
   const int ns = s1 - s0;
-  double2* rec = reinterpret_cast<double2*>(P->d_records + ((int64_t)P->rank * P->Lg + s0) * P->lay.rec_bytes);
+  double2* rec = reinterpret_cast<double2*>(P->d_records + ((int64_t)P->lrank * P->Lg + s0) * P->lay.rec_bytes);
   const int64_t rec_e = P->lay.rec_bytes / 16;
-  const int* kidx = P->sel_slots_h.empty() ? nullptr : P->d_key_index + s0;
+  // signal-sharded: the spectra are partial here, keys come after the all-reduce (launch_keys)
+  const int* kidx = (P->sel_slots_h.empty() || P->xshard) ? nullptr : P->d_key_index + s0;
   if (P->B1 > 1) {
     if (!P->fused1) {  // pass 1: B1-point FFTs over columns c (stride B2), twiddle e^{-2 pi i c k1 / B}
       FftPassArgs a1{P->d_u + (size_t)s0 * B, P->d_v + (size_t)s0 * B, P->d_tw, B, P->logB2, ns * P->B2, B, B, 1,
@@ -807,6 +829,20 @@ int launch_select(cusfft_plan_t P, cudaStream_t st) {
   return CUSFFT_SUCCESS;
 }
 
+// Cutoff keys from the summed spectra (signal-sharded plans, after the exchange).
+int launch_keys(cusfft_plan_t P, cudaStream_t st) {
+  if (P->sel_slots_h.empty()) return CUSFFT_SUCCESS;
+  KeysArgs ka{};
+  for (size_t i = 0; i < P->sel_slots_h.size(); ++i)
+    ka.rec[i] = reinterpret_cast<const double2*>(P->d_records + (int64_t)P->sel_slots_h[i] * P->lay.rec_bytes);
+  ka.keys = P->d_keys;
+  ka.hist = P->d_hist;
+  ka.B = (int)P->B;
+  const int gx = (int)std::max<int64_t>(1, std::min<int64_t>(P->B / 1024, 64));
+  CK(launch_k(k_keys, dim3(gx, (unsigned)P->sel_slots_h.size()), dim3(256), 0, st, P->cur_prio, ka));
+  return CUSFFT_SUCCESS;
+}
+
 int launch_local(cusfft_plan_t P, const double2* x) {
   cudaStream_t st = P->stream;
   int rc;
@@ -819,7 +855,7 @@ int launch_local(cusfft_plan_t P, const double2* x) {
   if (P->stage_limit < 2) return CUSFFT_SUCCESS;
   if ((rc = launch_bfft(P, 0, P->Lg, st))) return rc;
   mark(P, 2);
-  if (P->stage_limit < 3) return CUSFFT_SUCCESS;
+  if (P->stage_limit < 3 || P->xshard) return CUSFFT_SUCCESS;  // signal-sharded: cutoff after the all-reduce
   if ((rc = launch_select(P, st))) return rc;
   mark(P, 3);
   return CUSFFT_SUCCESS;
@@ -886,8 +922,16 @@ int launch_output(cusfft_plan_t P, int64_t* locs, double2* vals, cudaStream_t st
 int launch_finish(cusfft_plan_t P, int64_t* locs, double2* vals) {
   cudaStream_t st = P->stream;
   int rc;
-  if (P->stage_limit < 4) return CUSFFT_SUCCESS;
   g_pdl = !P->timing;  // every kernel waits for its predecessor before touching memory
+  if (P->xshard) {
+    g_pdl = false;  // follows the caller's all-reduce
+    if (P->stage_limit < 3) return CUSFFT_SUCCESS;
+    if ((rc = launch_keys(P, st))) return rc;
+    g_pdl = !P->timing;
+    if ((rc = launch_select(P, st))) return rc;
+    mark(P, 3);
+  }
+  if (P->stage_limit < 4) return CUSFFT_SUCCESS;
   if ((rc = launch_vote(P, st))) return rc;
   mark(P, 4);
   if (P->stage_limit < 5) return CUSFFT_SUCCESS;
@@ -998,7 +1042,7 @@ const char* cusfft_strerror(int code) {
     case CUSFFT_INVALID_N: return "n must be a power of two in [16, 2^31]";
     case CUSFFT_INVALID_B: return "B must be a power of two with 2 <= B < n";
     case CUSFFT_INVALID_K: return "need 1 <= k <= 8192 and k <= num_select <= B";
-    case CUSFFT_INVALID_LOOPS: return "need 1 <= T <= L_loc <= L <= 64 and world | L";
+    case CUSFFT_INVALID_LOOPS: return "need 1 <= T <= L_loc <= L <= 64, L_loc <= 32 and world | L (loop sharding)";
     case CUSFFT_INVALID_PARAM: return "invalid filter or plan parameter";
     case CUSFFT_NULL_PTR: return "null pointer argument";
     case CUSFFT_ALLOC: return "device allocation failed";
@@ -1039,6 +1083,7 @@ int cusfft_params_default(cusfft_params* p, int64_t n, int64_t k, int64_t B) {
   p->taps = nullptr;
   p->num_taps = 0;
   p->cutoff_mode = CUSFFT_CUTOFF_EXACT;
+  p->shard_mode = 0;
   p->cutoff_threshold = 0.0;
   return CUSFFT_SUCCESS;
 }
@@ -1141,6 +1186,11 @@ int cusfft_exchange_buffer(cusfft_plan_t plan, void** d_buf, int64_t* bytes_per_
   return CUSFFT_SUCCESS;
 }
 
+int32_t cusfft_exchange_kind(cusfft_plan_t plan) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  return plan->xshard ? 1 : 0;
+}
+
 int cusfft_get_info(cusfft_plan_t plan, int64_t* info, int64_t* a, int64_t* sigma, int64_t* tau) {
   if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
   if (info) {
@@ -1164,7 +1214,7 @@ int64_t cusfft_get_debug(cusfft_plan_t plan, int32_t what, void* dst, int64_t ca
   CK(cudaMemcpy(&hc, plan->d_flags, sizeof(unsigned), cudaMemcpyDeviceToHost));
   const int64_t H = std::min<int64_t>(hc, plan->max_hits);
   const int64_t B = plan->B, L = plan->L;
-  auto slot_of = [&](int r) { return (r % plan->world) * plan->Lg + r / plan->world; };
+  auto slot_of = [&](int r) { return (r % plan->lworld) * plan->Lg + r / plan->lworld; };
   int64_t need = 0;
   switch (what) {
     case CUSFFT_DEBUG_U: need = (int64_t)plan->Lg * B * 16; break;

@@ -46,10 +46,14 @@ __device__ __forceinline__ double2 ld_gather(const double2* p) {
   return v;
 }
 
+// x holds samples [xlo, xlo + xspan) of the signal (xlo = 0, xspan = n unless
+// the plan is signal-sharded): a gather outside the range
+// contributes nothing, so the ranks' partial buckets sum to the full fold.
 template <int RC>
 __global__ void __launch_bounds__(256) k_fold(const double2* __restrict__ x, const double* __restrict__ taps,
                                               const SlotParam* __restrict__ slots, double2* __restrict__ u,
-                                              int B, int w, int R, uint32_t nmask, ZeroArgs zero) {
+                                              int B, int w, int R, uint32_t nmask, uint32_t xlo, uint32_t xspan,
+                                              ZeroArgs zero) {
   pdl_wait();
   const int j = blockIdx.x * blockDim.x + threadIdx.x;
   const int s = blockIdx.y;
@@ -61,19 +65,20 @@ __global__ void __launch_bounds__(256) k_fold(const double2* __restrict__ x, con
   for (int r0 = 0; r0 < R; r0 += RC) {
     double2 v[RC];
     double g[RC];
+    bool ok[RC];
 #pragma unroll
     for (int c = 0; c < RC; ++c) {
       const int i = j + (r0 + c) * B;
-      if (r0 + c < R && i < w) {
-        const uint32_t idx = (sigma * (uint32_t)i + tau) & nmask;  // mod n, n | 2^32
-        v[c] = ld_gather(x + idx);
+      const uint32_t rel = ((sigma * (uint32_t)i + tau) & nmask) - xlo;  // mod n, n | 2^32
+      ok[c] = r0 + c < R && i < w && rel < xspan;
+      if (ok[c]) {
+        v[c] = ld_gather(x + rel);
         g[c] = __ldg(taps + i);
       }
     }
 #pragma unroll
     for (int c = 0; c < RC; ++c) {
-      const int i = j + (r0 + c) * B;
-      if (r0 + c < R && i < w) {
+      if (ok[c]) {
         ar = __dadd_rn(ar, __dmul_rn(g[c], v[c].x));
         ai = __dadd_rn(ai, __dmul_rn(g[c], v[c].y));
       }
@@ -149,7 +154,8 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict_
                                                                    const SlotParam* __restrict__ slots,
                                                                    double2* __restrict__ u, double2* __restrict__ v,
                                                                    const double2* __restrict__ tw, int B, int B2,
-                                                                   int w, int R, uint32_t nmask, ZeroArgs zero) {
+                                                                   int w, int R, uint32_t nmask, uint32_t xlo,
+                                                                   uint32_t xspan, ZeroArgs zero) {
   pdl_wait();
   constexpr int C = 256 / B1T;
   __shared__ double2 S[256 + 256 / 8];
@@ -202,19 +208,20 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict_
     for (int r0 = 0; r0 < R; r0 += RC) {
       double2 xv[RC];
       double g[RC];
+      bool ok[RC];
 #pragma unroll
       for (int cc = 0; cc < RC; ++cc) {
         const int i = j + (r0 + cc) * B;
-        if (r0 + cc < R && i < w) {
-          const uint32_t idx = (sigma * (uint32_t)i + tau) & nmask;  // mod n, n | 2^32
-          xv[cc] = ld_gather(x + idx);
+        const uint32_t rel = ((sigma * (uint32_t)i + tau) & nmask) - xlo;  // mod n, n | 2^32; k_fold's range rule
+        ok[cc] = r0 + cc < R && i < w && rel < xspan;
+        if (ok[cc]) {
+          xv[cc] = ld_gather(x + rel);
           g[cc] = __ldg(tp + (int64_t)(r0 + cc) * B);
         }
       }
 #pragma unroll
       for (int cc = 0; cc < RC; ++cc) {
-        const int i = j + (r0 + cc) * B;
-        if (r0 + cc < R && i < w) {
+        if (ok[cc]) {
           ar = __dadd_rn(ar, __dmul_rn(g[cc], xv[cc].x));
           ai = __dadd_rn(ai, __dmul_rn(g[cc], xv[cc].y));
         }
@@ -389,8 +396,10 @@ __device__ void select_topk(int N, int K, uint32_t* ghist, KeyAt key_at, OnSel o
 constexpr int kSelCap = 4096;
 constexpr int kSelNT = 256;
 
+constexpr int kMaxSel = 32;  // location loops per plan (kMaxLoc)
+
 struct SelArgs {
-  uint8_t* recs[32];  // record of each location slot of this rank (by value)
+  uint8_t* recs[kMaxSel];  // record of each location slot of this rank (by value)
   RecLayout lay;
   int B, num, S;
   int threshold_mode;  // Alg. 6: keep every key >= thr_key, no selection
@@ -412,6 +421,35 @@ struct GKeySrc {
     lo = ~(uint32_t)i;
   }
 };
+
+// Cutoff keys of the location loops from the summed bucket spectra
+// (signal-sharded plans only, after the all-reduce; otherwise FFT pass 2
+// emits them): key = bits(|u^|^2) and the 4096-bin top-digit histogram,
+// exactly as the FFT epilogue (fft.cuh) computes them.
+struct KeysArgs {
+  const double2* rec[kMaxSel];  // u^ of selection index i (record start)
+  uint64_t* keys;               // [n_sel][B]
+  uint32_t* hist;               // [n_sel][4096]
+  int B;
+};
+
+__global__ void __launch_bounds__(256) k_keys(KeysArgs A) {
+  pdl_wait();
+  __shared__ uint32_t sh[4096];
+  const int i = blockIdx.y;
+  for (int t = threadIdx.x; t < 4096; t += 256) sh[t] = 0;
+  __syncthreads();
+  const double2* u = A.rec[i];
+  for (int p = blockIdx.x * 256 + threadIdx.x; p < A.B; p += gridDim.x * 256) {
+    const double2 v = __ldcg(u + p);
+    const uint64_t key = (uint64_t)__double_as_longlong(__dadd_rn(__dmul_rn(v.x, v.x), __dmul_rn(v.y, v.y)));
+    A.keys[(int64_t)i * A.B + p] = key;
+    atomicAdd(&sh[(uint32_t)(key >> 51) & 0xFFFu], 1u);
+  }
+  __syncthreads();
+  for (int t = threadIdx.x; t < 4096; t += 256)
+    if (sh[t]) atomicAdd(&A.hist[(int64_t)i * 4096 + t], sh[t]);
+}
 
 __global__ void __launch_bounds__(kSelNT) k_select(SelArgs A) {
   pdl_wait();

@@ -1,5 +1,8 @@
-"""Loop-sharded multi-GPU execution (one process per GPU, torch.distributed).
+"""Multi-GPU execution (one process per GPU, torch.distributed).
 
+Two shardings:
+
+* loops (default) --
 The L loops of the sFFT are independent until the vote and all
 share B and the filter (one batched B-point FFT, L232), so rank g of G runs
 Steps 1-4 for the loops r with r mod G == g on a replicated signal.  The only
@@ -7,13 +10,24 @@ exchange is ONE all-gather of the per-loop records (u^_r, the cutoff bitmap
 and winner list of location loops) over NCCL / NVLink; then every rank runs
 the vote, the estimation and the output selection redundantly, so outputs are
 identical on all ranks and identical to the single-GPU plan (the loop draws
-depend only on (seed, r)).  See DESIGN.md §7.
+depend only on (seed, r)).
+
+* signal (``shard_mode=1``) -- rank g holds only the slice
+x[g n/G, (g+1) n/G) and folds the samples it owns for ALL L loops (Step 1-2
+restricted to its range; PAPER.md:L92 -- the fold is a sum over samples, and the
+B-point FFT of Step 3 is linear, so the partial bucket spectra add).  The
+exchange is ONE sum all-reduce (fp64) of the per-loop spectra; every rank then
+runs the cutoff, vote, estimation and output.  x never has to be replicated
+(n up to G x the single-GPU memory); outputs equal the single-GPU plan up to
+fp64 rounding of the sum order.
 
 The engine interface keeps the exchange logic independent of the compute
 engine, so the gloo CPU tests drive this exact code with a test engine:
   engine.local(x)            Steps 1-4 for this rank's loops
-  engine.exchange_tensor()   the all-gather buffer (uint8 [world * per_rank])
-  engine.finish()            Steps 5-6 + output, returns (locs, vals)
+  engine.exchange_tensor()   the exchange buffer (uint8 [world * per_rank] for
+                             the all-gather; float64 [...] for the all-reduce)
+  engine.exchange_kind       0 = all-gather (loops), 1 = sum all-reduce (signal)
+  engine.finish()            Steps 4-6 + output, returns (locs, vals)
 """
 from __future__ import annotations
 
@@ -34,12 +48,20 @@ def slot_of_loop(r: int, L: int, world: int) -> int:
     return (r % world) * (L // world) + r // world
 
 
+def signal_range(rank: int, n: int, world: int):
+    """Samples [lo, hi) of x rank `rank` holds under signal sharding."""
+    if n % world:
+        raise ValueError("world must divide n")
+    span = n // world
+    return rank * span, (rank + 1) * span
+
+
 class _CudaBuffer:
     """__cuda_array_interface__ view of a device allocation owned by the plan."""
 
-    def __init__(self, ptr: int, nbytes: int):
+    def __init__(self, ptr: int, nbytes: int, typestr: str = "|u1", itemsize: int = 1):
         self.__cuda_array_interface__ = {
-            "shape": (nbytes,), "typestr": "|u1", "data": (ptr, False), "version": 3, "strides": None,
+            "shape": (nbytes // itemsize,), "typestr": typestr, "data": (ptr, False), "version": 3, "strides": None,
         }
 
 
@@ -54,11 +76,16 @@ class CudaEngine:
         self.plan = Plan(n, k, B=B, L=L, rank=rank, world=world, device=device, **params)
         ptr, per = self.plan.exchange_buffer()
         self.per_rank = per
-        self._buf = torch.as_tensor(_CudaBuffer(ptr, per * world), device=self.device)
+        self.exchange_kind = self.plan.exchange_kind()
+        if self.exchange_kind == 1:  # the whole buffer, summed as float64
+            self._buf = torch.as_tensor(_CudaBuffer(ptr, per, "<f8", 8), device=self.device)
+        else:
+            self._buf = torch.as_tensor(_CudaBuffer(ptr, per * world), device=self.device)
         self.locs = torch.empty(k, dtype=torch.int64, device=self.device)
         self.vals = torch.empty(k, dtype=torch.complex128, device=self.device)
 
     def local(self, x):
+        """x: the whole signal (loop sharding) or this rank's slice (signal sharding)."""
         self.plan.execute_local(x)
 
     def exchange_tensor(self):
@@ -73,7 +100,10 @@ class CudaEngine:
 
 
 class LoopShardedSfft:
-    """execute(x) = local Steps 1-4, one all-gather, then Steps 5-6 everywhere."""
+    """execute(x) = local steps, ONE collective (the engine's exchange kind:
+    all-gather for loop sharding, sum all-reduce for signal sharding), then
+    the remaining steps on every rank.  x is the whole signal or this rank's
+    slice, as the engine expects."""
 
     def __init__(self, engine, group=None):
         self.engine = engine
@@ -85,6 +115,9 @@ class LoopShardedSfft:
         self.engine.local(x)
         if self.world > 1:
             buf = self.engine.exchange_tensor()
+            if getattr(self.engine, "exchange_kind", 0) == 1:
+                dist.all_reduce(buf, op=dist.ReduceOp.SUM, group=self.group)
+                return self.engine.finish()
             per = buf.numel() // self.world
             mine = buf[self.rank * per:(self.rank + 1) * per]
             # in place: input is this rank's slice of the output (NCCL in-place all-gather)
@@ -92,4 +125,4 @@ class LoopShardedSfft:
         return self.engine.finish()
 
 
-__all__ = ["loops_of_rank", "slot_of_loop", "CudaEngine", "LoopShardedSfft"]
+__all__ = ["loops_of_rank", "slot_of_loop", "signal_range", "CudaEngine", "LoopShardedSfft"]

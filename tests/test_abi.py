@@ -105,6 +105,33 @@ def test_plan_validation_before_device(kw, code):
     assert not h.value
 
 
+@pytest.mark.parametrize("world,L,shard,code", [
+    (3, 16, 0, b.INVALID_LOOPS),   # loop sharding: world must divide L
+    (2, 16, 2, b.INVALID_PARAM),   # unknown shard mode
+    (3, 16, 1, b.INVALID_PARAM),   # signal sharding: world must divide n
+])
+def test_dist_plan_validation(world, L, shard, code):
+    lib = pkg.load_library()
+    p = pkg.default_params(2 ** 14, 8, 64)
+    p.shard_mode = shard
+    h = ctypes.c_void_p()
+    assert lib.cusfft_plan_dist(ctypes.byref(h), 2 ** 14, 8, 64, L, ctypes.byref(p), 0, world) == code
+    assert not h.value
+
+
+def test_signal_sharding_accepts_any_L():
+    """Signal sharding does not need world | L: validation passes and only the
+    device probe fails here (no GPU), i.e. CUSFFT_CUDA, not a parameter code."""
+    torch = pytest.importorskip("torch")
+    if torch.cuda.is_available():
+        pytest.skip("a GPU is present")
+    lib = pkg.load_library()
+    p = pkg.default_params(2 ** 14, 8, 64)
+    p.shard_mode = 1
+    h = ctypes.c_void_p()
+    assert lib.cusfft_plan_dist(ctypes.byref(h), 2 ** 14, 8, 64, 15, ctypes.byref(p), 1, 4) == b.CUDA
+
+
 def test_no_cpu_fallback_without_device():
     """Without a CUDA device plan creation fails loudly (CUSFFT_CUDA)."""
     torch = pytest.importorskip("torch")

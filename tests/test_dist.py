@@ -1,4 +1,5 @@
-"""Loop-sharded multi-GPU execution (paper_conf_ipps_wangcc16_b200.dist).
+"""Multi-GPU execution (paper_conf_ipps_wangcc16_b200.dist): loop sharding
+(all-gather) and signal sharding (sum all-reduce).
 
 CPU (gloo, world_size 2): the exchange logic of LoopShardedSfft — loop
 ownership, rank-major slot layout, one all-gather, rank-identical outputs —
@@ -17,7 +18,7 @@ import torch.distributed as dist
 import torch.multiprocessing as mp
 
 import oracle as O
-from paper_conf_ipps_wangcc16_b200.dist import LoopShardedSfft, loops_of_rank, slot_of_loop
+from paper_conf_ipps_wangcc16_b200.dist import LoopShardedSfft, loops_of_rank, signal_range, slot_of_loop
 from paper_conf_ipps_wangcc16_b200.workload import planted_signal
 
 
@@ -73,6 +74,70 @@ class OracleEngine:
         return O.select_output(hits, vals, p.k)
 
 
+class OracleSignalEngine:
+    """Signal-sharded test engine: this rank holds x[lo, hi) and folds only
+    those samples for every loop (the oracle's Step 1-2 on the slice
+    zero-extended to n), Step 3 on the partial buckets; the exchange buffer
+    is the L x B partial spectra as float64, summed by the all-reduce."""
+
+    exchange_kind = 1
+
+    def __init__(self, p: O.SfftParams, rank: int, world: int):
+        self.p, self.rank, self.world = p, rank, world
+        self.a, self.sigma, self.tau = O.draw_permutations(p.seed, p.n, p.L, p.tau_mode)
+        self.g = O.filter_taps(p)
+        self.lo, self.hi = signal_range(rank, p.n, world)
+        self.buf = torch.zeros(p.L * p.B * 2, dtype=torch.float64)
+
+    def local(self, xs):
+        assert len(xs) == self.hi - self.lo
+        xz = np.zeros(self.p.n, np.complex128)
+        xz[self.lo:self.hi] = xs
+        for r in range(self.p.L):
+            uh = O.bucket_fft(O.perm_filter(xz, self.g, int(self.sigma[r]), int(self.tau[r]), self.p.B))
+            self.buf[r * 2 * self.p.B:(r + 1) * 2 * self.p.B] = torch.from_numpy(uh.view(np.float64))
+
+    def exchange_tensor(self):
+        return self.buf
+
+    def finish(self):
+        p = self.p
+        uhat = self.buf.numpy().view(np.complex128).reshape(p.L, p.B)
+        J = [O.cutoff(uhat[r], p.num_select) for r in range(p.loc_loops)]
+        hits = np.sort(O.location_recovery(J, self.a[:p.loc_loops], p.n, p.B, p.vote_threshold))
+        G = O.filter_response(self.g, p.n, p.n // p.B)
+        vals, _ = O.estimate(hits, uhat, self.sigma, self.tau, G, p.n, p.B)
+        return O.select_output(hits, vals, p.k)
+
+
+def test_signal_range_partitions_x():
+    for n, world in [(2 ** 12, 1), (2 ** 12, 2), (2 ** 12, 8)]:
+        rs = [signal_range(g, n, world) for g in range(world)]
+        assert rs[0][0] == 0 and rs[-1][1] == n
+        assert all(rs[i][1] == rs[i + 1][0] for i in range(world - 1))
+    with pytest.raises(ValueError):
+        signal_range(0, 2 ** 12, 3)
+
+
+def test_partial_folds_sum_to_full_fold():
+    """The property signal sharding rests on: Steps 1-3 are linear in x, so
+    the spectra of the range-restricted folds sum to the full one."""
+    n, k = 2 ** 12, 6
+    x, S, X = planted_signal(n, k, seed=6)
+    p = O.make_params(n, k, L=3, seed=1)
+    a, sigma, tau = O.draw_permutations(p.seed, n, p.L, p.tau_mode)
+    g = O.filter_taps(p)
+    for r in range(p.L):
+        full = O.bucket_fft(O.perm_filter(x, g, int(sigma[r]), int(tau[r]), p.B))
+        part = np.zeros_like(full)
+        for rank in range(4):
+            lo, hi = signal_range(rank, n, 4)
+            xz = np.zeros_like(x)
+            xz[lo:hi] = x[lo:hi]
+            part += O.bucket_fft(O.perm_filter(xz, g, int(sigma[r]), int(tau[r]), p.B))
+        np.testing.assert_allclose(part, full, rtol=0, atol=1e-12 * np.abs(full).max())
+
+
 def _free_port():
     with socket.socket() as s:
         s.bind(("127.0.0.1", 0))
@@ -91,6 +156,43 @@ def _worker(rank, world, port, q):
         q.put((rank, locs.tolist(), vals.tolist()))
     finally:
         dist.destroy_process_group()
+
+
+def _signal_worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        n, k = 2 ** 12, 6
+        x, S, X = planted_signal(n, k, seed=4)
+        p = O.make_params(n, k, L=7, loc_loops=5, vote_threshold=3, seed=9)  # world need not divide L
+        lo, hi = signal_range(rank, n, world)
+        locs, vals = LoopShardedSfft(OracleSignalEngine(p, rank, world)).execute(x[lo:hi])
+        q.put((rank, locs.tolist(), vals.tolist()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_signal_sharded_allreduce_gloo(world):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_signal_worker, args=(r, world, port, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    out = [q.get(timeout=300) for _ in range(world)]
+    for pr in procs:
+        pr.join(timeout=60)
+        assert pr.exitcode == 0
+    n, k = 2 ** 12, 6
+    x, S, X = planted_signal(n, k, seed=4)
+    ref = O.sfft(x, O.make_params(n, k, L=7, loc_loops=5, vote_threshold=3, seed=9))
+    assert sorted(ref.locs.tolist()) == sorted(S.tolist())
+    for rank, locs, vals in out:
+        assert locs == ref.locs.tolist(), rank
+        # the all-reduce sums partial spectra in another order: fp64 rounding only
+        np.testing.assert_allclose(np.array(vals), ref.vals, rtol=1e-9, atol=1e-12)
+        assert vals == out[0][2]  # every rank finishes from the same summed buffer
 
 
 @pytest.mark.parametrize("world", [2, 4])
@@ -150,3 +252,46 @@ def test_dist_plans_emulated_allgather_match_single_gpu(world):
         assert e.plan.status() == 0
         assert torch.equal(locs, ref_l)
         assert torch.equal(vals, ref_v)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("world,n,k,L", [(2, 2 ** 20, 100, 16), (4, 2 ** 20, 100, 16), (8, 2 ** 18, 50, 12)])
+def test_signal_sharded_plans_emulated_allreduce(world, n, k, L):
+    """Signal-sharded cusfft_plan_dist ranks on one GPU, each given only its
+    slice of x; the all-reduce is emulated by summing the ranks' exchange
+    buffers (fp64).  Equal to the single-GPU plan: locations and winners
+    exactly, values within fp64 rounding of the reordered sum."""
+    from paper_conf_ipps_wangcc16_b200 import Plan
+    from paper_conf_ipps_wangcc16_b200.dist import CudaEngine
+    x, S, X = planted_signal(n, k, seed=11)
+    xd = torch.from_numpy(x).cuda()
+    ref = Plan(n, k, L=L, seed=3)
+    ref_l, ref_v = ref.execute(xd)
+    engines = [CudaEngine(n, k, L=L, rank=r, world=world, seed=3, shard_mode=1) for r in range(world)]
+    assert all(e.exchange_kind == 1 for e in engines)
+    for r, e in enumerate(engines):
+        lo, hi = signal_range(r, n, world)
+        e.local(xd[lo:hi].clone())  # the rank holds only its slice
+    torch.cuda.synchronize()
+    total = sum(e.exchange_tensor().clone() for e in engines)
+    for e in engines:
+        e.exchange_tensor().copy_(total)
+    torch.cuda.synchronize()
+    for e in engines:
+        locs, vals = e.finish()
+        torch.cuda.synchronize()
+        assert e.plan.status() == 0
+        assert torch.equal(locs, ref_l)
+        torch.testing.assert_close(vals, ref_v, rtol=1e-9, atol=1e-12 * float(ref_v.abs().max()))
+        assert sorted(locs.tolist()) == sorted(S.tolist())
+    # a second execution reuses the captured graphs
+    for r, e in enumerate(engines):
+        lo, hi = signal_range(r, n, world)
+        e.local(xd[lo:hi].clone())
+    torch.cuda.synchronize()
+    total = sum(e.exchange_tensor().clone() for e in engines)
+    for e in engines:
+        e.exchange_tensor().copy_(total)
+        locs, vals = e.finish()
+        torch.cuda.synchronize()
+        assert torch.equal(locs, ref_l)
