@@ -22,7 +22,20 @@ __device__ __forceinline__ unsigned long long gtimer() {
   do { if (threadIdx.x == 0) g_trace[(slot)] = gtimer(); } while (0)
 #define TRACE_END(slot) \
   do { if (threadIdx.x == 0) atomicMax(&g_trace[(slot)], gtimer()); } while (0)
+// Per-kernel span: g_trace[128 + 2 id] = earliest CTA start (after pdl_wait),
+// g_trace[129 + 2 id] = latest CTA end (thread 0; any return path).
+struct KTraceScope {
+  int id;
+  __device__ explicit KTraceScope(int i) : id(i) {
+    if (threadIdx.x == 0) atomicMin(&g_trace[128 + 2 * id], gtimer());
+  }
+  __device__ ~KTraceScope() {
+    if (threadIdx.x == 0) atomicMax(&g_trace[129 + 2 * id], gtimer());
+  }
+};
+#define KTRACE(id) KTraceScope ktrace_scope_(id)
 #else
+#define KTRACE(id) do { } while (0)
 #define TRACE(slot) do { } while (0)
 #define TRACE_END(slot) do { } while (0)
 #endif

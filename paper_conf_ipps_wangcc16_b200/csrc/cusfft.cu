@@ -10,6 +10,7 @@
 #include <cstring>
 #include <new>
 #include <utility>
+#include <string>
 #include <vector>
 
 #include "../../include/cusfft.h"
@@ -121,6 +122,12 @@ struct cusfft_plan_s {
   bool fused1 = false;
   // staged gather: address-sorted gather schedule of this rank
   bool staged = false;
+  // Phase 2 variant (CUSFFT_STAGE_MODE): scatter = phase 1 writes each sample at
+  // phase 2's position (coalesced phase 2) instead of in sorted order (read
+  // through an index); split = phase 2 is a plain fold (k_fold_staged) followed
+  // by the stand-alone FFT pass 1, instead of k_fold_fft1.
+  bool stage_scatter = false;
+  bool stage_split = false;
   int64_t sectors = 0;            // distinct 32-B sectors of x gathered by this rank (the fold's DRAM floor)
   // Slot groups, each with its own sorted schedule (default: one group of all
   // local slots; CUSFFT_STAGE_GROUPS=2 splits location / estimation loops,
@@ -129,7 +136,8 @@ struct cusfft_plan_s {
     int s0 = 0, s1 = 0;          // local slots [s0, s1)
     int64_t total = 0;           // (s1 - s0) * w samples
     uint32_t* spos = nullptr;    // [total] sorted gather positions
-    uint32_t* inv = nullptr;     // [s1 - s0][R][B] staging index in the fused kernel's thread order
+    uint32_t* inv = nullptr;     // [s1 - s0][R][B] staging index in the fused kernel's thread order (index mode)
+    uint32_t* dst = nullptr;     // [total] thread-order staging position of sorted gather q (scatter mode)
   };
   std::vector<StageGroup> groups;
   double2* d_staging = nullptr;   // [max group total]
@@ -154,6 +162,10 @@ struct cusfft_plan_s {
   int* d_ccount = nullptr;        // [n_sel] candidate counters (self-resetting)
   int* d_done = nullptr;          // [n_sel] finished-CTA counters (self-resetting)
   int sel_S = 1;                  // CTAs per location loop in k_select
+  bool vote_packed = false;       // k_vote8 (L_loc <= 8, B <= 16384; CUSFFT_VOTE_BITMAP=1 forces k_vote)
+  int vote8_grid = 1;
+  bool vote_pairs = true;         // k_vote8 pair enumeration when T > ceil(L_loc/2) (CUSFFT_VOTE_PAIRS=0: off)
+  bool sel_multi = false;         // force the multi-CTA k_select (CUSFFT_SELECT_MULTI=1); else k_select1 for B <= 65536
   int* d_hits = nullptr;
   double2* d_hit_vals = nullptr;
   uint64_t* d_hit_keys = nullptr;
@@ -207,6 +219,7 @@ void free_plan(cusfft_plan_t p) {
   for (auto& g : p->groups) {
     if (g.spos) cudaFree(g.spos);
     if (g.inv) cudaFree(g.inv);
+    if (g.dst) cudaFree(g.dst);
   }
   void* ptrs[] = {p->d_taps, p->d_taps_perm, p->d_staging, p->d_ghat, p->d_tw, p->d_slots, p->d_loc_slots, p->d_loc_sigma, p->d_loc_a,
                   p->d_sel_slots, p->d_u, p->d_v, p->d_records, p->d_keys, p->d_zero, p->d_key_index, p->d_ckey, p->d_cidx, p->d_hits, p->d_hit_vals,
@@ -458,6 +471,10 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   P->stream = nullptr;
   if (const char* e = std::getenv("CUSFFT_NO_GRAPH")) P->use_graph = !(e[0] == '1');
   if (const char* e = std::getenv("CUSFFT_BRANCH")) P->branched = (e[0] == '1');
+  if (const char* e = std::getenv("CUSFFT_SELECT_MULTI")) P->sel_multi = (e[0] == '1');
+  P->vote_packed = q.loc_loops <= 8 && B <= kPk && B >= 32;
+  if (const char* e = std::getenv("CUSFFT_VOTE_BITMAP")) P->vote_packed = P->vote_packed && !(e[0] == '1');
+  if (const char* e = std::getenv("CUSFFT_VOTE_PAIRS")) P->vote_pairs = !(e[0] == '0');
   // measurement only: skip the staged gather's phase 1 (valid only for a repeated x)
   if (const char* e = std::getenv("CUSFFT_SKIP_STAGE")) P->skip_stage = (e[0] == '1');
 
@@ -519,6 +536,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     int sms = 148;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     P->vote_grid = (int)std::max<int64_t>(1, std::min<int64_t>((units + 7) / 8, (int64_t)sms * 4));
+    const int64_t units8 = (int64_t)std::max(P->Lloc - P->T + 1, P->Lloc / 2) * P->num;
+    P->vote8_grid = (int)std::max<int64_t>(1, std::min<int64_t>((units8 + 31) / 32, (int64_t)sms));
     P->est_grid = std::max(1, std::min((P->max_hits + 7) / 8, sms * 4));
   }
   if (P->vote_smem > 200 * 1024) {
@@ -589,6 +608,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   }
   if (set_fft_attrs() != cudaSuccess ||
       cudaFuncSetAttribute(k_select, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
+      cudaFuncSetAttribute(k_select1, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_select_sort, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_vote, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_output, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess) {
@@ -638,8 +658,14 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       ranges = {{0, P->nloc_local}, {P->nloc_local, P->Lg}};
     else
       ranges = {{0, P->Lg}};
-    int64_t maxtot = 0;
-    for (auto& r : ranges) maxtot = std::max<int64_t>(maxtot, (int64_t)(r.second - r.first) * P->w);
+    if (const char* em = std::getenv("CUSFFT_STAGE_MODE")) {  // fused_index | fused_scatter | split_index | split_scatter
+      const std::string m(em);
+      P->stage_split = m.rfind("split", 0) == 0;
+      P->stage_scatter = m.find("scatter") != std::string::npos;
+    }
+    int64_t maxtot = 0;  // staging elements: w per slot (index mode) or R B per slot (scatter mode)
+    for (auto& r : ranges)
+      maxtot = std::max<int64_t>(maxtot, (int64_t)(r.second - r.first) * (P->stage_scatter ? P->R * B : P->w));
     // the staging buffer must be (mostly) L2-resident between the two phases
     // (the staging schedule gathers from the whole signal: not for signal-sharded plans)
     P->staged = P->fused1 && !P->xshard && maxtot * 16 <= (int64_t)64 << 20 && !(e && e[0] == '1');
@@ -661,7 +687,11 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
           }
         }
         std::sort(ev.begin(), ev.end());
-        std::vector<uint32_t> spos((size_t)g.total), inv((size_t)(g.s1 - g.s0) * P->R * B, 0u);
+        std::vector<uint32_t> spos((size_t)g.total), dst, inv;
+        if (P->stage_scatter)
+          dst.assign((size_t)g.total, 0u);
+        else
+          inv.assign((size_t)(g.s1 - g.s0) * P->R * B, 0u);
         for (int64_t q = 0; q < g.total; ++q) {
           spos[(size_t)q] = (uint32_t)(ev[(size_t)q] >> 32);
           const uint64_t id = ev[(size_t)q] & 0xFFFFFFFFull;
@@ -669,14 +699,23 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
           const int64_t rr = i / B, j = i % B;
           const int64_t c = j % P->B2, j1 = j / P->B2;
           const int64_t cta = c / C, t = (c % C) * P->B1 + j1;
-          inv[(size_t)((sl * P->R + rr) * B + cta * 256 + t)] = (uint32_t)q;
+          const uint32_t tpos = (uint32_t)((sl * P->R + rr) * B + (P->stage_split ? j : cta * 256 + t));
+          if (P->stage_scatter)
+            dst[(size_t)q] = tpos;
+          else
+            inv[(size_t)tpos] = (uint32_t)q;
         }
         P->groups.push_back(g);
         auto& gg = P->groups.back();
         if ((rc = dalloc(&gg.spos, (size_t)g.total))) return fail(rc);
-        if ((rc = dalloc(&gg.inv, inv.size()))) return fail(rc);
         if ((rc = upload(gg.spos, spos.data(), spos.size() * sizeof(uint32_t)))) return fail(rc);
-        if ((rc = upload(gg.inv, inv.data(), inv.size() * sizeof(uint32_t)))) return fail(rc);
+        if (P->stage_scatter) {
+          if ((rc = dalloc(&gg.dst, dst.size()))) return fail(rc);
+          if ((rc = upload(gg.dst, dst.data(), dst.size() * sizeof(uint32_t)))) return fail(rc);
+        } else {
+          if ((rc = dalloc(&gg.inv, inv.size()))) return fail(rc);
+          if ((rc = upload(gg.inv, inv.data(), inv.size() * sizeof(uint32_t)))) return fail(rc);
+        }
       }
       if ((rc = dalloc(&P->d_staging, (size_t)maxtot))) return fail(rc);
       // Persisting-L2 set-aside for the staging buffer (a device-wide limit: raised, never lowered).
@@ -704,23 +743,27 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
 
 template <int B1T>
 cudaError_t launch_fold_fft1_t(cusfft_plan_t P, const double2* x, const uint32_t* inv, const SlotParam* sp, double2* u,
-                               double2* v, int nslots, ZeroArgs z, cudaStream_t st) {
+                               double2* v, int nslots, ZeroArgs z, cudaStream_t st, bool staged_tord) {
   dim3 grid((unsigned)(P->B / 256), (unsigned)nslots);
   if (inv)  // staged: x is the staging buffer of the group, inv its index
-    return launch_k(k_fold_fft1<B1T, 16, true>, grid, dim3(256), 0, st, P->cur_prio, x, inv,
+    return launch_k(k_fold_fft1<B1T, 16, 1>, grid, dim3(256), 0, st, P->cur_prio, x, inv,
                     (const double*)P->d_taps_perm, sp, u, v, (const double2*)P->d_tw,
                     (int)P->B, P->B2, P->w, P->R, (uint32_t)(P->n - 1), 0u, (uint32_t)P->n, z);
-  return launch_k(k_fold_fft1<B1T, 8, false>, grid, dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)nullptr,
+  if (staged_tord)  // staged in thread order: x is the group's staging buffer
+    return launch_k(k_fold_fft1<B1T, 16, 2>, grid, dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)nullptr,
+                    (const double*)P->d_taps_perm, sp, u, v, (const double2*)P->d_tw,
+                    (int)P->B, P->B2, P->w, P->R, (uint32_t)(P->n - 1), 0u, (uint32_t)P->n, z);
+  return launch_k(k_fold_fft1<B1T, 8, 0>, grid, dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)nullptr,
                   (const double*)P->d_taps_perm, sp, u, v, (const double2*)P->d_tw, (int)P->B, P->B2, P->w, P->R,
                   (uint32_t)(P->n - 1), P->xlo, P->xspan, z);
 }
 
 cudaError_t launch_fold_fft1(cusfft_plan_t P, const double2* x, const uint32_t* inv, const SlotParam* sp, double2* u,
-                             double2* v, int nslots, ZeroArgs z, cudaStream_t st) {
+                             double2* v, int nslots, ZeroArgs z, cudaStream_t st, bool staged_tord = false) {
   switch (P->B1) {
-    case 64: return launch_fold_fft1_t<64>(P, x, inv, sp, u, v, nslots, z, st);
-    case 128: return launch_fold_fft1_t<128>(P, x, inv, sp, u, v, nslots, z, st);
-    case 256: return launch_fold_fft1_t<256>(P, x, inv, sp, u, v, nslots, z, st);
+    case 64: return launch_fold_fft1_t<64>(P, x, inv, sp, u, v, nslots, z, st, staged_tord);
+    case 128: return launch_fold_fft1_t<128>(P, x, inv, sp, u, v, nslots, z, st, staged_tord);
+    case 256: return launch_fold_fft1_t<256>(P, x, inv, sp, u, v, nslots, z, st, staged_tord);
     default: return cudaErrorInvalidValue;
   }
 }
@@ -746,14 +789,23 @@ int launch_fold(cusfft_plan_t P, const double2* x, int s0, int s1, cudaStream_t 
       const int grid = std::max(1, std::min((tot + 8 * 256 - 1) / (8 * 256), sms * 8));
       cudaError_t e = cudaSuccess;
       if (!P->skip_stage) {
-        e = launch_k(k_stage, dim3(grid), dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)g.spos, P->d_staging, tot,
-                     z);
+        e = launch_k(k_stage, dim3(grid), dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)g.spos,
+                     (const uint32_t*)g.dst, P->d_staging, tot, z);
         z = ZeroArgs{nullptr, 0};
       }
       g_pdl = !P->timing;
-      if (e == cudaSuccess)
+      if (e == cudaSuccess && P->stage_split) {
+        dim3 grid2((unsigned)(B / 256), (unsigned)(g.s1 - g.s0));
+        if (g.dst)
+          e = launch_k(k_fold_staged<true>, grid2, dim3(256), 0, st, P->cur_prio, (const double2*)P->d_staging,
+                       (const uint32_t*)nullptr, (const double*)P->d_taps, P->d_u + (size_t)g.s0 * B, B, P->w, P->R, z);
+        else
+          e = launch_k(k_fold_staged<false>, grid2, dim3(256), 0, st, P->cur_prio, (const double2*)P->d_staging,
+                       (const uint32_t*)g.inv, (const double*)P->d_taps, P->d_u + (size_t)g.s0 * B, B, P->w, P->R, z);
+      } else if (e == cudaSuccess)
         e = launch_fold_fft1(P, P->d_staging, g.inv, P->d_slots + (size_t)P->lrank * P->Lg + g.s0,
-                             P->d_u + (size_t)g.s0 * B, P->d_v + (size_t)g.s0 * B, g.s1 - g.s0, z, st);
+                             P->d_u + (size_t)g.s0 * B, P->d_v + (size_t)g.s0 * B, g.s1 - g.s0, z, st,
+                             g.dst != nullptr);
       g_apw = cudaAccessPolicyWindow{};
       CK(e);
     }
@@ -777,7 +829,7 @@ int launch_bfft(cusfft_plan_t P, int s0, int s1, cudaStream_t st) {
   // signal-sharded: the spectra are partial here, keys come after the all-reduce (launch_keys)
   const int* kidx = (P->sel_slots_h.empty() || P->xshard) ? nullptr : P->d_key_index + s0;
   if (P->B1 > 1) {
-    if (!P->fused1) {  // pass 1: B1-point FFTs over columns c (stride B2), twiddle e^{-2 pi i c k1 / B}
+    if (!P->fused1 || (P->staged && P->stage_split)) {  // pass 1: B1-point FFTs over columns c (stride B2), twiddle e^{-2 pi i c k1 / B}
       FftPassArgs a1{P->d_u + (size_t)s0 * B, P->d_v + (size_t)s0 * B, P->d_tw, B, P->logB2, ns * P->B2, B, B, 1,
                      P->B2, 1, P->B2, 1, nullptr, nullptr, nullptr};
       CK(launch_fft(P->B1, a1, P->fft_smem1, st, P->cur_prio));
@@ -822,6 +874,11 @@ int launch_select(cusfft_plan_t P, cudaStream_t st) {
   if (P->prm.cutoff_mode == CUSFFT_CUTOFF_SORT) {
     const int smem = (int)P->B * 12 + (int)((P->B + 31) / 32) * 4;
     CK(launch_k(k_select_sort, dim3((int)P->sel_slots_h.size()), dim3(1024), smem, st, P->cur_prio, sa));
+    return CUSFFT_SUCCESS;
+  }
+  if (P->B <= kSel1MaxB && !P->sel_multi) {
+    const int smem = 4096 * 4 + 64 * 4 + kSelCap * 12 + (int)((P->B + 31) / 32) * 4;
+    CK(launch_k(k_select1, dim3((int)P->sel_slots_h.size()), dim3(1024), smem, st, P->cur_prio, sa));
     return CUSFFT_SUCCESS;
   }
   CK(launch_k(k_select, dim3((int)P->sel_slots_h.size() * P->sel_S), dim3(kSelNT), P->select_smem, st, P->cur_prio,
@@ -881,9 +938,14 @@ int launch_vote(cusfft_plan_t P, cudaStream_t st) {
   va.log2n = ilog2(P->n);
   va.log2B = ilog2(P->B);
   va.nmask = (uint32_t)(P->n - 1);
+  va.pairs = (P->vote_pairs && P->T > (P->Lloc + 1) / 2) ? 1 : 0;
   va.hits = P->d_hits;
   va.hit_count = reinterpret_cast<unsigned*>(P->d_flags);
   va.max_hits = P->max_hits;
+  if (P->vote_packed) {  // L_loc <= 8, B <= kPk: byte-per-bucket probes, one CTA per SM
+    CK(launch_k(k_vote8, dim3(P->vote8_grid), dim3(1024), 0, st, P->cur_prio, va));
+    return CUSFFT_SUCCESS;
+  }
   CK(launch_k(k_vote, dim3(P->vote_grid), dim3(256), P->vote_smem, st, P->cur_prio, va));
   return CUSFFT_SUCCESS;
 }
@@ -1322,11 +1384,21 @@ int cusfft_debug_trace(unsigned long long* host, int32_t n) {
   CK(cudaMemcpyFromSymbol(host, g_trace, sizeof(unsigned long long) * (n < 256 ? n : 256)));
   return CUSFFT_SUCCESS;
 }
+// Reset the trace: phase slots 0, per-kernel start slots (128 + 2 id) ~0.
+int cusfft_debug_trace_reset() {
+  unsigned long long init[256];
+  for (int i = 0; i < 256; ++i) init[i] = (i >= 128 && (i % 2) == 0) ? ~0ull : 0ull;
+  CK(cudaDeviceSynchronize());
+  CK(cudaMemcpyToSymbol(g_trace, init, sizeof(init)));
+  return CUSFFT_SUCCESS;
+}
 #endif
 
 int32_t cusfft_launches_per_execute(cusfft_plan_t plan) {
   if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
-  int n = (plan->staged ? 2 * (int)plan->groups.size() : 1) /*stage + fold per group*/ + (plan->B1 > 1 && !plan->fused1 ? 2 : 1) /*fft*/ + (plan->sel_slots_h.empty() ? 0 : 1) +
+  const bool pass1 = plan->B1 > 1 && (!plan->fused1 || (plan->staged && plan->stage_split));
+  int n = (plan->staged ? 2 * (int)plan->groups.size() : 1) /*stage + fold per group*/ + (pass1 ? 2 : 1) /*fft*/ +
+          (plan->sel_slots_h.empty() ? 0 : 1) + (plan->xshard && !plan->sel_slots_h.empty() ? 1 : 0) /*keys*/ +
           3 /*vote,est,out*/;
   return n;
 }

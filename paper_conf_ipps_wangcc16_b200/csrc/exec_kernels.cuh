@@ -55,6 +55,7 @@ __global__ void __launch_bounds__(256) k_fold(const double2* __restrict__ x, con
                                               int B, int w, int R, uint32_t nmask, uint32_t xlo, uint32_t xspan,
                                               ZeroArgs zero) {
   pdl_wait();
+  KTRACE(4);
   const int j = blockIdx.x * blockDim.x + threadIdx.x;
   const int s = blockIdx.y;
   if (blockIdx.x == 0 && blockIdx.y == 0) TRACE(0);
@@ -107,9 +108,14 @@ __device__ __forceinline__ uint64_t l2_policy_last() {
   return p;
 }
 
+// dst (optional): staging position of sorted gather q in the fused kernel's
+// thread order (scatter staging: phase 2 then reads coalesced, no index);
+// null: staging[q] in sorted order (phase 2 reads it through inv_perm).
 __global__ void __launch_bounds__(256) k_stage(const double2* __restrict__ x, const uint32_t* __restrict__ spos,
-                                               double2* __restrict__ staging, int total, ZeroArgs zero) {
+                                               const uint32_t* __restrict__ dst, double2* __restrict__ staging,
+                                               int total, ZeroArgs zero) {
   pdl_wait();
+  KTRACE(1);
   if (blockIdx.x == 0) TRACE(0);
   zero_part(zero);
   const uint64_t pf = l2_policy_first(), pl = l2_policy_last();
@@ -128,12 +134,60 @@ __global__ void __launch_bounds__(256) k_stage(const double2* __restrict__ x, co
 #pragma unroll
     for (int c = 0; c < 8; ++c) {
       const int q = q0 + c * T;
-      if (q < total)
-        asm volatile("st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %3;" ::"l"(staging + q), "d"(v[c].x),
-                     "d"(v[c].y), "l"(pl));
+      if (q < total) {
+        double2* o = staging + (dst ? __ldg(dst + q) : (uint32_t)q);
+        asm volatile("st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %3;" ::"l"(o), "d"(v[c].x), "d"(v[c].y),
+                     "l"(pl));
+      }
     }
   }
   TRACE_END(6);
+}
+
+// ---------------------------------------------------------------------------
+// Staged gather, phase 2 without the FFT (split mode): thread per (slot,
+// bucket j), natural order.  SCATTER: staging[(s R + rr) B + j] holds round
+// rr's sample (coalesced reads); else staging[inv[(s R + rr) B + j]].  Light
+// enough for 4 CTAs per SM; the rounds are accumulated in Alg. 1's order.
+// ---------------------------------------------------------------------------
+template <bool SCATTER>
+__global__ void __launch_bounds__(256, 4) k_fold_staged(const double2* __restrict__ staging,
+                                                        const uint32_t* __restrict__ inv,
+                                                        const double* __restrict__ taps, double2* __restrict__ u,
+                                                        int B, int w, int R, ZeroArgs zero) {
+  pdl_wait();
+  KTRACE(3);
+  if (blockIdx.x == 0 && blockIdx.y == 0) TRACE(0);
+  zero_part(zero);
+  const int j = blockIdx.x * 256 + threadIdx.x;
+  const int s = blockIdx.y;
+  const int64_t base = (int64_t)s * R * B + j;
+  double ar = 0.0, ai = 0.0;
+  constexpr int RC = 8;
+  for (int r0 = 0; r0 < R; r0 += RC) {
+    uint32_t q[RC];
+    double2 xv[RC];
+    if constexpr (!SCATTER) {
+#pragma unroll
+      for (int c = 0; c < RC; ++c)
+        if (r0 + c < R && j + (r0 + c) * B < w) q[c] = __ldcs(inv + base + (int64_t)(r0 + c) * B);
+    }
+#pragma unroll
+    for (int c = 0; c < RC; ++c)
+      if (r0 + c < R && j + (r0 + c) * B < w)
+        xv[c] = __ldcs(staging + (SCATTER ? base + (int64_t)(r0 + c) * B : (int64_t)q[c]));
+#pragma unroll
+    for (int c = 0; c < RC; ++c) {
+      const int i = j + (r0 + c) * B;
+      if (r0 + c < R && i < w) {
+        const double g = __ldg(taps + i);
+        ar = __dadd_rn(ar, __dmul_rn(g, xv[c].x));
+        ai = __dadd_rn(ai, __dmul_rn(g, xv[c].y));
+      }
+    }
+  }
+  u[(int64_t)s * B + j] = make_double2(ar, ai);
+  TRACE_END(1);
 }
 
 // ---------------------------------------------------------------------------
@@ -147,7 +201,9 @@ __global__ void __launch_bounds__(256) k_stage(const double2* __restrict__ x, co
 // loads of a CTA stay contiguous.  RC gathers per thread in flight; two CTAs
 // per SM so one CTA's FFT epilogue overlaps the other's gathers.
 // ---------------------------------------------------------------------------
-template <int B1T, int RC, bool STAGED>
+// MODE 0: direct gather from x; 1: staged, read through inv_perm; 2: staged in
+// this kernel's thread order (scatter staging), read coalesced.
+template <int B1T, int RC, int MODE>
 __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict__ x,
                                                                    const uint32_t* __restrict__ inv_perm,
                                                                    const double* __restrict__ taps_perm,
@@ -157,6 +213,7 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict_
                                                                    int w, int R, uint32_t nmask, uint32_t xlo,
                                                                    uint32_t xspan, ZeroArgs zero) {
   pdl_wait();
+  KTRACE(2);
   constexpr int C = 256 / B1T;
   __shared__ double2 S[256 + 256 / 8];
   __shared__ double2 twl[B1T];
@@ -170,7 +227,32 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict_
   for (int i = t; i < B1T; i += 256) twl[i] = __ldg(tw + (int64_t)i * B2);  // omega_B1^i
   const double* tp = taps_perm + (int64_t)blockIdx.x * 256 + t;
   double ar = 0.0, ai = 0.0;
-  if constexpr (STAGED) {
+  if constexpr (MODE == 2) {
+    // phase 2, scatter staging: staging[(s R + rr) B + cta 256 + t] is this
+    // thread's round-rr sample; all rounds in flight, coalesced L2 reads.
+    constexpr int RMAX = 16;
+    const double2* sp2 = x + (int64_t)s * R * B + (int64_t)blockIdx.x * 256 + t;
+    double2 xv[RMAX];
+#pragma unroll
+    for (int rr = 0; rr < RMAX; ++rr)
+      if (rr < R && j + rr * B < w) xv[rr] = __ldcs(sp2 + (int64_t)rr * B);
+#pragma unroll
+    for (int rr = 0; rr < RMAX; ++rr) {
+      if (rr < R && j + rr * B < w) {
+        const double g = __ldg(tp + (int64_t)rr * B);
+        ar = __dadd_rn(ar, __dmul_rn(g, xv[rr].x));
+        ai = __dadd_rn(ai, __dmul_rn(g, xv[rr].y));
+      }
+    }
+    for (int rr = RMAX; rr < R; ++rr) {  // R > 16 (small tolerance / Gaussian filters)
+      if (j + rr * B < w) {
+        const double2 v2 = __ldcs(sp2 + (int64_t)rr * B);
+        const double g = __ldg(tp + (int64_t)rr * B);
+        ar = __dadd_rn(ar, __dmul_rn(g, v2.x));
+        ai = __dadd_rn(ai, __dmul_rn(g, v2.y));
+      }
+    }
+  } else if constexpr (MODE == 1) {
     // phase 2: every round's staging index first (one dependent step), then
     // the L2-resident samples in chunks of RC, accumulated in round order.
     constexpr int RMAX = 16;
@@ -435,6 +517,7 @@ struct KeysArgs {
 
 __global__ void __launch_bounds__(256) k_keys(KeysArgs A) {
   pdl_wait();
+  KTRACE(7);
   __shared__ uint32_t sh[4096];
   const int i = blockIdx.y;
   for (int t = threadIdx.x; t < 4096; t += 256) sh[t] = 0;
@@ -453,6 +536,7 @@ __global__ void __launch_bounds__(256) k_keys(KeysArgs A) {
 
 __global__ void __launch_bounds__(kSelNT) k_select(SelArgs A) {
   pdl_wait();
+  KTRACE(8);
   extern __shared__ __align__(16) uint8_t smem[];
   uint32_t* hist = reinterpret_cast<uint32_t*>(smem);
   int* sm = reinterpret_cast<int*>(smem + 4096 * 4);
@@ -611,6 +695,131 @@ __global__ void __launch_bounds__(kSelNT) k_select(SelArgs A) {
 }
 
 // ---------------------------------------------------------------------------
+// Step 4, single-CTA form (B <= kSel1MaxB, the common case): one CTA of 1024
+// threads per location slot does the whole exact selection in shared memory.
+// Level 0 comes from the FFT epilogue's histogram; one pass over the keys
+// (8 chunks of 1024 in flight) writes the bitmap words by ballot and appends
+// boundary-bin candidates to shared memory (warp-aggregated); the boundary is
+// resolved by rank counting (nc <= 256) or a radix select over the candidates
+// (or over all keys of the bin when they overflow kSelCap); then the bitmap
+// and the ascending winner list go out.  Same result as k_select.
+// Dynamic smem: 4096 u32 + 64 int + kSelCap (u64 + int) + ceil(B/32) u32.
+// ---------------------------------------------------------------------------
+constexpr int kSel1MaxB = 65536;
+
+__global__ void __launch_bounds__(1024) k_select1(SelArgs A) {
+  pdl_wait();
+  KTRACE(8);
+  extern __shared__ __align__(16) uint8_t smem[];
+  uint32_t* hist = reinterpret_cast<uint32_t*>(smem);
+  int* sm = reinterpret_cast<int*>(smem + 4096 * 4);
+  uint64_t* skey = reinterpret_cast<uint64_t*>(smem + 4096 * 4 + 64 * 4);
+  int* sidx = reinterpret_cast<int*>(skey + kSelCap);
+  uint32_t* sbits = reinterpret_cast<uint32_t*>(sidx + kSelCap);
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int sel = blockIdx.x;
+  const int B = A.B;
+  uint8_t* rec = A.recs[sel];
+  const uint64_t* keys = A.keys + (int64_t)sel * B;
+  const int words = (B + 31) >> 5;
+  if (sel == 0) TRACE(10);
+  BinPick b0{0, 0, 0};
+  if (!A.threshold_mode) b0 = pick_bin<1024>(A.hist0 + (int64_t)sel * 4096, A.num, sm);
+  const uint32_t d0 = (uint32_t)b0.d;
+  const int k2 = A.num - b0.above;
+  const bool whole = A.threshold_mode || (k2 == b0.cnt);
+  if (tid == 0) sm[41] = 0;
+  __syncthreads();
+  if (sel == 0) TRACE(11);
+  const unsigned lt = (1u << lane) - 1u;
+  for (int c0 = 0; c0 < B; c0 += 8 * 1024) {
+    uint64_t kb[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int i = c0 + u * 1024 + tid;
+      kb[u] = i < B ? __ldg(keys + i) : 0ull;
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int i = c0 + u * 1024 + tid;
+      if (c0 + u * 1024 >= B) break;
+      const uint32_t d = (uint32_t)(kb[u] >> 51) & 0xFFFu;
+      const bool take = i < B && (A.threshold_mode ? kb[u] >= A.thr_key : (d > d0 || (d == d0 && whole)));
+      const bool cand = i < B && !A.threshold_mode && d == d0 && !whole;
+      const uint32_t word = __ballot_sync(kFull, take);
+      if (lane == 0 && (i >> 5) < words) sbits[i >> 5] = word;
+      const unsigned cm = __ballot_sync(kFull, cand);
+      if (cm) {
+        int base = 0;
+        if (lane == __ffs(cm) - 1) base = atomicAdd(&sm[41], __popc(cm));
+        base = __shfl_sync(kFull, base, __ffs(cm) - 1);
+        if (cand) {
+          const int pos = base + __popc(cm & lt);
+          if (pos < kSelCap) {
+            skey[pos] = kb[u];
+            sidx[pos] = i;
+          }
+        }
+      }
+    }
+  }
+  __syncthreads();
+  if (sel == 0) TRACE(12);
+#ifdef CUSFFT_TRACE
+  if (tid == 0 && sel < 16) g_trace[96 + sel] = (unsigned long long)sm[41] | ((unsigned long long)whole << 32);
+#endif
+  if (!whole) {
+    const int nc = sm[41];
+    Prefix96 p{0, 0, 0, 0};
+    or96(p.phi, p.plo, d0, pass_shift(0));
+    or96(p.mhi, p.mlo, 0xFFFu, pass_shift(0));
+    if (nc <= 256) {  // few candidates: exact rank counting
+      if (tid < nc) {
+        const uint64_t mk = skey[tid];
+        const int mi = sidx[tid];
+        int rank = 0;  // candidates preferred to mine: larger key, or equal key and smaller bucket
+        for (int c = 0; c < nc; ++c) rank += (skey[c] > mk) || (skey[c] == mk && sidx[c] < mi);
+        if (rank < k2) atomicOr(&sbits[mi >> 5], 1u << (mi & 31));
+      }
+    } else if (nc <= kSelCap) {
+      p = block_radix_select<PairSrc, 1024>(PairSrc{skey, sidx}, nc, k2, hist, sm, 1, p, false);
+      for (int c = tid; c < nc; c += 1024)
+        if (ge96(p, skey[c], ~(uint32_t)sidx[c])) atomicOr(&sbits[sidx[c] >> 5], 1u << (sidx[c] & 31));
+    } else {  // crowded boundary bin: radix over every key of the bin
+      p = block_radix_select<GKeySrc, 1024>(GKeySrc{keys}, B, k2, hist, sm, 1, p, false);
+      for (int i = tid; i < B; i += 1024) {
+        const uint64_t kk = __ldcg(keys + i);
+        if (((kk >> 51) & 0xFFFu) == d0 && ge96(p, kk, ~(uint32_t)i)) atomicOr(&sbits[i >> 5], 1u << (i & 31));
+      }
+    }
+  }
+  __syncthreads();
+  if (sel == 0) TRACE(13);
+  // bitmap out + ascending winner list (thread t owns words [t wpt, (t+1) wpt))
+  uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap);
+  int* J = reinterpret_cast<int*>(rec + A.lay.off_J);
+  for (int w = tid; w < words; w += 1024) bitmap[w] = sbits[w];
+  const int wpt = (words + 1023) / 1024;
+  int cnt = 0;
+  for (int w = tid * wpt; w < min(words, (tid + 1) * wpt); ++w) cnt += __popc(sbits[w]);
+  int total;
+  int pos = block_excl_scan<1024>(cnt, &total, sm);
+  for (int w = tid * wpt; w < min(words, (tid + 1) * wpt); ++w) {
+    uint32_t bits = sbits[w];
+    while (bits) {
+      const int b = __ffs(bits) - 1;
+      bits &= bits - 1;
+      J[pos++] = w * 32 + b;  // pos < total <= Jcap
+    }
+  }
+  if (tid == 0) {
+    *reinterpret_cast<int*>(rec + A.lay.off_cnt) = total;
+    if (!A.threshold_mode && total != A.num) atomicOr(A.status + 1, 1);
+  }
+  if (sel == 0) TRACE(14);
+}
+
+// ---------------------------------------------------------------------------
 // Step 4, Alg. 3 (L238-L250) as an ablation: one CTA of 1024 threads per
 // location slot sorts all B (|u^|^2, bucket) pairs in shared memory (bitonic,
 // larger key first, ties to the smaller bucket) and keeps the first num.
@@ -618,6 +827,7 @@ __global__ void __launch_bounds__(kSelNT) k_select(SelArgs A) {
 // ---------------------------------------------------------------------------
 __global__ void __launch_bounds__(1024) k_select_sort(SelArgs A) {
   pdl_wait();
+  KTRACE(8);
   extern __shared__ __align__(16) uint8_t smem[];
   const int B = A.B, tid = threadIdx.x;
   uint64_t* sk = reinterpret_cast<uint64_t*>(smem);
@@ -703,6 +913,7 @@ struct VoteArgs {
   uint32_t aa[kMaxLoc];          // a = sigma^-1
   const uint32_t* loc_sigma;     // the same sigmas in global memory (register-resident loads)
   int Lloc, T, num, B, nb, log2nb, log2n, log2B;
+  int pairs;  // k_vote8: pair enumeration (T > ceil(L_loc / 2))
   uint32_t nmask;
   int* hits;
   unsigned* hit_count;
@@ -752,11 +963,16 @@ __device__ __forceinline__ void vote_emit(const VoteArgs& A, bool hit, uint32_t 
   }
 }
 
-// One (q0, J) preimage range per warp, two candidates per lane per step.
-// M = mandatory probes (compile time; M == 0: runtime count mrt).  Survivors
-// of the mandatory probes are queued in shared memory (qF: scaled f, qG:
-// votes so far) and finished 32 at a time (convergent).
-template <int M>
+// One (q0, J) preimage range per warp, VC candidates per lane per step.
+// M = mandatory probes m = min(L_loc - T - q0 + 1, L_loc - 1 - q0) at compile
+// time (M == 0: runtime count mrt): a candidate with m - g > L_loc - T - q0
+// misses among them cannot reach T - 1 later votes and is dropped.  Survivors
+// are queued in shared memory (qF: scaled f, qG: votes so far) and finished
+// 32 at a time (convergent).
+constexpr int kVCmax = 4;
+constexpr int kVQ = 32 + 32 * kVCmax;  // per-warp survivor queue capacity
+
+template <int M, int VC>
 __device__ __forceinline__ void vote_unit(const VoteArgs& A, const uint32_t* __restrict__ bm, const uint32_t* ssig,
                                           int words, int q0, uint32_t Jv, uint32_t a, int mrt, uint32_t* qF,
                                           uint8_t* qG) {
@@ -781,45 +997,52 @@ __device__ __forceinline__ void vote_unit(const VoteArgs& A, const uint32_t* __r
   const uint32_t p0 = Jv * (uint32_t)A.nb - half;
   uint32_t F0 = a * ((p0 + (uint32_t)lane) << sh);
   const uint32_t d32 = a * (32u << sh);
-  const uint32_t d64 = a * (64u << sh);
+  const uint32_t dstep = a * ((32u * VC) << sh);
+  const unsigned lt = (1u << lane) - 1;
   int qn = 0;  // queued survivors (warp-uniform)
-  for (int t0 = 0; t0 < A.nb; t0 += 64, F0 += d64) {
-    const uint32_t F1 = F0 + d32;
-    int g0 = 0, g1 = 0;
+  for (int t0 = 0; t0 < A.nb; t0 += 32 * VC, F0 += dstep) {
+    uint32_t F[VC];
+    int g[VC];
+#pragma unroll
+    for (int c = 0; c < VC; ++c) {
+      F[c] = F0 + (uint32_t)c * d32;
+      g[c] = 0;
+    }
     if (M > 0) {
 #pragma unroll
       for (int qq = 0; qq < MM; ++qq) {
-        const uint32_t h0 = sg[qq] * F0 + half_s, h1 = sg[qq] * F1 + half_s;
-        const uint32_t w0 = lds_u32(base[qq] + ((h0 >> wsh) << 2));
-        const uint32_t w1 = lds_u32(base[qq] + ((h1 >> wsh) << 2));
-        g0 += __funnelshift_r(w0, w0, h0 >> bsh) & 1u;
-        g1 += __funnelshift_r(w1, w1, h1 >> bsh) & 1u;
+#pragma unroll
+        for (int c = 0; c < VC; ++c) {
+          const uint32_t h = sg[qq] * F[c] + half_s;
+          const uint32_t w = lds_u32(base[qq] + ((h >> wsh) << 2));
+          g[c] += __funnelshift_r(w, w, h >> bsh) & 1u;
+        }
       }
     } else {
       for (int qq = 0; qq < m; ++qq) {
         const uint32_t row = bm_s + (uint32_t)((q0 + 1 + qq) * words) * 4u;
-        g0 += probe_sa(row, ssig[q0 + 1 + qq], F0, half_s, bsh);
-        g1 += probe_sa(row, ssig[q0 + 1 + qq], F1, half_s, bsh);
+#pragma unroll
+        for (int c = 0; c < VC; ++c) g[c] += probe_sa(row, ssig[q0 + 1 + qq], F[c], half_s, bsh);
       }
     }
-    const bool s0 = (t0 + lane < A.nb) && (m - g0) <= allowed;
-    const bool s1 = (t0 + 32 + lane < A.nb) && (m - g1) <= allowed;
-    const unsigned b0 = __ballot_sync(kFull, s0);
-    const unsigned b1 = __ballot_sync(kFull, s1);
-    if (b0 | b1) {
-      const unsigned lt = (1u << lane) - 1;
-      if (s0) {
-        const int pos = qn + __popc(b0 & lt);
-        qF[pos] = F0;
-        qG[pos] = (uint8_t)g0;
+    unsigned bal[VC];
+    unsigned any = 0u;
+#pragma unroll
+    for (int c = 0; c < VC; ++c) {
+      const bool sv = (t0 + c * 32 + lane < A.nb) && (m - g[c]) <= allowed;
+      bal[c] = __ballot_sync(kFull, sv);
+      any |= bal[c];
+    }
+    if (any) {
+#pragma unroll
+      for (int c = 0; c < VC; ++c) {
+        if (bal[c] & (1u << lane)) {
+          const int pos = qn + __popc(bal[c] & lt);
+          qF[pos] = F[c];
+          qG[pos] = (uint8_t)g[c];
+        }
+        qn += __popc(bal[c]);
       }
-      const int qn1 = qn + __popc(b0);
-      if (s1) {
-        const int pos = qn1 + __popc(b1 & lt);
-        qF[pos] = F1;
-        qG[pos] = (uint8_t)g1;
-      }
-      qn = qn1 + __popc(b1);
       __syncwarp();
       while (qn >= 32) {  // finish 32 queued survivors, one per lane
         const uint32_t Fq = qF[qn - 32 + lane];
@@ -843,12 +1066,13 @@ __device__ __forceinline__ void vote_unit(const VoteArgs& A, const uint32_t* __r
 
 __global__ void __launch_bounds__(256) k_vote(VoteArgs A) {
   pdl_wait();
+  KTRACE(9);
   extern __shared__ __align__(16) uint8_t smem[];
   if (blockIdx.x == 0) TRACE(30);
   uint32_t* bm = reinterpret_cast<uint32_t*>(smem);
   __shared__ uint32_t ssig[64];
-  __shared__ uint32_t queueF[8][96];
-  __shared__ uint8_t queueG[8][96];
+  __shared__ uint32_t queueF[8][kVQ];
+  __shared__ uint8_t queueG[8][kVQ];
   const int words = (A.B + 31) >> 5;
   if ((words & 3) == 0) {  // 16-B vector loads, all loops' words in flight before the first store
     const int lv4 = A.log2B - 7;  // log2(words / 4)
@@ -897,11 +1121,240 @@ __global__ void __launch_bounds__(256) k_vote(VoteArgs A) {
     const uint32_t a = A.aa[q0];
     const int m = min(A.Lloc - A.T - q0 + 1, A.Lloc - 1 - q0);  // mandatory probes
     switch (m) {
-      case 1: vote_unit<1>(A, bm, ssig, words, q0, Jv, a, 1, qF, qG); break;
-      case 2: vote_unit<2>(A, bm, ssig, words, q0, Jv, a, 2, qF, qG); break;
-      case 3: vote_unit<3>(A, bm, ssig, words, q0, Jv, a, 3, qF, qG); break;
-      case 4: vote_unit<4>(A, bm, ssig, words, q0, Jv, a, 4, qF, qG); break;
-      default: vote_unit<0>(A, bm, ssig, words, q0, Jv, a, m, qF, qG); break;
+      case 1: vote_unit<1, 2>(A, bm, ssig, words, q0, Jv, a, 1, qF, qG); break;
+      case 2: vote_unit<2, 2>(A, bm, ssig, words, q0, Jv, a, 2, qF, qG); break;
+      case 3: vote_unit<3, 2>(A, bm, ssig, words, q0, Jv, a, 3, qF, qG); break;
+      case 4: vote_unit<4, 2>(A, bm, ssig, words, q0, Jv, a, 4, qF, qG); break;
+      default: vote_unit<0, 2>(A, bm, ssig, words, q0, Jv, a, m, qF, qG); break;
+    }
+  }
+  TRACE_END(32);
+}
+
+// ---------------------------------------------------------------------------
+// Step 5, packed form (L_loc <= 8, B <= kPk): the location loops' bitmaps are
+// transposed into one byte per bucket (bit q = bucket selected in loop q) in
+// a static shared array, so a probe is IMAD, SHF, LDS.U8 [b + const], LOP3.
+// One CTA of 1024 threads per SM builds the byte array once; then the same
+// warp-per-(q0, J) enumeration, mandatory probes and survivor queue as k_vote.
+// ---------------------------------------------------------------------------
+constexpr int kPk = 16384;
+
+__device__ __forceinline__ bool vote8_finish(const VoteArgs& A, const uint8_t* pk, const uint32_t* ssig, int q0, int m,
+                                             uint32_t F, int got, uint32_t half_s, int bsh) {
+  int votes = got;
+  for (int q = q0 + 1 + m; q < A.Lloc; ++q) votes += (pk[(ssig[q] * F + half_s) >> bsh] >> q) & 1;
+  bool hit = votes >= A.T - 1;
+  for (int q = 0; q < q0; ++q) hit = hit && !((pk[(ssig[q] * F + half_s) >> bsh] >> q) & 1);
+  return hit;
+}
+
+template <int M>
+__device__ __forceinline__ void vote8_unit(const VoteArgs& A, const uint8_t* pk, const uint32_t* ssig, int q0,
+                                           uint32_t Jv, uint32_t a, int mrt, uint32_t* qF, uint8_t* qG) {
+  constexpr int MM = M > 0 ? M : 1;
+  constexpr int VC = 2;
+  const int lane = threadIdx.x & 31;
+  const int sh = 32 - A.log2n, bsh = 32 - A.log2B;
+  const uint32_t half = (uint32_t)(A.nb >> 1);
+  const uint32_t half_s = half << sh;
+  const int m = M > 0 ? M : mrt;
+  const int allowed = A.Lloc - A.T - q0;
+  uint32_t sg[MM], mk[MM];
+#pragma unroll
+  for (int qq = 0; qq < MM; ++qq) {
+    sg[qq] = __ldg(A.loc_sigma + q0 + 1 + qq);
+    mk[qq] = 1u << (q0 + 1 + qq);
+  }
+  const uint32_t p0 = Jv * (uint32_t)A.nb - half;
+  uint32_t F0 = a * ((p0 + (uint32_t)lane) << sh);
+  const uint32_t d32 = a * (32u << sh);
+  const uint32_t dstep = a * ((32u * VC) << sh);
+  const unsigned lt = (1u << lane) - 1;
+  int qn = 0;
+  for (int t0 = 0; t0 < A.nb; t0 += 32 * VC, F0 += dstep) {
+    uint32_t F[VC], acc[VC];
+#pragma unroll
+    for (int c = 0; c < VC; ++c) {
+      F[c] = F0 + (uint32_t)c * d32;
+      acc[c] = 0u;
+    }
+    if (M > 0) {
+#pragma unroll
+      for (int qq = 0; qq < MM; ++qq)
+#pragma unroll
+        for (int c = 0; c < VC; ++c) acc[c] |= pk[(sg[qq] * F[c] + half_s) >> bsh] & mk[qq];
+    } else {
+      for (int qq = 0; qq < m; ++qq) {
+        const uint32_t sq = ssig[q0 + 1 + qq], mq = 1u << (q0 + 1 + qq);
+#pragma unroll
+        for (int c = 0; c < VC; ++c) acc[c] |= pk[(sq * F[c] + half_s) >> bsh] & mq;
+      }
+    }
+    unsigned bal[VC];
+    int g[VC];
+    unsigned any = 0u;
+#pragma unroll
+    for (int c = 0; c < VC; ++c) {
+      g[c] = __popc(acc[c]);
+      const bool sv = (t0 + c * 32 + lane < A.nb) && (m - g[c]) <= allowed;
+      bal[c] = __ballot_sync(kFull, sv);
+      any |= bal[c];
+    }
+    if (any) {
+#pragma unroll
+      for (int c = 0; c < VC; ++c) {
+        if (bal[c] & (1u << lane)) {
+          const int pos = qn + __popc(bal[c] & lt);
+          qF[pos] = F[c];
+          qG[pos] = (uint8_t)g[c];
+        }
+        qn += __popc(bal[c]);
+      }
+      __syncwarp();
+      while (qn >= 32) {
+        const uint32_t Fq = qF[qn - 32 + lane];
+        const int gq = qG[qn - 32 + lane];
+        __syncwarp();
+        qn -= 32;
+        const bool hit = vote8_finish(A, pk, ssig, q0, m, Fq, gq, half_s, bsh);
+        vote_emit(A, hit, Fq >> sh);
+      }
+    }
+  }
+  if (qn > 0) {
+    const bool has = lane < qn;
+    const uint32_t Fq = has ? qF[lane] : 0u;
+    const int gq = has ? qG[lane] : 0;
+    __syncwarp();
+    const bool hit = has && vote8_finish(A, pk, ssig, q0, m, Fq, gq, half_s, bsh);
+    vote_emit(A, hit, Fq >> sh);
+  }
+}
+
+// Pair enumeration (when T > ceil(L_loc / 2)): with the location loops in
+// pairs (2i, 2i+1), a frequency with >= T votes has some pair voting twice
+// (else it has at most ceil(L_loc/2) votes).  So candidates f = a_{2i} p run
+// over loop 2i's preimage ranges with ONE mandatory probe of loop 2i+1, and
+// f is counted at its first doubly-voting pair: survivors probe every other
+// loop, need >= T votes in all and no earlier pair voting twice.
+__device__ __forceinline__ bool vote8_pair_finish(const VoteArgs& A, const uint8_t* pk, const uint32_t* ssig, int pr,
+                                                  uint32_t F, uint32_t half_s, int bsh) {
+  uint32_t bits = 3u << (2 * pr);
+  for (int q = 0; q < A.Lloc; ++q)
+    if ((q >> 1) != pr) bits |= pk[(ssig[q] * F + half_s) >> bsh] & (1u << q);
+  bool hit = __popc(bits) >= A.T;
+  for (int j = 0; j < pr; ++j) hit = hit && ((bits >> (2 * j)) & 3u) != 3u;
+  return hit;
+}
+
+__device__ __forceinline__ void vote8_pair_unit(const VoteArgs& A, const uint8_t* pk, const uint32_t* ssig, int pr,
+                                                uint32_t Jv, uint32_t a, uint32_t* qF) {
+  constexpr int VC = 2;
+  const int lane = threadIdx.x & 31;
+  const int sh = 32 - A.log2n, bsh = 32 - A.log2B;
+  const uint32_t half = (uint32_t)(A.nb >> 1);
+  const uint32_t half_s = half << sh;
+  const uint32_t sg = __ldg(A.loc_sigma + 2 * pr + 1), mk = 1u << (2 * pr + 1);
+  const uint32_t p0 = Jv * (uint32_t)A.nb - half;
+  uint32_t F0 = a * ((p0 + (uint32_t)lane) << sh);
+  const uint32_t d32 = a * (32u << sh);
+  const uint32_t dstep = a * ((32u * VC) << sh);
+  const unsigned lt = (1u << lane) - 1;
+  int qn = 0;
+  for (int t0 = 0; t0 < A.nb; t0 += 32 * VC, F0 += dstep) {
+    const uint32_t F1 = F0 + d32;
+    const bool s0 = (t0 + lane < A.nb) && (pk[(sg * F0 + half_s) >> bsh] & mk);
+    const bool s1 = (t0 + 32 + lane < A.nb) && (pk[(sg * F1 + half_s) >> bsh] & mk);
+    const unsigned b0 = __ballot_sync(kFull, s0), b1 = __ballot_sync(kFull, s1);
+    if (b0 | b1) {
+      if (s0) qF[qn + __popc(b0 & lt)] = F0;
+      const int qn1 = qn + __popc(b0);
+      if (s1) qF[qn1 + __popc(b1 & lt)] = F1;
+      qn = qn1 + __popc(b1);
+      __syncwarp();
+      while (qn >= 32) {
+        const uint32_t Fq = qF[qn - 32 + lane];
+        __syncwarp();
+        qn -= 32;
+        vote_emit(A, vote8_pair_finish(A, pk, ssig, pr, Fq, half_s, bsh), Fq >> sh);
+      }
+    }
+  }
+  if (qn > 0) {
+    const bool has = lane < qn;
+    const uint32_t Fq = has ? qF[lane] : 0u;
+    __syncwarp();
+    vote_emit(A, has && vote8_pair_finish(A, pk, ssig, pr, Fq, half_s, bsh), Fq >> sh);
+  }
+}
+
+__global__ void __launch_bounds__(1024, 1) k_vote8(VoteArgs A) {
+  pdl_wait();
+  KTRACE(9);
+  __shared__ __align__(16) uint8_t pk[kPk];
+  __shared__ uint32_t ssig[kMaxLoc];
+  __shared__ uint32_t queueF[32][kVQ];
+  __shared__ uint8_t queueG[32][kVQ];
+  __shared__ int scnt[kMaxLoc + 1];
+  if (blockIdx.x == 0) TRACE(30);
+  const int tid = threadIdx.x;
+  const int words = (A.B + 31) >> 5;
+  // transpose: bucket 32 w + 4 j + i -> byte (w 8 + j) * 4 + i, bit q = loop q
+  for (int w = tid; w < words; w += 1024) {
+    uint32_t bw[8];
+#pragma unroll
+    for (int q = 0; q < 8; ++q) bw[q] = q < A.Lloc ? __ldg(A.bmp[q] + w) : 0u;
+    auto nib = [&](int j) {
+      uint32_t v = 0u;
+#pragma unroll
+      for (int q = 0; q < 8; ++q) v |= ((((bw[q] >> (4 * j)) & 0xFu) * 0x00204081u) & 0x01010101u) << q;
+      return v;
+    };
+    reinterpret_cast<uint4*>(pk)[w * 2] = make_uint4(nib(0), nib(1), nib(2), nib(3));
+    reinterpret_cast<uint4*>(pk)[w * 2 + 1] = make_uint4(nib(4), nib(5), nib(6), nib(7));
+  }
+  // enumerated loops: pairs' first loops 0, 2, 4, ... (pair mode) or 0 .. L_loc - T
+  const int nenum = A.pairs ? A.Lloc / 2 : A.Lloc - A.T + 1;
+  if (tid < A.Lloc) ssig[tid] = A.sig[tid];
+  if (tid == 0) {
+    int acc = 0;
+    scnt[0] = 0;
+    for (int e = 0; e < nenum; ++e) {
+      acc += __ldg(A.cntp[A.pairs ? 2 * e : e]);
+      scnt[e + 1] = acc;
+    }
+  }
+  __syncthreads();
+  if (blockIdx.x == 0) TRACE(31);
+  const int units = scnt[nenum];
+  uint32_t* qF = queueF[tid >> 5];
+  uint8_t* qG = queueG[tid >> 5];
+  const int warp = (blockIdx.x * 1024 + tid) >> 5;
+  const int nwarps = gridDim.x * 32;
+  if (A.pairs) {
+    for (int unit = warp; unit < units; unit += nwarps) {
+      int pr = 0;
+      while (unit >= scnt[pr + 1]) ++pr;
+      const uint32_t Jv = (uint32_t)__ldg(A.Jp[2 * pr] + (unit - scnt[pr]));
+      vote8_pair_unit(A, pk, ssig, pr, Jv, A.aa[2 * pr], qF);
+    }
+    TRACE_END(32);
+    return;
+  }
+  for (int unit = warp; unit < units; unit += nwarps) {
+    int q0 = 0;
+    while (unit >= scnt[q0 + 1]) ++q0;
+    const int jidx = unit - scnt[q0];
+    const uint32_t Jv = (uint32_t)__ldg(A.Jp[q0] + jidx);
+    const uint32_t a = A.aa[q0];
+    const int m = min(A.Lloc - A.T - q0 + 1, A.Lloc - 1 - q0);
+    switch (m) {
+      case 1: vote8_unit<1>(A, pk, ssig, q0, Jv, a, 1, qF, qG); break;
+      case 2: vote8_unit<2>(A, pk, ssig, q0, Jv, a, 2, qF, qG); break;
+      case 3: vote8_unit<3>(A, pk, ssig, q0, Jv, a, 3, qF, qG); break;
+      case 4: vote8_unit<4>(A, pk, ssig, q0, Jv, a, 4, qF, qG); break;
+      default: vote8_unit<0>(A, pk, ssig, q0, Jv, a, m, qF, qG); break;
     }
   }
   TRACE_END(32);
@@ -980,6 +1433,7 @@ __device__ __forceinline__ double warp_rank_select(double a0, double a1, int L, 
 
 __global__ void __launch_bounds__(256) k_estimate(EstArgs A) {
   pdl_wait();
+  KTRACE(10);
   __shared__ uint32_t sdig[8];
   if (blockIdx.x == 0) TRACE(40);
   const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
@@ -1042,6 +1496,7 @@ __global__ void __launch_bounds__(1024) k_output(const int* __restrict__ hits, c
                                                  int k, int kp2, int log2n, int64_t* __restrict__ locs,
                                                  double2* __restrict__ vals, int* __restrict__ status) {
   pdl_wait();
+  KTRACE(11);
   extern __shared__ __align__(16) uint8_t smem[];
   uint32_t* hist = reinterpret_cast<uint32_t*>(smem);
   int* sm = reinterpret_cast<int*>(smem + 4096 * 4);

@@ -40,7 +40,9 @@ want = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "lts__t_sectors_srcunit_tex_op_read.sum", "sm__warps_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread",
         "smsp__inst_executed.sum", "sm__throughput.avg.pct_of_peak_sustained_elapsed", "launch__grid_size", "launch__block_size"]
 traffic = None
-for name, rep in [("k_fold_fft1 (fold + FFT pass 1)", f"{G}/prof_fold_full.ncu-rep"), ("k_fft (pass 2 + keys)", f"{G}/prof_k_fft.ncu-rep"),
+fold_parts = {}
+for name, rep in [("k_stage (staged gather, phase 1)", f"{G}/prof_k_stage.ncu-rep"),
+                  ("k_fold_fft1 (fold phase 2 + FFT pass 1)", f"{G}/prof_fold_full.ncu-rep"), ("k_fft (pass 2 + keys)", f"{G}/prof_k_fft.ncu-rep"),
                   ("k_select", f"{G}/prof_k_select.ncu-rep"), ("k_vote", f"{G}/prof_k_vote.ncu-rep"),
                   ("k_estimate", f"{G}/prof_k_estimate.ncu-rep"), ("k_output", f"{G}/prof_k_output.ncu-rep")]:
     if not os.path.exists(rep):
@@ -51,15 +53,20 @@ for name, rep in [("k_fold_fft1 (fold + FFT pass 1)", f"{G}/prof_fold_full.ncu-r
     for w in want:
         if w in m:
             lines.append(f"| {w} | {m[w]} |")
-    if "fold" in name and "dram__bytes_read.sum" in m:
+    if ("fold" in name or "stage" in name) and "dram__bytes_read.sum" in m:
         out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
         rows = list(csv.reader(out.splitlines()))
         unit = dict(zip(rows[0], rows[1]))
         scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
         rd = float(m["dram__bytes_read.sum"]) * scale[unit["dram__bytes_read.sum"]]
         wr = float(m["dram__bytes_write.sum"]) * scale[unit["dram__bytes_write.sum"]]
-        traffic = {"kernel": "k_fold_fft1", "config": "C3", "source": f"{tag}_ncu_summary.md (ncu --set full)",
-                   "dram_bytes_read": rd, "dram_bytes_write": wr, "dram_bytes_per_launch": rd + wr}
+        fold_parts[name.split()[0]] = (rd, wr)
+if fold_parts:
+    rd = sum(v[0] for v in fold_parts.values())
+    wr = sum(v[1] for v in fold_parts.values())
+    traffic = {"kernel": " + ".join(sorted(fold_parts)), "config": "C3", "source": f"{tag}_ncu_summary.md (ncu --set full)",
+               "parts": {k: {"dram_bytes_read": v[0], "dram_bytes_write": v[1]} for k, v in fold_parts.items()},
+               "dram_bytes_read": rd, "dram_bytes_write": wr, "dram_bytes_per_launch": rd + wr}
 if traffic:
     json.dump(traffic, open(f"{P}/fold_traffic_C3.json", "w"), indent=1)
 open(f"{P}/{tag}_ncu_summary.md", "w").write("\n".join(lines) + "\n")

@@ -10,7 +10,8 @@ reps = int(sys.argv[2]) if len(sys.argv) > 2 else 4
 LL = int(sys.argv[3]) if len(sys.argv) > 3 else 16
 x, S, X = planted_signal(n, k, 1)
 xd = torch.from_numpy(x).cuda()
-plan = Plan(n, k, L=LL, seed=3)
+tol = {"C3": 1e-7}.get(cfg, 1e-8)  # bench.py TOLERANCE
+plan = Plan(n, k, L=LL, seed=3, tolerance=tol)
 for _ in range(reps):
     locs, vals = plan.execute(xd)
 torch.cuda.synchronize()

@@ -1,4 +1,5 @@
-"""Phase trace of the C3 pipeline (needs the -DCUSFFT_TRACE build, CUSFFT_LIB=libcusfft_trace.so)."""
+"""In-graph per-kernel spans of the C3 pipeline (needs the -DCUSFFT_TRACE build:
+CUSFFT_LIB=libcusfft_trace.so).  Usage: trace_c3.py [L] [tolerance] [reps]"""
 import ctypes, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
@@ -6,23 +7,40 @@ from paper_conf_ipps_wangcc16_b200 import Plan, load_library
 from paper_conf_ipps_wangcc16_b200.workload import planted_signal
 n, k = 2**24, 1000
 L = int(sys.argv[1]) if len(sys.argv) > 1 else 16
+tol = float(sys.argv[2]) if len(sys.argv) > 2 else 1e-7
+reps = int(sys.argv[3]) if len(sys.argv) > 3 else 5
 x, S, X = planted_signal(n, k, 1)
 xd = torch.from_numpy(x).cuda()
-plan = Plan(n, k, L=L, seed=3)
+plan = Plan(n, k, L=L, seed=3, tolerance=tol)
 lib = load_library()
 fl = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 fr = torch.ones(64 << 20, dtype=torch.int32, device="cuda")
-os.environ.get("X")
-for rep in range(4):
+names = {1: "k_stage", 2: "k_fold_fft1", 3: "k_fold_staged", 4: "k_fold", 5: "k_fft pass1", 6: "k_fft pass2",
+         7: "k_keys", 8: "k_select", 9: "k_vote", 10: "k_estimate", 11: "k_output"}
+acc = {}
+for rep in range(reps):
     fl.zero_(); fr.sum()
+    torch.cuda.synchronize()
+    lib.cusfft_debug_trace_reset()
     plan.execute(xd)
     torch.cuda.synchronize()
-buf = (ctypes.c_ulonglong * 256)()
-# one more run on a zeroed trace buffer
-zero = (ctypes.c_ulonglong * 256)()
-lib.cusfft_debug_trace(buf, 256)
-t = np.array(list(buf), dtype=np.float64)
-nz = {i: t[i] for i in range(256) if t[i] > 0}
-t0 = min(nz.values())
-for i, v in sorted(nz.items(), key=lambda kv: kv[1]):
-    print(f"slot {i:3d}  +{(v - t0) / 1e3:8.2f} us")
+    buf = (ctypes.c_ulonglong * 256)()
+    lib.cusfft_debug_trace(buf, 256)
+    t = np.array(list(buf), dtype=np.float64)
+    spans = {i: (t[128 + 2 * i], t[129 + 2 * i]) for i in names if t[129 + 2 * i] > 0}
+    t0 = min(s for s, e in spans.values())
+    end = max(e for s, e in spans.values())
+    if rep == 0:
+        continue  # first run captures the graph
+    if rep == reps - 1:
+        phases = {i: (t[i] - t0) / 1e3 for i in range(96) if t[i] > 0}
+        print("phase slots (us):", " ".join(f"{i}:{v:.2f}" for i, v in sorted(phases.items(), key=lambda kv: kv[1])))
+        print("select candidates per loop:", [int(t[96 + i]) & 0xFFFFFFFF for i in range(16) if t[96 + i] > 0])
+    for i, (s, e) in spans.items():
+        acc.setdefault(i, []).append(((s - t0) / 1e3, (e - t0) / 1e3))
+    acc.setdefault(0, []).append((0.0, (end - t0) / 1e3))
+print(f"C3 L={L} tol={tol:g} staged={plan.info()['staged'] if hasattr(plan, 'info') else '?'} mode={os.environ.get('CUSFFT_STAGE_MODE', 'default')}")
+print(f"{'kernel':16s} {'start us':>9s} {'end us':>9s} {'span us':>9s}")
+for i, v in sorted(acc.items(), key=lambda kv: np.mean([a for a, b in kv[1]])):
+    s = np.median([a for a, b in v]); e = np.median([b for a, b in v])
+    print(f"{names.get(i, 'TOTAL'):16s} {s:9.2f} {e:9.2f} {e - s:9.2f}")

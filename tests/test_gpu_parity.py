@@ -112,6 +112,10 @@ CASES = [
     (2 ** 16, 20, None, 12, dict(filter=1)),          # Gaussian filter
     (2 ** 16, 20, None, 16, dict(tau_mode=0)),        # Alg. 2 literal tau = 0
     (2 ** 15, 1, None, 16, {}),                       # k = 1
+    (2 ** 16, 32, None, 16, dict(loc_loops=8, vote_threshold=4)),   # vote: no pair enumeration (T <= L_loc/2)
+    (2 ** 16, 32, None, 14, dict(loc_loops=7, vote_threshold=5)),   # vote: pairs + odd singleton loop
+    (2 ** 16, 32, None, 16, dict(loc_loops=12, vote_threshold=7)),  # vote: L_loc > 8, bitmap kernel
+    (2 ** 21, 60, 32768, 8, dict(loc_loops=6, vote_threshold=4)),   # vote: B > 16384, bitmap kernel; multi-pass FFT
 ]
 
 
@@ -281,3 +285,30 @@ def test_parity_snr_sweep(snr_db):
     x, S, X = planted_signal(n, k, seed=11, snr_db=snr_db)
     plan, ref, locs, vals = run_pair(x, n, k, None, 16, shared_taps=True, seed=6)
     check_all(plan, ref, locs, vals, fold_bit_exact=True)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("env", [{"CUSFFT_VOTE_PAIRS": "0"}, {"CUSFFT_VOTE_BITMAP": "1"}, {"CUSFFT_SELECT_MULTI": "1"},
+                                 {"CUSFFT_STAGE_MODE": "split_index"}, {"CUSFFT_STAGE_MODE": "fused_scatter"},
+                                 {"CUSFFT_STAGE_MODE": "split_scatter"}, {"CUSFFT_NO_STAGE": "1"}])
+def test_kernel_variants_agree(env, monkeypatch):
+    """Every alternative kernel path (selected at plan time by environment
+    switches, used for A/B measurements) gives the default path's hits and
+    output exactly (same fold order, same selection rule)."""
+    import torch
+    from paper_conf_ipps_wangcc16_b200 import Plan
+    n, k = 2 ** 20, 100
+    x, S, X = planted_signal(n, k, seed=21)
+    xd = torch.from_numpy(x).cuda()
+    base = Plan(n, k, L=16, seed=4, debug=1)
+    l0, v0 = base.execute(xd)
+    h0 = np.sort(base.debug(DEBUG_HITS))
+    for key, val in env.items():
+        monkeypatch.setenv(key, val)
+    alt = Plan(n, k, L=16, seed=4, debug=1)
+    l1, v1 = alt.execute(xd)
+    torch.cuda.synchronize()
+    assert alt.status() == 0
+    assert np.array_equal(np.sort(alt.debug(DEBUG_HITS)), h0)
+    assert torch.equal(l1, l0)
+    assert torch.equal(v1, v0)
