@@ -165,7 +165,8 @@ struct cusfft_plan_s {
   bool vote_packed = false;       // k_vote8 (L_loc <= 8, B <= 16384; CUSFFT_VOTE_BITMAP=1 forces k_vote)
   int vote8_grid = 1;
   bool vote_pairs = true;         // k_vote8 pair enumeration when T > ceil(L_loc/2) (CUSFFT_VOTE_PAIRS=0: off)
-  bool sel_multi = false;         // force the multi-CTA k_select (CUSFFT_SELECT_MULTI=1); else k_select1 for B <= 65536
+  bool sel_multi = false;
+  bool sel_cluster = false;       // k_select_cluster (256 <= B <= 65536; CUSFFT_SELECT=single|multi to A/B)         // force the multi-CTA k_select (CUSFFT_SELECT_MULTI=1); else k_select1 for B <= 65536
   int* d_hits = nullptr;
   double2* d_hit_vals = nullptr;
   uint64_t* d_hit_keys = nullptr;
@@ -472,6 +473,11 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   if (const char* e = std::getenv("CUSFFT_NO_GRAPH")) P->use_graph = !(e[0] == '1');
   if (const char* e = std::getenv("CUSFFT_BRANCH")) P->branched = (e[0] == '1');
   if (const char* e = std::getenv("CUSFFT_SELECT_MULTI")) P->sel_multi = (e[0] == '1');
+  P->sel_cluster = B >= 256 && B <= 65536 && !P->sel_multi && q.cutoff_mode != CUSFFT_CUTOFF_SORT;
+  if (const char* e = std::getenv("CUSFFT_SELECT")) {
+    if (e[0] == 's') P->sel_cluster = false;                        // single CTA (k_select1)
+    if (e[0] == 'm') { P->sel_cluster = false; P->sel_multi = true; }  // multi-CTA (k_select)
+  }
   P->vote_packed = q.loc_loops <= 8 && B <= kPk && B >= 32;
   if (const char* e = std::getenv("CUSFFT_VOTE_BITMAP")) P->vote_packed = P->vote_packed && !(e[0] == '1');
   if (const char* e = std::getenv("CUSFFT_VOTE_PAIRS")) P->vote_pairs = !(e[0] == '0');
@@ -609,6 +615,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   if (set_fft_attrs() != cudaSuccess ||
       cudaFuncSetAttribute(k_select, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_select1, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
+      cudaFuncSetAttribute(k_select_cluster, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_select_sort, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_vote, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_output, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess) {
@@ -874,6 +881,27 @@ int launch_select(cusfft_plan_t P, cudaStream_t st) {
   if (P->prm.cutoff_mode == CUSFFT_CUTOFF_SORT) {
     const int smem = (int)P->B * 12 + (int)((P->B + 31) / 32) * 4;
     CK(launch_k(k_select_sort, dim3((int)P->sel_slots_h.size()), dim3(1024), smem, st, P->cur_prio, sa));
+    return CUSFFT_SUCCESS;
+  }
+  if (P->sel_cluster) {
+    const int smem = (int)sizeof(SelClusterSmem) + (int)(P->B / kSelCL / 32) * 4;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)(P->sel_slots_h.size() * kSelCL));
+    cfg.blockDim = dim3(kSelCNT);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[3];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = kSelCL;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[1].val.programmaticStreamSerializationAllowed = g_pdl ? 1 : 0;
+    attr[2].id = cudaLaunchAttributePriority;
+    attr[2].val.priority = P->cur_prio;
+    cfg.attrs = attr;
+    cfg.numAttrs = 3;
+    CK(cudaLaunchKernelEx(&cfg, k_select_cluster, sa));
     return CUSFFT_SUCCESS;
   }
   if (P->B <= kSel1MaxB && !P->sel_multi) {

@@ -6,6 +6,8 @@
 //   k_estimate  Step 6     per-loop estimates and their median
 //   k_output    output     top-k hits by |val|^2, sorted by location
 #pragma once
+#include <cooperative_groups.h>
+
 #include "common.cuh"
 #include "fft.cuh"
 
@@ -705,6 +707,24 @@ __global__ void __launch_bounds__(kSelNT) k_select(SelArgs A) {
 // and the ascending winner list go out.  Same result as k_select.
 // Dynamic smem: 4096 u32 + 64 int + kSelCap (u64 + int) + ceil(B/32) u32.
 // ---------------------------------------------------------------------------
+// Warp-parallel rank of candidate (mk, mi) among n (key, index) pairs in
+// shared memory: how many are preferred to it (larger key, or equal key and
+// smaller bucket).  Lanes split the pairs; one ballot per 32.
+__device__ __forceinline__ int warp_rank(const uint64_t* ck, const int* ci, int n, uint64_t mk, int mi) {
+  const int lane = threadIdx.x & 31;
+  int rank = 0;
+  for (int c0 = 0; c0 < n; c0 += 32) {
+    const int c = c0 + lane;
+    bool pref = false;
+    if (c < n) {
+      const uint64_t kc = ck[c];
+      pref = (kc > mk) | ((kc == mk) & (ci[c] < mi));
+    }
+    rank += __popc(__ballot_sync(kFull, pref));
+  }
+  return rank;
+}
+
 constexpr int kSel1MaxB = 65536;
 
 __global__ void __launch_bounds__(1024) k_select1(SelArgs A) {
@@ -773,13 +793,11 @@ __global__ void __launch_bounds__(1024) k_select1(SelArgs A) {
     Prefix96 p{0, 0, 0, 0};
     or96(p.phi, p.plo, d0, pass_shift(0));
     or96(p.mhi, p.mlo, 0xFFFu, pass_shift(0));
-    if (nc <= 256) {  // few candidates: exact rank counting
-      if (tid < nc) {
-        const uint64_t mk = skey[tid];
-        const int mi = sidx[tid];
-        int rank = 0;  // candidates preferred to mine: larger key, or equal key and smaller bucket
-        for (int c = 0; c < nc; ++c) rank += (skey[c] > mk) || (skey[c] == mk && sidx[c] < mi);
-        if (rank < k2) atomicOr(&sbits[mi >> 5], 1u << (mi & 31));
+    if (nc <= 256) {  // few candidates: exact rank counting, warp per candidate
+      for (int j = tid >> 5; j < nc; j += 32) {
+        const int mi = sidx[j];
+        const int rank = warp_rank(skey, sidx, nc, skey[j], mi);
+        if (lane == 0 && rank < k2) atomicOr(&sbits[mi >> 5], 1u << (mi & 31));
       }
     } else if (nc <= kSelCap) {
       p = block_radix_select<PairSrc, 1024>(PairSrc{skey, sidx}, nc, k2, hist, sm, 1, p, false);
@@ -817,6 +835,216 @@ __global__ void __launch_bounds__(1024) k_select1(SelArgs A) {
     if (!A.threshold_mode && total != A.num) atomicOr(A.status + 1, 1);
   }
   if (sel == 0) TRACE(14);
+}
+
+// ---------------------------------------------------------------------------
+// Step 4, cluster form (default for 256 <= B <= 65536): a cluster of kSelCL
+// CTAs per location slot, CTA r owning keys [r B/kSelCL, (r+1) B/kSelCL) and
+// level-0 bins [r 4096/kSelCL, ...).  Distributed shared memory replaces the
+// global candidate list and the last-CTA hand-off of k_select:
+//   1. each CTA sums its bin slice; cluster barrier
+//   2. the CTA holding the boundary bin finds d0 (block scan); barrier
+//   3. every CTA classifies its keys: bitmap words by ballot in its own smem,
+//      boundary-bin candidates appended to CTA 0's smem (remote atomics),
+//      its "take" count to CTA 0; barrier
+//   4. CTA 0 resolves the boundary exactly (rank counting, or radix over the
+//      candidates / over all keys of the bin if they overflowed), ORs the
+//      winners' bits into the owners' smem words, hands out J offsets; barrier
+//   5. every CTA writes its bitmap words and its part of the ascending J.
+// Same result as k_select / k_select1.
+// ---------------------------------------------------------------------------
+constexpr int kSelCL = 8;     // CTAs per cluster (portable maximum)
+constexpr int kSelCNT = 256;  // threads per CTA
+
+struct SelClusterSmem {
+  uint32_t hist[4096];          // radix scratch
+  int sm[64];
+  uint64_t ckey[kSelCap];       // candidates (appended into CTA 0, copied by every CTA)
+  int cidx[kSelCap];
+  int ncand;                    // candidate counter (CTA 0)
+  int part[kSelCL];             // bin-slice totals (pushed to every CTA)
+  int pick[3];                  // d0, above, cnt (pushed by the boundary CTA)
+  int cnt[kSelCL];              // final winners per CTA (pushed to every CTA)
+};
+
+__global__ void __launch_bounds__(kSelCNT, 1) k_select_cluster(SelArgs A) {
+  pdl_wait();
+  KTRACE(8);
+  namespace cg = cooperative_groups;
+  cg::cluster_group cl = cg::this_cluster();
+  extern __shared__ __align__(16) uint8_t smem[];
+  SelClusterSmem& S = *reinterpret_cast<SelClusterSmem*>(smem);
+  uint32_t* sbits = reinterpret_cast<uint32_t*>(smem + sizeof(SelClusterSmem));  // this CTA's words
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int r = (int)cl.block_rank();
+  const int sel = blockIdx.x / kSelCL;
+  const int B = A.B;
+  const int per = B / kSelCL;           // keys per CTA (multiple of 32)
+  const int wpc = per >> 5;             // words per CTA
+  const int k0 = r * per;
+  uint8_t* rec = A.recs[sel];
+  const uint64_t* keys = A.keys + (int64_t)sel * B;
+  const uint32_t* h0 = A.hist0 + (int64_t)sel * 4096;
+  if (sel == 0 && r == 0) TRACE(10);
+  // my keys (first chunk) and my two level-0 bins, all in flight at once
+  constexpr int KC = 8;
+  constexpr int BPC = 4096 / kSelCL;    // bins per CTA; thread t holds bins base, base - 1 (descending)
+  const int hbase = r * BPC + BPC - 1 - 2 * tid;
+  int c0 = 0, c1 = 0;
+  if (!A.threshold_mode) {
+    c0 = (int)__ldg(h0 + hbase);
+    c1 = (int)__ldg(h0 + hbase - 1);
+  }
+  uint64_t kb[KC];
+#pragma unroll
+  for (int u = 0; u < KC; ++u) {
+    const int i = u * kSelCNT + tid;
+    kb[u] = i < per ? __ldg(keys + k0 + i) : 0ull;
+  }
+  if (r == 0 && tid == 0) S.ncand = 0;
+  // 1. slice totals, pushed to every CTA of the cluster
+  int tot, ex = 0;
+  if (!A.threshold_mode) {
+    ex = block_excl_scan<kSelCNT>(c0 + c1, &tot, S.sm);
+    if (tid < kSelCL) cl.map_shared_rank(&S, tid)->part[r] = tot;
+  }
+  cl.sync();
+  // 2. the boundary slice (slices descending r = kSelCL-1 .. 0) finds d0 and pushes it
+  int d0 = 0, k2 = 0;
+  bool whole = true;
+  if (!A.threshold_mode) {
+    int above = 0, bs = 0;
+#pragma unroll
+    for (int c = kSelCL - 1; c >= 0; --c) {
+      const int pc = S.part[c];
+      if (above + pc >= A.num) { bs = c; break; }
+      above += pc;
+    }
+    if (r == bs) {
+      const int e = ex + above, kr = A.num;
+      int pk0 = -1, pk1 = 0, pk2 = 0;
+      if (e < kr && kr <= e + c0) { pk0 = hbase; pk1 = e; pk2 = c0; }
+      else if (e + c0 < kr && kr <= e + c0 + c1) { pk0 = hbase - 1; pk1 = e + c0; pk2 = c1; }
+      if (pk0 >= 0)
+        for (int c = 0; c < kSelCL; ++c) {
+          int* dst = cl.map_shared_rank(&S, c)->pick;
+          dst[0] = pk0; dst[1] = pk1; dst[2] = pk2;
+        }
+    }
+    cl.sync();
+    d0 = S.pick[0];
+    k2 = A.num - S.pick[1];
+    whole = (k2 == S.pick[2]);
+  }
+  if (sel == 0 && r == 0) TRACE(11);
+  // 3. classify my keys: bitmap words in my smem, candidates appended to CTA 0
+  SelClusterSmem* S0 = cl.map_shared_rank(&S, 0);
+  const unsigned lt = (1u << lane) - 1u;
+  for (int cb = 0; cb < per; cb += KC * kSelCNT) {
+    if (cb > 0) {
+#pragma unroll
+      for (int u = 0; u < KC; ++u) {
+        const int i = cb + u * kSelCNT + tid;
+        kb[u] = i < per ? __ldg(keys + k0 + i) : 0ull;
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < KC; ++u) {
+      const int i = cb + u * kSelCNT + tid;
+      if (cb + u * kSelCNT >= per) break;
+      const uint32_t d = (uint32_t)(kb[u] >> 51) & 0xFFFu;
+      const bool take = i < per && (A.threshold_mode ? kb[u] >= A.thr_key : (d > (uint32_t)d0 || (d == (uint32_t)d0 && whole)));
+      const bool cand = i < per && !A.threshold_mode && d == (uint32_t)d0 && !whole;
+      const uint32_t word = __ballot_sync(kFull, take);
+      if (lane == 0 && i < per) sbits[i >> 5] = word;  // per is a multiple of 32: whole warps in or out
+      const unsigned cm = __ballot_sync(kFull, cand);
+      if (cm) {
+        int bpos = 0;
+        if (lane == __ffs(cm) - 1) bpos = atomicAdd(&S0->ncand, __popc(cm));
+        bpos = __shfl_sync(kFull, bpos, __ffs(cm) - 1);
+        if (cand) {
+          const int pos = bpos + __popc(cm & lt);
+          if (pos < kSelCap) {
+            S0->ckey[pos] = kb[u];
+            S0->cidx[pos] = k0 + i;
+          }
+        }
+      }
+    }
+  }
+  cl.sync();
+  if (sel == 0 && r == 0) TRACE(12);
+  // 4. every CTA resolves its own candidates against the whole list
+  if (!whole) {
+    const int nc = S0->ncand;
+    Prefix96 p{0, 0, 0, 0};
+    or96(p.phi, p.plo, (uint32_t)d0, pass_shift(0));
+    or96(p.mhi, p.mlo, 0xFFFu, pass_shift(0));
+    if (nc <= kSelCap) {
+      if (r != 0)  // local copy of the candidate list (one remote round trip per thread)
+        for (int c = tid; c < nc; c += kSelCNT) {
+          S.ckey[c] = S0->ckey[c];
+          S.cidx[c] = S0->cidx[c];
+        }
+      __syncthreads();
+      if (nc <= kSelCNT) {  // warp per candidate of mine, lanes split the comparisons
+        for (int j = tid >> 5; j < nc; j += kSelCNT / 32) {
+          const int mi = S.cidx[j];
+          if (mi < k0 || mi >= k0 + per) continue;  // warp-uniform
+          const int rank = warp_rank(S.ckey, S.cidx, nc, S.ckey[j], mi);
+          if (lane == 0 && rank < k2) atomicOr(&sbits[(mi - k0) >> 5], 1u << (mi & 31));
+        }
+      } else {
+        p = block_radix_select<PairSrc, kSelCNT>(PairSrc{S.ckey, S.cidx}, nc, k2, S.hist, S.sm, 1, p, false);
+        for (int c = tid; c < nc; c += kSelCNT) {
+          const int mi = S.cidx[c];
+          if (mi >= k0 && mi < k0 + per && ge96(p, S.ckey[c], ~(uint32_t)mi)) atomicOr(&sbits[(mi - k0) >> 5], 1u << (mi & 31));
+        }
+      }
+    } else {  // crowded boundary bin: every CTA runs the radix over all keys of the bin, keeps its own
+      p = block_radix_select<GKeySrc, kSelCNT>(GKeySrc{keys}, B, k2, S.hist, S.sm, 1, p, false);
+      for (int i = tid; i < per; i += kSelCNT) {
+        const uint64_t kk = __ldcg(keys + k0 + i);
+        if (((kk >> 51) & 0xFFFu) == (uint32_t)d0 && ge96(p, kk, ~(uint32_t)(k0 + i)))
+          atomicOr(&sbits[i >> 5], 1u << (i & 31));
+      }
+    }
+    __syncthreads();
+  }
+  // my winner count, pushed to every CTA
+  const int wpt = (wpc + kSelCNT - 1) / kSelCNT;
+  int cnt = 0;
+  for (int w = tid * wpt; w < min(wpc, (tid + 1) * wpt); ++w) cnt += __popc(sbits[w]);
+  int mine;
+  int pos = block_excl_scan<kSelCNT>(cnt, &mine, S.sm);
+  if (tid < kSelCL) cl.map_shared_rank(&S, tid)->cnt[r] = mine;
+  cl.sync();
+  if (sel == 0 && r == 0) TRACE(13);
+  // 5. bitmap words and my part of the ascending J
+  int jofs = 0, total = 0;
+#pragma unroll
+  for (int c = 0; c < kSelCL; ++c) {
+    jofs += c < r ? S.cnt[c] : 0;
+    total += S.cnt[c];
+  }
+  uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap) + r * wpc;
+  int* J = reinterpret_cast<int*>(rec + A.lay.off_J);
+  for (int w = tid; w < wpc; w += kSelCNT) bitmap[w] = sbits[w];
+  pos += jofs;
+  for (int w = tid * wpt; w < min(wpc, (tid + 1) * wpt); ++w) {
+    uint32_t bits = sbits[w];
+    while (bits) {
+      const int b = __ffs(bits) - 1;
+      bits &= bits - 1;
+      J[pos++] = k0 + w * 32 + b;
+    }
+  }
+  if (r == 0 && tid == 0) {
+    *reinterpret_cast<int*>(rec + A.lay.off_cnt) = total;
+    if (!A.threshold_mode && total != A.num) atomicOr(A.status + 1, 1);
+  }
+  if (sel == 0 && r == 0) TRACE(14);
+  // (no remote smem access after the last barrier: CTAs may exit)
 }
 
 // ---------------------------------------------------------------------------

@@ -288,7 +288,7 @@ def test_parity_snr_sweep(snr_db):
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("env", [{"CUSFFT_VOTE_PAIRS": "0"}, {"CUSFFT_VOTE_BITMAP": "1"}, {"CUSFFT_SELECT_MULTI": "1"},
+@pytest.mark.parametrize("env", [{"CUSFFT_VOTE_PAIRS": "0"}, {"CUSFFT_VOTE_BITMAP": "1"}, {"CUSFFT_SELECT": "multi"}, {"CUSFFT_SELECT": "single"},
                                  {"CUSFFT_STAGE_MODE": "split_index"}, {"CUSFFT_STAGE_MODE": "fused_scatter"},
                                  {"CUSFFT_STAGE_MODE": "split_scatter"}, {"CUSFFT_NO_STAGE": "1"}])
 def test_kernel_variants_agree(env, monkeypatch):
