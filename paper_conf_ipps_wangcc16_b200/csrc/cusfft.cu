@@ -126,8 +126,10 @@ struct cusfft_plan_s {
   // phase 2's position (coalesced phase 2) instead of in sorted order (read
   // through an index); split = phase 2 is a plain fold (k_fold_staged) followed
   // by the stand-alone FFT pass 1, instead of k_fold_fft1.
-  bool stage_scatter = false;
+  bool stage_scatter = true;   // default: scatter staging + bulk-copy phase 2 (measured fastest)
   bool stage_split = false;
+  bool p2_tma = true;             // scatter phase 2 through bulk copies (k_fold_fft1_tma; CUSFFT_P2=ldg: k_fold_fft1 MODE 2)
+  bool p2_discard = true;         // drop consumed staging lines from L2 (CUSFFT_DISCARD=0: keep)
   int64_t sectors = 0;            // distinct 32-B sectors of x gathered by this rank (the fold's DRAM floor)
   // Slot groups, each with its own sorted schedule (default: one group of all
   // local slots; CUSFFT_STAGE_GROUPS=2 splits location / estimation loops,
@@ -483,6 +485,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   if (const char* e = std::getenv("CUSFFT_VOTE_PAIRS")) P->vote_pairs = !(e[0] == '0');
   // measurement only: skip the staged gather's phase 1 (valid only for a repeated x)
   if (const char* e = std::getenv("CUSFFT_SKIP_STAGE")) P->skip_stage = (e[0] == '1');
+  if (const char* e = std::getenv("CUSFFT_P2")) P->p2_tma = std::string(e) != "ldg";
+  if (const char* e = std::getenv("CUSFFT_DISCARD")) P->p2_discard = (e[0] == '1');
 
   // ---- draws (loop order), Alg. 1, Def. 1
   SplitMix64 rng{q.seed};
@@ -756,6 +760,17 @@ cudaError_t launch_fold_fft1_t(cusfft_plan_t P, const double2* x, const uint32_t
     return launch_k(k_fold_fft1<B1T, 16, 1>, grid, dim3(256), 0, st, P->cur_prio, x, inv,
                     (const double*)P->d_taps_perm, sp, u, v, (const double2*)P->d_tw,
                     (int)P->B, P->B2, P->w, P->R, (uint32_t)(P->n - 1), 0u, (uint32_t)P->n, z);
+  if (staged_tord && P->p2_tma && P->R <= 48) {  // staged in thread order, rows moved by bulk copies
+    const size_t smem = (size_t)P->R * 4096;
+    static thread_local bool attr_set[4] = {false, false, false, false};
+    if (!attr_set[B1T / 64]) {  // static + dynamic smem may exceed the 48 KB default
+      cudaFuncSetAttribute(k_fold_fft1_tma<B1T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+      attr_set[B1T / 64] = true;
+    }
+    return launch_k(k_fold_fft1_tma<B1T>, grid, dim3(256), smem, st, P->cur_prio, x,
+                    (const double*)P->d_taps_perm, u, v, (const double2*)P->d_tw, (int)P->B, P->B2, P->w, P->R,
+                    (int)P->p2_discard, z);
+  }
   if (staged_tord)  // staged in thread order: x is the group's staging buffer
     return launch_k(k_fold_fft1<B1T, 16, 2>, grid, dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)nullptr,
                     (const double*)P->d_taps_perm, sp, u, v, (const double2*)P->d_tw,

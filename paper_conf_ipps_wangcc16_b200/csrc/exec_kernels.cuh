@@ -328,6 +328,86 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict_
 }
 
 // ---------------------------------------------------------------------------
+// Phase 2 of the scatter-staged fold with bulk copies: the
+// CTA's R rows of 256 staged samples (row rr = staging[(s R + rr) B + cta 256
+// ...], 4 KB each, already in this kernel's thread order) are moved to shared
+// memory by the bulk-copy engine onto one mbarrier while the threads fetch
+// their taps, so no gathered sample occupies a register and four CTAs fit per
+// SM.  Then exactly k_fold_fft1's arithmetic: rounds accumulated in Alg. 1's
+// order (fp64 mul + add per component), u written, the C columns' B1-point
+// FFTs in shared memory, v = FFT x omega_B^(c k1).  discard != 0: the consumed
+// staging lines are dropped from L2 without write-back (the next execution
+// rewrites every staged sample that is read).
+// ---------------------------------------------------------------------------
+template <int B1T>
+__global__ void __launch_bounds__(256, 4) k_fold_fft1_tma(const double2* __restrict__ staging,
+                                                          const double* __restrict__ taps_perm,
+                                                          double2* __restrict__ u, double2* __restrict__ v,
+                                                          const double2* __restrict__ tw, int B, int B2, int w, int R,
+                                                          int discard, ZeroArgs zero) {
+  pdl_wait();
+  KTRACE(2);
+  constexpr int C = 256 / B1T;
+  constexpr int RMAX = 16;
+  extern __shared__ __align__(128) double2 Tile[];  // [R][256]
+  __shared__ double2 S[256 + 256 / 8];
+  __shared__ double2 twl[B1T];
+  __shared__ __align__(8) uint64_t bar;
+  const int t = threadIdx.x;
+  const int s = blockIdx.y;
+  if (blockIdx.x == 0 && blockIdx.y == 0) TRACE(0);
+  const double2* src = staging + (int64_t)s * R * B + (int64_t)blockIdx.x * 256;
+  if (t == 0) {
+    mbar_init(&bar, 1);
+    mbar_expect_tx(&bar, (uint32_t)R * 4096u);
+  }
+  __syncthreads();
+  if (t < 32) {
+    const uint64_t pol = l2_policy_first();
+    for (int rr = t; rr < R; rr += 32) bulk_g2s(Tile + rr * 256, src + (int64_t)rr * B, 4096u, &bar, pol);
+  }
+  zero_part(zero);
+  const int cl = t / B1T, j1 = t % B1T;
+  const int c = blockIdx.x * C + cl;
+  const int j = c + B2 * j1;
+  for (int i = t; i < B1T; i += 256) twl[i] = __ldg(tw + (int64_t)i * B2);  // omega_B1^i
+  const double* tp = taps_perm + (int64_t)blockIdx.x * 256 + t;
+  double g[RMAX];
+#pragma unroll
+  for (int rr = 0; rr < RMAX; ++rr) g[rr] = (rr < R && j + rr * B < w) ? __ldg(tp + (int64_t)rr * B) : 0.0;
+  mbar_wait(&bar, 0);
+  double ar = 0.0, ai = 0.0;
+#pragma unroll
+  for (int rr = 0; rr < RMAX; ++rr) {
+    if (rr < R && j + rr * B < w) {
+      const double2 q = Tile[rr * 256 + t];
+      ar = __dadd_rn(ar, __dmul_rn(g[rr], q.x));
+      ai = __dadd_rn(ai, __dmul_rn(g[rr], q.y));
+    }
+  }
+  for (int rr = RMAX; rr < R; ++rr) {  // R > 16 (small tolerance / Gaussian filters)
+    if (j + rr * B < w) {
+      const double2 q = Tile[rr * 256 + t];
+      const double gg = __ldg(tp + (int64_t)rr * B);
+      ar = __dadd_rn(ar, __dmul_rn(gg, q.x));
+      ai = __dadd_rn(ai, __dmul_rn(gg, q.y));
+    }
+  }
+  if (discard)
+    for (int q = t; q < R * 32; q += 256) l2_discard(src + (int64_t)(q >> 5) * B + (q & 31) * 8);
+  S[fft_pad(cl * B1T + j1)] = make_double2(ar, ai);
+  __syncthreads();
+  const int wc = t % C, wj = t / C;
+  const size_t wpos = (size_t)s * B + (size_t)blockIdx.x * C + wc + (size_t)B2 * wj;
+  u[wpos] = S[fft_pad(wc * B1T + wj)];
+  __syncthreads();
+  fft_smem<B1T, 256, 256, true>(S, twl, B1T);
+  const double2 wv = __ldg(tw + (((int64_t)(blockIdx.x * C + wc) * wj) & (B - 1)));
+  v[wpos] = cmul(S[fft_pad(wc * B1T + wj)], wv);
+  TRACE_END(1);
+}
+
+// ---------------------------------------------------------------------------
 // Record layout of one slot in the exchange buffer:
 //   [u^ : B x double2][bitmap : B/32 x u32][count : int32][J : Jcap x int32],
 //   256-B aligned; Jcap = num (B in THRESHOLD mode).
