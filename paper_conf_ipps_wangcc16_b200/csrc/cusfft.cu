@@ -130,6 +130,10 @@ struct cusfft_plan_s {
   bool stage_split = false;
   bool p2_tma = true;             // scatter phase 2 through bulk copies (k_fold_fft1_tma; CUSFFT_P2=ldg: k_fold_fft1 MODE 2)
   bool p2_discard = true;         // drop consumed staging lines from L2 (CUSFFT_DISCARD=0: keep)
+  bool slot_fused = false;        // FFT pass 2 (+ fold) + cutoff in one cluster kernel per slot (k_slot; CUSFFT_SLOT=1|2)
+  bool slot_select = false;       // k_slot also runs the cutoff (cluster selection)
+  bool slot_phase_a = false;      // k_slot also folds (phase A, CUSFFT_SLOT=2); default: after k_fold_fft1_tma
+  int slot_smem = 0;
   int64_t sectors = 0;            // distinct 32-B sectors of x gathered by this rank (the fold's DRAM floor)
   // Slot groups, each with its own sorted schedule (default: one group of all
   // local slots; CUSFFT_STAGE_GROUPS=2 splits location / estimation loops,
@@ -140,6 +144,7 @@ struct cusfft_plan_s {
     uint32_t* spos = nullptr;    // [total] sorted gather positions
     uint32_t* inv = nullptr;     // [s1 - s0][R][B] staging index in the fused kernel's thread order (index mode)
     uint32_t* dst = nullptr;     // [total] thread-order staging position of sorted gather q (scatter mode)
+    double2* staging = nullptr;  // this group's staging buffer (groups share one unless branched)
   };
   std::vector<StageGroup> groups;
   double2* d_staging = nullptr;   // [max group total]
@@ -188,6 +193,7 @@ struct cusfft_plan_s {
   bool use_graph = true;
   bool branched = false;          // two-branch graph (location chain || estimation folds); opt-in
   bool skip_stage = false;        // measurement only (CUSFFT_SKIP_STAGE)
+  int stage_cps = 8;              // k_stage CTAs per SM (CUSFFT_STAGE_CPS; branched default 2: room for the chain)
   int nloc_local = 0;             // local slots [0, nloc_local) are location loops
   cudaStream_t cap_stream = nullptr, cap_stream2 = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
@@ -205,6 +211,12 @@ struct cusfft_plan_s {
 namespace {
 
 bool valid_plan(cusfft_plan_t p) { return p && p->magic == kMagic; }
+
+// B1 x B2 splits with a k_slot instantiation
+bool slot_shape_ok(int B1, int B2) {
+  return (B1 == 64 && (B2 == 32 || B2 == 64)) || (B1 == 128 && (B2 == 64 || B2 == 128)) ||
+         (B1 == 256 && (B2 == 128 || B2 == 256));
+}
 
 struct DeviceGuard {
   int prev = -1;
@@ -485,6 +497,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   if (const char* e = std::getenv("CUSFFT_VOTE_PAIRS")) P->vote_pairs = !(e[0] == '0');
   // measurement only: skip the staged gather's phase 1 (valid only for a repeated x)
   if (const char* e = std::getenv("CUSFFT_SKIP_STAGE")) P->skip_stage = (e[0] == '1');
+  if (P->branched) P->stage_cps = 2;
+  if (const char* e = std::getenv("CUSFFT_STAGE_CPS")) P->stage_cps = std::max(1, std::atoi(e));
   if (const char* e = std::getenv("CUSFFT_P2")) P->p2_tma = std::string(e) != "ldg";
   if (const char* e = std::getenv("CUSFFT_DISCARD")) P->p2_discard = (e[0] == '1');
 
@@ -665,7 +679,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     const char* e = std::getenv("CUSFFT_NO_STAGE");
     const char* eg = std::getenv("CUSFFT_STAGE_GROUPS");
     std::vector<std::pair<int, int>> ranges;
-    if (P->nloc_local > 0 && P->nloc_local < P->Lg && eg && eg[0] == '2')  // opt-in: two groups
+    // two groups (location / estimation slots): opt-in, and always for the branched graph
+    if (P->nloc_local > 0 && P->nloc_local < P->Lg && ((eg && eg[0] == '2') || P->branched))
       ranges = {{0, P->nloc_local}, {P->nloc_local, P->Lg}};
     else
       ranges = {{0, P->Lg}};
@@ -674,9 +689,13 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       P->stage_split = m.rfind("split", 0) == 0;
       P->stage_scatter = m.find("scatter") != std::string::npos;
     }
-    int64_t maxtot = 0;  // staging elements: w per slot (index mode) or R B per slot (scatter mode)
-    for (auto& r : ranges)
-      maxtot = std::max<int64_t>(maxtot, (int64_t)(r.second - r.first) * (P->stage_scatter ? P->R * B : P->w));
+    int64_t maxtot = 0, sumtot = 0;  // staging elements: w per slot (index mode) or R B per slot (scatter mode)
+    for (auto& r : ranges) {
+      const int64_t t = (int64_t)(r.second - r.first) * (P->stage_scatter ? P->R * B : P->w);
+      maxtot = std::max<int64_t>(maxtot, t);
+      sumtot += t;
+    }
+    if (P->branched) maxtot = sumtot;  // concurrent groups: one staging buffer each
     // the staging buffer must be (mostly) L2-resident between the two phases
     // (the staging schedule gathers from the whole signal: not for signal-sharded plans)
     P->staged = P->fused1 && !P->xshard && maxtot * 16 <= (int64_t)64 << 20 && !(e && e[0] == '1');
@@ -729,6 +748,13 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
         }
       }
       if ((rc = dalloc(&P->d_staging, (size_t)maxtot))) return fail(rc);
+      {
+        int64_t off = 0;
+        for (auto& g : P->groups) {
+          g.staging = P->d_staging + off;
+          if (P->branched) off += (g.s1 - g.s0) * (P->stage_scatter ? (int64_t)P->R * B : (int64_t)P->w);
+        }
+      }
       // Persisting-L2 set-aside for the staging buffer (a device-wide limit: raised, never lowered).
       int maxp = 0;
       cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev);
@@ -744,12 +770,49 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       P->stage_window.missProp = cudaAccessPropertyStreaming;
     }
   }
+  {  // fused slot kernel (k_slot): scatter-staged plans whose B1 x B2 split has an instantiation
+    const char* e = std::getenv("CUSFFT_SLOT");
+    const bool shape = slot_shape_ok(P->B1, P->B2);
+    P->slot_smem = shape ? slot_smem_bytes(P->B1, P->B2, P->R) : 0;
+    // opt-in (CUSFFT_SLOT=1: FFT pass 2 + cutoff fused; 2: also the fold): measured no faster
+    // than the separate kernels on B200, kept for the A/B
+    P->slot_phase_a = e && e[0] == '2';
+    P->slot_fused = P->staged && P->stage_scatter && !P->stage_split && shape &&
+                    (!P->slot_phase_a || P->slot_smem <= 220 * 1024) && e && (e[0] == '1' || e[0] == '2');
+    P->slot_select = P->slot_fused && P->sel_cluster && !P->sel_slots_h.empty();
+  }
   if (cudaStreamSynchronize(P->stream) != cudaSuccess) {
     g_last_cuda_error = (int)cudaGetLastError();
     return fail(CUSFFT_CUDA);
   }
   *out = P;
   return CUSFFT_SUCCESS;
+}
+
+template <int B1T, int B2T, bool FV>
+cudaError_t launch_slot_t(cusfft_plan_t P, const SlotArgs& a, int nslots, cudaStream_t st) {
+  static thread_local bool attr_set = false;
+  if (!attr_set) {
+    cudaFuncSetAttribute(k_slot<B1T, B2T, FV>, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    attr_set = true;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(nslots * kSlotCS));
+  cfg.blockDim = dim3(256);
+  cfg.dynamicSmemBytes = FV ? (size_t)slot_smem_bytes_v(B1T, B2T) : (size_t)P->slot_smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[3];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = kSlotCS;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = g_pdl ? 1 : 0;
+  attr[2].id = cudaLaunchAttributePriority;
+  attr[2].val.priority = P->cur_prio;
+  cfg.attrs = attr;
+  cfg.numAttrs = 3;
+  return cudaLaunchKernelEx(&cfg, k_slot<B1T, B2T, FV>, a);
 }
 
 template <int B1T>
@@ -794,6 +857,84 @@ inline void mark(cusfft_plan_t P, int i) {
   if (P->timing) cudaEventRecord(P->ev[i], P->stream);
 }
 
+// Staged fold, phase 1: address-sorted gather of the group's samples into its staging buffer.
+int launch_stage1(cusfft_plan_t P, const cusfft_plan_s::StageGroup& g, const double2* x, cudaStream_t st, ZeroArgs z) {
+  if (P->skip_stage) return CUSFFT_SUCCESS;
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, P->device);
+  const int tot = (int)g.total;
+  const int grid = std::max(1, std::min((tot + 8 * 256 - 1) / (8 * 256), sms * P->stage_cps));
+  g_apw = P->stage_window;  // keep the staging buffer L2-resident for phase 2
+  const cudaError_t e = launch_k(k_stage, dim3(grid), dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)g.spos,
+                                 (const uint32_t*)g.dst, g.staging, tot, z);
+  g_apw = cudaAccessPolicyWindow{};
+  CK(e);
+  return CUSFFT_SUCCESS;
+}
+
+// Staged fold, phase 2: the fold (+ FFT pass 1) of the group's slots from its staging buffer.
+int launch_stage2(cusfft_plan_t P, const cusfft_plan_s::StageGroup& g, cudaStream_t st, ZeroArgs z) {
+  const int B = (int)P->B;
+  g_pdl = !P->timing;
+  cudaError_t e;
+  if (P->stage_split) {
+    dim3 grid2((unsigned)(B / 256), (unsigned)(g.s1 - g.s0));
+    if (g.dst)
+      e = launch_k(k_fold_staged<true>, grid2, dim3(256), 0, st, P->cur_prio, (const double2*)g.staging,
+                   (const uint32_t*)nullptr, (const double*)P->d_taps, P->d_u + (size_t)g.s0 * B, B, P->w, P->R, z);
+    else
+      e = launch_k(k_fold_staged<false>, grid2, dim3(256), 0, st, P->cur_prio, (const double2*)g.staging,
+                   (const uint32_t*)g.inv, (const double*)P->d_taps, P->d_u + (size_t)g.s0 * B, B, P->w, P->R, z);
+  } else {
+    e = launch_fold_fft1(P, g.staging, g.inv, P->d_slots + (size_t)P->lrank * P->Lg + g.s0,
+                         P->d_u + (size_t)g.s0 * B, P->d_v + (size_t)g.s0 * B, g.s1 - g.s0, z, st, g.dst != nullptr);
+  }
+  CK(e);
+  return CUSFFT_SUCCESS;
+}
+
+SelArgs make_sel_args(cusfft_plan_t P);
+
+// Steps 2-4 of a staged group in the fused cluster kernel (do_select: with the cutoff).
+int launch_slot(cusfft_plan_t P, const cusfft_plan_s::StageGroup& g, cudaStream_t st, bool do_select) {
+  const int B = (int)P->B;
+  SlotArgs a{};
+  a.staging = g.staging;
+  a.taps_perm = P->d_taps_perm;
+  a.u = P->d_u + (size_t)g.s0 * B;
+  a.recs = P->d_records + ((int64_t)P->lrank * P->Lg + g.s0) * P->lay.rec_bytes;
+  a.rec_bytes = P->lay.rec_bytes;
+  a.tw = P->d_tw;
+  a.key_index = P->sel_slots_h.empty() ? nullptr : P->d_key_index + g.s0;
+  a.keys = P->d_keys;
+  a.hist = P->d_hist;
+  a.B = B;
+  a.w = P->w;
+  a.R = P->R;
+  a.discard = P->p2_discard ? 1 : 0;
+  a.do_select = do_select ? 1 : 0;
+  a.sel = make_sel_args(P);
+  g_pdl = !P->timing;
+  const int ns = g.s1 - g.s0;
+  cudaError_t e = cudaErrorInvalidValue;
+  const bool fv = !P->slot_phase_a;
+  a.v = P->d_v + (size_t)g.s0 * B;
+  switch (P->B1 * 1000 + P->B2) {
+#define SLOT_CASE(b1, b2) \
+  case b1 * 1000 + b2: e = fv ? launch_slot_t<b1, b2, true>(P, a, ns, st) : launch_slot_t<b1, b2, false>(P, a, ns, st); break;
+    SLOT_CASE(64, 32)
+    SLOT_CASE(64, 64)
+    SLOT_CASE(128, 64)
+    SLOT_CASE(128, 128)
+    SLOT_CASE(256, 128)
+    SLOT_CASE(256, 256)
+#undef SLOT_CASE
+    default: break;
+  }
+  CK(e);
+  return CUSFFT_SUCCESS;
+}
+
 // Steps 1+2 (and the fused FFT pass 1) for this rank's local slots [s0, s1).
 // zero_block: this launch also zeroes the per-execution block (first fold only).
 int launch_fold(cusfft_plan_t P, const double2* x, int s0, int s1, cudaStream_t st, bool zero_block) {
@@ -802,34 +943,12 @@ int launch_fold(cusfft_plan_t P, const double2* x, int s0, int s1, cudaStream_t 
   const SlotParam* sp = P->d_slots + (size_t)P->lrank * P->Lg + s0;
   ZeroArgs z{zero_block ? P->d_zero : nullptr, zero_block ? P->nzero : 0};
   if (P->staged) {  // per slot group: phase 1 (address-sorted gather into staging), phase 2 (fused fold)
-    int sms = 148;
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, P->device);
     for (const auto& g : P->groups) {
       if (g.s1 <= s0 || g.s0 >= s1) continue;  // callers pass whole groups
-      const int tot = (int)g.total;
-      g_apw = P->stage_window;  // keep the staging buffer L2-resident for phase 2
-      const int grid = std::max(1, std::min((tot + 8 * 256 - 1) / (8 * 256), sms * 8));
-      cudaError_t e = cudaSuccess;
-      if (!P->skip_stage) {
-        e = launch_k(k_stage, dim3(grid), dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)g.spos,
-                     (const uint32_t*)g.dst, P->d_staging, tot, z);
-        z = ZeroArgs{nullptr, 0};
-      }
-      g_pdl = !P->timing;
-      if (e == cudaSuccess && P->stage_split) {
-        dim3 grid2((unsigned)(B / 256), (unsigned)(g.s1 - g.s0));
-        if (g.dst)
-          e = launch_k(k_fold_staged<true>, grid2, dim3(256), 0, st, P->cur_prio, (const double2*)P->d_staging,
-                       (const uint32_t*)nullptr, (const double*)P->d_taps, P->d_u + (size_t)g.s0 * B, B, P->w, P->R, z);
-        else
-          e = launch_k(k_fold_staged<false>, grid2, dim3(256), 0, st, P->cur_prio, (const double2*)P->d_staging,
-                       (const uint32_t*)g.inv, (const double*)P->d_taps, P->d_u + (size_t)g.s0 * B, B, P->w, P->R, z);
-      } else if (e == cudaSuccess)
-        e = launch_fold_fft1(P, P->d_staging, g.inv, P->d_slots + (size_t)P->lrank * P->Lg + g.s0,
-                             P->d_u + (size_t)g.s0 * B, P->d_v + (size_t)g.s0 * B, g.s1 - g.s0, z, st,
-                             g.dst != nullptr);
-      g_apw = cudaAccessPolicyWindow{};
-      CK(e);
+      int rc;
+      if ((rc = launch_stage1(P, g, x, st, z))) return rc;
+      if (!P->skip_stage) z = ZeroArgs{nullptr, 0};
+      if ((rc = launch_stage2(P, g, st, z))) return rc;
     }
   } else if (P->fused1) {
     CK(launch_fold_fft1(P, x, nullptr, sp, P->d_u + (size_t)s0 * B, P->d_v + (size_t)s0 * B, s1 - s0, z, st));
@@ -869,8 +988,7 @@ int launch_bfft(cusfft_plan_t P, int s0, int s1, cudaStream_t st) {
 }
 
 // Step 4 for this rank's location slots.
-int launch_select(cusfft_plan_t P, cudaStream_t st) {
-  if (P->sel_slots_h.empty()) return CUSFFT_SUCCESS;
+SelArgs make_sel_args(cusfft_plan_t P) {
   SelArgs sa{};
   for (size_t i = 0; i < P->sel_slots_h.size(); ++i)
     sa.recs[i] = P->d_records + (int64_t)P->sel_slots_h[i] * P->lay.rec_bytes;
@@ -893,6 +1011,12 @@ int launch_select(cusfft_plan_t P, cudaStream_t st) {
     std::memcpy(&bits, &th, 8);
     sa.thr_key = bits;
   }
+  return sa;
+}
+
+int launch_select(cusfft_plan_t P, cudaStream_t st) {
+  if (P->sel_slots_h.empty()) return CUSFFT_SUCCESS;
+  const SelArgs sa = make_sel_args(P);
   if (P->prm.cutoff_mode == CUSFFT_CUTOFF_SORT) {
     const int smem = (int)P->B * 12 + (int)((P->B + 31) / 32) * 4;
     CK(launch_k(k_select_sort, dim3((int)P->sel_slots_h.size()), dim3(1024), smem, st, P->cur_prio, sa));
@@ -948,6 +1072,25 @@ int launch_local(cusfft_plan_t P, const double2* x) {
   int rc;
   mark(P, 0);
   g_pdl = false;  // the first kernel follows arbitrary caller work
+  if (P->slot_fused) {  // phase 1 per group, then one cluster kernel per group for steps 2-4
+    ZeroArgs z{P->d_zero, P->nzero};
+    for (const auto& g : P->groups) {  // stage 1 "fold": phase 1 (+ phase 2 unless k_slot folds)
+      if ((rc = launch_stage1(P, g, x, st, z))) return rc;
+      z = ZeroArgs{nullptr, 0};
+      g_pdl = !P->timing;
+      if (!P->slot_phase_a && (rc = launch_stage2(P, g, st, z))) return rc;
+    }
+    mark(P, 1);
+    if (P->stage_limit < 2) return CUSFFT_SUCCESS;
+    const bool sel = P->slot_select && P->stage_limit >= 3 && !P->xshard;
+    for (const auto& g : P->groups)
+      if ((rc = launch_slot(P, g, st, sel))) return rc;
+    mark(P, 2);
+    if (P->stage_limit < 3 || P->xshard) return CUSFFT_SUCCESS;
+    if (!sel && (rc = launch_select(P, st))) return rc;
+    mark(P, 3);
+    return CUSFFT_SUCCESS;
+  }
   rc = launch_fold(P, x, 0, P->Lg, st, true);
   g_pdl = !P->timing;
   if (rc) return rc;
@@ -1075,11 +1218,45 @@ int launch_branched(cusfft_plan_t P, const double2* x, int64_t* locs, double2* v
   return launch_output(P, locs, vals, a);
 }
 
+// Staged variant of the two-branch graph: the location group's phase 1 runs
+// alone; then the estimation group's phase 1 (DRAM-bound, k_stage at
+// stage_cps CTAs per SM) overlaps the location chain (phase 2, FFT, cutoff,
+// vote: L2/latency-bound) on the high-priority stream; the estimation group's
+// phase 2 and FFT follow on the second stream and join before the estimation.
+int launch_branched_staged(cusfft_plan_t P, const double2* x, int64_t* locs, double2* vals) {
+  cudaStream_t a = P->stream, b = P->cap_stream2;
+  const auto& gl = P->groups[0];
+  const auto& ge = P->groups[1];
+  int rc;
+  P->cur_prio = P->prio_hi;
+  g_pdl = false;
+  if ((rc = launch_stage1(P, gl, x, a, ZeroArgs{P->d_zero, P->nzero}))) return rc;
+  CK(cudaEventRecord(P->ev_fork, a));
+  CK(cudaStreamWaitEvent(b, P->ev_fork, 0));
+  P->cur_prio = P->prio_lo;
+  g_pdl = false;
+  if ((rc = launch_stage1(P, ge, x, b, ZeroArgs{nullptr, 0}))) return rc;
+  if ((rc = launch_stage2(P, ge, b, ZeroArgs{nullptr, 0}))) return rc;
+  if ((rc = launch_bfft(P, ge.s0, ge.s1, b))) return rc;
+  CK(cudaEventRecord(P->ev_join, b));
+  P->cur_prio = P->prio_hi;
+  if ((rc = launch_stage2(P, gl, a, ZeroArgs{nullptr, 0}))) return rc;
+  if ((rc = launch_bfft(P, gl.s0, gl.s1, a))) return rc;
+  if ((rc = launch_select(P, a))) return rc;
+  if ((rc = launch_vote(P, a))) return rc;
+  P->cur_prio = 0;
+  CK(cudaStreamWaitEvent(a, P->ev_join, 0));
+  g_pdl = false;
+  if ((rc = launch_estimate(P, a))) return rc;
+  g_pdl = !P->timing;
+  return launch_output(P, locs, vals, a);
+}
+
 // Branched execution only inside graph capture, for full-stage runs with both
 // location and estimation-only slots on this rank.
 inline bool use_branches(cusfft_plan_t P) {
-  return !P->staged && P->branched && P->use_graph && !P->timing && P->stage_limit == 6 && P->nloc_local > 0 &&
-         P->nloc_local < P->Lg;
+  return P->branched && !P->slot_fused && P->use_graph && !P->timing && P->stage_limit == 6 && P->nloc_local > 0 &&
+         P->nloc_local < P->Lg && (!P->staged || (P->groups.size() == 2 && !P->stage_split && !P->skip_stage));
 }
 
 // Run `body` (which enqueues on P->stream) either directly or through a cached
@@ -1240,7 +1417,8 @@ int cusfft_execute(cusfft_plan_t plan, const void* d_x, int64_t* d_locs, void* d
   return run_graphed(plan, plan->g_full, plan->g_full_t, d_x, d_locs, d_vals, [&] {
     const double2* x = reinterpret_cast<const double2*>(d_x);
     double2* v = reinterpret_cast<double2*>(d_vals);
-    if (use_branches(plan)) return launch_branched(plan, x, d_locs, v);
+    if (use_branches(plan))
+      return plan->staged ? launch_branched_staged(plan, x, d_locs, v) : launch_branched(plan, x, d_locs, v);
     int rc = launch_local(plan, x);
     if (rc) return rc;
     return launch_finish(plan, d_locs, v);
@@ -1272,7 +1450,9 @@ int cusfft_execute_host(cusfft_plan_t plan, const void* h_x, int64_t* h_locs, vo
   cudaStream_t st = plan->stream;
   CK(cudaMemcpyAsync(plan->d_xbuf, h_x, (size_t)plan->n * 16, cudaMemcpyHostToDevice, st));
   rc = run_graphed(plan, plan->g_full, plan->g_full_t, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf, [&] {
-    if (use_branches(plan)) return launch_branched(plan, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf);
+    if (use_branches(plan))
+      return plan->staged ? launch_branched_staged(plan, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf)
+                          : launch_branched(plan, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf);
     int r = launch_local(plan, plan->d_xbuf);
     if (r) return r;
     return launch_finish(plan, plan->d_locs_buf, plan->d_vals_buf);

@@ -947,17 +947,17 @@ struct SelClusterSmem {
   int cnt[kSelCL];              // final winners per CTA (pushed to every CTA)
 };
 
-__global__ void __launch_bounds__(kSelCNT, 1) k_select_cluster(SelArgs A) {
-  pdl_wait();
-  KTRACE(8);
+// The cluster selection of location slot `sel` by the calling cluster of kSelCL
+// CTAs x kSelCNT threads; smem: sizeof(SelClusterSmem) + B / kSelCL / 8 bytes.
+// Reads keys and histograms through L2 (__ldcg): they may have been written by
+// other CTAs of the cluster in the same kernel (k_slot), before a cluster barrier.
+__device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, uint8_t* smem) {
   namespace cg = cooperative_groups;
   cg::cluster_group cl = cg::this_cluster();
-  extern __shared__ __align__(16) uint8_t smem[];
   SelClusterSmem& S = *reinterpret_cast<SelClusterSmem*>(smem);
   uint32_t* sbits = reinterpret_cast<uint32_t*>(smem + sizeof(SelClusterSmem));  // this CTA's words
   const int tid = threadIdx.x, lane = tid & 31;
   const int r = (int)cl.block_rank();
-  const int sel = blockIdx.x / kSelCL;
   const int B = A.B;
   const int per = B / kSelCL;           // keys per CTA (multiple of 32)
   const int wpc = per >> 5;             // words per CTA
@@ -972,14 +972,14 @@ __global__ void __launch_bounds__(kSelCNT, 1) k_select_cluster(SelArgs A) {
   const int hbase = r * BPC + BPC - 1 - 2 * tid;
   int c0 = 0, c1 = 0;
   if (!A.threshold_mode) {
-    c0 = (int)__ldg(h0 + hbase);
-    c1 = (int)__ldg(h0 + hbase - 1);
+    c0 = (int)__ldcg(h0 + hbase);
+    c1 = (int)__ldcg(h0 + hbase - 1);
   }
   uint64_t kb[KC];
 #pragma unroll
   for (int u = 0; u < KC; ++u) {
     const int i = u * kSelCNT + tid;
-    kb[u] = i < per ? __ldg(keys + k0 + i) : 0ull;
+    kb[u] = i < per ? __ldcg(keys + k0 + i) : 0ull;
   }
   if (r == 0 && tid == 0) S.ncand = 0;
   // 1. slice totals, pushed to every CTA of the cluster
@@ -1025,7 +1025,7 @@ __global__ void __launch_bounds__(kSelCNT, 1) k_select_cluster(SelArgs A) {
 #pragma unroll
       for (int u = 0; u < KC; ++u) {
         const int i = cb + u * kSelCNT + tid;
-        kb[u] = i < per ? __ldg(keys + k0 + i) : 0ull;
+        kb[u] = i < per ? __ldcg(keys + k0 + i) : 0ull;
       }
     }
 #pragma unroll
@@ -1125,6 +1125,215 @@ __global__ void __launch_bounds__(kSelCNT, 1) k_select_cluster(SelArgs A) {
   }
   if (sel == 0 && r == 0) TRACE(14);
   // (no remote smem access after the last barrier: CTAs may exit)
+}
+
+__global__ void __launch_bounds__(kSelCNT, 1) k_select_cluster(SelArgs A) {
+  pdl_wait();
+  KTRACE(8);
+  extern __shared__ __align__(16) uint8_t smem[];
+  select_cluster_body(A, blockIdx.x / kSelCL, smem);
+}
+
+// ---------------------------------------------------------------------------
+// Steps 2-4 of one slot in ONE cluster of kSlotCS CTAs, after
+// the scatter-staged phase 1 (k_stage).  B = B1 x B2, CTA r of the cluster
+// owns columns c in [r COLS, (r+1) COLS) (COLS = B2 / kSlotCS) and pass-2
+// rows k1 in [r ROWS, (r+1) ROWS) (ROWS = B1 / kSlotCS):
+//   A. fold + FFT pass 1: its TPC tiles of 256 buckets (C = 256 / B1 columns
+//      x B1 rows each) stream from the staging buffer through shared memory
+//      (bulk copies, two buffers on two mbarriers); per tile exactly
+//      k_fold_fft1_tma's arithmetic (Alg. 1 round order, B1-point FFTs),
+//      u written to global, V[c][k1] = FFT x omega_B^(c k1) kept in smem.
+//   B. cluster barrier; pass 2: row k1 gathers V[c][k1] of all B2 columns
+//      from the owners' shared memory (DSMEM), B2-point FFTs (k_fft's
+//      arithmetic), u^[k1 + B1 k2] to the slot's record, cutoff keys and the
+//      top-digit histogram (location slots).
+//   C. location slots (do_select): cluster barrier, then the cluster
+//      selection (select_cluster_body, same result as k_select_cluster).
+// Replaces k_fold_fft1_tma + k_fft pass 2 + k_select: two launches and the
+// spill of V through L2 disappear.
+// ---------------------------------------------------------------------------
+constexpr int kSlotCS = 8;  // CTAs per cluster (= kSelCL: phase C reuses the cluster selection)
+static_assert(kSlotCS == kSelCL, "slot cluster must match the selection cluster");
+
+struct SlotArgs {
+  const double2* v;         // FROM_V: FFT pass-1 output v[s][c + B2 k1] (k_fold_fft1*), else unused
+  const double2* staging;   // group staging, scatter layout [(s R + rr) B + tile 256 + t]
+  const double* taps_perm;  // [R][B] tile-contiguous taps
+  double2* u;               // [ns][B] (group slot 0)
+  uint8_t* recs;            // record of group slot 0
+  int64_t rec_bytes;
+  const double2* tw;        // e^{-2 pi i t / B}, t < B
+  const int* key_index;     // [ns] selection index of each group slot or -1
+  uint64_t* keys;           // [n_sel][B]
+  uint32_t* hist;           // [n_sel][4096]
+  int B, w, R, discard, do_select;
+  SelArgs sel;
+};
+
+__host__ __device__ constexpr int slot_max3(int a, int b, int c) { return a > b ? (a > c ? a : c) : (b > c ? b : c); }
+__host__ __device__ constexpr int slot_smem_bytes(int B1, int B2, int R) {
+  // V (padded FFT layout) + max(phase A: 2 tiles + twl, phase B: S2 + twl2 + hist, phase C: selection) + 2 mbarriers
+  return ((B1 * B2 / kSlotCS) + (B1 * B2 / kSlotCS) / 8) * 16 +
+         slot_max3(2 * R * 256 * 16 + B1 * 16, ((B1 * B2 / kSlotCS) + (B1 * B2 / kSlotCS) / 8) * 16 + B2 * 16 + 4096 * 4,
+                   (int)sizeof(SelClusterSmem) + 1024) +
+         16;
+}
+
+__host__ __device__ constexpr int slot_smem_bytes_v(int B1, int B2) {
+  // FROM_V: no V region; max(phase B, phase C)
+  return slot_max3(0, ((B1 * B2 / kSlotCS) + (B1 * B2 / kSlotCS) / 8) * 16 + B2 * 16 + 4096 * 4,
+                   (int)sizeof(SelClusterSmem) + 1024);
+}
+
+// FROM_V: phase A was done by k_fold_fft1_tma (v in global, L2-resident);
+// the kernel is then FFT pass 2 + keys + the cluster cutoff (k_fft + k_select).
+template <int B1T, int B2T, bool FROM_V>
+__global__ void __launch_bounds__(256, 1) k_slot(SlotArgs A) {
+  pdl_wait();
+  KTRACE(2);
+  namespace cg = cooperative_groups;
+  cg::cluster_group cl = cg::this_cluster();
+  constexpr int C = 256 / B1T;
+  constexpr int COLS = B2T / kSlotCS;
+  constexpr int TPC = COLS / C;
+  constexpr int ROWS = B1T / kSlotCS;
+  constexpr int E2 = ROWS * B2T;  // == COLS * B1T
+  static_assert(TPC >= 1 && COLS % C == 0 && ROWS >= 1 && E2 >= 256, "slot kernel shape");
+  extern __shared__ __align__(16) uint8_t smem[];
+  double2* V = reinterpret_cast<double2*>(smem);                    // [COLS][B1T], fft_pad layout
+  uint8_t* X = FROM_V ? smem : smem + (E2 + E2 / 8) * 16;           // phase-dependent region
+  const int B = A.B, R = A.R, w = A.w;
+  const int t = threadIdx.x;
+  const int r = (int)cl.block_rank();
+  const int s = blockIdx.x / kSlotCS;
+  if (blockIdx.x == 0) TRACE(0);
+  if constexpr (!FROM_V) {
+  // ---- phase A: fold the CTA's TPC tiles into V (sequence = local column, element = row j1)
+  double2* Tile = reinterpret_cast<double2*>(X);                     // [2][R][256]
+  double2* twl = Tile + 2 * R * 256;                                // [B1T]
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + slot_smem_bytes(B1T, B2T, R) - 16);
+  const double2* src0 = A.staging + (int64_t)s * R * B + (int64_t)r * TPC * 256;
+  auto issue = [&](int tl) {  // thread 0: the R rows of tile tl into buffer tl & 1
+    uint64_t* b = bar + (tl & 1);
+    mbar_expect_tx(b, (uint32_t)R * 4096u);
+    const uint64_t pol = l2_policy_first();
+    for (int rr = 0; rr < R; ++rr)
+      bulk_g2s(Tile + ((tl & 1) * R + rr) * 256, src0 + (int64_t)rr * B + tl * 256, 4096u, b, pol);
+  };
+  if (t == 0) {
+    mbar_init(bar, 1);
+    mbar_init(bar + 1, 1);
+  }
+  __syncthreads();
+  if (t == 0) {
+    issue(0);
+    if (TPC > 1) issue(1);
+  }
+  for (int i = t; i < B1T; i += 256) twl[i] = __ldg(A.tw + (int64_t)i * B2T);  // omega_B1^i
+  const int cl_ = t / B1T, j1 = t % B1T;
+  constexpr int RMAX = 16;
+#pragma unroll 1
+  for (int tl = 0; tl < TPC; ++tl) {
+    const int cta = r * TPC + tl;  // tile index within the slot (k_fold_fft1's blockIdx.x)
+    const int j = cta * C + cl_ + B2T * j1;
+    const double* tp = A.taps_perm + (int64_t)cta * 256 + t;
+    double g[RMAX];
+#pragma unroll
+    for (int rr = 0; rr < RMAX; ++rr) g[rr] = (rr < R && j + rr * B < w) ? __ldg(tp + (int64_t)rr * B) : 0.0;
+    mbar_wait(bar + (tl & 1), (uint32_t)((tl >> 1) & 1));
+    const double2* T = Tile + (tl & 1) * R * 256;
+    double ar = 0.0, ai = 0.0;
+#pragma unroll
+    for (int rr = 0; rr < RMAX; ++rr) {
+      if (rr < R && j + rr * B < w) {
+        const double2 q = T[rr * 256 + t];
+        ar = __dadd_rn(ar, __dmul_rn(g[rr], q.x));
+        ai = __dadd_rn(ai, __dmul_rn(g[rr], q.y));
+      }
+    }
+    for (int rr = RMAX; rr < R; ++rr) {
+      if (j + rr * B < w) {
+        const double2 q = T[rr * 256 + t];
+        const double gg = __ldg(tp + (int64_t)rr * B);
+        ar = __dadd_rn(ar, __dmul_rn(gg, q.x));
+        ai = __dadd_rn(ai, __dmul_rn(gg, q.y));
+      }
+    }
+    if (A.discard)
+      for (int q = t; q < R * 32; q += 256) l2_discard(src0 + (int64_t)(q >> 5) * B + tl * 256 + (q & 31) * 8);
+    V[fft_pad((tl * C + cl_) * B1T + j1)] = make_double2(ar, ai);
+    __syncthreads();  // buffer (tl & 1) consumed: refill it with tile tl + 2
+    if (t == 0 && tl + 2 < TPC) issue(tl + 2);
+  }
+  // u (kept for parity checks): runs of COLS consecutive columns per row j1
+  for (int e = t; e < E2; e += 256) {
+    const int cc = e % COLS, jj = e / COLS;
+    A.u[(size_t)s * B + (size_t)r * COLS + cc + (size_t)B2T * jj] = V[fft_pad(cc * B1T + jj)];
+  }
+  fft_smem<B1T, E2, 256, true>(V, twl, B1T);  // the COLS columns' B1-point FFTs (syncs inside)
+  for (int e = t; e < E2; e += 256) {          // twiddle omega_B^(c k1)
+    const int cc = e / B1T, k1 = e % B1T;
+    const int cg_ = r * COLS + cc;
+    V[fft_pad(e)] = cmul(V[fft_pad(e)], __ldg(A.tw + (((int64_t)cg_ * k1) & (B - 1))));
+  }
+  if (blockIdx.x == 0) TRACE(1);
+  cl.sync();  // every CTA's V complete
+  }  // !FROM_V
+  // ---- phase B: rows k1 = r ROWS + rl, element c of row from CTA c / COLS
+  double2* S2 = reinterpret_cast<double2*>(X);                      // [E2 + E2/8]
+  double2* tw2 = S2 + E2 + E2 / 8;                                  // [B2T]
+  uint32_t* shist = reinterpret_cast<uint32_t*>(tw2 + B2T);         // [4096]
+  for (int i = t; i < B2T; i += 256) tw2[i] = __ldg(A.tw + (int64_t)i * B1T);  // omega_B2^i
+  const int ki = A.key_index ? A.key_index[s] : -1;
+  if (ki >= 0)
+    for (int i = t; i < 4096; i += 256) shist[i] = 0;
+  {
+    constexpr int PER = E2 / 256;
+    double2 buf[PER];
+#pragma unroll
+    for (int u2 = 0; u2 < PER; ++u2) {
+      const int e = t + u2 * 256;
+      const int rl = e / B2T, cc = e % B2T;  // consecutive threads: consecutive columns (owners rotate)
+      if constexpr (FROM_V) {
+        buf[u2] = __ldg(A.v + (int64_t)s * B + (int64_t)(r * ROWS + rl) * B2T + cc);
+      } else {
+        const double2* rv = cl.map_shared_rank(V, cc / COLS);
+        buf[u2] = rv[fft_pad((cc % COLS) * B1T + r * ROWS + rl)];
+      }
+    }
+#pragma unroll
+    for (int u2 = 0; u2 < PER; ++u2) {
+      const int e = t + u2 * 256;
+      S2[fft_pad(e)] = buf[u2];
+    }
+  }
+  __syncthreads();
+  fft_smem<B2T, E2, 256, true>(S2, tw2, B2T);
+  {
+    double2* rec = reinterpret_cast<double2*>(A.recs + (int64_t)s * A.rec_bytes);
+    uint64_t* keys = ki >= 0 ? A.keys + (int64_t)ki * B : nullptr;
+    for (int e = t; e < E2; e += 256) {
+      const int rl = e % ROWS, k2 = e / ROWS;  // consecutive threads: consecutive k1 (contiguous m)
+      const double2 v = S2[fft_pad(rl * B2T + k2)];
+      const int m = r * ROWS + rl + B1T * k2;
+      rec[m] = v;
+      if (ki >= 0) {
+        const uint64_t key = (uint64_t)__double_as_longlong(__dadd_rn(__dmul_rn(v.x, v.x), __dmul_rn(v.y, v.y)));
+        keys[m] = key;
+        atomicAdd(&shist[(uint32_t)(key >> 51) & 0xFFFu], 1u);
+      }
+    }
+  }
+  if (ki >= 0) {
+    __syncthreads();
+    for (int i = t; i < 4096; i += 256)
+      if (shist[i]) atomicAdd(&A.hist[(int64_t)ki * 4096 + i], shist[i]);
+  }
+  if (blockIdx.x == 0) TRACE(4);
+  // ---- phase C (the whole cluster takes the same branch: one slot per cluster)
+  cl.sync();  // remote V reads done; keys and histogram of the slot complete
+  if (ki >= 0 && A.do_select) select_cluster_body(A.sel, ki, X);
 }
 
 // ---------------------------------------------------------------------------

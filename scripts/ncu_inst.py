@@ -1,7 +1,7 @@
 """Per-CUDA-source-line stall samples and executed instructions from an ncu report (needs -lineinfo)."""
 import csv, subprocess, sys, os
 rep = sys.argv[1]; top = int(sys.argv[2]) if len(sys.argv) > 2 else 20
-out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source=cuda,sass"],
+out = subprocess.run(["ncu", "-i", rep] + (["-k", sys.argv[3]] if len(sys.argv) > 3 else []) + ["--page", "source", "--csv", "--print-source=cuda,sass"],
                      capture_output=True, text=True).stdout.splitlines()
 fname = "?"; hdr = None; agg = []
 for r in csv.reader(out):
