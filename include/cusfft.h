@@ -139,6 +139,26 @@ int cusfft_set_stream(cusfft_plan_t plan, void* cuda_stream);
  * Asynchronous; hit-buffer overflow is reported by cusfft_status. */
 int cusfft_execute(cusfft_plan_t plan, const void* d_x, int64_t* d_locs, void* d_vals);
 
+/* Batched transform of `count` independent signals of length n (the batched
+ * configuration of SURVEY.md §8(e); each signal is the problem of L13/L77):
+ *   d_x    : device, read-only, complex fp64; signal b at d_x + b * x_stride
+ *            elements (x_stride >= n)
+ *   d_locs : device, int64 [count][k];  d_vals : device, complex fp64 [count][k]
+ * Signal b's outputs equal cusfft_execute on it (same plan draws).  With a
+ * pipeline depth D > 1 (cusfft_set_pipeline) signal b runs on internal clone
+ * b mod D, each on its own stream forked from and joined back to the plan's
+ * stream, so one signal's DRAM-bound gather overlaps another's latency-bound
+ * cutoff / vote / estimation.  Asynchronous; count = 0 is a no-op.  Errors:
+ * CUSFFT_INVALID_PARAM (count < 0 or x_stride < n), CUSFFT_NULL_PTR. */
+int cusfft_execute_batch(cusfft_plan_t plan, const void* d_x, int64_t count, int64_t x_stride, int64_t* d_locs,
+                         void* d_vals);
+
+/* Pipeline depth D in [1, 8] of cusfft_execute_batch: creates (or frees) D - 1
+ * internal clones of the plan (same parameters and draws, own workspace and
+ * stream).  Synchronises the plan's stream.  cusfft_status also reports the
+ * clones; cusfft_destroy frees them.  world = 1 plans only. */
+int cusfft_set_pipeline(cusfft_plan_t plan, int32_t depth);
+
 /* Same transform from HOST buffers: copies h_x [n] to a plan-owned device
  * buffer, executes, copies k locations / values back and synchronises the
  * stream.  Pinned host memory gives asynchronous copies.  Returns the

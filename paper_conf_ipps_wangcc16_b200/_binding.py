@@ -30,7 +30,8 @@ DEBUG_PER_LOOP, DEBUG_TAPS, DEBUG_GHAT, DEBUG_NUM_HITS = 5, 6, 7, 8
 # Every symbol include/cusfft.h declares (checked by tests/test_abi.py).
 EXPORTED = (
     "cusfft_params_default", "cusfft_default_B", "cusfft_plan", "cusfft_plan_dist",
-    "cusfft_destroy", "cusfft_set_stream", "cusfft_execute", "cusfft_execute_host",
+    "cusfft_destroy", "cusfft_set_stream", "cusfft_execute", "cusfft_execute_host", "cusfft_execute_batch",
+    "cusfft_set_pipeline",
     "cusfft_execute_local", "cusfft_execute_finish", "cusfft_exchange_buffer", "cusfft_exchange_kind",
     "cusfft_get_info", "cusfft_get_debug", "cusfft_status", "cusfft_set_timing",
     "cusfft_get_stage_times", "cusfft_set_stage_limit", "cusfft_launches_per_execute", "cusfft_strerror",
@@ -85,6 +86,8 @@ def load_library():
         "cusfft_set_stream": (ctypes.c_int, [P, P]),
         "cusfft_execute": (ctypes.c_int, [P, P, P, P]),
         "cusfft_execute_host": (ctypes.c_int, [P, P, P, P]),
+        "cusfft_execute_batch": (ctypes.c_int, [P, P, i64, i64, P, P]),
+        "cusfft_set_pipeline": (ctypes.c_int, [P, i32]),
         "cusfft_execute_local": (ctypes.c_int, [P, P]),
         "cusfft_execute_finish": (ctypes.c_int, [P, P, P]),
         "cusfft_exchange_buffer": (ctypes.c_int, [P, ctypes.POINTER(P), ctypes.POINTER(i64)]),
@@ -219,6 +222,33 @@ class Plan:
         check(self._lib.cusfft_execute(self._h, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(locs.data_ptr()),
                                        ctypes.c_void_p(vals.data_ptr())), "cusfft_execute")
         return locs, vals
+
+    def execute_batch(self, xb, locs=None, vals=None):
+        """xb: complex128 CUDA tensor [count, n] (rows may be strided: row stride >= n
+        elements, unit element stride).  Returns (locs int64[count, k], vals complex128[count, k]);
+        row b equals execute(xb[b]).  See set_pipeline."""
+        import torch
+        if (xb.dtype != torch.complex128 or not xb.is_cuda or xb.dim() != 2 or xb.shape[1] != self.n
+                or xb.stride(1) != 1):
+            raise ValueError("xb must be a complex128 CUDA tensor [count, n] with unit element stride")
+        count = xb.shape[0]
+        if locs is None:
+            locs = torch.empty(count, self.k, dtype=torch.int64, device=xb.device)
+        if vals is None:
+            vals = torch.empty(count, self.k, dtype=torch.complex128, device=xb.device)
+        if not (locs.is_contiguous() and vals.is_contiguous() and locs.shape == (count, self.k)
+                and vals.shape == (count, self.k)):
+            raise ValueError("locs / vals must be contiguous [count, k]")
+        self._use_current_stream()
+        check(self._lib.cusfft_execute_batch(self._h, ctypes.c_void_p(xb.data_ptr()), count,
+                                             max(xb.stride(0), self.n) if count > 1 else self.n,
+                                             ctypes.c_void_p(locs.data_ptr()), ctypes.c_void_p(vals.data_ptr())),
+              "cusfft_execute_batch")
+        return locs, vals
+
+    def set_pipeline(self, depth: int):
+        """Pipeline depth of execute_batch (1..8 in-flight signals on internal clone plans)."""
+        check(self._lib.cusfft_set_pipeline(self._h, int(depth)), "cusfft_set_pipeline")
 
     def execute_raw(self, x_ptr: int, locs_ptr: int, vals_ptr: int):
         """Enqueue on the plan's current stream with raw device pointers."""

@@ -185,6 +185,7 @@ struct cusfft_plan_s {
   int64_t* d_locs_buf = nullptr;
   double2* d_vals_buf = nullptr;
   cudaStream_t stream = nullptr;
+  bool own_stream = false;        // clone plans (batched execution) own their stream
   int device = 0;
   bool timing = false;
   cudaEvent_t ev[7] = {};
@@ -206,7 +207,16 @@ struct cusfft_plan_s {
     const void* c = nullptr;
     cudaGraphExec_t exec = nullptr;
   } g_full, g_local, g_finish, g_full_t, g_local_t, g_finish_t;  // *_t: with timing event nodes
+  // whole-transform graphs by (x, locs, vals): up to kGraphCache, least recently used replaced
+  std::vector<GraphEntry> g_cache;
+  std::vector<uint64_t> g_used;
+  uint64_t g_tick = 0;
+  // batched execution (cusfft_execute_batch): depth-1 clones of this plan, each on its own stream
+  std::vector<cusfft_plan_s*> subs;
+  std::vector<cudaEvent_t> sub_ev;  // [depth] join events (+ fork event at the end)
 };
+
+constexpr size_t kGraphCache = 64;
 
 namespace {
 
@@ -245,6 +255,11 @@ void free_plan(cusfft_plan_t p) {
     for (auto& e : p->ev) cudaEventDestroy(e);
   for (auto* g : {&p->g_full, &p->g_local, &p->g_finish, &p->g_full_t, &p->g_local_t, &p->g_finish_t})
     if (g->exec) cudaGraphExecDestroy(g->exec);
+  for (auto& g : p->g_cache)
+    if (g.exec) cudaGraphExecDestroy(g.exec);
+  for (auto* sp : p->subs) free_plan(sp);
+  for (auto e : p->sub_ev) cudaEventDestroy(e);
+  if (p->own_stream && p->stream) cudaStreamDestroy(p->stream);
   if (p->cap_stream) cudaStreamDestroy(p->cap_stream);
   if (p->cap_stream2) cudaStreamDestroy(p->cap_stream2);
   if (p->ev_fork) cudaEventDestroy(p->ev_fork);
@@ -1308,6 +1323,39 @@ int run_graphed(cusfft_plan_t P, cusfft_plan_s::GraphEntry& g_plain, cusfft_plan
   return CUSFFT_SUCCESS;
 }
 
+// The cache entry for a whole-transform graph of (a, b, c) at the current stage limit.
+cusfft_plan_s::GraphEntry& full_entry(cusfft_plan_t P, const void* a, const void* b, const void* c) {
+  if (P->timing) return P->g_full;  // timing mode launches directly
+  size_t lru = 0;
+  for (size_t i = 0; i < P->g_cache.size(); ++i) {
+    const auto& g = P->g_cache[i];
+    if (g.exec && g.a == a && g.b == b && g.c == c && g.lim == P->stage_limit) {
+      P->g_used[i] = ++P->g_tick;
+      return P->g_cache[i];
+    }
+    if (P->g_used[i] < P->g_used[lru]) lru = i;
+  }
+  if (P->g_cache.size() < kGraphCache) {
+    P->g_cache.emplace_back();
+    P->g_used.push_back(++P->g_tick);
+    return P->g_cache.back();
+  }
+  P->g_used[lru] = ++P->g_tick;
+  return P->g_cache[lru];  // run_graphed re-captures it
+}
+
+int execute_full(cusfft_plan_t plan, const void* d_x, int64_t* d_locs, void* d_vals) {
+  return run_graphed(plan, full_entry(plan, d_x, d_locs, d_vals), plan->g_full_t, d_x, d_locs, d_vals, [&] {
+    const double2* x = reinterpret_cast<const double2*>(d_x);
+    double2* v = reinterpret_cast<double2*>(d_vals);
+    if (use_branches(plan))
+      return plan->staged ? launch_branched_staged(plan, x, d_locs, v) : launch_branched(plan, x, d_locs, v);
+    int rc = launch_local(plan, x);
+    if (rc) return rc;
+    return launch_finish(plan, d_locs, v);
+  });
+}
+
 }  // namespace
 
 // ===========================================================================
@@ -1414,15 +1462,66 @@ int cusfft_execute(cusfft_plan_t plan, const void* d_x, int64_t* d_locs, void* d
   if (!d_x || !d_locs || !d_vals) return CUSFFT_NULL_PTR;
   if (plan->world != 1) return CUSFFT_INVALID_LOOPS;
   DeviceGuard g(plan->device);
-  return run_graphed(plan, plan->g_full, plan->g_full_t, d_x, d_locs, d_vals, [&] {
-    const double2* x = reinterpret_cast<const double2*>(d_x);
-    double2* v = reinterpret_cast<double2*>(d_vals);
-    if (use_branches(plan))
-      return plan->staged ? launch_branched_staged(plan, x, d_locs, v) : launch_branched(plan, x, d_locs, v);
-    int rc = launch_local(plan, x);
+  return execute_full(plan, d_x, d_locs, d_vals);
+}
+
+int cusfft_set_pipeline(cusfft_plan_t plan, int32_t depth) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  if (depth < 1 || depth > 8) return CUSFFT_INVALID_PARAM;
+  if (plan->world != 1) return CUSFFT_INVALID_LOOPS;
+  DeviceGuard g(plan->device);
+  CK(cudaStreamSynchronize(plan->stream));
+  while ((int)plan->subs.size() > depth - 1) {
+    free_plan(plan->subs.back());
+    plan->subs.pop_back();
+  }
+  while ((int)plan->subs.size() < depth - 1) {
+    cusfft_plan_t sp = nullptr;
+    const int rc = cusfft_plan(&sp, plan->n, plan->k, plan->B, plan->L, &plan->prm);
     if (rc) return rc;
-    return launch_finish(plan, d_locs, v);
-  });
+    cudaStream_t st = nullptr;
+    CK(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
+    sp->stream = st;
+    sp->own_stream = true;
+    plan->subs.push_back(sp);
+  }
+  while ((int)plan->sub_ev.size() < depth + 1) {
+    cudaEvent_t e;
+    CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    plan->sub_ev.push_back(e);
+  }
+  return CUSFFT_SUCCESS;
+}
+
+int cusfft_execute_batch(cusfft_plan_t plan, const void* d_x, int64_t count, int64_t x_stride, int64_t* d_locs,
+                         void* d_vals) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  if (count < 0 || x_stride < plan->n) return CUSFFT_INVALID_PARAM;
+  if (count == 0) return CUSFFT_SUCCESS;
+  if (!d_x || !d_locs || !d_vals) return CUSFFT_NULL_PTR;
+  if (plan->world != 1) return CUSFFT_INVALID_LOOPS;
+  DeviceGuard g(plan->device);
+  const double2* x = reinterpret_cast<const double2*>(d_x);
+  double2* v = reinterpret_cast<double2*>(d_vals);
+  const int depth = 1 + (int)plan->subs.size();
+  if (depth > 1) {  // fork the clones' streams off the caller's stream
+    CK(cudaEventRecord(plan->sub_ev[depth], plan->stream));
+    for (auto* sp : plan->subs) CK(cudaStreamWaitEvent(sp->stream, plan->sub_ev[depth], 0));
+  }
+  for (int64_t b = 0; b < count; ++b) {
+    const int lane = (int)(b % depth);
+    cusfft_plan_t P = lane == 0 ? plan : plan->subs[lane - 1];
+    P->stage_limit = plan->stage_limit;
+    const int rc = execute_full(P, x + b * x_stride, d_locs + b * plan->k, v + b * plan->k);
+    if (rc) return rc;
+  }
+  if (depth > 1) {  // join
+    for (int l = 1; l < depth; ++l) {
+      CK(cudaEventRecord(plan->sub_ev[l], plan->subs[l - 1]->stream));
+      CK(cudaStreamWaitEvent(plan->stream, plan->sub_ev[l], 0));
+    }
+  }
+  return CUSFFT_SUCCESS;
 }
 
 int cusfft_status(cusfft_plan_t plan) {
@@ -1433,6 +1532,10 @@ int cusfft_status(cusfft_plan_t plan) {
   CK(cudaMemcpy(flags, plan->d_flags, sizeof(flags), cudaMemcpyDeviceToHost));
   if (flags[1]) return CUSFFT_HIT_OVERFLOW;
   if (flags[2] || flags[3]) return CUSFFT_INTERNAL;
+  for (auto* sp : plan->subs) {
+    const int rc = cusfft_status(sp);
+    if (rc) return rc;
+  }
   return CUSFFT_SUCCESS;
 }
 
@@ -1449,7 +1552,8 @@ int cusfft_execute_host(cusfft_plan_t plan, const void* h_x, int64_t* h_locs, vo
   }
   cudaStream_t st = plan->stream;
   CK(cudaMemcpyAsync(plan->d_xbuf, h_x, (size_t)plan->n * 16, cudaMemcpyHostToDevice, st));
-  rc = run_graphed(plan, plan->g_full, plan->g_full_t, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf, [&] {
+  rc = run_graphed(plan, full_entry(plan, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf), plan->g_full_t,
+                   plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf, [&] {
     if (use_branches(plan))
       return plan->staged ? launch_branched_staged(plan, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf)
                           : launch_branched(plan, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf);

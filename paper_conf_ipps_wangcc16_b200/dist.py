@@ -125,4 +125,58 @@ class LoopShardedSfft:
         return self.engine.finish()
 
 
-__all__ = ["loops_of_rank", "slot_of_loop", "signal_range", "CudaEngine", "LoopShardedSfft"]
+def batch_range(rank: int, count: int, world: int):
+    """Signals [lo, hi) of a batch of `count` independent signals owned by
+    `rank` (batched configuration): contiguous, sizes differ by
+    at most one, every signal owned once."""
+    if world < 1 or not 0 <= rank < world or count < 0:
+        raise ValueError("bad rank / world / count")
+    base, extra = divmod(count, world)
+    lo = rank * base + min(rank, extra)
+    return lo, lo + base + (1 if rank < extra else 0)
+
+
+class BatchShardedSfft:
+    """Independent signals sharded across ranks with NO collective on the data
+    path: rank g transforms signals batch_range(g, count, world) with its own
+    single-GPU plan (engine.execute_batch).  gather_outputs() is optional output
+    plumbing (an all-gather of the k-sparse results), outside the transform."""
+
+    def __init__(self, engine, count: int, group=None):
+        self.engine = engine
+        self.count = int(count)
+        self.group = group
+        self.world = dist.get_world_size(group) if dist.is_initialized() else 1
+        self.rank = dist.get_rank(group) if dist.is_initialized() else 0
+        self.lo, self.hi = batch_range(self.rank, self.count, self.world)
+
+    def execute(self, xb_local):
+        """xb_local: this rank's signals [hi - lo, n].  Returns its (locs, vals)."""
+        if xb_local.shape[0] != self.hi - self.lo:
+            raise ValueError("xb_local must hold exactly this rank's signals")
+        return self.engine.execute_batch(xb_local)
+
+    def gather_outputs(self, locs, vals):
+        """All ranks' (locs, vals) in batch order (pads ranks to the largest share)."""
+        if self.world == 1:
+            return locs, vals
+        share = -(-self.count // self.world)
+        k = locs.shape[1]
+        pl = locs.new_full((share, k), -1)
+        pv = vals.new_zeros((share, k))
+        pl[:locs.shape[0]] = locs
+        pv[:vals.shape[0]] = vals
+        al = [torch.empty_like(pl) for _ in range(self.world)]
+        av = [torch.empty_like(pv) for _ in range(self.world)]
+        dist.all_gather(al, pl, group=self.group)
+        dist.all_gather(av, pv, group=self.group)
+        out_l, out_v = [], []
+        for g in range(self.world):
+            lo, hi = batch_range(g, self.count, self.world)
+            out_l.append(al[g][:hi - lo])
+            out_v.append(av[g][:hi - lo])
+        return torch.cat(out_l), torch.cat(out_v)
+
+
+__all__ = ["loops_of_rank", "slot_of_loop", "signal_range", "batch_range", "CudaEngine", "LoopShardedSfft",
+           "BatchShardedSfft"]

@@ -85,6 +85,8 @@ def test_null_pointers_and_invalid_plan():
     assert lib.cusfft_execute(None, None, None, None) == b.INVALID_PLAN
     assert lib.cusfft_status(None) == b.INVALID_PLAN
     assert lib.cusfft_launches_per_execute(None) == b.INVALID_PLAN
+    assert lib.cusfft_execute_batch(None, None, 0, 0, None, None) == b.INVALID_PLAN
+    assert lib.cusfft_set_pipeline(None, 2) == b.INVALID_PLAN
 
 
 @pytest.mark.parametrize("kw,code", [

@@ -295,3 +295,71 @@ def test_signal_sharded_plans_emulated_allreduce(world, n, k, L):
         locs, vals = e.finish()
         torch.cuda.synchronize()
         assert torch.equal(locs, ref_l)
+
+
+# ---------------------------------------------------------------------------
+# Batched independent signals (SURVEY.md §8(e) batched config): no collective
+# on the data path; each rank transforms its contiguous share.
+# ---------------------------------------------------------------------------
+def test_batch_range_partitions_signals():
+    from paper_conf_ipps_wangcc16_b200.dist import batch_range
+    for count, world in [(64, 8), (64, 3), (5, 8), (0, 2), (7, 1)]:
+        spans = [batch_range(g, count, world) for g in range(world)]
+        assert spans[0][0] == 0 and spans[-1][1] == count
+        for (a, b), (c, d) in zip(spans, spans[1:]):
+            assert b == c
+        sizes = [b - a for a, b in spans]
+        assert max(sizes) - min(sizes) <= 1
+    with pytest.raises(ValueError):
+        batch_range(2, 4, 2)
+
+
+class OracleBatchEngine:
+    """execute_batch with the oracle's arithmetic (test infrastructure)."""
+
+    def __init__(self, p):
+        self.p = p
+
+    def execute_batch(self, xb):
+        outs = [O.sfft(np.asarray(x), self.p) for x in xb]
+        return (torch.from_numpy(np.stack([o.locs for o in outs])),
+                torch.from_numpy(np.stack([o.vals for o in outs])))
+
+
+def _batch_worker(rank, world, port, q):
+    from paper_conf_ipps_wangcc16_b200.dist import BatchShardedSfft
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        n, k, count = 2 ** 12, 6, 5
+        xs = np.stack([planted_signal(n, k, seed=40 + b)[0] for b in range(count)])
+        p = O.make_params(n, k, L=8, loc_loops=5, vote_threshold=3, seed=9)
+        drv = BatchShardedSfft(OracleBatchEngine(p), count)
+        locs, vals = drv.execute(xs[drv.lo:drv.hi])
+        gl, gv = drv.gather_outputs(locs, vals)
+        q.put((rank, drv.lo, drv.hi, gl.tolist(), gv.tolist()))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_batch_sharded_gloo():
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_batch_worker, args=(r, world, port, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    out = sorted(q.get(timeout=300) for _ in range(world))
+    for pr in procs:
+        pr.join(timeout=60)
+        assert pr.exitcode == 0
+    n, k, count = 2 ** 12, 6, 5
+    p = O.make_params(n, k, L=8, loc_loops=5, vote_threshold=3, seed=9)
+    assert [(lo, hi) for _, lo, hi, _, _ in out] == [(0, 3), (3, 5)]
+    for b in range(count):
+        x, S, X = planted_signal(n, k, seed=40 + b)
+        ref = O.sfft(x, p)
+        for _, _, _, gl, gv in out:  # every rank holds every result after the (optional) gather
+            assert gl[b] == ref.locs.tolist()
+            np.testing.assert_array_equal(np.array(gv[b]), ref.vals)

@@ -315,3 +315,56 @@ def test_kernel_variants_agree(env, monkeypatch):
     assert np.array_equal(np.sort(alt.debug(DEBUG_HITS)), h0)
     assert torch.equal(l1, l0)
     assert torch.equal(v1, v0)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("depth", [1, 2, 3])
+def test_execute_batch_matches_single(depth):
+    """cusfft_execute_batch: signal b's outputs equal cusfft_execute on it, for
+    any pipeline depth (clone plans on their own streams), with a row stride
+    larger than n; status covers the clones."""
+    import torch
+    from paper_conf_ipps_wangcc16_b200 import Plan
+    n, k, count = 2 ** 18, 50, 5
+    xs = np.stack([planted_signal(n, k, seed=60 + b)[0] for b in range(count)])
+    xpad = torch.zeros(count, n + 64, dtype=torch.complex128, device="cuda")
+    xpad[:, :n] = torch.from_numpy(xs).cuda()
+    xb = xpad[:, :n]
+    with Plan(n, k, L=16, seed=5) as plan:
+        ref = [plan.execute(xb[b].contiguous()) for b in range(count)]
+        ref = [(l.clone(), v.clone()) for l, v in ref]
+        plan.set_pipeline(depth)
+        for _ in range(2):  # second call replays the cached graphs
+            locs, vals = plan.execute_batch(xb)
+            torch.cuda.synchronize()
+            assert plan.status() == 0
+            for b in range(count):
+                assert torch.equal(locs[b], ref[b][0])
+                assert torch.equal(vals[b], ref[b][1])
+    for b in range(count):
+        x, S, X = planted_signal(n, k, seed=60 + b)
+        assert set(ref[b][0].cpu().tolist()) == set(S.tolist())
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("k,bcst", [(50, 1.0), (200, 1.0), (1000, 1.0), (2000, 2.0), (4096, 2.0)])
+def test_C5_k_sweep_parity(k, bcst):
+    """C5 (BASELINE.json configs[4]): n = 2^22, k = 50 ... 4096 (B from the
+    formula; Bcst = 2 for k >= 2000).  GPU = oracle on the
+    recovered set (exact) and values (1e-9), planted support recovered."""
+    import torch
+    import oracle as O
+    from paper_conf_ipps_wangcc16_b200 import Plan, default_B
+    n = 2 ** 22
+    B = default_B(n, k, bcst)
+    x, S, X = planted_signal(n, k, seed=70 + k)
+    with Plan(n, k, B=B, L=16, seed=8) as plan:
+        locs, vals = plan.execute(torch.from_numpy(x).cuda())
+        torch.cuda.synchronize()
+        assert plan.status() == 0
+        locs, vals = locs.cpu().numpy(), vals.cpu().numpy()
+    ref = O.sfft(x, O.make_params(n, k, B=B, L=16, seed=8))
+    assert np.array_equal(locs, ref.locs)
+    np.testing.assert_allclose(vals, ref.vals, rtol=1e-9, atol=1e-12)
+    assert set(locs.tolist()) == set(S.tolist())
+    assert O.l1_error(locs, vals, S, X, k) <= 1e-6
