@@ -128,6 +128,8 @@ struct cusfft_plan_s {
   // by the stand-alone FFT pass 1, instead of k_fold_fft1.
   bool stage_scatter = true;   // default: scatter staging + bulk-copy phase 2 (measured fastest)
   bool stage_split = false;
+  bool stage_packed = false;      // scatter schedule as packed (slot, i) words (k_stage_packed; CUSFFT_PACKED=0: off)
+  int stage_ibits = 0;
   bool p2_tma = true;             // scatter phase 2 through bulk copies (k_fold_fft1_tma; CUSFFT_P2=ldg: k_fold_fft1 MODE 2)
   bool p2_discard = true;         // drop consumed staging lines from L2 (CUSFFT_DISCARD=0: keep)
   bool slot_fused = false;        // FFT pass 2 (+ fold) + cutoff in one cluster kernel per slot (k_slot; CUSFFT_SLOT=1|2)
@@ -144,6 +146,7 @@ struct cusfft_plan_s {
     uint32_t* spos = nullptr;    // [total] sorted gather positions
     uint32_t* inv = nullptr;     // [s1 - s0][R][B] staging index in the fused kernel's thread order (index mode)
     uint32_t* dst = nullptr;     // [total] thread-order staging position of sorted gather q (scatter mode)
+    uint32_t* code = nullptr;    // [total] packed (local slot << ibits | i) in address order (packed scatter mode)
     double2* staging = nullptr;  // this group's staging buffer (groups share one unless branched)
   };
   std::vector<StageGroup> groups;
@@ -245,6 +248,7 @@ void free_plan(cusfft_plan_t p) {
     if (g.spos) cudaFree(g.spos);
     if (g.inv) cudaFree(g.inv);
     if (g.dst) cudaFree(g.dst);
+    if (g.code) cudaFree(g.code);
   }
   void* ptrs[] = {p->d_taps, p->d_taps_perm, p->d_staging, p->d_ghat, p->d_tw, p->d_slots, p->d_loc_slots, p->d_loc_sigma, p->d_loc_a,
                   p->d_sel_slots, p->d_u, p->d_v, p->d_records, p->d_keys, p->d_zero, p->d_key_index, p->d_ckey, p->d_cidx, p->d_hits, p->d_hit_vals,
@@ -704,6 +708,15 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       P->stage_split = m.rfind("split", 0) == 0;
       P->stage_scatter = m.find("scatter") != std::string::npos;
     }
+    {  // packed (slot, i) schedule words: fused scatter mode when local slot and tap index fit 32 bits
+      int ib = 1;
+      while ((int64_t(1) << ib) < P->w) ++ib;
+      int sb = 0;
+      while ((1 << sb) < P->Lg) ++sb;
+      const char* ep = std::getenv("CUSFFT_PACKED");
+      P->stage_ibits = ib;
+      P->stage_packed = P->stage_scatter && !P->stage_split && ib + sb <= 32 && !(ep && ep[0] == '0');
+    }
     int64_t maxtot = 0, sumtot = 0;  // staging elements: w per slot (index mode) or R B per slot (scatter mode)
     for (auto& r : ranges) {
       const int64_t t = (int64_t)(r.second - r.first) * (P->stage_scatter ? P->R * B : P->w);
@@ -732,8 +745,10 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
           }
         }
         std::sort(ev.begin(), ev.end());
-        std::vector<uint32_t> spos((size_t)g.total), dst, inv;
-        if (P->stage_scatter)
+        std::vector<uint32_t> spos((size_t)g.total), dst, inv, code;
+        if (P->stage_packed)
+          code.assign((size_t)g.total, 0u);
+        else if (P->stage_scatter)
           dst.assign((size_t)g.total, 0u);
         else
           inv.assign((size_t)(g.s1 - g.s0) * P->R * B, 0u);
@@ -745,16 +760,24 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
           const int64_t c = j % P->B2, j1 = j / P->B2;
           const int64_t cta = c / C, t = (c % C) * P->B1 + j1;
           const uint32_t tpos = (uint32_t)((sl * P->R + rr) * B + (P->stage_split ? j : cta * 256 + t));
-          if (P->stage_scatter)
+          if (P->stage_packed)
+            code[(size_t)q] = ((uint32_t)sl << P->stage_ibits) | (uint32_t)i;
+          else if (P->stage_scatter)
             dst[(size_t)q] = tpos;
           else
             inv[(size_t)tpos] = (uint32_t)q;
         }
         P->groups.push_back(g);
         auto& gg = P->groups.back();
-        if ((rc = dalloc(&gg.spos, (size_t)g.total))) return fail(rc);
-        if ((rc = upload(gg.spos, spos.data(), spos.size() * sizeof(uint32_t)))) return fail(rc);
-        if (P->stage_scatter) {
+        if (P->stage_packed) {
+          if ((rc = dalloc(&gg.code, code.size()))) return fail(rc);
+          if ((rc = upload(gg.code, code.data(), code.size() * sizeof(uint32_t)))) return fail(rc);
+        } else if ((rc = dalloc(&gg.spos, (size_t)g.total)) ||
+                   (rc = upload(gg.spos, spos.data(), spos.size() * sizeof(uint32_t)))) {
+          return fail(rc);
+        }
+        if (P->stage_packed) {
+        } else if (P->stage_scatter) {
           if ((rc = dalloc(&gg.dst, dst.size()))) return fail(rc);
           if ((rc = upload(gg.dst, dst.data(), dst.size() * sizeof(uint32_t)))) return fail(rc);
         } else {
@@ -880,8 +903,16 @@ int launch_stage1(cusfft_plan_t P, const cusfft_plan_s::StageGroup& g, const dou
   const int tot = (int)g.total;
   const int grid = std::max(1, std::min((tot + 8 * 256 - 1) / (8 * 256), sms * P->stage_cps));
   g_apw = P->stage_window;  // keep the staging buffer L2-resident for phase 2
-  const cudaError_t e = launch_k(k_stage, dim3(grid), dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)g.spos,
-                                 (const uint32_t*)g.dst, g.staging, tot, z);
+  cudaError_t e;
+  if (g.code) {
+    StagePackArgs a{x, g.code, g.staging, P->d_slots + (size_t)P->lrank * P->Lg + g.s0, tot, g.s1 - g.s0,
+                    P->stage_ibits, P->R, ilog2(P->B), P->logB2, P->logB1, ilog2(256 / P->B1),
+                    (uint32_t)(P->n - 1), z};
+    e = launch_k(k_stage_packed, dim3(grid), dim3(256), 0, st, P->cur_prio, a);
+  } else {
+    e = launch_k(k_stage, dim3(grid), dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)g.spos,
+                 (const uint32_t*)g.dst, g.staging, tot, z);
+  }
   g_apw = cudaAccessPolicyWindow{};
   CK(e);
   return CUSFFT_SUCCESS;
@@ -902,7 +933,7 @@ int launch_stage2(cusfft_plan_t P, const cusfft_plan_s::StageGroup& g, cudaStrea
                    (const uint32_t*)g.inv, (const double*)P->d_taps, P->d_u + (size_t)g.s0 * B, B, P->w, P->R, z);
   } else {
     e = launch_fold_fft1(P, g.staging, g.inv, P->d_slots + (size_t)P->lrank * P->Lg + g.s0,
-                         P->d_u + (size_t)g.s0 * B, P->d_v + (size_t)g.s0 * B, g.s1 - g.s0, z, st, g.dst != nullptr);
+                         P->d_u + (size_t)g.s0 * B, P->d_v + (size_t)g.s0 * B, g.s1 - g.s0, z, st, g.dst != nullptr || g.code != nullptr);
   }
   CK(e);
   return CUSFFT_SUCCESS;

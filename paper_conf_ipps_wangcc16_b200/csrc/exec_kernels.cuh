@@ -24,6 +24,8 @@ namespace cusfft {
 // ---------------------------------------------------------------------------
 // Per-execution block zeroed by the CTAs of the first fold launch (the fold is
 // memory-latency bound, so the stores are free): flags, histograms, counters.
+constexpr int kMaxLoops = 64;  // L limit (plan validation)
+
 struct ZeroArgs {
   int* p;
   int n;
@@ -140,6 +142,67 @@ __global__ void __launch_bounds__(256) k_stage(const double2* __restrict__ x, co
         double2* o = staging + (dst ? __ldg(dst + q) : (uint32_t)q);
         asm volatile("st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %3;" ::"l"(o), "d"(v[c].x), "d"(v[c].y),
                      "l"(pl));
+      }
+    }
+  }
+  TRACE_END(6);
+}
+
+// Packed form of the scatter staging (default): the schedule holds one word
+// per gather, (local slot << ibits) | tap index i, in address order; the
+// position sigma_s i + tau_s and phase 2's thread-order destination
+//   (s R + rr) B + tile 256 + (c mod C) B1 + j1,  i = rr B + j, j = c + B2 j1,
+// are recomputed here (shifts and masks), halving the schedule bytes.
+struct StagePackArgs {
+  const double2* x;
+  const uint32_t* code;
+  double2* staging;
+  const SlotParam* slots;  // group slot 0
+  int total, nslots, ibits, R, logB, logB2, logB1, logC;
+  uint32_t nmask;
+  ZeroArgs zero;
+};
+
+__global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
+  pdl_wait();
+  KTRACE(1);
+  if (blockIdx.x == 0) TRACE(0);
+  __shared__ uint32_t ssig[kMaxLoops], stau[kMaxLoops];
+  for (int i = threadIdx.x; i < A.nslots; i += blockDim.x) {
+    ssig[i] = A.slots[i].sigma;
+    stau[i] = A.slots[i].tau;
+  }
+  zero_part(A.zero);
+  __syncthreads();
+  const uint64_t pf = l2_policy_first(), pl = l2_policy_last();
+  const uint32_t imask = (1u << A.ibits) - 1u;
+  const uint32_t Bm = (1u << A.logB) - 1u, B2m = (1u << A.logB2) - 1u, Cm = (1u << A.logC) - 1u;
+  const int T = gridDim.x * blockDim.x;
+  for (int q0 = blockIdx.x * blockDim.x + threadIdx.x; q0 < A.total; q0 += 8 * T) {
+    double2 v[8];
+    uint32_t cd[8];
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      const int q = q0 + c * T;
+      if (q < A.total) {
+        cd[c] = __ldg(A.code + q);
+        const uint32_t sl = cd[c] >> A.ibits, i = cd[c] & imask;
+        const double2* p = A.x + ((ssig[sl] * i + stau[sl]) & A.nmask);
+        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.L2::64B.v2.f64 {%0, %1}, [%2], %3;"
+                     : "=d"(v[c].x), "=d"(v[c].y) : "l"(p), "l"(pf));
+      }
+    }
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      const int q = q0 + c * T;
+      if (q < A.total) {
+        const uint32_t sl = cd[c] >> A.ibits, i = cd[c] & imask;
+        const uint32_t rr = i >> A.logB, j = i & Bm;
+        const uint32_t col = j & B2m, j1 = j >> A.logB2;
+        const uint32_t dst = ((sl * (uint32_t)A.R + rr) << A.logB) + ((col >> A.logC) << 8) +
+                             ((col & Cm) << A.logB1) + j1;
+        asm volatile("st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %3;" ::"l"(A.staging + dst), "d"(v[c].x),
+                     "d"(v[c].y), "l"(pl));
       }
     }
   }
@@ -1903,7 +1966,6 @@ struct EstArgs {
   uint32_t* out_hist;  // [4096] level-0 histogram of hit_keys
 };
 
-constexpr int kMaxLoops = 64;
 
 __device__ __forceinline__ double2 loop_estimate(const EstArgs& A, const SlotParam& sp, int l, uint32_t f) {
   const uint32_t p = (sp.sigma * f) & A.nmask;

@@ -293,7 +293,7 @@ def test_parity_snr_sweep(snr_db):
                                  {"CUSFFT_STAGE_MODE": "split_scatter"}, {"CUSFFT_NO_STAGE": "1"},
                                  {"CUSFFT_STAGE_MODE": "fused_index"}, {"CUSFFT_P2": "ldg"}, {"CUSFFT_DISCARD": "0"},
                                  {"CUSFFT_SLOT": "1"}, {"CUSFFT_SLOT": "2"}, {"CUSFFT_BRANCH": "1"},
-                                 {"CUSFFT_STAGE_GROUPS": "2"}])
+                                 {"CUSFFT_STAGE_GROUPS": "2"}, {"CUSFFT_PACKED": "0"}])
 def test_kernel_variants_agree(env, monkeypatch):
     """Every alternative kernel path (selected at plan time by environment
     switches, used for A/B measurements) gives the default path's hits and
