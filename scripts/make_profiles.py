@@ -34,33 +34,35 @@ if os.path.exists(f"{G}/launches.csv"):
     lines.append("| kernel | launches | mean µs |\n|---|---|---|")
     for k, v in sorted(other.items(), key=lambda kv: -sum(kv[1]) / len(kv[1])):
         lines.append(f"| `{k[:70]}` | {len(v)} | {sum(v) / len(v) / 1e3:.2f} |")
-# full captures
+# full captures: ONE application-replay report of one whole execution
+# (--cache-control none: phase 2 sees the staging buffer phase 1 left in L2,
+# as in the timed step; x itself is cold because run_c3 flushes L2 first)
 want = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum", "dram__throughput.avg.pct_of_peak_sustained_elapsed",
-        "lts__t_sector_hit_rate.pct", "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum", "l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum",
+        "lts__t_sector_hit_rate.pct", "lts__throughput.avg.pct_of_peak_sustained_elapsed",
+        "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum", "l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum",
         "lts__t_sectors_srcunit_tex_op_read.sum", "sm__warps_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread",
         "smsp__inst_executed.sum", "sm__throughput.avg.pct_of_peak_sustained_elapsed", "launch__grid_size", "launch__block_size"]
+scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
+rep = f"{G}/prof_all.ncu-rep"
 traffic = None
 fold_parts = {}
-for name, rep in [("k_stage (staged gather, phase 1)", f"{G}/prof_k_stage.ncu-rep"),
-                  ("k_fold_fft1 (fold phase 2 + FFT pass 1)", f"{G}/prof_fold_full.ncu-rep"), ("k_fft (pass 2 + keys)", f"{G}/prof_k_fft.ncu-rep"),
-                  ("k_select", f"{G}/prof_k_select.ncu-rep"), ("k_vote", f"{G}/prof_k_vote.ncu-rep"),
-                  ("k_estimate", f"{G}/prof_k_estimate.ncu-rep"), ("k_output", f"{G}/prof_k_output.ncu-rep")]:
-    if not os.path.exists(rep):
-        continue
-    m = raw(rep)
-    lines.append(f"\n## {name} — `ncu --set full --clock-control none` (C3, `scripts/run_c3.py`)\n")
-    lines.append("| metric | value |\n|---|---|")
+if os.path.exists(rep):
+    out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(out.splitlines()))
+    hdr, units = rows[0], dict(zip(rows[0], rows[1]))
+    lines.append("\n## Full captures of one C3 execution — `ncu --set full --cache-control none --replay-mode application "
+                 "--clock-control none` (`scripts/run_c3.py`, L2 flushed before the execution)\n")
+    names = [r[hdr.index("Kernel Name")].split("(")[0].replace("void ", "") for r in rows[2:]]
+    lines.append("| metric | " + " | ".join(f"`{n}`" for n in names) + " |")
+    lines.append("|---|" + "---|" * len(names))
     for w in want:
-        if w in m:
-            lines.append(f"| {w} | {m[w]} |")
-    if ("fold" in name or "stage" in name) and "dram__bytes_read.sum" in m:
-        out = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
-        rows = list(csv.reader(out.splitlines()))
-        unit = dict(zip(rows[0], rows[1]))
-        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
-        rd = float(m["dram__bytes_read.sum"]) * scale[unit["dram__bytes_read.sum"]]
-        wr = float(m["dram__bytes_write.sum"]) * scale[unit["dram__bytes_write.sum"]]
-        fold_parts[name.split()[0]] = (rd, wr)
+        if w in hdr:
+            lines.append(f"| {w} ({units.get(w, '')}) | " + " | ".join(r[hdr.index(w)] for r in rows[2:]) + " |")
+    for n, r in zip(names, rows[2:]):
+        if "k_stage" in n or "k_fold" in n:
+            rd = float(r[hdr.index("dram__bytes_read.sum")]) * scale[units["dram__bytes_read.sum"]]
+            wr = float(r[hdr.index("dram__bytes_write.sum")]) * scale[units["dram__bytes_write.sum"]]
+            fold_parts[n] = (rd, wr)
 if fold_parts:
     rd = sum(v[0] for v in fold_parts.values())
     wr = sum(v[1] for v in fold_parts.values())
@@ -70,4 +72,4 @@ if fold_parts:
 if traffic:
     json.dump(traffic, open(f"{P}/fold_traffic_C3.json", "w"), indent=1)
 open(f"{P}/{tag}_ncu_summary.md", "w").write("\n".join(lines) + "\n")
-print("\n".join(lines[:40]))
+print("\n".join(lines[:60]))

@@ -12,7 +12,10 @@ x, S, X = planted_signal(n, k, 1)
 xd = torch.from_numpy(x).cuda()
 tol = {"C3": 1e-7}.get(cfg, 1e-8)  # bench.py TOLERANCE
 plan = Plan(n, k, L=LL, seed=3, tolerance=tol)
+fl = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+fr = torch.ones(64 << 20, dtype=torch.int32, device="cuda")
 for _ in range(reps):
+    fl.zero_(); fr.sum()  # L2 flush as in bench.py: x cold, nothing of the last execution resident
     locs, vals = plan.execute(xd)
 torch.cuda.synchronize()
 print("ok", plan.status(), set(locs.cpu().tolist()) == set(S.tolist()))
