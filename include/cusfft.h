@@ -210,7 +210,9 @@ int64_t cusfft_get_debug(cusfft_plan_t plan, int32_t what, void* host_dst, int64
 int cusfft_status(cusfft_plan_t plan);
 
 /* Per-stage device times (ms) of the last execution when timing is enabled:
- * ms[0..5] = fold, B-point FFT, cutoff, vote, estimate, output.  Enabling
+ * ms[0..5] = fold, B-point FFT, cutoff, vote, estimate, output; with cap >= 7,
+ * ms[6] = phase 1 of the staged fold alone (the address-ordered permute
+ * gather k_stage*), -1 when the plan is not staged.  Enabling
  * records CUDA events between the kernels on the plan's stream.  get syncs. */
 int cusfft_set_timing(cusfft_plan_t plan, int32_t enable);
 int cusfft_get_stage_times(cusfft_plan_t plan, float* ms, int32_t cap);

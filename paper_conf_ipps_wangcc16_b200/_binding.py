@@ -336,9 +336,11 @@ class Plan:
         check(self._lib.cusfft_set_timing(self._h, 1 if enable else 0), "cusfft_set_timing")
 
     def stage_times(self):
-        ms = (ctypes.c_float * 6)()
-        check(self._lib.cusfft_get_stage_times(self._h, ms, 6), "cusfft_get_stage_times")
-        return dict(zip(("fold", "fft", "cutoff", "vote", "estimate", "output"), list(ms)))
+        """Stage times (ms) of the last timed execution; 'gather' is phase 1 of
+        the staged fold alone (-1 when the plan is not staged)."""
+        ms = (ctypes.c_float * 7)()
+        check(self._lib.cusfft_get_stage_times(self._h, ms, 7), "cusfft_get_stage_times")
+        return dict(zip(("fold", "fft", "cutoff", "vote", "estimate", "output", "gather"), list(ms)))
 
     def set_stage_limit(self, stages: int):
         check(self._lib.cusfft_set_stage_limit(self._h, stages), "cusfft_set_stage_limit")

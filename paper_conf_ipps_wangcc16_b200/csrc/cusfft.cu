@@ -128,6 +128,8 @@ struct cusfft_plan_s {
   // by the stand-alone FFT pass 1, instead of k_fold_fft1.
   bool stage_scatter = true;   // default: scatter staging + bulk-copy phase 2 (measured fastest)
   bool stage_split = false;
+  bool stage_atomic = false;      // phase 1 multiplies by the tap and adds into u with fp64 L2 reductions, no staging
+                                  // (CUSFFT_STAGE_MODE=atomic; bucket sums then not in Alg. 1's order: opt-in A/B)
   bool stage_packed = false;      // scatter schedule as packed (slot, i) words (k_stage_packed; CUSFFT_PACKED=0: off)
   int stage_ibits = 0;
   bool p2_tma = true;             // scatter phase 2 through bulk copies (k_fold_fft1_tma; CUSFFT_P2=ldg: k_fold_fft1 MODE 2)
@@ -191,11 +193,14 @@ struct cusfft_plan_s {
   bool own_stream = false;        // clone plans (batched execution) own their stream
   int device = 0;
   bool timing = false;
-  cudaEvent_t ev[7] = {};
+  cudaEvent_t ev[8] = {};  // stage boundaries 0..6; [7] after phase 1 of the staged fold
   bool ev_made = false;
   // CUDA graphs of the launch sequences, keyed by the caller's pointers
   bool use_graph = true;
   bool branched = false;          // two-branch graph (location chain || estimation folds); opt-in
+  int branch_fork = 0;            // CUSFFT_BRANCH=2..5: the estimation branch forks after phase 1 / the location
+                                  // slots' phase 2 / their FFT pass 2 / the cutoff
+  bool branch_p2 = true;          // CUSFFT_BRANCH=2: one phase 1, then location chain || estimation phase 2 + FFT
   bool skip_stage = false;        // measurement only (CUSFFT_SKIP_STAGE)
   int stage_cps = 8;              // k_stage CTAs per SM (CUSFFT_STAGE_CPS; branched default 2: room for the chain)
   int nloc_local = 0;             // local slots [0, nloc_local) are location loops
@@ -504,7 +509,11 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   P->R = (int)((w64 + B - 1) / B);
   P->stream = nullptr;
   if (const char* e = std::getenv("CUSFFT_NO_GRAPH")) P->use_graph = !(e[0] == '1');
-  if (const char* e = std::getenv("CUSFFT_BRANCH")) P->branched = (e[0] == '1');
+  if (const char* e = std::getenv("CUSFFT_BRANCH")) {
+    P->branched = (e[0] == '1');
+    P->branch_p2 = (e[0] >= '2' && e[0] <= '5');  // 0: one serial chain, 1: the two-group staged graph
+    if (P->branch_p2) P->branch_fork = e[0] - '2';
+  }
   if (const char* e = std::getenv("CUSFFT_SELECT_MULTI")) P->sel_multi = (e[0] == '1');
   P->sel_cluster = B >= 256 && B <= 65536 && !P->sel_multi && q.cutoff_mode != CUSFFT_CUTOFF_SORT;
   if (const char* e = std::getenv("CUSFFT_SELECT")) {
@@ -705,8 +714,9 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       ranges = {{0, P->Lg}};
     if (const char* em = std::getenv("CUSFFT_STAGE_MODE")) {  // fused_index | fused_scatter | split_index | split_scatter
       const std::string m(em);
-      P->stage_split = m.rfind("split", 0) == 0;
-      P->stage_scatter = m.find("scatter") != std::string::npos;
+      P->stage_atomic = m == "atomic";
+      P->stage_split = m.rfind("split", 0) == 0 || P->stage_atomic;
+      P->stage_scatter = m.find("scatter") != std::string::npos || P->stage_atomic;
     }
     {  // packed (slot, i) schedule words: fused scatter mode when local slot and tap index fit 32 bits
       int ib = 1;
@@ -716,6 +726,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       const char* ep = std::getenv("CUSFFT_PACKED");
       P->stage_ibits = ib;
       P->stage_packed = P->stage_scatter && !P->stage_split && ib + sb <= 32 && !(ep && ep[0] == '0');
+      if (P->stage_atomic && ib + sb > 32) P->stage_atomic = P->stage_split = false;
+      P->stage_packed = P->stage_packed || P->stage_atomic;
     }
     int64_t maxtot = 0, sumtot = 0;  // staging elements: w per slot (index mode) or R B per slot (scatter mode)
     for (auto& r : ranges) {
@@ -785,7 +797,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
           if ((rc = upload(gg.inv, inv.data(), inv.size() * sizeof(uint32_t)))) return fail(rc);
         }
       }
-      if ((rc = dalloc(&P->d_staging, (size_t)maxtot))) return fail(rc);
+      if ((rc = dalloc(&P->d_staging, P->stage_atomic ? (size_t)1 : (size_t)maxtot))) return fail(rc);
       {
         int64_t off = 0;
         for (auto& g : P->groups) {
@@ -796,7 +808,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       // Persisting-L2 set-aside for the staging buffer (a device-wide limit: raised, never lowered).
       int maxp = 0;
       cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev);
-      const size_t win = std::min<size_t>((size_t)maxtot * 16, (size_t)maxp);
+      const size_t win = P->stage_atomic ? 0 : std::min<size_t>((size_t)maxtot * 16, (size_t)maxp);
       size_t cur = 0;
       cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
       if (win > cur) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, win);
@@ -904,7 +916,14 @@ int launch_stage1(cusfft_plan_t P, const cusfft_plan_s::StageGroup& g, const dou
   const int grid = std::max(1, std::min((tot + 8 * 256 - 1) / (8 * 256), sms * P->stage_cps));
   g_apw = P->stage_window;  // keep the staging buffer L2-resident for phase 2
   cudaError_t e;
-  if (g.code) {
+  if (g.code && P->stage_atomic) {
+    double2* u = P->d_u + (size_t)g.s0 * P->B;
+    CK(cudaMemsetAsync(u, 0, (size_t)(g.s1 - g.s0) * P->B * sizeof(double2), st));
+    StagePackArgs a{x, g.code, nullptr, P->d_slots + (size_t)P->lrank * P->Lg + g.s0, tot, g.s1 - g.s0,
+                    P->stage_ibits, P->R, ilog2(P->B), P->logB2, P->logB1, ilog2(256 / P->B1),
+                    (uint32_t)(P->n - 1), z};
+    e = launch_k(k_stage_atomic, dim3(grid), dim3(256), 0, st, P->cur_prio, a, (const double*)P->d_taps, u);
+  } else if (g.code) {
     StagePackArgs a{x, g.code, g.staging, P->d_slots + (size_t)P->lrank * P->Lg + g.s0, tot, g.s1 - g.s0,
                     P->stage_ibits, P->R, ilog2(P->B), P->logB2, P->logB1, ilog2(256 / P->B1),
                     (uint32_t)(P->n - 1), z};
@@ -923,6 +942,7 @@ int launch_stage2(cusfft_plan_t P, const cusfft_plan_s::StageGroup& g, cudaStrea
   const int B = (int)P->B;
   g_pdl = !P->timing;
   cudaError_t e;
+  if (P->stage_atomic) return CUSFFT_SUCCESS;  // phase 1 already summed the buckets into u
   if (P->stage_split) {
     dim3 grid2((unsigned)(B / 256), (unsigned)(g.s1 - g.s0));
     if (g.dst)
@@ -993,6 +1013,7 @@ int launch_fold(cusfft_plan_t P, const double2* x, int s0, int s1, cudaStream_t 
       if (g.s1 <= s0 || g.s0 >= s1) continue;  // callers pass whole groups
       int rc;
       if ((rc = launch_stage1(P, g, x, st, z))) return rc;
+      if (&g == &P->groups.front()) mark(P, 7);
       if (!P->skip_stage) z = ZeroArgs{nullptr, 0};
       if ((rc = launch_stage2(P, g, st, z))) return rc;
     }
@@ -1298,6 +1319,66 @@ int launch_branched_staged(cusfft_plan_t P, const double2* x, int64_t* locs, dou
   return launch_output(P, locs, vals, a);
 }
 
+// Two branches after ONE address-ordered phase 1 of all slots (the DRAM pass
+// stays whole): the location slots' phase 2, FFT pass 2, cutoff and vote on
+// the high-priority stream, the estimation slots' phase 2 and FFT pass 2 on a
+// second stream (filling the SMs the latency-bound chain leaves idle); they
+// join before the estimation.
+int launch_branched_p2(cusfft_plan_t P, const double2* x, int64_t* locs, double2* vals) {
+  cudaStream_t a = P->stream, b = P->cap_stream2;
+  const auto& g = P->groups[0];
+  const int nl = P->nloc_local, B = (int)P->B;
+  const SlotParam* sp = P->d_slots + (size_t)P->lrank * P->Lg;
+  const ZeroArgs z0{nullptr, 0};
+  int rc;
+  // the estimation branch, forked from stream a at the current point
+  auto fork = [&]() -> int {
+    CK(cudaEventRecord(P->ev_fork, a));
+    CK(cudaStreamWaitEvent(b, P->ev_fork, 0));
+    P->cur_prio = P->prio_lo;
+    g_pdl = false;
+    CK(launch_fold_fft1(P, g.staging + (size_t)nl * P->R * B, nullptr, sp + nl, P->d_u + (size_t)nl * B,
+                        P->d_v + (size_t)nl * B, P->Lg - nl, z0, b, true));
+    g_pdl = true;
+    int r = launch_bfft(P, nl, P->Lg, b);
+    if (r) return r;
+    CK(cudaEventRecord(P->ev_join, b));
+    P->cur_prio = P->prio_hi;
+    // the next kernel on a keeps its programmatic edge to its predecessor on a
+    // (the fork's event record adds no node): its CTAs become resident early,
+    // ahead of the estimation branch's
+    g_pdl = true;
+    return CUSFFT_SUCCESS;
+  };
+  P->cur_prio = P->prio_hi;
+  g_pdl = false;
+  if ((rc = launch_stage1(P, g, x, a, ZeroArgs{P->d_zero, P->nzero}))) return rc;
+  g_pdl = true;
+  if (P->branch_fork == 0 && (rc = fork())) return rc;
+  CK(launch_fold_fft1(P, g.staging, nullptr, sp, P->d_u, P->d_v, nl, z0, a, true));
+  g_pdl = true;
+  if (P->branch_fork == 1 && (rc = fork())) return rc;
+  if ((rc = launch_bfft(P, 0, nl, a))) return rc;
+  g_pdl = true;
+  if (P->branch_fork == 2 && (rc = fork())) return rc;
+  if ((rc = launch_select(P, a))) return rc;
+  g_pdl = true;
+  if (P->branch_fork == 3 && (rc = fork())) return rc;
+  if ((rc = launch_vote(P, a))) return rc;
+  P->cur_prio = 0;
+  CK(cudaStreamWaitEvent(a, P->ev_join, 0));
+  g_pdl = false;
+  if ((rc = launch_estimate(P, a))) return rc;
+  g_pdl = true;
+  return launch_output(P, locs, vals, a);
+}
+
+inline bool use_branch_p2(cusfft_plan_t P) {
+  return P->branch_p2 && !P->slot_fused && P->use_graph && !P->timing && P->stage_limit == 6 && P->nloc_local > 0 &&
+         P->nloc_local < P->Lg && P->staged && P->groups.size() == 1 && P->stage_scatter && !P->stage_split &&
+         !P->skip_stage && !P->xshard;
+}
+
 // Branched execution only inside graph capture, for full-stage runs with both
 // location and estimation-only slots on this rank.
 inline bool use_branches(cusfft_plan_t P) {
@@ -1379,6 +1460,7 @@ int execute_full(cusfft_plan_t plan, const void* d_x, int64_t* d_locs, void* d_v
   return run_graphed(plan, full_entry(plan, d_x, d_locs, d_vals), plan->g_full_t, d_x, d_locs, d_vals, [&] {
     const double2* x = reinterpret_cast<const double2*>(d_x);
     double2* v = reinterpret_cast<double2*>(d_vals);
+    if (use_branch_p2(plan)) return launch_branched_p2(plan, x, d_locs, v);
     if (use_branches(plan))
       return plan->staged ? launch_branched_staged(plan, x, d_locs, v) : launch_branched(plan, x, d_locs, v);
     int rc = launch_local(plan, x);
@@ -1585,6 +1667,7 @@ int cusfft_execute_host(cusfft_plan_t plan, const void* h_x, int64_t* h_locs, vo
   CK(cudaMemcpyAsync(plan->d_xbuf, h_x, (size_t)plan->n * 16, cudaMemcpyHostToDevice, st));
   rc = run_graphed(plan, full_entry(plan, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf), plan->g_full_t,
                    plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf, [&] {
+    if (use_branch_p2(plan)) return launch_branched_p2(plan, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf);
     if (use_branches(plan))
       return plan->staged ? launch_branched_staged(plan, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf)
                           : launch_branched(plan, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf);
@@ -1724,6 +1807,14 @@ int cusfft_get_stage_times(cusfft_plan_t plan, float* ms, int32_t cap) {
     }
     ms[i] = t;
   }
+  if (cap >= 7) {
+    float t = -1.f;
+    if (!plan->staged || cudaEventElapsedTime(&t, plan->ev[0], plan->ev[7]) != cudaSuccess) {
+      t = -1.f;
+      cudaGetLastError();
+    }
+    ms[6] = t;
+  }
   return CUSFFT_SUCCESS;
 }
 
@@ -1758,6 +1849,7 @@ int32_t cusfft_launches_per_execute(cusfft_plan_t plan) {
   int n = (plan->staged ? 2 * (int)plan->groups.size() : 1) /*stage + fold per group*/ + (pass1 ? 2 : 1) /*fft*/ +
           (plan->sel_slots_h.empty() ? 0 : 1) + (plan->xshard && !plan->sel_slots_h.empty() ? 1 : 0) /*keys*/ +
           3 /*vote,est,out*/;
+  if (use_branch_p2(plan)) n += 2;  // phase 2 and FFT pass 2 launched per branch
   return n;
 }
 

@@ -209,6 +209,57 @@ __global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
   TRACE_END(6);
 }
 
+// Atomic form of phase 1 (opt-in, CUSFFT_STAGE_MODE=atomic): the same
+// address-ordered gathers, each multiplied by its tap g_i and added straight
+// into u_s[i mod B] with fp64 L2 reductions (u zeroed by a memset node), so
+// there is no staging round trip; the FFT pass 1 then reads u.  The order of
+// the additions into a bucket is whatever order the L2 sees them in, so u is
+// reproducible only to rounding (not bit-exact with Alg. 1's order).
+__global__ void __launch_bounds__(256) k_stage_atomic(StagePackArgs A, const double* __restrict__ taps,
+                                                      double2* __restrict__ u) {
+  pdl_wait();
+  KTRACE(1);
+  if (blockIdx.x == 0) TRACE(0);
+  __shared__ uint32_t ssig[kMaxLoops], stau[kMaxLoops];
+  for (int i = threadIdx.x; i < A.nslots; i += blockDim.x) {
+    ssig[i] = A.slots[i].sigma;
+    stau[i] = A.slots[i].tau;
+  }
+  zero_part(A.zero);
+  __syncthreads();
+  const uint64_t pf = l2_policy_first();
+  const uint32_t imask = (1u << A.ibits) - 1u;
+  const uint32_t Bm = (1u << A.logB) - 1u;
+  const int T = gridDim.x * blockDim.x;
+  for (int q0 = blockIdx.x * blockDim.x + threadIdx.x; q0 < A.total; q0 += 8 * T) {
+    double2 v[8];
+    uint32_t cd[8];
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      const int q = q0 + c * T;
+      if (q < A.total) {
+        cd[c] = __ldg(A.code + q);
+        const uint32_t sl = cd[c] >> A.ibits, i = cd[c] & imask;
+        const double2* p = A.x + ((ssig[sl] * i + stau[sl]) & A.nmask);
+        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.L2::64B.v2.f64 {%0, %1}, [%2], %3;"
+                     : "=d"(v[c].x), "=d"(v[c].y) : "l"(p), "l"(pf));
+      }
+    }
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      const int q = q0 + c * T;
+      if (q < A.total) {
+        const uint32_t sl = cd[c] >> A.ibits, i = cd[c] & imask;
+        const double g = __ldg(taps + i);
+        double* o = reinterpret_cast<double*>(u + ((sl << A.logB) | (i & Bm)));
+        asm volatile("red.relaxed.gpu.global.add.f64 [%0], %1;" ::"l"(o), "d"(__dmul_rn(g, v[c].x)) : "memory");
+        asm volatile("red.relaxed.gpu.global.add.f64 [%0], %1;" ::"l"(o + 1), "d"(__dmul_rn(g, v[c].y)) : "memory");
+      }
+    }
+  }
+  TRACE_END(6);
+}
+
 // ---------------------------------------------------------------------------
 // Staged gather, phase 2 without the FFT (split mode): thread per (slot,
 // bucket j), natural order.  SCATTER: staging[(s R + rr) B + j] holds round

@@ -62,12 +62,14 @@ if os.path.exists(rep):
         if "k_stage" in n or "k_fold" in n:
             rd = float(r[hdr.index("dram__bytes_read.sum")]) * scale[units["dram__bytes_read.sum"]]
             wr = float(r[hdr.index("dram__bytes_write.sum")]) * scale[units["dram__bytes_write.sum"]]
-            fold_parts[n] = (rd, wr)
+            a = fold_parts.get(n, (0.0, 0.0))  # several launches per execution (branched graph): summed
+            fold_parts[n] = (a[0] + rd, a[1] + wr)
 if fold_parts:
     rd = sum(v[0] for v in fold_parts.values())
     wr = sum(v[1] for v in fold_parts.values())
     traffic = {"kernel": " + ".join(sorted(fold_parts)), "config": "C3", "source": f"{tag}_ncu_summary.md (ncu --set full)",
-               "parts": {k: {"dram_bytes_read": v[0], "dram_bytes_write": v[1]} for k, v in fold_parts.items()},
+               "parts": {k: {"dram_bytes_read": v[0], "dram_bytes_write": v[1], "dram_bytes_per_launch": v[0] + v[1]}
+                         for k, v in fold_parts.items()},
                "dram_bytes_read": rd, "dram_bytes_write": wr, "dram_bytes_per_launch": rd + wr}
 if traffic:
     json.dump(traffic, open(f"{P}/fold_traffic_C3.json", "w"), indent=1)
