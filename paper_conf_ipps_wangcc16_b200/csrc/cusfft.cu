@@ -112,6 +112,7 @@ struct cusfft_plan_s {
   int select_smem = 0, vote_smem = 0, output_smem = 0;
   int vote_grid = 1, est_grid = 1;
   int fft_smem1 = 0, fft_smem2 = 0;
+  int fft_E = 512;                // elements per CTA of the FFT passes (CUSFFT_FFT_E=256|512|1024; 512 measured best at C3)
   std::vector<SlotParam> slots_h;       // slot order
   std::vector<int64_t> a_r, sigma_r, tau_r;  // loop order
   std::vector<int> loc_slots_h, sel_slots_h;
@@ -174,6 +175,8 @@ struct cusfft_plan_s {
   int* d_ccount = nullptr;        // [n_sel] candidate counters (self-resetting)
   int* d_done = nullptr;          // [n_sel] finished-CTA counters (self-resetting)
   int sel_S = 1;                  // CTAs per location loop in k_select
+  bool pk_direct = false;         // the cutoff writes k_vote8's byte-per-bucket array (d_pk, in the zero block)
+  uint32_t* d_pk = nullptr;
   bool vote_packed = false;       // k_vote8 (L_loc <= 8, B <= 16384; CUSFFT_VOTE_BITMAP=1 forces k_vote)
   int vote8_grid = 1;
   bool vote_pairs = true;         // k_vote8 pair enumeration when T > ceil(L_loc/2) (CUSFFT_VOTE_PAIRS=0: off)
@@ -405,15 +408,27 @@ cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem,
   return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
 }
 
-template <int M>
-constexpr int fft_E() { return M < 1024 ? 1024 : M; }
+// Elements per CTA of the batched B1/B2-point FFT passes: g_fft_E (1024
+// default; CUSFFT_FFT_E=512|256 for more, smaller CTAs), at least M.
+thread_local int g_fft_E = 1024;
+
+template <int M, int E>
+cudaError_t launch_fft_e(const FftPassArgs& a, int smem, cudaStream_t st, int prio) {
+  constexpr int NSEQ = E / M;
+  const int grid = (a.total_seq + NSEQ - 1) / NSEQ;
+  return launch_k(k_fft<M, E, 128>, dim3(grid), dim3(128), fft_smem_bytes(E), st, prio, a);
+}
 
 template <int M>
 cudaError_t launch_fft_t(const FftPassArgs& a, int smem, cudaStream_t st, int prio) {
-  constexpr int E = fft_E<M>();
-  constexpr int NSEQ = E / M;
-  const int grid = (a.total_seq + NSEQ - 1) / NSEQ;
-  return launch_k(k_fft<M, E, 128>, dim3(grid), dim3(128), smem, st, prio, a);
+  (void)smem;
+  if constexpr (M >= 1024) {
+    return launch_fft_e<M, M>(a, 0, st, prio);
+  } else {
+    if (g_fft_E <= 256 && M <= 256) return launch_fft_e<M, (M < 256 ? 256 : M)>(a, 0, st, prio);
+    if (g_fft_E <= 512 && M <= 512) return launch_fft_e<M, 512>(a, 0, st, prio);
+    return launch_fft_e<M, 1024>(a, 0, st, prio);
+  }
 }
 
 cudaError_t launch_fft(int M, const FftPassArgs& a, int smem, cudaStream_t st, int prio = 0) {
@@ -434,10 +449,27 @@ cudaError_t launch_fft(int M, const FftPassArgs& a, int smem, cudaStream_t st, i
   }
 }
 
+template <int M, int E>
+cudaError_t set_fft_attr_e() {
+  return cudaFuncSetAttribute(k_fft<M, E, 128>, cudaFuncAttributeMaxDynamicSharedMemorySize, fft_smem_bytes(E));
+}
+
 template <int M>
 cudaError_t set_fft_attr_t() {
-  return cudaFuncSetAttribute(k_fft<M, fft_E<M>(), 128>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                              fft_smem_bytes(fft_E<M>()));
+  if constexpr (M >= 1024) {
+    return set_fft_attr_e<M, M>();
+  } else {
+    cudaError_t e = set_fft_attr_e<M, 1024>();
+    if constexpr (M <= 512) {
+      cudaError_t e2 = set_fft_attr_e<M, 512>();
+      if (e2 != cudaSuccess) e = e2;
+    }
+    if constexpr (M <= 256) {
+      cudaError_t e3 = set_fft_attr_e<M, (M < 256 ? 256 : M)>();
+      if (e3 != cudaSuccess) e = e3;
+    }
+    return e;
+  }
 }
 
 cudaError_t set_fft_attrs() {
@@ -529,6 +561,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   if (const char* e = std::getenv("CUSFFT_STAGE_CPS")) P->stage_cps = std::max(1, std::atoi(e));
   if (const char* e = std::getenv("CUSFFT_P2")) P->p2_tma = std::string(e) != "ldg";
   if (const char* e = std::getenv("CUSFFT_DISCARD")) P->p2_discard = (e[0] == '1');
+  if (const char* e = std::getenv("CUSFFT_FFT_E")) P->fft_E = std::max(256, std::min(1024, std::atoi(e)));
 
   // ---- draws (loop order), Alg. 1, Def. 1
   SplitMix64 rng{q.seed};
@@ -617,7 +650,10 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     const size_t nsel = std::max<size_t>(1, P->sel_slots_h.size());
     if ((rc = dalloc(&P->d_keys, nsel * B))) return fail(rc);
     // per-execution counters and histograms: one block, zeroed by the first fold kernel
-    P->nzero = 8 + (int)(2 * nsel * 4096 + 4096 + 2 * nsel);
+    // cutoff-built vote bytes: every location loop selected on this rank, cluster cutoff, k_vote8
+    P->pk_direct = P->vote_packed && P->sel_cluster && P->sel_slots_h == P->loc_slots_h && B % 32 == 0 &&
+                   !(std::getenv("CUSFFT_PK") && std::getenv("CUSFFT_PK")[0] == '0');
+    P->nzero = 8 + (int)(2 * nsel * 4096 + 4096 + 2 * nsel) + (P->pk_direct ? (int)(B / 4) : 0);
     if ((rc = dalloc(&P->d_zero, (size_t)P->nzero))) return fail(rc);
     P->d_flags = P->d_zero;
     P->d_hist = reinterpret_cast<uint32_t*>(P->d_zero + 8);
@@ -625,6 +661,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     P->d_ohist = P->d_hist1 + nsel * 4096;
     P->d_ccount = reinterpret_cast<int*>(P->d_ohist + 4096);
     P->d_done = P->d_ccount + nsel;
+    if (P->pk_direct) P->d_pk = reinterpret_cast<uint32_t*>(P->d_done + nsel);
     if ((rc = dalloc(&P->d_key_index, (size_t)P->Lg))) return fail(rc);
 
     if ((rc = dalloc(&P->d_ckey, nsel * kSelCap))) return fail(rc);
@@ -1032,6 +1069,7 @@ int launch_bfft(cusfft_plan_t P, int s0, int s1, cudaStream_t st) {
   if (s1 <= s0) return CUSFFT_SUCCESS;
   const int B = (int)P->B;
   const int ns = s1 - s0;
+  g_fft_E = P->fft_E;
   double2* rec = reinterpret_cast<double2*>(P->d_records + ((int64_t)P->lrank * P->Lg + s0) * P->lay.rec_bytes);
   const int64_t rec_e = P->lay.rec_bytes / 16;
   // signal-sharded: the spectra are partial here, keys come after the all-reduce (launch_keys)
@@ -1071,6 +1109,7 @@ SelArgs make_sel_args(cusfft_plan_t P) {
   sa.ccount = P->d_ccount;
   sa.done = P->d_done;
   sa.status = P->d_flags + 1;
+  sa.pk = P->d_pk;
   sa.threshold_mode = P->prm.cutoff_mode == CUSFFT_CUTOFF_THRESHOLD ? 1 : 0;
   {
     const double th = P->prm.cutoff_threshold;
@@ -1195,6 +1234,7 @@ int launch_vote(cusfft_plan_t P, cudaStream_t st) {
   va.hits = P->d_hits;
   va.hit_count = reinterpret_cast<unsigned*>(P->d_flags);
   va.max_hits = P->max_hits;
+  va.pk = P->d_pk;
   if (P->vote_packed) {  // L_loc <= 8, B <= kPk: byte-per-bucket probes, one CTA per SM
     CK(launch_k(k_vote8, dim3(P->vote8_grid), dim3(1024), 0, st, P->cur_prio, va));
     return CUSFFT_SUCCESS;

@@ -690,6 +690,10 @@ struct SelArgs {
   int* ccount;           // [n_sel]
   int* done;             // [n_sel]
   int* status;
+  // optional (single-rank plans with every location loop selected here): the
+  // vote's byte-per-bucket array (bit q = bucket kept in location loop q,
+  // selection index == vote index), ORed in by the cutoff; zeroed per execution
+  uint32_t* pk;
 };
 
 struct GKeySrc {
@@ -1224,6 +1228,18 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
   uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap) + r * wpc;
   int* J = reinterpret_cast<int*>(rec + A.lay.off_J);
   for (int w = tid; w < wpc; w += kSelCNT) bitmap[w] = sbits[w];
+  if (A.pk) {  // bucket 32 gw + 4 j + i -> byte i of word gw 8 + j, bit sel (k_vote8's layout)
+    for (int w = tid; w < wpc; w += kSelCNT) {
+      const uint32_t bits = sbits[w];
+      if (!bits) continue;
+      uint32_t* dst = A.pk + (int64_t)(r * wpc + w) * 8;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        const uint32_t nib = (bits >> (4 * j)) & 0xFu;
+        if (nib) atomicOr(dst + j, ((nib * 0x00204081u) & 0x01010101u) << sel);
+      }
+    }
+  }
   pos += jofs;
   for (int w = tid * wpt; w < min(wpc, (tid + 1) * wpt); ++w) {
     uint32_t bits = sbits[w];
@@ -1549,6 +1565,7 @@ struct VoteArgs {
   int* hits;
   unsigned* hit_count;
   int max_hits;
+  const uint32_t* pk;  // k_vote8: the byte-per-bucket array already built by the cutoff (or null: transpose bmp)
 };
 
 // Scaled arithmetic: with F = f << (32 - log2 n), sigma * F + (nb/2 << (32 - log2 n))
@@ -1932,7 +1949,12 @@ __global__ void __launch_bounds__(1024, 1) k_vote8(VoteArgs A) {
   const int tid = threadIdx.x;
   const int words = (A.B + 31) >> 5;
   // transpose: bucket 32 w + 4 j + i -> byte (w 8 + j) * 4 + i, bit q = loop q
-  for (int w = tid; w < words; w += 1024) {
+  // (or copy it: the cutoff already ORed the bits into A.pk)
+  if (A.pk) {
+    for (int i = tid; i < (words << 1); i += 1024)
+      reinterpret_cast<uint4*>(pk)[i] = __ldcg(reinterpret_cast<const uint4*>(A.pk) + i);
+  }
+  for (int w = A.pk ? words : tid; w < words; w += 1024) {
     uint32_t bw[8];
 #pragma unroll
     for (int q = 0; q < 8; ++q) bw[q] = q < A.Lloc ? __ldg(A.bmp[q] + w) : 0u;
@@ -1963,7 +1985,7 @@ __global__ void __launch_bounds__(1024, 1) k_vote8(VoteArgs A) {
   uint8_t* qG = queueG[tid >> 5];
   const int warp = (blockIdx.x * 1024 + tid) >> 5;
   const int nwarps = gridDim.x * 32;
-  if (A.pairs) {
+  if (A.pairs) {  // unit = (pair, winner J, part h of its nb candidates), split parts per winner
     for (int unit = warp; unit < units; unit += nwarps) {
       int pr = 0;
       while (unit >= scnt[pr + 1]) ++pr;

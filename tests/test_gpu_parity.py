@@ -294,17 +294,20 @@ def test_parity_snr_sweep(snr_db):
                                  {"CUSFFT_STAGE_MODE": "split_scatter"}, {"CUSFFT_NO_STAGE": "1"},
                                  {"CUSFFT_STAGE_MODE": "fused_index"}, {"CUSFFT_P2": "ldg"}, {"CUSFFT_DISCARD": "0"},
                                  {"CUSFFT_SLOT": "1"}, {"CUSFFT_SLOT": "2"}, {"CUSFFT_BRANCH": "1"}, {"CUSFFT_BRANCH": "2"}, {"CUSFFT_BRANCH": "3"}, {"CUSFFT_BRANCH": "4"}, {"CUSFFT_BRANCH": "5"},
-                                 {"CUSFFT_STAGE_GROUPS": "2"}, {"CUSFFT_PACKED": "0"}])
+                                 {"CUSFFT_STAGE_GROUPS": "2"}, {"CUSFFT_PACKED": "0"},
+                                 {"CUSFFT_FFT_E": "1024"}, {"CUSFFT_FFT_E": "256"}, {"CUSFFT_PK": "0"}, {"CUSFFT_BRANCH": "0"}])
 def test_kernel_variants_agree(env, monkeypatch):
     """Every alternative kernel path (selected at plan time by environment
     switches, used for A/B measurements) gives the default path's hits and
     output exactly (same fold order, same selection rule)."""
     import torch
     from paper_conf_ipps_wangcc16_b200 import Plan
-    n, k = 2 ** 20, 100
+    # n = 2^22, k = 1000: B = 8192, two FFT passes, staged fold, branched graph
+    n, k = 2 ** 22, 1000
     x, S, X = planted_signal(n, k, seed=21)
     xd = torch.from_numpy(x).cuda()
     base = Plan(n, k, L=16, seed=4, debug=1)
+    assert base.info()["staged"]
     l0, v0 = base.execute(xd)
     h0 = np.sort(base.debug(DEBUG_HITS))
     for key, val in env.items():
