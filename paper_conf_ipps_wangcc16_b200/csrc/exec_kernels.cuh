@@ -2164,24 +2164,83 @@ __global__ void __launch_bounds__(1024) k_output(const int* __restrict__ hits, c
   const int H = min((int)hc, max_hits);
   if (tid == 0 && (int)hc > max_hits) atomicOr(status, 1);
   const int K = min(k, H);
+  // Fast path (H <= 4096 items, k <= 2048): every item's key, f and value are
+  // loaded into registers while the level-0 boundary bin is found; if that
+  // bin is taken whole (the usual case: the k planted coefficients stand far
+  // above the false hits), one classification pass selects, and the values
+  // go to shared memory (aliasing the unused candidate arrays), so neither the
+  // sort nor the write-out touches global memory again.
+  constexpr int PF = 4;
+  double2* selv = reinterpret_cast<double2*>(ckey);  // [kp2] values of the selected entries (fast path)
+  const bool fast = H <= PF * 1024 && kp2 * 16 <= kOutCap * 12;
+  uint64_t pk[PF];
+  uint32_t pf[PF];
+  double2 pv[PF];
+  if (fast) {
+#pragma unroll
+    for (int u = 0; u < PF; ++u) {
+      const int i = u * 1024 + tid;
+      if (i < H) {
+        pk[u] = __ldg(hit_keys + i);
+        pf[u] = (uint32_t)__ldg(hits + i);
+        pv[u] = __ldg(hit_vals + i);
+      }
+    }
+  }
   if (tid == 0) sm[41] = 0;
   bcnt[tid] = 0;
-  __syncthreads();
-  auto add = [&](int i) {
-    const int pos = atomicAdd(&sm[41], 1);
-    if (pos < kp2) sel[pos] = ((uint64_t)(uint32_t)__ldg(hits + i) << 32) | (uint32_t)i;
-  };
-  if (H > K) {
-    select_topk(
-        H, K, ghist,
-        [&](int i, uint64_t& kk, uint32_t& t) {
-          kk = __ldg(hit_keys + i);
-          t = (uint32_t)__ldg(hits + i);
-        },
-        add, ckey, cidx, kOutCap, hist, sm);
+  bool direct = false;  // selv holds the values
+  if (fast) {
+    uint32_t d0 = 0;
+    bool whole = true;
+    if (H > K) {
+      const BinPick b0 = pick_bin(ghist, K, sm);  // syncs
+      d0 = (uint32_t)b0.d;
+      whole = (K - b0.above) == b0.cnt;
+    } else {
+      __syncthreads();
+    }
+    if (whole) {
+      direct = true;
+      const int lane = tid & 31;
+#pragma unroll
+      for (int u = 0; u < PF; ++u) {
+        const int i = u * 1024 + tid;
+        const bool take = i < H && ((uint32_t)(pk[u] >> 51) & 0xFFFu) >= d0;
+        const unsigned bal = __ballot_sync(kFull, take);
+        int base = 0;
+        if (lane == 0 && bal) base = atomicAdd(&sm[41], __popc(bal));
+        base = __shfl_sync(kFull, base, 0);
+        if (take) {
+          const int pos = base + __popc(bal & ((1u << lane) - 1u));
+          if (pos < kp2) {
+            sel[pos] = ((uint64_t)pf[u] << 32) | (uint32_t)pos;
+            selv[pos] = pv[u];
+          }
+        }
+      }
+      __syncthreads();
+    }
   } else {
-    for (int i = tid; i < H; i += 1024) add(i);
     __syncthreads();
+  }
+  if (!direct) {
+    auto add = [&](int i) {
+      const int pos = atomicAdd(&sm[41], 1);
+      if (pos < kp2) sel[pos] = ((uint64_t)(uint32_t)__ldg(hits + i) << 32) | (uint32_t)i;
+    };
+    if (H > K) {
+      select_topk(
+          H, K, ghist,
+          [&](int i, uint64_t& kk, uint32_t& t) {
+            kk = __ldg(hit_keys + i);
+            t = (uint32_t)__ldg(hits + i);
+          },
+          add, ckey, cidx, kOutCap, hist, sm);
+    } else {
+      for (int i = tid; i < H; i += 1024) add(i);
+      __syncthreads();
+    }
   }
   TRACE(51);
   const int ns = min(sm[41], kp2);
@@ -2240,7 +2299,7 @@ __global__ void __launch_bounds__(1024) k_output(const int* __restrict__ hits, c
     if (j < ns) {
       const uint64_t v = srt[j];
       locs[j] = (int64_t)(v >> 32);
-      vals[j] = hit_vals[(uint32_t)v];
+      vals[j] = direct ? selv[(uint32_t)v] : hit_vals[(uint32_t)v];
     } else {
       locs[j] = -1;
       vals[j] = make_double2(0.0, 0.0);
