@@ -188,7 +188,9 @@ int32_t cusfft_exchange_kind(cusfft_plan_t plan);
 int cusfft_get_info(cusfft_plan_t plan, int64_t* info, int64_t* a, int64_t* sigma, int64_t* tau);
 
 typedef enum {
-  CUSFFT_DEBUG_U = 0,        /* complex fp64 [L_local][B]: fold output, this rank's loops  */
+  CUSFFT_DEBUG_U = 0,        /* complex fp64 [L_local][B]: fold output, this rank's loops;
+                                 staged plans write it only with params.debug = 1 (else
+                                 CUSFFT_INVALID_PARAM)                                      */
   CUSFFT_DEBUG_UHAT = 1,     /* complex fp64 [L][B]: B-point FFTs, loop order                */
   CUSFFT_DEBUG_WINNERS = 2,  /* int32 [L_loc][cap]: kept buckets, ascending, -1 padded; cap =
                                 num_select (B in THRESHOLD mode)                              */

@@ -46,6 +46,15 @@ struct KTraceScope {
 // for ordinary launches.
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 
+// Early launch of the dependent kernel (programmatic dependent launch): kernel
+// `bit` of the chain lets its successor's CTAs become resident (they block in
+// pdl_wait until this grid completes) when bit is set in c_pdl_trigger
+// (CUSFFT_PDL_TRIGGER, process-wide, set at plan creation; A/B switch).
+__constant__ int c_pdl_trigger;
+__device__ __forceinline__ void pdl_trigger(int bit) {
+  if ((c_pdl_trigger >> bit) & 1) asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
 // Bulk (TMA engine) global -> shared copies completing on an mbarrier.
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
 __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {

@@ -201,6 +201,7 @@ struct cusfft_plan_s {
   // CUDA graphs of the launch sequences, keyed by the caller's pointers
   bool use_graph = true;
   bool branched = false;          // two-branch graph (location chain || estimation folds); opt-in
+  bool split_launch = false;      // CUSFFT_SPLIT_LAUNCH=1: phase 1 as a plain launch before the graph of the rest
   int branch_fork = 0;            // CUSFFT_BRANCH=2..5: the estimation branch forks after phase 1 / the location
                                   // slots' phase 2 / their FFT pass 2 / the cutoff
   bool branch_p2 = true;          // CUSFFT_BRANCH=2: one phase 1, then location chain || estimation phase 2 + FFT
@@ -561,6 +562,14 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   if (const char* e = std::getenv("CUSFFT_STAGE_CPS")) P->stage_cps = std::max(1, std::atoi(e));
   if (const char* e = std::getenv("CUSFFT_P2")) P->p2_tma = std::string(e) != "ldg";
   if (const char* e = std::getenv("CUSFFT_DISCARD")) P->p2_discard = (e[0] == '1');
+  {
+    const char* e = std::getenv("CUSFFT_PDL_TRIGGER");
+    // default: only the estimation lets the output CTA launch early (measured: -0.8 us at C3;
+    // early-resident vote / estimate / FFT CTAs slow their predecessors)
+    const int m = e ? std::atoi(e) : 32;
+    cudaMemcpyToSymbol(c_pdl_trigger, &m, sizeof(int));
+  }
+  if (const char* e = std::getenv("CUSFFT_SPLIT_LAUNCH")) P->split_launch = (e[0] == '1');
   if (const char* e = std::getenv("CUSFFT_FFT_E")) P->fft_E = std::max(256, std::min(1024, std::atoi(e)));
 
   // ---- draws (loop order), Alg. 1, Def. 1
@@ -653,7 +662,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     // cutoff-built vote bytes: every location loop selected on this rank, cluster cutoff, k_vote8
     P->pk_direct = P->vote_packed && P->sel_cluster && P->sel_slots_h == P->loc_slots_h && B % 32 == 0 &&
                    !(std::getenv("CUSFFT_PK") && std::getenv("CUSFFT_PK")[0] == '0');
-    P->nzero = 8 + (int)(2 * nsel * 4096 + 4096 + 2 * nsel) + (P->pk_direct ? (int)(B / 4) : 0);
+    const int pk_off = (8 + (int)(2 * nsel * 4096 + 4096 + 2 * nsel) + 3) & ~3;  // 16-B aligned (uint4 copies)
+    P->nzero = P->pk_direct ? pk_off + (int)(B / 4) : 8 + (int)(2 * nsel * 4096 + 4096 + 2 * nsel);
     if ((rc = dalloc(&P->d_zero, (size_t)P->nzero))) return fail(rc);
     P->d_flags = P->d_zero;
     P->d_hist = reinterpret_cast<uint32_t*>(P->d_zero + 8);
@@ -661,7 +671,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     P->d_ohist = P->d_hist1 + nsel * 4096;
     P->d_ccount = reinterpret_cast<int*>(P->d_ohist + 4096);
     P->d_done = P->d_ccount + nsel;
-    if (P->pk_direct) P->d_pk = reinterpret_cast<uint32_t*>(P->d_done + nsel);
+    if (P->pk_direct) P->d_pk = reinterpret_cast<uint32_t*>(P->d_zero + pk_off);
     if ((rc = dalloc(&P->d_key_index, (size_t)P->Lg))) return fail(rc);
 
     if ((rc = dalloc(&P->d_ckey, nsel * kSelCap))) return fail(rc);
@@ -918,7 +928,7 @@ cudaError_t launch_fold_fft1_t(cusfft_plan_t P, const double2* x, const uint32_t
       attr_set[B1T / 64] = true;
     }
     return launch_k(k_fold_fft1_tma<B1T>, grid, dim3(256), smem, st, P->cur_prio, x,
-                    (const double*)P->d_taps_perm, u, v, (const double2*)P->d_tw, (int)P->B, P->B2, P->w, P->R,
+                    (const double*)P->d_taps_perm, P->prm.debug ? u : nullptr, v, (const double2*)P->d_tw, (int)P->B, P->B2, P->w, P->R,
                     (int)P->p2_discard, z);
   }
   if (staged_tord)  // staged in thread order: x is the group's staging buffer
@@ -938,6 +948,11 @@ cudaError_t launch_fold_fft1(cusfft_plan_t P, const double2* x, const uint32_t* 
     case 256: return launch_fold_fft1_t<256>(P, x, inv, sp, u, v, nslots, z, st, staged_tord);
     default: return cudaErrorInvalidValue;
   }
+}
+
+// The bulk-copy fold + FFT pass 1 writes u only for debug plans (the FFT reads v).
+inline bool u_debug_only(cusfft_plan_t P) {
+  return P->staged && P->stage_scatter && !P->stage_split && P->p2_tma && P->R <= 48 && !(P->slot_fused && P->slot_phase_a);
 }
 
 inline void mark(cusfft_plan_t P, int i) {
@@ -1364,7 +1379,9 @@ int launch_branched_staged(cusfft_plan_t P, const double2* x, int64_t* locs, dou
 // the high-priority stream, the estimation slots' phase 2 and FFT pass 2 on a
 // second stream (filling the SMs the latency-bound chain leaves idle); they
 // join before the estimation.
-int launch_branched_p2(cusfft_plan_t P, const double2* x, int64_t* locs, double2* vals) {
+// stage1_outside: phase 1 was launched directly on the caller's stream just
+// before this graph (so the graph's launch latency overlaps it).
+int launch_branched_p2(cusfft_plan_t P, const double2* x, int64_t* locs, double2* vals, bool stage1_outside = false) {
   cudaStream_t a = P->stream, b = P->cap_stream2;
   const auto& g = P->groups[0];
   const int nl = P->nloc_local, B = (int)P->B;
@@ -1392,9 +1409,10 @@ int launch_branched_p2(cusfft_plan_t P, const double2* x, int64_t* locs, double2
   };
   P->cur_prio = P->prio_hi;
   g_pdl = false;
-  if ((rc = launch_stage1(P, g, x, a, ZeroArgs{P->d_zero, P->nzero}))) return rc;
-  g_pdl = true;
+  if (!stage1_outside && (rc = launch_stage1(P, g, x, a, ZeroArgs{P->d_zero, P->nzero}))) return rc;
+  g_pdl = !stage1_outside;
   if (P->branch_fork == 0 && (rc = fork())) return rc;
+  if (stage1_outside) g_pdl = false;  // the graph's first node on a
   CK(launch_fold_fft1(P, g.staging, nullptr, sp, P->d_u, P->d_v, nl, z0, a, true));
   g_pdl = true;
   if (P->branch_fork == 1 && (rc = fork())) return rc;
@@ -1497,6 +1515,16 @@ cusfft_plan_s::GraphEntry& full_entry(cusfft_plan_t P, const void* a, const void
 }
 
 int execute_full(cusfft_plan_t plan, const void* d_x, int64_t* d_locs, void* d_vals) {
+  if (plan->split_launch && use_branch_p2(plan)) {  // phase 1 launched directly, the rest as a graph
+    const double2* x = reinterpret_cast<const double2*>(d_x);
+    g_pdl = false;
+    plan->cur_prio = 0;
+    int rc = launch_stage1(plan, plan->groups[0], x, plan->stream, ZeroArgs{plan->d_zero, plan->nzero});
+    if (rc) return rc;
+    return run_graphed(plan, full_entry(plan, d_x, d_locs, d_vals), plan->g_full_t, d_x, d_locs, d_vals, [&] {
+      return launch_branched_p2(plan, x, d_locs, reinterpret_cast<double2*>(d_vals), true);
+    });
+  }
   return run_graphed(plan, full_entry(plan, d_x, d_locs, d_vals), plan->g_full_t, d_x, d_locs, d_vals, [&] {
     const double2* x = reinterpret_cast<const double2*>(d_x);
     double2* v = reinterpret_cast<double2*>(d_vals);
@@ -1775,6 +1803,7 @@ int64_t cusfft_get_debug(cusfft_plan_t plan, int32_t what, void* dst, int64_t ca
   uint8_t* out = reinterpret_cast<uint8_t*>(dst);
   switch (what) {
     case CUSFFT_DEBUG_U:
+      if (!plan->prm.debug && u_debug_only(plan)) return CUSFFT_INVALID_PARAM;  // not written
       CK(cudaMemcpy(out, plan->d_u, need, cudaMemcpyDeviceToHost));
       break;
     case CUSFFT_DEBUG_UHAT:

@@ -164,6 +164,7 @@ struct StagePackArgs {
 };
 
 __global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
+  pdl_trigger(0);
   pdl_wait();
   KTRACE(1);
   if (blockIdx.x == 0) TRACE(0);
@@ -432,7 +433,7 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict_
   // elements from neighbouring threads (full 32-B sectors when C >= 2)
   const int wc = t % C, wj = t / C;  // writer's (column, row)
   const size_t wpos = (size_t)s * B + (size_t)blockIdx.x * C + wc + (size_t)B2 * wj;
-  u[wpos] = S[fft_pad(wc * B1T + wj)];
+  if (u) u[wpos] = S[fft_pad(wc * B1T + wj)];  // the fold output itself: debug plans only
   __syncthreads();
   fft_smem<B1T, 256, 256, true>(S, twl, B1T);
   // v = FFT result times omega_B^(c k1); the writer's own twiddle
@@ -459,6 +460,7 @@ __global__ void __launch_bounds__(256, 4) k_fold_fft1_tma(const double2* __restr
                                                           double2* __restrict__ u, double2* __restrict__ v,
                                                           const double2* __restrict__ tw, int B, int B2, int w, int R,
                                                           int discard, ZeroArgs zero) {
+  pdl_trigger(1);
   pdl_wait();
   KTRACE(2);
   constexpr int C = 256 / B1T;
@@ -513,7 +515,7 @@ __global__ void __launch_bounds__(256, 4) k_fold_fft1_tma(const double2* __restr
   __syncthreads();
   const int wc = t % C, wj = t / C;
   const size_t wpos = (size_t)s * B + (size_t)blockIdx.x * C + wc + (size_t)B2 * wj;
-  u[wpos] = S[fft_pad(wc * B1T + wj)];
+  if (u) u[wpos] = S[fft_pad(wc * B1T + wj)];  // the fold output itself: debug plans only
   __syncthreads();
   fft_smem<B1T, 256, 256, true>(S, twl, B1T);
   const double2 wv = __ldg(tw + (((int64_t)(blockIdx.x * C + wc) * wj) & (B - 1)));
@@ -1258,6 +1260,7 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
 }
 
 __global__ void __launch_bounds__(kSelCNT, 1) k_select_cluster(SelArgs A) {
+  pdl_trigger(3);
   pdl_wait();
   KTRACE(8);
   extern __shared__ __align__(16) uint8_t smem[];
@@ -1938,6 +1941,7 @@ __device__ __forceinline__ void vote8_pair_unit(const VoteArgs& A, const uint8_t
 }
 
 __global__ void __launch_bounds__(1024, 1) k_vote8(VoteArgs A) {
+  pdl_trigger(4);
   pdl_wait();
   KTRACE(9);
   __shared__ __align__(16) uint8_t pk[kPk];
@@ -2084,6 +2088,7 @@ __device__ __forceinline__ double warp_rank_select(double a0, double a1, int L, 
 }
 
 __global__ void __launch_bounds__(256) k_estimate(EstArgs A) {
+  pdl_trigger(5);
   pdl_wait();
   KTRACE(10);
   __shared__ uint32_t sdig[8];

@@ -295,7 +295,7 @@ def test_parity_snr_sweep(snr_db):
                                  {"CUSFFT_STAGE_MODE": "fused_index"}, {"CUSFFT_P2": "ldg"}, {"CUSFFT_DISCARD": "0"},
                                  {"CUSFFT_SLOT": "1"}, {"CUSFFT_SLOT": "2"}, {"CUSFFT_BRANCH": "1"}, {"CUSFFT_BRANCH": "2"}, {"CUSFFT_BRANCH": "3"}, {"CUSFFT_BRANCH": "4"}, {"CUSFFT_BRANCH": "5"},
                                  {"CUSFFT_STAGE_GROUPS": "2"}, {"CUSFFT_PACKED": "0"},
-                                 {"CUSFFT_FFT_E": "1024"}, {"CUSFFT_FFT_E": "256"}, {"CUSFFT_PK": "0"}, {"CUSFFT_BRANCH": "0"}])
+                                 {"CUSFFT_FFT_E": "1024"}, {"CUSFFT_FFT_E": "256"}, {"CUSFFT_PK": "0"}, {"CUSFFT_PDL_TRIGGER": "0"}, {"CUSFFT_PDL_TRIGGER": "63"}, {"CUSFFT_SPLIT_LAUNCH": "1"}, {"CUSFFT_BRANCH": "0"}])
 def test_kernel_variants_agree(env, monkeypatch):
     """Every alternative kernel path (selected at plan time by environment
     switches, used for A/B measurements) gives the default path's hits and
@@ -372,3 +372,24 @@ def test_C5_k_sweep_parity(k, bcst):
     np.testing.assert_allclose(vals, ref.vals, rtol=1e-9, atol=1e-12)
     assert set(locs.tolist()) == set(S.tolist())
     assert O.l1_error(locs, vals, S, X, k) <= 1e-6
+
+
+@pytest.mark.gpu
+def test_debug_and_plain_plans_agree():
+    """A plan without debug buffers (the fold output u is then not written by
+    the bulk-copy fold; the FFT reads v) returns exactly the debug plan's
+    output, and refuses the U artefact instead of returning stale data."""
+    from paper_conf_ipps_wangcc16_b200 import Plan
+    n, k = 2 ** 22, 1000
+    x, S, X = planted_signal(n, k, seed=33)
+    xd = torch.from_numpy(x).to(DEV)
+    dbg = Plan(n, k, L=16, seed=9, debug=1)
+    plain = Plan(n, k, L=16, seed=9)
+    assert plain.info()["staged"]
+    l0, v0 = dbg.execute(xd)
+    l1, v1 = plain.execute(xd)
+    torch.cuda.synchronize()
+    assert torch.equal(l0, l1) and torch.equal(v0, v1)
+    assert set(l1.cpu().tolist()) == set(S.tolist())
+    with pytest.raises(Exception):
+        plain.debug(DEBUG_U)
