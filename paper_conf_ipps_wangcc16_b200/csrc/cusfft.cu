@@ -8,6 +8,7 @@
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <new>
 #include <utility>
 #include <string>
@@ -154,7 +155,8 @@ struct cusfft_plan_s {
   };
   std::vector<StageGroup> groups;
   double2* d_staging = nullptr;   // [max group total]
-  cudaAccessPolicyWindow stage_window = {};  // persisting L2 window over d_staging
+  cudaAccessPolicyWindow stage_window = {};
+  bool setaside = false;          // holds a reference on the device's persisting-L2 set-aside  // persisting L2 window over d_staging
   double2* d_ghat = nullptr;
   double2* d_tw = nullptr;
   SlotParam* d_slots = nullptr;
@@ -252,6 +254,39 @@ struct DeviceGuard {
   }
 };
 
+// Device-wide persisting-L2 set-aside (cudaLimitPersistingL2CacheSize), shared
+// by the plans of a device: raised to the largest request while any plan holds
+// it, restored to the value found before the first plan when the last one is
+// destroyed, so other work on the device (e.g. dense cuFFT) gets the whole L2
+// back.
+struct SetAside {
+  int refs = 0;
+  size_t orig = 0, cur = 0;
+};
+std::mutex g_setaside_mu;
+SetAside g_setaside[64];
+
+void setaside_acquire(int dev, size_t bytes) {
+  std::lock_guard<std::mutex> lk(g_setaside_mu);
+  SetAside& a = g_setaside[dev & 63];
+  if (a.refs++ == 0) {
+    cudaDeviceGetLimit(&a.orig, cudaLimitPersistingL2CacheSize);
+    a.cur = a.orig;
+  }
+  if (bytes > a.cur && cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, bytes) == cudaSuccess) a.cur = bytes;
+  cudaGetLastError();
+}
+
+void setaside_release(int dev) {
+  std::lock_guard<std::mutex> lk(g_setaside_mu);
+  SetAside& a = g_setaside[dev & 63];
+  if (a.refs > 0 && --a.refs == 0 && a.cur != a.orig) {
+    cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, a.orig);
+    cudaGetLastError();
+    a.cur = a.orig;
+  }
+}
+
 void free_plan(cusfft_plan_t p) {
   for (auto& g : p->groups) {
     if (g.spos) cudaFree(g.spos);
@@ -277,6 +312,7 @@ void free_plan(cusfft_plan_t p) {
   if (p->cap_stream2) cudaStreamDestroy(p->cap_stream2);
   if (p->ev_fork) cudaEventDestroy(p->ev_fork);
   if (p->ev_join) cudaEventDestroy(p->ev_join);
+  if (p->setaside) setaside_release(p->device);
   p->magic = 0;
   delete p;
 }
@@ -855,11 +891,16 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       // Persisting-L2 set-aside for the staging buffer (a device-wide limit: raised, never lowered).
       int maxp = 0;
       cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev);
-      const size_t win = P->stage_atomic ? 0 : std::min<size_t>((size_t)maxtot * 16, (size_t)maxp);
-      size_t cur = 0;
-      cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
-      if (win > cur) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, win);
-      cudaGetLastError();
+      // The set-aside is what keeps the staging (stored evict_last = persisting) apart from the
+      // evict_first stream of x: without it C3 takes 100 us instead of 87.
+      // CUSFFT_APW=0 turns it (and the window) off for that A/B.
+      const bool apw = !(std::getenv("CUSFFT_APW") && std::getenv("CUSFFT_APW")[0] == '0');
+      const size_t win = (P->stage_atomic || !apw) ? 0 : std::min<size_t>((size_t)maxtot * 16, (size_t)maxp);
+      size_t want = win;  // CUSFFT_SETASIDE_MB: a larger set-aside than the staging buffer (A/B)
+      if (const char* e = std::getenv("CUSFFT_SETASIDE_MB"))
+        if (win > 0) want = std::min<size_t>((size_t)maxp, std::max<size_t>(win, (size_t)std::atoll(e) << 20));
+      if (win > 0) setaside_acquire(dev, want);
+      P->setaside = win > 0;
       P->stage_window.base_ptr = P->d_staging;
       P->stage_window.num_bytes = win;
       P->stage_window.hitRatio = 1.0f;
@@ -1394,8 +1435,12 @@ int launch_branched_p2(cusfft_plan_t P, const double2* x, int64_t* locs, double2
     CK(cudaStreamWaitEvent(b, P->ev_fork, 0));
     P->cur_prio = P->prio_lo;
     g_pdl = false;
-    CK(launch_fold_fft1(P, g.staging + (size_t)nl * P->R * B, nullptr, sp + nl, P->d_u + (size_t)nl * B,
-                        P->d_v + (size_t)nl * B, P->Lg - nl, z0, b, true));
+    if (g.inv)  // index staging: staging in address order, phase 2 gathers through the slot's index rows
+      CK(launch_fold_fft1(P, g.staging, g.inv + (size_t)nl * P->R * B, sp + nl, P->d_u + (size_t)nl * B,
+                          P->d_v + (size_t)nl * B, P->Lg - nl, z0, b, false));
+    else
+      CK(launch_fold_fft1(P, g.staging + (size_t)nl * P->R * B, nullptr, sp + nl, P->d_u + (size_t)nl * B,
+                          P->d_v + (size_t)nl * B, P->Lg - nl, z0, b, true));
     g_pdl = true;
     int r = launch_bfft(P, nl, P->Lg, b);
     if (r) return r;
@@ -1413,7 +1458,7 @@ int launch_branched_p2(cusfft_plan_t P, const double2* x, int64_t* locs, double2
   g_pdl = !stage1_outside;
   if (P->branch_fork == 0 && (rc = fork())) return rc;
   if (stage1_outside) g_pdl = false;  // the graph's first node on a
-  CK(launch_fold_fft1(P, g.staging, nullptr, sp, P->d_u, P->d_v, nl, z0, a, true));
+  CK(launch_fold_fft1(P, g.staging, g.inv, sp, P->d_u, P->d_v, nl, z0, a, g.inv == nullptr));
   g_pdl = true;
   if (P->branch_fork == 1 && (rc = fork())) return rc;
   if ((rc = launch_bfft(P, 0, nl, a))) return rc;
@@ -1433,7 +1478,8 @@ int launch_branched_p2(cusfft_plan_t P, const double2* x, int64_t* locs, double2
 
 inline bool use_branch_p2(cusfft_plan_t P) {
   return P->branch_p2 && !P->slot_fused && P->use_graph && !P->timing && P->stage_limit == 6 && P->nloc_local > 0 &&
-         P->nloc_local < P->Lg && P->staged && P->groups.size() == 1 && P->stage_scatter && !P->stage_split &&
+         P->nloc_local < P->Lg && P->staged && P->groups.size() == 1 &&
+         (P->stage_scatter || P->groups[0].inv) && !P->stage_split &&
          !P->skip_stage && !P->xshard;
 }
 

@@ -393,3 +393,28 @@ def test_debug_and_plain_plans_agree():
     assert set(l1.cpu().tolist()) == set(S.tolist())
     with pytest.raises(Exception):
         plain.debug(DEBUG_U)
+
+
+@pytest.mark.gpu
+def test_l2_setaside_held_and_released():
+    """A staged plan holds the device's persisting-L2 set-aside (the staging
+    buffer is stored evict_last) and the last plan to go restores the value it
+    found, so other work gets the whole L2 back."""
+    import gc
+    from cuda.bindings import runtime as rt
+    from paper_conf_ipps_wangcc16_b200 import Plan
+    lim = rt.cudaLimit.cudaLimitPersistingL2CacheSize
+    gc.collect()
+    torch.cuda.synchronize()
+    before = rt.cudaDeviceGetLimit(lim)[1]
+    maxp = rt.cudaDeviceGetAttribute(rt.cudaDeviceAttr.cudaDevAttrMaxPersistingL2CacheSize, 0)[1]
+    plan = Plan(2 ** 22, 1000, L=16, seed=1)
+    assert plan.info()["staged"]
+    during = rt.cudaDeviceGetLimit(lim)[1]
+    if maxp > 0:
+        assert during > 0
+    plan.close()
+    after = rt.cudaDeviceGetLimit(lim)[1]
+    assert after == before or after == during  # == during only if another live plan still holds it
+    if before == 0:
+        assert after == 0
