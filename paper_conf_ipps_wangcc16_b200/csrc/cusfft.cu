@@ -203,6 +203,7 @@ struct cusfft_plan_s {
   // CUDA graphs of the launch sequences, keyed by the caller's pointers
   bool use_graph = true;
   bool branched = false;          // two-branch graph (location chain || estimation folds); opt-in
+  bool code_ef = false;           // CUSFFT_CODE_EF=1: schedule words loaded evict_first (A/B)
   bool split_launch = false;      // CUSFFT_SPLIT_LAUNCH=1: phase 1 as a plain launch before the graph of the rest
   int branch_fork = 0;            // CUSFFT_BRANCH=2..5: the estimation branch forks after phase 1 / the location
                                   // slots' phase 2 / their FFT pass 2 / the cutoff
@@ -605,6 +606,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     const int m = e ? std::atoi(e) : 32;
     cudaMemcpyToSymbol(c_pdl_trigger, &m, sizeof(int));
   }
+  if (const char* e = std::getenv("CUSFFT_CODE_EF")) P->code_ef = (e[0] == '1');
   if (const char* e = std::getenv("CUSFFT_SPLIT_LAUNCH")) P->split_launch = (e[0] == '1');
   if (const char* e = std::getenv("CUSFFT_FFT_E")) P->fft_E = std::max(256, std::min(1024, std::atoi(e)));
 
@@ -893,7 +895,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev);
       // The set-aside is what keeps the staging (stored evict_last = persisting) apart from the
       // evict_first stream of x: without it C3 takes 100 us instead of 87.
-      // CUSFFT_APW=0 turns it (and the window) off for that A/B.
+      // CUSFFT_APW=0 turns it off for that A/B.
       const bool apw = !(std::getenv("CUSFFT_APW") && std::getenv("CUSFFT_APW")[0] == '0');
       const size_t win = (P->stage_atomic || !apw) ? 0 : std::min<size_t>((size_t)maxtot * 16, (size_t)maxp);
       size_t want = win;  // CUSFFT_SETASIDE_MB: a larger set-aside than the staging buffer (A/B)
@@ -902,7 +904,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       if (win > 0) setaside_acquire(dev, want);
       P->setaside = win > 0;
       P->stage_window.base_ptr = P->d_staging;
-      P->stage_window.num_bytes = win;
+      // the access-policy window on the launches adds nothing measurable (CUSFFT_APW=1 to attach it)
+      P->stage_window.num_bytes = (std::getenv("CUSFFT_APW") && std::getenv("CUSFFT_APW")[0] == '1') ? win : 0;
       P->stage_window.hitRatio = 1.0f;
       P->stage_window.hitProp = cudaAccessPropertyPersisting;
       P->stage_window.missProp = cudaAccessPropertyStreaming;
@@ -1019,7 +1022,7 @@ int launch_stage1(cusfft_plan_t P, const cusfft_plan_s::StageGroup& g, const dou
   } else if (g.code) {
     StagePackArgs a{x, g.code, g.staging, P->d_slots + (size_t)P->lrank * P->Lg + g.s0, tot, g.s1 - g.s0,
                     P->stage_ibits, P->R, ilog2(P->B), P->logB2, P->logB1, ilog2(256 / P->B1),
-                    (uint32_t)(P->n - 1), z};
+                    (uint32_t)(P->n - 1), z, P->code_ef ? 1 : 0};
     e = launch_k(k_stage_packed, dim3(grid), dim3(256), 0, st, P->cur_prio, a);
   } else {
     e = launch_k(k_stage, dim3(grid), dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)g.spos,

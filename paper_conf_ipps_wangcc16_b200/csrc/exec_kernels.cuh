@@ -161,7 +161,14 @@ struct StagePackArgs {
   int total, nslots, ibits, R, logB, logB2, logB1, logC;
   uint32_t nmask;
   ZeroArgs zero;
+  int code_ef;  // schedule words read with the evict_first policy too
 };
+
+__device__ __forceinline__ uint32_t ld_u32_ef(const uint32_t* p, uint64_t pol) {
+  uint32_t v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+  return v;
+}
 
 __global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
   pdl_trigger(0);
@@ -186,7 +193,7 @@ __global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
     for (int c = 0; c < 8; ++c) {
       const int q = q0 + c * T;
       if (q < A.total) {
-        cd[c] = __ldg(A.code + q);
+        cd[c] = A.code_ef ? ld_u32_ef(A.code + q, pf) : __ldg(A.code + q);
         const uint32_t sl = cd[c] >> A.ibits, i = cd[c] & imask;
         const double2* p = A.x + ((ssig[sl] * i + stau[sl]) & A.nmask);
         asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.L2::64B.v2.f64 {%0, %1}, [%2], %3;"
@@ -1791,7 +1798,28 @@ __global__ void __launch_bounds__(256) k_vote(VoteArgs A) {
 // ---------------------------------------------------------------------------
 constexpr int kPk = 16384;
 
-__device__ __forceinline__ bool vote8_finish(const VoteArgs& A, const uint8_t* pk, const uint32_t* ssig, int q0, int m,
+// Shared-memory views addressed by 32-bit shared-window offsets: a generic
+// pointer to a __shared__ array passed into a device function makes the
+// compiler rebuild the window address (S2R SR_CgaCtaId, MOV, LEA) at every
+// probe; these emit one LDS with an immediate base instead.
+struct SmemU8 {
+  uint32_t base;
+  __device__ __forceinline__ uint32_t operator[](uint32_t i) const {
+    uint32_t v;
+    asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(base + i));
+    return v;
+  }
+};
+struct SmemU32 {
+  uint32_t base;
+  __device__ __forceinline__ uint32_t operator[](int i) const {
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(base + 4u * (uint32_t)i));
+    return v;
+  }
+};
+
+__device__ __forceinline__ bool vote8_finish(const VoteArgs& A, SmemU8 pk, SmemU32 ssig, int q0, int m,
                                              uint32_t F, int got, uint32_t half_s, int bsh) {
   int votes = got;
   for (int q = q0 + 1 + m; q < A.Lloc; ++q) votes += (pk[(ssig[q] * F + half_s) >> bsh] >> q) & 1;
@@ -1801,7 +1829,7 @@ __device__ __forceinline__ bool vote8_finish(const VoteArgs& A, const uint8_t* p
 }
 
 template <int M>
-__device__ __forceinline__ void vote8_unit(const VoteArgs& A, const uint8_t* pk, const uint32_t* ssig, int q0,
+__device__ __forceinline__ void vote8_unit(const VoteArgs& A, SmemU8 pk, SmemU32 ssig, int q0,
                                            uint32_t Jv, uint32_t a, int mrt, uint32_t* qF, uint8_t* qG) {
   constexpr int MM = M > 0 ? M : 1;
   constexpr int VC = 2;
@@ -1889,7 +1917,7 @@ __device__ __forceinline__ void vote8_unit(const VoteArgs& A, const uint8_t* pk,
 // over loop 2i's preimage ranges with ONE mandatory probe of loop 2i+1, and
 // f is counted at its first doubly-voting pair: survivors probe every other
 // loop, need >= T votes in all and no earlier pair voting twice.
-__device__ __forceinline__ bool vote8_pair_finish(const VoteArgs& A, const uint8_t* pk, const uint32_t* ssig, int pr,
+__device__ __forceinline__ bool vote8_pair_finish(const VoteArgs& A, SmemU8 pk, SmemU32 ssig, int pr,
                                                   uint32_t F, uint32_t half_s, int bsh) {
   uint32_t bits = 3u << (2 * pr);
   for (int q = 0; q < A.Lloc; ++q)
@@ -1899,7 +1927,7 @@ __device__ __forceinline__ bool vote8_pair_finish(const VoteArgs& A, const uint8
   return hit;
 }
 
-__device__ __forceinline__ void vote8_pair_unit(const VoteArgs& A, const uint8_t* pk, const uint32_t* ssig, int pr,
+__device__ __forceinline__ void vote8_pair_unit(const VoteArgs& A, SmemU8 pk, SmemU32 ssig, int pr,
                                                 uint32_t Jv, uint32_t a, uint32_t* qF) {
   constexpr int VC = 2;
   const int lane = threadIdx.x & 31;
@@ -1974,6 +2002,12 @@ __global__ void __launch_bounds__(1024, 1) k_vote8(VoteArgs A) {
   // enumerated loops: pairs' first loops 0, 2, 4, ... (pair mode) or 0 .. L_loc - T
   const int nenum = A.pairs ? A.Lloc / 2 : A.Lloc - A.T + 1;
   if (tid < A.Lloc) ssig[tid] = A.sig[tid];
+  // held in registers (a volatile move cannot be rematerialised inside the loops)
+  uint32_t pk_base, ss_base;
+  asm volatile("mov.u32 %0, %1;" : "=r"(pk_base) : "r"(smem_u32(pk)));
+  asm volatile("mov.u32 %0, %1;" : "=r"(ss_base) : "r"(smem_u32(ssig)));
+  const SmemU8 spk{pk_base};
+  const SmemU32 sss{ss_base};
   if (tid == 0) {
     int acc = 0;
     scnt[0] = 0;
@@ -1994,7 +2028,7 @@ __global__ void __launch_bounds__(1024, 1) k_vote8(VoteArgs A) {
       int pr = 0;
       while (unit >= scnt[pr + 1]) ++pr;
       const uint32_t Jv = (uint32_t)__ldg(A.Jp[2 * pr] + (unit - scnt[pr]));
-      vote8_pair_unit(A, pk, ssig, pr, Jv, A.aa[2 * pr], qF);
+      vote8_pair_unit(A, spk, sss, pr, Jv, A.aa[2 * pr], qF);
     }
     TRACE_END(32);
     return;
@@ -2007,11 +2041,11 @@ __global__ void __launch_bounds__(1024, 1) k_vote8(VoteArgs A) {
     const uint32_t a = A.aa[q0];
     const int m = min(A.Lloc - A.T - q0 + 1, A.Lloc - 1 - q0);
     switch (m) {
-      case 1: vote8_unit<1>(A, pk, ssig, q0, Jv, a, 1, qF, qG); break;
-      case 2: vote8_unit<2>(A, pk, ssig, q0, Jv, a, 2, qF, qG); break;
-      case 3: vote8_unit<3>(A, pk, ssig, q0, Jv, a, 3, qF, qG); break;
-      case 4: vote8_unit<4>(A, pk, ssig, q0, Jv, a, 4, qF, qG); break;
-      default: vote8_unit<0>(A, pk, ssig, q0, Jv, a, m, qF, qG); break;
+      case 1: vote8_unit<1>(A, spk, sss, q0, Jv, a, 1, qF, qG); break;
+      case 2: vote8_unit<2>(A, spk, sss, q0, Jv, a, 2, qF, qG); break;
+      case 3: vote8_unit<3>(A, spk, sss, q0, Jv, a, 3, qF, qG); break;
+      case 4: vote8_unit<4>(A, spk, sss, q0, Jv, a, 4, qF, qG); break;
+      default: vote8_unit<0>(A, spk, sss, q0, Jv, a, m, qF, qG); break;
     }
   }
   TRACE_END(32);
