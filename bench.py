@@ -197,7 +197,7 @@ def run_gpu(args):
     from paper_conf_ipps_wangcc16_b200.dist import CudaEngine, LoopShardedSfft, signal_range
 
     n, k, L, desc = CONFIGS[args.config]
-    B = default_B(n, k)
+    B = args.B or default_B(n, k)
     x_np, S, X = make_signal(n, k, args.signal_seed)
     x_pin = torch.from_numpy(x_np).pin_memory()
     x = x_pin.to(dev)
@@ -615,6 +615,7 @@ def main():
     ap.add_argument("--plan-seed", type=int, default=3)
     ap.add_argument("--shard", default="loops", choices=["loops", "signal"],
                     help="N>1: loop sharding (all-gather) or signal sharding (SURVEY N1, all-reduce)")
+    ap.add_argument("--B", type=int, default=0, help="bucket count (default: the paper's formula, DESIGN.md Z3)")
     ap.add_argument("--pipeline", type=int, default=2, help="C5 batch: clone plans in flight per GPU")
     ap.add_argument("--cpu-budget-s", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -193,13 +193,14 @@ def test_num_select_equals_B():
     check_all(plan, ref, locs, vals, fold_bit_exact=True)
 
 
-@pytest.mark.parametrize("tol", [1e-8, 1e-7])
-def test_C3_full_size_parity_and_recovery(tol):
+@pytest.mark.parametrize("tol,B", [(1e-8, None), (1e-7, None), (1e-7, 8192)])
+def test_C3_full_size_parity_and_recovery(tol, B):
     """BASELINE.json configs[2]: n = 2^24, k = 1000, L = 16, in the bench's launch
-    config (delta = 1e-7, staged fold) and at the library default delta."""
+    config (delta = 1e-7, staged fold), at the library default delta, and with
+    half the formula's buckets (B = 8192, DESIGN.md §3 study)."""
     n, k = 2 ** 24, 1000
     x, S, X = planted_signal(n, k, seed=1)
-    plan, ref, locs, vals = run_pair(x, n, k, None, 16, shared_taps=False, seed=3, tolerance=tol)
+    plan, ref, locs, vals = run_pair(x, n, k, B, 16, shared_taps=False, seed=3, tolerance=tol)
     assert plan.info()["staged"] == 1
     check_all(plan, ref, locs, vals, fold_bit_exact=False)
     assert set(locs.tolist()) == set(S.tolist())
