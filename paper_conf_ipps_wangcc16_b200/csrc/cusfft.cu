@@ -203,6 +203,7 @@ struct cusfft_plan_s {
   // CUDA graphs of the launch sequences, keyed by the caller's pointers
   bool use_graph = true;
   bool branched = false;          // two-branch graph (location chain || estimation folds); opt-in
+  bool est_seg = true;            // k_estimate_seg for L <= 16 (CUSFFT_EST_SEG=0: k_estimate)
   bool code_ef = false;           // CUSFFT_CODE_EF=1: schedule words loaded evict_first (A/B)
   bool split_launch = false;      // CUSFFT_SPLIT_LAUNCH=1: phase 1 as a plain launch before the graph of the rest
   int branch_fork = 0;            // CUSFFT_BRANCH=2..5: the estimation branch forks after phase 1 / the location
@@ -606,6 +607,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     const int m = e ? std::atoi(e) : 32;
     cudaMemcpyToSymbol(c_pdl_trigger, &m, sizeof(int));
   }
+  if (const char* e = std::getenv("CUSFFT_EST_SEG")) P->est_seg = (e[0] != '0');
   if (const char* e = std::getenv("CUSFFT_CODE_EF")) P->code_ef = (e[0] == '1');
   if (const char* e = std::getenv("CUSFFT_SPLIT_LAUNCH")) P->split_launch = (e[0] == '1');
   if (const char* e = std::getenv("CUSFFT_FFT_E")) P->fft_E = std::max(256, std::min(1024, std::atoi(e)));
@@ -1321,7 +1323,14 @@ int launch_estimate(cusfft_plan_t P, cudaStream_t st) {
   ea.hit_keys = P->d_hit_keys;
   ea.per_loop = P->d_per_loop;
   ea.out_hist = P->d_ohist;
-  CK(launch_k(k_estimate, dim3(P->est_grid), dim3(256), 0, st, P->cur_prio, ea));
+  // segmented kernel (2 hits per warp at L = 16, 4 at L <= 8); CUSFFT_EST_SEG=0: warp per hit
+  if (P->est_seg && P->L <= 8) {
+    CK(launch_k(k_estimate_seg<8>, dim3(P->est_grid), dim3(256), 0, st, P->cur_prio, ea));
+  } else if (P->est_seg && P->L <= 16) {
+    CK(launch_k(k_estimate_seg<16>, dim3(P->est_grid), dim3(256), 0, st, P->cur_prio, ea));
+  } else {
+    CK(launch_k(k_estimate, dim3(P->est_grid), dim3(256), 0, st, P->cur_prio, ea));
+  }
   return CUSFFT_SUCCESS;
 }
 

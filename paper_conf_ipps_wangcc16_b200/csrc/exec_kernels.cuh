@@ -2171,6 +2171,78 @@ __global__ void __launch_bounds__(256) k_estimate(EstArgs A) {
   TRACE_END(41);
 }
 
+// Segmented form for L <= LP (LP = 8 or 16): a warp holds 32 / LP hits, one
+// segment of LP lanes per hit, lane li of a segment = loop li; the same
+// per-loop estimate and the same rank rule (ties by loop) inside the segment.
+// Twice (L = 16) the hits per warp of k_estimate with all 32 lanes busy.
+template <int LP>
+__global__ void __launch_bounds__(256) k_estimate_seg(EstArgs A) {
+  pdl_trigger(5);
+  pdl_wait();
+  KTRACE(10);
+  constexpr int G = 32 / LP;    // hits per warp
+  constexpr int NH = 8 * G;     // hits per CTA iteration
+  __shared__ uint32_t sdig[NH];
+  if (blockIdx.x == 0) TRACE(40);
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const int seg = lane / LP, li = lane % LP, sbase = seg * LP;
+  const bool act = li < A.L;
+  SlotParam sp{0, 0, 0, 0};
+  if (act) sp = A.slots[li];
+  const int H = min((int)*A.hit_count, A.max_hits);
+  const int med = (A.L - 1) >> 1;
+  const unsigned segmask = (LP == 32 ? kFull : ((1u << LP) - 1u)) << sbase;
+  for (int h0 = blockIdx.x * NH; h0 < H; h0 += gridDim.x * NH) {  // CTA-uniform
+    const int h = h0 + wib * G + seg;
+    const bool valid = h < H;
+    double2 v = make_double2(0.0, 0.0);
+    if (valid && act) {
+      const uint32_t f = (uint32_t)__ldg(A.hits + h);
+      v = loop_estimate(A, sp, li, f);
+      if (A.per_loop) A.per_loop[(int64_t)h * A.L + li] = v;
+    }
+    // element of rank med among the segment's L values (ties by loop), re and im separately
+    double vr = 0.0, vi = 0.0;
+#pragma unroll
+    for (int part = 0; part < 2; ++part) {
+      const double a = part ? v.y : v.x;
+      int r = 0;
+#pragma unroll
+      for (int j = 0; j < LP; ++j) {
+        const double b = __shfl_sync(kFull, a, sbase + j);
+        r += (j < A.L) && ((b < a) || (b == a && j < li));
+      }
+      const unsigned bal = __ballot_sync(kFull, act && r == med) & segmask;
+      const int src = bal ? __ffs(bal) - 1 : sbase;
+      const double m = __shfl_sync(kFull, a, src);
+      if (part) vi = m; else vr = m;
+    }
+    uint32_t dig = 0xFFFFFFFFu;
+    if (valid) {
+      const uint64_t key = (uint64_t)__double_as_longlong(__dadd_rn(__dmul_rn(vr, vr), __dmul_rn(vi, vi)));
+      if (li == 0) {
+        A.hit_vals[h] = make_double2(vr, vi);
+        A.hit_keys[h] = key;
+      }
+      dig = (uint32_t)(key >> 51) & 0xFFFu;
+    }
+    if (li == 0) sdig[wib * G + seg] = dig;
+    __syncthreads();
+    if (threadIdx.x < NH) {  // one atomic per distinct digit of this CTA's hits
+      const uint32_t d = sdig[threadIdx.x];
+      bool first = d != 0xFFFFFFFFu;
+      uint32_t c = 0;
+      for (int j = 0; j < NH; ++j) {
+        first = first && !(j < (int)threadIdx.x && sdig[j] == d);
+        c += sdig[j] == d;
+      }
+      if (first) atomicAdd(A.out_hist + d, c);
+    }
+    __syncthreads();
+  }
+  TRACE_END(41);
+}
+
 // ---------------------------------------------------------------------------
 // Output: the k hits of largest |val|^2 (ties to the smaller f), written in
 // ascending f; pads loc = -1, val = 0.  One CTA of 1024 threads: two-level
