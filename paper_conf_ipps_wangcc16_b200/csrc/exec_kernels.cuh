@@ -2281,13 +2281,13 @@ __global__ void __launch_bounds__(1024) k_output(const int* __restrict__ hits, c
   // above the false hits), one classification pass selects, and the values
   // go to shared memory (aliasing the unused candidate arrays), so neither the
   // sort nor the write-out touches global memory again.
-  constexpr int PF = 4;
+  constexpr int PF = 4, NCH = 4;  // items per thread per chunk, chunks (H <= 16384 on the fast path)
   double2* selv = reinterpret_cast<double2*>(ckey);  // [kp2] values of the selected entries (fast path)
-  const bool fast = H <= PF * 1024 && kp2 * 16 <= kOutCap * 12;
+  const bool fast = H <= NCH * PF * 1024 && kp2 * 16 <= kOutCap * 12;
   uint64_t pk[PF];
   uint32_t pf[PF];
   double2 pv[PF];
-  if (fast) {
+  if (fast) {  // chunk 0: keys, f and values
 #pragma unroll
     for (int u = 0; u < PF; ++u) {
       const int i = u * 1024 + tid;
@@ -2314,19 +2314,31 @@ __global__ void __launch_bounds__(1024) k_output(const int* __restrict__ hits, c
     if (whole) {
       direct = true;
       const int lane = tid & 31;
+      for (int ch = 0; ch < NCH && ch * PF * 1024 < H; ++ch) {  // block-uniform
+        if (ch > 0) {  // later chunks (many false hits): keys and f here, values only for the selected
 #pragma unroll
-      for (int u = 0; u < PF; ++u) {
-        const int i = u * 1024 + tid;
-        const bool take = i < H && ((uint32_t)(pk[u] >> 51) & 0xFFFu) >= d0;
-        const unsigned bal = __ballot_sync(kFull, take);
-        int base = 0;
-        if (lane == 0 && bal) base = atomicAdd(&sm[41], __popc(bal));
-        base = __shfl_sync(kFull, base, 0);
-        if (take) {
-          const int pos = base + __popc(bal & ((1u << lane) - 1u));
-          if (pos < kp2) {
-            sel[pos] = ((uint64_t)pf[u] << 32) | (uint32_t)pos;
-            selv[pos] = pv[u];
+          for (int u = 0; u < PF; ++u) {
+            const int i = ch * PF * 1024 + u * 1024 + tid;
+            if (i < H) {
+              pk[u] = __ldg(hit_keys + i);
+              pf[u] = (uint32_t)__ldg(hits + i);
+            }
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < PF; ++u) {
+          const int i = ch * PF * 1024 + u * 1024 + tid;
+          const bool take = i < H && ((uint32_t)(pk[u] >> 51) & 0xFFFu) >= d0;
+          const unsigned bal = __ballot_sync(kFull, take);
+          int base = 0;
+          if (lane == 0 && bal) base = atomicAdd(&sm[41], __popc(bal));
+          base = __shfl_sync(kFull, base, 0);
+          if (take) {
+            const int pos = base + __popc(bal & ((1u << lane) - 1u));
+            if (pos < kp2) {
+              sel[pos] = ((uint64_t)pf[u] << 32) | (uint32_t)pos;
+              selv[pos] = ch == 0 ? pv[u] : __ldg(hit_vals + i);
+            }
           }
         }
       }
