@@ -423,7 +423,7 @@ def run_gpu(args):
             p2.close()
 
     cpu = None
-    if rank == 0 and not args.no_cpu_baseline:
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:  # N = 1 only (bench contract)
         times, _ = oracle_time(n, k, L, B, x_np, args.plan_seed, budget_s=args.cpu_budget_s, min_runs=1,
                                tolerance=TOLERANCE[args.config])
         cpu = {"value": 1e3 * sum(times) / len(times), "unit": "ms", "cores": 1, "kind": "oracle",

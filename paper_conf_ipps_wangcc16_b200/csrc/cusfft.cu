@@ -203,6 +203,8 @@ struct cusfft_plan_s {
   // CUDA graphs of the launch sequences, keyed by the caller's pointers
   bool use_graph = true;
   bool branched = false;          // two-branch graph (location chain || estimation folds); opt-in
+  bool sel_local_pick = false;    // cluster cutoff picks the boundary bin per CTA (CUSFFT_SEL_LOCALPICK=1; slower)
+  int est_p2_pad = 0;             // extra dynamic smem (bytes) of the estimation branch's phase 2 (CUSFFT_EST_P2_PAD)
   bool est_seg = true;            // k_estimate_seg for L <= 16 (CUSFFT_EST_SEG=0: k_estimate)
   bool code_ef = false;           // CUSFFT_CODE_EF=1: schedule words loaded evict_first (A/B)
   bool split_launch = false;      // CUSFFT_SPLIT_LAUNCH=1: phase 1 as a plain launch before the graph of the rest
@@ -607,6 +609,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     const int m = e ? std::atoi(e) : 32;
     cudaMemcpyToSymbol(c_pdl_trigger, &m, sizeof(int));
   }
+  if (const char* e = std::getenv("CUSFFT_SEL_LOCALPICK")) P->sel_local_pick = (e[0] == '1');
+  if (const char* e = std::getenv("CUSFFT_EST_P2_PAD")) P->est_p2_pad = std::max(0, std::atoi(e));
   if (const char* e = std::getenv("CUSFFT_EST_SEG")) P->est_seg = (e[0] != '0');
   if (const char* e = std::getenv("CUSFFT_CODE_EF")) P->code_ef = (e[0] == '1');
   if (const char* e = std::getenv("CUSFFT_SPLIT_LAUNCH")) P->split_launch = (e[0] == '1');
@@ -958,6 +962,9 @@ cudaError_t launch_slot_t(cusfft_plan_t P, const SlotArgs& a, int nslots, cudaSt
   return cudaLaunchKernelEx(&cfg, k_slot<B1T, B2T, FV>, a);
 }
 
+// extra dynamic smem of the next bulk-copy phase-2 launch (fewer CTAs per SM)
+thread_local int g_p2_pad = 0;
+
 template <int B1T>
 cudaError_t launch_fold_fft1_t(cusfft_plan_t P, const double2* x, const uint32_t* inv, const SlotParam* sp, double2* u,
                                double2* v, int nslots, ZeroArgs z, cudaStream_t st, bool staged_tord) {
@@ -967,7 +974,7 @@ cudaError_t launch_fold_fft1_t(cusfft_plan_t P, const double2* x, const uint32_t
                     (const double*)P->d_taps_perm, sp, u, v, (const double2*)P->d_tw,
                     (int)P->B, P->B2, P->w, P->R, (uint32_t)(P->n - 1), 0u, (uint32_t)P->n, z);
   if (staged_tord && P->p2_tma && P->R <= 48) {  // staged in thread order, rows moved by bulk copies
-    const size_t smem = (size_t)P->R * 4096;
+    const size_t smem = (size_t)P->R * 4096 + (size_t)g_p2_pad;
     static thread_local bool attr_set[4] = {false, false, false, false};
     if (!attr_set[B1T / 64]) {  // static + dynamic smem may exceed the 48 KB default
       cudaFuncSetAttribute(k_fold_fft1_tma<B1T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
@@ -1171,6 +1178,7 @@ SelArgs make_sel_args(cusfft_plan_t P) {
   sa.done = P->d_done;
   sa.status = P->d_flags + 1;
   sa.pk = P->d_pk;
+  sa.local_pick = P->sel_local_pick ? 1 : 0;
   sa.threshold_mode = P->prm.cutoff_mode == CUSFFT_CUTOFF_THRESHOLD ? 1 : 0;
   {
     const double th = P->prm.cutoff_threshold;
@@ -1447,12 +1455,14 @@ int launch_branched_p2(cusfft_plan_t P, const double2* x, int64_t* locs, double2
     CK(cudaStreamWaitEvent(b, P->ev_fork, 0));
     P->cur_prio = P->prio_lo;
     g_pdl = false;
+    g_p2_pad = P->est_p2_pad;
     if (g.inv)  // index staging: staging in address order, phase 2 gathers through the slot's index rows
       CK(launch_fold_fft1(P, g.staging, g.inv + (size_t)nl * P->R * B, sp + nl, P->d_u + (size_t)nl * B,
                           P->d_v + (size_t)nl * B, P->Lg - nl, z0, b, false));
     else
       CK(launch_fold_fft1(P, g.staging + (size_t)nl * P->R * B, nullptr, sp + nl, P->d_u + (size_t)nl * B,
                           P->d_v + (size_t)nl * B, P->Lg - nl, z0, b, true));
+    g_p2_pad = 0;
     g_pdl = true;
     int r = launch_bfft(P, nl, P->Lg, b);
     if (r) return r;

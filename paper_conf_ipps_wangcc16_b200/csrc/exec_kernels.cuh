@@ -703,6 +703,7 @@ struct SelArgs {
   // vote's byte-per-bucket array (bit q = bucket kept in location loop q,
   // selection index == vote index), ORed in by the cutoff; zeroed per execution
   uint32_t* pk;
+  int local_pick;  // cluster cutoff: each CTA scans the whole level-0 histogram (no pick round trips)
 };
 
 struct GKeySrc {
@@ -1109,6 +1110,45 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
     kb[u] = i < per ? __ldcg(keys + k0 + i) : 0ull;
   }
   if (r == 0 && tid == 0) S.ncand = 0;
+  int d0 = 0, k2 = 0;
+  bool whole = true;
+  if (A.local_pick) {
+    // 1+2 without cluster round trips: every CTA finds the boundary bin itself
+    // from the whole 4096-bin histogram (16 KB of L2 reads per CTA) while the
+    // split cluster barrier (arrive now, wait before the first DSMEM access)
+    // completes in the background
+    asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+    if (!A.threshold_mode) {
+      constexpr int PER = 4096 / kSelCNT;
+      const int base = 4095 - PER * tid;
+      int c[PER];
+      int mine = 0;
+#pragma unroll
+      for (int j = 0; j < PER; ++j) {
+        c[j] = (int)__ldcg(h0 + base - j);
+        mine += c[j];
+      }
+      int total;
+      const int ex2 = block_excl_scan<kSelCNT>(mine, &total, S.sm);
+      if (ex2 < A.num && A.num <= ex2 + mine) {
+        int cum = ex2;
+#pragma unroll
+        for (int j = 0; j < PER; ++j) {
+          if (cum + c[j] >= A.num) {
+            S.sm[32] = base - j; S.sm[33] = cum; S.sm[34] = c[j];
+            break;
+          }
+          cum += c[j];
+        }
+      }
+      __syncthreads();
+      d0 = S.sm[32];
+      k2 = A.num - S.sm[33];
+      whole = (k2 == S.sm[34]);
+      __syncthreads();
+    }
+    asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+  } else {
   // 1. slice totals, pushed to every CTA of the cluster
   int tot, ex = 0;
   if (!A.threshold_mode) {
@@ -1117,8 +1157,6 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
   }
   cl.sync();
   // 2. the boundary slice (slices descending r = kSelCL-1 .. 0) finds d0 and pushes it
-  int d0 = 0, k2 = 0;
-  bool whole = true;
   if (!A.threshold_mode) {
     int above = 0, bs = 0;
 #pragma unroll
@@ -1142,6 +1180,7 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
     d0 = S.pick[0];
     k2 = A.num - S.pick[1];
     whole = (k2 == S.pick[2]);
+  }
   }
   if (sel == 0 && r == 0) TRACE(11);
   // 3. classify my keys: bitmap words in my smem, candidates appended to CTA 0
