@@ -1549,7 +1549,11 @@ int run_graphed(cusfft_plan_t P, cusfft_plan_s::GraphEntry& g_plain, cusfft_plan
       return rc;
     }
     CK(ce);
-    const cudaError_t ie = cudaGraphInstantiate(&g.exec, graph, 0);
+    // node priorities (location branch high, estimation branch low) are honoured only
+    // with UseNodePriority (CUSFFT_NODE_PRIO=0: the launching stream's priority for all)
+    const char* np = std::getenv("CUSFFT_NODE_PRIO");
+    const unsigned long long iflags = (np && np[0] == '0') ? 0ull : (unsigned long long)cudaGraphInstantiateFlagUseNodePriority;
+    const cudaError_t ie = cudaGraphInstantiateWithFlags(&g.exec, graph, iflags);
     cudaGraphDestroy(graph);
     CK(ie);
     g.a = a;

@@ -296,7 +296,7 @@ def test_parity_snr_sweep(snr_db):
                                  {"CUSFFT_STAGE_MODE": "fused_index"}, {"CUSFFT_P2": "ldg"}, {"CUSFFT_DISCARD": "0"},
                                  {"CUSFFT_SLOT": "1"}, {"CUSFFT_SLOT": "2"}, {"CUSFFT_BRANCH": "1"}, {"CUSFFT_BRANCH": "2"}, {"CUSFFT_BRANCH": "3"}, {"CUSFFT_BRANCH": "4"}, {"CUSFFT_BRANCH": "5"},
                                  {"CUSFFT_STAGE_GROUPS": "2"}, {"CUSFFT_PACKED": "0"},
-                                 {"CUSFFT_FFT_E": "1024"}, {"CUSFFT_FFT_E": "256"}, {"CUSFFT_PK": "0"}, {"CUSFFT_PDL_TRIGGER": "0"}, {"CUSFFT_PDL_TRIGGER": "63"}, {"CUSFFT_SPLIT_LAUNCH": "1"}, {"CUSFFT_EST_SEG": "0"}, {"CUSFFT_SEL_LOCALPICK": "0"}, {"CUSFFT_BRANCH": "0"}])
+                                 {"CUSFFT_FFT_E": "1024"}, {"CUSFFT_FFT_E": "256"}, {"CUSFFT_PK": "0"}, {"CUSFFT_PDL_TRIGGER": "0"}, {"CUSFFT_PDL_TRIGGER": "63"}, {"CUSFFT_SPLIT_LAUNCH": "1"}, {"CUSFFT_EST_SEG": "0"}, {"CUSFFT_SEL_LOCALPICK": "1"}, {"CUSFFT_NODE_PRIO": "0"}, {"CUSFFT_BRANCH": "0"}])
 def test_kernel_variants_agree(env, monkeypatch):
     """Every alternative kernel path (selected at plan time by environment
     switches, used for A/B measurements) gives the default path's hits and
