@@ -212,7 +212,7 @@ struct cusfft_plan_s {
                                   // slots' phase 2 / their FFT pass 2 / the cutoff
   bool branch_p2 = true;          // CUSFFT_BRANCH=2: one phase 1, then location chain || estimation phase 2 + FFT
   bool skip_stage = false;        // measurement only (CUSFFT_SKIP_STAGE)
-  int stage_cps = 8;              // k_stage CTAs per SM (CUSFFT_STAGE_CPS; branched default 2: room for the chain)
+  int stage_cps = 4;              // phase-1 CTAs per SM: one resident wave (occupancy query; CUSFFT_STAGE_CPS overrides)
   int nloc_local = 0;             // local slots [0, nloc_local) are location loops
   cudaStream_t cap_stream = nullptr, cap_stream2 = nullptr;
   cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
@@ -598,6 +598,13 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   if (const char* e = std::getenv("CUSFFT_VOTE_PAIRS")) P->vote_pairs = !(e[0] == '0');
   // measurement only: skip the staged gather's phase 1 (valid only for a repeated x)
   if (const char* e = std::getenv("CUSFFT_SKIP_STAGE")) P->skip_stage = (e[0] == '1');
+  {  // one resident wave of phase-1 CTAs (grid-stride loop): measured best (C3: 4 per SM at 64 registers,
+     // 84.8 us vs 86.1 with 8 per SM = two waves, 86.1 with 3, 90.6 with 2)
+    int occ = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_stage_packed, 256, 0) == cudaSuccess && occ > 0)
+      P->stage_cps = occ;
+    cudaGetLastError();
+  }
   if (P->branched) P->stage_cps = 2;
   if (const char* e = std::getenv("CUSFFT_STAGE_CPS")) P->stage_cps = std::max(1, std::atoi(e));
   if (const char* e = std::getenv("CUSFFT_P2")) P->p2_tma = std::string(e) != "ldg";
