@@ -135,7 +135,8 @@ struct cusfft_plan_s {
   bool stage_packed = false;      // scatter schedule as packed (slot, i) words (k_stage_packed; CUSFFT_PACKED=0: off)
   int stage_ibits = 0;
   bool p2_tma = true;             // scatter phase 2 through bulk copies (k_fold_fft1_tma; CUSFFT_P2=ldg: k_fold_fft1 MODE 2)
-  bool p2_discard = true;         // drop consumed staging lines from L2 (CUSFFT_DISCARD=0: keep)
+  bool p2_discard = false;        // CUSFFT_DISCARD=1: drop consumed staging lines from L2 (default keeps them:
+                                  // the next execution's phase-1 stores then hit valid set-aside lines)
   bool slot_fused = false;        // FFT pass 2 (+ fold) + cutoff in one cluster kernel per slot (k_slot; CUSFFT_SLOT=1|2)
   bool slot_select = false;       // k_slot also runs the cutoff (cluster selection)
   bool slot_phase_a = false;      // k_slot also folds (phase A, CUSFFT_SLOT=2); default: after k_fold_fft1_tma
