@@ -446,7 +446,8 @@ def run_gpu(args):
         try:
             with open(tf) as f:
                 tj = json.load(f)
-            traffic = (tj.get("parts", {}).get("k_stage_packed", {}).get("dram_bytes_per_launch")
+            parts = {kk.split("<")[0]: vv for kk, vv in tj.get("parts", {}).items()}
+            traffic = (parts.get("k_stage_packed", {}).get("dram_bytes_per_launch")
                        if gather_ms else tj.get("dram_bytes_per_launch"))
         except Exception:
             traffic = None

@@ -135,6 +135,7 @@ struct cusfft_plan_s {
   bool stage_packed = false;      // scatter schedule as packed (slot, i) words (k_stage_packed; CUSFFT_PACKED=0: off)
   int stage_ibits = 0;
   bool p2_tma = true;             // scatter phase 2 through bulk copies (k_fold_fft1_tma; CUSFFT_P2=ldg: k_fold_fft1 MODE 2)
+  int stage_u = 4;                // gathers in flight per phase-1 thread (CUSFFT_STAGE_U = 2 / 4 / 8 / 16)
   bool p2_discard = false;        // CUSFFT_DISCARD=1: drop consumed staging lines from L2 (default keeps them:
                                   // the next execution's phase-1 stores then hit valid set-aside lines)
   bool slot_fused = false;        // FFT pass 2 (+ fold) + cutoff in one cluster kernel per slot (k_slot; CUSFFT_SLOT=1|2)
@@ -599,15 +600,17 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   if (const char* e = std::getenv("CUSFFT_VOTE_PAIRS")) P->vote_pairs = !(e[0] == '0');
   // measurement only: skip the staged gather's phase 1 (valid only for a repeated x)
   if (const char* e = std::getenv("CUSFFT_SKIP_STAGE")) P->skip_stage = (e[0] == '1');
-  {  // one resident wave of phase-1 CTAs (grid-stride loop): measured best (C3: 4 per SM at 64 registers,
-     // 84.8 us vs 86.1 with 8 per SM = two waves, 86.1 with 3, 90.6 with 2)
+  {  // one resident wave of phase-1 CTAs (grid-stride loop), at most 4 per SM: with 4 gathers in flight per
+     // thread that is 4096 per SM, measured best (C3: 81.5-81.9 us; 8 in flight at 4 per SM 83.6-83.9,
+     // 4 in flight at 8 per SM 83.9-84.1, at 3 per SM 83.2-83.5, at 2 per SM 88.2-88.7)
     int occ = 0;
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_stage_packed, 256, 0) == cudaSuccess && occ > 0)
-      P->stage_cps = occ;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_stage_packed<4>, 256, 0) == cudaSuccess && occ > 0)
+      P->stage_cps = std::min(occ, 4);
     cudaGetLastError();
   }
   if (P->branched) P->stage_cps = 2;
   if (const char* e = std::getenv("CUSFFT_STAGE_CPS")) P->stage_cps = std::max(1, std::atoi(e));
+  if (const char* e = std::getenv("CUSFFT_STAGE_U")) P->stage_u = std::atoi(e);
   if (const char* e = std::getenv("CUSFFT_P2")) P->p2_tma = std::string(e) != "ldg";
   if (const char* e = std::getenv("CUSFFT_DISCARD")) P->p2_discard = (e[0] == '1');
   {
@@ -1026,7 +1029,8 @@ int launch_stage1(cusfft_plan_t P, const cusfft_plan_s::StageGroup& g, const dou
   int sms = 148;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, P->device);
   const int tot = (int)g.total;
-  const int grid = std::max(1, std::min((tot + 8 * 256 - 1) / (8 * 256), sms * P->stage_cps));
+  const int per = 256 * std::max(1, P->stage_u);
+  const int grid = std::max(1, std::min((tot + per - 1) / per, sms * P->stage_cps));
   g_apw = P->stage_window;  // keep the staging buffer L2-resident for phase 2
   cudaError_t e;
   if (g.code && P->stage_atomic) {
@@ -1040,7 +1044,16 @@ int launch_stage1(cusfft_plan_t P, const cusfft_plan_s::StageGroup& g, const dou
     StagePackArgs a{x, g.code, g.staging, P->d_slots + (size_t)P->lrank * P->Lg + g.s0, tot, g.s1 - g.s0,
                     P->stage_ibits, P->R, ilog2(P->B), P->logB2, P->logB1, ilog2(256 / P->B1),
                     (uint32_t)(P->n - 1), z, P->code_ef ? 1 : 0};
-    e = launch_k(k_stage_packed, dim3(grid), dim3(256), 0, st, P->cur_prio, a);
+    if (P->stage_u == 2)
+      e = launch_k(k_stage_packed<2>, dim3(grid), dim3(256), 0, st, P->cur_prio, a);
+    else if (P->stage_u == 4)
+      e = launch_k(k_stage_packed<4>, dim3(grid), dim3(256), 0, st, P->cur_prio, a);
+    else if (P->stage_u == 16)
+      e = launch_k(k_stage_packed<16>, dim3(grid), dim3(256), 0, st, P->cur_prio, a);
+    else if (P->stage_u == 8)
+      e = launch_k(k_stage_packed<8>, dim3(grid), dim3(256), 0, st, P->cur_prio, a);
+    else
+      e = launch_k(k_stage_packed<4>, dim3(grid), dim3(256), 0, st, P->cur_prio, a);
   } else {
     e = launch_k(k_stage, dim3(grid), dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)g.spos,
                  (const uint32_t*)g.dst, g.staging, tot, z);

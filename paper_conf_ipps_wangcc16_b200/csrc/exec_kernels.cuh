@@ -170,6 +170,8 @@ __device__ __forceinline__ uint32_t ld_u32_ef(const uint32_t* p, uint64_t pol) {
   return v;
 }
 
+// U: gathers in flight per thread (CUSFFT_STAGE_U = 2 / 4 / 8 / 16; 4 by default).
+template <int U>
 __global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
   pdl_trigger(0);
   pdl_wait();
@@ -186,11 +188,11 @@ __global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
   const uint32_t imask = (1u << A.ibits) - 1u;
   const uint32_t Bm = (1u << A.logB) - 1u, B2m = (1u << A.logB2) - 1u, Cm = (1u << A.logC) - 1u;
   const int T = gridDim.x * blockDim.x;
-  for (int q0 = blockIdx.x * blockDim.x + threadIdx.x; q0 < A.total; q0 += 8 * T) {
-    double2 v[8];
-    uint32_t cd[8];
+  for (int q0 = blockIdx.x * blockDim.x + threadIdx.x; q0 < A.total; q0 += U * T) {
+    double2 v[U];
+    uint32_t cd[U];
 #pragma unroll
-    for (int c = 0; c < 8; ++c) {
+    for (int c = 0; c < U; ++c) {
       const int q = q0 + c * T;
       if (q < A.total) {
         cd[c] = A.code_ef ? ld_u32_ef(A.code + q, pf) : __ldg(A.code + q);
@@ -201,7 +203,7 @@ __global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
       }
     }
 #pragma unroll
-    for (int c = 0; c < 8; ++c) {
+    for (int c = 0; c < U; ++c) {
       const int q = q0 + c * T;
       if (q < A.total) {
         const uint32_t sl = cd[c] >> A.ibits, i = cd[c] & imask;

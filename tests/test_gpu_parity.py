@@ -293,7 +293,7 @@ def test_parity_snr_sweep(snr_db):
 @pytest.mark.parametrize("env", [{"CUSFFT_VOTE_PAIRS": "0"}, {"CUSFFT_VOTE_BITMAP": "1"}, {"CUSFFT_SELECT": "multi"}, {"CUSFFT_SELECT": "single"},
                                  {"CUSFFT_STAGE_MODE": "split_index"}, {"CUSFFT_STAGE_MODE": "fused_scatter"},
                                  {"CUSFFT_STAGE_MODE": "split_scatter"}, {"CUSFFT_NO_STAGE": "1"},
-                                 {"CUSFFT_STAGE_MODE": "fused_index"}, {"CUSFFT_P2": "ldg"}, {"CUSFFT_DISCARD": "1"},
+                                 {"CUSFFT_STAGE_MODE": "fused_index"}, {"CUSFFT_P2": "ldg"}, {"CUSFFT_DISCARD": "1"}, {"CUSFFT_STAGE_U": "8"}, {"CUSFFT_STAGE_U": "2"},
                                  {"CUSFFT_SLOT": "1"}, {"CUSFFT_SLOT": "2"}, {"CUSFFT_BRANCH": "1"}, {"CUSFFT_BRANCH": "2"}, {"CUSFFT_BRANCH": "3"}, {"CUSFFT_BRANCH": "4"}, {"CUSFFT_BRANCH": "5"},
                                  {"CUSFFT_STAGE_GROUPS": "2"}, {"CUSFFT_PACKED": "0"},
                                  {"CUSFFT_FFT_E": "1024"}, {"CUSFFT_FFT_E": "256"}, {"CUSFFT_PK": "0"}, {"CUSFFT_PDL_TRIGGER": "0"}, {"CUSFFT_PDL_TRIGGER": "63"}, {"CUSFFT_SPLIT_LAUNCH": "1"}, {"CUSFFT_EST_SEG": "0"}, {"CUSFFT_SEL_LOCALPICK": "1"}, {"CUSFFT_NODE_PRIO": "0"}, {"CUSFFT_BRANCH": "0"}])
