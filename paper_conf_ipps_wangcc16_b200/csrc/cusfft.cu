@@ -135,6 +135,7 @@ struct cusfft_plan_s {
   bool stage_packed = false;      // scatter schedule as packed (slot, i) words (k_stage_packed; CUSFFT_PACKED=0: off)
   int stage_ibits = 0;
   bool p2_tma = true;             // scatter phase 2 through bulk copies (k_fold_fft1_tma; CUSFFT_P2=ldg: k_fold_fft1 MODE 2)
+  int stage_bs = 256;             // phase-1 CTA size (CUSFFT_STAGE_BS = 128: A/B)
   int stage_u = 4;                // gathers in flight per phase-1 thread (CUSFFT_STAGE_U = 2 / 4 / 8 / 16)
   bool p2_discard = false;        // CUSFFT_DISCARD=1: drop consumed staging lines from L2 (default keeps them:
                                   // the next execution's phase-1 stores then hit valid set-aside lines)
@@ -611,6 +612,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   if (P->branched) P->stage_cps = 2;
   if (const char* e = std::getenv("CUSFFT_STAGE_CPS")) P->stage_cps = std::max(1, std::atoi(e));
   if (const char* e = std::getenv("CUSFFT_STAGE_U")) P->stage_u = std::atoi(e);
+  if (const char* e = std::getenv("CUSFFT_STAGE_BS")) P->stage_bs = std::atoi(e);
   if (const char* e = std::getenv("CUSFFT_P2")) P->p2_tma = std::string(e) != "ldg";
   if (const char* e = std::getenv("CUSFFT_DISCARD")) P->p2_discard = (e[0] == '1');
   {
@@ -1044,16 +1046,17 @@ int launch_stage1(cusfft_plan_t P, const cusfft_plan_s::StageGroup& g, const dou
     StagePackArgs a{x, g.code, g.staging, P->d_slots + (size_t)P->lrank * P->Lg + g.s0, tot, g.s1 - g.s0,
                     P->stage_ibits, P->R, ilog2(P->B), P->logB2, P->logB1, ilog2(256 / P->B1),
                     (uint32_t)(P->n - 1), z, P->code_ef ? 1 : 0};
+    // CUSFFT_STAGE_BS = 128: half-size CTAs (A/B; the grid keeps the same threads per SM)
+    const int bs = P->stage_bs == 128 ? 128 : 256;
+    const dim3 gr((unsigned)(bs == 128 ? 2 * grid : grid)), bl((unsigned)bs);
     if (P->stage_u == 2)
-      e = launch_k(k_stage_packed<2>, dim3(grid), dim3(256), 0, st, P->cur_prio, a);
-    else if (P->stage_u == 4)
-      e = launch_k(k_stage_packed<4>, dim3(grid), dim3(256), 0, st, P->cur_prio, a);
+      e = launch_k(k_stage_packed<2>, gr, bl, 0, st, P->cur_prio, a);
     else if (P->stage_u == 16)
-      e = launch_k(k_stage_packed<16>, dim3(grid), dim3(256), 0, st, P->cur_prio, a);
+      e = launch_k(k_stage_packed<16>, gr, bl, 0, st, P->cur_prio, a);
     else if (P->stage_u == 8)
-      e = launch_k(k_stage_packed<8>, dim3(grid), dim3(256), 0, st, P->cur_prio, a);
+      e = launch_k(k_stage_packed<8>, gr, bl, 0, st, P->cur_prio, a);
     else
-      e = launch_k(k_stage_packed<4>, dim3(grid), dim3(256), 0, st, P->cur_prio, a);
+      e = launch_k(k_stage_packed<4>, gr, bl, 0, st, P->cur_prio, a);
   } else {
     e = launch_k(k_stage, dim3(grid), dim3(256), 0, st, P->cur_prio, x, (const uint32_t*)g.spos,
                  (const uint32_t*)g.dst, g.staging, tot, z);
