@@ -105,7 +105,8 @@ struct cusfft_plan_s {
   bool xshard = false;
   int lrank = 0, lworld = 1;
   uint32_t xlo = 0, xspan = 0;
-  cusfft_params prm{};
+  cusfft_params prm{};            // prm.taps points at user_taps (plan-owned copy) or is NULL
+  std::vector<double> user_taps;  // host copy of caller-supplied taps (clones are built from it)
   int log2nb = 0, w = 0, R = 0, num = 0, Lloc = 0, T = 0, max_hits = 0;
   int Jcap = 0;  // winner-list capacity per loop (num, or B in THRESHOLD mode)
   int B1 = 1, B2 = 1, logB1 = 0, logB2 = 0;
@@ -563,6 +564,10 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   cusfft_plan_t P = new (std::nothrow) cusfft_plan_s();
   if (!P) return CUSFFT_ALLOC;
   P->n = n; P->k = k; P->B = B; P->L = L; P->prm = q; P->rank = rank; P->world = world;
+  if (q.taps) {  // the caller keeps ownership of its array: keep a copy (cusfft_set_pipeline clones read it)
+    P->user_taps.assign(q.taps, q.taps + q.num_taps);
+    P->prm.taps = P->user_taps.data();
+  }
   P->device = dev;
   P->nb = n / B;
   P->log2nb = ilog2(P->nb);
@@ -762,13 +767,17 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     g_last_cuda_error = (int)cudaGetLastError();
     return fail(CUSFFT_CUDA);
   }
+  // k_output needs up to 205 KB at k = 8192 (kp2 = 8192): allow the device's opt-in maximum
+  int smem_optin = 200 * 1024;
+  cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
   if (set_fft_attrs() != cudaSuccess ||
       cudaFuncSetAttribute(k_select, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_select1, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_select_cluster, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_select_sort, cudaFuncAttributeMaxDynamicSharedMemorySize, 210 * 1024) != cudaSuccess ||
       cudaFuncSetAttribute(k_vote, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess ||
-      cudaFuncSetAttribute(k_output, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024) != cudaSuccess) {
+      cudaFuncSetAttribute(k_output, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_optin) != cudaSuccess ||
+      P->output_smem > smem_optin) {
     g_last_cuda_error = (int)cudaGetLastError();
     return fail(CUSFFT_CUDA);
   }
@@ -988,10 +997,10 @@ cudaError_t launch_fold_fft1_t(cusfft_plan_t P, const double2* x, const uint32_t
                     (int)P->B, P->B2, P->w, P->R, (uint32_t)(P->n - 1), 0u, (uint32_t)P->n, z);
   if (staged_tord && P->p2_tma && P->R <= 48) {  // staged in thread order, rows moved by bulk copies
     const size_t smem = (size_t)P->R * 4096 + (size_t)g_p2_pad;
-    static thread_local bool attr_set[4] = {false, false, false, false};
-    if (!attr_set[B1T / 64]) {  // static + dynamic smem may exceed the 48 KB default
+    static thread_local bool attr_set = false;  // one flag per B1T instantiation
+    if (!attr_set) {  // static + dynamic smem may exceed the 48 KB default
       cudaFuncSetAttribute(k_fold_fft1_tma<B1T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-      attr_set[B1T / 64] = true;
+      attr_set = true;
     }
     return launch_k(k_fold_fft1_tma<B1T>, grid, dim3(256), smem, st, P->cur_prio, x,
                     (const double*)P->d_taps_perm, P->prm.debug ? u : nullptr, v, (const double2*)P->d_tw, (int)P->B, P->B2, P->w, P->R,
@@ -1752,20 +1761,26 @@ int cusfft_set_pipeline(cusfft_plan_t plan, int32_t depth) {
     free_plan(plan->subs.back());
     plan->subs.pop_back();
   }
-  while ((int)plan->subs.size() < depth - 1) {
-    cusfft_plan_t sp = nullptr;
-    const int rc = cusfft_plan(&sp, plan->n, plan->k, plan->B, plan->L, &plan->prm);
-    if (rc) return rc;
-    cudaStream_t st = nullptr;
-    CK(cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking));
-    sp->stream = st;
-    sp->own_stream = true;
-    plan->subs.push_back(sp);
-  }
+  // events first: execute_batch indexes sub_ev[depth] for depth = 1 + subs.size()
   while ((int)plan->sub_ev.size() < depth + 1) {
     cudaEvent_t e;
     CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     plan->sub_ev.push_back(e);
+  }
+  while ((int)plan->subs.size() < depth - 1) {
+    cusfft_plan_t sp = nullptr;
+    const int rc = cusfft_plan(&sp, plan->n, plan->k, plan->B, plan->L, &plan->prm);  // prm.taps: the plan's own copy
+    if (rc) return rc;  // subs keeps its previous (consistent) size
+    cudaStream_t st = nullptr;
+    const cudaError_t e = cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking);
+    if (e != cudaSuccess) {
+      g_last_cuda_error = (int)e;
+      free_plan(sp);
+      return CUSFFT_CUDA;
+    }
+    sp->stream = st;
+    sp->own_stream = true;
+    plan->subs.push_back(sp);
   }
   return CUSFFT_SUCCESS;
 }
