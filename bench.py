@@ -14,6 +14,7 @@ from __future__ import annotations
 
 import argparse
 import json
+import math
 import os
 import statistics
 import subprocess
@@ -38,10 +39,48 @@ CONFIGS = {
     "C5": (2 ** 22, 1000, 16, "n=2^22, k=1000, batch of 64 independent noiseless fp64 signals, signals sharded over GPUs"),
 }
 BATCH = {"C5": 64}
-# Filter tolerance delta per config (the paper leaves it open).  C3: 1e-7 keeps
-# exact recovery and L1 <= 1.75e-7 on 48/48 oracle seeds (DESIGN.md §3 study)
-# with 12% fewer taps than the library default 1e-8.
-TOLERANCE = {"C1": 1e-8, "C2": 1e-8, "C3": 1e-7, "C4": 1e-8, "C5": 1e-8}
+# Filter and cutoff parameters per config (the paper leaves them open, DESIGN.md
+# §3 [Z1], [Z17], [Z21]): tolerance delta, main-lobe half width lambda = lam_B / B,
+# optionally the location loops' own (loc_tol, loc_lam_B), and num_select = num_k * k.
+# C3: delta = 1e-7 with lambda = 0.75 / B (2/3 of the taps of lambda = 0.5 / B):
+# exact recovery and L1 <= 2.1e-7 on 48 + 192 oracle seeds (scripts/study/n3_study*.jsonl).
+FILTERS = {
+    "C1": dict(tol=1e-8, lam_B=0.5),
+    "C2": dict(tol=1e-8, lam_B=0.5),
+    "C3": dict(tol=1e-7, lam_B=0.75),
+    "C4": dict(tol=1e-8, lam_B=0.5),
+    "C5": dict(tol=1e-8, lam_B=0.5),
+}
+# the library defaults (cusfft_params_default), reported beside the tuned line
+DEFAULT_FILTER = dict(tol=1e-8, lam_B=0.5)
+
+
+def plan_params(config: str, B: int | None = None, filt: dict | None = None) -> dict:
+    """Plan keyword arguments (cusfft_params fields) of a config's filter / cutoff."""
+    n, k = CONFIGS[config][:2]
+    if B is None:  # the paper's formula B = floor_pow2(sqrt(n k / log2 n)) (PAPER.md:L196, L228)
+        B = 1 << int(math.floor(math.log2(math.sqrt(n * k / math.log2(n)))))
+    f = dict(FILTERS[config] if filt is None else filt)
+    out = dict(tolerance=f["tol"], lobefrac=f["lam_B"] / B)
+    if "loc_tol" in f:
+        out["loc_tolerance"] = f["loc_tol"]
+    if "loc_lam_B" in f:
+        out["loc_lobefrac"] = f["loc_lam_B"] / B
+    if "num_k" in f:
+        out["num_select"] = int(round(f["num_k"] * k))
+    return out
+
+
+def filter_desc(config: str, filt: dict | None = None) -> str:
+    f = FILTERS[config] if filt is None else filt
+    d = f"Dolph-Chebyshev delta={f['tol']:g}, lambda={f['lam_B']:g}/B"
+    if "loc_tol" in f or "loc_lam_B" in f:
+        d += f"; location loops delta={f.get('loc_tol', f['tol']):g}, lambda={f.get('loc_lam_B', f['lam_B']):g}/B"
+    if "num_k" in f:
+        d += f"; num={f['num_k']:g}k"
+    return d
+
+
 METRIC = "ms per sparse FFT at n=2^24,k=1000 (1/2/4/8 B200); x vs dense cuFFT; HBM GB/s"
 PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
 FALLBACK_HBM = 6650.0
@@ -53,17 +92,6 @@ def hbm_peak():
             return float(json.load(f)["hbm_gbs"]), "measured (MEASURED_PEAKS.json copy bandwidth)"
     except Exception:
         return FALLBACK_HBM, "fallback (B200_PROFILING.md)"
-
-
-def fold_bytes(L: int, w: int, B: int, sectors: int):
-    """Algorithmic bytes of the fold stage: the distinct
-    32-B DRAM sectors of x that the plan's L*w gather positions touch (exact,
-    counted at plan time; a random 16-B sample cannot cost less than its
-    sector, and a sector shared by several loops need be read once), the w fp64
-    taps, and the L*B complex fp64 buckets written (u, plus v when the first
-    FFT pass is fused, B > 2048).  `useful` counts 16 B per sample instead."""
-    out = L * B * 16 * (2 if 2048 < B <= 65536 else 1)
-    return sectors * 32 + w * 8 + out, L * w * 16 + w * 8 + out
 
 
 class ClockSampler:
@@ -128,22 +156,42 @@ def make_signal(n, k, seed):
 # ---------------------------------------------------------------------------
 # CPU oracle legs (the oracle is test infrastructure; bench may time it here)
 # ---------------------------------------------------------------------------
-def oracle_time(n, k, L, B, x, seed, budget_s=20.0, min_runs=1, max_runs=None, tolerance=1e-8):
+def host_cores() -> int:
+    return len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else (os.cpu_count() or 1)
+
+
+def oracle_time(config, n, k, L, B, x, seed, budget_s=20.0, min_runs=1, max_runs=None):
+    """The oracle transform as it stands (plan-time filter excluded), pinned to
+    one host core (sched_setaffinity, like taskset -c) with one BLAS thread."""
     import oracle
-    p = oracle.make_params(n, k, B=B, L=L, seed=seed, tolerance=tolerance)
+    prm = plan_params(config, B)
+    okw = {kk: prm[kk] for kk in ("tolerance", "lobefrac", "loc_tolerance", "loc_lobefrac", "num_select") if kk in prm}
+    p = oracle.make_params(n, k, B=B, L=L, seed=seed, **okw)
     g = oracle.filter_taps(p)
     Ghat = oracle.filter_response(g, n, n // B)
+    gl = oracle.filter_taps(oracle.loc_filter_params(p)) if oracle.separate_filters(p) else None
+    cores = host_cores()
+    pinned = None
+    if hasattr(os, "sched_setaffinity"):
+        before = os.sched_getaffinity(0)
+        core = min(before)
+        os.sched_setaffinity(0, {core})
+        pinned = core
     times = []
-    t_start = time.perf_counter()
-    while True:
-        t0 = time.perf_counter()
-        res = oracle.sfft(x, p, taps=g, Ghat=Ghat)
-        times.append(time.perf_counter() - t0)
-        if max_runs is not None and len(times) >= max_runs:
-            break
-        if len(times) >= min_runs and time.perf_counter() - t_start >= budget_s:
-            break
-    return times, res
+    try:
+        t_start = time.perf_counter()
+        while True:
+            t0 = time.perf_counter()
+            res = oracle.sfft(x, p, taps=g, Ghat=Ghat, taps_loc=gl)
+            times.append(time.perf_counter() - t0)
+            if max_runs is not None and len(times) >= max_runs:
+                break
+            if len(times) >= min_runs and time.perf_counter() - t_start >= budget_s:
+                break
+    finally:
+        if pinned is not None:
+            os.sched_setaffinity(0, before)
+    return times, res, cores, pinned
 
 
 def run_reference(args):
@@ -155,19 +203,20 @@ def run_reference(args):
     from oracle import default_B
     B = default_B(n, k)
     x, S, X = make_signal(n, k, args.signal_seed)
-    times, _ = oracle_time(n, k, L, B, x, args.plan_seed, budget_s=0, min_runs=args.warmup + args.steps,
-                           max_runs=args.warmup + args.steps, tolerance=TOLERANCE[args.config])
+    times, _, cores, core = oracle_time(args.config, n, k, L, B, x, args.plan_seed, budget_s=0,
+                                        min_runs=args.warmup + args.steps, max_runs=args.warmup + args.steps)
     t = times[args.warmup:]
     ms = 1e3 * sum(t) / len(t)
     line = {
         "impl": "reference", "metric": METRIC, "value": ms, "unit": "ms", "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": False,
         "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": f"{args.config}: {desc}, L={L}, B={B}, delta={TOLERANCE[args.config]:g}",
-                   "n": n, "k": k, "B": B, "L": L, "tolerance": TOLERANCE[args.config]},
+        "config": {"workload": f"{args.config}: {desc}, L={L}, B={B}, {filter_desc(args.config)}",
+                   "n": n, "k": k, "B": B, "L": L, **plan_params(args.config, B)},
         "cpu_baseline": {"value": ms, "unit": "ms", "cores": 1, "kind": "oracle",
                          "sample": f"{len(t)} full oracle transforms of the {args.config} workload "
-                                   "(plan-time filter construction excluded), numpy single thread"},
+                                   f"(plan-time filter construction excluded), numpy, pinned to core {core}: "
+                                   f"1 of {cores} host cores"},
         "e2e": {"value": ms, "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -177,6 +226,35 @@ def run_reference(args):
 # ---------------------------------------------------------------------------
 # GPU arm
 # ---------------------------------------------------------------------------
+class L2Flush:
+    """L2 flush between timed steps: write 256 MiB (evicts every normal line),
+    then read another 256 MiB so the write-backs happen here, not in the step.
+    cold=True first returns every persisting line to normal
+    (cudaCtxResetPersistingL2Cache), so a staged plan's staging buffer is
+    flushed too (the persisting set-aside otherwise keeps it resident)."""
+
+    def __init__(self, dev):
+        import torch
+        self.w = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=dev)
+        self.r = torch.ones(64 * 1024 * 1024, dtype=torch.int32, device=dev)
+        self._reset = None
+
+    def __call__(self, cold: bool = False):
+        if cold:
+            if self._reset is None:
+                from cuda.bindings import runtime as rt
+                self._reset = rt.cudaCtxResetPersistingL2Cache
+            self._reset()
+        self.w.zero_()
+        self.r.sum()
+
+
+PAPER_CONTEXT = ("cusFFT (PAPER.md, fp64, Tesla K20x: Kepler GK110, 14 SMs, 250 GB/s, CUDA 5.5; Table I L412-L414): "
+                 "15x over cuFFT at n=2^27 (>9x baseline, L406), faster than cuFFT for n > 2^22 (L402); "
+                 "0.5x-29x over parallel FFTW 3.3 on a 6-core Xeon E5-2640 Sandy Bridge (Table II L418-L420, L426); "
+                 "up to 6.6x over PsFFT (OpenMP sFFT) at n=2^24, transfers included (L426)")
+
+
 def run_gpu(args):
     import torch
     import torch.distributed as dist
@@ -193,67 +271,56 @@ def run_gpu(args):
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
 
-    from paper_conf_ipps_wangcc16_b200 import Plan, default_B
-    from paper_conf_ipps_wangcc16_b200.dist import CudaEngine, LoopShardedSfft, signal_range
+    from paper_conf_ipps_wangcc16_b200 import Plan, default_B, nccl_unique_id
 
     n, k, L, desc = CONFIGS[args.config]
     B = args.B or default_B(n, k)
+    prm = plan_params(args.config, B)
     x_np, S, X = make_signal(n, k, args.signal_seed)
     x_pin = torch.from_numpy(x_np).pin_memory()
     x = x_pin.to(dev)
+    flush = L2Flush(dev)
+    stream = torch.cuda.current_stream()
 
-    flush_w = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=dev)
-    flush_r = torch.ones(64 * 1024 * 1024, dtype=torch.int32, device=dev)
-
-    class _Flush:
-        """L2 flush between timed steps: write 256 MiB (evicts everything), then
-        read another 256 MiB so the write-backs happen here, not in the step."""
-
-        @staticmethod
-        def zero_():
-            flush_w.zero_()
-            flush_r.sum()
-
-    flush = _Flush()
+    def time_steps(fn, reps, cold=False):
+        ts = []
+        for _ in range(reps):
+            flush(cold)
+            a = torch.cuda.Event(enable_timing=True)
+            b = torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            fn()
+            b.record(stream)
+            torch.cuda.synchronize()
+            ts.append(a.elapsed_time(b))
+        return ts
 
     # ---- dense cuFFT of the same n (context), complex128, L2 flushed; timed
     # before any plan exists, so cuFFT has the whole L2 (a staged plan holds a
-    # persisting-L2 set-aside while it lives, DESIGN.md §6.2)
-    dense = []
-    for i in range(args.warmup + 10):
-        flush.zero_()
-        a = torch.cuda.Event(enable_timing=True)
-        b = torch.cuda.Event(enable_timing=True)
-        a.record(torch.cuda.current_stream())
-        torch.fft.fft(x)
-        b.record(torch.cuda.current_stream())
-        torch.cuda.synchronize()
-        if i >= args.warmup:
-            dense.append(a.elapsed_time(b))
-    dense_ms = statistics.median(dense)
+    # persisting-L2 set-aside while it lives, include/cusfft.h)
+    dense_ms = statistics.median(time_steps(lambda: torch.fft.fft(x), args.warmup + 10)[args.warmup:])
 
+    t_plan0 = time.perf_counter()
     if world == 1:
-        plan = Plan(n, k, B=B, L=L, seed=args.plan_seed, device=local_rank, tolerance=TOLERANCE[args.config])
-        locs = torch.empty(k, dtype=torch.int64, device=dev)
-        vals = torch.empty(k, dtype=torch.complex128, device=dev)
-
-        def step():
-            plan.execute(x, locs, vals)
-            return locs, vals
-        launches = plan.launches_per_execute()
-    else:
+        plan = Plan(n, k, B=B, L=L, seed=args.plan_seed, device=local_rank, **prm)
+    else:  # the plan owns the exchange: rank 0's ncclUniqueId broadcast once over the process group
+        uid = [nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(uid, src=0)
         shard = 1 if args.shard == "signal" else 0
-        eng = CudaEngine(n, k, B=B, L=L, rank=rank, world=world, device=local_rank, seed=args.plan_seed,
-                         tolerance=TOLERANCE[args.config], shard_mode=shard)
-        runner = LoopShardedSfft(eng)
-        plan = eng.plan
+        plan = Plan(n, k, B=B, L=L, seed=args.plan_seed, device=local_rank, rank=rank, world=world,
+                    nccl_id=uid[0], shard_mode=shard, **prm)
         if shard:  # this rank holds only its slice of x
-            lo, hi = signal_range(rank, n, world)
-            x = x[lo:hi].clone()
+            span = n // world
+            x = x[rank * span:(rank + 1) * span].clone()
+    plan_ms = 1e3 * (time.perf_counter() - t_plan0)
+    locs = torch.empty(k, dtype=torch.int64, device=dev)
+    vals = torch.empty(k, dtype=torch.complex128, device=dev)
 
-        def step():
-            return runner.execute(x)
-        launches = eng.launches_per_execute()
+    def step():
+        plan.execute(x, locs, vals)
+        return locs, vals
+    launches = plan.launches_per_execute()
+    info = plan.info()
 
     # correctness of the benchmarked configuration (untimed)
     l_out, v_out = step()
@@ -265,8 +332,6 @@ def run_gpu(args):
     got = {int(f): complex(v) for f, v in zip(l_np, v_np) if f >= 0}
     l1 = sum(abs(got.get(f, 0) - truth.get(f, 0)) for f in set(truth) | set(got)) / k
 
-    stream = torch.cuda.current_stream()
-
     def barrier():
         if world > 1:
             dist.barrier()
@@ -276,7 +341,7 @@ def run_gpu(args):
         t0 = time.perf_counter()
         i = 0
         while i < args.warmup or time.perf_counter() - t0 < 0.3:
-            flush.zero_()
+            flush()
             step()
             i += 1
         torch.cuda.synchronize()
@@ -288,84 +353,78 @@ def run_gpu(args):
         reg1 = torch.cuda.Event(enable_timing=True)
         reg0.record(stream)
         for s in range(args.steps):
-            flush.zero_()                       # L2 flush, outside the step's events
+            flush()                             # L2 flush, outside the step's events
             ev[s][0].record(stream)
             step()
             ev[s][1].record(stream)
         reg1.record(stream)
         torch.cuda.synchronize()
         barrier()
-        # keep load on for the sampler a little longer
-        t1 = time.perf_counter()
-        while time.perf_counter() - t1 < 0.2:
-            step()
+        # the cold arm: the same steps with the persisting lines reset before each flush
+        cold_ms = time_steps(step, args.steps, cold=True)
         torch.cuda.synchronize()
     step_ms = [a.elapsed_time(b) for a, b in ev]
     ms = sum(step_ms) / len(step_ms)
+    cold = sum(cold_ms) / len(cold_ms)
     region_ms = reg0.elapsed_time(reg1)
     if world > 1:
-        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        t = torch.tensor([ms, cold], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms = float(t.item())
+        ms, cold = float(t[0].item()), float(t[1].item())
+
+    # ---- the roofline kernel (phase 1 of the staged fold, the permute gather)
+    # timed INSIDE the bench's CUDA graph: event-record nodes before and after it
+    # (cusfft_set_timing mode 2), same flush, warm and cold
+    gather = {}
+    if info["staged"]:
+        for nm, cold_flag in (("warm", False), ("cold", True)):
+            plan.set_timing(2)
+            g, tot = [], []
+            for _ in range(max(10, args.steps)):
+                flush(cold_flag)
+                step()
+                st = plan.stage_times()
+                g.append(st["gather"])
+                tot.append(st["fold"])
+            plan.set_timing(0)
+            if all(v > 0 for v in g):
+                gather[nm] = {"ms": sum(g) / len(g), "graph_ms": sum(tot) / len(tot)}
 
     # ---- per-stage times inside the CUDA graph: T_s = time of the graph that
-    # runs stages 1..s (cusfft_set_stage_limit), stage s = T_s - T_{s-1}.
-    # T_1 is the fold kernel alone (+ an 8-int memset node): the roofline's
-    # kernel time, measured with CUDA events on the plan's (current) stream.
-    def timed_mean(reps):
-        ts = []
-        for _ in range(reps):
-            flush.zero_()
-            a = torch.cuda.Event(enable_timing=True)
-            b = torch.cuda.Event(enable_timing=True)
-            a.record(stream)
-            step()
-            b.record(stream)
-            torch.cuda.synchronize()
-            ts.append(a.elapsed_time(b))
-        return sum(ts) / len(ts)
-
+    # runs stages 1..s (cusfft_set_stage_limit), stage s = T_s - T_{s-1}
     names = ("fold", "fft", "cutoff", "vote", "estimate", "output")
     stage_ms = {}
     if world == 1:
         prev = 0.0
         reps = max(10, args.steps)
         for si, nm in enumerate(names, start=1):
+            if info["tail"] and si > 4:
+                break
             plan.set_stage_limit(si)
             step()
-            tsi = timed_mean(reps)
-            stage_ms[nm] = tsi - prev
+            tsi = sum(time_steps(step, reps)) / reps
+            stage_ms["tail (vote + estimate + output)" if (info["tail"] and si == 4) else nm] = tsi - prev
             prev = tsi
         plan.set_stage_limit(6)
-        fold_ms = stage_ms["fold"]
-    else:
-        plan.set_timing(True)
-        acc = {nm: [] for nm in names}
-        for _ in range(max(5, args.steps)):
-            flush.zero_()
-            step()
-            st = plan.stage_times()
-            for nm in names:
-                acc[nm].append(st[nm])
-        plan.set_timing(False)
-        stage_ms = {nm: sum(v) / len(v) for nm, v in acc.items()}
-        fold_ms = stage_ms["fold"]
 
-    # ---- the gather kernel alone (phase 1 of the staged fold, k_stage*): events
-    # recorded on the plan's stream right before and after its launch (timing
-    # mode: direct launches, no graph), L2 flushed before every execution
-    gather_ms = None
-    if plan.info()["staged"]:
-        plan.set_timing(True)
-        g = []
-        for _ in range(max(10, args.steps)):
-            flush.zero_()
-            step()
-            g.append(plan.stage_times()["gather"])
-        plan.set_timing(False)
-        if all(v > 0 for v in g):
-            gather_ms = sum(g) / len(g)
-
+    # ---- CUPTI cross-check of the kernel durations (torch.profiler: no replay)
+    cupti = None
+    if world == 1 and not args.no_cupti:
+        try:
+            acts = [torch.profiler.ProfilerActivity.CUDA]
+            with torch.profiler.profile(activities=acts) as prof:
+                for _ in range(10):
+                    flush()
+                    step()
+                torch.cuda.synchronize()
+            per = {}
+            for e in prof.events():
+                if e.device_type == torch.autograd.DeviceType.CUDA and "cusfft::" in e.name:
+                    short = e.name.split("(")[0].replace("void ", "").replace("cusfft::", "")
+                    per.setdefault(short, []).append(e.device_time)
+            cupti = {kk: {"launches": len(v), "mean_us": sum(v) / len(v)} for kk, v in sorted(per.items())}
+        except Exception as exc:  # pragma: no cover
+            cupti = {"error": str(exc)[:200]}
 
     # ---- e2e through the C ABI with host buffers (world == 1 path)
     e2e = None
@@ -376,7 +435,7 @@ def run_gpu(args):
             plan.execute_host(x_pin, h_locs, h_vals)
         e_ms = []
         for _ in range(args.steps):
-            flush.zero_()
+            flush()
             torch.cuda.synchronize()
             t0 = time.perf_counter()
             plan.execute_host(x_pin, h_locs, h_vals)
@@ -385,105 +444,101 @@ def run_gpu(args):
                "d2h_bytes_per_step": k * (8 + 16),
                "note": "cusfft_execute_host: pinned H2D of x, transform, D2H of locs/vals, host wall clock"}
 
+    # ---- the library-default filter (delta = 1e-8, lambda = 0.5/B) on the same signal
+    default_line = None
+    if world == 1 and args.config == "C3" and not args.no_default_line:
+        pd = Plan(n, k, B=B, L=L, seed=args.plan_seed, device=local_rank, **plan_params(args.config, B, DEFAULT_FILTER))
+        l2_, v2_ = torch.empty_like(locs), torch.empty_like(vals)
+        for _ in range(3):
+            flush()
+            pd.execute(x, l2_, v2_)
+        ts = time_steps(lambda: pd.execute(x, l2_, v2_), args.steps)
+        default_line = {"filter": filter_desc(args.config, DEFAULT_FILTER), "taps": pd.w,
+                        "ms": sum(ts) / len(ts), "exact_recovery": set(l2_.cpu().tolist()) == set(S.tolist()),
+                        "status": pd.status()}
+        pd.close()
+
     ablations = None
     if world == 1 and args.ablations:
         ablations = {}
-        variants = [("cutoff_sort_alg3", dict(cutoff_mode=1), {}),
-                    ("cutoff_threshold_alg6", dict(cutoff_mode=2, cutoff_threshold=1e-3), {}),
-                    ("direct_gather_no_stage", {}, {"CUSFFT_NO_STAGE": "1"})]
-        for name, kw, env in variants:
-            old = {e: os.environ.get(e) for e in env}
-            os.environ.update(env)
-            try:
-                p2 = Plan(n, k, B=B, L=L, seed=args.plan_seed, device=local_rank, tolerance=TOLERANCE[args.config], **kw)
-            finally:
-                for e, v in old.items():
-                    if v is None:
-                        os.environ.pop(e, None)
-                    else:
-                        os.environ[e] = v
+        variants = [("cutoff_sort_alg3", dict(cutoff_mode=1)),
+                    ("cutoff_threshold_alg6", dict(cutoff_mode=2, cutoff_threshold=1e-3)),
+                    ("direct_gather_no_stage", dict(gather=1)),
+                    ("no_l2_persist", dict(l2_persist=0))]
+        for name, kw in variants:
+            p2 = Plan(n, k, B=B, L=L, seed=args.plan_seed, device=local_rank, **{**prm, **kw})
             l2_, v2_ = torch.empty_like(locs), torch.empty_like(vals)
-
-            def step2():
-                p2.execute(x, l2_, v2_)
             for _ in range(3):
-                step2()
-            ts = []
-            for _ in range(max(10, args.steps)):
-                flush.zero_()
-                a = torch.cuda.Event(enable_timing=True)
-                b = torch.cuda.Event(enable_timing=True)
-                a.record(stream)
-                step2()
-                b.record(stream)
-                torch.cuda.synchronize()
-                ts.append(a.elapsed_time(b))
+                p2.execute(x, l2_, v2_)
+            ts = time_steps(lambda: p2.execute(x, l2_, v2_), max(10, args.steps))
             ok = set(l2_.cpu().tolist()) == set(S.tolist())
             ablations[name] = {"ms": sum(ts) / len(ts), "exact_recovery": ok, "status": p2.status()}
             p2.close()
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:  # N = 1 only (bench contract)
-        times, _ = oracle_time(n, k, L, B, x_np, args.plan_seed, budget_s=args.cpu_budget_s, min_runs=1,
-                               tolerance=TOLERANCE[args.config])
+        times, _, cores, core = oracle_time(args.config, n, k, L, B, x_np, args.plan_seed,
+                                            budget_s=args.cpu_budget_s, min_runs=1)
         cpu = {"value": 1e3 * sum(times) / len(times), "unit": "ms", "cores": 1, "kind": "oracle",
                "sample": f"{len(times)} full oracle transform(s) of the same {args.config} signal "
-                         "(plan-time filter construction excluded), numpy single thread"}
+                         f"(plan-time filter construction excluded), numpy, pinned to core {core}: "
+                         f"1 of {cores} host cores"}
 
     peak, peak_src = hbm_peak()
-    info = plan.info()
-    sector, useful = fold_bytes(plan.L // world if world > 1 else L, plan.w, B, int(info["sectors"]))
-    # roofline kernel: the address-ordered permute gather (fold phase 1) when
-    # the plan is staged -- it carries all of the fold's HBM traffic; phase 2
-    # streams the staging buffer from L2 (reported as fold_stage below)
+    # roofline kernel: the address-ordered permute gather (fold phase 1) -- it
+    # carries all of the transform's HBM traffic.  Algorithmic bytes: 32 B per
+    # distinct sector of x the plan's gathers touch.
     gather_bytes = int(info["sectors"]) * 32
-    rk_ms = gather_ms if gather_ms else fold_ms
-    rk_bytes = gather_bytes if gather_ms else sector
-    achieved = rk_bytes / (rk_ms * 1e-3) / 1e9
+    sum_w = int(info["w_loc"]) * plan.loc_loops + int(info["w"]) * (L - plan.loc_loops) if info["filters"] == 2 else L * plan.w
+    rk_ms = gather["warm"]["ms"] if "warm" in gather else stage_ms.get("fold", 0.0)
+    achieved = gather_bytes / (rk_ms * 1e-3) / 1e9
     traffic = None
     tf = os.path.join(ROOT, "profiles", f"fold_traffic_{args.config}.json")
     if os.path.exists(tf):
         try:
             with open(tf) as f:
                 tj = json.load(f)
-            parts = {kk.split("<")[0]: vv for kk, vv in tj.get("parts", {}).items()}
-            traffic = (parts.get("k_stage_packed", {}).get("dram_bytes_per_launch")
-                       if gather_ms else tj.get("dram_bytes_per_launch"))
+            if tj.get("sum_w") == sum_w:  # only a capture of this very plan counts
+                traffic = tj.get("k_stage_packed_dram_bytes_per_launch")
         except Exception:
             traffic = None
     line = {
         "metric": METRIC, "value": ms, "unit": "ms", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": False,
         "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": f"{args.config}: {desc}, L={L}, B={B}, w={plan.w} taps "
-                               f"(Dolph-Chebyshev, delta={TOLERANCE[args.config]:g})",
-                   "n": n, "k": k, "B": B, "L": L, "taps": plan.w, "tolerance": TOLERANCE[args.config],
-                   "loc_loops": plan.loc_loops,
-                   "vote_threshold": plan.T, "parallelism": f"{args.shard}-sharded x{world}" if world > 1 else "single GPU",
-                   "l2": "flushed between timed steps (256 MiB write + 256 MiB read), outside the step events",
+        "config": {"workload": f"{args.config}: {desc}, L={L}, B={B}, {filter_desc(args.config)}, "
+                               f"{sum_w} gathers (taps x loops)",
+                   "n": n, "k": k, "B": B, "L": L, "taps": plan.w, "taps_loc": int(info["w_loc"]),
+                   **prm, "loc_loops": plan.loc_loops, "vote_threshold": plan.T,
+                   "parallelism": f"{args.shard}-sharded x{world} (NCCL in the plan's graph)" if world > 1 else "single GPU",
+                   "l2": "flushed between timed steps (256 MiB write + 256 MiB read), outside the step events; "
+                         "the staging buffer's persisting lines survive it (warm); value_cold resets them too",
                    "signal_seed": args.signal_seed, "plan_seed": args.plan_seed},
+        "value_cold": cold,
+        "plan_ms": plan_ms,
         "gpu_launches": launches * args.steps,
         "timed_region_ms_incl_flush": region_ms,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic,
-                     "kernel": ("k_stage_packed (fold phase 1: address-ordered permute gather of x)" if gather_ms
-                                else "fold stage (k_fold_fft1)"),
-                     "algorithmic_bytes_per_launch": rk_bytes, "kernel_ms": rk_ms,
-                     "algorithmic_bytes_note": "distinct 32-B sectors of x the plan's L*w gather positions touch x 32 B",
-                     "peak_source": peak_src,
-                     "fold_stage": {"kernels": "k_stage_packed + k_fold_fft1_tma" if info["staged"] else "k_fold_fft1",
-                                    "ms": fold_ms, "algorithmic_bytes": sector, "useful_bytes": useful,
-                                    "gbs": sector / (fold_ms * 1e-3) / 1e9,
-                                    "frac": sector / (fold_ms * 1e-3) / 1e9 / peak,
-                                    "note": "graph-prefix time (includes the graph launch)"}},
+                     "kernel": "k_stage_packed (fold phase 1: address-ordered permute gather of x)",
+                     "algorithmic_bytes_per_launch": gather_bytes, "kernel_ms": rk_ms,
+                     "algorithmic_bytes_note": "32 B per distinct 32-B sector of x the plan's gathers touch "
+                                               f"({int(info['sectors'])} sectors; L*w*32 = {sum_w * 32} B before sharing)",
+                     "kernel_ms_how": "CUDA event-record nodes around the kernel inside the bench's graph, "
+                                      "L2 flushed before each execution",
+                     "kernel_ms_cold": gather.get("cold", {}).get("ms"),
+                     "frac_cold": (gather_bytes / (gather["cold"]["ms"] * 1e-3) / 1e9 / peak) if "cold" in gather else None,
+                     "peak_source": peak_src},
         "stage_ms": stage_ms,
+        "kernels_cupti_us": cupti,
+        "default_filter": default_line,
         "ablations": ablations,
         "dense_cufft_ms": dense_ms, "speedup_vs_dense_cufft": dense_ms / ms,
         "accuracy": {"exact_recovery": exact, "l1_per_coefficient": l1, "status": status},
         "clocks": clocks.summary(),
         "e2e": e2e,
         "cpu_baseline": cpu,
-        "paper_context": "cusFFT (K20x, fp64): 15x over cuFFT at n=2^27, >9x baseline (PAPER.md:L406)",
+        "paper_context": PAPER_CONTEXT,
     }
     if rank == 0:
         print(json.dumps(line), flush=True)
@@ -513,7 +568,7 @@ def run_gpu_batch(args):
     n, k, L, desc = CONFIGS[args.config]
     count = BATCH[args.config]
     B = default_B(n, k)
-    plan = Plan(n, k, B=B, L=L, seed=args.plan_seed, device=local_rank, tolerance=TOLERANCE[args.config])
+    plan = Plan(n, k, B=B, L=L, seed=args.plan_seed, device=local_rank, **plan_params(args.config, B))
     plan.set_pipeline(args.pipeline)
 
     class _Eng:
@@ -525,15 +580,11 @@ def run_gpu_batch(args):
     xb = xb_pin.to(dev)
     locs = torch.empty(len(mine), k, dtype=torch.int64, device=dev)
     vals = torch.empty(len(mine), k, dtype=torch.complex128, device=dev)
-
-    def step():
-        return drv.execute(xb) if len(mine) else (locs, vals)
     plan.execute_batch(xb, locs, vals)
     torch.cuda.synchronize()
     status = plan.status()
     exact = all(set(locs[i].cpu().tolist()) == set(sigs[i][1].tolist()) for i in range(len(mine)))
-    flush_w = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=dev)
-    flush_r = torch.ones(64 * 1024 * 1024, dtype=torch.int32, device=dev)
+    flush = L2Flush(dev)
     stream = torch.cuda.current_stream()
 
     def barrier():
@@ -541,14 +592,14 @@ def run_gpu_batch(args):
             dist.barrier()
     with ClockSampler(local_rank) as clocks:
         for _ in range(args.warmup):
-            flush_w.zero_(); flush_r.sum()
+            flush()
             plan.execute_batch(xb, locs, vals)
         torch.cuda.synchronize()
         ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
         barrier()
         torch.cuda.synchronize()
         for s_ in range(args.steps):
-            flush_w.zero_(); flush_r.sum()
+            flush()
             ev[s_][0].record(stream)
             plan.execute_batch(xb, locs, vals)
             ev[s_][1].record(stream)
@@ -585,7 +636,7 @@ def run_gpu_batch(args):
     line = {
         "metric": METRIC, "value": ms, "unit": "ms", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": batch_ms, "higher_is_better": False,
-        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "scaling": "weak" if world > 1 else "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
         "config": {"workload": f"{args.config}: {desc}, L={L}, B={B}, w={plan.w}, pipeline depth {args.pipeline}",
                    "n": n, "k": k, "B": B, "L": L, "batch": count, "per_rank": len(mine),
                    "parallelism": f"signal-batch sharded x{world} (no collective)",
@@ -620,8 +671,10 @@ def main():
     ap.add_argument("--pipeline", type=int, default=2, help="C5 batch: clone plans in flight per GPU")
     ap.add_argument("--cpu-budget-s", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-cupti", action="store_true")
+    ap.add_argument("--no-default-line", action="store_true")
     ap.add_argument("--ablations", action="store_true",
-                    help="also time the cutoff variants (Alg. 3 sort, Alg. 6 threshold) and the direct gather")
+                    help="also time the cutoff variants (Alg. 3 sort, Alg. 6 threshold), the direct gather, no L2 set-aside")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

@@ -37,7 +37,7 @@
 extern "C" {
 #endif
 
-#define CUSFFT_ABI_VERSION 1
+#define CUSFFT_ABI_VERSION 2
 
 typedef struct cusfft_plan_s* cusfft_plan_t; /* opaque; owns all device workspace */
 
@@ -53,7 +53,8 @@ typedef enum {
   CUSFFT_CUDA = -8,           /* a CUDA runtime call failed (cusfft_last_cuda_error)  */
   CUSFFT_HIT_OVERFLOW = -9,   /* more than max_hits frequencies reached T votes       */
   CUSFFT_INVALID_PLAN = -10,  /* NULL or destroyed plan                               */
-  CUSFFT_INTERNAL = -11       /* a device-side consistency check failed               */
+  CUSFFT_INTERNAL = -11,      /* a device-side consistency check failed               */
+  CUSFFT_NCCL = -12           /* NCCL not loadable, or an NCCL call failed (cusfft_last_nccl_error) */
 } cusfft_status_t;
 
 typedef enum {
@@ -72,7 +73,27 @@ typedef enum {
   CUSFFT_CUTOFF_THRESHOLD = 2
 } cusfft_cutoff_t;
 
-/* Plan parameters.  Fill with cusfft_params_default, then override. */
+/* Plan parameters.  Fill with cusfft_params_default, then override.
+ *
+ * Filters (DESIGN.md §3 [Z1]): the taps are a Dolph-Chebyshev or Gaussian
+ * window of w taps, w = floor(acosh(1/delta) / (pi lambda)) (Dolph-Chebyshev)
+ * or floor(2 ln(1/delta) / (pi lambda)) (Gaussian), forced odd, times a
+ * box of width b, normalised to sum 1 ("nearly flat inside the pass region",
+ * L85).  The location loops r < L_loc may use their own (delta, lambda)
+ * (loc_tolerance, loc_lobefrac; the paper's location loops, L93,
+ * against the loops the estimation runs over, L232 / Alg. 5); every loop
+ * still estimates with its own filter's response G^.
+ *
+ * Persisting L2 (l2_persist = 1, the default): a plan whose fold is staged
+ * (cusfft_get_info info[11] = 1) raises the DEVICE-WIDE limit
+ * cudaLimitPersistingL2CacheSize to its staging buffer size (at most the
+ * device maximum, 82 MB on B200) while it lives; its staging stores are
+ * evict_last (persisting) so they survive the x stream.  That set-aside is
+ * taken from the L2 every kernel of the process sees (dense cuFFT of n = 2^24
+ * slows from 292 to 340 us while a C3 plan lives).  Plans share one
+ * reference-counted raise per device; the last one destroyed restores the
+ * value found before the first.  l2_persist = 0 leaves the limit alone (the
+ * staging then competes with x for the normal L2: C3 ~13 us slower). */
 typedef struct {
   int32_t filter;          /* cusfft_filter_t; default DOLPH_CHEBYSHEV (L85)                     */
   double tolerance;        /* delta: filter side-lobe / leakage level; default 1e-8              */
@@ -85,14 +106,21 @@ typedef struct {
   uint64_t seed;           /* drives (a_r, sigma_r, tau_r) through SplitMix64      */
   int64_t max_hits;        /* hit-buffer capacity; default from the expected false-hit count      */
   int32_t device;          /* CUDA device ordinal; default: the current device                   */
-  int32_t debug;           /* 1: keep per-loop estimates for cusfft_get_debug; default 0          */
-  const double* taps;      /* optional HOST array of num_taps real taps g_i (Alg. 1 filter[]);
-                              NULL: build the filter from filter/tolerance/lobefrac/box_width.
-                              Copied at plan time; the caller keeps ownership.                    */
+  int32_t debug;           /* 1: keep u and per-loop estimates for cusfft_get_debug; default 0   */
+  const double* taps;      /* optional HOST array of num_taps real taps g_i (Alg. 1 filter[]) used
+                              by every loop; NULL: build the filters from filter / tolerance /
+                              lobefrac / box_width (and loc_*).  Copied at plan time; the caller
+                              keeps ownership.                                                    */
   int64_t num_taps;        /* length of taps when taps != NULL (odd not required)                */
   int32_t cutoff_mode;     /* cusfft_cutoff_t; default EXACT                                      */
   int32_t shard_mode;      /* cusfft_plan_dist only: 0 = loops (default), 1 = signal range       */
   double cutoff_threshold; /* THRESHOLD mode: absolute |u^|^2 threshold (> 0)                    */
+  double loc_tolerance;    /* delta of the location loops' filter; 0 (default): tolerance        */
+  double loc_lobefrac;     /* lambda of the location loops' filter; 0 (default): lobefrac        */
+  int32_t l2_persist;      /* 1 (default): staged plans raise the device's persisting-L2 set-aside
+                              while they live (see above); 0: never touch the device limit       */
+  int32_t gather;          /* 0 (default): address-sorted staged gather when its staging buffer fits
+                              L2, else direct; 1: always the direct gather       */
 } cusfft_params;
 
 /* Fill *p with the defaults for (n, k, B).  Returns CUSFFT_NULL_PTR / INVALID_*. */
@@ -112,17 +140,31 @@ int cusfft_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L,
 /* Multi-GPU plan for rank `rank` of `world` processes (one GPU each).
  * shard_mode 0 (loops): world must divide L; loop r is owned by rank r mod
  * world, every rank passes the whole signal; outputs are identical on every
- * rank and bit-identical to a world = 1 plan.  The exchange between
- * cusfft_execute_local and cusfft_execute_finish is an ALL-GATHER of the
- * buffer returned by cusfft_exchange_buffer (rank-major slices).
+ * rank and bit-identical to a world = 1 plan.  The exchange is an ALL-GATHER
+ * of the buffer returned by cusfft_exchange_buffer (rank-major slices).
  * shard_mode 1 (signal): world must divide n; rank g passes only
- * its slice x[g n/world, (g+1) n/world) to cusfft_execute_local and folds
- * the samples it owns for all L loops; the exchange is a SUM ALL-REDUCE (fp64)
- * of the whole buffer (the B-point FFT is linear, so partial bucket spectra
- * add); every rank then runs Steps 4-6.  Equal to world = 1 within fp64
- * rounding (the sum order differs).  See cusfft_exchange_kind. */
+ * its slice x[g n/world, (g+1) n/world) and folds the samples it owns for all
+ * L loops; the exchange is a SUM ALL-REDUCE (fp64) of the whole buffer (the
+ * B-point FFT is linear, so partial bucket spectra add); every rank then runs
+ * Steps 4-6.  Equal to world = 1 within fp64 rounding (the sum order differs).
+ *
+ * nccl_unique_id: NULL, or 128 bytes from cusfft_nccl_unique_id on one rank,
+ * distributed to every rank by the caller (any channel).  With an id the plan
+ * owns an NCCL communicator (ncclCommInitRank over the `world` ranks; this
+ * call then blocks until every rank has called it) and cusfft_execute runs the
+ * whole transform including the collective, stream-ordered and captured in
+ * the plan's CUDA graph.  NCCL is loaded at run time (libnccl.so.2: the one
+ * already in the process, e.g. PyTorch's, else the system's); CUSFFT_NCCL if
+ * it cannot be loaded or initialised.  Without an id the caller runs the
+ * exchange between cusfft_execute_local and cusfft_execute_finish
+ * (cusfft_exchange_kind) and cusfft_execute returns CUSFFT_INVALID_LOOPS for
+ * world > 1. */
 int cusfft_plan_dist(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L,
-                     const cusfft_params* p, int32_t rank, int32_t world);
+                     const cusfft_params* p, int32_t rank, int32_t world, const void* nccl_unique_id);
+
+/* Write a fresh 128-byte ncclUniqueId to out (ncclGetUniqueId).  CUSFFT_NCCL
+ * when NCCL cannot be loaded. */
+int cusfft_nccl_unique_id(void* out);
 
 /* Release every device allocation of the plan.  Synchronises the plan's stream.
  * Destroying NULL returns CUSFFT_INVALID_PLAN. */
@@ -131,7 +173,7 @@ int cusfft_destroy(cusfft_plan_t plan);
 /* Set the CUDA stream (a cudaStream_t; NULL = legacy default stream). */
 int cusfft_set_stream(cusfft_plan_t plan, void* cuda_stream);
 
-/* The whole transform on one GPU (world = 1 plans only):
+/* The whole transform (world = 1 plans, or multi-GPU plans that own a communicator):
  *   d_x    : device, read-only, complex fp64 [n]
  *   d_locs : device, int64 [k]      output: recovered frequencies, ascending; -1 pads
  *   d_vals : device, complex fp64 [k] output: x^_f / n at d_locs; 0 pads
@@ -180,9 +222,12 @@ int cusfft_exchange_buffer(cusfft_plan_t plan, void** d_buf, int64_t* bytes_per_
 int32_t cusfft_exchange_kind(cusfft_plan_t plan);
 
 /* Plan facts (host arrays, caller-owned):
- *   info[0..11] = n, k, B, L, w (taps), n/B, num_select, loc_loops, vote_threshold, max_hits,
- *                 distinct 32-B sectors of x this rank's gathers touch (the fold's DRAM floor),
- *                 staged (1: address-sorted two-phase gather)
+ *   info[0..15] = n, k, B, L, w (taps of the estimation filter), n/B, num_select, loc_loops,
+ *                 vote_threshold, max_hits, distinct 32-B sectors of x this rank's gathers
+ *                 touch (the fold's DRAM floor), staged (1: address-sorted two-phase gather,
+ *                 DESIGN.md §6.2), w of the location filter, number of filters (1 or 2),
+ *                 fused tail (1: vote + estimation + output in one kernel), owns an NCCL
+ *                 communicator (1)
  *   a, sigma, tau : int64 [L], in loop order r = 0..L-1 (NULL to skip).  sigma is
  *   the gather stride (Alg. 1's ai), a = sigma^-1 mod n, tau the offset. */
 int cusfft_get_info(cusfft_plan_t plan, int64_t* info, int64_t* a, int64_t* sigma, int64_t* tau);
@@ -197,9 +242,11 @@ typedef enum {
   CUSFFT_DEBUG_HITS = 3,     /* int32 [H]: frequencies with >= T votes (unordered)           */
   CUSFFT_DEBUG_HIT_VALS = 4, /* complex fp64 [H]: median estimates aligned with HITS          */
   CUSFFT_DEBUG_PER_LOOP = 5, /* complex fp64 [H][L]: per-loop estimates (params.debug = 1)    */
-  CUSFFT_DEBUG_TAPS = 6,     /* fp64 [w]: filter taps g_i                                    */
-  CUSFFT_DEBUG_GHAT = 7,     /* complex fp64 [n/B + 1]: G^(q), q = -n/(2B) .. n/(2B)          */
-  CUSFFT_DEBUG_NUM_HITS = 8  /* int64 [1]: H (may exceed max_hits on overflow)               */
+  CUSFFT_DEBUG_TAPS = 6,     /* fp64 [w]: filter taps g_i (the estimation loops' filter)     */
+  CUSFFT_DEBUG_GHAT = 7,     /* complex fp64 [n/B + 1]: its G^(q), q = -n/(2B) .. n/(2B)      */
+  CUSFFT_DEBUG_NUM_HITS = 8, /* int64 [1]: H (may exceed max_hits on overflow)               */
+  CUSFFT_DEBUG_LOC_TAPS = 9, /* fp64 [w_loc]: the location loops' filter taps (= TAPS with one filter) */
+  CUSFFT_DEBUG_LOC_GHAT = 10 /* complex fp64 [n/B + 1]: its G^                                */
 } cusfft_debug_t;
 
 /* Copy a debug artefact of the last execution to host memory.  cap is the
@@ -211,11 +258,17 @@ int64_t cusfft_get_debug(cusfft_plan_t plan, int32_t what, void* host_dst, int64
  * execution: CUSFFT_SUCCESS, CUSFFT_HIT_OVERFLOW or CUSFFT_INTERNAL. */
 int cusfft_status(cusfft_plan_t plan);
 
-/* Per-stage device times (ms) of the last execution when timing is enabled:
- * ms[0..5] = fold, B-point FFT, cutoff, vote, estimate, output; with cap >= 7,
+/* Timing (enable): 0 off; 1 direct launches (no graph) with CUDA events
+ * between the stages; 2 the normal CUDA graph with event-record nodes before
+ * and after phase 1 and at the end (times the gather inside the graph that is
+ * otherwise executed).
+ * Per-stage device times (ms) of the last execution when timing is enabled:
+ * ms[0..5] = fold, B-point FFT, cutoff, vote, estimate, output (with the fused
+ * tail, info[14] = 1, the vote entry holds vote + estimate + output and the
+ * next two are 0); with cap >= 7,
  * ms[6] = phase 1 of the staged fold alone (the address-ordered permute
- * gather k_stage*), -1 when the plan is not staged.  Enabling
- * records CUDA events between the kernels on the plan's stream.  get syncs. */
+ * gather k_stage*), -1 when the plan is not staged.  In mode 2
+ * ms[0] is the whole graph and ms[1..5] are -1.  get syncs. */
 int cusfft_set_timing(cusfft_plan_t plan, int32_t enable);
 int cusfft_get_stage_times(cusfft_plan_t plan, float* ms, int32_t cap);
 
@@ -229,6 +282,7 @@ int32_t cusfft_launches_per_execute(cusfft_plan_t plan);
 
 const char* cusfft_strerror(int code);
 int32_t cusfft_last_cuda_error(void);
+int32_t cusfft_last_nccl_error(void);
 int32_t cusfft_abi_version(void);
 
 #ifdef __cplusplus

@@ -9,8 +9,8 @@ fallback.
 """
 from ._binding import (  # noqa: F401
     DEBUG_GHAT, DEBUG_HIT_VALS, DEBUG_HITS, DEBUG_NUM_HITS, DEBUG_PER_LOOP, DEBUG_TAPS,
-    DEBUG_U, DEBUG_UHAT, DEBUG_WINNERS, FILTER_DOLPH_CHEBYSHEV, FILTER_GAUSSIAN,
-    CusfftError, CusfftParams, Plan, default_B, default_params, load_library,
+    DEBUG_LOC_GHAT, DEBUG_LOC_TAPS, DEBUG_U, DEBUG_UHAT, DEBUG_WINNERS, FILTER_DOLPH_CHEBYSHEV, FILTER_GAUSSIAN,
+    CusfftError, CusfftParams, Plan, default_B, default_params, load_library, nccl_unique_id,
 )
 
-__all__ = ["Plan", "default_B", "default_params", "load_library", "CusfftError", "CusfftParams"]
+__all__ = ["Plan", "default_B", "default_params", "load_library", "nccl_unique_id", "CusfftError", "CusfftParams"]

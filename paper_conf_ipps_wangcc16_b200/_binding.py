@@ -17,7 +17,7 @@ LIB_PATH = os.path.join(_HERE, os.environ.get("CUSFFT_LIB", "libcusfft.so"))
 
 SUCCESS = 0
 INVALID_N, INVALID_B, INVALID_K, INVALID_LOOPS, INVALID_PARAM = -1, -2, -3, -4, -5
-NULL_PTR, ALLOC, CUDA, HIT_OVERFLOW, INVALID_PLAN, INTERNAL = -6, -7, -8, -9, -10, -11
+NULL_PTR, ALLOC, CUDA, HIT_OVERFLOW, INVALID_PLAN, INTERNAL, NCCL = -6, -7, -8, -9, -10, -11, -12
 
 FILTER_DOLPH_CHEBYSHEV = 0
 FILTER_GAUSSIAN = 1
@@ -26,16 +26,17 @@ CUTOFF_EXACT, CUTOFF_SORT, CUTOFF_THRESHOLD = 0, 1, 2
 
 DEBUG_U, DEBUG_UHAT, DEBUG_WINNERS, DEBUG_HITS, DEBUG_HIT_VALS = 0, 1, 2, 3, 4
 DEBUG_PER_LOOP, DEBUG_TAPS, DEBUG_GHAT, DEBUG_NUM_HITS = 5, 6, 7, 8
+DEBUG_LOC_TAPS, DEBUG_LOC_GHAT = 9, 10
 
 # Every symbol include/cusfft.h declares (checked by tests/test_abi.py).
 EXPORTED = (
-    "cusfft_params_default", "cusfft_default_B", "cusfft_plan", "cusfft_plan_dist",
+    "cusfft_params_default", "cusfft_default_B", "cusfft_plan", "cusfft_plan_dist", "cusfft_nccl_unique_id",
     "cusfft_destroy", "cusfft_set_stream", "cusfft_execute", "cusfft_execute_host", "cusfft_execute_batch",
     "cusfft_set_pipeline",
     "cusfft_execute_local", "cusfft_execute_finish", "cusfft_exchange_buffer", "cusfft_exchange_kind",
     "cusfft_get_info", "cusfft_get_debug", "cusfft_status", "cusfft_set_timing",
     "cusfft_get_stage_times", "cusfft_set_stage_limit", "cusfft_launches_per_execute", "cusfft_strerror",
-    "cusfft_last_cuda_error", "cusfft_abi_version",
+    "cusfft_last_cuda_error", "cusfft_last_nccl_error", "cusfft_abi_version",
 )
 
 
@@ -58,6 +59,10 @@ class CusfftParams(ctypes.Structure):
         ("cutoff_mode", ctypes.c_int32),
         ("shard_mode", ctypes.c_int32),
         ("cutoff_threshold", ctypes.c_double),
+        ("loc_tolerance", ctypes.c_double),
+        ("loc_lobefrac", ctypes.c_double),
+        ("l2_persist", ctypes.c_int32),
+        ("gather", ctypes.c_int32),
     ]
 
 
@@ -81,7 +86,8 @@ def load_library():
         "cusfft_params_default": (ctypes.c_int, [pp, i64, i64, i64]),
         "cusfft_default_B": (i64, [i64, i64, ctypes.c_double]),
         "cusfft_plan": (ctypes.c_int, [ctypes.POINTER(P), i64, i64, i64, i32, pp]),
-        "cusfft_plan_dist": (ctypes.c_int, [ctypes.POINTER(P), i64, i64, i64, i32, pp, i32, i32]),
+        "cusfft_plan_dist": (ctypes.c_int, [ctypes.POINTER(P), i64, i64, i64, i32, pp, i32, i32, P]),
+        "cusfft_nccl_unique_id": (ctypes.c_int, [P]),
         "cusfft_destroy": (ctypes.c_int, [P]),
         "cusfft_set_stream": (ctypes.c_int, [P, P]),
         "cusfft_execute": (ctypes.c_int, [P, P, P, P]),
@@ -101,6 +107,7 @@ def load_library():
         "cusfft_launches_per_execute": (i32, [P]),
         "cusfft_strerror": (ctypes.c_char_p, [ctypes.c_int]),
         "cusfft_last_cuda_error": (i32, []),
+        "cusfft_last_nccl_error": (i32, []),
         "cusfft_abi_version": (i32, []),
     }
     for name, (res, args) in sig.items():
@@ -117,6 +124,8 @@ class CusfftError(RuntimeError):
         msg = lib.cusfft_strerror(code).decode()
         if code == CUDA:
             msg += f" (cudaError {lib.cusfft_last_cuda_error()})"
+        if code == NCCL:
+            msg += f" (ncclResult {lib.cusfft_last_nccl_error()})"
         super().__init__(f"{what}: {msg} [{code}]" if what else f"{msg} [{code}]")
         self.code = code
 
@@ -137,6 +146,13 @@ def default_params(n: int, k: int, B: int) -> CusfftParams:
     return p
 
 
+def nccl_unique_id() -> bytes:
+    """128 bytes of a fresh ncclUniqueId (cusfft_nccl_unique_id) for cusfft_plan_dist."""
+    buf = ctypes.create_string_buffer(128)
+    check(load_library().cusfft_nccl_unique_id(buf), "cusfft_nccl_unique_id")
+    return buf.raw
+
+
 def _ptr(t) -> int:
     """Raw data pointer of a torch tensor or numpy array."""
     if hasattr(t, "data_ptr"):
@@ -149,12 +165,15 @@ class Plan:
 
     ``params`` are the fields of ``cusfft_params`` (filter, tolerance,
     lobefrac, box_width, loc_loops, vote_threshold, num_select, tau_mode,
-    seed, max_hits, device, debug) plus ``taps`` (a float64 array of user
-    taps).  ``rank`` / ``world`` make a loop-sharded plan (cusfft_plan_dist).
+    seed, max_hits, device, debug, cutoff_mode, shard_mode, cutoff_threshold,
+    loc_tolerance, loc_lobefrac, l2_persist, gather) plus ``taps`` (a float64
+    array of user taps).  ``rank`` / ``world`` make a multi-GPU plan
+    (cusfft_plan_dist); ``nccl_id`` (128 bytes from ``nccl_unique_id()`` on
+    one rank, shared by the caller) lets the plan own the exchange.
     """
 
     def __init__(self, n: int, k: int, B: int | None = None, L: int = 16, rank: int = 0,
-                 world: int = 1, **params):
+                 world: int = 1, nccl_id: bytes | None = None, **params):
         self._lib = load_library()
         self._h = ctypes.c_void_p()
         if B is None:
@@ -172,11 +191,17 @@ class Plan:
             prm.taps = self._taps.ctypes.data_as(ctypes.POINTER(ctypes.c_double))
             prm.num_taps = self._taps.shape[0]
         self.params = prm
-        if self.world == 1:
+        if self.world == 1 and nccl_id is None:
             rc = self._lib.cusfft_plan(ctypes.byref(self._h), self.n, self.k, self.B, self.L, ctypes.byref(prm))
         else:
+            uid = None
+            if nccl_id is not None:
+                if len(nccl_id) != 128:
+                    raise ValueError("nccl_id must be 128 bytes")
+                self._uid = ctypes.create_string_buffer(bytes(nccl_id), 128)
+                uid = ctypes.cast(self._uid, ctypes.c_void_p)
             rc = self._lib.cusfft_plan_dist(ctypes.byref(self._h), self.n, self.k, self.B, self.L,
-                                            ctypes.byref(prm), self.rank, self.world)
+                                            ctypes.byref(prm), self.rank, self.world, uid)
         check(rc, "cusfft_plan")
         info = self.info()
         self.w, self.nb, self.num, self.loc_loops, self.T, self.max_hits = (
@@ -298,14 +323,15 @@ class Plan:
 
     # -- introspection
     def info(self):
-        info = np.zeros(12, dtype=np.int64)
+        info = np.zeros(16, dtype=np.int64)
         a = np.zeros(self.L, dtype=np.int64)
         s = np.zeros(self.L, dtype=np.int64)
         t = np.zeros(self.L, dtype=np.int64)
         check(self._lib.cusfft_get_info(self._h, ctypes.c_void_p(info.ctypes.data), ctypes.c_void_p(a.ctypes.data),
                                         ctypes.c_void_p(s.ctypes.data), ctypes.c_void_p(t.ctypes.data)),
               "cusfft_get_info")
-        keys = ("n", "k", "B", "L", "w", "nb", "num", "loc_loops", "T", "max_hits", "sectors", "staged")
+        keys = ("n", "k", "B", "L", "w", "nb", "num", "loc_loops", "T", "max_hits", "sectors", "staged",
+                "w_loc", "filters", "tail", "owns_comm")
         d = dict(zip(keys, info.tolist()))
         d.update(a=a, sigma=s, tau=t)
         return d
@@ -313,7 +339,8 @@ class Plan:
     def debug(self, what: int):
         dtype = {DEBUG_U: np.complex128, DEBUG_UHAT: np.complex128, DEBUG_WINNERS: np.int32,
                  DEBUG_HITS: np.int32, DEBUG_HIT_VALS: np.complex128, DEBUG_PER_LOOP: np.complex128,
-                 DEBUG_TAPS: np.float64, DEBUG_GHAT: np.complex128, DEBUG_NUM_HITS: np.int64}[what]
+                 DEBUG_TAPS: np.float64, DEBUG_GHAT: np.complex128, DEBUG_NUM_HITS: np.int64,
+                 DEBUG_LOC_TAPS: np.float64, DEBUG_LOC_GHAT: np.complex128}[what]
         need = int(self._lib.cusfft_get_debug(self._h, what, None, 0))
         if need < 0:
             check(need, "cusfft_get_debug")
@@ -332,12 +359,14 @@ class Plan:
             buf = buf.reshape(-1, self.L)
         return buf
 
-    def set_timing(self, enable: bool = True):
-        check(self._lib.cusfft_set_timing(self._h, 1 if enable else 0), "cusfft_set_timing")
+    def set_timing(self, mode: int = 1):
+        """0 off; 1 direct launches with stage events; 2 events around phase 1 inside the CUDA graph."""
+        check(self._lib.cusfft_set_timing(self._h, int(mode)), "cusfft_set_timing")
 
     def stage_times(self):
         """Stage times (ms) of the last timed execution; 'gather' is phase 1 of
-        the staged fold alone (-1 when the plan is not staged)."""
+        the staged fold alone (-1 when the plan is not staged).  With the fused
+        tail (info()['tail'] == 1) 'vote' covers vote + estimate + output."""
         ms = (ctypes.c_float * 7)()
         check(self._lib.cusfft_get_stage_times(self._h, ms, 7), "cusfft_get_stage_times")
         return dict(zip(("fold", "fft", "cutoff", "vote", "estimate", "output", "gather"), list(ms)))

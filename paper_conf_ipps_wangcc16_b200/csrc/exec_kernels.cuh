@@ -95,10 +95,11 @@ __global__ void __launch_bounds__(256) k_fold(const double2* __restrict__ x, con
 
 // ---------------------------------------------------------------------------
 // Staged gather, phase 1: the plan sorted every (slot, tap)
-// gather position of this rank; staging[q] = x[spos[q]] in that address order,
-// so DRAM rows are opened once for all loops' samples that share them (the
-// random-order gather is bound by row activations).  x is read evict-first
-// with 64-B L2 fetches; staging (L2-sized) is written evict-last for phase 2.
+// gather of this rank by address; the kernel walks them in that order, so
+// DRAM rows are opened once for all loops' samples that share them (the
+// random-order gather is bound by row activations), and stores each sample
+// where phase 2 reads it (scatter).  x is read evict-first with 64-B L2
+// fetches; the staging buffer (L2-sized) is written evict-last for phase 2.
 // Also zeroes the per-execution block (first kernel of the execution).
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ uint64_t l2_policy_first() {
@@ -112,75 +113,34 @@ __device__ __forceinline__ uint64_t l2_policy_last() {
   return p;
 }
 
-// dst (optional): staging position of sorted gather q in the fused kernel's
-// thread order (scatter staging: phase 2 then reads coalesced, no index);
-// null: staging[q] in sorted order (phase 2 reads it through inv_perm).
-__global__ void __launch_bounds__(256) k_stage(const double2* __restrict__ x, const uint32_t* __restrict__ spos,
-                                               const uint32_t* __restrict__ dst, double2* __restrict__ staging,
-                                               int total, ZeroArgs zero) {
-  pdl_wait();
-  KTRACE(1);
-  if (blockIdx.x == 0) TRACE(0);
-  zero_part(zero);
-  const uint64_t pf = l2_policy_first(), pl = l2_policy_last();
-  const int T = gridDim.x * blockDim.x;
-  for (int q0 = blockIdx.x * blockDim.x + threadIdx.x; q0 < total; q0 += 8 * T) {
-    double2 v[8];
-#pragma unroll
-    for (int c = 0; c < 8; ++c) {
-      const int q = q0 + c * T;
-      if (q < total) {
-        const double2* p = x + __ldg(spos + q);
-        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.L2::64B.v2.f64 {%0, %1}, [%2], %3;"
-                     : "=d"(v[c].x), "=d"(v[c].y) : "l"(p), "l"(pf));
-      }
-    }
-#pragma unroll
-    for (int c = 0; c < 8; ++c) {
-      const int q = q0 + c * T;
-      if (q < total) {
-        double2* o = staging + (dst ? __ldg(dst + q) : (uint32_t)q);
-        asm volatile("st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %3;" ::"l"(o), "d"(v[c].x), "d"(v[c].y),
-                     "l"(pl));
-      }
-    }
-  }
-  TRACE_END(6);
-}
-
-// Packed form of the scatter staging (default): the schedule holds one word
-// per gather, (local slot << ibits) | tap index i, in address order; the
-// position sigma_s i + tau_s and phase 2's thread-order destination
-//   (s R + rr) B + tile 256 + (c mod C) B1 + j1,  i = rr B + j, j = c + B2 j1,
-// are recomputed here (shifts and masks), halving the schedule bytes.
+// The schedule holds one word per gather, (local slot << ibits) | tap index
+// i, in address order; the position sigma_s i + tau_s and phase 2's
+// thread-order destination
+//   (row0_s + rr) B + tile 256 + (c mod C) B1 + j1,  i = rr B + j, j = c + B2 j1,
+// are recomputed here (shifts and masks; row0_s = first staging row of slot
+// s, slots of a filter group have R_g rows each).
 struct StagePackArgs {
   const double2* x;
   const uint32_t* code;
   double2* staging;
-  const SlotParam* slots;  // group slot 0
-  int total, nslots, ibits, R, logB, logB2, logB1, logC;
+  const SlotParam* slots;  // local slot 0
+  const uint32_t* row0;    // [nslots] first staging row of each local slot
+  int total, nslots, ibits, logB, logB2, logB1, logC;
   uint32_t nmask;
   ZeroArgs zero;
-  int code_ef;  // schedule words read with the evict_first policy too
 };
 
-__device__ __forceinline__ uint32_t ld_u32_ef(const uint32_t* p, uint64_t pol) {
-  uint32_t v;
-  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
-  return v;
-}
-
-// U: gathers in flight per thread (CUSFFT_STAGE_U = 2 / 4 / 8 / 16; 4 by default).
+// U: gathers in flight per thread (4: 4096 per SM at 4 CTAs of 256).
 template <int U>
 __global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
-  pdl_trigger(0);
   pdl_wait();
   KTRACE(1);
   if (blockIdx.x == 0) TRACE(0);
-  __shared__ uint32_t ssig[kMaxLoops], stau[kMaxLoops];
+  __shared__ uint32_t ssig[kMaxLoops], stau[kMaxLoops], srow[kMaxLoops];
   for (int i = threadIdx.x; i < A.nslots; i += blockDim.x) {
     ssig[i] = A.slots[i].sigma;
     stau[i] = A.slots[i].tau;
+    srow[i] = A.row0[i];
   }
   zero_part(A.zero);
   __syncthreads();
@@ -195,7 +155,7 @@ __global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
     for (int c = 0; c < U; ++c) {
       const int q = q0 + c * T;
       if (q < A.total) {
-        cd[c] = A.code_ef ? ld_u32_ef(A.code + q, pf) : __ldg(A.code + q);
+        cd[c] = __ldg(A.code + q);
         const uint32_t sl = cd[c] >> A.ibits, i = cd[c] & imask;
         const double2* p = A.x + ((ssig[sl] * i + stau[sl]) & A.nmask);
         asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.L2::64B.v2.f64 {%0, %1}, [%2], %3;"
@@ -209,111 +169,13 @@ __global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
         const uint32_t sl = cd[c] >> A.ibits, i = cd[c] & imask;
         const uint32_t rr = i >> A.logB, j = i & Bm;
         const uint32_t col = j & B2m, j1 = j >> A.logB2;
-        const uint32_t dst = ((sl * (uint32_t)A.R + rr) << A.logB) + ((col >> A.logC) << 8) +
-                             ((col & Cm) << A.logB1) + j1;
+        const uint32_t dst = ((srow[sl] + rr) << A.logB) + ((col >> A.logC) << 8) + ((col & Cm) << A.logB1) + j1;
         asm volatile("st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %3;" ::"l"(A.staging + dst), "d"(v[c].x),
                      "d"(v[c].y), "l"(pl));
       }
     }
   }
   TRACE_END(6);
-}
-
-// Atomic form of phase 1 (opt-in, CUSFFT_STAGE_MODE=atomic): the same
-// address-ordered gathers, each multiplied by its tap g_i and added straight
-// into u_s[i mod B] with fp64 L2 reductions (u zeroed by a memset node), so
-// there is no staging round trip; the FFT pass 1 then reads u.  The order of
-// the additions into a bucket is whatever order the L2 sees them in, so u is
-// reproducible only to rounding (not bit-exact with Alg. 1's order).
-__global__ void __launch_bounds__(256) k_stage_atomic(StagePackArgs A, const double* __restrict__ taps,
-                                                      double2* __restrict__ u) {
-  pdl_wait();
-  KTRACE(1);
-  if (blockIdx.x == 0) TRACE(0);
-  __shared__ uint32_t ssig[kMaxLoops], stau[kMaxLoops];
-  for (int i = threadIdx.x; i < A.nslots; i += blockDim.x) {
-    ssig[i] = A.slots[i].sigma;
-    stau[i] = A.slots[i].tau;
-  }
-  zero_part(A.zero);
-  __syncthreads();
-  const uint64_t pf = l2_policy_first();
-  const uint32_t imask = (1u << A.ibits) - 1u;
-  const uint32_t Bm = (1u << A.logB) - 1u;
-  const int T = gridDim.x * blockDim.x;
-  for (int q0 = blockIdx.x * blockDim.x + threadIdx.x; q0 < A.total; q0 += 8 * T) {
-    double2 v[8];
-    uint32_t cd[8];
-#pragma unroll
-    for (int c = 0; c < 8; ++c) {
-      const int q = q0 + c * T;
-      if (q < A.total) {
-        cd[c] = __ldg(A.code + q);
-        const uint32_t sl = cd[c] >> A.ibits, i = cd[c] & imask;
-        const double2* p = A.x + ((ssig[sl] * i + stau[sl]) & A.nmask);
-        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.L2::64B.v2.f64 {%0, %1}, [%2], %3;"
-                     : "=d"(v[c].x), "=d"(v[c].y) : "l"(p), "l"(pf));
-      }
-    }
-#pragma unroll
-    for (int c = 0; c < 8; ++c) {
-      const int q = q0 + c * T;
-      if (q < A.total) {
-        const uint32_t sl = cd[c] >> A.ibits, i = cd[c] & imask;
-        const double g = __ldg(taps + i);
-        double* o = reinterpret_cast<double*>(u + ((sl << A.logB) | (i & Bm)));
-        asm volatile("red.relaxed.gpu.global.add.f64 [%0], %1;" ::"l"(o), "d"(__dmul_rn(g, v[c].x)) : "memory");
-        asm volatile("red.relaxed.gpu.global.add.f64 [%0], %1;" ::"l"(o + 1), "d"(__dmul_rn(g, v[c].y)) : "memory");
-      }
-    }
-  }
-  TRACE_END(6);
-}
-
-// ---------------------------------------------------------------------------
-// Staged gather, phase 2 without the FFT (split mode): thread per (slot,
-// bucket j), natural order.  SCATTER: staging[(s R + rr) B + j] holds round
-// rr's sample (coalesced reads); else staging[inv[(s R + rr) B + j]].  Light
-// enough for 4 CTAs per SM; the rounds are accumulated in Alg. 1's order.
-// ---------------------------------------------------------------------------
-template <bool SCATTER>
-__global__ void __launch_bounds__(256, 4) k_fold_staged(const double2* __restrict__ staging,
-                                                        const uint32_t* __restrict__ inv,
-                                                        const double* __restrict__ taps, double2* __restrict__ u,
-                                                        int B, int w, int R, ZeroArgs zero) {
-  pdl_wait();
-  KTRACE(3);
-  if (blockIdx.x == 0 && blockIdx.y == 0) TRACE(0);
-  zero_part(zero);
-  const int j = blockIdx.x * 256 + threadIdx.x;
-  const int s = blockIdx.y;
-  const int64_t base = (int64_t)s * R * B + j;
-  double ar = 0.0, ai = 0.0;
-  constexpr int RC = 8;
-  for (int r0 = 0; r0 < R; r0 += RC) {
-    uint32_t q[RC];
-    double2 xv[RC];
-    if constexpr (!SCATTER) {
-#pragma unroll
-      for (int c = 0; c < RC; ++c)
-        if (r0 + c < R && j + (r0 + c) * B < w) q[c] = __ldcs(inv + base + (int64_t)(r0 + c) * B);
-    }
-#pragma unroll
-    for (int c = 0; c < RC; ++c)
-      if (r0 + c < R && j + (r0 + c) * B < w)
-        xv[c] = __ldcs(staging + (SCATTER ? base + (int64_t)(r0 + c) * B : (int64_t)q[c]));
-#pragma unroll
-    for (int c = 0; c < RC; ++c) {
-      const int i = j + (r0 + c) * B;
-      if (r0 + c < R && i < w) {
-        const double g = __ldg(taps + i);
-        ar = __dadd_rn(ar, __dmul_rn(g, xv[c].x));
-        ai = __dadd_rn(ai, __dmul_rn(g, xv[c].y));
-      }
-    }
-  }
-  u[(int64_t)s * B + j] = make_double2(ar, ai);
-  TRACE_END(1);
 }
 
 // ---------------------------------------------------------------------------
@@ -327,17 +189,15 @@ __global__ void __launch_bounds__(256, 4) k_fold_staged(const double2* __restric
 // loads of a CTA stay contiguous.  RC gathers per thread in flight; two CTAs
 // per SM so one CTA's FFT epilogue overlaps the other's gathers.
 // ---------------------------------------------------------------------------
-// MODE 0: direct gather from x; 1: staged, read through inv_perm; 2: staged in
-// this kernel's thread order (scatter staging), read coalesced.
-template <int B1T, int RC, int MODE>
+// Direct gather from x (plans whose staging buffer would not fit L2).
+template <int B1T, int RC>
 __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict__ x,
-                                                                   const uint32_t* __restrict__ inv_perm,
-                                                                   const double* __restrict__ taps_perm,
-                                                                   const SlotParam* __restrict__ slots,
-                                                                   double2* __restrict__ u, double2* __restrict__ v,
-                                                                   const double2* __restrict__ tw, int B, int B2,
-                                                                   int w, int R, uint32_t nmask, uint32_t xlo,
-                                                                   uint32_t xspan, ZeroArgs zero) {
+                                                      const double* __restrict__ taps_perm,
+                                                      const SlotParam* __restrict__ slots,
+                                                      double2* __restrict__ u, double2* __restrict__ v,
+                                                      const double2* __restrict__ tw, int B, int B2,
+                                                      int w, int R, uint32_t nmask, uint32_t xlo,
+                                                      uint32_t xspan, ZeroArgs zero) {
   pdl_wait();
   KTRACE(2);
   constexpr int C = 256 / B1T;
@@ -353,65 +213,7 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict_
   for (int i = t; i < B1T; i += 256) twl[i] = __ldg(tw + (int64_t)i * B2);  // omega_B1^i
   const double* tp = taps_perm + (int64_t)blockIdx.x * 256 + t;
   double ar = 0.0, ai = 0.0;
-  if constexpr (MODE == 2) {
-    // phase 2, scatter staging: staging[(s R + rr) B + cta 256 + t] is this
-    // thread's round-rr sample; all rounds in flight, coalesced L2 reads.
-    constexpr int RMAX = 16;
-    const double2* sp2 = x + (int64_t)s * R * B + (int64_t)blockIdx.x * 256 + t;
-    double2 xv[RMAX];
-#pragma unroll
-    for (int rr = 0; rr < RMAX; ++rr)
-      if (rr < R && j + rr * B < w) xv[rr] = __ldcs(sp2 + (int64_t)rr * B);
-#pragma unroll
-    for (int rr = 0; rr < RMAX; ++rr) {
-      if (rr < R && j + rr * B < w) {
-        const double g = __ldg(tp + (int64_t)rr * B);
-        ar = __dadd_rn(ar, __dmul_rn(g, xv[rr].x));
-        ai = __dadd_rn(ai, __dmul_rn(g, xv[rr].y));
-      }
-    }
-    for (int rr = RMAX; rr < R; ++rr) {  // R > 16 (small tolerance / Gaussian filters)
-      if (j + rr * B < w) {
-        const double2 v2 = __ldcs(sp2 + (int64_t)rr * B);
-        const double g = __ldg(tp + (int64_t)rr * B);
-        ar = __dadd_rn(ar, __dmul_rn(g, v2.x));
-        ai = __dadd_rn(ai, __dmul_rn(g, v2.y));
-      }
-    }
-  } else if constexpr (MODE == 1) {
-    // phase 2: every round's staging index first (one dependent step), then
-    // the L2-resident samples in chunks of RC, accumulated in round order.
-    constexpr int RMAX = 16;
-    const uint32_t* ip = inv_perm + (int64_t)s * R * B + (int64_t)blockIdx.x * 256 + t;
-    uint32_t q[RMAX];
-#pragma unroll
-    for (int rr = 0; rr < RMAX; ++rr) q[rr] = (rr < R && j + rr * B < w) ? __ldg(ip + (int64_t)rr * B) : 0xFFFFFFFFu;
-#pragma unroll
-    for (int r0 = 0; r0 < RMAX; r0 += RC) {
-      double2 xv[RC];
-#pragma unroll
-      for (int cc = 0; cc < RC; ++cc)
-        if (q[r0 + cc] != 0xFFFFFFFFu) xv[cc] = __ldcg(x + q[r0 + cc]);
-#pragma unroll
-      for (int cc = 0; cc < RC; ++cc) {
-        if (q[r0 + cc] != 0xFFFFFFFFu) {
-          const double g = __ldg(tp + (int64_t)(r0 + cc) * B);
-          ar = __dadd_rn(ar, __dmul_rn(g, xv[cc].x));
-          ai = __dadd_rn(ai, __dmul_rn(g, xv[cc].y));
-        }
-      }
-    }
-    for (int rr = RMAX; rr < R; ++rr) {  // R > 16 (small tolerance / Gaussian filters)
-      const int i = j + rr * B;
-      if (i < w) {
-        const double2 xv = __ldcg(x + __ldg(inv_perm + (int64_t)s * R * B + (int64_t)rr * B +
-                                            (int64_t)blockIdx.x * 256 + t));
-        const double g = __ldg(tp + (int64_t)rr * B);
-        ar = __dadd_rn(ar, __dmul_rn(g, xv.x));
-        ai = __dadd_rn(ai, __dmul_rn(g, xv.y));
-      }
-    }
-  } else {
+  {
     const uint32_t sigma = slots[s].sigma, tau = slots[s].tau;
     for (int r0 = 0; r0 < R; r0 += RC) {
       double2 xv[RC];
@@ -459,17 +261,16 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict_
 // their taps, so no gathered sample occupies a register and four CTAs fit per
 // SM.  Then exactly k_fold_fft1's arithmetic: rounds accumulated in Alg. 1's
 // order (fp64 mul + add per component), u written, the C columns' B1-point
-// FFTs in shared memory, v = FFT x omega_B^(c k1).  discard != 0: the consumed
-// staging lines are dropped from L2 without write-back (the next execution
-// rewrites every staged sample that is read).
+// FFTs in shared memory, v = FFT x omega_B^(c k1).  The consumed staging
+// lines stay in L2 (the persisting set-aside): the next execution's phase-1
+// stores then hit valid lines.
 // ---------------------------------------------------------------------------
 template <int B1T>
 __global__ void __launch_bounds__(256, 4) k_fold_fft1_tma(const double2* __restrict__ staging,
                                                           const double* __restrict__ taps_perm,
                                                           double2* __restrict__ u, double2* __restrict__ v,
                                                           const double2* __restrict__ tw, int B, int B2, int w, int R,
-                                                          int discard, ZeroArgs zero) {
-  pdl_trigger(1);
+                                                          ZeroArgs zero) {
   pdl_wait();
   KTRACE(2);
   constexpr int C = 256 / B1T;
@@ -518,8 +319,6 @@ __global__ void __launch_bounds__(256, 4) k_fold_fft1_tma(const double2* __restr
       ai = __dadd_rn(ai, __dmul_rn(gg, q.y));
     }
   }
-  if (discard)
-    for (int q = t; q < R * 32; q += 256) l2_discard(src + (int64_t)(q >> 5) * B + (q & 31) * 8);
   S[fft_pad(cl * B1T + j1)] = make_double2(ar, ai);
   __syncthreads();
   const int wc = t % C, wj = t / C;
@@ -690,22 +489,18 @@ constexpr int kMaxSel = 32;  // location loops per plan (kMaxLoc)
 struct SelArgs {
   uint8_t* recs[kMaxSel];  // record of each location slot of this rank (by value)
   RecLayout lay;
-  int B, num, S;
+  int B, num;
   int threshold_mode;  // Alg. 6: keep every key >= thr_key, no selection
   uint64_t thr_key;    // bits of the |u^|^2 threshold
   const uint64_t* keys;  // [n_sel][B]
   uint32_t* hist0;       // [n_sel][4096] (FFT epilogue)
-  uint32_t* hist1;       // [n_sel][4096]
-  uint64_t* ckey;        // [n_sel][kSelCap]
-  int* cidx;             // [n_sel][kSelCap]
-  int* ccount;           // [n_sel]
-  int* done;             // [n_sel]
   int* status;
   // optional (single-rank plans with every location loop selected here): the
-  // vote's byte-per-bucket array (bit q = bucket kept in location loop q,
-  // selection index == vote index), ORed in by the cutoff; zeroed per execution
+  // vote table of k_tail (element b = bucket b, bit q = kept in location loop
+  // q, selection index == vote index), ORed in by the cluster cutoff; zeroed
+  // per execution
   uint32_t* pk;
-  int local_pick;  // cluster cutoff: each CTA scans the whole level-0 histogram (no pick round trips)
+  int pk_esz;      // bytes per pk element (1 / 2 / 4: L_loc <= 8 / 16 / 32)
 };
 
 struct GKeySrc {
@@ -744,166 +539,6 @@ __global__ void __launch_bounds__(256) k_keys(KeysArgs A) {
   __syncthreads();
   for (int t = threadIdx.x; t < 4096; t += 256)
     if (sh[t]) atomicAdd(&A.hist[(int64_t)i * 4096 + t], sh[t]);
-}
-
-__global__ void __launch_bounds__(kSelNT) k_select(SelArgs A) {
-  pdl_wait();
-  KTRACE(8);
-  extern __shared__ __align__(16) uint8_t smem[];
-  uint32_t* hist = reinterpret_cast<uint32_t*>(smem);
-  int* sm = reinterpret_cast<int*>(smem + 4096 * 4);
-  uint64_t* skey = reinterpret_cast<uint64_t*>(smem + 4096 * 4 + 64 * 4);
-  int* sidx = reinterpret_cast<int*>(skey + kSelCap);
-  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
-  const int sel = blockIdx.x / A.S, part = blockIdx.x - sel * A.S;
-  uint8_t* rec = A.recs[sel];
-  uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap);
-  const uint64_t* keys = A.keys + (int64_t)sel * A.B;
-  uint32_t* h0 = A.hist0 + (int64_t)sel * 4096;
-  uint32_t* h1 = A.hist1 + (int64_t)sel * 4096;
-  const int words = (A.B + 31) >> 5;
-  if (blockIdx.x == 0) TRACE(10);
-  BinPick b0{0, 0, 0};
-  if (!A.threshold_mode) b0 = pick_bin<kSelNT>(h0, A.num, sm);
-  if (blockIdx.x == 0) TRACE(11);
-  const uint32_t d0 = (uint32_t)b0.d;
-  const int k2 = A.num - b0.above;
-  const bool whole = A.threshold_mode || (k2 == b0.cnt);
-  // this CTA's words
-  const int wpc = (words + A.S - 1) / A.S;
-  const int w_begin = part * wpc, w_end = min(words, w_begin + wpc);
-  for (int w0 = w_begin + wid; w0 < w_end; w0 += 8 * (kSelNT / 32)) {
-    uint64_t kb[8];
-#pragma unroll
-    for (int u = 0; u < 8; ++u) {  // 8 words' keys in flight per warp
-      const int w = w0 + u * (kSelNT / 32), i = w * 32 + lane;
-      kb[u] = (w < w_end && i < A.B) ? __ldg(keys + i) : 0ull;
-    }
-#pragma unroll
-    for (int u = 0; u < 8; ++u) {
-      const int w = w0 + u * (kSelNT / 32), i = w * 32 + lane;
-      if (w >= w_end) break;
-      const uint32_t d = (uint32_t)(kb[u] >> 51) & 0xFFFu;
-      const bool take = i < A.B && (A.threshold_mode ? kb[u] >= A.thr_key : (d > d0 || (d == d0 && whole)));
-      const bool cand = i < A.B && !A.threshold_mode && d == d0 && !whole;
-      const uint32_t word = __ballot_sync(kFull, take);
-      if (lane == 0) bitmap[w] = word;
-      if (cand) {
-        const int pos = atomicAdd(A.ccount + sel, 1);
-        if (pos < kSelCap) {
-          A.ckey[(int64_t)sel * kSelCap + pos] = kb[u];
-          A.cidx[(int64_t)sel * kSelCap + pos] = i;
-        }
-        atomicAdd(h1 + digit96(kb[u], ~(uint32_t)i, pass_shift(1)), 1u);
-      }
-    }
-  }
-  if (blockIdx.x == 0) TRACE(12);
-  __threadfence();
-  __syncthreads();
-  if (blockIdx.x == 0) TRACE(13);
-  if (tid == 0) sm[40] = atomicAdd(A.done + sel, 1);
-  __syncthreads();
-  if (blockIdx.x == 0) TRACE(14);
-  if (sm[40] != A.S - 1) return;  // not the last CTA of this loop
-  __threadfence();
-  if (sel == 0) TRACE(20);
-  // ---- finalize (last CTA of the loop)
-  if (!whole) {
-    const int nc = __ldcg(A.ccount + sel);
-    if (nc > kSelNT) {  // level-1 histogram for the radix paths, 16 loads in flight per thread
-      uint32_t hb[4096 / kSelNT];
-#pragma unroll
-      for (int u = 0; u < 4096 / kSelNT; ++u) hb[u] = __ldcg(h1 + tid + u * kSelNT);
-#pragma unroll
-      for (int u = 0; u < 4096 / kSelNT; ++u) hist[tid + u * kSelNT] = hb[u];
-    }
-    Prefix96 p{0, 0, 0, 0};
-    or96(p.phi, p.plo, d0, pass_shift(0));
-    or96(p.mhi, p.mlo, 0xFFFu, pass_shift(0));
-    if (nc <= kSelNT) {  // few candidates: exact rank counting, one pass
-      uint64_t mk = 0;
-      int mi = 0x7FFFFFFF;
-      if (tid < nc) {
-        mk = __ldcg(A.ckey + (int64_t)sel * kSelCap + tid);
-        mi = __ldcg(A.cidx + (int64_t)sel * kSelCap + tid);
-        skey[tid] = mk;
-        sidx[tid] = mi;
-      }
-      __syncthreads();
-      if (tid < nc) {
-        int rank = 0;  // candidates preferred to mine: larger key, or equal key and smaller bucket
-        for (int c = 0; c < nc; ++c) rank += (skey[c] > mk) || (skey[c] == mk && sidx[c] < mi);
-        if (rank < k2) atomicOr(&bitmap[mi >> 5], 1u << (mi & 31));
-      }
-    } else if (nc <= kSelCap) {
-      for (int c0 = 0; c0 < nc; c0 += 4 * kSelNT) {
-        uint64_t kb[4];
-        int ib[4];
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const int c = c0 + u * kSelNT + tid;
-          if (c < nc) {
-            kb[u] = __ldcg(A.ckey + (int64_t)sel * kSelCap + c);
-            ib[u] = __ldcg(A.cidx + (int64_t)sel * kSelCap + c);
-          }
-        }
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const int c = c0 + u * kSelNT + tid;
-          if (c < nc) {
-            skey[c] = kb[u];
-            sidx[c] = ib[u];
-          }
-        }
-      }
-      __syncthreads();
-      p = block_radix_select<PairSrc, kSelNT>(PairSrc{skey, sidx}, nc, k2, hist, sm, 1, p, true);
-      for (int c = tid; c < nc; c += kSelNT)
-        if (ge96(p, skey[c], ~(uint32_t)sidx[c])) atomicOr(&bitmap[sidx[c] >> 5], 1u << (sidx[c] & 31));
-    } else {  // crowded boundary bin: radix over every key matching d0
-      __syncthreads();
-      p = block_radix_select<GKeySrc, kSelNT>(GKeySrc{keys}, A.B, k2, hist, sm, 1, p, true);
-      for (int i = tid; i < A.B; i += kSelNT) {
-        const uint64_t kk = __ldcg(keys + i);
-        if (((kk >> 51) & 0xFFFu) == d0 && ge96(p, kk, ~(uint32_t)i)) atomicOr(&bitmap[i >> 5], 1u << (i & 31));
-      }
-    }
-  }
-  if (sel == 0) TRACE(21);
-  __syncthreads();
-  // ascending winner list
-  int* J = reinterpret_cast<int*>(rec + A.lay.off_J);
-  const int wpt = (words + kSelNT - 1) / kSelNT;
-  constexpr int kWB = 8;  // words held in registers per thread (B <= 65536)
-  uint32_t wb[kWB];
-  int cnt = 0;
-#pragma unroll
-  for (int u = 0; u < kWB; ++u) {
-    const int w = tid * wpt + u;
-    wb[u] = (u < wpt && w < words) ? __ldcg(bitmap + w) : 0u;
-  }
-  for (int w = tid * wpt + kWB; w < min(words, (tid + 1) * wpt); ++w) cnt += __popc(__ldcg(bitmap + w));
-#pragma unroll
-  for (int u = 0; u < kWB; ++u) cnt += __popc(wb[u]);
-  int total;
-  int pos = block_excl_scan<kSelNT>(cnt, &total, sm);
-  for (int w = tid * wpt; w < min(words, (tid + 1) * wpt); ++w) {
-    const int u = w - tid * wpt;
-    uint32_t bits = u < kWB ? wb[u] : __ldcg(bitmap + w);
-    while (bits) {
-      const int b = __ffs(bits) - 1;
-      bits &= bits - 1;
-      J[pos] = w * 32 + b;  // pos < total <= Jcap
-      ++pos;
-    }
-  }
-  if (tid == 0) {
-    *reinterpret_cast<int*>(rec + A.lay.off_cnt) = total;
-    if (!A.threshold_mode && total != A.num) atomicOr(A.status + 1, 1);
-  }
-  if (sel == 0) TRACE(22);
-  TRACE_END(15);
 }
 
 // ---------------------------------------------------------------------------
@@ -1114,43 +749,7 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
   if (r == 0 && tid == 0) S.ncand = 0;
   int d0 = 0, k2 = 0;
   bool whole = true;
-  if (A.local_pick) {
-    // 1+2 without cluster round trips: every CTA finds the boundary bin itself
-    // from the whole 4096-bin histogram (16 KB of L2 reads per CTA) while the
-    // split cluster barrier (arrive now, wait before the first DSMEM access)
-    // completes in the background
-    asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
-    if (!A.threshold_mode) {
-      constexpr int PER = 4096 / kSelCNT;
-      const int base = 4095 - PER * tid;
-      int c[PER];
-      int mine = 0;
-#pragma unroll
-      for (int j = 0; j < PER; ++j) {
-        c[j] = (int)__ldcg(h0 + base - j);
-        mine += c[j];
-      }
-      int total;
-      const int ex2 = block_excl_scan<kSelCNT>(mine, &total, S.sm);
-      if (ex2 < A.num && A.num <= ex2 + mine) {
-        int cum = ex2;
-#pragma unroll
-        for (int j = 0; j < PER; ++j) {
-          if (cum + c[j] >= A.num) {
-            S.sm[32] = base - j; S.sm[33] = cum; S.sm[34] = c[j];
-            break;
-          }
-          cum += c[j];
-        }
-      }
-      __syncthreads();
-      d0 = S.sm[32];
-      k2 = A.num - S.sm[33];
-      whole = (k2 == S.sm[34]);
-      __syncthreads();
-    }
-    asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
-  } else {
+  {
   // 1. slice totals, pushed to every CTA of the cluster
   int tot, ex = 0;
   if (!A.threshold_mode) {
@@ -1278,15 +877,24 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
   uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap) + r * wpc;
   int* J = reinterpret_cast<int*>(rec + A.lay.off_J);
   for (int w = tid; w < wpc; w += kSelCNT) bitmap[w] = sbits[w];
-  if (A.pk) {  // bucket 32 gw + 4 j + i -> byte i of word gw 8 + j, bit sel (k_vote8's layout)
+  if (A.pk) {  // k_tail's vote table: element b (pk_esz bytes) = bucket b, bit sel = kept in location loop sel
     for (int w = tid; w < wpc; w += kSelCNT) {
       const uint32_t bits = sbits[w];
       if (!bits) continue;
-      uint32_t* dst = A.pk + (int64_t)(r * wpc + w) * 8;
+      const int64_t b0 = (int64_t)(r * wpc + w) * 32;  // first bucket of the word
+      if (A.pk_esz == 1) {  // 4 buckets per u32: spread each nibble of bits over 4 bytes
+        uint32_t* dst = A.pk + b0 / 4;
 #pragma unroll
-      for (int j = 0; j < 8; ++j) {
-        const uint32_t nib = (bits >> (4 * j)) & 0xFu;
-        if (nib) atomicOr(dst + j, ((nib * 0x00204081u) & 0x01010101u) << sel);
+        for (int j = 0; j < 8; ++j) {
+          const uint32_t nib = (bits >> (4 * j)) & 0xFu;
+          if (nib) atomicOr(dst + j, ((nib * 0x00204081u) & 0x01010101u) << sel);
+        }
+      } else {
+        for (uint32_t bb = bits; bb; bb &= bb - 1) {
+          const int64_t bkt = b0 + __ffs(bb) - 1;
+          const int per = 4 / A.pk_esz;  // buckets per u32 word
+          atomicOr(A.pk + bkt / per, (1u << sel) << (8 * A.pk_esz * (int)(bkt % per)));
+        }
       }
     }
   }
@@ -1308,213 +916,10 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
 }
 
 __global__ void __launch_bounds__(kSelCNT, 1) k_select_cluster(SelArgs A) {
-  pdl_trigger(3);
   pdl_wait();
   KTRACE(8);
   extern __shared__ __align__(16) uint8_t smem[];
   select_cluster_body(A, blockIdx.x / kSelCL, smem);
-}
-
-// ---------------------------------------------------------------------------
-// Steps 2-4 of one slot in ONE cluster of kSlotCS CTAs, after
-// the scatter-staged phase 1 (k_stage).  B = B1 x B2, CTA r of the cluster
-// owns columns c in [r COLS, (r+1) COLS) (COLS = B2 / kSlotCS) and pass-2
-// rows k1 in [r ROWS, (r+1) ROWS) (ROWS = B1 / kSlotCS):
-//   A. fold + FFT pass 1: its TPC tiles of 256 buckets (C = 256 / B1 columns
-//      x B1 rows each) stream from the staging buffer through shared memory
-//      (bulk copies, two buffers on two mbarriers); per tile exactly
-//      k_fold_fft1_tma's arithmetic (Alg. 1 round order, B1-point FFTs),
-//      u written to global, V[c][k1] = FFT x omega_B^(c k1) kept in smem.
-//   B. cluster barrier; pass 2: row k1 gathers V[c][k1] of all B2 columns
-//      from the owners' shared memory (DSMEM), B2-point FFTs (k_fft's
-//      arithmetic), u^[k1 + B1 k2] to the slot's record, cutoff keys and the
-//      top-digit histogram (location slots).
-//   C. location slots (do_select): cluster barrier, then the cluster
-//      selection (select_cluster_body, same result as k_select_cluster).
-// Replaces k_fold_fft1_tma + k_fft pass 2 + k_select: two launches and the
-// spill of V through L2 disappear.
-// ---------------------------------------------------------------------------
-constexpr int kSlotCS = 8;  // CTAs per cluster (= kSelCL: phase C reuses the cluster selection)
-static_assert(kSlotCS == kSelCL, "slot cluster must match the selection cluster");
-
-struct SlotArgs {
-  const double2* v;         // FROM_V: FFT pass-1 output v[s][c + B2 k1] (k_fold_fft1*), else unused
-  const double2* staging;   // group staging, scatter layout [(s R + rr) B + tile 256 + t]
-  const double* taps_perm;  // [R][B] tile-contiguous taps
-  double2* u;               // [ns][B] (group slot 0)
-  uint8_t* recs;            // record of group slot 0
-  int64_t rec_bytes;
-  const double2* tw;        // e^{-2 pi i t / B}, t < B
-  const int* key_index;     // [ns] selection index of each group slot or -1
-  uint64_t* keys;           // [n_sel][B]
-  uint32_t* hist;           // [n_sel][4096]
-  int B, w, R, discard, do_select;
-  SelArgs sel;
-};
-
-__host__ __device__ constexpr int slot_max3(int a, int b, int c) { return a > b ? (a > c ? a : c) : (b > c ? b : c); }
-__host__ __device__ constexpr int slot_smem_bytes(int B1, int B2, int R) {
-  // V (padded FFT layout) + max(phase A: 2 tiles + twl, phase B: S2 + twl2 + hist, phase C: selection) + 2 mbarriers
-  return ((B1 * B2 / kSlotCS) + (B1 * B2 / kSlotCS) / 8) * 16 +
-         slot_max3(2 * R * 256 * 16 + B1 * 16, ((B1 * B2 / kSlotCS) + (B1 * B2 / kSlotCS) / 8) * 16 + B2 * 16 + 4096 * 4,
-                   (int)sizeof(SelClusterSmem) + 1024) +
-         16;
-}
-
-__host__ __device__ constexpr int slot_smem_bytes_v(int B1, int B2) {
-  // FROM_V: no V region; max(phase B, phase C)
-  return slot_max3(0, ((B1 * B2 / kSlotCS) + (B1 * B2 / kSlotCS) / 8) * 16 + B2 * 16 + 4096 * 4,
-                   (int)sizeof(SelClusterSmem) + 1024);
-}
-
-// FROM_V: phase A was done by k_fold_fft1_tma (v in global, L2-resident);
-// the kernel is then FFT pass 2 + keys + the cluster cutoff (k_fft + k_select).
-template <int B1T, int B2T, bool FROM_V>
-__global__ void __launch_bounds__(256, 1) k_slot(SlotArgs A) {
-  pdl_wait();
-  KTRACE(2);
-  namespace cg = cooperative_groups;
-  cg::cluster_group cl = cg::this_cluster();
-  constexpr int C = 256 / B1T;
-  constexpr int COLS = B2T / kSlotCS;
-  constexpr int TPC = COLS / C;
-  constexpr int ROWS = B1T / kSlotCS;
-  constexpr int E2 = ROWS * B2T;  // == COLS * B1T
-  static_assert(TPC >= 1 && COLS % C == 0 && ROWS >= 1 && E2 >= 256, "slot kernel shape");
-  extern __shared__ __align__(16) uint8_t smem[];
-  double2* V = reinterpret_cast<double2*>(smem);                    // [COLS][B1T], fft_pad layout
-  uint8_t* X = FROM_V ? smem : smem + (E2 + E2 / 8) * 16;           // phase-dependent region
-  const int B = A.B, R = A.R, w = A.w;
-  const int t = threadIdx.x;
-  const int r = (int)cl.block_rank();
-  const int s = blockIdx.x / kSlotCS;
-  if (blockIdx.x == 0) TRACE(0);
-  if constexpr (!FROM_V) {
-  // ---- phase A: fold the CTA's TPC tiles into V (sequence = local column, element = row j1)
-  double2* Tile = reinterpret_cast<double2*>(X);                     // [2][R][256]
-  double2* twl = Tile + 2 * R * 256;                                // [B1T]
-  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + slot_smem_bytes(B1T, B2T, R) - 16);
-  const double2* src0 = A.staging + (int64_t)s * R * B + (int64_t)r * TPC * 256;
-  auto issue = [&](int tl) {  // thread 0: the R rows of tile tl into buffer tl & 1
-    uint64_t* b = bar + (tl & 1);
-    mbar_expect_tx(b, (uint32_t)R * 4096u);
-    const uint64_t pol = l2_policy_first();
-    for (int rr = 0; rr < R; ++rr)
-      bulk_g2s(Tile + ((tl & 1) * R + rr) * 256, src0 + (int64_t)rr * B + tl * 256, 4096u, b, pol);
-  };
-  if (t == 0) {
-    mbar_init(bar, 1);
-    mbar_init(bar + 1, 1);
-  }
-  __syncthreads();
-  if (t == 0) {
-    issue(0);
-    if (TPC > 1) issue(1);
-  }
-  for (int i = t; i < B1T; i += 256) twl[i] = __ldg(A.tw + (int64_t)i * B2T);  // omega_B1^i
-  const int cl_ = t / B1T, j1 = t % B1T;
-  constexpr int RMAX = 16;
-#pragma unroll 1
-  for (int tl = 0; tl < TPC; ++tl) {
-    const int cta = r * TPC + tl;  // tile index within the slot (k_fold_fft1's blockIdx.x)
-    const int j = cta * C + cl_ + B2T * j1;
-    const double* tp = A.taps_perm + (int64_t)cta * 256 + t;
-    double g[RMAX];
-#pragma unroll
-    for (int rr = 0; rr < RMAX; ++rr) g[rr] = (rr < R && j + rr * B < w) ? __ldg(tp + (int64_t)rr * B) : 0.0;
-    mbar_wait(bar + (tl & 1), (uint32_t)((tl >> 1) & 1));
-    const double2* T = Tile + (tl & 1) * R * 256;
-    double ar = 0.0, ai = 0.0;
-#pragma unroll
-    for (int rr = 0; rr < RMAX; ++rr) {
-      if (rr < R && j + rr * B < w) {
-        const double2 q = T[rr * 256 + t];
-        ar = __dadd_rn(ar, __dmul_rn(g[rr], q.x));
-        ai = __dadd_rn(ai, __dmul_rn(g[rr], q.y));
-      }
-    }
-    for (int rr = RMAX; rr < R; ++rr) {
-      if (j + rr * B < w) {
-        const double2 q = T[rr * 256 + t];
-        const double gg = __ldg(tp + (int64_t)rr * B);
-        ar = __dadd_rn(ar, __dmul_rn(gg, q.x));
-        ai = __dadd_rn(ai, __dmul_rn(gg, q.y));
-      }
-    }
-    if (A.discard)
-      for (int q = t; q < R * 32; q += 256) l2_discard(src0 + (int64_t)(q >> 5) * B + tl * 256 + (q & 31) * 8);
-    V[fft_pad((tl * C + cl_) * B1T + j1)] = make_double2(ar, ai);
-    __syncthreads();  // buffer (tl & 1) consumed: refill it with tile tl + 2
-    if (t == 0 && tl + 2 < TPC) issue(tl + 2);
-  }
-  // u (kept for parity checks): runs of COLS consecutive columns per row j1
-  for (int e = t; e < E2; e += 256) {
-    const int cc = e % COLS, jj = e / COLS;
-    A.u[(size_t)s * B + (size_t)r * COLS + cc + (size_t)B2T * jj] = V[fft_pad(cc * B1T + jj)];
-  }
-  fft_smem<B1T, E2, 256, true>(V, twl, B1T);  // the COLS columns' B1-point FFTs (syncs inside)
-  for (int e = t; e < E2; e += 256) {          // twiddle omega_B^(c k1)
-    const int cc = e / B1T, k1 = e % B1T;
-    const int cg_ = r * COLS + cc;
-    V[fft_pad(e)] = cmul(V[fft_pad(e)], __ldg(A.tw + (((int64_t)cg_ * k1) & (B - 1))));
-  }
-  if (blockIdx.x == 0) TRACE(1);
-  cl.sync();  // every CTA's V complete
-  }  // !FROM_V
-  // ---- phase B: rows k1 = r ROWS + rl, element c of row from CTA c / COLS
-  double2* S2 = reinterpret_cast<double2*>(X);                      // [E2 + E2/8]
-  double2* tw2 = S2 + E2 + E2 / 8;                                  // [B2T]
-  uint32_t* shist = reinterpret_cast<uint32_t*>(tw2 + B2T);         // [4096]
-  for (int i = t; i < B2T; i += 256) tw2[i] = __ldg(A.tw + (int64_t)i * B1T);  // omega_B2^i
-  const int ki = A.key_index ? A.key_index[s] : -1;
-  if (ki >= 0)
-    for (int i = t; i < 4096; i += 256) shist[i] = 0;
-  {
-    constexpr int PER = E2 / 256;
-    double2 buf[PER];
-#pragma unroll
-    for (int u2 = 0; u2 < PER; ++u2) {
-      const int e = t + u2 * 256;
-      const int rl = e / B2T, cc = e % B2T;  // consecutive threads: consecutive columns (owners rotate)
-      if constexpr (FROM_V) {
-        buf[u2] = __ldg(A.v + (int64_t)s * B + (int64_t)(r * ROWS + rl) * B2T + cc);
-      } else {
-        const double2* rv = cl.map_shared_rank(V, cc / COLS);
-        buf[u2] = rv[fft_pad((cc % COLS) * B1T + r * ROWS + rl)];
-      }
-    }
-#pragma unroll
-    for (int u2 = 0; u2 < PER; ++u2) {
-      const int e = t + u2 * 256;
-      S2[fft_pad(e)] = buf[u2];
-    }
-  }
-  __syncthreads();
-  fft_smem<B2T, E2, 256, true>(S2, tw2, B2T);
-  {
-    double2* rec = reinterpret_cast<double2*>(A.recs + (int64_t)s * A.rec_bytes);
-    uint64_t* keys = ki >= 0 ? A.keys + (int64_t)ki * B : nullptr;
-    for (int e = t; e < E2; e += 256) {
-      const int rl = e % ROWS, k2 = e / ROWS;  // consecutive threads: consecutive k1 (contiguous m)
-      const double2 v = S2[fft_pad(rl * B2T + k2)];
-      const int m = r * ROWS + rl + B1T * k2;
-      rec[m] = v;
-      if (ki >= 0) {
-        const uint64_t key = (uint64_t)__double_as_longlong(__dadd_rn(__dmul_rn(v.x, v.x), __dmul_rn(v.y, v.y)));
-        keys[m] = key;
-        atomicAdd(&shist[(uint32_t)(key >> 51) & 0xFFFu], 1u);
-      }
-    }
-  }
-  if (ki >= 0) {
-    __syncthreads();
-    for (int i = t; i < 4096; i += 256)
-      if (shist[i]) atomicAdd(&A.hist[(int64_t)ki * 4096 + i], shist[i]);
-  }
-  if (blockIdx.x == 0) TRACE(4);
-  // ---- phase C (the whole cluster takes the same branch: one slot per cluster)
-  cl.sync();  // remote V reads done; keys and histogram of the slot complete
-  if (ki >= 0 && A.do_select) select_cluster_body(A.sel, ki, X);
 }
 
 // ---------------------------------------------------------------------------
@@ -1831,268 +1236,6 @@ __global__ void __launch_bounds__(256) k_vote(VoteArgs A) {
 }
 
 // ---------------------------------------------------------------------------
-// Step 5, packed form (L_loc <= 8, B <= kPk): the location loops' bitmaps are
-// transposed into one byte per bucket (bit q = bucket selected in loop q) in
-// a static shared array, so a probe is IMAD, SHF, LDS.U8 [b + const], LOP3.
-// One CTA of 1024 threads per SM builds the byte array once; then the same
-// warp-per-(q0, J) enumeration, mandatory probes and survivor queue as k_vote.
-// ---------------------------------------------------------------------------
-constexpr int kPk = 16384;
-
-// Shared-memory views addressed by 32-bit shared-window offsets: a generic
-// pointer to a __shared__ array passed into a device function makes the
-// compiler rebuild the window address (S2R SR_CgaCtaId, MOV, LEA) at every
-// probe; these emit one LDS with an immediate base instead.
-struct SmemU8 {
-  uint32_t base;
-  __device__ __forceinline__ uint32_t operator[](uint32_t i) const {
-    uint32_t v;
-    asm volatile("ld.shared.u8 %0, [%1];" : "=r"(v) : "r"(base + i));
-    return v;
-  }
-};
-struct SmemU32 {
-  uint32_t base;
-  __device__ __forceinline__ uint32_t operator[](int i) const {
-    uint32_t v;
-    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(base + 4u * (uint32_t)i));
-    return v;
-  }
-};
-
-__device__ __forceinline__ bool vote8_finish(const VoteArgs& A, SmemU8 pk, SmemU32 ssig, int q0, int m,
-                                             uint32_t F, int got, uint32_t half_s, int bsh) {
-  int votes = got;
-  for (int q = q0 + 1 + m; q < A.Lloc; ++q) votes += (pk[(ssig[q] * F + half_s) >> bsh] >> q) & 1;
-  bool hit = votes >= A.T - 1;
-  for (int q = 0; q < q0; ++q) hit = hit && !((pk[(ssig[q] * F + half_s) >> bsh] >> q) & 1);
-  return hit;
-}
-
-template <int M>
-__device__ __forceinline__ void vote8_unit(const VoteArgs& A, SmemU8 pk, SmemU32 ssig, int q0,
-                                           uint32_t Jv, uint32_t a, int mrt, uint32_t* qF, uint8_t* qG) {
-  constexpr int MM = M > 0 ? M : 1;
-  constexpr int VC = 2;
-  const int lane = threadIdx.x & 31;
-  const int sh = 32 - A.log2n, bsh = 32 - A.log2B;
-  const uint32_t half = (uint32_t)(A.nb >> 1);
-  const uint32_t half_s = half << sh;
-  const int m = M > 0 ? M : mrt;
-  const int allowed = A.Lloc - A.T - q0;
-  uint32_t sg[MM], mk[MM];
-#pragma unroll
-  for (int qq = 0; qq < MM; ++qq) {
-    sg[qq] = __ldg(A.loc_sigma + q0 + 1 + qq);
-    mk[qq] = 1u << (q0 + 1 + qq);
-  }
-  const uint32_t p0 = Jv * (uint32_t)A.nb - half;
-  uint32_t F0 = a * ((p0 + (uint32_t)lane) << sh);
-  const uint32_t d32 = a * (32u << sh);
-  const uint32_t dstep = a * ((32u * VC) << sh);
-  const unsigned lt = (1u << lane) - 1;
-  int qn = 0;
-  for (int t0 = 0; t0 < A.nb; t0 += 32 * VC, F0 += dstep) {
-    uint32_t F[VC], acc[VC];
-#pragma unroll
-    for (int c = 0; c < VC; ++c) {
-      F[c] = F0 + (uint32_t)c * d32;
-      acc[c] = 0u;
-    }
-    if (M > 0) {
-#pragma unroll
-      for (int qq = 0; qq < MM; ++qq)
-#pragma unroll
-        for (int c = 0; c < VC; ++c) acc[c] |= pk[(sg[qq] * F[c] + half_s) >> bsh] & mk[qq];
-    } else {
-      for (int qq = 0; qq < m; ++qq) {
-        const uint32_t sq = ssig[q0 + 1 + qq], mq = 1u << (q0 + 1 + qq);
-#pragma unroll
-        for (int c = 0; c < VC; ++c) acc[c] |= pk[(sq * F[c] + half_s) >> bsh] & mq;
-      }
-    }
-    unsigned bal[VC];
-    int g[VC];
-    unsigned any = 0u;
-#pragma unroll
-    for (int c = 0; c < VC; ++c) {
-      g[c] = __popc(acc[c]);
-      const bool sv = (t0 + c * 32 + lane < A.nb) && (m - g[c]) <= allowed;
-      bal[c] = __ballot_sync(kFull, sv);
-      any |= bal[c];
-    }
-    if (any) {
-#pragma unroll
-      for (int c = 0; c < VC; ++c) {
-        if (bal[c] & (1u << lane)) {
-          const int pos = qn + __popc(bal[c] & lt);
-          qF[pos] = F[c];
-          qG[pos] = (uint8_t)g[c];
-        }
-        qn += __popc(bal[c]);
-      }
-      __syncwarp();
-      while (qn >= 32) {
-        const uint32_t Fq = qF[qn - 32 + lane];
-        const int gq = qG[qn - 32 + lane];
-        __syncwarp();
-        qn -= 32;
-        const bool hit = vote8_finish(A, pk, ssig, q0, m, Fq, gq, half_s, bsh);
-        vote_emit(A, hit, Fq >> sh);
-      }
-    }
-  }
-  if (qn > 0) {
-    const bool has = lane < qn;
-    const uint32_t Fq = has ? qF[lane] : 0u;
-    const int gq = has ? qG[lane] : 0;
-    __syncwarp();
-    const bool hit = has && vote8_finish(A, pk, ssig, q0, m, Fq, gq, half_s, bsh);
-    vote_emit(A, hit, Fq >> sh);
-  }
-}
-
-// Pair enumeration (when T > ceil(L_loc / 2)): with the location loops in
-// pairs (2i, 2i+1), a frequency with >= T votes has some pair voting twice
-// (else it has at most ceil(L_loc/2) votes).  So candidates f = a_{2i} p run
-// over loop 2i's preimage ranges with ONE mandatory probe of loop 2i+1, and
-// f is counted at its first doubly-voting pair: survivors probe every other
-// loop, need >= T votes in all and no earlier pair voting twice.
-__device__ __forceinline__ bool vote8_pair_finish(const VoteArgs& A, SmemU8 pk, SmemU32 ssig, int pr,
-                                                  uint32_t F, uint32_t half_s, int bsh) {
-  uint32_t bits = 3u << (2 * pr);
-  for (int q = 0; q < A.Lloc; ++q)
-    if ((q >> 1) != pr) bits |= pk[(ssig[q] * F + half_s) >> bsh] & (1u << q);
-  bool hit = __popc(bits) >= A.T;
-  for (int j = 0; j < pr; ++j) hit = hit && ((bits >> (2 * j)) & 3u) != 3u;
-  return hit;
-}
-
-__device__ __forceinline__ void vote8_pair_unit(const VoteArgs& A, SmemU8 pk, SmemU32 ssig, int pr,
-                                                uint32_t Jv, uint32_t a, uint32_t* qF) {
-  constexpr int VC = 2;
-  const int lane = threadIdx.x & 31;
-  const int sh = 32 - A.log2n, bsh = 32 - A.log2B;
-  const uint32_t half = (uint32_t)(A.nb >> 1);
-  const uint32_t half_s = half << sh;
-  const uint32_t sg = __ldg(A.loc_sigma + 2 * pr + 1), mk = 1u << (2 * pr + 1);
-  const uint32_t p0 = Jv * (uint32_t)A.nb - half;
-  uint32_t F0 = a * ((p0 + (uint32_t)lane) << sh);
-  const uint32_t d32 = a * (32u << sh);
-  const uint32_t dstep = a * ((32u * VC) << sh);
-  const unsigned lt = (1u << lane) - 1;
-  int qn = 0;
-  for (int t0 = 0; t0 < A.nb; t0 += 32 * VC, F0 += dstep) {
-    const uint32_t F1 = F0 + d32;
-    const bool s0 = (t0 + lane < A.nb) && (pk[(sg * F0 + half_s) >> bsh] & mk);
-    const bool s1 = (t0 + 32 + lane < A.nb) && (pk[(sg * F1 + half_s) >> bsh] & mk);
-    const unsigned b0 = __ballot_sync(kFull, s0), b1 = __ballot_sync(kFull, s1);
-    if (b0 | b1) {
-      if (s0) qF[qn + __popc(b0 & lt)] = F0;
-      const int qn1 = qn + __popc(b0);
-      if (s1) qF[qn1 + __popc(b1 & lt)] = F1;
-      qn = qn1 + __popc(b1);
-      __syncwarp();
-      while (qn >= 32) {
-        const uint32_t Fq = qF[qn - 32 + lane];
-        __syncwarp();
-        qn -= 32;
-        vote_emit(A, vote8_pair_finish(A, pk, ssig, pr, Fq, half_s, bsh), Fq >> sh);
-      }
-    }
-  }
-  if (qn > 0) {
-    const bool has = lane < qn;
-    const uint32_t Fq = has ? qF[lane] : 0u;
-    __syncwarp();
-    vote_emit(A, has && vote8_pair_finish(A, pk, ssig, pr, Fq, half_s, bsh), Fq >> sh);
-  }
-}
-
-__global__ void __launch_bounds__(1024, 1) k_vote8(VoteArgs A) {
-  pdl_trigger(4);
-  pdl_wait();
-  KTRACE(9);
-  __shared__ __align__(16) uint8_t pk[kPk];
-  __shared__ uint32_t ssig[kMaxLoc];
-  __shared__ uint32_t queueF[32][kVQ];
-  __shared__ uint8_t queueG[32][kVQ];
-  __shared__ int scnt[kMaxLoc + 1];
-  if (blockIdx.x == 0) TRACE(30);
-  const int tid = threadIdx.x;
-  const int words = (A.B + 31) >> 5;
-  // transpose: bucket 32 w + 4 j + i -> byte (w 8 + j) * 4 + i, bit q = loop q
-  // (or copy it: the cutoff already ORed the bits into A.pk)
-  if (A.pk) {
-    for (int i = tid; i < (words << 1); i += 1024)
-      reinterpret_cast<uint4*>(pk)[i] = __ldcg(reinterpret_cast<const uint4*>(A.pk) + i);
-  }
-  for (int w = A.pk ? words : tid; w < words; w += 1024) {
-    uint32_t bw[8];
-#pragma unroll
-    for (int q = 0; q < 8; ++q) bw[q] = q < A.Lloc ? __ldg(A.bmp[q] + w) : 0u;
-    auto nib = [&](int j) {
-      uint32_t v = 0u;
-#pragma unroll
-      for (int q = 0; q < 8; ++q) v |= ((((bw[q] >> (4 * j)) & 0xFu) * 0x00204081u) & 0x01010101u) << q;
-      return v;
-    };
-    reinterpret_cast<uint4*>(pk)[w * 2] = make_uint4(nib(0), nib(1), nib(2), nib(3));
-    reinterpret_cast<uint4*>(pk)[w * 2 + 1] = make_uint4(nib(4), nib(5), nib(6), nib(7));
-  }
-  // enumerated loops: pairs' first loops 0, 2, 4, ... (pair mode) or 0 .. L_loc - T
-  const int nenum = A.pairs ? A.Lloc / 2 : A.Lloc - A.T + 1;
-  if (tid < A.Lloc) ssig[tid] = A.sig[tid];
-  // held in registers (a volatile move cannot be rematerialised inside the loops)
-  uint32_t pk_base, ss_base;
-  asm volatile("mov.u32 %0, %1;" : "=r"(pk_base) : "r"(smem_u32(pk)));
-  asm volatile("mov.u32 %0, %1;" : "=r"(ss_base) : "r"(smem_u32(ssig)));
-  const SmemU8 spk{pk_base};
-  const SmemU32 sss{ss_base};
-  if (tid == 0) {
-    int acc = 0;
-    scnt[0] = 0;
-    for (int e = 0; e < nenum; ++e) {
-      acc += __ldg(A.cntp[A.pairs ? 2 * e : e]);
-      scnt[e + 1] = acc;
-    }
-  }
-  __syncthreads();
-  if (blockIdx.x == 0) TRACE(31);
-  const int units = scnt[nenum];
-  uint32_t* qF = queueF[tid >> 5];
-  uint8_t* qG = queueG[tid >> 5];
-  const int warp = (blockIdx.x * 1024 + tid) >> 5;
-  const int nwarps = gridDim.x * 32;
-  if (A.pairs) {  // unit = (pair, winner J, part h of its nb candidates), split parts per winner
-    for (int unit = warp; unit < units; unit += nwarps) {
-      int pr = 0;
-      while (unit >= scnt[pr + 1]) ++pr;
-      const uint32_t Jv = (uint32_t)__ldg(A.Jp[2 * pr] + (unit - scnt[pr]));
-      vote8_pair_unit(A, spk, sss, pr, Jv, A.aa[2 * pr], qF);
-    }
-    TRACE_END(32);
-    return;
-  }
-  for (int unit = warp; unit < units; unit += nwarps) {
-    int q0 = 0;
-    while (unit >= scnt[q0 + 1]) ++q0;
-    const int jidx = unit - scnt[q0];
-    const uint32_t Jv = (uint32_t)__ldg(A.Jp[q0] + jidx);
-    const uint32_t a = A.aa[q0];
-    const int m = min(A.Lloc - A.T - q0 + 1, A.Lloc - 1 - q0);
-    switch (m) {
-      case 1: vote8_unit<1>(A, spk, sss, q0, Jv, a, 1, qF, qG); break;
-      case 2: vote8_unit<2>(A, spk, sss, q0, Jv, a, 2, qF, qG); break;
-      case 3: vote8_unit<3>(A, spk, sss, q0, Jv, a, 3, qF, qG); break;
-      case 4: vote8_unit<4>(A, spk, sss, q0, Jv, a, 4, qF, qG); break;
-      default: vote8_unit<0>(A, spk, sss, q0, Jv, a, m, qF, qG); break;
-    }
-  }
-  TRACE_END(32);
-}
-
-// ---------------------------------------------------------------------------
 // Step 6 (L95, Alg. 5), one warp per hit, one lane per loop (slot).
 // For hit f and loop l:  p = sigma_l f mod n, h = p / nb, d = p mod nb;
 //   if d > nb/2: h = h+1 mod B, d -= nb;
@@ -2105,7 +1248,9 @@ struct EstArgs {
   RecLayout lay;
   const SlotParam* slots;
   int L;
-  const double2* ghat;
+  const double2* ghat;      // G^ of the location loops' filter, q = -nb/2 .. nb/2
+  const double2* ghat_est;  // G^ of loops r >= ghat_split (the estimation-only filter)
+  int ghat_split;           // L_loc with separate filters, else L
   const int* hits;
   const unsigned* hit_count;
   int max_hits;
@@ -2127,7 +1272,7 @@ __device__ __forceinline__ double2 loop_estimate(const EstArgs& A, const SlotPar
     hb = (hb + 1) & (A.B - 1);
     d -= A.nb;
   }
-  const double2 g = __ldg(A.ghat + (A.nb >> 1) - d);  // G^(-d)
+  const double2 g = __ldg((sp.loop < (uint32_t)A.ghat_split ? A.ghat : A.ghat_est) + (A.nb >> 1) - d);  // G^(-d)
   const double2 b = __ldg(reinterpret_cast<const double2*>(A.records + (int64_t)l * A.lay.rec_bytes) + hb);
   const uint32_t tph = (sp.tau * f) & A.nmask;
   double sn, cs;
@@ -2163,7 +1308,7 @@ __device__ __forceinline__ double warp_rank_select(double a0, double a1, int L, 
 }
 
 __global__ void __launch_bounds__(256) k_estimate(EstArgs A) {
-  pdl_trigger(5);
+  pdl_launch_dependents();
   pdl_wait();
   KTRACE(10);
   __shared__ uint32_t sdig[8];
@@ -2218,7 +1363,7 @@ __global__ void __launch_bounds__(256) k_estimate(EstArgs A) {
 // Twice (L = 16) the hits per warp of k_estimate with all 32 lanes busy.
 template <int LP>
 __global__ void __launch_bounds__(256) k_estimate_seg(EstArgs A) {
-  pdl_trigger(5);
+  pdl_launch_dependents();
   pdl_wait();
   KTRACE(10);
   constexpr int G = 32 / LP;    // hits per warp
@@ -2282,194 +1427,6 @@ __global__ void __launch_bounds__(256) k_estimate_seg(EstArgs A) {
     __syncthreads();
   }
   TRACE_END(41);
-}
-
-// ---------------------------------------------------------------------------
-// Output: the k hits of largest |val|^2 (ties to the smaller f), written in
-// ascending f; pads loc = -1, val = 0.  One CTA of 1024 threads: two-level
-// selection (level 0 counted by k_estimate), then a bucket sort by the top 10
-// bits of f with a per-bucket insertion sort (bitonic fallback for crowded
-// buckets).  Dynamic smem: 4096 u32 hist + 64 ints + kOutCap x (u64 + int)
-// + kp2 x u64 + 1024 x 2 ints.
-// ---------------------------------------------------------------------------
-constexpr int kOutCap = 4096;
-
-__global__ void __launch_bounds__(1024) k_output(const int* __restrict__ hits, const unsigned* __restrict__ hit_count,
-                                                 int max_hits, const double2* __restrict__ hit_vals,
-                                                 const uint64_t* __restrict__ hit_keys, uint32_t* __restrict__ ghist,
-                                                 int k, int kp2, int log2n, int64_t* __restrict__ locs,
-                                                 double2* __restrict__ vals, int* __restrict__ status) {
-  pdl_wait();
-  KTRACE(11);
-  extern __shared__ __align__(16) uint8_t smem[];
-  uint32_t* hist = reinterpret_cast<uint32_t*>(smem);
-  int* sm = reinterpret_cast<int*>(smem + 4096 * 4);
-  uint64_t* ckey = reinterpret_cast<uint64_t*>(smem + 4096 * 4 + 64 * 4);
-  int* cidx = reinterpret_cast<int*>(ckey + kOutCap);
-  uint64_t* sel = reinterpret_cast<uint64_t*>(cidx + kOutCap);  // (f << 32 | i), kp2 entries
-  uint64_t* srt = sel + kp2;                                     // bucket-sorted copy
-  int* bcnt = reinterpret_cast<int*>(srt + kp2);                 // 1024 bucket counters
-  int* bstart = bcnt + 1024;                                     // 1024 bucket starts
-  const int tid = threadIdx.x;
-  TRACE(50);
-  const unsigned hc = *hit_count;
-  const int H = min((int)hc, max_hits);
-  if (tid == 0 && (int)hc > max_hits) atomicOr(status, 1);
-  const int K = min(k, H);
-  // Fast path (H <= 4096 items, k <= 2048): every item's key, f and value are
-  // loaded into registers while the level-0 boundary bin is found; if that
-  // bin is taken whole (the usual case: the k planted coefficients stand far
-  // above the false hits), one classification pass selects, and the values
-  // go to shared memory (aliasing the unused candidate arrays), so neither the
-  // sort nor the write-out touches global memory again.
-  constexpr int PF = 4, NCH = 4;  // items per thread per chunk, chunks (H <= 16384 on the fast path)
-  double2* selv = reinterpret_cast<double2*>(ckey);  // [kp2] values of the selected entries (fast path)
-  const bool fast = H <= NCH * PF * 1024 && kp2 * 16 <= kOutCap * 12;
-  uint64_t pk[PF];
-  uint32_t pf[PF];
-  double2 pv[PF];
-  if (fast) {  // chunk 0: keys, f and values
-#pragma unroll
-    for (int u = 0; u < PF; ++u) {
-      const int i = u * 1024 + tid;
-      if (i < H) {
-        pk[u] = __ldg(hit_keys + i);
-        pf[u] = (uint32_t)__ldg(hits + i);
-        pv[u] = __ldg(hit_vals + i);
-      }
-    }
-  }
-  if (tid == 0) sm[41] = 0;
-  bcnt[tid] = 0;
-  bool direct = false;  // selv holds the values
-  if (fast) {
-    uint32_t d0 = 0;
-    bool whole = true;
-    if (H > K) {
-      const BinPick b0 = pick_bin(ghist, K, sm);  // syncs
-      d0 = (uint32_t)b0.d;
-      whole = (K - b0.above) == b0.cnt;
-    } else {
-      __syncthreads();
-    }
-    if (whole) {
-      direct = true;
-      const int lane = tid & 31;
-      for (int ch = 0; ch < NCH && ch * PF * 1024 < H; ++ch) {  // block-uniform
-        if (ch > 0) {  // later chunks (many false hits): keys and f here, values only for the selected
-#pragma unroll
-          for (int u = 0; u < PF; ++u) {
-            const int i = ch * PF * 1024 + u * 1024 + tid;
-            if (i < H) {
-              pk[u] = __ldg(hit_keys + i);
-              pf[u] = (uint32_t)__ldg(hits + i);
-            }
-          }
-        }
-#pragma unroll
-        for (int u = 0; u < PF; ++u) {
-          const int i = ch * PF * 1024 + u * 1024 + tid;
-          const bool take = i < H && ((uint32_t)(pk[u] >> 51) & 0xFFFu) >= d0;
-          const unsigned bal = __ballot_sync(kFull, take);
-          int base = 0;
-          if (lane == 0 && bal) base = atomicAdd(&sm[41], __popc(bal));
-          base = __shfl_sync(kFull, base, 0);
-          if (take) {
-            const int pos = base + __popc(bal & ((1u << lane) - 1u));
-            if (pos < kp2) {
-              sel[pos] = ((uint64_t)pf[u] << 32) | (uint32_t)pos;
-              selv[pos] = ch == 0 ? pv[u] : __ldg(hit_vals + i);
-            }
-          }
-        }
-      }
-      __syncthreads();
-    }
-  } else {
-    __syncthreads();
-  }
-  if (!direct) {
-    auto add = [&](int i) {
-      const int pos = atomicAdd(&sm[41], 1);
-      if (pos < kp2) sel[pos] = ((uint64_t)(uint32_t)__ldg(hits + i) << 32) | (uint32_t)i;
-    };
-    if (H > K) {
-      select_topk(
-          H, K, ghist,
-          [&](int i, uint64_t& kk, uint32_t& t) {
-            kk = __ldg(hit_keys + i);
-            t = (uint32_t)__ldg(hits + i);
-          },
-          add, ckey, cidx, kOutCap, hist, sm);
-    } else {
-      for (int i = tid; i < H; i += 1024) add(i);
-      __syncthreads();
-    }
-  }
-  TRACE(51);
-  const int ns = min(sm[41], kp2);
-  if (tid == 0 && sm[41] != K) atomicOr(status + 2, 1);
-  // bucket sort by the top 10 bits of f
-  const int sh = max(0, log2n - 10);
-  for (int i = tid; i < ns; i += 1024) atomicAdd(&bcnt[(int)(sel[i] >> 32) >> sh], 1);
-  __syncthreads();
-  const int c = bcnt[tid];
-  int total;
-  const int st = block_excl_scan<1024>(c, &total, sm);
-  bstart[tid] = st;
-  if (tid == 0) sm[42] = 0;
-  __syncthreads();
-  atomicMax(&sm[42], c);
-  bcnt[tid] = 0;
-  __syncthreads();
-  for (int i = tid; i < ns; i += 1024) {
-    const int bkt = (int)(sel[i] >> 32) >> sh;
-    srt[bstart[bkt] + atomicAdd(&bcnt[bkt], 1)] = sel[i];
-  }
-  __syncthreads();
-  if (sm[42] <= 32) {
-    const int b0 = bstart[tid];
-    for (int i = 1; i < c; ++i) {  // insertion sort of this thread's bucket
-      const uint64_t v = srt[b0 + i];
-      int j = i - 1;
-      while (j >= 0 && srt[b0 + j] > v) {
-        srt[b0 + j + 1] = srt[b0 + j];
-        --j;
-      }
-      srt[b0 + j + 1] = v;
-    }
-  } else {  // crowded bucket: bitonic over all selected entries
-    for (int i = ns + tid; i < kp2; i += 1024) srt[i] = ~0ull;
-    __syncthreads();
-    for (int size = 2; size <= kp2; size <<= 1) {
-      for (int stride = size >> 1; stride > 0; stride >>= 1) {
-        for (int t = tid; t < (kp2 >> 1); t += 1024) {
-          const int i = 2 * t - (t & (stride - 1));
-          const int jn = i + stride;
-          const bool up = (i & size) == 0;
-          const uint64_t a = srt[i], b = srt[jn];
-          if ((a > b) == up) {
-            srt[i] = b;
-            srt[jn] = a;
-          }
-        }
-        __syncthreads();
-      }
-    }
-  }
-  __syncthreads();
-  TRACE(52);
-  for (int j = tid; j < k; j += 1024) {
-    if (j < ns) {
-      const uint64_t v = srt[j];
-      locs[j] = (int64_t)(v >> 32);
-      vals[j] = direct ? selv[(uint32_t)v] : hit_vals[(uint32_t)v];
-    } else {
-      locs[j] = -1;
-      vals[j] = make_double2(0.0, 0.0);
-    }
-  }
-  TRACE(53);
 }
 
 }  // namespace cusfft

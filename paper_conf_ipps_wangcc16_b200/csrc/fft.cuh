@@ -152,7 +152,6 @@ __host__ __device__ constexpr int fft_smem_bytes(int E) { return (E + E / 8) * 1
 
 template <int M, int E, int NT>
 __global__ void __launch_bounds__(NT) k_fft(FftPassArgs A) {
-  pdl_trigger(2);
   pdl_wait();
   KTRACE(A.twiddle ? 5 : 6);
   constexpr int NSEQ = E / M;

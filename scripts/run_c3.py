@@ -2,6 +2,7 @@
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
+import bench
 from paper_conf_ipps_wangcc16_b200 import Plan
 from paper_conf_ipps_wangcc16_b200.workload import planted_signal
 cfg = sys.argv[1] if len(sys.argv) > 1 else "C3"
@@ -10,8 +11,7 @@ reps = int(sys.argv[2]) if len(sys.argv) > 2 else 4
 LL = int(sys.argv[3]) if len(sys.argv) > 3 else 16
 x, S, X = planted_signal(n, k, 1)
 xd = torch.from_numpy(x).cuda()
-tol = {"C3": 1e-7}.get(cfg, 1e-8)  # bench.py TOLERANCE
-plan = Plan(n, k, L=LL, seed=3, tolerance=tol)
+plan = Plan(n, k, L=LL, seed=3, **bench.plan_params(cfg))  # the bench's filter parameters
 fl = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 fr = torch.ones(64 << 20, dtype=torch.int32, device="cuda")
 for _ in range(reps):

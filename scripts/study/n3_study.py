@@ -58,8 +58,26 @@ SETTINGS2 = {
     "loc_d1e-6_lam2.0_est_lam1.0": (1e-6, 2.0, 1e-7, 1, 1.0),
     "loc_d1e-6_lam1.0_est_lam1.0": (1e-6, 1.0, 1e-7, 1, 1.0),
 }
+# third round (N3_SET=3): the candidates over more seeds; num = 1.25 k gives the
+# cutoff slack against buckets a wide main lobe lets a neighbour share
+SETTINGS3 = {
+    "all_d1e-7_lam0.75": (1e-7, 0.75, 1e-7, 1, 0.75),
+    "all_d1e-7_lam1.0": (1e-7, 1.0, 1e-7, 1, 1.0),
+    "all_d1e-7_lam1.0_num1.25k": (1e-7, 1.0, 1e-7, 1.25, 1.0),
+    "loc_d1e-7_lam1.25_est_lam1.0_num1.25k": (1e-7, 1.25, 1e-7, 1.25, 1.0),
+}
+# fourth round (N3_SET=4): a looser location filter next to the lambda = 0.75/B estimation filter
+SETTINGS4 = {
+    "loc_d1e-6_lam0.75_est_d1e-7_lam0.75": (1e-6, 0.75, 1e-7, 1, 0.75),
+    "loc_d1e-5_lam0.75_est_d1e-7_lam0.75": (1e-5, 0.75, 1e-7, 1, 0.75),
+    "loc_d1e-5_lam0.875_est_d1e-7_lam0.75": (1e-5, 0.875, 1e-7, 1, 0.75),
+}
+if os.environ.get("N3_SET") == "4":
+    SETTINGS = SETTINGS4
 if os.environ.get("N3_SET") == "2":
     SETTINGS = SETTINGS2
+if os.environ.get("N3_SET") == "3":
+    SETTINGS = SETTINGS3
 
 _taps = {}
 
@@ -81,7 +99,7 @@ def run_setting(x, S, X, seed, name):
     u = np.stack([O.perm_filter(x, g_loc if r < L_loc else g_est, int(sigma[r]), int(tau[r]), B)
                   for r in range(L_loc + L_est)])
     uhat = O.bucket_fft(u)
-    J = [O.cutoff(uhat[r], numf * k) for r in range(L_loc)]
+    J = [O.cutoff(uhat[r], int(numf * k)) for r in range(L_loc)]
     hits = np.sort(O.location_recovery(J, a[:L_loc], n, B, T))
     _, pl_loc = O.estimate(hits, uhat[:L_loc], sigma[:L_loc], tau[:L_loc], G_loc, n, B)
     _, pl_est = O.estimate(hits, uhat[L_loc:], sigma[L_loc:], tau[L_loc:], G_est, n, B)
@@ -90,7 +108,7 @@ def run_setting(x, S, X, seed, name):
     vals = np.sort(per_loop.real, axis=1)[:, med] + 1j * np.sort(per_loop.imag, axis=1)[:, med]
     locs, out = O.select_output(hits, vals, k)
     return {"setting": name, "seed": seed, "delta_loc": d_loc, "lambda_loc_B": lam_loc, "delta_est": d_est,
-            "lambda_est_B": lam_est, "num": numf * k, "w_loc": len(g_loc), "w_est": len(g_est),
+            "lambda_est_B": lam_est, "num": int(numf * k), "w_loc": len(g_loc), "w_est": len(g_est),
             "sum_w": L_loc * len(g_loc) + L_est * len(g_est),
             "exact": bool(set(locs.tolist()) == set(S.tolist())),
             "l1": O.l1_error(locs, out, S, X, k), "hits": int(len(hits))}

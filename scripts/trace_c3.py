@@ -3,6 +3,7 @@ CUSFFT_LIB=libcusfft_trace.so).  Usage: trace_c3.py [L] [tolerance] [reps]"""
 import ctypes, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
+import bench
 from paper_conf_ipps_wangcc16_b200 import Plan, load_library
 from paper_conf_ipps_wangcc16_b200.workload import planted_signal
 n, k = 2**24, 1000
@@ -11,12 +12,15 @@ tol = float(sys.argv[2]) if len(sys.argv) > 2 else 1e-7
 reps = int(sys.argv[3]) if len(sys.argv) > 3 else 5
 x, S, X = planted_signal(n, k, 1)
 xd = torch.from_numpy(x).cuda()
-plan = Plan(n, k, L=L, seed=3, tolerance=tol)
+prm = bench.plan_params("C3")
+if len(sys.argv) > 2:
+    prm["tolerance"] = tol
+plan = Plan(n, k, L=L, seed=3, **prm)
 lib = load_library()
 fl = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 fr = torch.ones(64 << 20, dtype=torch.int32, device="cuda")
-names = {1: "k_stage", 2: "k_fold_fft1", 3: "k_fold_staged", 4: "k_fold", 5: "k_fft pass1", 6: "k_fft pass2",
-         7: "k_keys", 8: "k_select", 9: "k_vote", 10: "k_estimate", 11: "k_output"}
+names = {1: "k_stage_packed", 2: "k_fold_fft1*", 4: "k_fold", 5: "k_fft pass1", 6: "k_fft pass2",
+         7: "k_keys", 8: "k_select*", 9: "k_tail / k_vote", 10: "k_estimate", 11: "k_output"}
 acc = {}
 for rep in range(reps):
     fl.zero_(); fr.sum()

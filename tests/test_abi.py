@@ -40,13 +40,16 @@ def test_library_is_sm100a():
 
 
 def test_params_struct_layout():
-    assert ctypes.sizeof(b.CusfftParams) == 104
+    # include/cusfft.h cusfft_params (x86-64 SysV layout): 17 v1 fields (104 B) +
+    # loc_tolerance, loc_lobefrac, l2_persist, gather
+    assert ctypes.sizeof(b.CusfftParams) == 128
+    assert b.CusfftParams.loc_tolerance.offset == 104 and b.CusfftParams.gather.offset == 124
 
 
 def test_abi_version_and_strerror():
     lib = pkg.load_library()
-    assert lib.cusfft_abi_version() == 1
-    for code in range(0, -12, -1):
+    assert lib.cusfft_abi_version() == 2
+    for code in range(0, -13, -1):
         assert lib.cusfft_strerror(code)
     assert b"unknown" in lib.cusfft_strerror(-99)
 
@@ -65,6 +68,7 @@ def test_params_default_values():
     assert p.filter == 0 and p.tolerance == 1e-8 and p.lobefrac == 0.5 / 16384
     assert p.box_width == 1023 and p.num_select == 1000 and p.tau_mode == 1
     assert p.loc_loops == 0 and p.vote_threshold == 0 and p.device == -1
+    assert p.loc_tolerance == 0.0 and p.loc_lobefrac == 0.0 and p.l2_persist == 1 and p.gather == 0
 
 
 @pytest.mark.parametrize("n,k,B,code", [
@@ -95,6 +99,8 @@ def test_null_pointers_and_invalid_plan():
     (dict(tolerance=0.0), b.INVALID_PARAM), (dict(box_width=256), b.INVALID_PARAM),
     (dict(tau_mode=2), b.INVALID_PARAM), (dict(cutoff_mode=3), b.INVALID_PARAM),
     (dict(cutoff_mode=2, cutoff_threshold=0.0), b.INVALID_PARAM),
+    (dict(loc_tolerance=1.5), b.INVALID_PARAM), (dict(loc_lobefrac=0.6), b.INVALID_PARAM),
+    (dict(l2_persist=2), b.INVALID_PARAM), (dict(gather=3), b.INVALID_PARAM),
 ])
 def test_plan_validation_before_device(kw, code):
     """Parameter validation happens before any CUDA call, so it is testable here."""
@@ -117,7 +123,7 @@ def test_dist_plan_validation(world, L, shard, code):
     p = pkg.default_params(2 ** 14, 8, 64)
     p.shard_mode = shard
     h = ctypes.c_void_p()
-    assert lib.cusfft_plan_dist(ctypes.byref(h), 2 ** 14, 8, 64, L, ctypes.byref(p), 0, world) == code
+    assert lib.cusfft_plan_dist(ctypes.byref(h), 2 ** 14, 8, 64, L, ctypes.byref(p), 0, world, None) == code
     assert not h.value
 
 
@@ -131,7 +137,7 @@ def test_signal_sharding_accepts_any_L():
     p = pkg.default_params(2 ** 14, 8, 64)
     p.shard_mode = 1
     h = ctypes.c_void_p()
-    assert lib.cusfft_plan_dist(ctypes.byref(h), 2 ** 14, 8, 64, 15, ctypes.byref(p), 1, 4) == b.CUDA
+    assert lib.cusfft_plan_dist(ctypes.byref(h), 2 ** 14, 8, 64, 15, ctypes.byref(p), 1, 4, None) == b.CUDA
 
 
 def test_no_cpu_fallback_without_device():
@@ -142,3 +148,16 @@ def test_no_cpu_fallback_without_device():
     with pytest.raises(b.CusfftError) as e:
         pkg.Plan(2 ** 14, 8)
     assert e.value.code == b.CUDA
+
+
+def test_nccl_unique_id_host_only():
+    """cusfft_nccl_unique_id loads NCCL at run time (no link dependency) and
+    returns 128 bytes; a NULL destination is refused."""
+    lib = pkg.load_library()
+    assert lib.cusfft_nccl_unique_id(None) == b.NULL_PTR
+    try:
+        uid = pkg.nccl_unique_id()
+    except b.CusfftError as e:  # NCCL not loadable in this environment
+        assert e.code == b.NCCL
+        return
+    assert isinstance(uid, bytes) and len(uid) == 128

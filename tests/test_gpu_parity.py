@@ -25,7 +25,8 @@ REL = 1e-9
 
 def _oracle_params(n, k, B, L, **kw):
     okw = {key: kw[key] for key in ("loc_loops", "vote_threshold", "num_select", "filter", "tolerance",
-                                    "tau_mode", "seed", "cutoff_mode", "cutoff_threshold") if key in kw}
+                                    "lobefrac", "loc_tolerance", "loc_lobefrac", "tau_mode", "seed",
+                                    "cutoff_mode", "cutoff_threshold") if key in kw}
     return O.make_params(n, k, B=B, L=L, **okw)
 
 
@@ -114,8 +115,9 @@ CASES = [
     (2 ** 15, 1, None, 16, {}),                       # k = 1
     (2 ** 16, 32, None, 16, dict(loc_loops=8, vote_threshold=4)),   # vote: no pair enumeration (T <= L_loc/2)
     (2 ** 16, 32, None, 14, dict(loc_loops=7, vote_threshold=5)),   # vote: pairs + odd singleton loop
-    (2 ** 16, 32, None, 16, dict(loc_loops=12, vote_threshold=7)),  # vote: L_loc > 8, bitmap kernel
-    (2 ** 21, 60, 32768, 8, dict(loc_loops=6, vote_threshold=4)),   # vote: B > 16384, bitmap kernel; multi-pass FFT
+    (2 ** 16, 32, None, 16, dict(loc_loops=12, vote_threshold=7)),  # tail: 16-bit vote table (L_loc > 8)
+    (2 ** 16, 32, None, 24, dict(loc_loops=20, vote_threshold=11)),  # tail: 32-bit table, warp-per-hit estimate (L > 16)
+    (2 ** 21, 60, 32768, 8, dict(loc_loops=6, vote_threshold=4)),   # B > 16384, q0 enumeration (T <= L_loc/2)
 ]
 
 
@@ -264,7 +266,8 @@ def test_stage_timing_and_launch_count():
     t = plan.stage_times()
     assert all(v >= 0 for nm, v in t.items() if nm != "gather") and t["fold"] > 0
     assert (t["gather"] > 0) == bool(plan.info()["staged"])
-    assert plan.launches_per_execute() == 6
+    # C2 (B = 2048: one FFT pass, direct fold): fold x 2 slot ranges, FFT, cutoff, tail
+    assert plan.info()["tail"] == 1 and plan.launches_per_execute() == 5
 
 
 def test_C4_full_size_parity():
@@ -290,33 +293,32 @@ def test_parity_snr_sweep(snr_db):
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("env", [{"CUSFFT_VOTE_PAIRS": "0"}, {"CUSFFT_VOTE_BITMAP": "1"}, {"CUSFFT_SELECT": "multi"}, {"CUSFFT_SELECT": "single"},
-                                 {"CUSFFT_STAGE_MODE": "split_index"}, {"CUSFFT_STAGE_MODE": "fused_scatter"},
-                                 {"CUSFFT_STAGE_MODE": "split_scatter"}, {"CUSFFT_NO_STAGE": "1"},
-                                 {"CUSFFT_STAGE_MODE": "fused_index"}, {"CUSFFT_P2": "ldg"}, {"CUSFFT_DISCARD": "1"}, {"CUSFFT_STAGE_U": "8"}, {"CUSFFT_STAGE_U": "2"},
-                                 {"CUSFFT_SLOT": "1"}, {"CUSFFT_SLOT": "2"}, {"CUSFFT_BRANCH": "1"}, {"CUSFFT_BRANCH": "2"}, {"CUSFFT_BRANCH": "3"}, {"CUSFFT_BRANCH": "4"}, {"CUSFFT_BRANCH": "5"},
-                                 {"CUSFFT_STAGE_GROUPS": "2"}, {"CUSFFT_PACKED": "0"},
-                                 {"CUSFFT_FFT_E": "1024"}, {"CUSFFT_FFT_E": "256"}, {"CUSFFT_PK": "0"}, {"CUSFFT_PDL_TRIGGER": "0"}, {"CUSFFT_PDL_TRIGGER": "63"}, {"CUSFFT_SPLIT_LAUNCH": "1"}, {"CUSFFT_EST_SEG": "0"}, {"CUSFFT_SEL_LOCALPICK": "1"}, {"CUSFFT_NODE_PRIO": "0"}, {"CUSFFT_BRANCH": "0"}])
-def test_kernel_variants_agree(env, monkeypatch):
-    """Every alternative kernel path (selected at plan time by environment
-    switches, used for A/B measurements) gives the default path's hits and
-    output exactly (same fold order, same selection rule)."""
+@pytest.mark.parametrize("env,kw", [({"CUSFFT_NO_GRAPH": "1"}, {}), ({"CUSFFT_TAIL": "0"}, {}),
+                                    ({}, dict(gather=1)), ({}, dict(l2_persist=0)),
+                                    ({"CUSFFT_TAIL": "0", "CUSFFT_NO_GRAPH": "1"}, dict(gather=1))])
+def test_kernel_paths_agree(env, kw, monkeypatch):
+    """Every alternative path (no CUDA graph, the k_vote / k_estimate /
+    k_output chain instead of the fused tail, the direct gather instead of
+    the staged one, no persisting-L2 set-aside) gives the default path's hits
+    and output exactly (same fold order, same selection rules)."""
     import torch
     from paper_conf_ipps_wangcc16_b200 import Plan
-    # n = 2^22, k = 1000: B = 8192, two FFT passes, staged fold, branched graph
+    # n = 2^22, k = 1000: B = 8192, two FFT passes, staged fold, two-branch graph
     n, k = 2 ** 22, 1000
     x, S, X = planted_signal(n, k, seed=21)
     xd = torch.from_numpy(x).cuda()
     base = Plan(n, k, L=16, seed=4, debug=1)
-    assert base.info()["staged"]
+    assert base.info()["staged"] and base.info()["tail"]
     l0, v0 = base.execute(xd)
     h0 = np.sort(base.debug(DEBUG_HITS))
     for key, val in env.items():
         monkeypatch.setenv(key, val)
-    alt = Plan(n, k, L=16, seed=4, debug=1)
+    alt = Plan(n, k, L=16, seed=4, debug=1, **kw)
     l1, v1 = alt.execute(xd)
     torch.cuda.synchronize()
     assert alt.status() == 0
+    assert alt.info()["tail"] == (0 if env.get("CUSFFT_TAIL") == "0" else 1)
+    assert alt.info()["staged"] == (0 if kw.get("gather") == 1 else 1)
     assert np.array_equal(np.sort(alt.debug(DEBUG_HITS)), h0)
     assert torch.equal(l1, l0)
     assert torch.equal(v1, v0)
@@ -419,3 +421,124 @@ def test_l2_setaside_held_and_released():
     assert after == before or after == during  # == during only if another live plan still holds it
     if before == 0:
         assert after == 0
+
+
+@pytest.mark.gpu
+def test_C3_bench_plan_elementwise():
+    """The bench's own plan (bench.py C3 configuration, debug = 0, default
+    launch path) against the oracle element by element: locations exact,
+    values within 1e-9 relative (north_star), planted truth recovered."""
+    import bench
+    n, k, L = bench.CONFIGS["C3"][:3]
+    prm = bench.plan_params("C3")
+    x, S, X = planted_signal(n, k, seed=1)
+    B = O.default_B(n, k)
+    plan = Plan(n, k, B=B, L=L, seed=3, **prm)
+    assert plan.info()["staged"] == 1 and plan.info()["tail"] == 1
+    locs, vals = plan.execute(torch.from_numpy(x).to(DEV))
+    torch.cuda.synchronize()
+    assert plan.status() == 0
+    locs, vals = locs.cpu().numpy(), vals.cpu().numpy()
+    ref = O.sfft(x, _oracle_params(n, k, B, L, seed=3, **prm))
+    assert np.array_equal(locs, ref.locs)
+    assert_close(vals, ref.vals)
+    assert set(locs.tolist()) == set(S.tolist())
+    assert O.l1_error(locs, vals, S, X, k) <= 1e-6
+
+
+@pytest.mark.gpu
+def test_C4_noisy_parity():
+    """BASELINE.json configs[3]: n = 2^27, k = 1000 with additive Gaussian
+    noise (SNR 20 dB), full size: GPU = oracle (debug artefacts, hits,
+    outputs) whatever the noise does to recovery."""
+    n, k = 2 ** 27, 1000
+    x, S, X = planted_signal(n, k, seed=12, snr_db=20.0)
+    plan, ref, locs, vals = run_pair(x, n, k, None, 16, shared_taps=False, seed=7)
+    check_all(plan, ref, locs, vals, fold_bit_exact=False)
+
+
+@pytest.mark.gpu
+def test_C1_gpu_values_equal_direct_dft():
+    """BASELINE.json configs[0] (C1): the GPU's recovered values
+    equal (1/n) x^_f by direct summation, at fixed seeds."""
+    n, k = 2 ** 14, 8
+    t = np.arange(n)
+    for seed in range(4):
+        x, S, X = planted_signal(n, k, seed)
+        with Plan(n, k, L=16, seed=200 + seed, num_select=2 * k) as plan:
+            locs, vals = plan.execute(torch.from_numpy(x).to(DEV))
+            locs, vals = locs.cpu().numpy(), vals.cpu().numpy()
+        assert set(locs.tolist()) == set(S.tolist())
+        ref = np.array([np.sum(x * np.exp(-2j * np.pi * ((int(f) * t) % n) / n)) for f in locs]) / n
+        np.testing.assert_allclose(vals, ref, rtol=0, atol=1e-9)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("n,k,extra", [
+    (2 ** 16, 32, dict(loc_tolerance=1e-6, loc_lobefrac=1.0 / 512, tolerance=1e-8, num_select=64)),
+    (2 ** 22, 1000, dict(loc_tolerance=1e-6, loc_lobefrac=1.0 / 8192, tolerance=1e-7, lobefrac=0.75 / 8192)),
+])
+def test_parity_separate_filters(n, k, extra):
+    """location loops with their own (delta, lambda) filter; GPU-built
+    filters against the oracle's, staged or direct fold, the fused tail with
+    two G^ tables.  The 2^22 case is staged (two filter groups in one
+    address-sorted schedule)."""
+    x, S, X = planted_signal(n, k, seed=5)
+    plan, ref, locs, vals = run_pair(x, n, k, None, 16, shared_taps=False, seed=8, **extra)
+    info = plan.info()
+    assert info["filters"] == 2 and info["w_loc"] < info["w"]
+    gl = plan.debug(b.DEBUG_LOC_TAPS)
+    assert np.abs(gl - ref.extra["taps_loc"]).max() <= 1e-12 * np.abs(gl).max()
+    check_all(plan, ref, locs, vals, fold_bit_exact=False)
+    assert set(locs.tolist()) == set(S.tolist())
+
+
+@pytest.mark.gpu
+def test_library_owned_nccl_exchange_world1():
+    """cusfft_plan_dist with an ncclUniqueId: the plan owns a communicator and
+    cusfft_execute runs the whole transform with the collective inside the
+    plan's CUDA graph (a one-rank communicator on the single test GPU); the
+    output equals the plain plan's bit for bit."""
+    from paper_conf_ipps_wangcc16_b200 import nccl_unique_id
+    n, k = 2 ** 22, 1000
+    x, S, X = planted_signal(n, k, seed=27)
+    xd = torch.from_numpy(x).to(DEV)
+    plain = Plan(n, k, L=16, seed=6)
+    l0, v0 = plain.execute(xd)
+    owned = Plan(n, k, L=16, seed=6, rank=0, world=1, nccl_id=nccl_unique_id())
+    assert owned.info()["owns_comm"] == 1
+    for _ in range(2):  # capture, then replay
+        l1, v1 = owned.execute(xd)
+        torch.cuda.synchronize()
+        assert owned.status() == 0
+        assert torch.equal(l0, l1) and torch.equal(v0, v1)
+
+
+@pytest.mark.gpu
+def test_k8192_output_smem():
+    """k up to 8192 (include/cusfft.h limit): the output selection's shared
+    memory (205 KB at kp2 = 8192) fits; the plan runs and recovers a planted signal."""
+    n, k = 2 ** 22, 8192
+    B = 65536
+    x, S, X = planted_signal(n, k, seed=31)
+    with Plan(n, k, B=B, L=16, seed=2) as plan:
+        locs, vals = plan.execute(torch.from_numpy(x).to(DEV))
+        torch.cuda.synchronize()
+        assert plan.status() == 0
+        got = set(locs.cpu().tolist())
+    assert len(got & set(S.tolist())) >= int(0.99 * k)
+
+
+@pytest.mark.gpu
+def test_l2_persist_opt_out():
+    """params.l2_persist = 0: a staged plan leaves the device's persisting-L2 limit alone."""
+    import gc
+    from cuda.bindings import runtime as rt
+    lim = rt.cudaLimit.cudaLimitPersistingL2CacheSize
+    gc.collect()
+    torch.cuda.synchronize()
+    before = rt.cudaDeviceGetLimit(lim)[1]
+    plan = Plan(2 ** 22, 1000, L=16, seed=1, l2_persist=0)
+    assert plan.info()["staged"]
+    assert rt.cudaDeviceGetLimit(lim)[1] == before
+    plan.close()
