@@ -226,7 +226,7 @@ int32_t cusfft_exchange_kind(cusfft_plan_t plan);
  *                 vote_threshold, max_hits, distinct 32-B sectors of x this rank's gathers
  *                 touch (the fold's DRAM floor), staged (1: address-sorted two-phase gather,
  *                 DESIGN.md §6.2), w of the location filter, number of filters (1 or 2),
- *                 fused tail (1: vote + estimation + output in one kernel), owns an NCCL
+ *                 fused tail (1: vote + estimation in one kernel), owns an NCCL
  *                 communicator (1)
  *   a, sigma, tau : int64 [L], in loop order r = 0..L-1 (NULL to skip).  sigma is
  *   the gather stride (Alg. 1's ai), a = sigma^-1 mod n, tau the offset. */
@@ -264,8 +264,8 @@ int cusfft_status(cusfft_plan_t plan);
  * otherwise executed).
  * Per-stage device times (ms) of the last execution when timing is enabled:
  * ms[0..5] = fold, B-point FFT, cutoff, vote, estimate, output (with the fused
- * tail, info[14] = 1, the vote entry holds vote + estimate + output and the
- * next two are 0); with cap >= 7,
+ * vote + estimation kernel, info[14] = 1, the vote entry holds both and the
+ * estimate entry is 0); with cap >= 7,
  * ms[6] = phase 1 of the staged fold alone (the address-ordered permute
  * gather k_stage*), -1 when the plan is not staged.  In mode 2
  * ms[0] is the whole graph and ms[1..5] are -1.  get syncs. */

@@ -34,7 +34,15 @@ struct KTraceScope {
   }
 };
 #define KTRACE(id) KTraceScope ktrace_scope_(id)
+// SM-clock stamps (cheap to read; differences only within one CTA):
+// CTRACE(slot) stores clock64() of thread 0; CTRACE_MAX(slot, cycles) keeps the largest value.
+#define CTRACE(slot) \
+  do { if (threadIdx.x == 0) g_trace[(slot)] = (unsigned long long)clock64(); } while (0)
+#define CTRACE_MAX(slot, v) \
+  do { if (threadIdx.x == 0) atomicMax(&g_trace[(slot)], (unsigned long long)(v)); } while (0)
 #else
+#define CTRACE(slot) do { } while (0)
+#define CTRACE_MAX(slot, v) do { } while (0)
 #define KTRACE(id) do { } while (0)
 #define TRACE(slot) do { } while (0)
 #define TRACE_END(slot) do { } while (0)

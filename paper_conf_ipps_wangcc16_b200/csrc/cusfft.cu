@@ -148,6 +148,7 @@ struct Filter {
   double* d_taps = nullptr;         // [R B] zero-padded past w
   double* d_taps_perm = nullptr;    // [R B] tile-permuted (fused fold + FFT pass 1 layout)
   double2* d_ghat = nullptr;        // [nb + 1] G^(q), q = -nb/2 .. nb/2
+  double2* d_ginv = nullptr;        // [nb + 1] 1 / G^(q)
 };
 
 struct cusfft_plan_s {
@@ -187,6 +188,9 @@ struct cusfft_plan_s {
   bool setaside = false;                     // holds a reference on the device's persisting-L2 set-aside
   int64_t sectors = 0;                       // distinct 32-B sectors of x gathered by this rank
   double2* d_tw = nullptr;
+  double2* d_ph_hi = nullptr;     // e^{-2 pi i (j << plo) / n}: the estimation's phase, high bits
+  double2* d_ph_lo = nullptr;     // e^{-2 pi i j / n}, j < 2^plo: low bits
+  int plo = 0;
   SlotParam* d_slots = nullptr;
   uint32_t* d_loc_sigma = nullptr;
   double2* d_u = nullptr;
@@ -196,7 +200,6 @@ struct cusfft_plan_s {
   uint32_t* d_hist = nullptr;     // [n_sel][4096] top-digit histograms (zero block)
   int* d_key_index = nullptr;     // [Lg] local slot -> selection index or -1
   uint32_t* d_ohist = nullptr;    // [4096] top-digit histogram of the output keys (zero block)
-  unsigned* d_tail_done = nullptr;  // finished-CTA counter of k_tail (zero block)
   bool sel_cluster = false;       // k_select_cluster (256 <= B <= 65536, EXACT / THRESHOLD modes)
   int select1_smem = 0;
   // fused vote + estimate + output (k_tail) when its table fits shared memory
@@ -210,7 +213,7 @@ struct cusfft_plan_s {
   uint64_t* d_hit_keys = nullptr;
   double2* d_per_loop = nullptr;
   int* d_zero = nullptr;   // per-execution block, zeroed by the first kernel of each execution:
-  int nzero = 0;           //   flags[8] | hist0[n_sel][4096] | ohist[4096] | tail counter [4] | pk
+  int nzero = 0;           //   flags[8] | hist0[n_sel][4096] | ohist[4096] | pad [4] | pk
   int* d_flags = nullptr;  // [0] hit_count (unsigned), [1] overflow, [2] select mismatch, [3] output mismatch
   double2* d_xbuf = nullptr;
   int64_t* d_locs_buf = nullptr;
@@ -302,8 +305,9 @@ void free_plan(cusfft_plan_t p) {
     if (f.d_taps) cudaFree(f.d_taps);
     if (f.d_taps_perm) cudaFree(f.d_taps_perm);
     if (f.d_ghat) cudaFree(f.d_ghat);
+    if (f.d_ginv) cudaFree(f.d_ginv);
   }
-  void* ptrs[] = {p->d_code, p->d_row0, p->d_staging, p->d_tw, p->d_slots, p->d_loc_sigma, p->d_u, p->d_v,
+  void* ptrs[] = {p->d_code, p->d_row0, p->d_staging, p->d_tw, p->d_ph_hi, p->d_ph_lo, p->d_slots, p->d_loc_sigma, p->d_u, p->d_v,
                   p->d_records, p->d_keys, p->d_zero, p->d_key_index, p->d_hits, p->d_hit_vals, p->d_hit_keys,
                   p->d_per_loop, p->d_xbuf, p->d_locs_buf, p->d_vals_buf};
   for (void* q : ptrs)
@@ -400,6 +404,7 @@ int build_filter(cusfft_plan_t P, Filter& F) {
   cudaStream_t st = P->stream;
   TRY(dalloc(&F.d_taps, (size_t)padded));
   TRY(dalloc(&F.d_ghat, (size_t)P->nb + 1));
+  TRY(dalloc(&F.d_ginv, (size_t)P->nb + 1));
   if (q.taps) {
     CK(cudaMemsetAsync(F.d_taps, 0, (size_t)padded * sizeof(double), st));
     CK(cudaMemcpyAsync(F.d_taps, q.taps, (size_t)w * sizeof(double), cudaMemcpyHostToDevice, st));
@@ -428,6 +433,8 @@ int build_filter(cusfft_plan_t P, Filter& F) {
     if (pj) cudaFree(pj);
   }
   k_ghat<<<(int)P->nb + 1, 256, 0, st>>>(F.d_taps, F.d_ghat, w, P->n, (int)P->nb);
+  CKL();
+  k_ginv<<<(int)((P->nb + 256) / 256), 256, 0, st>>>(F.d_ghat, F.d_ginv, (int)P->nb + 1);
   CKL();
   if (P->fused1) {  // taps_perm[rr B + cta 256 + t] = g[j(cta, t) + rr B], j = c + B2 j1
     std::vector<double> g((size_t)padded), gp((size_t)padded);
@@ -667,23 +674,21 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   P->select1_smem = 4096 * 4 + 64 * 4 + kSelCap * 12 + (int)((B + 31) / 32) * 4;
   if (!P->sel_cluster && q.cutoff_mode != CUSFFT_CUTOFF_SORT && P->select1_smem > smem_optin)
     return fail(CUSFFT_INVALID_B);
-  // ---- fused tail (vote + estimate + output): table element by L_loc, table + queues in smem
+  // ---- fused vote + estimation (k_tail): table element by L_loc, table + queues in smem
   {
     const int esz = P->Lloc <= 8 ? 1 : P->Lloc <= 16 ? 2 : 4;
     const int64_t tab = ((int64_t)B * esz + 15) & ~int64_t(15);
-    const int64_t need_vote = tab + (kTailNT / 32) * kTailQ * 2;
-    const int64_t need = std::max<int64_t>(need_vote, output_smem_total(P->kp2));
-    const char* et = std::getenv("CUSFFT_TAIL");  // CUSFFT_TAIL=0: the k_vote / k_estimate / k_output chain (tests, A/B)
-    if (need + 1024 <= smem_optin && !(et && et[0] == '0')) {
+    const int64_t need = tab + (kTailNT / 32) * kTailQ * 2;
+    const char* et = std::getenv("CUSFFT_TAIL");  // CUSFFT_TAIL=0: the k_vote / k_estimate chain (tests, A/B)
+    if (need + 8 * 1024 <= smem_optin && !(et && et[0] == '0')) {  // + k_tail's static smem (hit queue)
       P->tail_esz = esz;
       P->tail_qoff = (int)tab;
       P->tail_smem = (int)need;
-      P->tail_grid = P->sms;
     }
   }
   P->vote_smem = P->Lloc * (int)((B + 31) / 32) * 4;
   P->output_smem = output_smem_total(P->kp2);
-  if (!P->tail_esz && (P->vote_smem > smem_optin || P->output_smem > smem_optin)) return fail(CUSFFT_INVALID_B);
+  if ((!P->tail_esz && P->vote_smem > smem_optin) || P->output_smem + 1024 > smem_optin) return fail(CUSFFT_INVALID_B);
   {
     const int64_t units = (int64_t)(P->Lloc - P->T + 1) * P->num;  // k_vote: one warp per (q0, J) range
     P->vote_grid = (int)std::max<int64_t>(1, std::min<int64_t>((units + 7) / 8, (int64_t)P->sms * 4));
@@ -708,7 +713,6 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     P->d_flags = P->d_zero;
     P->d_hist = reinterpret_cast<uint32_t*>(P->d_zero + 8);
     P->d_ohist = P->d_hist + (size_t)nsel * 4096;
-    P->d_tail_done = reinterpret_cast<unsigned*>(P->d_ohist + 4096);
     if (P->pk_direct) P->d_pk = reinterpret_cast<uint32_t*>(P->d_zero + pk_off);
     if ((rc = dalloc(&P->d_key_index, (size_t)P->Lg))) return fail(rc);
     std::vector<int> kidx(P->Lg, -1);
@@ -749,10 +753,36 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     g_last_cuda_error = (int)ae;
     return fail(CUSFFT_CUDA);
   }
+  if (P->tail_esz) {  // a warp per (enumerated loop, J) unit; CTAs up to the resident limit
+    int occ = 0;
+    const bool seg = L <= 16;
+    cudaError_t oe = cudaErrorInvalidValue;
+    if (P->tail_esz == 1)
+      oe = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, seg ? k_tail<uint8_t, 16> : k_tail<uint8_t, 32>, kTailNT, P->tail_smem);
+    else if (P->tail_esz == 2)
+      oe = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, seg ? k_tail<uint16_t, 16> : k_tail<uint16_t, 32>, kTailNT, P->tail_smem);
+    else
+      oe = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, seg ? k_tail<uint32_t, 16> : k_tail<uint32_t, 32>, kTailNT, P->tail_smem);
+    if (oe != cudaSuccess || occ < 1) occ = 1;
+    cudaGetLastError();
+    const int nenum = (P->T > (P->Lloc + 1) / 2) ? P->Lloc / 2 : P->Lloc - P->T + 1;
+    const int64_t units = (int64_t)nenum * (q.cutoff_mode == CUSFFT_CUTOFF_THRESHOLD ? B : P->num);
+    const int64_t ctas = (units + kTailNT / 32 - 1) / (kTailNT / 32);
+    P->tail_grid = (int)std::max<int64_t>(1, std::min<int64_t>(ctas, (int64_t)P->sms * occ));
+  }
   for (int f = 0; f < P->nfilt; ++f)
     if ((rc = build_filter(P, P->filt[f]))) return fail(rc);
   k_twiddles<<<(int)((B + 255) / 256), 256, 0, P->stream>>>(P->d_tw, (int)B);
   if (cudaGetLastError() != cudaSuccess) return fail(CUSFFT_CUDA);
+  {  // the estimation's phase e^{-2 pi i m / n} as a product of two tables (m's high / low bits)
+    const int log2n = ilog2(n);
+    P->plo = (log2n + 1) / 2;
+    const int nhi = (int)(n >> P->plo), nlo = 1 << P->plo;
+    if ((rc = dalloc(&P->d_ph_hi, (size_t)nhi)) || (rc = dalloc(&P->d_ph_lo, (size_t)nlo))) return fail(rc);
+    k_phase_table<<<(nhi + 255) / 256, 256, 0, P->stream>>>(P->d_ph_hi, nhi, P->plo, log2n);
+    k_phase_table<<<(nlo + 255) / 256, 256, 0, P->stream>>>(P->d_ph_lo, nlo, 0, log2n);
+    if (cudaGetLastError() != cudaSuccess) return fail(CUSFFT_CUDA);
+  }
   // ---- distinct 32-B sectors (2 complex samples) of x this rank gathers (the fold's DRAM floor)
   {
     std::vector<uint64_t> bits((size_t)((n / 2 + 63) / 64), 0ull);
@@ -1049,6 +1079,7 @@ VoteArgs make_vote_args(cusfft_plan_t P) {
   va.log2B = ilog2(P->B);
   va.nmask = (uint32_t)(P->n - 1);
   va.pairs = P->T > (P->Lloc + 1) / 2 ? 1 : 0;
+  va.cnt_fixed = P->prm.cutoff_mode == CUSFFT_CUTOFF_THRESHOLD ? 0 : 1;
   va.hits = P->d_hits;
   va.hit_count = reinterpret_cast<unsigned*>(P->d_flags);
   va.max_hits = P->max_hits;
@@ -1062,9 +1093,12 @@ EstArgs make_est_args(cusfft_plan_t P) {
   ea.lay = P->lay;
   ea.slots = P->d_slots;
   ea.L = P->L;
-  ea.ghat = P->filt[0].d_ghat;
-  ea.ghat_est = P->filt[P->nfilt - 1].d_ghat;
+  ea.ginv = P->filt[0].d_ginv;
+  ea.ginv_est = P->filt[P->nfilt - 1].d_ginv;
   ea.ghat_split = P->nfilt > 1 ? P->Lloc : P->L;
+  ea.ph_hi = P->d_ph_hi;
+  ea.ph_lo = P->d_ph_lo;
+  ea.plo = P->plo;
   ea.hits = P->d_hits;
   ea.hit_count = reinterpret_cast<const unsigned*>(P->d_flags);
   ea.max_hits = P->max_hits;
@@ -1080,18 +1114,11 @@ EstArgs make_est_args(cusfft_plan_t P) {
   return ea;
 }
 
-// Steps 5 + 6 + output in one kernel (tail.cuh).
-int launch_tail(cusfft_plan_t P, int64_t* locs, double2* vals, cudaStream_t st) {
+// Steps 5 + 6 in one kernel (tail.cuh).
+int launch_tail(cusfft_plan_t P, cudaStream_t st) {
   TailArgs ta{};
   ta.v = make_vote_args(P);
   ta.e = make_est_args(P);
-  ta.k = (int)P->k;
-  ta.kp2 = P->kp2;
-  ta.log2n = ilog2(P->n);
-  ta.locs = locs;
-  ta.vals = vals;
-  ta.status = P->d_flags + 1;
-  ta.done = P->d_tail_done;
   ta.q_off = P->tail_qoff;
   const bool seg = P->L <= 16;
   const dim3 g((unsigned)P->tail_grid), b(kTailNT);
@@ -1107,39 +1134,36 @@ int launch_tail(cusfft_plan_t P, int64_t* locs, double2* vals, cudaStream_t st) 
   return CUSFFT_SUCCESS;
 }
 
-// The chain k_vote -> k_estimate* -> k_output (plans whose vote table does not fit shared memory).
-int launch_vote_chain(cusfft_plan_t P, int64_t* locs, double2* vals, cudaStream_t st) {
-  CK(launch_k(k_vote, dim3(P->vote_grid), dim3(256), P->vote_smem, st, P->cur_prio, make_vote_args(P)));
-  mark(P, 4);
-  if (P->stage_limit < 5) return CUSFFT_SUCCESS;
-  const EstArgs ea = make_est_args(P);
-  if (P->L <= 8)
-    CK(launch_k(k_estimate_seg<8>, dim3(P->est_grid), dim3(256), 0, st, P->cur_prio, ea));
-  else if (P->L <= 16)
-    CK(launch_k(k_estimate_seg<16>, dim3(P->est_grid), dim3(256), 0, st, P->cur_prio, ea));
-  else
-    CK(launch_k(k_estimate, dim3(P->est_grid), dim3(256), 0, st, P->cur_prio, ea));
-  mark(P, 5);
+// Steps 5-6 (the fused k_tail, or the chain k_vote -> k_estimate* for plans
+// whose vote table does not fit shared memory) and the output (stage limits 4..6).
+int launch_after_cutoff(cusfft_plan_t P, int64_t* locs, double2* vals, cudaStream_t st) {
+  if (P->stage_limit < 4) return CUSFFT_SUCCESS;
+  if (P->tail_esz) {
+    TRY(launch_tail(P, st));
+    mark(P, 4);
+    mark(P, 5);
+  } else {
+    CK(launch_k(k_vote, dim3(P->vote_grid), dim3(256), P->vote_smem, st, P->cur_prio, make_vote_args(P)));
+    mark(P, 4);
+    if (P->stage_limit < 5) return CUSFFT_SUCCESS;
+    const EstArgs ea = make_est_args(P);
+    g_pdl = P->timing != 1;
+    if (P->L <= 8)
+      CK(launch_k(k_estimate_seg<8>, dim3(P->est_grid), dim3(256), 0, st, P->cur_prio, ea));
+    else if (P->L <= 16)
+      CK(launch_k(k_estimate_seg<16>, dim3(P->est_grid), dim3(256), 0, st, P->cur_prio, ea));
+    else
+      CK(launch_k(k_estimate, dim3(P->est_grid), dim3(256), 0, st, P->cur_prio, ea));
+    mark(P, 5);
+  }
   if (P->stage_limit < 6) return CUSFFT_SUCCESS;
+  g_pdl = P->timing != 1;
   CK(launch_k(k_output, dim3(1), dim3(1024), P->output_smem, st, P->cur_prio, (const int*)P->d_hits,
               reinterpret_cast<const unsigned*>(P->d_flags), P->max_hits, (const double2*)P->d_hit_vals,
               (const uint64_t*)P->d_hit_keys, P->d_ohist, (int)P->k, P->kp2, ilog2(P->n), locs, vals,
               P->d_flags + 1));
   mark(P, 6);
   return CUSFFT_SUCCESS;
-}
-
-// Steps 5-6 and the output (stage limits 4..6).
-int launch_after_cutoff(cusfft_plan_t P, int64_t* locs, double2* vals, cudaStream_t st) {
-  if (P->stage_limit < 4) return CUSFFT_SUCCESS;
-  if (P->tail_esz) {
-    TRY(launch_tail(P, locs, vals, st));
-    mark(P, 4);
-    mark(P, 5);
-    mark(P, 6);
-    return CUSFFT_SUCCESS;
-  }
-  return launch_vote_chain(P, locs, vals, st);
 }
 
 // Steps 1-4 of this rank's loops, one serial chain on P->stream.
@@ -1740,7 +1764,7 @@ int32_t cusfft_launches_per_execute(cusfft_plan_t plan) {
   const bool branched = use_branches(plan);
   int n = (plan->staged ? 1 : 0) + ranges /*fold per slot range*/ +
           (branched ? ranges : 1) * (pass1 ? 2 : 1) /*fft*/ + (plan->sel_slots_h.empty() ? 0 : 1) +
-          (plan->xshard && !plan->sel_slots_h.empty() ? 1 : 0) /*keys*/ + (plan->tail_esz ? 1 : 3);
+          (plan->xshard && !plan->sel_slots_h.empty() ? 1 : 0) /*keys*/ + (plan->tail_esz ? 2 : 3);
   return n;
 }
 

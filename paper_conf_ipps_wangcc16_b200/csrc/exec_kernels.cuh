@@ -1016,12 +1016,13 @@ struct VoteArgs {
   uint32_t aa[kMaxLoc];          // a = sigma^-1
   const uint32_t* loc_sigma;     // the same sigmas in global memory (register-resident loads)
   int Lloc, T, num, B, nb, log2nb, log2n, log2B;
-  int pairs;  // k_vote8: pair enumeration (T > ceil(L_loc / 2))
+  int pairs;      // pair enumeration (T > ceil(L_loc / 2))
+  int cnt_fixed;  // every winner list holds exactly num buckets (EXACT / SORT cutoffs)
   uint32_t nmask;
   int* hits;
   unsigned* hit_count;
   int max_hits;
-  const uint32_t* pk;  // k_vote8: the byte-per-bucket array already built by the cutoff (or null: transpose bmp)
+  const uint32_t* pk;  // k_tail: the vote table already built by the cutoff (or null: transpose bmp)
 };
 
 // Scaled arithmetic: with F = f << (32 - log2 n), sigma * F + (nb/2 << (32 - log2 n))
@@ -1248,9 +1249,12 @@ struct EstArgs {
   RecLayout lay;
   const SlotParam* slots;
   int L;
-  const double2* ghat;      // G^ of the location loops' filter, q = -nb/2 .. nb/2
-  const double2* ghat_est;  // G^ of loops r >= ghat_split (the estimation-only filter)
+  const double2* ginv;      // 1 / G^(q) of the location loops' filter, q = -nb/2 .. nb/2 (plan time)
+  const double2* ginv_est;  // the same for loops r >= ghat_split (the estimation-only filter)
   int ghat_split;           // L_loc with separate filters, else L
+  const double2* ph_hi;     // e^{-2 pi i (j << plo) / n}, j < n >> plo   (plan time)
+  const double2* ph_lo;     // e^{-2 pi i j / n}, j < 2^plo
+  int plo;
   const int* hits;
   const unsigned* hit_count;
   int max_hits;
@@ -1264,6 +1268,12 @@ struct EstArgs {
 };
 
 
+// v_l = u^_l[h] e^{-2 pi i tau_l f / n} / G^(-d) (Alg. 5 L311-L325 with the
+// permutation's phase removed [Z4]).  The phase e^{-2 pi i m / n}, m = tau f
+// mod n, is the product of two plan-time table entries (m's high and low
+// bits, each computed by sincospi of an exact fraction) and the division by
+// G^ a multiplication by its plan-time reciprocal: every load of the
+// estimate is independent, so its latency is one L2 round trip.
 __device__ __forceinline__ double2 loop_estimate(const EstArgs& A, const SlotParam& sp, int l, uint32_t f) {
   const uint32_t p = (sp.sigma * f) & A.nmask;
   int hb = (int)(p >> A.log2nb);
@@ -1272,15 +1282,15 @@ __device__ __forceinline__ double2 loop_estimate(const EstArgs& A, const SlotPar
     hb = (hb + 1) & (A.B - 1);
     d -= A.nb;
   }
-  const double2 g = __ldg((sp.loop < (uint32_t)A.ghat_split ? A.ghat : A.ghat_est) + (A.nb >> 1) - d);  // G^(-d)
-  const double2 b = __ldg(reinterpret_cast<const double2*>(A.records + (int64_t)l * A.lay.rec_bytes) + hb);
   const uint32_t tph = (sp.tau * f) & A.nmask;
-  double sn, cs;
-  sincospi(2.0 * (double)tph / A.n, &sn, &cs);
-  const double zr = b.x * cs + b.y * sn;  // b * e^{-i phi}
-  const double zi = b.y * cs - b.x * sn;
-  const double den = g.x * g.x + g.y * g.y;
-  return make_double2((zr * g.x + zi * g.y) / den, (zi * g.x - zr * g.y) / den);
+  const double2 gi = __ldg((sp.loop < (uint32_t)A.ghat_split ? A.ginv : A.ginv_est) + (A.nb >> 1) - d);  // 1 / G^(-d)
+  const double2 b = __ldg(reinterpret_cast<const double2*>(A.records + (int64_t)l * A.lay.rec_bytes) + hb);
+  const double2 e1 = __ldg(A.ph_hi + (tph >> A.plo));
+  const double2 e0 = __ldg(A.ph_lo + (tph & ((1u << A.plo) - 1u)));
+  const double2 ph = make_double2(e1.x * e0.x - e1.y * e0.y, e1.x * e0.y + e1.y * e0.x);
+  const double zr = b.x * ph.x - b.y * ph.y;  // b * e^{-i phi}
+  const double zi = b.x * ph.y + b.y * ph.x;
+  return make_double2(zr * gi.x - zi * gi.y, zr * gi.y + zi * gi.x);
 }
 
 // Element of rank `med` among the L values held as (lane: a0 = slot lane,

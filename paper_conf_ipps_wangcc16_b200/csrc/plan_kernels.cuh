@@ -140,4 +140,26 @@ __global__ void __launch_bounds__(256) k_ghat(const double* __restrict__ taps, d
   }
 }
 
+// Estimation tables (Alg. 5's filter_freq division and the phase of Def. 1):
+// ginv[q] = 1 / G^(q) (complex reciprocal, q = -nb/2 .. nb/2, entry q + nb/2).
+__global__ void k_ginv(const double2* __restrict__ ghat, double2* ginv, int m) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < m) {
+    const double2 g = ghat[i];
+    const double den = g.x * g.x + g.y * g.y;
+    ginv[i] = make_double2(g.x / den, -g.y / den);
+  }
+}
+
+// e^{-2 pi i m / n} for m = j << shift, j < count (the exact fraction m / n
+// = j / 2^(log2n - shift) handed to sincospi).
+__global__ void k_phase_table(double2* tab, int count, int shift, int log2n) {
+  const int j = blockIdx.x * blockDim.x + threadIdx.x;
+  if (j < count) {
+    double s, c;
+    sincospi(2.0 * ldexp((double)j, shift - log2n), &s, &c);
+    tab[j] = make_double2(c, -s);
+  }
+}
+
 }  // namespace cusfft

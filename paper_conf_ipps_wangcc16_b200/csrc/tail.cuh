@@ -4,7 +4,7 @@
 //   Step 6  median estimation        PAPER.md:L95, Alg. 5
 //   output  k strongest, by f        PAPER.md:L13 (k large coefficients), Alg. 5
 //
-// One CTA of 1024 threads per SM.  Every CTA holds the location loops' cutoff
+// CTAs of 256 threads, several per SM.  Every CTA holds the location loops' cutoff
 // results as one table element per bucket (bit q = bucket kept in location
 // loop q; uint8_t for L_loc <= 8, uint16_t <= 16, uint32_t <= 32) in shared
 // memory, copied from the array the cluster cutoff ORs its winners into or
@@ -35,9 +35,9 @@
 // element of rank floor((L-1)/2) of the real and of the imaginary parts (L95,
 // Alg. 5; ties by slot).
 //
-// Output (fused): the last CTA to finish (threadfence + counter) selects the
-// k hits of largest |val|^2 (ties to the smaller f) and writes them sorted by
-// f (output_body, shared with the stand-alone k_output).
+// Output: k_output (one CTA of 1024 threads, launched programmatically after
+// k_tail) selects the k hits of largest |val|^2 (ties to the smaller f) and
+// writes them sorted by f.
 #pragma once
 #include "exec_kernels.cuh"
 
@@ -45,16 +45,11 @@ namespace cusfft {
 
 struct TailArgs {
   VoteArgs v;          // location loops in vote order: bitmaps, winner lists, sigma, a (pk: ET table or null)
-  EstArgs e;           // every slot: records, slot params, G^, hit buffers, output-key histogram
-  int k, kp2, log2n;
-  int64_t* locs;
-  double2* vals;
-  int* status;         // d_flags + 1
-  unsigned* done;      // finished-CTA counter (per-execution zero block)
+  EstArgs e;           // every slot: records, slot params, 1/G^, phase tables, hit buffers, output-key histogram
   int q_off;           // byte offset of the per-warp queues in dynamic smem
 };
 
-constexpr int kTailNT = 1024;
+constexpr int kTailNT = 256;  // threads per CTA (several CTAs per SM: a CTA waits only for its own 8 warps)
 constexpr int kTailQ = 1024;  // per-warp queue entries (u16 candidate offsets): one whole chunk
 
 // Output selection (Alg. 5 L333-L335 emits all hits, the k
@@ -85,42 +80,42 @@ __device__ void output_body(uint8_t* smem, const int* __restrict__ hits, const u
   uint64_t* srt = sel + kp2;                                     // bucket-sorted copy
   int* bcnt = reinterpret_cast<int*>(srt + kp2);                 // 1024 bucket counters
   int* bstart = bcnt + 1024;                                     // 1024 bucket starts
-  const int tid = threadIdx.x;
-  TRACE(50);
-  // the level-0 histogram through L2 into shared memory (other CTAs of k_tail
-  // counted into it; it is the selection's read-only level 0 from here on)
+  const int tid = threadIdx.x, lane = tid & 31;
+  CTRACE(80);
+  // Every load of the fast path is issued before the first barrier: the
+  // hit count, the level-0 histogram (other CTAs of k_tail counted into it;
+  // copied to shared memory) and up to PF items per thread (keys, f, values),
+  // read speculatively below max_hits and masked once H is known.
+  constexpr int PF = 4;  // fast path: H <= PF * 1024 items, kp2 <= 1024
   uint32_t* h0 = reinterpret_cast<uint32_t*>(smem + output_smem_bytes(kp2));
-  for (int i = tid; i < 4096; i += 1024) h0[i] = __ldcg(ghist + i);
-  ghist = h0;
-  __syncthreads();
-  const unsigned hc = __ldcg(hit_count);
-  const int H = min((int)hc, max_hits);
-  if (tid == 0 && (int)hc > max_hits) atomicOr(status, 1);
-  const int K = min(k, H);
-  // Fast path (H <= 16384 items, k <= 2048): every item's key, f and value
-  // are loaded into registers while the level-0 boundary bin is found; if that
-  // bin is taken whole (the usual case: the k planted coefficients stand far
-  // above the false hits), one classification pass selects, and the values go
-  // to shared memory (aliasing the unused candidate arrays).
-  constexpr int PF = 4, NCH = 4;  // items per thread per chunk, chunks
   double2* selv = reinterpret_cast<double2*>(ckey);  // [kp2] values of the selected entries (fast path)
-  const bool fast = H <= NCH * PF * 1024 && kp2 * 16 <= kOutCap * 12;
+  const unsigned hc = __ldcg(hit_count);
+  uint32_t hb[4];
+#pragma unroll
+  for (int j = 0; j < 4; ++j) hb[j] = __ldcg(ghist + tid + j * 1024);
   uint64_t pk[PF];
   uint32_t pf[PF];
   double2 pv[PF];
-  if (fast) {  // chunk 0: keys, f and values
 #pragma unroll
-    for (int u = 0; u < PF; ++u) {
-      const int i = u * 1024 + tid;
-      if (i < H) {
-        pk[u] = __ldcg(hit_keys + i);
-        pf[u] = (uint32_t)__ldcg(hits + i);
-        pv[u] = __ldcg(hit_vals + i);
-      }
+  for (int u = 0; u < PF; ++u) {
+    const int i = u * 1024 + tid;
+    if (i < max_hits) {
+      pk[u] = __ldcg(hit_keys + i);
+      pf[u] = (uint32_t)__ldcg(hits + i);
+      pv[u] = __ldcg(hit_vals + i);
     }
   }
+#pragma unroll
+  for (int j = 0; j < 4; ++j) h0[tid + j * 1024] = hb[j];
+  ghist = h0;
+  const int H = min((int)hc, max_hits);
+  if (tid == 0 && (int)hc > max_hits) atomicOr(status, 1);
+  const int K = min(k, H);
+  const bool fast = H <= PF * 1024 && kp2 <= 1024;
   if (tid == 0) sm[41] = 0;
   bcnt[tid] = 0;
+  __syncthreads();
+  CTRACE(81);
   bool direct = false;  // selv holds the values
   if (fast) {
     uint32_t d0 = 0;
@@ -129,44 +124,33 @@ __device__ void output_body(uint8_t* smem, const int* __restrict__ hits, const u
       const BinPick b0 = pick_bin(ghist, K, sm);  // syncs
       d0 = (uint32_t)b0.d;
       whole = (K - b0.above) == b0.cnt;
-    } else {
-      __syncthreads();
     }
-    if (whole) {
+    CTRACE(82);
+    if (whole) {  // the boundary bin is taken whole: selected = digit >= d0; positions by one block scan
       direct = true;
-      const int lane = tid & 31;
-      for (int ch = 0; ch < NCH && ch * PF * 1024 < H; ++ch) {  // block-uniform
-        if (ch > 0) {  // later chunks (many false hits): keys and f here, values only for the selected
+      bool take[PF];
+      int cnt = 0;
 #pragma unroll
-          for (int u = 0; u < PF; ++u) {
-            const int i = ch * PF * 1024 + u * 1024 + tid;
-            if (i < H) {
-              pk[u] = __ldcg(hit_keys + i);
-              pf[u] = (uint32_t)__ldcg(hits + i);
-            }
-          }
-        }
+      for (int u = 0; u < PF; ++u) {
+        const int i = u * 1024 + tid;
+        take[u] = i < H && ((uint32_t)(pk[u] >> 51) & 0xFFFu) >= d0;
+        cnt += take[u];
+      }
+      int total;
+      int pos = block_excl_scan<1024>(cnt, &total, sm);
 #pragma unroll
-        for (int u = 0; u < PF; ++u) {
-          const int i = ch * PF * 1024 + u * 1024 + tid;
-          const bool take = i < H && ((uint32_t)(pk[u] >> 51) & 0xFFFu) >= d0;
-          const unsigned bal = __ballot_sync(kFull, take);
-          int base = 0;
-          if (lane == 0 && bal) base = atomicAdd(&sm[41], __popc(bal));
-          base = __shfl_sync(kFull, base, 0);
-          if (take) {
-            const int pos = base + __popc(bal & ((1u << lane) - 1u));
-            if (pos < kp2) {
-              sel[pos] = ((uint64_t)pf[u] << 32) | (uint32_t)pos;
-              selv[pos] = ch == 0 ? pv[u] : __ldcg(hit_vals + i);
-            }
+      for (int u = 0; u < PF; ++u) {
+        if (take[u]) {
+          if (pos < kp2) {
+            sel[pos] = ((uint64_t)pf[u] << 32) | (uint32_t)pos;
+            selv[pos] = pv[u];
           }
+          ++pos;
         }
       }
+      if (tid == 0) sm[41] = total;
       __syncthreads();
     }
-  } else {
-    __syncthreads();
   }
   if (!direct) {
     auto add = [&](int i) {
@@ -186,27 +170,34 @@ __device__ void output_body(uint8_t* smem, const int* __restrict__ hits, const u
       __syncthreads();
     }
   }
-  TRACE(51);
+  CTRACE(83);
   const int ns = min(sm[41], kp2);
   if (tid == 0 && sm[41] != K) atomicOr(status + 2, 1);
-  // bucket sort by the top 10 bits of f
+  // bucket sort by the top 10 bits of f: an item's rank inside its bucket is
+  // the counter value its atomic returns; one scan places the buckets
   const int sh = max(0, log2n - 10);
-  for (int i = tid; i < ns; i += 1024) atomicAdd(&bcnt[(int)(sel[i] >> 32) >> sh], 1);
+  int rnk[8];  // kp2 <= 8192: at most 8 items per thread
+#pragma unroll
+  for (int u = 0; u < 8; ++u) {
+    const int i = tid + u * 1024;
+    if (i < ns) rnk[u] = atomicAdd(&bcnt[(int)(sel[i] >> 32) >> sh], 1);
+  }
   __syncthreads();
   const int c = bcnt[tid];
   int total;
   const int st = block_excl_scan<1024>(c, &total, sm);
   bstart[tid] = st;
+  const int cmax = __reduce_max_sync(kFull, c);
   if (tid == 0) sm[42] = 0;
   __syncthreads();
-  atomicMax(&sm[42], c);
-  bcnt[tid] = 0;
-  __syncthreads();
-  for (int i = tid; i < ns; i += 1024) {
-    const int bkt = (int)(sel[i] >> 32) >> sh;
-    srt[bstart[bkt] + atomicAdd(&bcnt[bkt], 1)] = sel[i];
+  if (lane == 0) atomicMax(&sm[42], cmax);
+#pragma unroll
+  for (int u = 0; u < 8; ++u) {
+    const int i = tid + u * 1024;
+    if (i < ns) srt[bstart[(int)(sel[i] >> 32) >> sh] + rnk[u]] = sel[i];
   }
   __syncthreads();
+  CTRACE(84);
   if (sm[42] <= 32) {
     const int b0 = bstart[tid];
     for (int i = 1; i < c; ++i) {  // insertion sort of this thread's bucket
@@ -238,7 +229,7 @@ __device__ void output_body(uint8_t* smem, const int* __restrict__ hits, const u
     }
   }
   __syncthreads();
-  TRACE(52);
+  CTRACE(85);
   for (int j = tid; j < k; j += 1024) {
     if (j < ns) {
       const uint64_t v = srt[j];
@@ -249,7 +240,7 @@ __device__ void output_body(uint8_t* smem, const int* __restrict__ hits, const u
       vals[j] = make_double2(0.0, 0.0);
     }
   }
-  TRACE(53);
+  CTRACE(86);
 }
 
 // Stand-alone output kernel (the fallback chain: k_vote / k_estimate* / k_output).
@@ -265,34 +256,108 @@ __global__ void __launch_bounds__(1024) k_output(const int* __restrict__ hits, c
 }
 
 
-// Estimate the hits of one finish round (hit: this lane's candidate is a hit,
-// f its frequency).  Warp-uniform control flow; all 32 lanes call it.
-// LP = 16: a 16-lane segment per hit, lane li = slot li (L <= 16);
-// LP = 32: a warp per hit, lanes hold slots li and li + 32 (L <= 64).
+// Step 6 for the hit each lane segment holds (frequency hf; valid = it
+// exists).  LP = 16: a 16-lane segment per hit, lane li = slot li (L <= 16);
+// LP = 32: one hit per warp, lanes hold slots li and li + 32 (L <= 64).
+// Per-loop values stay in v0 / v1, the median in (vr, vi).  Warp-uniform.
 template <int LP>
-__device__ __forceinline__ void tail_emit_estimate(const TailArgs& A, bool hit, uint32_t f, const SlotParam& sp0,
-                                                   const SlotParam& sp1) {
+__device__ __forceinline__ void tail_estimate(const EstArgs& E, uint32_t hf, bool valid, const SlotParam& sp0,
+                                              const SlotParam& sp1, double& vr, double& vi, double2& v0,
+                                              double2& v1) {
   const int lane = threadIdx.x & 31;
-  unsigned hb = __ballot_sync(kFull, hit);
-  if (!hb) return;
-  unsigned base = 0;
-  const int leader = __ffs(hb) - 1;
-  if (lane == leader) base = atomicAdd(A.v.hit_count, (unsigned)__popc(hb));
-  base = __shfl_sync(kFull, base, leader);
-  const unsigned myslot = base + __popc(hb & ((1u << lane) - 1u));
-  if (hit && (int)myslot < A.v.max_hits) A.v.hits[myslot] = (int)f;
-  const EstArgs& E = A.e;
   const int L = E.L;
   const int med = (L - 1) >> 1;
-  constexpr int G = 32 / LP;  // hits per step
-  while (hb) {  // warp-uniform
+  const int seg = lane / LP, li = lane % LP;
+  v0 = make_double2(0.0, 0.0);
+  v1 = make_double2(0.0, 0.0);
+  if (LP == 16) {
+    const unsigned segmask = 0xFFFFu << (seg * 16);
+    const bool act = li < L;
+    if (valid && act) v0 = loop_estimate(E, sp0, li, hf);
+#pragma unroll
+    for (int part = 0; part < 2; ++part) {
+      const double a = part ? v0.y : v0.x;
+      int r = 0;
+#pragma unroll
+      for (int j = 0; j < 16; ++j) {
+        const double b = __shfl_sync(kFull, a, seg * 16 + j);
+        r += (j < L) && ((b < a) || (b == a && j < li));
+      }
+      const unsigned bal = __ballot_sync(kFull, act && r == med) & segmask;
+      const int from = bal ? __ffs(bal) - 1 : seg * 16;
+      const double m = __shfl_sync(kFull, a, from);
+      if (part) vi = m; else vr = m;
+    }
+  } else {
+    if (valid) {
+      if (lane < L) v0 = loop_estimate(E, sp0, lane, hf);
+      if (lane + 32 < L) v1 = loop_estimate(E, sp1, lane + 32, hf);
+    }
+    vr = warp_rank_select(v0.x, v1.x, L, med);
+    vi = warp_rank_select(v0.y, v1.y, L, med);
+  }
+}
+
+// Results of tail_estimate for hit-list position hs (valid: hs < max_hits).
+template <int LP>
+__device__ __forceinline__ void tail_store(const EstArgs& E, unsigned hs, bool valid, double vr, double vi,
+                                           const double2& v0, const double2& v1) {
+  if (!valid) return;
+  const int lane = threadIdx.x & 31;
+  const int L = E.L, li = lane % LP;
+  if (E.per_loop) {
+    if (LP == 16) {
+      if (li < L) E.per_loop[(int64_t)hs * L + li] = v0;
+    } else {
+      if (lane < L) E.per_loop[(int64_t)hs * L + lane] = v0;
+      if (lane + 32 < L) E.per_loop[(int64_t)hs * L + lane + 32] = v1;
+    }
+  }
+  if (li == 0) {
+    const uint64_t key = (uint64_t)__double_as_longlong(__dadd_rn(__dmul_rn(vr, vr), __dmul_rn(vi, vi)));
+    E.hit_vals[hs] = make_double2(vr, vi);
+    E.hit_keys[hs] = key;
+    atomicAdd(E.out_hist + ((uint32_t)(key >> 51) & 0xFFFu), 1u);
+  }
+}
+
+// Hits of one finish round (hit: this lane's candidate is a hit, f its
+// frequency): queued in the CTA's shared list (estimated by the whole CTA
+// after its vote), or -- when that list is full -- given their hit-list
+// positions and estimated by this warp at once.
+constexpr int kTailHQ = 1024;  // CTA hit-queue capacity
+
+template <int LP>
+__device__ __forceinline__ void tail_emit(const TailArgs& A, bool hit, uint32_t f, uint32_t* hq, int* nq,
+                                          const SlotParam& sp0, const SlotParam& sp1) {
+  const int lane = threadIdx.x & 31;
+  const unsigned hb = __ballot_sync(kFull, hit);
+  if (!hb) return;
+  const int leader = __ffs(hb) - 1;
+  const unsigned rank = __popc(hb & ((1u << lane) - 1u));
+  int qpos = 0;
+  if (lane == leader) qpos = atomicAdd(nq, __popc(hb));
+  qpos = __shfl_sync(kFull, qpos, leader);
+  if (qpos + __popc(hb) <= kTailHQ) {  // warp-uniform
+    if (hit) hq[qpos + rank] = f;
+    return;
+  }
+  if (lane == leader) atomicSub(nq, __popc(hb));  // overflow: this warp places and estimates them itself
+  unsigned base = 0;
+  if (lane == leader) base = atomicAdd(A.v.hit_count, (unsigned)__popc(hb));
+  base = __shfl_sync(kFull, base, leader);
+  const unsigned myslot = base + rank;
+  if (hit && (int)myslot < A.v.max_hits) A.v.hits[myslot] = (int)f;
+  constexpr int G = 32 / LP;
+  unsigned rem = hb;
+  while (rem) {  // warp-uniform
     int src[G];
 #pragma unroll
     for (int g = 0; g < G; ++g) {
-      src[g] = hb ? __ffs(hb) - 1 : -1;
-      if (hb) hb &= hb - 1;
+      src[g] = rem ? __ffs(rem) - 1 : -1;
+      if (rem) rem &= rem - 1;
     }
-    const int seg = lane / LP, li = lane % LP;
+    const int seg = lane / LP;
     int s = src[0];
 #pragma unroll
     for (int g = 1; g < G; ++g)
@@ -301,47 +366,9 @@ __device__ __forceinline__ void tail_emit_estimate(const TailArgs& A, bool hit, 
     const unsigned hs = __shfl_sync(kFull, myslot, s < 0 ? 0 : s);
     const bool valid = s >= 0 && (int)hs < A.v.max_hits;
     double vr, vi;
-    if (LP == 16) {
-      const unsigned segmask = 0xFFFFu << (seg * 16);
-      const bool act = li < L;
-      double2 v = make_double2(0.0, 0.0);
-      if (valid && act) {
-        v = loop_estimate(E, sp0, li, hf);
-        if (E.per_loop) E.per_loop[(int64_t)hs * L + li] = v;
-      }
-#pragma unroll
-      for (int part = 0; part < 2; ++part) {
-        const double a = part ? v.y : v.x;
-        int r = 0;
-#pragma unroll
-        for (int j = 0; j < 16; ++j) {
-          const double b = __shfl_sync(kFull, a, seg * 16 + j);
-          r += (j < L) && ((b < a) || (b == a && j < li));
-        }
-        const unsigned bal = __ballot_sync(kFull, act && r == med) & segmask;
-        const int from = bal ? __ffs(bal) - 1 : seg * 16;
-        const double m = __shfl_sync(kFull, a, from);
-        if (part) vi = m; else vr = m;
-      }
-    } else {
-      double2 v0 = make_double2(0.0, 0.0), v1 = make_double2(0.0, 0.0);
-      if (valid) {
-        if (lane < L) v0 = loop_estimate(E, sp0, lane, hf);
-        if (lane + 32 < L) v1 = loop_estimate(E, sp1, lane + 32, hf);
-        if (E.per_loop) {
-          if (lane < L) E.per_loop[(int64_t)hs * L + lane] = v0;
-          if (lane + 32 < L) E.per_loop[(int64_t)hs * L + lane + 32] = v1;
-        }
-      }
-      vr = warp_rank_select(v0.x, v1.x, L, med);
-      vi = warp_rank_select(v0.y, v1.y, L, med);
-    }
-    if (valid && li == 0) {
-      const uint64_t key = (uint64_t)__double_as_longlong(__dadd_rn(__dmul_rn(vr, vr), __dmul_rn(vi, vi)));
-      E.hit_vals[hs] = make_double2(vr, vi);
-      E.hit_keys[hs] = key;
-      atomicAdd(E.out_hist + ((uint32_t)(key >> 51) & 0xFFFu), 1u);
-    }
+    double2 v0, v1;
+    tail_estimate<LP>(A.e, hf, valid, sp0, sp1, vr, vi, v0, v1);
+    tail_store<LP>(A.e, hs, valid, vr, vi, v0, v1);
   }
 }
 
@@ -359,17 +386,27 @@ __device__ __forceinline__ uint32_t tab_at(uint32_t base, uint32_t i) {
 
 // ET: vote table element; LP: estimation lanes per hit (16 or 32).
 template <typename ET, int LP>
-__global__ void __launch_bounds__(kTailNT, 1) k_tail(TailArgs A) {
+__global__ void __launch_bounds__(kTailNT, 4) k_tail(TailArgs A) {
   pdl_wait();
   KTRACE(9);
   extern __shared__ __align__(16) uint8_t smem[];
   __shared__ uint32_t ssig[kMaxLoc], saa[kMaxLoc];
   __shared__ int scnt[kMaxLoc + 1];
-  __shared__ int s_last;
+  __shared__ int s_nq;
+  __shared__ unsigned s_base;
+  __shared__ uint32_t s_hq[kTailHQ];  // this CTA's hits (frequencies), estimated after its vote
   const VoteArgs& V = A.v;
   const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
   if (blockIdx.x == 0) TRACE(30);
   const int B = V.B, Lloc = V.Lloc;
+  const int nenum = V.pairs ? Lloc / 2 : Lloc - V.T + 1;
+  const int warp = blockIdx.x * (kTailNT / 32) + wid;
+  // the warp's first winner bucket J, loaded now so its latency overlaps the table copy
+  uint32_t Jpre = 0u;
+  if (V.cnt_fixed && warp < nenum * V.num) {
+    const int e0 = warp / V.num;
+    Jpre = (uint32_t)__ldcg(V.Jp[V.pairs ? 2 * e0 : e0] + (warp - e0 * V.num));
+  }
   // ---- the vote table: copy (the cutoff ORed the winners into V.pk) or transpose the bitmaps
   if (V.pk) {
     const int n16 = (int)(((int64_t)B * sizeof(ET) + 15) / 16);
@@ -391,13 +428,13 @@ __global__ void __launch_bounds__(kTailNT, 1) k_tail(TailArgs A) {
       }
     }
   }
-  const int nenum = V.pairs ? Lloc / 2 : Lloc - V.T + 1;
   if (tid < Lloc) {
     ssig[tid] = V.sig[tid];
     saa[tid] = V.aa[tid];
   }
   if (tid == 0) {
     int acc = 0;
+    s_nq = 0;
     scnt[0] = 0;
     for (int e = 0; e < nenum; ++e) {
       acc += __ldcg(V.cntp[V.pairs ? 2 * e : e]);
@@ -413,6 +450,9 @@ __global__ void __launch_bounds__(kTailNT, 1) k_tail(TailArgs A) {
   }
   __syncthreads();
   if (blockIdx.x == 0) TRACE(31);
+#ifdef CUSFFT_TRACE
+  const long long c_vote0 = clock64();
+#endif
   uint32_t tab_s;
   asm volatile("mov.u32 %0, %1;" : "=r"(tab_s) : "r"(smem_u32(smem)));
   uint16_t* q = reinterpret_cast<uint16_t*>(smem + A.q_off) + wid * kTailQ;
@@ -420,13 +460,12 @@ __global__ void __launch_bounds__(kTailNT, 1) k_tail(TailArgs A) {
   const uint32_t nb = (uint32_t)V.nb, half = nb >> 1;
   const uint32_t half_s = half << sh;
   const int units = scnt[nenum];
-  const int warp = blockIdx.x * (kTailNT / 32) + wid;
   const int nwarps = gridDim.x * (kTailNT / 32);
   for (int unit = warp; unit < units; unit += nwarps) {  // warp-uniform
     int e = 0;
     while (unit >= scnt[e + 1]) ++e;
     const int eq = V.pairs ? 2 * e : e;  // enumerated loop
-    const uint32_t J = (uint32_t)__ldcg(V.Jp[eq] + (unit - scnt[e]));
+    const uint32_t J = (V.cnt_fixed && unit == warp) ? Jpre : (uint32_t)__ldcg(V.Jp[eq] + (unit - scnt[e]));
     const uint32_t a = saa[eq];
     const uint32_t p0 = J * nb - half;  // first preimage of J (mod n via the scaled arithmetic below)
     // mandatory probes: pairs -> loop eq + 1; else loops e + 1 .. e + m with <= allowed misses
@@ -490,23 +529,50 @@ __global__ void __launch_bounds__(kTailNT, 1) k_tail(TailArgs A) {
             hit = __popc(bits) >= V.T && (bits & ((1u << e) - 1u)) == 0u;
           }
         }
-        tail_emit_estimate<LP>(A, hit, f, sp0, sp1);
+        tail_emit<LP>(A, hit, f, s_hq, &s_nq, sp0, sp1);
       }
       __syncwarp();
     }
   }
-  // ---- the last CTA to finish selects the output
+  // ---- Step 6 for this CTA's queued hits: one block of hit-list positions,
+  // then 32 / LP hits per warp per pass
+  pdl_launch_dependents();  // the output kernel may become resident as CTAs drain
+  TRACE_END(33);  // (trace builds) latest end of a CTA's vote
+#ifdef CUSFFT_TRACE
+  CTRACE_MAX(70, clock64() - c_vote0);  // longest warp-0 vote (cycles)
+#endif
+  // (the first pass is computed while thread 0's reservation of hit-list
+  // positions is in flight; it is stored once the base is known)
   __syncthreads();
-  if (tid == 0) {
-    __threadfence();
-    s_last = atomicAdd(A.done, 1u) == gridDim.x - 1;
+#ifdef CUSFFT_TRACE
+  const long long c_est0 = clock64();
+  CTRACE_MAX(71, c_est0 - c_vote0);  // longest CTA vote incl. its barrier (cycles)
+#endif
+  const int nq = s_nq;
+  if (tid == 0 && nq > 0) s_base = atomicAdd(V.hit_count, (unsigned)nq);
+  constexpr int G = 32 / LP;
+  constexpr int PASS = (kTailNT / 32) * G;  // hits per CTA pass
+  const int h1 = wid * G + lane / LP;
+  double vr = 0.0, vi = 0.0;
+  double2 v0, v1;
+  if (wid * G < nq)  // warp-uniform
+    tail_estimate<LP>(A.e, h1 < nq ? s_hq[h1] : 0u, h1 < nq, sp0, sp1, vr, vi, v0, v1);
+  __syncthreads();
+  if (nq > 0) {
+    const unsigned base = s_base;
+    for (int i = tid; i < nq; i += kTailNT)
+      if ((int)(base + i) < V.max_hits) V.hits[base + i] = (int)s_hq[i];
+    if (wid * G < nq) tail_store<LP>(A.e, base + (unsigned)h1, h1 < nq && (int)(base + h1) < V.max_hits, vr, vi, v0, v1);
+    for (int hh = wid * G + PASS; hh < nq; hh += PASS) {  // more than one pass of hits (warp-uniform)
+      const int h = hh + lane / LP;
+      tail_estimate<LP>(A.e, h < nq ? s_hq[h] : 0u, h < nq, sp0, sp1, vr, vi, v0, v1);
+      tail_store<LP>(A.e, base + (unsigned)h, h < nq && (int)(base + h) < V.max_hits, vr, vi, v0, v1);
+    }
   }
-  __syncthreads();
-  if (blockIdx.x == 0) TRACE(32);
-  if (!s_last) return;
-  __threadfence();
-  output_body(smem, V.hits, V.hit_count, V.max_hits, A.e.hit_vals, A.e.hit_keys, A.e.out_hist, A.k, A.kp2, A.log2n,
-              A.locs, A.vals, A.status);
+  TRACE_END(34);  // (trace builds) latest end of a CTA's estimation
+#ifdef CUSFFT_TRACE
+  CTRACE_MAX(72, clock64() - c_est0);  // longest CTA estimation (cycles)
+#endif
 }
 
 }  // namespace cusfft

@@ -40,6 +40,13 @@ for rep in range(reps):
         phases = {i: (t[i] - t0) / 1e3 for i in range(96) if t[i] > 0}
         print("phase slots (us):", " ".join(f"{i}:{v:.2f}" for i, v in sorted(phases.items(), key=lambda kv: kv[1])))
         print("select candidates per loop:", [int(t[96 + i]) & 0xFFFFFFFF for i in range(16) if t[96 + i] > 0])
+        cyc = {i: int(t[i]) for i in range(64, 96) if t[i] > 0}
+        if cyc:
+            print("tail cycles: vote(w0 max)", cyc.get(70), "vote(CTA max)", cyc.get(71), "estimate(CTA max)", cyc.get(72))
+            o = [cyc.get(i) for i in range(80, 87)]
+            if all(o):
+                print("output phases (cycles): load", o[1] - o[0], "pick", o[2] - o[1], "classify", o[3] - o[2],
+                      "count+scan+scatter", o[4] - o[3], "insertion", o[5] - o[4], "write", o[6] - o[5], "total", o[6] - o[0])
     for i, (s, e) in spans.items():
         acc.setdefault(i, []).append(((s - t0) / 1e3, (e - t0) / 1e3))
     acc.setdefault(0, []).append((0.0, (end - t0) / 1e3))
