@@ -37,6 +37,7 @@ CONFIGS = {
     "C3": (2 ** 24, 1000, 16, "n=2^24, k=1000, noiseless fp64 planted spectrum"),
     "C4": (2 ** 27, 1000, 16, "n=2^27, k=1000, noiseless fp64 planted spectrum"),
     "C5": (2 ** 22, 1000, 16, "n=2^22, k=1000, batch of 64 independent noiseless fp64 signals, signals sharded over GPUs"),
+    "C5k": (2 ** 22, 1000, 16, "n=2^22, one noiseless fp64 signal, k from --k (the k sweep 50..4096)"),
 }
 BATCH = {"C5": 64}
 # Filter and cutoff parameters per config (the paper leaves them open, DESIGN.md
@@ -50,6 +51,7 @@ FILTERS = {
     "C3": dict(tol=1e-7, lam_B=0.75),
     "C4": dict(tol=1e-8, lam_B=0.5),
     "C5": dict(tol=1e-8, lam_B=0.5),
+    "C5k": dict(tol=1e-8, lam_B=0.5),
 }
 # the library defaults (cusfft_params_default), reported beside the tuned line
 DEFAULT_FILTER = dict(tol=1e-8, lam_B=0.5)
@@ -148,9 +150,12 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
+SNR_DB = None  # --snr: additive complex white Gaussian noise (workload.planted_signal)
+
+
 def make_signal(n, k, seed):
     from paper_conf_ipps_wangcc16_b200.workload import planted_signal
-    return planted_signal(n, k, seed)
+    return planted_signal(n, k, seed, snr_db=SNR_DB)
 
 
 # ---------------------------------------------------------------------------
@@ -201,7 +206,7 @@ def run_reference(args):
         return 0
     n, k, L, desc = CONFIGS[args.config]
     from oracle import default_B
-    B = default_B(n, k)
+    B = args.B or default_B(n, k)
     x, S, X = make_signal(n, k, args.signal_seed)
     times, _, cores, core = oracle_time(args.config, n, k, L, B, x, args.plan_seed, budget_s=0,
                                         min_runs=args.warmup + args.steps, max_runs=args.warmup + args.steps)
@@ -513,7 +518,8 @@ def run_gpu(args):
                    "parallelism": f"{args.shard}-sharded x{world} (NCCL in the plan's graph)" if world > 1 else "single GPU",
                    "l2": "flushed between timed steps (256 MiB write + 256 MiB read), outside the step events; "
                          "the staging buffer's persisting lines survive it (warm); value_cold resets them too",
-                   "signal_seed": args.signal_seed, "plan_seed": args.plan_seed},
+                   "signal_seed": args.signal_seed, "plan_seed": args.plan_seed,
+                   "snr_db": SNR_DB},
         "value_cold": cold,
         "plan_ms": plan_ms,
         "gpu_launches": launches * args.steps,
@@ -675,9 +681,20 @@ def main():
     ap.add_argument("--no-default-line", action="store_true")
     ap.add_argument("--ablations", action="store_true",
                     help="also time the cutoff variants (Alg. 3 sort, Alg. 6 threshold), the direct gather, no L2 set-aside")
+    ap.add_argument("--k", type=int, default=0, help="C5k: sparsity k (the k sweep)")
+    ap.add_argument("--bcst", type=float, default=1.0, help="B = floor_pow2(bcst sqrt(n k / log2 n)) (k sweep: 2 for k >= 2000)")
+    ap.add_argument("--snr", type=float, default=None, help="additive noise SNR in dB (C4 sweep); default noiseless")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
+    global SNR_DB
+    SNR_DB = args.snr
+    if args.k:
+        n_, _, L_, d_ = CONFIGS[args.config]
+        CONFIGS[args.config] = (n_, args.k, L_, d_.replace("k from --k", f"k={args.k}"))
+    if args.bcst != 1.0 and not args.B:
+        n_, k_ = CONFIGS[args.config][:2]
+        args.B = 1 << int(math.floor(math.log2(args.bcst * math.sqrt(n_ * k_ / math.log2(n_)))))
     if args.impl == "reference":
         return run_reference(args)
     if args.config in BATCH:

@@ -123,13 +123,20 @@ typedef struct {
                               L2, else direct; 1: always the direct gather       */
 } cusfft_params;
 
-/* Fill *p with the defaults for (n, k, B).  Returns CUSFFT_NULL_PTR / INVALID_*. */
+/* Fill *p with the defaults for (n, k, B).  Returns CUSFFT_NULL_PTR / INVALID_*.
+ * Paper: the parameters of Steps 1-6 (L81-L95); the values the paper leaves
+ * open are DESIGN.md §3's readings [Z1, Z6, Z8, Z17]. */
 int cusfft_params_default(cusfft_params* p, int64_t n, int64_t k, int64_t B);
 
-/* B = floor_pow2(bcst * sqrt(n k / log2 n)) (L85, L196, L228); 0 on bad input. */
+/* B = floor_pow2(bcst * sqrt(n k / log2 n)); 0 on bad input.
+ * Paper: B = O(sqrt(nk / log n)) (L85), = sqrt(nk / log n) (L196, worked
+ * example 3,816 at n = 2^18, k = 1000), a power of 2 (L228). */
 int64_t cusfft_default_B(int64_t n, int64_t k, double bcst);
 
 /* Create a plan for length-n signals, k outputs, B buckets and L loops.
+ * Paper: the per-loop draws a <- random() mod n with gcd(a, n) = 1 and
+ * ai = a^-1 (Alg. 1, Def. 1), the flat-window filter (L25, L85)
+ * and its response G^ used by the estimation (Alg. 5).
  * p may be NULL (defaults).  Draws (a_r, sigma_r, tau_r), builds the filter
  * taps, the filter response G^(q) for |q| <= n/(2B) and the B-point twiddles
  * on the device, allocates all workspace.  Synchronous.  *out is written only
@@ -138,6 +145,8 @@ int cusfft_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L,
                 const cusfft_params* p);
 
 /* Multi-GPU plan for rank `rank` of `world` processes (one GPU each).
+ * Paper: the L loops are independent until the vote (L93) and are batched
+ * over one B-point FFT (L232); the paper itself runs on one GPU (L119, L398).
  * shard_mode 0 (loops): world must divide L; loop r is owned by rank r mod
  * world, every rank passes the whole signal; outputs are identical on every
  * rank and bit-identical to a world = 1 plan.  The exchange is an ALL-GATHER
@@ -163,17 +172,20 @@ int cusfft_plan_dist(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_
                      const cusfft_params* p, int32_t rank, int32_t world, const void* nccl_unique_id);
 
 /* Write a fresh 128-byte ncclUniqueId to out (ncclGetUniqueId).  CUSFFT_NCCL
- * when NCCL cannot be loaded. */
+ * when NCCL cannot be loaded.  Plumbing for cusfft_plan_dist (no paper passage). */
 int cusfft_nccl_unique_id(void* out);
 
 /* Release every device allocation of the plan.  Synchronises the plan's stream.
- * Destroying NULL returns CUSFFT_INVALID_PLAN. */
+ * Destroying NULL returns CUSFFT_INVALID_PLAN.  Plumbing (no paper passage). */
 int cusfft_destroy(cusfft_plan_t plan);
 
-/* Set the CUDA stream (a cudaStream_t; NULL = legacy default stream). */
+/* Set the CUDA stream (a cudaStream_t; NULL = legacy default stream).
+ * Plumbing (no paper passage); the paper overlaps work on CUDA streams (L345-L351). */
 int cusfft_set_stream(cusfft_plan_t plan, void* cuda_stream);
 
-/* The whole transform (world = 1 plans, or multi-GPU plans that own a communicator):
+/* The whole transform (world = 1 plans, or multi-GPU plans that own a communicator).
+ * Paper: Steps 1-6 (L81-L95; Alg. 1, Alg. 2, Alg. 3
+ * L238-L250, Alg. 4, Alg. 5) for the problem of L13/L77.
  *   d_x    : device, read-only, complex fp64 [n]
  *   d_locs : device, int64 [k]      output: recovered frequencies, ascending; -1 pads
  *   d_vals : device, complex fp64 [k] output: x^_f / n at d_locs; 0 pads
@@ -195,25 +207,30 @@ int cusfft_execute(cusfft_plan_t plan, const void* d_x, int64_t* d_locs, void* d
 int cusfft_execute_batch(cusfft_plan_t plan, const void* d_x, int64_t count, int64_t x_stride, int64_t* d_locs,
                          void* d_vals);
 
-/* Pipeline depth D in [1, 8] of cusfft_execute_batch: creates (or frees) D - 1
+/* Paper: none (engine scheduling); cf. the paper's concurrent streams (L345-L351).
+ * Pipeline depth D in [1, 8] of cusfft_execute_batch: creates (or frees) D - 1
  * internal clones of the plan (same parameters and draws, own workspace and
  * stream).  Synchronises the plan's stream.  cusfft_status also reports the
  * clones; cusfft_destroy frees them.  world = 1 plans only. */
 int cusfft_set_pipeline(cusfft_plan_t plan, int32_t depth);
 
-/* Same transform from HOST buffers: copies h_x [n] to a plan-owned device
+/* Paper: the transfer-inclusive timing of the PsFFT comparison (L426).
+ * Same transform from HOST buffers: copies h_x [n] to a plan-owned device
  * buffer, executes, copies k locations / values back and synchronises the
  * stream.  Pinned host memory gives asynchronous copies.  Returns the
  * cusfft_status result of the transform. */
 int cusfft_execute_host(cusfft_plan_t plan, const void* h_x, int64_t* h_locs, void* h_vals);
 
 /* Loop-sharded execution (any world): Steps 1-4 for this rank's loops, written
- * into this rank's slice of the exchange buffer. */
+ * into this rank's slice of the exchange buffer.  Paper: Steps 1-4 per loop
+ * (L81-L89), independent across loops until the vote (L93). */
 int cusfft_execute_local(cusfft_plan_t plan, const void* d_x);
 /* Steps 5-6 plus output selection, after the exchange buffer holds every
- * rank's slice.  Outputs as in cusfft_execute. */
+ * rank's slice.  Outputs as in cusfft_execute.  Paper: Steps 5-6 (L91-L95,
+ * Alg. 4, Alg. 5). */
 int cusfft_execute_finish(cusfft_plan_t plan, int64_t* d_locs, void* d_vals);
-/* The exchange buffer: *d_buf points at world * (*bytes_per_rank) bytes of
+/* Plumbing of the caller-run exchange (no paper passage).
+ * The exchange buffer: *d_buf points at world * (*bytes_per_rank) bytes of
  * device memory, rank r's slice at offset r * (*bytes_per_rank) (loop
  * sharding); for signal sharding *bytes_per_rank is the whole buffer. */
 int cusfft_exchange_buffer(cusfft_plan_t plan, void** d_buf, int64_t* bytes_per_rank);
@@ -221,7 +238,9 @@ int cusfft_exchange_buffer(cusfft_plan_t plan, void** d_buf, int64_t* bytes_per_
  * all-reduce of the whole buffer (signal sharding); negative: error. */
 int32_t cusfft_exchange_kind(cusfft_plan_t plan);
 
-/* Plan facts (host arrays, caller-owned):
+/* Paper: a and ai of Alg. 1 (L146-L153), the offset of Def. 1 (L81), the
+ * filter length of Alg. 1's filter[filter_size] (L140).
+ * Plan facts (host arrays, caller-owned):
  *   info[0..15] = n, k, B, L, w (taps of the estimation filter), n/B, num_select, loc_loops,
  *                 vote_threshold, max_hits, distinct 32-B sectors of x this rank's gathers
  *                 touch (the fold's DRAM floor), staged (1: address-sorted two-phase gather,
@@ -249,16 +268,22 @@ typedef enum {
   CUSFFT_DEBUG_LOC_GHAT = 10 /* complex fp64 [n/B + 1]: its G^                                */
 } cusfft_debug_t;
 
-/* Copy a debug artefact of the last execution to host memory.  cap is the
+/* Paper: the intermediate arrays of Alg. 1-5 (buckets L164-L168, the FFT
+ * output L87, J of Alg. 3, the hit list of Alg. 4, the
+ * per-loop estimates of Alg. 5) for parity checks.
+ * Copy a debug artefact of the last execution to host memory.  cap is the
  * destination size in bytes; returns the number of bytes the artefact needs
  * (>= 0; nothing copied if cap is smaller) or a negative status.  Synchronises. */
 int64_t cusfft_get_debug(cusfft_plan_t plan, int32_t what, void* host_dst, int64_t cap);
 
 /* Synchronise the plan's stream and report device-side status of the last
- * execution: CUSFFT_SUCCESS, CUSFFT_HIT_OVERFLOW or CUSFFT_INTERNAL. */
+ * execution: CUSFFT_SUCCESS, CUSFFT_HIT_OVERFLOW (more hits than max_hits;
+ * Alg. 4's hit array L279-L281 is unbounded) or CUSFFT_INTERNAL. */
 int cusfft_status(cusfft_plan_t plan);
 
-/* Timing (enable): 0 off; 1 direct launches (no graph) with CUDA events
+/* Paper: the per-step timing of Fig. 2 (L119) and the average execution
+ * times of §VI (L402).
+ * Timing (enable): 0 off; 1 direct launches (no graph) with CUDA events
  * between the stages; 2 the normal CUDA graph with event-record nodes before
  * and after phase 1 and at the end (times the gather inside the graph that is
  * otherwise executed).
@@ -272,14 +297,16 @@ int cusfft_status(cusfft_plan_t plan);
 int cusfft_set_timing(cusfft_plan_t plan, int32_t enable);
 int cusfft_get_stage_times(cusfft_plan_t plan, float* ms, int32_t cap);
 
-/* Profiling: run only the first `stages` stages (1 = fold ... 6 = output,
+/* Profiling (no paper passage; the per-step breakdown of Fig. 2):
+ * run only the first `stages` stages (1 = fold ... 6 = output,
  * the default) so per-stage times can be taken inside the CUDA graph by
  * differences of whole-execution times.  Outputs are undefined when < 6. */
 int cusfft_set_stage_limit(cusfft_plan_t plan, int32_t stages);
 
-/* Number of kernel launches one cusfft_execute issues for this plan. */
+/* Number of kernel launches one cusfft_execute issues for this plan (plumbing). */
 int32_t cusfft_launches_per_execute(cusfft_plan_t plan);
 
+/* Plumbing: status text, the last CUDA / NCCL error codes, the ABI version. */
 const char* cusfft_strerror(int code);
 int32_t cusfft_last_cuda_error(void);
 int32_t cusfft_last_nccl_error(void);

@@ -185,6 +185,8 @@ struct cusfft_plan_s {
   std::vector<uint32_t> row0_h;              // same, host (+ total rows at [Lg])
   double2* d_staging = nullptr;              // [rows][B]
   int stage_grid = 1;
+  int p2_spc = 2;                            // phase-2 slots per CTA (taps reused across them; 1 / 4 slower)
+  int fork_at = 1;                           // estimation branch forks after phase 1 (0) or after the location phase 2 (1, measured ~0.5 us faster)
   bool setaside = false;                     // holds a reference on the device's persisting-L2 set-aside
   int64_t sectors = 0;                       // distinct 32-B sectors of x gathered by this rank
   double2* d_tw = nullptr;
@@ -534,9 +536,15 @@ cudaError_t set_dyn_smem(K* kern, int want, int optin) {
   return cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, std::min(want, cap));
 }
 
-template <typename ET, int LP>
-cudaError_t set_tail_attr(int smem, int optin) {
-  return set_dyn_smem(k_tail<ET, LP>, smem, optin);
+// k_tail instantiation of a plan: vote-table element (tail_esz), estimation
+// lanes per hit (L <= 16: 16), compile-time L_loc = 8 for the default plans.
+using TailKernel = void (*)(TailArgs);
+TailKernel tail_kernel(int esz, int L, int Lloc) {
+  const bool seg = L <= 16;
+  if (esz == 1 && Lloc == 8) return seg ? k_tail<uint8_t, 16, 8> : k_tail<uint8_t, 32, 8>;
+  if (esz == 1) return seg ? k_tail<uint8_t, 16, 0> : k_tail<uint8_t, 32, 0>;
+  if (esz == 2) return seg ? k_tail<uint16_t, 16, 0> : k_tail<uint16_t, 32, 0>;
+  return seg ? k_tail<uint32_t, 16, 0> : k_tail<uint32_t, 32, 0>;
 }
 
 int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, const cusfft_params* pin, int rank,
@@ -600,7 +608,9 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   P->Lloc = q.loc_loops;
   P->T = q.vote_threshold;
   P->max_hits = (int)q.max_hits;
-  if (const char* e = std::getenv("CUSFFT_NO_GRAPH")) P->use_graph = !(e[0] == '1');
+  if (const char* e = std::getenv("CUSFFT_NO_GRAPH")) P->use_graph = !(e[0] == '1');                    // A/B (measurement)
+  if (const char* e = std::getenv("CUSFFT_P2_SPC")) P->p2_spc = std::max(1, std::min(8, std::atoi(e)));  // A/B (measurement)
+  if (const char* e = std::getenv("CUSFFT_FORK")) P->fork_at = e[0] == '1' ? 1 : 0;                       // A/B (measurement)
   // ---- filters (group 0: location loops; group 1: estimation-only loops)
   {
     const double tl = q.loc_tolerance > 0.0 ? q.loc_tolerance : q.tolerance;
@@ -742,27 +752,15 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   attr(set_dyn_smem(k_select_sort, 210 * 1024, smem_optin));
   attr(set_dyn_smem(k_vote, smem_optin, smem_optin));
   attr(set_dyn_smem(k_output, smem_optin, smem_optin));
-  if (P->tail_esz) {
-    const bool seg = L <= 16;
-    const int ts = P->tail_smem;
-    if (P->tail_esz == 1) attr(seg ? set_tail_attr<uint8_t, 16>(ts, smem_optin) : set_tail_attr<uint8_t, 32>(ts, smem_optin));
-    if (P->tail_esz == 2) attr(seg ? set_tail_attr<uint16_t, 16>(ts, smem_optin) : set_tail_attr<uint16_t, 32>(ts, smem_optin));
-    if (P->tail_esz == 4) attr(seg ? set_tail_attr<uint32_t, 16>(ts, smem_optin) : set_tail_attr<uint32_t, 32>(ts, smem_optin));
-  }
+  if (P->tail_esz) attr(set_dyn_smem(tail_kernel(P->tail_esz, L, P->Lloc), P->tail_smem, smem_optin));
   if (ae != cudaSuccess) {
     g_last_cuda_error = (int)ae;
     return fail(CUSFFT_CUDA);
   }
   if (P->tail_esz) {  // a warp per (enumerated loop, J) unit; CTAs up to the resident limit
     int occ = 0;
-    const bool seg = L <= 16;
-    cudaError_t oe = cudaErrorInvalidValue;
-    if (P->tail_esz == 1)
-      oe = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, seg ? k_tail<uint8_t, 16> : k_tail<uint8_t, 32>, kTailNT, P->tail_smem);
-    else if (P->tail_esz == 2)
-      oe = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, seg ? k_tail<uint16_t, 16> : k_tail<uint16_t, 32>, kTailNT, P->tail_smem);
-    else
-      oe = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, seg ? k_tail<uint32_t, 16> : k_tail<uint32_t, 32>, kTailNT, P->tail_smem);
+    const cudaError_t oe =
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, tail_kernel(P->tail_esz, L, P->Lloc), kTailNT, P->tail_smem);
     if (oe != cudaSuccess || occ < 1) occ = 1;
     cudaGetLastError();
     const int nenum = (P->T > (P->Lloc + 1) / 2) ? P->Lloc / 2 : P->Lloc - P->T + 1;
@@ -910,13 +908,18 @@ cudaError_t launch_p2_t(cusfft_plan_t P, const Filter& F, const double2* staging
                         ZeroArgs z, cudaStream_t st) {
   static thread_local bool attr_set = false;  // one flag per B1T instantiation
   if (!attr_set) {  // static + dynamic smem may exceed the 48 KB default
-    cudaFuncSetAttribute(k_fold_fft1_tma<B1T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    cudaFuncSetAttribute(k_fold_fft1_tma<B1T, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    cudaFuncSetAttribute(k_fold_fft1_tma<B1T, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
     attr_set = true;
   }
-  dim3 grid((unsigned)(P->B / 256), (unsigned)nslots);
-  return launch_k(k_fold_fft1_tma<B1T>, grid, dim3(256), (size_t)F.R * 4096, st, P->cur_prio, staging,
+  // spc slots per CTA (their taps loaded once), double-buffered rows while two fit in shared memory
+  const int spc = (2 * F.R * 4096 <= 160 * 1024) ? std::min(P->p2_spc, nslots) : 1;
+  const size_t smem = (size_t)(spc > 1 ? 2 : 1) * F.R * 4096;
+  dim3 grid((unsigned)(P->B / 256), (unsigned)((nslots + spc - 1) / spc));
+  auto kern = F.R <= 8 ? k_fold_fft1_tma<B1T, 8> : k_fold_fft1_tma<B1T, 16>;
+  return launch_k(kern, grid, dim3(256), smem, st, P->cur_prio, staging,
                   (const double*)F.d_taps_perm, P->prm.debug ? u : nullptr, v, (const double2*)P->d_tw, (int)P->B,
-                  P->B2, F.w, F.R, z);
+                  P->B2, F.w, F.R, nslots, spc, z);
 }
 
 template <int B1T>
@@ -1120,17 +1123,8 @@ int launch_tail(cusfft_plan_t P, cudaStream_t st) {
   ta.v = make_vote_args(P);
   ta.e = make_est_args(P);
   ta.q_off = P->tail_qoff;
-  const bool seg = P->L <= 16;
-  const dim3 g((unsigned)P->tail_grid), b(kTailNT);
-  const size_t sm = (size_t)P->tail_smem;
-  cudaError_t e = cudaErrorInvalidValue;
-  if (P->tail_esz == 1)
-    e = seg ? launch_k(k_tail<uint8_t, 16>, g, b, sm, st, P->cur_prio, ta) : launch_k(k_tail<uint8_t, 32>, g, b, sm, st, P->cur_prio, ta);
-  else if (P->tail_esz == 2)
-    e = seg ? launch_k(k_tail<uint16_t, 16>, g, b, sm, st, P->cur_prio, ta) : launch_k(k_tail<uint16_t, 32>, g, b, sm, st, P->cur_prio, ta);
-  else if (P->tail_esz == 4)
-    e = seg ? launch_k(k_tail<uint32_t, 16>, g, b, sm, st, P->cur_prio, ta) : launch_k(k_tail<uint32_t, 32>, g, b, sm, st, P->cur_prio, ta);
-  CK(e);
+  CK(launch_k(tail_kernel(P->tail_esz, P->L, P->Lloc), dim3((unsigned)P->tail_grid), dim3(kTailNT),
+              (size_t)P->tail_smem, st, P->cur_prio, ta));
   return CUSFFT_SUCCESS;
 }
 
@@ -1232,31 +1226,42 @@ int launch_exchange(cusfft_plan_t P, cudaStream_t st) {
 // address-ordered phase 1 of every slot, then the location slots' phase 2,
 // FFT pass 2 and cutoff on a high-priority stream while the estimation
 // slots' phase 2 and FFT pass 2 fill the SMs the latency-bound chain leaves
-// idle on a second stream; they join before the exchange / the tail.
+// idle on a second stream; they join before the exchange / the tail.  The
+// estimation branch forks after phase 1 (fork_at 0) or after the location
+// slots' phase 2 (fork_at 1: that phase 2 then has the L2 bandwidth alone).
+// Stage limits below 6 end the graph early (both branches joined).
 int launch_branched(cusfft_plan_t P, const double2* x, int64_t* locs, double2* vals) {
   cudaStream_t a = P->stream, b = P->cap_stream2;
   const int nl = P->nloc_local;
+  const int lim = P->stage_limit;
+  auto fork = [&]() -> int {
+    CK(cudaEventRecord(P->ev_fork, a));
+    CK(cudaStreamWaitEvent(b, P->ev_fork, 0));
+    P->cur_prio = P->prio_lo;
+    g_pdl = false;
+    TRY(launch_fold_range(P, x, nl, P->Lg, b, false));
+    g_pdl = true;
+    if (lim >= 2) TRY(launch_bfft(P, nl, P->Lg, b));
+    CK(cudaEventRecord(P->ev_join, b));
+    P->cur_prio = P->prio_hi;
+    g_pdl = true;  // the next kernel on a keeps its programmatic edge (the event record adds no node)
+    return CUSFFT_SUCCESS;
+  };
   P->cur_prio = P->prio_hi;
   g_pdl = false;
   mark(P, 0);
   TRY(launch_stage1(P, x, a));
   mark(P, 7);
-  CK(cudaEventRecord(P->ev_fork, a));
-  CK(cudaStreamWaitEvent(b, P->ev_fork, 0));
-  P->cur_prio = P->prio_lo;
-  g_pdl = false;
-  TRY(launch_fold_range(P, x, nl, P->Lg, b, false));
+  if (P->fork_at == 0) TRY(fork());
   g_pdl = true;
-  TRY(launch_bfft(P, nl, P->Lg, b));
-  CK(cudaEventRecord(P->ev_join, b));
-  P->cur_prio = P->prio_hi;
-  g_pdl = true;  // keeps its programmatic edge to phase 1 (the fork's event record adds no node)
   TRY(launch_fold_range(P, x, 0, nl, a, false));
-  TRY(launch_bfft(P, 0, nl, a));
-  if (!P->xshard) TRY(launch_select(P, a));
+  if (P->fork_at == 1) TRY(fork());
+  if (lim >= 2) TRY(launch_bfft(P, 0, nl, a));
+  if (lim >= 3 && !P->xshard) TRY(launch_select(P, a));
   P->cur_prio = 0;
   CK(cudaStreamWaitEvent(a, P->ev_join, 0));
   g_pdl = false;
+  if (lim < 4) return CUSFFT_SUCCESS;
   if (P->comm) {
     TRY(launch_exchange(P, a));
     return launch_finish(P, locs, vals);
@@ -1265,8 +1270,22 @@ int launch_branched(cusfft_plan_t P, const double2* x, int64_t* locs, double2* v
 }
 
 inline bool use_branches(cusfft_plan_t P) {
-  return P->use_graph && P->timing != 1 && P->stage_limit == 6 && P->staged && P->nloc_local > 0 &&
+  return P->timing != 1 && P->staged && P->nloc_local > 0 &&
          P->nloc_local < P->Lg && !P->xshard;
+}
+
+// The plan-owned capture stream, the estimation branch's stream and the fork / join events.
+int ensure_streams(cusfft_plan_t P) {
+  if (P->cap_stream) return CUSFFT_SUCCESS;
+  int lo = 0, hi = 0;
+  CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+  P->prio_lo = lo;
+  P->prio_hi = hi;
+  CK(cudaStreamCreateWithPriority(&P->cap_stream, cudaStreamNonBlocking, hi));   // location chain
+  CK(cudaStreamCreateWithPriority(&P->cap_stream2, cudaStreamNonBlocking, lo));  // estimation folds
+  CK(cudaEventCreateWithFlags(&P->ev_fork, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&P->ev_join, cudaEventDisableTiming));
+  return CUSFFT_SUCCESS;
 }
 
 // Run `body` (which enqueues on P->stream) either directly or through a cached
@@ -1281,16 +1300,7 @@ int run_graphed(cusfft_plan_t P, cusfft_plan_s::GraphEntry& g, const void* a, co
       cudaGraphExecDestroy(g.exec);
       g.exec = nullptr;
     }
-    if (!P->cap_stream) {
-      int lo = 0, hi = 0;
-      CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
-      P->prio_lo = lo;
-      P->prio_hi = hi;
-      CK(cudaStreamCreateWithPriority(&P->cap_stream, cudaStreamNonBlocking, hi));   // location chain
-      CK(cudaStreamCreateWithPriority(&P->cap_stream2, cudaStreamNonBlocking, lo));  // estimation folds
-      CK(cudaEventCreateWithFlags(&P->ev_fork, cudaEventDisableTiming));
-      CK(cudaEventCreateWithFlags(&P->ev_join, cudaEventDisableTiming));
-    }
+    TRY(ensure_streams(P));
     CK(cudaStreamBeginCapture(P->cap_stream, cudaStreamCaptureModeThreadLocal));
     cudaStream_t user = P->stream;
     P->stream = P->cap_stream;
@@ -1342,7 +1352,10 @@ int execute_full(cusfft_plan_t plan, const void* d_x, int64_t* d_locs, void* d_v
   return run_graphed(plan, full_entry(plan, d_x, d_locs, d_vals), d_x, d_locs, d_vals, [&] {
     const double2* x = reinterpret_cast<const double2*>(d_x);
     double2* v = reinterpret_cast<double2*>(d_vals);
-    if (use_branches(plan)) return launch_branched(plan, x, d_locs, v);
+    if (use_branches(plan)) {
+      TRY(ensure_streams(plan));  // (graph-less runs: the second stream is used directly)
+      return launch_branched(plan, x, d_locs, v);
+    }
     TRY(launch_local(plan, x));
     if (plan->comm) {
       g_pdl = false;

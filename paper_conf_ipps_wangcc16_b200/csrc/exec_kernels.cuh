@@ -254,43 +254,53 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict_
 }
 
 // ---------------------------------------------------------------------------
-// Phase 2 of the scatter-staged fold with bulk copies: the
-// CTA's R rows of 256 staged samples (row rr = staging[(s R + rr) B + cta 256
-// ...], 4 KB each, already in this kernel's thread order) are moved to shared
-// memory by the bulk-copy engine onto one mbarrier while the threads fetch
-// their taps, so no gathered sample occupies a register and four CTAs fit per
-// SM.  Then exactly k_fold_fft1's arithmetic: rounds accumulated in Alg. 1's
-// order (fp64 mul + add per component), u written, the C columns' B1-point
-// FFTs in shared memory, v = FFT x omega_B^(c k1).  The consumed staging
-// lines stay in L2 (the persisting set-aside): the next execution's phase-1
-// stores then hit valid lines.
+// Phase 2 of the scatter-staged fold with bulk copies: a CTA
+// owns one tile of 256 buckets of `spc` consecutive slots of one filter.  Its
+// taps (R per thread) are loaded once and serve every slot; each slot's R rows
+// of 256 staged samples (row rr = staging[(s R + rr) B + tile 256 ...], 4 KB
+// each, already in this kernel's thread order) are moved to shared memory by
+// the bulk-copy engine onto an mbarrier, double-buffered so the next slot's
+// rows stream in while this one is folded.  Per slot exactly k_fold_fft1's
+// arithmetic: rounds accumulated in Alg. 1's order (fp64 mul + add per
+// component), u written (debug plans), the C columns' B1-point FFTs in shared
+// memory, v = FFT x omega_B^(c k1).  The consumed staging lines stay in L2
+// (the persisting set-aside): the next execution's phase-1 stores then hit
+// valid lines.
 // ---------------------------------------------------------------------------
-template <int B1T>
-__global__ void __launch_bounds__(256, 4) k_fold_fft1_tma(const double2* __restrict__ staging,
+// RMAX: taps held in registers (8 when R <= 8, else 16; rounds beyond reload theirs).
+template <int B1T, int RMAX>
+__global__ void __launch_bounds__(256, 3) k_fold_fft1_tma(const double2* __restrict__ staging,
                                                           const double* __restrict__ taps_perm,
                                                           double2* __restrict__ u, double2* __restrict__ v,
                                                           const double2* __restrict__ tw, int B, int B2, int w, int R,
-                                                          ZeroArgs zero) {
+                                                          int nslots, int spc, ZeroArgs zero) {
   pdl_wait();
   KTRACE(2);
   constexpr int C = 256 / B1T;
-  constexpr int RMAX = 16;
-  extern __shared__ __align__(128) double2 Tile[];  // [R][256]
+  extern __shared__ __align__(128) double2 Tile[];  // [nbuf][R][256]
   __shared__ double2 S[256 + 256 / 8];
   __shared__ double2 twl[B1T];
-  __shared__ __align__(8) uint64_t bar;
+  __shared__ __align__(8) uint64_t bar[2];
   const int t = threadIdx.x;
-  const int s = blockIdx.y;
+  const int s0 = blockIdx.y * spc;
+  const int ns = min(spc, nslots - s0);
   if (blockIdx.x == 0 && blockIdx.y == 0) TRACE(0);
-  const double2* src = staging + (int64_t)s * R * B + (int64_t)blockIdx.x * 256;
-  if (t == 0) {
-    mbar_init(&bar, 1);
-    mbar_expect_tx(&bar, (uint32_t)R * 4096u);
-  }
-  __syncthreads();
-  if (t < 32) {
+  const double2* src0 = staging + (int64_t)s0 * R * B + (int64_t)blockIdx.x * 256;
+  const uint32_t bytes = (uint32_t)R * 4096u;
+  // thread 0: slot i's R rows into buffer i & 1 (its barrier's next phase)
+  auto issue = [&](int i) {
+    uint64_t* b = bar + (i & 1);
+    mbar_expect_tx(b, bytes);
     const uint64_t pol = l2_policy_first();
-    for (int rr = t; rr < R; rr += 32) bulk_g2s(Tile + rr * 256, src + (int64_t)rr * B, 4096u, &bar, pol);
+    const double2* src = src0 + (int64_t)i * R * B;
+    double2* dst = Tile + (size_t)(i & 1) * R * 256;
+    for (int rr = 0; rr < R; ++rr) bulk_g2s(dst + rr * 256, src + (int64_t)rr * B, 4096u, b, pol);
+  };
+  if (t == 0) {
+    mbar_init(bar, 1);
+    mbar_init(bar + 1, 1);
+    issue(0);
+    if (ns > 1) issue(1);
   }
   zero_part(zero);
   const int cl = t / B1T, j1 = t % B1T;
@@ -301,33 +311,39 @@ __global__ void __launch_bounds__(256, 4) k_fold_fft1_tma(const double2* __restr
   double g[RMAX];
 #pragma unroll
   for (int rr = 0; rr < RMAX; ++rr) g[rr] = (rr < R && j + rr * B < w) ? __ldg(tp + (int64_t)rr * B) : 0.0;
-  mbar_wait(&bar, 0);
-  double ar = 0.0, ai = 0.0;
-#pragma unroll
-  for (int rr = 0; rr < RMAX; ++rr) {
-    if (rr < R && j + rr * B < w) {
-      const double2 q = Tile[rr * 256 + t];
-      ar = __dadd_rn(ar, __dmul_rn(g[rr], q.x));
-      ai = __dadd_rn(ai, __dmul_rn(g[rr], q.y));
-    }
-  }
-  for (int rr = RMAX; rr < R; ++rr) {  // R > 16 (small tolerance / Gaussian filters)
-    if (j + rr * B < w) {
-      const double2 q = Tile[rr * 256 + t];
-      const double gg = __ldg(tp + (int64_t)rr * B);
-      ar = __dadd_rn(ar, __dmul_rn(gg, q.x));
-      ai = __dadd_rn(ai, __dmul_rn(gg, q.y));
-    }
-  }
-  S[fft_pad(cl * B1T + j1)] = make_double2(ar, ai);
-  __syncthreads();
-  const int wc = t % C, wj = t / C;
-  const size_t wpos = (size_t)s * B + (size_t)blockIdx.x * C + wc + (size_t)B2 * wj;
-  if (u) u[wpos] = S[fft_pad(wc * B1T + wj)];  // the fold output itself: debug plans only
-  __syncthreads();
-  fft_smem<B1T, 256, 256, true>(S, twl, B1T);
+  const int wc = t % C, wj = t / C;  // writer's (column, row)
   const double2 wv = __ldg(tw + (((int64_t)(blockIdx.x * C + wc) * wj) & (B - 1)));
-  v[wpos] = cmul(S[fft_pad(wc * B1T + wj)], wv);
+  __syncthreads();  // barrier init visible to every thread
+  for (int i = 0; i < ns; ++i) {
+    const double2* T = Tile + (size_t)(i & 1) * R * 256;
+    mbar_wait(bar + (i & 1), (uint32_t)((i >> 1) & 1));
+    double ar = 0.0, ai = 0.0;
+#pragma unroll
+    for (int rr = 0; rr < RMAX; ++rr) {
+      if (rr < R && j + rr * B < w) {
+        const double2 q = T[rr * 256 + t];
+        ar = __dadd_rn(ar, __dmul_rn(g[rr], q.x));
+        ai = __dadd_rn(ai, __dmul_rn(g[rr], q.y));
+      }
+    }
+    for (int rr = RMAX; rr < R; ++rr) {  // R > 16 (small tolerance / Gaussian filters)
+      if (j + rr * B < w) {
+        const double2 q = T[rr * 256 + t];
+        const double gg = __ldg(tp + (int64_t)rr * B);
+        ar = __dadd_rn(ar, __dmul_rn(gg, q.x));
+        ai = __dadd_rn(ai, __dmul_rn(gg, q.y));
+      }
+    }
+    S[fft_pad(cl * B1T + j1)] = make_double2(ar, ai);
+    __syncthreads();  // every thread is done with buffer i & 1
+    if (t == 0 && i + 2 < ns) issue(i + 2);
+    const size_t wpos = (size_t)(s0 + i) * B + (size_t)blockIdx.x * C + wc + (size_t)B2 * wj;
+    if (u) u[wpos] = S[fft_pad(wc * B1T + wj)];  // the fold output itself: debug plans only
+    __syncthreads();
+    fft_smem<B1T, 256, 256, true>(S, twl, B1T);
+    v[wpos] = cmul(S[fft_pad(wc * B1T + wj)], wv);
+    __syncthreads();  // S is rewritten by the next slot
+  }
   TRACE_END(1);
 }
 

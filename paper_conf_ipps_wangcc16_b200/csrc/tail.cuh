@@ -385,7 +385,8 @@ __device__ __forceinline__ uint32_t tab_at(uint32_t base, uint32_t i) {
 }
 
 // ET: vote table element; LP: estimation lanes per hit (16 or 32).
-template <typename ET, int LP>
+// LL: L_loc at compile time (8, the default plans) or 0 (any L_loc <= 8 sizeof(ET)).
+template <typename ET, int LP, int LL>
 __global__ void __launch_bounds__(kTailNT, 4) k_tail(TailArgs A) {
   pdl_wait();
   KTRACE(9);
@@ -453,6 +454,9 @@ __global__ void __launch_bounds__(kTailNT, 4) k_tail(TailArgs A) {
 #ifdef CUSFFT_TRACE
   const long long c_vote0 = clock64();
 #endif
+  uint32_t sig_r[LL > 0 ? LL : 1];
+#pragma unroll
+  for (int qq = 0; qq < (LL > 0 ? LL : 1); ++qq) sig_r[qq] = LL > 0 ? ssig[qq] : 0u;
   uint32_t tab_s;
   asm volatile("mov.u32 %0, %1;" : "=r"(tab_s) : "r"(smem_u32(smem)));
   uint16_t* q = reinterpret_cast<uint16_t*>(smem + A.q_off) + wid * kTailQ;
@@ -521,7 +525,13 @@ __global__ void __launch_bounds__(kTailNT, 4) k_tail(TailArgs A) {
           const uint32_t F = a * ((p0 + c0 + (uint32_t)q[b0 + lane]) << sh);
           f = F >> sh;
           uint32_t bits = 0u;
-          for (int qq = 0; qq < Lloc; ++qq) bits |= tab_at<ET>(tab_s, (ssig[qq] * F + half_s) >> bsh) & (1u << qq);
+          if (LL > 0) {  // compile-time L_loc: unrolled, sigmas in registers
+#pragma unroll
+            for (int qq = 0; qq < (LL > 0 ? LL : 1); ++qq)
+              bits |= tab_at<ET>(tab_s, (sig_r[qq] * F + half_s) >> bsh) & (1u << qq);
+          } else {
+            for (int qq = 0; qq < Lloc; ++qq) bits |= tab_at<ET>(tab_s, (ssig[qq] * F + half_s) >> bsh) & (1u << qq);
+          }
           if (V.pairs) {
             const uint32_t below = bits & ((1u << (2 * e)) - 1u);
             hit = __popc(bits) >= V.T && (below & (below >> 1) & 0x55555555u) == 0u;

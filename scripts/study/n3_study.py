@@ -27,7 +27,8 @@ import numpy as np
 import oracle as O
 from paper_conf_ipps_wangcc16_b200.workload import planted_signal
 
-n, k, B, L_loc, L_est, T = 2 ** 24, 1000, 16384, 8, 8, 5
+n, k, L_loc, L_est, T = 2 ** 24, 1000, 8, 8, 5
+B = int(os.environ.get("N3_B", "16384"))  # N3_B=8192: half the formula's buckets (Bcst = 1/2)
 nb = n // B
 
 # name: (delta_loc, lambda_loc * B, delta_est, num / k, lambda_est * B)
@@ -72,6 +73,13 @@ SETTINGS4 = {
     "loc_d1e-5_lam0.75_est_d1e-7_lam0.75": (1e-5, 0.75, 1e-7, 1, 0.75),
     "loc_d1e-5_lam0.875_est_d1e-7_lam0.75": (1e-5, 0.875, 1e-7, 1, 0.75),
 }
+# fifth round (N3_SET=5, with N3_B=8192): half the buckets, both main-lobe widths
+SETTINGS5 = {
+    "all_d1e-7_lam0.75": (1e-7, 0.75, 1e-7, 1, 0.75),
+    "all_d1e-7_lam0.5": (1e-7, 0.5, 1e-7, 1, 0.5),
+}
+if os.environ.get("N3_SET") == "5":
+    SETTINGS = SETTINGS5
 if os.environ.get("N3_SET") == "4":
     SETTINGS = SETTINGS4
 if os.environ.get("N3_SET") == "2":
@@ -107,7 +115,7 @@ def run_setting(x, S, X, seed, name):
     med = (per_loop.shape[1] - 1) // 2
     vals = np.sort(per_loop.real, axis=1)[:, med] + 1j * np.sort(per_loop.imag, axis=1)[:, med]
     locs, out = O.select_output(hits, vals, k)
-    return {"setting": name, "seed": seed, "delta_loc": d_loc, "lambda_loc_B": lam_loc, "delta_est": d_est,
+    return {"setting": name, "B": B, "seed": seed, "delta_loc": d_loc, "lambda_loc_B": lam_loc, "delta_est": d_est,
             "lambda_est_B": lam_est, "num": int(numf * k), "w_loc": len(g_loc), "w_est": len(g_est),
             "sum_w": L_loc * len(g_loc) + L_est * len(g_est),
             "exact": bool(set(locs.tolist()) == set(S.tolist())),
