@@ -466,7 +466,8 @@ def run_gpu(args):
     ablations = None
     if world == 1 and args.ablations:
         ablations = {}
-        variants = [("cutoff_sort_alg3", dict(cutoff_mode=1)),
+        variants = [("separate_filters_n3_loc_d1e-6", dict(loc_tolerance=1e-6, loc_lobefrac=prm["lobefrac"])),
+                    ("cutoff_sort_alg3", dict(cutoff_mode=1)),
                     ("cutoff_threshold_alg6", dict(cutoff_mode=2, cutoff_threshold=1e-3)),
                     ("direct_gather_no_stage", dict(gather=1)),
                     ("no_l2_persist", dict(l2_persist=0))]
@@ -493,10 +494,16 @@ def run_gpu(args):
     # roofline kernel: the address-ordered permute gather (fold phase 1) -- it
     # carries all of the transform's HBM traffic.  Algorithmic bytes: 32 B per
     # distinct sector of x the plan's gathers touch.
-    gather_bytes = int(info["sectors"]) * 32
     sum_w = int(info["w_loc"]) * plan.loc_loops + int(info["w"]) * (L - plan.loc_loops) if info["filters"] == 2 else L * plan.w
+    lw_local = sum_w // world if world > 1 and args.shard == "loops" else sum_w
+    gather_bytes = lw_local * 32  # one 32-B sector per gathered 16-B sample (L w 32 B)
     rk_ms = gather["warm"]["ms"] if "warm" in gather else stage_ms.get("fold", 0.0)
     achieved = gather_bytes / (rk_ms * 1e-3) / 1e9
+    cupti_gather_us = None
+    if isinstance(cupti, dict):
+        for kk, vv in cupti.items():
+            if kk.startswith("k_stage_packed") and isinstance(vv, dict):
+                cupti_gather_us = vv.get("mean_us")
     traffic = None
     tf = os.path.join(ROOT, "profiles", f"fold_traffic_{args.config}.json")
     if os.path.exists(tf):
@@ -528,10 +535,12 @@ def run_gpu(args):
                      "frac": achieved / peak, "traffic": traffic,
                      "kernel": "k_stage_packed (fold phase 1: address-ordered permute gather of x)",
                      "algorithmic_bytes_per_launch": gather_bytes, "kernel_ms": rk_ms,
-                     "algorithmic_bytes_note": "32 B per distinct 32-B sector of x the plan's gathers touch "
-                                               f"({int(info['sectors'])} sectors; L*w*32 = {sum_w * 32} B before sharing)",
-                     "kernel_ms_how": "CUDA event-record nodes around the kernel inside the bench's graph, "
-                                      "L2 flushed before each execution",
+                     "algorithmic_bytes_note": f"L*w*32 B: {lw_local} gathers x one 32-B sector (SURVEY 8(d)); "
+                                               f"{int(info['sectors'])} distinct sectors = {int(info['sectors']) * 32} B",
+                     "kernel_ms_how": "CUDA event-record nodes around the kernel inside the bench's graph "
+                                      "(adds the event latency), L2 flushed before each execution",
+                     "kernel_ms_cupti": cupti_gather_us * 1e-3 if cupti_gather_us else None,
+                     "frac_cupti": (gather_bytes / (cupti_gather_us * 1e-6) / 1e9 / peak) if cupti_gather_us else None,
                      "kernel_ms_cold": gather.get("cold", {}).get("ms"),
                      "frac_cold": (gather_bytes / (gather["cold"]["ms"] * 1e-3) / 1e9 / peak) if "cold" in gather else None,
                      "peak_source": peak_src},

@@ -715,7 +715,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   if ((rc = dalloc(&P->d_keys, (size_t)std::max(1, nsel) * B))) return fail(rc);
   {
     // per-execution counters and histograms: one block, zeroed by the first kernel
-    P->pk_direct = P->tail_esz && P->sel_cluster && P->sel_slots_h == P->loc_slots_h && B % 32 == 0;
+    P->pk_direct = P->tail_esz && P->sel_cluster && P->sel_slots_h == P->loc_slots_h && B % 32 == 0 &&
+                   q.cutoff_mode != CUSFFT_CUTOFF_SORT;
     const int base = 8 + nsel * 4096 + 4096 + 4;
     const int pk_off = (base + 3) & ~3;  // 16-B aligned (uint4 copies)
     P->nzero = P->pk_direct ? pk_off + (int)(((int64_t)B * P->tail_esz + 15) / 16) * 4 : base;

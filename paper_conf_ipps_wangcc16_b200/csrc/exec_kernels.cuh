@@ -739,6 +739,9 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
   uint32_t* sbits = reinterpret_cast<uint32_t*>(smem + sizeof(SelClusterSmem));  // this CTA's words
   const int tid = threadIdx.x, lane = tid & 31;
   const int r = (int)cl.block_rank();
+  // no remote shared memory may be touched before every CTA of the cluster has
+  // started: arrive now, wait before the first DSMEM store (step 1)
+  asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");
   const int B = A.B;
   const int per = B / kSelCL;           // keys per CTA (multiple of 32)
   const int wpc = per >> 5;             // words per CTA
@@ -766,12 +769,12 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
   int d0 = 0, k2 = 0;
   bool whole = true;
   {
-  // 1. slice totals, pushed to every CTA of the cluster
+  // 1. slice totals, pushed to every CTA of the cluster (once every CTA of the
+  //    cluster has started: the split barrier's arrive was issued at entry)
   int tot, ex = 0;
-  if (!A.threshold_mode) {
-    ex = block_excl_scan<kSelCNT>(c0 + c1, &tot, S.sm);
-    if (tid < kSelCL) cl.map_shared_rank(&S, tid)->part[r] = tot;
-  }
+  if (!A.threshold_mode) ex = block_excl_scan<kSelCNT>(c0 + c1, &tot, S.sm);
+  asm volatile("barrier.cluster.wait.aligned;" ::: "memory");
+  if (!A.threshold_mode && tid < kSelCL) cl.map_shared_rank(&S, tid)->part[r] = tot;
   cl.sync();
   // 2. the boundary slice (slices descending r = kSelCL-1 .. 0) finds d0 and pushes it
   if (!A.threshold_mode) {

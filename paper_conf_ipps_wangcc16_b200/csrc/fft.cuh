@@ -144,7 +144,7 @@ struct FftPassArgs {
   // cutoff keys (pass 2 / single pass only): slot -> location index or -1
   const int* key_index;   // [slots of this rank], may be null
   uint64_t* keys;         // [n_sel][B]
-  uint32_t* hist;         // [n_sel][4096]
+  uint32_t* hist;         // [n_sel][4096] top-digit histograms (null: none)
 };
 
 // E = elements per CTA, NT = threads per CTA.  Dynamic smem: fft_smem_bytes(E).
@@ -197,7 +197,8 @@ __global__ void __launch_bounds__(NT) k_fft(FftPassArgs A) {
   const bool one_slot = NSEQ <= (1 << A.log_seq_per_slot);
   int kidx = -1;
   if (A.key_index && one_slot) kidx = A.key_index[q0 >> A.log_seq_per_slot];
-  if (kidx >= 0) {
+  const bool hist = A.hist != nullptr;
+  if (kidx >= 0 && hist) {
     for (int i = threadIdx.x; i < 4096; i += NT) shist[i] = 0;
     __syncthreads();
   }
@@ -225,7 +226,8 @@ __global__ void __launch_bounds__(NT) k_fft(FftPassArgs A) {
               (uint64_t)__double_as_longlong(__dadd_rn(__dmul_rn(v.x, v.x), __dmul_rn(v.y, v.y)));
           A.keys[(int64_t)ki * A.B + opos] = key;
           const uint32_t d = (uint32_t)(key >> 51) & 0xFFFu;
-          if (one_slot) {
+          if (!hist) {
+          } else if (one_slot) {
             atomicAdd(&shist[d], 1u);
           } else {
             atomicAdd(&A.hist[(int64_t)ki * 4096 + d], 1u);
@@ -234,7 +236,7 @@ __global__ void __launch_bounds__(NT) k_fft(FftPassArgs A) {
       }
     }
   }
-  if (kidx >= 0) {
+  if (kidx >= 0 && hist) {
     __syncthreads();
     for (int i = threadIdx.x; i < 4096; i += NT)
       if (shist[i]) atomicAdd(&A.hist[(int64_t)kidx * 4096 + i], shist[i]);

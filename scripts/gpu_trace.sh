@@ -1,5 +1,5 @@
 # In-graph per-kernel spans (trace build).  VARIANTS: space-separated env
-# assignments joined by commas, e.g. "CUSFFT_VOTE_VC=2 CUSFFT_VOTE_VC=4,CUSFFT_STAGE_MODE=split_index".
+# assignments joined by commas, e.g. "CUSFFT_P2_SPC=1 CUSFFT_P2_SPC=2,CUSFFT_FORK=0".
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
 python -c "

@@ -21,10 +21,10 @@ if os.path.exists(f"{G}/launches.csv"):
     for r in rows[i + 1:]:
         if len(r) > vi:
             d[r[ki].split("(")[0]].append(float(r[vi].replace(",", "")))
-    hot = {k: v for k, v in d.items() if "cusfft::k_" in k and not any(s in k for s in ("cheb", "dc_window", "taps", "normalize", "ghat", "twiddles", "gauss"))}
+    hot = {k: v for k, v in d.items() if "cusfft::k_" in k and not any(s in k for s in ("cheb", "dc_window", "taps", "normalize", "ghat", "ginv", "phase_table", "twiddles", "gauss"))}
     step = sum(sum(v) / len(v) for v in hot.values())
     lines.append(f"## Launch list (ncu --metrics gpu__time_duration.sum --clock-control none; cold-cache, serialised)\n")
-    lines.append(f"Command: `ncu ... python bench.py --steps 2 --warmup 3 --no-cpu-baseline` (file `{tag}_launches.csv`).\n")
+    lines.append(f"Command: `ncu --metrics gpu__time_duration.sum --clock-control none ... python bench.py --steps 2 --warmup 3 --no-cpu-baseline --no-cupti --no-default-line` (file `{tag}_launches.csv`).  Per-launch times are cold-cache and serialised; the SHARES are what compare with the bench's in-graph numbers.\n")
     lines.append("| kernel | launches | mean µs | share of hot-path sum |\n|---|---|---|---|")
     for k, v in sorted(hot.items(), key=lambda kv: -sum(kv[1]) / len(kv[1])):
         m = sum(v) / len(v) / 1e3
@@ -43,7 +43,7 @@ want = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "lts__t_sectors_srcunit_tex_op_read.sum", "sm__warps_active.avg.pct_of_peak_sustained_active", "launch__registers_per_thread",
         "smsp__inst_executed.sum", "sm__throughput.avg.pct_of_peak_sustained_elapsed", "launch__grid_size", "launch__block_size"]
 scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9}
-rep = f"{G}/prof_all.ncu-rep"
+rep = f"{G}/prof_{tag}.ncu-rep" if os.path.exists(f"{G}/prof_{tag}.ncu-rep") else f"{G}/prof_all.ncu-rep"
 traffic = None
 fold_parts = {}
 if os.path.exists(rep):
@@ -67,7 +67,11 @@ if os.path.exists(rep):
 if fold_parts:
     rd = sum(v[0] for v in fold_parts.values())
     wr = sum(v[1] for v in fold_parts.values())
+    info = json.load(open(f"{G}/plan_info.json")) if os.path.exists(f"{G}/plan_info.json") else {}
+    sp = [v for k, v in fold_parts.items() if k.startswith("cusfft::k_stage_packed") or k.startswith("k_stage_packed")]
     traffic = {"kernel": " + ".join(sorted(fold_parts)), "config": "C3", "source": f"{tag}_ncu_summary.md (ncu --set full)",
+               "sum_w": info.get("sum_w"), "plan": info,
+               "k_stage_packed_dram_bytes_per_launch": (sp[0][0] + sp[0][1]) if sp else None,
                "parts": {k: {"dram_bytes_read": v[0], "dram_bytes_write": v[1], "dram_bytes_per_launch": v[0] + v[1]}
                          for k, v in fold_parts.items()},
                "dram_bytes_read": rd, "dram_bytes_write": wr, "dram_bytes_per_launch": rd + wr}

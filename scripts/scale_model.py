@@ -1,0 +1,97 @@
+"""Per-rank time model of loop-sharded C3 on G = 1, 2, 4, 8 GPUs, with the
+per-rank compute MEASURED on one B200.
+
+For each G the script builds rank 0's plan of a G-rank loop-sharded run
+(cusfft_plan_dist without a communicator), and times on the bench's terms
+(L2 flushed before every step, CUDA events, graphs):
+  local  = cusfft_execute_local  (Steps 1-4 of this rank's L/G loops)
+  finish = cusfft_execute_finish (vote + estimation + output over all L loops)
+The exchange buffer is filled with the records of a world = 1 plan of the same
+draws (the all-gather's result), so finish does the real work.  The
+all-gather itself cannot be timed on one GPU: it is modelled as
+alpha + (G-1)/G * bytes / bw with the bytes of the plan and stated alpha / bw.
+Usage: scale_model.py OUT.json
+"""
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+import bench  # noqa: E402
+from paper_conf_ipps_wangcc16_b200 import Plan, default_B  # noqa: E402
+from paper_conf_ipps_wangcc16_b200.dist import slot_of_loop  # noqa: E402
+
+ALPHA_US = 10.0   # assumed NCCL all-gather latency inside one NVSwitch domain (small messages)
+BW_GBS = 700.0    # assumed achieved all-gather bus bandwidth per GPU (NVLink 5, 900 GB/s per direction)
+
+n, k, L = bench.CONFIGS["C3"][:3]
+B = default_B(n, k)
+prm = bench.plan_params("C3", B)
+x_np, S, X = bench.make_signal(n, k, 1)
+dev = torch.device("cuda", 0)
+x = torch.from_numpy(x_np).to(dev)
+flush = bench.L2Flush(dev)
+stream = torch.cuda.current_stream()
+
+
+def timed(fn, reps=20):
+    for _ in range(3):
+        flush()
+        fn()
+    ts = []
+    for _ in range(reps):
+        flush()
+        a = torch.cuda.Event(enable_timing=True)
+        b = torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        fn()
+        b.record(stream)
+        torch.cuda.synchronize()
+        ts.append(a.elapsed_time(b) * 1e3)
+    return sum(ts) / len(ts)
+
+
+ref = Plan(n, k, B=B, L=L, seed=3, device=0, **prm)
+locs = torch.empty(k, dtype=torch.int64, device=dev)
+vals = torch.empty(k, dtype=torch.complex128, device=dev)
+full_us = timed(lambda: ref.execute(x, locs, vals))
+ref.execute(x, locs, vals)
+torch.cuda.synchronize()
+ref_ptr, ref_per = ref.exchange_buffer()
+rec_bytes = ref_per // L
+ref_buf = torch.as_tensor(__import__("paper_conf_ipps_wangcc16_b200.dist", fromlist=["_CudaBuffer"])._CudaBuffer(
+    ref_ptr, ref_per), device=dev)
+out = {"config": "C3", "filter": bench.filter_desc("C3"), "single_gpu_us": full_us,
+       "allgather_model": {"alpha_us": ALPHA_US, "bw_gbs": BW_GBS,
+                           "note": "assumed, not measured (one GPU in this environment)"},
+       "ranks": {}}
+for G in (1, 2, 4, 8):
+    p = Plan(n, k, B=B, L=L, seed=3, device=0, rank=0, world=G, **prm)
+    ptr, per = p.exchange_buffer()
+    buf = torch.as_tensor(__import__("paper_conf_ipps_wangcc16_b200.dist", fromlist=["_CudaBuffer"])._CudaBuffer(
+        ptr, per * G), device=dev)
+    local_us = timed(lambda: p.execute_local(x))
+    # the all-gather's result: every loop's record at its loop-sharded slot
+    for r in range(L):
+        s = slot_of_loop(r, L, G)
+        buf[s * rec_bytes:(s + 1) * rec_bytes].copy_(ref_buf[r * rec_bytes:(r + 1) * rec_bytes])
+    torch.cuda.synchronize()
+    l2 = torch.empty_like(locs)
+    v2 = torch.empty_like(vals)
+    finish_us = timed(lambda: p.execute_finish(l2, v2))
+    p.execute_finish(l2, v2)
+    torch.cuda.synchronize()
+    same = torch.equal(l2, locs) and torch.equal(v2, vals)
+    ag_bytes = per * G
+    ag_us = 0.0 if G == 1 else ALPHA_US + (G - 1) / G * ag_bytes / (BW_GBS * 1e3)
+    out["ranks"][G] = {"local_us": local_us, "finish_us": finish_us, "allgather_bytes": ag_bytes,
+                       "allgather_model_us": ag_us, "model_total_us": local_us + ag_us + finish_us,
+                       "finish_equals_single_gpu_output": same}
+    p.close()
+print(json.dumps(out, indent=1))
+with open(sys.argv[1], "w") as f:
+    json.dump(out, f, indent=1)

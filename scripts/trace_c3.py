@@ -50,7 +50,7 @@ for rep in range(reps):
     for i, (s, e) in spans.items():
         acc.setdefault(i, []).append(((s - t0) / 1e3, (e - t0) / 1e3))
     acc.setdefault(0, []).append((0.0, (end - t0) / 1e3))
-print(f"C3 L={L} tol={tol:g} staged={plan.info()['staged'] if hasattr(plan, 'info') else '?'} mode={os.environ.get('CUSFFT_STAGE_MODE', 'default')}")
+print(f"C3 L={L} {prm} staged={plan.info()['staged']}")
 print(f"{'kernel':16s} {'start us':>9s} {'end us':>9s} {'span us':>9s}")
 for i, v in sorted(acc.items(), key=lambda kv: np.mean([a for a, b in kv[1]])):
     s = np.median([a for a, b in v]); e = np.median([b for a, b in v])
