@@ -408,11 +408,17 @@ __global__ void __launch_bounds__(kTailNT, 4) k_tail(TailArgs A) {
     const int e0 = warp / V.num;
     Jpre = (uint32_t)__ldcg(V.Jp[V.pairs ? 2 * e0 : e0] + (warp - e0 * V.num));
   }
-  // ---- the vote table: copy (the cutoff ORed the winners into V.pk) or transpose the bitmaps
+  // ---- the vote table: bulk-copied (the cutoff ORed the winners into V.pk) or transposed from the bitmaps
+  __shared__ __align__(8) uint64_t tbar;
+  const uint32_t tbytes = (uint32_t)(((int64_t)B * sizeof(ET) + 15) & ~int64_t(15));
   if (V.pk) {
-    const int n16 = (int)(((int64_t)B * sizeof(ET) + 15) / 16);
-    for (int i = tid; i < n16; i += kTailNT)
-      reinterpret_cast<uint4*>(smem)[i] = __ldcg(reinterpret_cast<const uint4*>(V.pk) + i);
+    if (tid == 0) {
+      mbar_init(&tbar, 1);
+      mbar_expect_tx(&tbar, tbytes);
+      for (uint32_t o = 0; o < tbytes; o += 32768u)
+        bulk_g2s(smem + o, reinterpret_cast<const uint8_t*>(V.pk) + o, min(32768u, tbytes - o), &tbar,
+                 l2_policy_last());
+    }
   } else {
     ET* tab = reinterpret_cast<ET*>(smem);
     const int words = (B + 31) >> 5;
@@ -433,14 +439,14 @@ __global__ void __launch_bounds__(kTailNT, 4) k_tail(TailArgs A) {
     ssig[tid] = V.sig[tid];
     saa[tid] = V.aa[tid];
   }
+  // unit prefix over the enumerated loops' winner counts (exactly num each
+  // unless Alg. 6's threshold cutoff ran: then loaded in parallel, summed by one thread)
+  if (tid < nenum) scnt[tid + 1] = V.cnt_fixed ? V.num : __ldcg(V.cntp[V.pairs ? 2 * tid : tid]);
+  if (tid == 0) s_nq = 0;
+  __syncthreads();
   if (tid == 0) {
-    int acc = 0;
-    s_nq = 0;
     scnt[0] = 0;
-    for (int e = 0; e < nenum; ++e) {
-      acc += __ldcg(V.cntp[V.pairs ? 2 * e : e]);
-      scnt[e + 1] = acc;
-    }
+    for (int e = 0; e < nenum; ++e) scnt[e + 1] += scnt[e];
   }
   // slot parameters of the lanes' estimation slots
   SlotParam sp0{0, 0, 0, 0}, sp1{0, 0, 0, 0};
@@ -450,6 +456,7 @@ __global__ void __launch_bounds__(kTailNT, 4) k_tail(TailArgs A) {
     if (LP == 32 && lane + 32 < A.e.L) sp1 = A.e.slots[lane + 32];
   }
   __syncthreads();
+  if (V.pk) mbar_wait(&tbar, 0);
   if (blockIdx.x == 0) TRACE(31);
 #ifdef CUSFFT_TRACE
   const long long c_vote0 = clock64();

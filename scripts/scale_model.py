@@ -4,8 +4,8 @@ per-rank compute MEASURED on one B200.
 For each G the script builds rank 0's plan of a G-rank loop-sharded run
 (cusfft_plan_dist without a communicator), and times on the bench's terms
 (L2 flushed before every step, CUDA events, graphs):
-  local  = cusfft_execute_local  (Steps 1-4 of this rank's L/G loops)
-  finish = cusfft_execute_finish (vote + estimation + output over all L loops)
+  local  = cusfft_execute_local  (Steps 1-4 of this rank's L/G loops, one serial chain)
+  finish = (local + cusfft_execute_finish) - local (vote + estimation + output over all L loops)
 The exchange buffer is filled with the records of a world = 1 plan of the same
 draws (the all-gather's result), so finish does the real work.  The
 all-gather itself cannot be timed on one GPU: it is modelled as
@@ -75,15 +75,20 @@ for G in (1, 2, 4, 8):
     buf = torch.as_tensor(__import__("paper_conf_ipps_wangcc16_b200.dist", fromlist=["_CudaBuffer"])._CudaBuffer(
         ptr, per * G), device=dev)
     local_us = timed(lambda: p.execute_local(x))
-    # the all-gather's result: every loop's record at its loop-sharded slot
+    # the all-gather's result: every loop's record at its loop-sharded slot (the local steps
+    # rewrite only this rank's slice, so the other slices stay in place across repetitions)
     for r in range(L):
         s = slot_of_loop(r, L, G)
         buf[s * rec_bytes:(s + 1) * rec_bytes].copy_(ref_buf[r * rec_bytes:(r + 1) * rec_bytes])
     torch.cuda.synchronize()
     l2 = torch.empty_like(locs)
     v2 = torch.empty_like(vals)
-    finish_us = timed(lambda: p.execute_finish(l2, v2))
-    p.execute_finish(l2, v2)
+
+    def both():  # the per-execution counters are reset by the local steps' first kernel
+        p.execute_local(x)
+        p.execute_finish(l2, v2)
+    finish_us = timed(both) - local_us
+    both()
     torch.cuda.synchronize()
     same = torch.equal(l2, locs) and torch.equal(v2, vals)
     ag_bytes = per * G
