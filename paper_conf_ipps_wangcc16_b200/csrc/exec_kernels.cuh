@@ -269,7 +269,7 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict_
 // ---------------------------------------------------------------------------
 // RMAX: taps held in registers (8 when R <= 8, else 16; rounds beyond reload theirs).
 template <int B1T, int RMAX>
-__global__ void __launch_bounds__(256, 3) k_fold_fft1_tma(const double2* __restrict__ staging,
+__global__ void __launch_bounds__(256, 2) k_fold_fft1_tma(const double2* __restrict__ staging,
                                                           const double* __restrict__ taps_perm,
                                                           double2* __restrict__ u, double2* __restrict__ v,
                                                           const double2* __restrict__ tw, int B, int B2, int w, int R,

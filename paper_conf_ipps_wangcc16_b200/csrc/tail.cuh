@@ -82,10 +82,11 @@ __device__ void output_body(uint8_t* smem, const int* __restrict__ hits, const u
   int* bstart = bcnt + 1024;                                     // 1024 bucket starts
   const int tid = threadIdx.x, lane = tid & 31;
   CTRACE(80);
-  // Every load of the fast path is issued before the first barrier: the
-  // hit count, the level-0 histogram (other CTAs of k_tail counted into it;
-  // copied to shared memory) and up to PF items per thread (keys, f, values),
-  // read speculatively below max_hits and masked once H is known.
+  // The first loads of the fast path are issued before the first barrier: the
+  // hit count, the level-0 histogram (counted by the estimation; copied to
+  // shared memory) and up to PF keys per thread, read speculatively below
+  // max_hits and masked once H is known.  f and the value are loaded only for
+  // the selected items.
   constexpr int PF = 4;  // fast path: H <= PF * 1024 items, kp2 <= 1024
   uint32_t* h0 = reinterpret_cast<uint32_t*>(smem + output_smem_bytes(kp2));
   double2* selv = reinterpret_cast<double2*>(ckey);  // [kp2] values of the selected entries (fast path)
@@ -99,11 +100,7 @@ __device__ void output_body(uint8_t* smem, const int* __restrict__ hits, const u
 #pragma unroll
   for (int u = 0; u < PF; ++u) {
     const int i = u * 1024 + tid;
-    if (i < max_hits) {
-      pk[u] = __ldcg(hit_keys + i);
-      pf[u] = (uint32_t)__ldcg(hits + i);
-      pv[u] = __ldcg(hit_vals + i);
-    }
+    if (i < max_hits) pk[u] = __ldcg(hit_keys + i);
   }
 #pragma unroll
   for (int j = 0; j < 4; ++j) h0[tid + j * 1024] = hb[j];
@@ -135,6 +132,10 @@ __device__ void output_body(uint8_t* smem, const int* __restrict__ hits, const u
         const int i = u * 1024 + tid;
         take[u] = i < H && ((uint32_t)(pk[u] >> 51) & 0xFFFu) >= d0;
         cnt += take[u];
+        if (take[u]) {  // in flight across the scan's barriers
+          pf[u] = (uint32_t)__ldcg(hits + i);
+          pv[u] = __ldcg(hit_vals + i);
+        }
       }
       int total;
       int pos = block_excl_scan<1024>(cnt, &total, sm);
@@ -461,9 +462,6 @@ __global__ void __launch_bounds__(kTailNT, 4) k_tail(TailArgs A) {
 #ifdef CUSFFT_TRACE
   const long long c_vote0 = clock64();
 #endif
-  uint32_t sig_r[LL > 0 ? LL : 1];
-#pragma unroll
-  for (int qq = 0; qq < (LL > 0 ? LL : 1); ++qq) sig_r[qq] = LL > 0 ? ssig[qq] : 0u;
   uint32_t tab_s;
   asm volatile("mov.u32 %0, %1;" : "=r"(tab_s) : "r"(smem_u32(smem)));
   uint16_t* q = reinterpret_cast<uint16_t*>(smem + A.q_off) + wid * kTailQ;
@@ -532,10 +530,10 @@ __global__ void __launch_bounds__(kTailNT, 4) k_tail(TailArgs A) {
           const uint32_t F = a * ((p0 + c0 + (uint32_t)q[b0 + lane]) << sh);
           f = F >> sh;
           uint32_t bits = 0u;
-          if (LL > 0) {  // compile-time L_loc: unrolled, sigmas in registers
+          if (LL > 0) {  // compile-time L_loc: unrolled (sigmas by broadcast shared loads)
 #pragma unroll
             for (int qq = 0; qq < (LL > 0 ? LL : 1); ++qq)
-              bits |= tab_at<ET>(tab_s, (sig_r[qq] * F + half_s) >> bsh) & (1u << qq);
+              bits |= tab_at<ET>(tab_s, (ssig[qq] * F + half_s) >> bsh) & (1u << qq);
           } else {
             for (int qq = 0; qq < Lloc; ++qq) bits |= tab_at<ET>(tab_s, (ssig[qq] * F + half_s) >> bsh) & (1u << qq);
           }
