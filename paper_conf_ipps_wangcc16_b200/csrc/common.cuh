@@ -24,13 +24,33 @@ __device__ __forceinline__ unsigned long long gtimer() {
   do { if (threadIdx.x == 0) atomicMax(&g_trace[(slot)], gtimer()); } while (0)
 // Per-kernel span: g_trace[128 + 2 id] = earliest CTA start (after pdl_wait),
 // g_trace[129 + 2 id] = latest CTA end (thread 0; any return path).
+// Per-CTA records (start, end, id | smid << 8 | linear block << 16) in g_cta.
+constexpr int kCtaTraceMax = 16384;
+__device__ unsigned g_cta_n;
+__device__ unsigned long long g_cta[3 * kCtaTraceMax];
 struct KTraceScope {
   int id;
-  __device__ explicit KTraceScope(int i) : id(i) {
-    if (threadIdx.x == 0) atomicMin(&g_trace[128 + 2 * id], gtimer());
+  unsigned long long t0;
+  __device__ explicit KTraceScope(int i) : id(i), t0(0) {
+    if (threadIdx.x == 0) {
+      t0 = gtimer();
+      atomicMin(&g_trace[128 + 2 * id], t0);
+    }
   }
   __device__ ~KTraceScope() {
-    if (threadIdx.x == 0) atomicMax(&g_trace[129 + 2 * id], gtimer());
+    if (threadIdx.x == 0) {
+      const unsigned long long t1 = gtimer();
+      atomicMax(&g_trace[129 + 2 * id], t1);
+      unsigned smid;
+      asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+      const unsigned i = atomicAdd(&g_cta_n, 1u);
+      if (i < kCtaTraceMax) {
+        g_cta[3 * i] = t0;
+        g_cta[3 * i + 1] = t1;
+        g_cta[3 * i + 2] = (unsigned long long)id | ((unsigned long long)smid << 8) |
+                           ((unsigned long long)(blockIdx.x + blockIdx.y * gridDim.x) << 16);
+      }
+    }
   }
 };
 #define KTRACE(id) KTraceScope ktrace_scope_(id)

@@ -1760,12 +1760,25 @@ int cusfft_debug_trace(unsigned long long* host, int32_t n) {
   CK(cudaMemcpyFromSymbol(host, g_trace, sizeof(unsigned long long) * (n < 256 ? n : 256)));
   return CUSFFT_SUCCESS;
 }
+// Trace builds only: per-CTA records (3 u64 each, common.cuh KTraceScope); returns the count.
+int cusfft_debug_cta_trace(unsigned long long* host, int32_t max_records) {
+  if (!host) return CUSFFT_NULL_PTR;
+  CK(cudaDeviceSynchronize());
+  unsigned n = 0;
+  CK(cudaMemcpyFromSymbol(&n, g_cta_n, sizeof(n)));
+  int m = (int)(n < (unsigned)kCtaTraceMax ? n : (unsigned)kCtaTraceMax);
+  if (m > max_records) m = max_records;
+  if (m > 0) CK(cudaMemcpyFromSymbol(host, g_cta, sizeof(unsigned long long) * 3 * (size_t)m));
+  return m;
+}
 // Reset the trace: phase slots 0, per-kernel start slots (128 + 2 id) ~0.
 int cusfft_debug_trace_reset() {
   unsigned long long init[256];
   for (int i = 0; i < 256; ++i) init[i] = (i >= 128 && (i % 2) == 0) ? ~0ull : 0ull;
   CK(cudaDeviceSynchronize());
   CK(cudaMemcpyToSymbol(g_trace, init, sizeof(init)));
+  const unsigned zero = 0;
+  CK(cudaMemcpyToSymbol(g_cta_n, &zero, sizeof(zero)));
   return CUSFFT_SUCCESS;
 }
 #endif

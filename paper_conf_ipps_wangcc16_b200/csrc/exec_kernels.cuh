@@ -314,9 +314,18 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1_tma(const double2* __restr
   const int wc = t % C, wj = t / C;  // writer's (column, row)
   const double2 wv = __ldg(tw + (((int64_t)(blockIdx.x * C + wc) * wj) & (B - 1)));
   __syncthreads();  // barrier init visible to every thread
+#ifdef CUSFFT_TRACE
+  const long long fc0 = clock64();
+  const int fsel = blockIdx.y * gridDim.x + blockIdx.x;
+  if (t == 0) atomicMax(&g_trace[112 + (zero.p != nullptr)], gtimer());  // latest CTA start (per launch)
+#endif
   for (int i = 0; i < ns; ++i) {
     const double2* T = Tile + (size_t)(i & 1) * R * 256;
     mbar_wait(bar + (i & 1), (uint32_t)((i >> 1) & 1));
+#ifdef CUSFFT_TRACE
+    if (i == 0) CTRACE_MAX(114, clock64() - fc0);  // first slot's rows landed
+    const long long fc1 = clock64();
+#endif
     double ar = 0.0, ai = 0.0;
 #pragma unroll
     for (int rr = 0; rr < RMAX; ++rr) {
@@ -343,7 +352,14 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1_tma(const double2* __restr
     fft_smem<B1T, 256, 256, true>(S, twl, B1T);
     v[wpos] = cmul(S[fft_pad(wc * B1T + wj)], wv);
     __syncthreads();  // S is rewritten by the next slot
+#ifdef CUSFFT_TRACE
+    CTRACE_MAX(115, clock64() - fc1);  // one slot's fold + column FFT
+#endif
   }
+#ifdef CUSFFT_TRACE
+  CTRACE_MAX(116, clock64() - fc0);
+  (void)fsel;
+#endif
   TRACE_END(1);
 }
 
@@ -803,9 +819,12 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
   }
   }
   if (sel == 0 && r == 0) TRACE(11);
-  // 3. classify my keys: bitmap words in my smem, candidates appended to CTA 0
+  // 3. classify my keys: bitmap words in my smem, candidates appended to CTA 0,
+  //    my count of keys taken outright pushed to every CTA
   SelClusterSmem* S0 = cl.map_shared_rank(&S, 0);
   const unsigned lt = (1u << lane) - 1u;
+  if (tid == 0) S.sm[44] = 0;
+  __syncthreads();
   for (int cb = 0; cb < per; cb += KC * kSelCNT) {
     if (cb > 0) {
 #pragma unroll
@@ -822,7 +841,10 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
       const bool take = i < per && (A.threshold_mode ? kb[u] >= A.thr_key : (d > (uint32_t)d0 || (d == (uint32_t)d0 && whole)));
       const bool cand = i < per && !A.threshold_mode && d == (uint32_t)d0 && !whole;
       const uint32_t word = __ballot_sync(kFull, take);
-      if (lane == 0 && i < per) sbits[i >> 5] = word;  // per is a multiple of 32: whole warps in or out
+      if (lane == 0 && i < per) {  // per is a multiple of 32: whole warps in or out
+        sbits[i >> 5] = word;
+        atomicAdd(&S.sm[44], __popc(word));
+      }
       const unsigned cm = __ballot_sync(kFull, cand);
       if (cm) {
         int bpos = 0;
@@ -838,11 +860,25 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
       }
     }
   }
+  __syncthreads();
+  if (tid < kSelCL) cl.map_shared_rank(&S, tid)->cnt[r] = S.sm[44];
   cl.sync();
   if (sel == 0 && r == 0) TRACE(12);
-  // 4. every CTA resolves its own candidates against the whole list
+  // 4. the boundary bin's candidates.  Few (<= kSelCNT, the usual case): every
+  //    CTA copies the whole list, ranks every candidate and so knows every
+  //    CTA's final count (no further cluster round; CTA 0's list must outlive
+  //    the copies: arrive on a split cluster barrier now, wait before exit).
+  //    Many: every CTA resolves its own candidates, counts pushed in one more
+  //    cluster round.
+#ifdef CUSFFT_TRACE
+  if (r == 0 && tid == 0 && sel < 16) g_trace[96 + sel] = (unsigned long long)S0->ncand | ((unsigned long long)whole << 32);
+#endif
+  const int nc = whole ? 0 : S0->ncand;
+  const bool few = nc <= kSelCNT;
+  int wins[kSelCL];
+#pragma unroll
+  for (int c = 0; c < kSelCL; ++c) wins[c] = 0;
   if (!whole) {
-    const int nc = S0->ncand;
     Prefix96 p{0, 0, 0, 0};
     or96(p.phi, p.plo, (uint32_t)d0, pass_shift(0));
     or96(p.mhi, p.mlo, 0xFFFu, pass_shift(0));
@@ -852,13 +888,17 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
           S.ckey[c] = S0->ckey[c];
           S.cidx[c] = S0->cidx[c];
         }
+      if (few) asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+      if (tid < kSelCL) S.part[tid] = 0;  // winners per CTA (reuses the slice totals)
       __syncthreads();
-      if (nc <= kSelCNT) {  // warp per candidate of mine, lanes split the comparisons
+      if (few) {  // warp per candidate (every candidate), lanes split the comparisons
         for (int j = tid >> 5; j < nc; j += kSelCNT / 32) {
           const int mi = S.cidx[j];
-          if (mi < k0 || mi >= k0 + per) continue;  // warp-uniform
           const int rank = warp_rank(S.ckey, S.cidx, nc, S.ckey[j], mi);
-          if (lane == 0 && rank < k2) atomicOr(&sbits[(mi - k0) >> 5], 1u << (mi & 31));
+          if (lane == 0 && rank < k2) {
+            atomicAdd(&S.part[mi / per], 1);
+            if (mi >= k0 && mi < k0 + per) atomicOr(&sbits[(mi - k0) >> 5], 1u << (mi & 31));
+          }
         }
       } else {
         p = block_radix_select<PairSrc, kSelCNT>(PairSrc{S.ckey, S.cidx}, nc, k2, S.hist, S.sm, 1, p, false);
@@ -876,22 +916,29 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
       }
     }
     __syncthreads();
+    if (few) {
+#pragma unroll
+      for (int c = 0; c < kSelCL; ++c) wins[c] = S.part[c];
+    }
   }
-  // my winner count, pushed to every CTA
   const int wpt = (wpc + kSelCNT - 1) / kSelCNT;
   int cnt = 0;
   for (int w = tid * wpt; w < min(wpc, (tid + 1) * wpt); ++w) cnt += __popc(sbits[w]);
   int mine;
   int pos = block_excl_scan<kSelCNT>(cnt, &mine, S.sm);
-  if (tid < kSelCL) cl.map_shared_rank(&S, tid)->cnt[r] = mine;
-  cl.sync();
+  if (!whole && !few) {  // resolved locally: my final count to every CTA
+    if (tid < kSelCL) cl.map_shared_rank(&S, tid)->cnt[r] = mine;
+    cl.sync();
+  }
   if (sel == 0 && r == 0) TRACE(13);
   // 5. bitmap words and my part of the ascending J
   int jofs = 0, total = 0;
+  const bool exact_counts = whole || few;  // S.cnt holds taken-outright counts; add the candidate winners
 #pragma unroll
   for (int c = 0; c < kSelCL; ++c) {
-    jofs += c < r ? S.cnt[c] : 0;
-    total += S.cnt[c];
+    const int cc = S.cnt[c] + (exact_counts ? wins[c] : 0);
+    jofs += c < r ? cc : 0;
+    total += cc;
   }
   uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap) + r * wpc;
   int* J = reinterpret_cast<int*>(rec + A.lay.off_J);
@@ -931,6 +978,7 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
     if (!A.threshold_mode && total != A.num) atomicOr(A.status + 1, 1);
   }
   if (sel == 0 && r == 0) TRACE(14);
+  if (!whole && few && nc <= kSelCap) asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
   // (no remote smem access after the last barrier: CTAs may exit)
 }
 

@@ -39,7 +39,9 @@ for rep in range(reps):
     if rep == reps - 1:
         phases = {i: (t[i] - t0) / 1e3 for i in range(96) if t[i] > 0}
         print("phase slots (us):", " ".join(f"{i}:{v:.2f}" for i, v in sorted(phases.items(), key=lambda kv: kv[1])))
-        print("select candidates per loop:", [int(t[96 + i]) & 0xFFFFFFFF for i in range(16) if t[96 + i] > 0])
+        print("select candidates per loop:", [int(t[96 + i]) & 0xFFFFFFFF for i in range(16) if 0 < t[96 + i] < 2**40])
+        print("fold_fft1: latest CTA start (us) loc/est", [(t[112 + q] - t0) / 1e3 for q in (0, 1) if t[112 + q] > 0],
+              "cycles: first rows landed", int(t[114]), "slot compute", int(t[115]), "CTA", int(t[116]))
         cyc = {i: int(t[i]) for i in range(64, 96) if t[i] > 0}
         if cyc:
             print("tail cycles: vote(w0 max)", cyc.get(70), "vote(CTA max)", cyc.get(71), "estimate(CTA max)", cyc.get(72))
@@ -47,6 +49,23 @@ for rep in range(reps):
             if all(o):
                 print("output phases (cycles): load", o[1] - o[0], "pick", o[2] - o[1], "classify", o[3] - o[2],
                       "count+scan+scatter", o[4] - o[3], "insertion", o[5] - o[4], "write", o[6] - o[5], "total", o[6] - o[0])
+    if rep == reps - 1 and hasattr(lib, "cusfft_debug_cta_trace"):
+        cbuf = (ctypes.c_ulonglong * (3 * 16384))()
+        m = lib.cusfft_debug_cta_trace(cbuf, 16384)
+        rec = np.array(list(cbuf)[:3 * m], dtype=np.uint64).reshape(-1, 3) if m > 0 else np.zeros((0, 3), np.uint64)
+        print(f"per-CTA records: {m}")
+        for kid in sorted(set(int(r) & 0xFF for r in rec[:, 2])):
+            sel_ = rec[(rec[:, 2] & np.uint64(0xFF)) == np.uint64(kid)]
+            st = (sel_[:, 0].astype(np.float64) - t0) / 1e3
+            en = (sel_[:, 1].astype(np.float64) - t0) / 1e3
+            du = en - st
+            q = lambda a: " ".join(f"{np.percentile(a, p):6.2f}" for p in (0, 10, 50, 90, 100))
+            print(f"  {names.get(kid, kid)!s:16s} n={len(st):4d} start[0,10,50,90,100] {q(st)} | end {q(en)} | dur {q(du)}")
+            lo, hi = int(np.floor(st.min())), int(np.ceil(en.max()))
+            hist = [int(((st >= b) & (st < b + 1)).sum()) for b in range(lo, hi)]
+            live = [int(((st < b + 1) & (en > b)).sum()) for b in range(lo, hi)]
+            print(f"  {'':16s} starts/us from {lo}: {hist}")
+            print(f"  {'':16s} live CTAs/us     : {live}")
     for i, (s, e) in spans.items():
         acc.setdefault(i, []).append(((s - t0) / 1e3, (e - t0) / 1e3))
     acc.setdefault(0, []).append((0.0, (end - t0) / 1e3))
