@@ -202,6 +202,7 @@ struct cusfft_plan_s {
   uint32_t* d_hist = nullptr;     // [n_sel][4096] top-digit histograms (zero block)
   int* d_key_index = nullptr;     // [Lg] local slot -> selection index or -1
   uint32_t* d_ohist = nullptr;    // [4096] top-digit histogram of the output keys (zero block)
+  bool fft2sel = true;             // location slots' FFT pass 2 fused with the cutoff when the shape allows (use_fft2_select)
   bool sel_cluster = false;       // k_select_cluster (256 <= B <= 65536, EXACT / THRESHOLD modes)
   int select1_smem = 0;
   // fused vote + estimate + output (k_tail) when its table fits shared memory
@@ -610,7 +611,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   P->max_hits = (int)q.max_hits;
   if (const char* e = std::getenv("CUSFFT_NO_GRAPH")) P->use_graph = !(e[0] == '1');                    // A/B (measurement)
   if (const char* e = std::getenv("CUSFFT_P2_SPC")) P->p2_spc = std::max(1, std::min(8, std::atoi(e)));  // A/B (measurement)
-  if (const char* e = std::getenv("CUSFFT_FORK")) P->fork_at = e[0] == '1' ? 1 : 0;                       // A/B (measurement)
+  if (const char* e = std::getenv("CUSFFT_FFT2SEL")) P->fft2sel = std::atoi(e) != 0;                     // A/B (measurement)
+  if (const char* e = std::getenv("CUSFFT_FORK")) P->fork_at = std::atoi(e);                                 // A/B (measurement)
   // ---- filters (group 0: location loops; group 1: estimation-only loops)
   {
     const double tl = q.loc_tolerance > 0.0 ? q.loc_tolerance : q.tolerance;
@@ -751,6 +753,9 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   attr(set_dyn_smem(k_select1, smem_optin, smem_optin));
   attr(set_dyn_smem(k_select_cluster, 200 * 1024, smem_optin));
   attr(set_dyn_smem(k_select_sort, 210 * 1024, smem_optin));
+  attr(set_dyn_smem(k_fft2_select<64, 16>, fft2sel_smem_bytes<64, 16>(), smem_optin));
+  attr(set_dyn_smem(k_fft2_select<128, 16>, fft2sel_smem_bytes<128, 16>(), smem_optin));
+  attr(set_dyn_smem(k_fft2_select<128, 32>, fft2sel_smem_bytes<128, 32>(), smem_optin));
   attr(set_dyn_smem(k_vote, smem_optin, smem_optin));
   attr(set_dyn_smem(k_output, smem_optin, smem_optin));
   if (P->tail_esz) attr(set_dyn_smem(tail_kernel(P->tail_esz, L, P->Lloc), P->tail_smem, smem_optin));
@@ -1048,6 +1053,60 @@ int launch_select(cusfft_plan_t P, cudaStream_t st) {
   return CUSFFT_SUCCESS;
 }
 
+// FFT pass 2 + cutoff of the location slots in one cluster kernel
+// (k_fft2_select): exact mode, four-step B with B1 = 8 ROWS, the selected
+// slots = this rank's location slots [0, nloc_local) in order, shapes with
+// compiled instances (B = 8192, 16384, 32768).
+bool use_fft2_select(cusfft_plan_t P) {
+  if (!P->sel_cluster || P->xshard || P->prm.cutoff_mode != CUSFFT_CUTOFF_EXACT || P->B1 <= 1 || !P->fft2sel)
+    return false;
+  const int key = P->B2 * 1000 + P->B1 / kSelCL;
+  if (key != 64016 && key != 128016 && key != 128032) return false;
+  if ((int)P->sel_slots_h.size() != P->nloc_local) return false;
+  for (int i = 0; i < P->nloc_local; ++i)
+    if (P->sel_slots_h[(size_t)i] != (int64_t)P->lrank * P->Lg + i) return false;
+  return true;
+}
+
+template <int M, int ROWS>
+cudaError_t launch_f2s_t(cusfft_plan_t P, const Fft2SelArgs& fa, int nsel, cudaStream_t st) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(nsel * kSelCL));
+  cfg.blockDim = dim3(kF2SNT);
+  cfg.dynamicSmemBytes = (size_t)fft2sel_smem_bytes<M, ROWS>();
+  cfg.stream = st;
+  cudaLaunchAttribute attr[3];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = kSelCL;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = g_pdl ? 1 : 0;
+  attr[2].id = cudaLaunchAttributePriority;
+  attr[2].val.priority = P->cur_prio;
+  cfg.attrs = attr;
+  cfg.numAttrs = 3;
+  return cudaLaunchKernelEx(&cfg, k_fft2_select<M, ROWS>, fa);
+}
+
+int launch_fft2_select(cusfft_plan_t P, cudaStream_t st) {
+  const int nsel = (int)P->sel_slots_h.size();
+  if (nsel == 0) return CUSFFT_SUCCESS;
+  Fft2SelArgs fa{};
+  fa.s = make_sel_args(P);
+  for (int i = 0; i < nsel; ++i) fa.v[i] = P->d_v + (size_t)i * P->B;
+  fa.tw = P->d_tw;
+  fa.B1 = P->B1;
+  cudaError_t e = cudaErrorInvalidValue;
+  switch (P->B2 * 1000 + P->B1 / kSelCL) {
+    case 64016: e = launch_f2s_t<64, 16>(P, fa, nsel, st); break;
+    case 128016: e = launch_f2s_t<128, 16>(P, fa, nsel, st); break;
+    case 128032: e = launch_f2s_t<128, 32>(P, fa, nsel, st); break;
+  }
+  CK(e);
+  return CUSFFT_SUCCESS;
+}
+
 // Cutoff keys from the summed spectra (signal-sharded plans, after the exchange).
 int launch_keys(cusfft_plan_t P, cudaStream_t st) {
   if (P->sel_slots_h.empty()) return CUSFFT_SUCCESS;
@@ -1181,10 +1240,14 @@ int launch_local(cusfft_plan_t P, const double2* x) {
   g_pdl = P->timing != 1;
   mark(P, 1);
   if (P->stage_limit < 2) return CUSFFT_SUCCESS;
-  TRY(launch_bfft(P, 0, P->Lg, st));
+  const bool f2s = use_fft2_select(P) && P->stage_limit >= 3;
+  TRY(launch_bfft(P, f2s ? P->nloc_local : 0, P->Lg, st));  // fused: the location slots' pass 2 runs with their cutoff
   mark(P, 2);
   if (P->stage_limit < 3 || P->xshard) return CUSFFT_SUCCESS;  // signal-sharded: cutoff after the all-reduce
-  TRY(launch_select(P, st));
+  if (f2s)
+    TRY(launch_fft2_select(P, st));
+  else
+    TRY(launch_select(P, st));
   mark(P, 3);
   return CUSFFT_SUCCESS;
 }
@@ -1257,8 +1320,14 @@ int launch_branched(cusfft_plan_t P, const double2* x, int64_t* locs, double2* v
   g_pdl = true;
   TRY(launch_fold_range(P, x, 0, nl, a, false));
   if (P->fork_at == 1) TRY(fork());
-  if (lim >= 2) TRY(launch_bfft(P, 0, nl, a));
-  if (lim >= 3 && !P->xshard) TRY(launch_select(P, a));
+  const bool f2s = use_fft2_select(P) && lim >= 3;
+  if (lim >= 2 && !f2s) TRY(launch_bfft(P, 0, nl, a));
+  if (P->fork_at == 2) TRY(fork());
+  if (f2s)
+    TRY(launch_fft2_select(P, a));
+  else if (lim >= 3 && !P->xshard)
+    TRY(launch_select(P, a));
+  if (P->fork_at == 3) TRY(fork());
   P->cur_prio = 0;
   CK(cudaStreamWaitEvent(a, P->ev_join, 0));
   g_pdl = false;
@@ -1789,8 +1858,10 @@ int32_t cusfft_launches_per_execute(cusfft_plan_t plan) {
   const int ranges = (nl > 0) + (ne > 0);
   const bool pass1 = plan->B1 > 1 && !plan->fused1;
   const bool branched = use_branches(plan);
+  const bool f2s = use_fft2_select(plan) && plan->stage_limit >= 3;  // location pass 2 inside the cutoff kernel
+  const int ffts = f2s ? (ne > 0 ? 1 : 0) : (branched ? ranges : 1);
   int n = (plan->staged ? 1 : 0) + ranges /*fold per slot range*/ +
-          (branched ? ranges : 1) * (pass1 ? 2 : 1) /*fft*/ + (plan->sel_slots_h.empty() ? 0 : 1) +
+          ffts * (pass1 ? 2 : 1) /*fft*/ + (plan->sel_slots_h.empty() ? 0 : 1) +
           (plan->xshard && !plan->sel_slots_h.empty() ? 1 : 0) /*keys*/ + (plan->tail_esz ? 2 : 3);
   return n;
 }

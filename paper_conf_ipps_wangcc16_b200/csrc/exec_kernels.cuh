@@ -604,17 +604,35 @@ __device__ __forceinline__ int warp_rank(const uint64_t* ck, const int* ci, int 
 
 constexpr int kSel1MaxB = 65536;
 
-__global__ void __launch_bounds__(1024) k_select1(SelArgs A) {
-  pdl_wait();
-  KTRACE(8);
-  extern __shared__ __align__(16) uint8_t smem[];
+// k_tail's vote table (element b, pk_esz bytes = bucket b; bit sel = kept in
+// location loop sel): OR in the 32 buckets from b0 of one bitmap word.
+__device__ __forceinline__ void pk_or_word(const SelArgs& A, int sel, uint32_t bits, int64_t b0) {
+  if (!bits) return;
+  if (A.pk_esz == 1) {  // 4 buckets per u32: spread each nibble of bits over 4 bytes
+    uint32_t* dst = A.pk + b0 / 4;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const uint32_t nib = (bits >> (4 * j)) & 0xFu;
+      if (nib) atomicOr(dst + j, ((nib * 0x00204081u) & 0x01010101u) << sel);
+    }
+  } else {
+    for (uint32_t bb = bits; bb; bb &= bb - 1) {
+      const int64_t bkt = b0 + __ffs(bb) - 1;
+      const int per = 4 / A.pk_esz;  // buckets per u32 word
+      atomicOr(A.pk + bkt / per, (1u << sel) << (8 * A.pk_esz * (int)(bkt % per)));
+    }
+  }
+}
+
+// The whole single-CTA selection of slot `sel` (blockDim 1024); write_pk: also
+// OR the winners into k_tail's vote table (when called as a cluster cutoff's fallback).
+__device__ __forceinline__ void select1_body(const SelArgs& A, int sel, uint8_t* smem, bool write_pk) {
   uint32_t* hist = reinterpret_cast<uint32_t*>(smem);
   int* sm = reinterpret_cast<int*>(smem + 4096 * 4);
   uint64_t* skey = reinterpret_cast<uint64_t*>(smem + 4096 * 4 + 64 * 4);
   int* sidx = reinterpret_cast<int*>(skey + kSelCap);
   uint32_t* sbits = reinterpret_cast<uint32_t*>(sidx + kSelCap);
   const int tid = threadIdx.x, lane = tid & 31;
-  const int sel = blockIdx.x;
   const int B = A.B;
   uint8_t* rec = A.recs[sel];
   const uint64_t* keys = A.keys + (int64_t)sel * B;
@@ -693,7 +711,10 @@ __global__ void __launch_bounds__(1024) k_select1(SelArgs A) {
   // bitmap out + ascending winner list (thread t owns words [t wpt, (t+1) wpt))
   uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap);
   int* J = reinterpret_cast<int*>(rec + A.lay.off_J);
-  for (int w = tid; w < words; w += 1024) bitmap[w] = sbits[w];
+  for (int w = tid; w < words; w += 1024) {
+    bitmap[w] = sbits[w];
+    if (write_pk && A.pk) pk_or_word(A, sel, sbits[w], (int64_t)w * 32);
+  }
   const int wpt = (words + 1023) / 1024;
   int cnt = 0;
   for (int w = tid * wpt; w < min(words, (tid + 1) * wpt); ++w) cnt += __popc(sbits[w]);
@@ -712,6 +733,13 @@ __global__ void __launch_bounds__(1024) k_select1(SelArgs A) {
     if (!A.threshold_mode && total != A.num) atomicOr(A.status + 1, 1);
   }
   if (sel == 0) TRACE(14);
+}
+
+__global__ void __launch_bounds__(1024) k_select1(SelArgs A) {
+  pdl_wait();
+  KTRACE(8);
+  extern __shared__ __align__(16) uint8_t smem[];
+  select1_body(A, blockIdx.x, smem, false);
 }
 
 // ---------------------------------------------------------------------------
@@ -744,6 +772,249 @@ struct SelClusterSmem {
   int cnt[kSelCL];              // final winners per CTA (pushed to every CTA)
 };
 
+// Step 5 of the cluster selection: this CTA's bitmap words, its vote-table
+// bits, its part of the ascending J (from position pos) and the count.
+template <int NT = kSelCNT>
+__device__ __forceinline__ void select_cluster_write(const SelArgs& A, uint8_t* rec, const uint32_t* sbits, int sel,
+                                                     int r, int wpc, int wpt, int k0, int pos, int total) {
+  const int tid = threadIdx.x;
+  uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap) + r * wpc;
+  int* J = reinterpret_cast<int*>(rec + A.lay.off_J);
+  for (int w = tid; w < wpc; w += NT) bitmap[w] = sbits[w];
+  if (A.pk)  // k_tail's vote table
+    for (int w = tid; w < wpc; w += NT) pk_or_word(A, sel, sbits[w], (int64_t)(r * wpc + w) * 32);
+  for (int w = tid * wpt; w < min(wpc, (tid + 1) * wpt); ++w) {
+    uint32_t bits = sbits[w];
+    while (bits) {
+      const int b = __ffs(bits) - 1;
+      bits &= bits - 1;
+      J[pos++] = k0 + w * 32 + b;
+    }
+  }
+  if (r == 0 && tid == 0) {
+    *reinterpret_cast<int*>(rec + A.lay.off_cnt) = total;
+    if (!A.threshold_mode && total != A.num) atomicOr(A.status + 1, 1);
+  }
+}
+
+// Fast form of the cluster selection (EXACT mode), one cluster barrier:
+//   1. every CTA reads the whole 4096-bin level-0 histogram and finds the
+//      boundary digit d0 itself (block scan, no exchange);
+//   2. classifies its keys (bitmap words by ballot), counts the keys taken
+//      outright and pushes that count and its boundary-bin candidates to
+//      every CTA of the cluster (remote stores);
+//   3. one cluster barrier; then every CTA holds every candidate and every
+//      take count: it ranks all candidates (ties to the smaller bucket), so it
+//      knows every CTA's final count (its J offset) without another round.
+// Returns false (uniformly over the cluster, after the barrier) when some CTA
+// holds more than kSelFastCap candidates: the caller then runs the general form.
+constexpr int kSelFastCap = 64;
+struct SelFastSmem {
+  int sm[64];
+  int take[kSelCL];                     // pushed: keys taken outright by CTA c
+  int ncand[kSelCL];                    // pushed: boundary candidates of CTA c
+  uint64_t ckey[kSelCL][kSelFastCap];   // pushed: candidates of CTA c
+  int cidx[kSelCL][kSelFastCap];
+  uint64_t fkey[kSelCL * kSelFastCap];  // local: all candidates, flat
+  int fidx[kSelCL * kSelFastCap];
+  int wins[kSelCL];                     // local: winners per owner CTA
+  int lkey_n;                           // local: my candidates
+  int pick[3];                          // local: d0, above, cnt
+};
+
+static_assert(sizeof(SelFastSmem) <= sizeof(SelClusterSmem), "fast selection smem must fit the general layout");
+__device__ __forceinline__ bool select_cluster_fast(const SelArgs& A, int sel, uint8_t* smem) {
+  namespace cg = cooperative_groups;
+  cg::cluster_group cl = cg::this_cluster();
+  SelFastSmem& S = *reinterpret_cast<SelFastSmem*>(smem);
+  uint32_t* sbits = reinterpret_cast<uint32_t*>(smem + sizeof(SelClusterSmem));  // this CTA's words
+  const int tid = threadIdx.x, lane = tid & 31;
+  const int r = (int)cl.block_rank();
+  asm volatile("barrier.cluster.arrive.relaxed.aligned;" ::: "memory");  // every CTA started (before remote stores)
+  const int B = A.B;
+  const int per = B / kSelCL;
+  const int wpc = per >> 5;
+  const int k0 = r * per;
+  uint8_t* rec = A.recs[sel];
+  const uint64_t* keys = A.keys + (int64_t)sel * B;
+  const uint4* h4 = reinterpret_cast<const uint4*>(A.hist0 + (int64_t)sel * 4096) + 4 * tid;  // bins [16 tid, 16 tid + 16)
+  if (sel == 0 && r == 0) TRACE(10);
+  constexpr int KC = 8;
+  uint4 hb[4];
+#pragma unroll
+  for (int j = 0; j < 4; ++j) hb[j] = __ldcg(h4 + j);
+  uint64_t kb[KC];
+#pragma unroll
+  for (int u = 0; u < KC; ++u) {
+    const int i = u * kSelCNT + tid;
+    kb[u] = i < per ? __ldcg(keys + k0 + i) : 0ull;
+  }
+  if (tid == 0) S.lkey_n = 0;
+  // 1. boundary digit: keys in bins above thread t's 16 = exclusive scan in reversed thread order
+  uint32_t hv[16];
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    hv[4 * j] = hb[j].x; hv[4 * j + 1] = hb[j].y; hv[4 * j + 2] = hb[j].z; hv[4 * j + 3] = hb[j].w;
+  }
+  int mys = 0;
+#pragma unroll
+  for (int j = 0; j < 16; ++j) mys += (int)hv[j];
+  int tot;
+  // block_excl_scan over threads in descending order: thread t gets sum over t' > t
+  {
+    const int wid = tid >> 5;
+    // reverse within the block: lane l of warp w plays position (255 - tid)
+    int v = mys, inc = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {  // suffix scan inside the warp (lanes above)
+      const int y = __shfl_down_sync(kFull, inc, o);
+      if (lane + o < 32) inc += y;
+    }
+    if (lane == 0) S.sm[wid] = inc;  // warp total
+    __syncthreads();
+    int above_w = 0;
+#pragma unroll
+    for (int w = 0; w < kSelCNT / 32; ++w) above_w += w > wid ? S.sm[w] : 0;
+    tot = 0;
+#pragma unroll
+    for (int w = 0; w < kSelCNT / 32; ++w) tot += S.sm[w];
+    const int ex = above_w + inc - v;  // keys in bins of threads above me
+    if (ex < A.num && A.num <= ex + mys) {
+      int e = ex;
+#pragma unroll
+      for (int j = 15; j >= 0; --j) {
+        const int c = (int)hv[j];
+        if (e < A.num && A.num <= e + c) {
+          S.pick[0] = 16 * tid + j;
+          S.pick[1] = e;
+          S.pick[2] = c;
+        }
+        e += c;
+      }
+    }
+  }
+  (void)tot;
+  __syncthreads();
+  const int d0 = S.pick[0];
+  const int k2 = A.num - S.pick[1];
+  const bool whole = (k2 == S.pick[2]);
+  if (sel == 0 && r == 0) TRACE(11);
+  // 2. classify my keys; candidates to my local list (fkey/fidx as scratch)
+  const unsigned lt = (1u << lane) - 1u;
+  int mytake = 0;
+  for (int cb = 0; cb < per; cb += KC * kSelCNT) {
+    if (cb > 0) {
+#pragma unroll
+      for (int u = 0; u < KC; ++u) {
+        const int i = cb + u * kSelCNT + tid;
+        kb[u] = i < per ? __ldcg(keys + k0 + i) : 0ull;
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < KC; ++u) {
+      const int i = cb + u * kSelCNT + tid;
+      if (cb + u * kSelCNT >= per) break;
+      const uint32_t d = (uint32_t)(kb[u] >> 51) & 0xFFFu;
+      const bool take = i < per && (d > (uint32_t)d0 || (d == (uint32_t)d0 && whole));
+      const bool cand = i < per && d == (uint32_t)d0 && !whole;
+      const uint32_t word = __ballot_sync(kFull, take);
+      if (lane == 0 && i < per) sbits[i >> 5] = word;  // per is a multiple of 32
+      mytake += __popc(word);
+      const unsigned cm = __ballot_sync(kFull, cand);
+      if (cm) {
+        int bpos = 0;
+        if (lane == __ffs(cm) - 1) bpos = atomicAdd(&S.lkey_n, __popc(cm));
+        bpos = __shfl_sync(kFull, bpos, __ffs(cm) - 1);
+        if (cand) {
+          const int pos = bpos + __popc(cm & lt);
+          if (pos < kSelFastCap) {
+            S.fkey[pos] = kb[u];
+            S.fidx[pos] = k0 + i;
+          }
+        }
+      }
+    }
+  }
+  if (lane == 0) S.sm[8 + (tid >> 5)] = mytake;  // warp totals (every lane holds the warp's count)
+  __syncthreads();
+  const int nmine = S.lkey_n;
+  asm volatile("barrier.cluster.wait.aligned;" ::: "memory");  // every CTA has started: remote stores allowed
+  if (tid < kSelCL) {
+    int t = 0;
+#pragma unroll
+    for (int w = 0; w < kSelCNT / 32; ++w) t += S.sm[8 + w];
+    SelFastSmem* D = cl.map_shared_rank(&S, tid);
+    D->take[r] = t;
+    D->ncand[r] = nmine;
+  }
+  const int ncopy = min(nmine, kSelFastCap);
+  for (int j = tid; j < ncopy * kSelCL; j += kSelCNT) {
+    const int c = j / ncopy, q = j - c * ncopy;
+    SelFastSmem* D = cl.map_shared_rank(&S, c);
+    D->ckey[r][q] = S.fkey[q];
+    D->cidx[r][q] = S.fidx[q];
+  }
+  cl.sync();
+  if (sel == 0 && r == 0) TRACE(12);
+  // 3. every candidate and every take count are here
+  int nc = 0, offs[kSelCL];
+  bool over = false;
+#pragma unroll
+  for (int c = 0; c < kSelCL; ++c) {
+    offs[c] = nc;
+    nc += S.ncand[c];
+    over |= S.ncand[c] > kSelFastCap;
+  }
+  if (over) return false;
+  if (tid < kSelCL) S.wins[tid] = 0;
+  if (!whole) {
+    for (int j = tid; j < nc; j += kSelCNT) {
+      int c = 0, base = 0;
+#pragma unroll
+      for (int q = 1; q < kSelCL; ++q)
+        if (j >= offs[q]) {
+          c = q;
+          base = offs[q];
+        }
+      S.fkey[j] = S.ckey[c][j - base];
+      S.fidx[j] = S.cidx[c][j - base];
+    }
+    __syncthreads();
+    const int lper = __ffs(per) - 1;  // per = B / kSelCL is a power of two
+    for (int j = tid; j < nc; j += kSelCNT) {  // thread per candidate: rank = candidates preferred to it
+      const uint64_t mk = S.fkey[j];
+      const int mi = S.fidx[j];
+      int rank = 0;
+#pragma unroll 4
+      for (int c = 0; c < nc; ++c) {
+        const uint64_t kc = S.fkey[c];  // same address for every thread: broadcast
+        rank += (kc > mk) | ((kc == mk) & (S.fidx[c] < mi));
+      }
+      if (rank < k2) {
+        atomicAdd(&S.wins[mi >> lper], 1);
+        if (mi >= k0 && mi < k0 + per) atomicOr(&sbits[(mi - k0) >> 5], 1u << (mi & 31));
+      }
+    }
+  }
+  __syncthreads();
+  int jofs = 0, total = 0;
+#pragma unroll
+  for (int c = 0; c < kSelCL; ++c) {
+    const int cc = S.take[c] + S.wins[c];
+    jofs += c < r ? cc : 0;
+    total += cc;
+  }
+  const int wpt = (wpc + kSelCNT - 1) / kSelCNT;
+  int cnt = 0;
+  for (int w = tid * wpt; w < min(wpc, (tid + 1) * wpt); ++w) cnt += __popc(sbits[w]);
+  int mine;
+  int pos = block_excl_scan<kSelCNT>(cnt, &mine, S.sm);
+  if (sel == 0 && r == 0) TRACE(13);
+  select_cluster_write(A, rec, sbits, sel, r, wpc, wpt, k0, pos + jofs, total);
+  if (sel == 0 && r == 0) TRACE(14);
+  return true;
+}
+
 // The cluster selection of location slot `sel` by the calling cluster of kSelCL
 // CTAs x kSelCNT threads; smem: sizeof(SelClusterSmem) + B / kSelCL / 8 bytes.
 // Reads keys and histograms through L2 (__ldcg): they may have been written by
@@ -751,6 +1022,7 @@ struct SelClusterSmem {
 __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, uint8_t* smem) {
   namespace cg = cooperative_groups;
   cg::cluster_group cl = cg::this_cluster();
+  if (!A.threshold_mode && select_cluster_fast(A, sel, smem)) return;
   SelClusterSmem& S = *reinterpret_cast<SelClusterSmem*>(smem);
   uint32_t* sbits = reinterpret_cast<uint32_t*>(smem + sizeof(SelClusterSmem));  // this CTA's words
   const int tid = threadIdx.x, lane = tid & 31;
@@ -766,6 +1038,12 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
   const uint64_t* keys = A.keys + (int64_t)sel * B;
   const uint32_t* h0 = A.hist0 + (int64_t)sel * 4096;
   if (sel == 0 && r == 0) TRACE(10);
+#ifdef CUSFFT_TRACE
+  const long long scs0 = clock64();
+#define SELT(slot) CTRACE_MAX(slot, clock64() - scs0)
+#else
+#define SELT(slot) do { } while (0)
+#endif
   // my keys (first chunk) and my two level-0 bins, all in flight at once
   constexpr int KC = 8;
   constexpr int BPC = 4096 / kSelCL;    // bins per CTA; thread t holds bins base, base - 1 (descending)
@@ -789,9 +1067,12 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
   //    cluster has started: the split barrier's arrive was issued at entry)
   int tot, ex = 0;
   if (!A.threshold_mode) ex = block_excl_scan<kSelCNT>(c0 + c1, &tot, S.sm);
+  SELT(117);
   asm volatile("barrier.cluster.wait.aligned;" ::: "memory");
+  SELT(118);
   if (!A.threshold_mode && tid < kSelCL) cl.map_shared_rank(&S, tid)->part[r] = tot;
   cl.sync();
+  SELT(119);
   // 2. the boundary slice (slices descending r = kSelCL-1 .. 0) finds d0 and pushes it
   if (!A.threshold_mode) {
     int above = 0, bs = 0;
@@ -813,6 +1094,7 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
         }
     }
     cl.sync();
+    SELT(120);
     d0 = S.pick[0];
     k2 = A.num - S.pick[1];
     whole = (k2 == S.pick[2]);
@@ -861,8 +1143,10 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
     }
   }
   __syncthreads();
+  SELT(121);
   if (tid < kSelCL) cl.map_shared_rank(&S, tid)->cnt[r] = S.sm[44];
   cl.sync();
+  SELT(122);
   if (sel == 0 && r == 0) TRACE(12);
   // 4. the boundary bin's candidates.  Few (<= kSelCNT, the usual case): every
   //    CTA copies the whole list, ranks every candidate and so knows every
@@ -891,6 +1175,7 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
       if (few) asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
       if (tid < kSelCL) S.part[tid] = 0;  // winners per CTA (reuses the slice totals)
       __syncthreads();
+      SELT(123);
       if (few) {  // warp per candidate (every candidate), lanes split the comparisons
         for (int j = tid >> 5; j < nc; j += kSelCNT / 32) {
           const int mi = S.cidx[j];
@@ -916,6 +1201,7 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
       }
     }
     __syncthreads();
+    SELT(124);
     if (few) {
 #pragma unroll
       for (int c = 0; c < kSelCL; ++c) wins[c] = S.part[c];
@@ -926,6 +1212,7 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
   for (int w = tid * wpt; w < min(wpc, (tid + 1) * wpt); ++w) cnt += __popc(sbits[w]);
   int mine;
   int pos = block_excl_scan<kSelCNT>(cnt, &mine, S.sm);
+  SELT(125);
   if (!whole && !few) {  // resolved locally: my final count to every CTA
     if (tid < kSelCL) cl.map_shared_rank(&S, tid)->cnt[r] = mine;
     cl.sync();
@@ -940,43 +1227,9 @@ __device__ __forceinline__ void select_cluster_body(const SelArgs& A, int sel, u
     jofs += c < r ? cc : 0;
     total += cc;
   }
-  uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap) + r * wpc;
-  int* J = reinterpret_cast<int*>(rec + A.lay.off_J);
-  for (int w = tid; w < wpc; w += kSelCNT) bitmap[w] = sbits[w];
-  if (A.pk) {  // k_tail's vote table: element b (pk_esz bytes) = bucket b, bit sel = kept in location loop sel
-    for (int w = tid; w < wpc; w += kSelCNT) {
-      const uint32_t bits = sbits[w];
-      if (!bits) continue;
-      const int64_t b0 = (int64_t)(r * wpc + w) * 32;  // first bucket of the word
-      if (A.pk_esz == 1) {  // 4 buckets per u32: spread each nibble of bits over 4 bytes
-        uint32_t* dst = A.pk + b0 / 4;
-#pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          const uint32_t nib = (bits >> (4 * j)) & 0xFu;
-          if (nib) atomicOr(dst + j, ((nib * 0x00204081u) & 0x01010101u) << sel);
-        }
-      } else {
-        for (uint32_t bb = bits; bb; bb &= bb - 1) {
-          const int64_t bkt = b0 + __ffs(bb) - 1;
-          const int per = 4 / A.pk_esz;  // buckets per u32 word
-          atomicOr(A.pk + bkt / per, (1u << sel) << (8 * A.pk_esz * (int)(bkt % per)));
-        }
-      }
-    }
-  }
-  pos += jofs;
-  for (int w = tid * wpt; w < min(wpc, (tid + 1) * wpt); ++w) {
-    uint32_t bits = sbits[w];
-    while (bits) {
-      const int b = __ffs(bits) - 1;
-      bits &= bits - 1;
-      J[pos++] = k0 + w * 32 + b;
-    }
-  }
-  if (r == 0 && tid == 0) {
-    *reinterpret_cast<int*>(rec + A.lay.off_cnt) = total;
-    if (!A.threshold_mode && total != A.num) atomicOr(A.status + 1, 1);
-  }
+  select_cluster_write(A, rec, sbits, sel, r, wpc, wpt, k0, pos + jofs, total);
+  SELT(126);
+#undef SELT
   if (sel == 0 && r == 0) TRACE(14);
   if (!whole && few && nc <= kSelCap) asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
   // (no remote smem access after the last barrier: CTAs may exit)
@@ -987,6 +1240,297 @@ __global__ void __launch_bounds__(kSelCNT, 1) k_select_cluster(SelArgs A) {
   KTRACE(8);
   extern __shared__ __align__(16) uint8_t smem[];
   select_cluster_body(A, blockIdx.x / kSelCL, smem);
+}
+
+// ---------------------------------------------------------------------------
+// Step 3 (pass 2, L87) fused with Step 4 (L89, the exact cutoff) for the
+// location slots: one cluster of kSelCL CTAs per location slot, CTA r owning
+// rows k1 in [r ROWS, r ROWS + ROWS) of the four-step FFT (B = B1 x M, B1 =
+// kSelCL ROWS).  Nothing of the cutoff goes through global memory:
+//   1. the CTA loads its ROWS contiguous rows of v (pass 1's output), runs the
+//      M-point row FFTs in shared memory and writes u^[k1 + B1 k2] to the
+//      record; keys bits(|u^|^2) stay in shared memory and are counted into a
+//      4096-bin top-digit histogram whose nonzero bins are added into every
+//      CTA's copy (remote shared-memory atomics); cluster barrier;
+//   2. every CTA finds the boundary digit d0 from the complete histogram,
+//      classifies its keys and stores its ROWS-bit pieces of the slot's take
+//      bitmap (bucket b = k1 + B1 k2: the piece of row k2 is bits [r ROWS,
+//      r ROWS + ROWS) of the B1 buckets B1 k2 ...) into every CTA, and pushes
+//      its boundary-bin candidates; cluster barrier;
+//   3. every CTA holds the whole take bitmap and every candidate: it ranks
+//      the candidates (ties to the smaller bucket), ORs the winners in, and
+//      writes buckets [r B/kSelCL, (r+1) B/kSelCL) of the bitmap, the vote
+//      table and the ascending J (offsets by one block scan of popcounts).
+// Same u^ as k_fft, same winners and J as the cutoff kernels.  When a CTA
+// holds more than kSelFastCap candidates the cluster falls back to the
+// general cluster selection over the keys and histogram it also wrote to
+// global memory.
+// ---------------------------------------------------------------------------
+struct Fft2SelArgs {
+  SelArgs s;
+  const double2* v[kMaxSel];  // pass-1 output of location slot i: row k1 = v[k1 M ... k1 M + M)
+  const double2* tw;          // e^{-2 pi i t / B}, t < B
+  int B1;
+};
+
+constexpr int kF2SNT = 1024;  // threads per CTA of k_fft2_select (32 warps: the chain is latency-bound)
+
+template <int M, int ROWS>
+__host__ __device__ constexpr int fft2sel_smem_bytes() {
+  return (M * ROWS + M * ROWS / 8) * 16 + M * 16 + 2 * 4096 * 4 + M * ROWS * 8 + M * ROWS * kSelCL / 8 +
+         (int)sizeof(SelFastSmem) + kF2SNT * 4;
+}
+
+template <int M, int ROWS>
+__global__ void __launch_bounds__(kF2SNT, 1) k_fft2_select(Fft2SelArgs F) {
+  pdl_wait();
+  KTRACE(8);
+  namespace cg = cooperative_groups;
+  cg::cluster_group cl = cg::this_cluster();
+  constexpr int NT = kF2SNT;
+  constexpr int E = M * ROWS;  // elements (and keys) of this CTA
+  constexpr int EPT = E / NT;
+  constexpr int HB = 4096 / NT;            // histogram bins per thread
+  constexpr int WORDS = E * kSelCL / 32;   // bitmap words of the slot
+  constexpr int WT = (WORDS + NT - 1) / NT;  // words per thread in the offset scan
+  static_assert(E % NT == 0 && (ROWS == 8 || ROWS == 16 || ROWS == 32) && M <= NT, "fft2_select shape");
+  const SelArgs& A = F.s;
+  extern __shared__ __align__(16) uint8_t smem[];
+  double2* S = reinterpret_cast<double2*>(smem);                 // E + E/8 (padded FFT workspace)
+  double2* twl = S + (E + E / 8);                                // omega_M^t, t < M
+  uint32_t* lh = reinterpret_cast<uint32_t*>(twl + M);           // 4096: my keys' top digits
+  uint32_t* gh = lh + 4096;                                      // 4096: the slot's (summed over the cluster)
+  uint64_t* skey = reinterpret_cast<uint64_t*>(gh + 4096);       // E: key of local t = k2 ROWS + j
+  uint32_t* full = reinterpret_cast<uint32_t*>(skey + E);        // WORDS: the slot's bitmap
+  SelFastSmem& C = *reinterpret_cast<SelFastSmem*>(full + WORDS);
+  int* pre = reinterpret_cast<int*>(&C + 1);                     // NT: offset scan
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  const int r = (int)cl.block_rank();
+  const int sel = blockIdx.x / kSelCL;
+  const int B = A.B, B1 = F.B1;
+  if (sel == 0 && r == 0) TRACE(10);
+#ifdef CUSFFT_TRACE
+  const long long fcs0 = clock64();
+#define F2T(slot) CTRACE_MAX(slot, clock64() - fcs0)
+#else
+#define F2T(slot) do { } while (0)
+#endif
+  {
+    const double2* vin = F.v[sel] + (int64_t)r * E;
+    double2 buf[EPT];
+#pragma unroll
+    for (int u = 0; u < EPT; ++u) buf[u] = __ldcg(vin + u * NT + tid);
+    // histograms zeroed before this CTA's arrive: the others add into gh only after their wait
+#pragma unroll
+    for (int j = 0; j < HB; ++j) {
+      lh[j * NT + tid] = 0;
+      gh[j * NT + tid] = 0;
+    }
+    if (tid == 0) C.lkey_n = 0;
+    asm volatile("barrier.cluster.arrive.release.aligned;" ::: "memory");
+    if (tid < M) twl[tid] = __ldg(F.tw + (int64_t)tid * (B / M));
+#pragma unroll
+    for (int u = 0; u < EPT; ++u) S[fft_pad(u * NT + tid)] = buf[u];
+  }
+  __syncthreads();
+  F2T(117);
+  fft_smem<M, E, NT, true>(S, twl, M);  // ROWS sequences of M: S[j M + k2] = row j's k2-th output
+  F2T(118);
+  uint8_t* rec = A.recs[sel];
+  double2* uh = reinterpret_cast<double2*>(rec);
+  uint64_t* gkeys = const_cast<uint64_t*>(A.keys) + (int64_t)sel * B;
+#pragma unroll
+  for (int u = 0; u < EPT; ++u) {
+    const int t = u * NT + tid;
+    const int j = t % ROWS, k2 = t / ROWS;
+    const double2 val = S[fft_pad(j * M + k2)];
+    const int b = r * ROWS + j + B1 * k2;
+    uh[b] = val;
+    const uint64_t key = (uint64_t)__double_as_longlong(__dadd_rn(__dmul_rn(val.x, val.x), __dmul_rn(val.y, val.y)));
+    skey[t] = key;
+    gkeys[b] = key;  // the general fallback reads keys and histogram through L2
+    atomicAdd(&lh[(uint32_t)(key >> 51) & 0xFFFu], 1u);
+  }
+  __syncthreads();
+  F2T(119);
+  asm volatile("barrier.cluster.wait.acquire.aligned;" ::: "memory");
+  F2T(120);
+#pragma unroll
+  for (int j = 0; j < HB; ++j) {
+    const int i = j * NT + tid;
+    const uint32_t c = lh[i];
+    if (c) {
+      atomicAdd(A.hist0 + (int64_t)sel * 4096 + i, c);
+#pragma unroll
+      for (int q = 0; q < kSelCL; ++q) {
+        const uint32_t ra = (uint32_t)__cvta_generic_to_shared(gh + i);
+        uint32_t rq;
+        asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(rq) : "r"(ra), "r"(q));
+        asm volatile("red.shared::cluster.add.u32 [%0], %1;" ::"r"(rq), "r"(c) : "memory");
+      }
+    }
+  }
+  F2T(121);
+  cl.sync();
+  F2T(122);
+  if (sel == 0 && r == 0) TRACE(11);
+  // 2. boundary digit (every CTA alike): keys in the bins of higher threads by a reversed scan
+  {
+    uint32_t hv[HB];
+    int mys = 0;
+#pragma unroll
+    for (int j = 0; j < HB; ++j) {
+      hv[j] = gh[HB * tid + j];
+      mys += (int)hv[j];
+    }
+    int inc = mys;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_down_sync(kFull, inc, o);
+      if (lane + o < 32) inc += y;
+    }
+    if (lane == 0) C.sm[wid] = inc;
+    __syncthreads();
+    int above_w = 0;
+    if (lane < NT / 32) above_w = lane > wid ? C.sm[lane] : 0;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) above_w += __shfl_xor_sync(kFull, above_w, o);
+    const int ex = above_w + inc - mys;
+    if (ex < A.num && A.num <= ex + mys) {
+      int e = ex;
+#pragma unroll
+      for (int j = HB - 1; j >= 0; --j) {
+        const int c = (int)hv[j];
+        if (e < A.num && A.num <= e + c) {
+          C.pick[0] = HB * tid + j;
+          C.pick[1] = e;
+          C.pick[2] = c;
+        }
+        e += c;
+      }
+    }
+  }
+  __syncthreads();
+  const int d0 = C.pick[0];
+  const int k2sel = A.num - C.pick[1];
+  const bool whole = (k2sel == C.pick[2]);
+  const unsigned lt = (1u << lane) - 1u;
+#pragma unroll
+  for (int u = 0; u < EPT; ++u) {
+    const int t = u * NT + tid;
+    const uint64_t key = skey[t];
+    const uint32_t d = (uint32_t)(key >> 51) & 0xFFFu;
+    const bool take = d > (uint32_t)d0 || (d == (uint32_t)d0 && whole);
+    const bool cand = d == (uint32_t)d0 && !whole;
+    const uint32_t word = __ballot_sync(kFull, take);
+    // this warp's 32 keys = 32 / ROWS pieces (rows k2 = t0 / ROWS ...) of ROWS bits each
+    const int t0 = t - lane;
+    if (ROWS == 32) {
+      if (lane < kSelCL) *cl.map_shared_rank(full + ((B1 * (t0 / ROWS) + r * ROWS) >> 5), lane) = word;
+    } else if (ROWS == 16) {
+      if (lane < 2 * kSelCL) {
+        const int p = lane / kSelCL, q = lane % kSelCL;
+        const int k2 = t0 / ROWS + p;
+        uint16_t* dst = reinterpret_cast<uint16_t*>(full) + ((B1 * k2 + r * ROWS) >> 4);
+        *cl.map_shared_rank(dst, q) = (uint16_t)(word >> (16 * p));
+      }
+    } else {
+      const int p = lane / kSelCL, q = lane % kSelCL;  // 4 pieces x 8 CTAs
+      const int k2 = t0 / ROWS + p;
+      uint8_t* dst = reinterpret_cast<uint8_t*>(full) + ((B1 * k2 + r * ROWS) >> 3);
+      *cl.map_shared_rank(dst, q) = (uint8_t)(word >> (8 * p));
+    }
+    const unsigned cm = __ballot_sync(kFull, cand);
+    if (cm) {
+      int bpos = 0;
+      if (lane == __ffs(cm) - 1) bpos = atomicAdd(&C.lkey_n, __popc(cm));
+      bpos = __shfl_sync(kFull, bpos, __ffs(cm) - 1);
+      if (cand) {
+        const int pos = bpos + __popc(cm & lt);
+        if (pos < kSelFastCap) {
+          C.fkey[pos] = key;
+          C.fidx[pos] = r * ROWS + t % ROWS + B1 * (t / ROWS);
+        }
+      }
+    }
+  }
+  __syncthreads();
+  {
+    const int nmine = C.lkey_n;
+    if (tid < kSelCL) cl.map_shared_rank(&C, tid)->ncand[r] = nmine;
+    const int ncopy = min(nmine, kSelFastCap);
+    for (int j = tid; j < ncopy * kSelCL; j += NT) {
+      const int q = j / ncopy, c = j - q * ncopy;
+      SelFastSmem* D = cl.map_shared_rank(&C, q);
+      D->ckey[r][c] = C.fkey[c];
+      D->cidx[r][c] = C.fidx[c];
+    }
+  }
+  F2T(123);
+  cl.sync();
+  F2T(124);
+  if (sel == 0 && r == 0) TRACE(12);
+  // 3. resolution, identical in every CTA
+  int nc = 0, offs[kSelCL];
+  bool over = false;
+#pragma unroll
+  for (int c = 0; c < kSelCL; ++c) {
+    offs[c] = nc;
+    nc += C.ncand[c];
+    over |= C.ncand[c] > kSelFastCap;
+  }
+  if (over) {  // crowded boundary bin: CTA 0 runs the single-CTA selection over the keys and histogram in L2
+    __threadfence();
+    cl.sync();
+    if (r == 0) select1_body(A, sel, smem, true);
+    return;
+  }
+  if (!whole) {
+    for (int j = tid; j < nc; j += NT) {
+      int c = 0, base = 0;
+#pragma unroll
+      for (int q = 1; q < kSelCL; ++q)
+        if (j >= offs[q]) {
+          c = q;
+          base = offs[q];
+        }
+      C.fkey[j] = C.ckey[c][j - base];
+      C.fidx[j] = C.cidx[c][j - base];
+    }
+    __syncthreads();
+    for (int j = tid; j < nc; j += NT) {
+      const uint64_t mk = C.fkey[j];
+      const int mi = C.fidx[j];
+      int rank = 0;
+#pragma unroll 4
+      for (int c = 0; c < nc; ++c) {
+        const uint64_t kc = C.fkey[c];
+        rank += (kc > mk) | ((kc == mk) & (C.fidx[c] < mi));
+      }
+      if (rank < k2sel) atomicOr(&full[mi >> 5], 1u << (mi & 31));
+    }
+    __syncthreads();
+  }
+  // offsets: popcounts of the whole bitmap, WT words per thread
+  int cnt = 0;
+#pragma unroll
+  for (int w = 0; w < WT; ++w) cnt += tid * WT + w < WORDS ? __popc(full[tid * WT + w]) : 0;
+  int total;
+  pre[tid] = block_excl_scan<NT>(cnt, &total, C.sm);
+  __syncthreads();
+  F2T(125);
+  if (sel == 0 && r == 0) TRACE(13);
+  const int wpc = WORDS / kSelCL;  // my words: [r wpc, r wpc + wpc), one per thread (wpc <= NT)
+  int pos = 0;
+  if (tid < wpc) {
+    const int w = r * wpc + tid;
+    pos = pre[w / WT];
+    for (int q = (w / WT) * WT; q < w; ++q) pos += __popc(full[q]);
+  }
+  select_cluster_write<NT>(A, rec, full + r * wpc, sel, r, wpc, 1, r * E, pos, total);
+  F2T(126);
+#undef F2T
+  if (sel == 0 && r == 0) TRACE(14);
 }
 
 // ---------------------------------------------------------------------------

@@ -12,6 +12,8 @@ for tool in memcheck racecheck synccheck; do
   run $tool n16_k32_L24 65536 32 0 L=24 loc_loops=20 vote_threshold=11
   run $tool n22_k1000_staged 4194304 1000
   run $tool n16_k32_B256 65536 32 256
+  run $tool n20_k1000_B16384 1048576 1000 16384
+  run $tool n18_zero_B16384 262144 64 16384 zero=1
 done
 run memcheck n22_k1000_chain 4194304 1000 0 gather=1
 CUSFFT_TAIL=0 run memcheck n22_k1000_tail0 4194304 1000

@@ -16,6 +16,8 @@ prm = bench.plan_params("C3")
 if len(sys.argv) > 2:
     prm["tolerance"] = tol
 plan = Plan(n, k, L=L, seed=3, **prm)
+if os.environ.get("TRACE_TIMING"):
+    plan.set_timing(int(os.environ["TRACE_TIMING"]))
 lib = load_library()
 fl = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 fr = torch.ones(64 << 20, dtype=torch.int32, device="cuda")
@@ -42,6 +44,9 @@ for rep in range(reps):
         print("select candidates per loop:", [int(t[96 + i]) & 0xFFFFFFFF for i in range(16) if 0 < t[96 + i] < 2**40])
         print("fold_fft1: latest CTA start (us) loc/est", [(t[112 + q] - t0) / 1e3 for q in (0, 1) if t[112 + q] > 0],
               "cycles: first rows landed", int(t[114]), "slot compute", int(t[115]), "CTA", int(t[116]))
+        print("fft2_select cycles (max over CTAs, from entry): loads", int(t[117]), "fft", int(t[118]),
+              "keys", int(t[119]), "cl.wait", int(t[120]), "hist push", int(t[121]), "sync1", int(t[122]),
+              "classify+push", int(t[123]), "sync2", int(t[124]), "resolve+scan", int(t[125]), "write", int(t[126]))
         cyc = {i: int(t[i]) for i in range(64, 96) if t[i] > 0}
         if cyc:
             print("tail cycles: vote(w0 max)", cyc.get(70), "vote(CTA max)", cyc.get(71), "estimate(CTA max)", cyc.get(72))

@@ -187,6 +187,24 @@ def test_zero_signal_ties():
     assert np.all(vals == 0)
 
 
+@pytest.mark.parametrize("B", [8192, 16384])
+def test_fft2_select_crowded_fallback(B):
+    """Shapes of the fused FFT-pass-2 + cutoff cluster kernel (k_fft2_select):
+    x = 0 puts every key of a slot in the boundary bin (the fallback to the
+    single-CTA selection inside the cluster kernel), a dense signal puts
+    hundreds of keys there (more than the per-CTA candidate cap); both match
+    the oracle's winners (ties to the smaller bucket) and outputs."""
+    n, k = 2 ** 18, 64
+    x = np.zeros(n, dtype=np.complex128)
+    plan, ref, locs, vals = run_pair(x, n, k, B, 8, shared_taps=True, seed=1)
+    win = plan.debug(DEBUG_WINNERS)
+    assert all(np.array_equal(w, np.arange(plan.num)) for w in win)
+    check_all(plan, ref, locs, vals, fold_bit_exact=True)
+    x = dense_signal(n, 12)
+    plan, ref, locs, vals = run_pair(x, n, k, B, 8, shared_taps=True, seed=2)
+    check_all(plan, ref, locs, vals, fold_bit_exact=True)
+
+
 def test_num_select_equals_B():
     n, k = 2 ** 10, 4
     x, S, X = planted_signal(n, k, seed=1)
@@ -294,6 +312,7 @@ def test_parity_snr_sweep(snr_db):
 
 @pytest.mark.gpu
 @pytest.mark.parametrize("env,kw", [({"CUSFFT_NO_GRAPH": "1"}, {}), ({"CUSFFT_TAIL": "0"}, {}),
+                                    ({"CUSFFT_FFT2SEL": "0"}, {}),
                                     ({}, dict(gather=1)), ({}, dict(l2_persist=0)),
                                     ({"CUSFFT_TAIL": "0", "CUSFFT_NO_GRAPH": "1"}, dict(gather=1))])
 def test_kernel_paths_agree(env, kw, monkeypatch):
