@@ -411,6 +411,8 @@ def run_gpu(args):
             stage_ms["vote + estimate (k_tail)" if (info["tail"] and si == 4) else nm] = tsi - prev
             prev = tsi
         plan.set_stage_limit(6)
+        # where the location slots' FFT pass 2 is fused with the cutoff (k_fft2_select),
+        # "fft" is the estimation slots' FFT and "cutoff" includes the location pass 2
 
     # ---- CUPTI cross-check of the kernel durations (torch.profiler: no replay)
     cupti = None

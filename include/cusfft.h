@@ -300,7 +300,10 @@ int cusfft_get_stage_times(cusfft_plan_t plan, float* ms, int32_t cap);
 /* Profiling (no paper passage; the per-step breakdown of Fig. 2):
  * run only the first `stages` stages (1 = fold ... 6 = output,
  * the default) so per-stage times can be taken inside the CUDA graph by
- * differences of whole-execution times.  Outputs are undefined when < 6. */
+ * differences of whole-execution times.  Outputs are undefined when < 6.
+ * Where the location slots' FFT pass 2 runs inside the cutoff kernel
+ * (B = 8192, 16384, 32768, exact cutoff), it belongs to stage 3: stage 2 is
+ * then the estimation slots' FFT only. */
 int cusfft_set_stage_limit(cusfft_plan_t plan, int32_t stages);
 
 /* Number of kernel launches one cusfft_execute issues for this plan (plumbing). */

@@ -185,6 +185,7 @@ struct cusfft_plan_s {
   std::vector<uint32_t> row0_h;              // same, host (+ total rows at [Lg])
   double2* d_staging = nullptr;              // [rows][B]
   int stage_grid = 1;
+  bool p2_ms = true;                         // phase 2 in the multi-slot form (k_fold_fft1_ms, R <= 16)
   int p2_spc = 2;                            // phase-2 slots per CTA (taps reused across them; 1 / 4 slower)
   int fork_at = 1;                           // estimation branch forks after phase 1 (0) or after the location phase 2 (1, measured ~0.5 us faster)
   bool setaside = false;                     // holds a reference on the device's persisting-L2 set-aside
@@ -610,6 +611,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   P->T = q.vote_threshold;
   P->max_hits = (int)q.max_hits;
   if (const char* e = std::getenv("CUSFFT_NO_GRAPH")) P->use_graph = !(e[0] == '1');                    // A/B (measurement)
+  if (const char* e = std::getenv("CUSFFT_P2_MS")) P->p2_ms = std::atoi(e) != 0;                         // A/B (measurement)
   if (const char* e = std::getenv("CUSFFT_P2_SPC")) P->p2_spc = std::max(1, std::min(8, std::atoi(e)));  // A/B (measurement)
   if (const char* e = std::getenv("CUSFFT_FFT2SEL")) P->fft2sel = std::atoi(e) != 0;                     // A/B (measurement)
   if (const char* e = std::getenv("CUSFFT_FORK")) P->fork_at = std::atoi(e);                                 // A/B (measurement)
@@ -917,6 +919,23 @@ cudaError_t launch_p2_t(cusfft_plan_t P, const Filter& F, const double2* staging
     cudaFuncSetAttribute(k_fold_fft1_tma<B1T, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
     cudaFuncSetAttribute(k_fold_fft1_tma<B1T, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
     attr_set = true;
+  }
+  if (P->p2_ms && F.R <= 16) {  // multi-slot form (k_fold_fft1_ms): 8 slots per CTA, 4 (R <= 8) or 2 in flight
+    constexpr int NSM = 8;
+    static thread_local bool ms_attr = false;
+    if (!ms_attr) {
+      cudaFuncSetAttribute(k_fold_fft1_ms<B1T, NSM, 4, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           fold_ms_smem_bytes<B1T, NSM, 4, 8>());
+      cudaFuncSetAttribute(k_fold_fft1_ms<B1T, NSM, 2, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           fold_ms_smem_bytes<B1T, NSM, 2, 16>());
+      ms_attr = true;
+    }
+    dim3 grid((unsigned)(P->B / 256), (unsigned)((nslots + NSM - 1) / NSM));
+    const bool r8 = F.R <= 8;
+    return launch_k(r8 ? k_fold_fft1_ms<B1T, NSM, 4, 8> : k_fold_fft1_ms<B1T, NSM, 2, 16>, grid, dim3(256),
+                    (size_t)(r8 ? fold_ms_smem_bytes<B1T, NSM, 4, 8>() : fold_ms_smem_bytes<B1T, NSM, 2, 16>()),
+                    st, P->cur_prio, staging, (const double*)F.d_taps_perm, P->prm.debug ? u : nullptr, v,
+                    (const double2*)P->d_tw, (int)P->B, P->B2, F.w, F.R, nslots, z);
   }
   // spc slots per CTA (their taps loaded once), double-buffered rows while two fit in shared memory
   const int spc = (2 * F.R * 4096 <= 160 * 1024) ? std::min(P->p2_spc, nslots) : 1;
@@ -1240,8 +1259,8 @@ int launch_local(cusfft_plan_t P, const double2* x) {
   g_pdl = P->timing != 1;
   mark(P, 1);
   if (P->stage_limit < 2) return CUSFFT_SUCCESS;
-  const bool f2s = use_fft2_select(P) && P->stage_limit >= 3;
-  TRY(launch_bfft(P, f2s ? P->nloc_local : 0, P->Lg, st));  // fused: the location slots' pass 2 runs with their cutoff
+  const bool f2s = use_fft2_select(P);
+  TRY(launch_bfft(P, f2s ? P->nloc_local : 0, P->Lg, st));  // fused: the location slots' pass 2 runs with their cutoff (stage 3)
   mark(P, 2);
   if (P->stage_limit < 3 || P->xshard) return CUSFFT_SUCCESS;  // signal-sharded: cutoff after the all-reduce
   if (f2s)
@@ -1320,10 +1339,10 @@ int launch_branched(cusfft_plan_t P, const double2* x, int64_t* locs, double2* v
   g_pdl = true;
   TRY(launch_fold_range(P, x, 0, nl, a, false));
   if (P->fork_at == 1) TRY(fork());
-  const bool f2s = use_fft2_select(P) && lim >= 3;
+  const bool f2s = use_fft2_select(P);  // location slots: FFT pass 2 inside the cutoff kernel (stage 3)
   if (lim >= 2 && !f2s) TRY(launch_bfft(P, 0, nl, a));
   if (P->fork_at == 2) TRY(fork());
-  if (f2s)
+  if (f2s && lim >= 3)
     TRY(launch_fft2_select(P, a));
   else if (lim >= 3 && !P->xshard)
     TRY(launch_select(P, a));
@@ -1858,7 +1877,7 @@ int32_t cusfft_launches_per_execute(cusfft_plan_t plan) {
   const int ranges = (nl > 0) + (ne > 0);
   const bool pass1 = plan->B1 > 1 && !plan->fused1;
   const bool branched = use_branches(plan);
-  const bool f2s = use_fft2_select(plan) && plan->stage_limit >= 3;  // location pass 2 inside the cutoff kernel
+  const bool f2s = use_fft2_select(plan);  // location pass 2 inside the cutoff kernel
   const int ffts = f2s ? (ne > 0 ? 1 : 0) : (branched ? ranges : 1);
   int n = (plan->staged ? 1 : 0) + ranges /*fold per slot range*/ +
           ffts * (pass1 ? 2 : 1) /*fft*/ + (plan->sel_slots_h.empty() ? 0 : 1) +

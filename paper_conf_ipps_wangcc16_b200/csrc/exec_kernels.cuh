@@ -364,6 +364,97 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1_tma(const double2* __restr
 }
 
 // ---------------------------------------------------------------------------
+// Phase 2, multi-slot form: a CTA owns one tile of 256 buckets (C = 256 / B1
+// columns) of up to NSMAX slots of one filter.  Thread t folds bucket
+// (c, j1) of every slot; its R staged samples of each slot (row rr element t
+// of the tile: exactly the ones it folds) are copied to shared memory by
+// cp.async, NBUF slots in flight (a per-thread ring: no barrier between
+// slots).  After the last slot the CTA runs the column FFTs of ALL its slots
+// at once (NSMAX C sequences of B1) and writes v.  Per slot the arithmetic is
+// k_fold_fft1_tma's (Alg. 1 order).  Dynamic smem: fold_ms_smem_bytes.
+// ---------------------------------------------------------------------------
+template <int B1T, int NSMAX, int NBUF, int RMAX>
+__host__ __device__ constexpr int fold_ms_smem_bytes() {
+  return NBUF * RMAX * 256 * 16 + (NSMAX * 256 + NSMAX * 256 / 8) * 16 + B1T * 16;
+}
+
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+template <int B1T, int NSMAX, int NBUF, int RMAX>
+__global__ void __launch_bounds__(256, 1) k_fold_fft1_ms(const double2* __restrict__ staging,
+                                                         const double* __restrict__ taps_perm,
+                                                         double2* __restrict__ u, double2* __restrict__ v,
+                                                         const double2* __restrict__ tw, int B, int B2, int w, int R,
+                                                         int nslots, ZeroArgs zero) {
+  pdl_wait();
+  KTRACE(2);
+  constexpr int C = 256 / B1T;
+  constexpr int E = NSMAX * 256;
+  extern __shared__ __align__(16) uint8_t msm[];
+  double2* Ring = reinterpret_cast<double2*>(msm);  // [NBUF][RMAX][256]
+  double2* S = Ring + NBUF * RMAX * 256;            // E + E/8
+  double2* twl = S + (E + E / 8);                   // B1T
+  const int t = threadIdx.x;
+  const int s0 = blockIdx.y * NSMAX;
+  const int ns = min(NSMAX, nslots - s0);
+  if (blockIdx.x == 0 && blockIdx.y == 0) TRACE(0);
+  const int cl = t / B1T, j1 = t % B1T;
+  const int c = blockIdx.x * C + cl;
+  const int j = c + B2 * j1;
+  const double2* src0 = staging + (int64_t)s0 * R * B + (int64_t)blockIdx.x * 256 + t;
+  auto issue = [&](int i) {  // my R samples of slot i into ring slot i mod NBUF
+    if (i < ns) {
+      double2* dst = Ring + (i % NBUF) * RMAX * 256 + t;
+      const double2* src = src0 + (int64_t)i * R * B;
+#pragma unroll
+      for (int rr = 0; rr < RMAX; ++rr)
+        if (rr < R && j + rr * B < w) cp_async16(dst + rr * 256, src + (int64_t)rr * B);
+    }
+    cp_async_commit();  // (empty groups keep the count uniform)
+  };
+#pragma unroll
+  for (int i = 0; i < NBUF; ++i) issue(i);
+  zero_part(zero);
+  for (int i = t; i < B1T; i += 256) twl[i] = __ldg(tw + (int64_t)i * B2);  // omega_B1^i
+  const double* tp = taps_perm + (int64_t)blockIdx.x * 256 + t;
+  double g[RMAX];
+#pragma unroll
+  for (int rr = 0; rr < RMAX; ++rr) g[rr] = (rr < R && j + rr * B < w) ? __ldg(tp + (int64_t)rr * B) : 0.0;
+  const int wc = t % C, wj = t / C;  // writer's (column, row)
+  const double2 wv = __ldg(tw + (((int64_t)(blockIdx.x * C + wc) * wj) & (B - 1)));
+  for (int i = 0; i < ns; ++i) {
+    cp_async_wait<NBUF - 1>();  // slot i's group (my own copies: no barrier)
+    const double2* T = Ring + (i % NBUF) * RMAX * 256 + t;
+    double ar = 0.0, ai = 0.0;
+#pragma unroll
+    for (int rr = 0; rr < RMAX; ++rr) {
+      if (rr < R && j + rr * B < w) {
+        const double2 q = T[rr * 256];
+        ar = __dadd_rn(ar, __dmul_rn(g[rr], q.x));
+        ai = __dadd_rn(ai, __dmul_rn(g[rr], q.y));
+      }
+    }
+    S[fft_pad(i * 256 + cl * B1T + j1)] = make_double2(ar, ai);
+    issue(i + NBUF);  // into the ring slot just consumed (by this thread only)
+  }
+  cp_async_wait<0>();
+  __syncthreads();
+  if (u)  // the fold output itself: debug plans only
+    for (int i = 0; i < ns; ++i)
+      u[(size_t)(s0 + i) * B + (size_t)blockIdx.x * C + wc + (size_t)B2 * wj] = S[fft_pad(i * 256 + wc * B1T + wj)];
+  fft_smem<B1T, E, 256, true>(S, twl, B1T);
+  for (int i = 0; i < ns; ++i)
+    v[(size_t)(s0 + i) * B + (size_t)blockIdx.x * C + wc + (size_t)B2 * wj] =
+        cmul(S[fft_pad(i * 256 + wc * B1T + wj)], wv);
+  TRACE_END(1);
+}
+
+// ---------------------------------------------------------------------------
 // Record layout of one slot in the exchange buffer:
 //   [u^ : B x double2][bitmap : B/32 x u32][count : int32][J : Jcap x int32],
 //   256-B aligned; Jcap = num (B in THRESHOLD mode).
