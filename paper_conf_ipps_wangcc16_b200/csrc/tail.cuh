@@ -274,7 +274,17 @@ __device__ __forceinline__ void tail_estimate(const EstArgs& E, uint32_t hf, boo
   if (LP == 16) {
     const unsigned segmask = 0xFFFFu << (seg * 16);
     const bool act = li < L;
+#ifdef CUSFFT_TRACE
+    const long long te0 = clock64();
+#endif
     if (valid && act) v0 = loop_estimate(E, sp0, li, hf);
+#ifdef CUSFFT_TRACE
+    {
+      const bool nanv = v0.x != v0.x;  // waits for the loads
+      const long long te1 = clock64();
+      if (lane == 0 && valid) atomicMax(&g_trace[75], (unsigned long long)(te1 - te0 + (nanv ? 1 : 0)));
+    }
+#endif
 #pragma unroll
     for (int part = 0; part < 2; ++part) {
       const double a = part ? v0.y : v0.x;
@@ -572,7 +582,13 @@ __global__ void __launch_bounds__(kTailNT, 4) k_tail(TailArgs A) {
   double2 v0, v1;
   if (wid * G < nq)  // warp-uniform
     tail_estimate<LP>(A.e, h1 < nq ? s_hq[h1] : 0u, h1 < nq, sp0, sp1, vr, vi, v0, v1);
+#ifdef CUSFFT_TRACE
+  if (wid * G < nq && lane == 0) atomicMax(&g_trace[73], (unsigned long long)(clock64() - c_est0));  // first pass estimated
+#endif
   __syncthreads();
+#ifdef CUSFFT_TRACE
+  CTRACE_MAX(74, clock64() - c_est0);  // + the block barrier (hit-list base known)
+#endif
   if (nq > 0) {
     const unsigned base = s_base;
     for (int i = tid; i < nq; i += kTailNT)

@@ -49,7 +49,8 @@ for rep in range(reps):
               "classify+push", int(t[123]), "sync2", int(t[124]), "resolve+scan", int(t[125]), "write", int(t[126]))
         cyc = {i: int(t[i]) for i in range(64, 96) if t[i] > 0}
         if cyc:
-            print("tail cycles: vote(w0 max)", cyc.get(70), "vote(CTA max)", cyc.get(71), "estimate(CTA max)", cyc.get(72))
+            print("tail cycles: vote(w0 max)", cyc.get(70), "vote(CTA max)", cyc.get(71), "estimate(CTA max)", cyc.get(72),
+                  "first pass (warp max)", cyc.get(73), "+barrier", cyc.get(74), "loop_estimate loads", cyc.get(75))
             o = [cyc.get(i) for i in range(80, 87)]
             if all(o):
                 print("output phases (cycles): load", o[1] - o[0], "pick", o[2] - o[1], "classify", o[3] - o[2],
