@@ -201,7 +201,7 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1(const double2* __restrict_
   pdl_wait();
   KTRACE(2);
   constexpr int C = 256 / B1T;
-  __shared__ double2 S[256 + 256 / 8];
+  __shared__ double2 S[fft_pad_n(256)];
   __shared__ double2 twl[B1T];
   const int t = threadIdx.x;
   const int s = blockIdx.y;
@@ -278,7 +278,7 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1_tma(const double2* __restr
   KTRACE(2);
   constexpr int C = 256 / B1T;
   extern __shared__ __align__(128) double2 Tile[];  // [nbuf][R][256]
-  __shared__ double2 S[256 + 256 / 8];
+  __shared__ double2 S[fft_pad_n(256)];
   __shared__ double2 twl[B1T];
   __shared__ __align__(8) uint64_t bar[2];
   const int t = threadIdx.x;
@@ -375,7 +375,7 @@ __global__ void __launch_bounds__(256, 2) k_fold_fft1_tma(const double2* __restr
 // ---------------------------------------------------------------------------
 template <int B1T, int NSMAX, int NBUF, int RMAX>
 __host__ __device__ constexpr int fold_ms_smem_bytes() {
-  return NBUF * RMAX * 256 * 16 + (NSMAX * 256 + NSMAX * 256 / 8) * 16 + B1T * 16;
+  return NBUF * RMAX * 256 * 16 + fft_pad_n(NSMAX * 256) * 16 + B1T * 16;
 }
 
 __device__ __forceinline__ void cp_async16(void* dst, const void* src) {
@@ -397,8 +397,8 @@ __global__ void __launch_bounds__(256, 1) k_fold_fft1_ms(const double2* __restri
   constexpr int E = NSMAX * 256;
   extern __shared__ __align__(16) uint8_t msm[];
   double2* Ring = reinterpret_cast<double2*>(msm);  // [NBUF][RMAX][256]
-  double2* S = Ring + NBUF * RMAX * 256;            // E + E/8
-  double2* twl = S + (E + E / 8);                   // B1T
+  double2* S = Ring + NBUF * RMAX * 256;            // fft_pad_n(E)
+  double2* twl = S + fft_pad_n(E);                  // B1T
   const int t = threadIdx.x;
   const int s0 = blockIdx.y * NSMAX;
   const int ns = min(NSMAX, nslots - s0);
@@ -1368,7 +1368,7 @@ constexpr int kF2SNT = 1024;  // threads per CTA of k_fft2_select (32 warps: the
 
 template <int M, int ROWS>
 __host__ __device__ constexpr int fft2sel_smem_bytes() {
-  return (M * ROWS + M * ROWS / 8) * 16 + M * 16 + 2 * 4096 * 4 + M * ROWS * 8 + M * ROWS * kSelCL / 8 +
+  return fft_pad_n(M * ROWS) * 16 + M * 16 + 2 * 4096 * 4 + M * ROWS * 8 + M * ROWS * kSelCL / 8 +
          (int)sizeof(SelFastSmem) + kF2SNT * 4;
 }
 
@@ -1387,8 +1387,8 @@ __global__ void __launch_bounds__(kF2SNT, 1) k_fft2_select(Fft2SelArgs F) {
   static_assert(E % NT == 0 && (ROWS == 8 || ROWS == 16 || ROWS == 32) && M <= NT, "fft2_select shape");
   const SelArgs& A = F.s;
   extern __shared__ __align__(16) uint8_t smem[];
-  double2* S = reinterpret_cast<double2*>(smem);                 // E + E/8 (padded FFT workspace)
-  double2* twl = S + (E + E / 8);                                // omega_M^t, t < M
+  double2* S = reinterpret_cast<double2*>(smem);                 // fft_pad_n(E) (padded FFT workspace)
+  double2* twl = S + fft_pad_n(E);                                // omega_M^t, t < M
   uint32_t* lh = reinterpret_cast<uint32_t*>(twl + M);           // 4096: my keys' top digits
   uint32_t* gh = lh + 4096;                                      // 4096: the slot's (summed over the cluster)
   uint64_t* skey = reinterpret_cast<uint64_t*>(gh + 4096);       // E: key of local t = k2 ROWS + j

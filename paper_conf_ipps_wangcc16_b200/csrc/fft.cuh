@@ -10,7 +10,9 @@
 //           stored at u^[k1 + B1 k2].
 // Inside a CTA: Stockham autosort (natural order in and out), radix-8 stages
 // after one radix-2/4 stage when log2(M) is not a multiple of 3, with
-// conflict-free padded smem indexing pad(i) = i + i/8.
+// padded smem indexing pad(i) = i + i/8 + i/128 (conflict-free radix-8
+// strides; the extra element per 128 skews consecutive 128-point sequences
+// so that reading one element of each of them is not a bank conflict).
 //
 // Pass 2 (and the single pass) also produce the cutoff keys of the location
 // loops: key = bits(re*re + im*im) (non-negative fp64 orders like its bit
@@ -21,7 +23,9 @@
 
 namespace cusfft {
 
-__device__ __forceinline__ int fft_pad(int i) { return i + (i >> 3); }
+__device__ __forceinline__ int fft_pad(int i) { return i + (i >> 3) + (i >> 7); }
+// elements of a padded workspace holding E
+__host__ __device__ constexpr int fft_pad_n(int E) { return E + E / 8 + E / 128 + 1; }
 
 __device__ __forceinline__ double2 cmul(double2 a, double2 b) {
   return make_double2(a.x * b.x - a.y * b.y, a.x * b.y + a.y * b.x);
@@ -148,7 +152,7 @@ struct FftPassArgs {
 };
 
 // E = elements per CTA, NT = threads per CTA.  Dynamic smem: fft_smem_bytes(E).
-__host__ __device__ constexpr int fft_smem_bytes(int E) { return (E + E / 8) * 16 + 4096 * 4 + E * 16; }
+__host__ __device__ constexpr int fft_smem_bytes(int E) { return fft_pad_n(E) * 16 + 4096 * 4 + E * 16; }
 
 template <int M, int E, int NT>
 __global__ void __launch_bounds__(NT) k_fft(FftPassArgs A) {
@@ -157,8 +161,8 @@ __global__ void __launch_bounds__(NT) k_fft(FftPassArgs A) {
   constexpr int NSEQ = E / M;
   extern __shared__ __align__(16) uint8_t fsm[];
   double2* S = reinterpret_cast<double2*>(fsm);
-  uint32_t* shist = reinterpret_cast<uint32_t*>(fsm + (E + E / 8) * sizeof(double2));
-  double2* twl = reinterpret_cast<double2*>(fsm + (E + E / 8) * sizeof(double2) + 4096 * 4);  // omega_M^t, t < M
+  uint32_t* shist = reinterpret_cast<uint32_t*>(fsm + fft_pad_n(E) * sizeof(double2));
+  double2* twl = reinterpret_cast<double2*>(fsm + fft_pad_n(E) * sizeof(double2) + 4096 * 4);  // omega_M^t, t < M
   const int q0 = blockIdx.x * NSEQ;
   for (int t = threadIdx.x; t < M; t += NT) twl[t] = __ldg(A.tw + (int64_t)t * (A.B / M));
   if (blockIdx.x == 0) TRACE(A.twiddle ? 2 : 4);
