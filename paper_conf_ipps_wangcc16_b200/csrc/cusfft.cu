@@ -855,10 +855,12 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       // one resident wave of phase-1 CTAs (grid-stride loop), at most 4 per SM: with 4 gathers in
       // flight per thread that is 4096 per SM, measured best
       int occ = 0;
-      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_stage_packed<4>, 256, 0) != cudaSuccess || occ < 1) occ = 4;
+      if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_stage_packed<kStageU>, 256, 0) != cudaSuccess || occ < 1) occ = 4;
       cudaGetLastError();
-      const int per = 256 * 4;
-      P->stage_grid = (int)std::max<int64_t>(1, std::min<int64_t>((total + per - 1) / per, (int64_t)P->sms * std::min(occ, 4)));
+      const int per = 256 * kStageU;
+      int cps = std::min(occ, 4);
+      if (const char* e = std::getenv("CUSFFT_STAGE_CPS")) cps = std::max(1, std::min(occ, std::atoi(e)));  // A/B (measurement)
+      P->stage_grid = (int)std::max<int64_t>(1, std::min<int64_t>((total + per - 1) / per, (int64_t)P->sms * cps));
       // Persisting-L2 set-aside for the staging buffer: the staging stores carry evict_last
       // (= persisting) and the x loads evict_first; without the set-aside C3 took 100 us
       // instead of 87.  Device-wide and optional (params.l2_persist).
@@ -907,7 +909,7 @@ int launch_stage1(cusfft_plan_t P, const double2* x, cudaStream_t st) {
   StagePackArgs a{x, P->d_code, P->d_staging, P->d_slots + (size_t)P->lrank * P->Lg, P->d_row0,
                   (int)P->stage_total, P->Lg, P->stage_ibits, ilog2(P->B), P->logB2, P->logB1,
                   ilog2(256 / P->B1), (uint32_t)(P->n - 1), ZeroArgs{P->d_zero, P->nzero}};
-  CK(launch_k(k_stage_packed<4>, dim3(P->stage_grid), dim3(256), 0, st, P->cur_prio, a));
+  CK(launch_k(k_stage_packed<kStageU>, dim3(P->stage_grid), dim3(256), 0, st, P->cur_prio, a));
   return CUSFFT_SUCCESS;
 }
 

@@ -130,7 +130,12 @@ struct StagePackArgs {
   ZeroArgs zero;
 };
 
-// U: gathers in flight per thread (4: 4096 per SM at 4 CTAs of 256).
+// U: gathers in flight per thread per pass (1 at 4 CTAs of 256 per SM; U = 2, 4, 8 and 2-3 CTAs
+// per SM measured equal or slower once the schedule words are prefetched).
+#ifndef CUSFFT_STAGE_U
+#define CUSFFT_STAGE_U 1
+#endif
+constexpr int kStageU = CUSFFT_STAGE_U;
 template <int U>
 __global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
   pdl_wait();
@@ -148,24 +153,38 @@ __global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
   const uint32_t imask = (1u << A.ibits) - 1u;
   const uint32_t Bm = (1u << A.logB) - 1u, B2m = (1u << A.logB2) - 1u, Cm = (1u << A.logC) - 1u;
   const int T = gridDim.x * blockDim.x;
-  for (int q0 = blockIdx.x * blockDim.x + threadIdx.x; q0 < A.total; q0 += U * T) {
-    double2 v[U];
-    uint32_t cd[U];
+  // The schedule words are software-pipelined one iteration ahead: the next
+  // iteration's U words are requested while this iteration's gathers are in
+  // flight, so no gather waits on a dependent schedule load (round 1 issued
+  // word c, waited for it, then gather c: U + 1 DRAM round trips per pass).
+  auto load_codes = [&](int q0, uint32_t* cd) {
 #pragma unroll
     for (int c = 0; c < U; ++c) {
       const int q = q0 + c * T;
-      if (q < A.total) {
-        cd[c] = __ldg(A.code + q);
+      cd[c] = 0u;
+      if (q < A.total)
+        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;"
+                     : "=r"(cd[c]) : "l"(A.code + q), "l"(pf));
+    }
+  };
+  uint32_t cd[U];
+  load_codes(blockIdx.x * blockDim.x + threadIdx.x, cd);
+  for (int q0 = blockIdx.x * blockDim.x + threadIdx.x; q0 < A.total; q0 += U * T) {
+    double2 v[U];
+#pragma unroll
+    for (int c = 0; c < U; ++c) {
+      if (q0 + c * T < A.total) {
         const uint32_t sl = cd[c] >> A.ibits, i = cd[c] & imask;
         const double2* p = A.x + ((ssig[sl] * i + stau[sl]) & A.nmask);
         asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.L2::64B.v2.f64 {%0, %1}, [%2], %3;"
                      : "=d"(v[c].x), "=d"(v[c].y) : "l"(p), "l"(pf));
       }
     }
+    uint32_t nx[U];
+    load_codes(q0 + U * T, nx);
 #pragma unroll
     for (int c = 0; c < U; ++c) {
-      const int q = q0 + c * T;
-      if (q < A.total) {
+      if (q0 + c * T < A.total) {
         const uint32_t sl = cd[c] >> A.ibits, i = cd[c] & imask;
         const uint32_t rr = i >> A.logB, j = i & Bm;
         const uint32_t col = j & B2m, j1 = j >> A.logB2;
@@ -173,6 +192,7 @@ __global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
         asm volatile("st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %3;" ::"l"(A.staging + dst), "d"(v[c].x),
                      "d"(v[c].y), "l"(pl));
       }
+      cd[c] = nx[c];
     }
   }
   TRACE_END(6);
