@@ -311,10 +311,11 @@ def run_gpu(args):
     else:  # the plan owns the exchange: rank 0's ncclUniqueId broadcast once over the process group
         uid = [nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(uid, src=0)
-        shard = 1 if args.shard == "signal" else 0
+        shard = {"loops": 0, "signal": 1, "loops2": 2}[args.shard]
+        extra = dict(max_hits=8192) if shard == 2 else {}  # exchange #2 moves max_hits x L x 16 B
         plan = Plan(n, k, B=B, L=L, seed=args.plan_seed, device=local_rank, rank=rank, world=world,
-                    nccl_id=uid[0], shard_mode=shard, **prm)
-        if shard:  # this rank holds only its slice of x
+                    nccl_id=uid[0], shard_mode=shard, **prm, **extra)
+        if shard == 1:  # this rank holds only its slice of x
             span = n // world
             x = x[rank * span:(rank + 1) * span].clone()
     plan_ms = 1e3 * (time.perf_counter() - t_plan0)
@@ -472,6 +473,7 @@ def run_gpu(args):
                     ("cutoff_sort_alg3", dict(cutoff_mode=1)),
                     ("cutoff_threshold_alg6", dict(cutoff_mode=2, cutoff_threshold=1e-3)),
                     ("direct_gather_no_stage", dict(gather=1)),
+                    ("remap_execute_paper_sec5a", dict(gather=2)),
                     ("no_l2_persist", dict(l2_persist=0))]
         for name, kw in variants:
             p2 = Plan(n, k, B=B, L=L, seed=args.plan_seed, device=local_rank, **{**prm, **kw})
@@ -497,7 +499,7 @@ def run_gpu(args):
     # carries all of the transform's HBM traffic.  Algorithmic bytes: 32 B per
     # distinct sector of x the plan's gathers touch.
     sum_w = int(info["w_loc"]) * plan.loc_loops + int(info["w"]) * (L - plan.loc_loops) if info["filters"] == 2 else L * plan.w
-    lw_local = sum_w // world if world > 1 and args.shard == "loops" else sum_w
+    lw_local = sum_w // world if world > 1 and args.shard in ("loops", "loops2") else sum_w
     gather_bytes = lw_local * 32  # one 32-B sector per gathered 16-B sample (L w 32 B)
     rk_ms = gather["warm"]["ms"] if "warm" in gather else stage_ms.get("fold", 0.0)
     achieved = gather_bytes / (rk_ms * 1e-3) / 1e9
@@ -682,8 +684,10 @@ def main():
     ap.add_argument("--config", default="C3", choices=sorted(CONFIGS))
     ap.add_argument("--signal-seed", type=int, default=1)
     ap.add_argument("--plan-seed", type=int, default=3)
-    ap.add_argument("--shard", default="loops", choices=["loops", "signal"],
-                    help="N>1: loop sharding (all-gather) or signal sharding (SURVEY N1, all-reduce)")
+    ap.add_argument("--shard", default="loops", choices=["loops", "signal", "loops2"],
+                    help="N>1: loop sharding (one all-gather of the per-loop records), signal sharding "
+                         "(SURVEY N1, all-reduce) or loop sharding with two all-gathers (candidates, then "
+                         "per-loop estimates: SURVEY 8(e) steps 1-5)")
     ap.add_argument("--B", type=int, default=0, help="bucket count (default: the paper's formula, DESIGN.md Z3)")
     ap.add_argument("--pipeline", type=int, default=2, help="C5 batch: clone plans in flight per GPU")
     ap.add_argument("--cpu-budget-s", type=float, default=15.0)

@@ -113,14 +113,17 @@ typedef struct {
                               keeps ownership.                                                    */
   int64_t num_taps;        /* length of taps when taps != NULL (odd not required)                */
   int32_t cutoff_mode;     /* cusfft_cutoff_t; default EXACT                                      */
-  int32_t shard_mode;      /* cusfft_plan_dist only: 0 = loops (default), 1 = signal range       */
+  int32_t shard_mode;      /* cusfft_plan_dist: 0 = loops, one all-gather (default); 1 = signal range;
+                              2 = loops, two all-gathers (candidates, then per-loop estimates)      */
   double cutoff_threshold; /* THRESHOLD mode: absolute |u^|^2 threshold (> 0)                    */
   double loc_tolerance;    /* delta of the location loops' filter; 0 (default): tolerance        */
   double loc_lobefrac;     /* lambda of the location loops' filter; 0 (default): lobefrac        */
   int32_t l2_persist;      /* 1 (default): staged plans raise the device's persisting-L2 set-aside
                               while they live (see above); 0: never touch the device limit       */
   int32_t gather;          /* 0 (default): address-sorted staged gather when its staging buffer fits
-                              L2, else direct; 1: always the direct gather       */
+                              L2, else direct; 1: always the direct gather;
+                              2: the paper's remap + execute kernels on concurrent streams
+                              (an ablation; not with shard_mode 1)           */
 } cusfft_params;
 
 /* Fill *p with the defaults for (n, k, B).  Returns CUSFFT_NULL_PTR / INVALID_*.
@@ -156,6 +159,17 @@ int cusfft_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L,
  * L loops; the exchange is a SUM ALL-REDUCE (fp64) of the whole buffer (the
  * B-point FFT is linear, so partial bucket spectra add); every rank then runs
  * Steps 4-6.  Equal to world = 1 within fp64 rounding (the sum order differs).
+ * shard_mode 2 (loops, TWO collectives, the
+ * north_star's "candidate-index and per-loop estimate lists combined by
+ * all-gather"): loops owned as in mode 0; exchange #1 all-gathers the
+ * location loops' candidate records (cutoff bitmap | count | J, no u^);
+ * every rank then votes over all location loops (identical hit set, L91-L93),
+ * sorts the hits ascending and estimates ITS loops for every hit (Alg. 5
+ * L308-L325); exchange #2 all-gathers those per-loop estimates; every rank
+ * takes the medians (L95, Alg. 5) and selects the output.  Bit-
+ * identical to world = 1.  Needs max_hits <= 32768 (the hit list is sorted in
+ * shared memory) and L <= 64; exchange #2 moves world x max_hits x L/world x 16
+ * bytes, so set max_hits near the expected hit count.
  *
  * nccl_unique_id: NULL, or 128 bytes from cusfft_nccl_unique_id on one rank,
  * distributed to every rank by the caller (any channel).  With an id the plan
@@ -226,16 +240,31 @@ int cusfft_execute_host(cusfft_plan_t plan, const void* h_x, int64_t* h_locs, vo
  * (L81-L89), independent across loops until the vote (L93). */
 int cusfft_execute_local(cusfft_plan_t plan, const void* d_x);
 /* Steps 5-6 plus output selection, after the exchange buffer holds every
- * rank's slice.  Outputs as in cusfft_execute.  Paper: Steps 5-6 (L91-L95,
+ * rank's slice (shard_mode 2: after the second exchange; the medians and the
+ * output only).  Outputs as in cusfft_execute.  Paper: Steps 5-6 (L91-L95,
  * Alg. 4, Alg. 5). */
 int cusfft_execute_finish(cusfft_plan_t plan, int64_t* d_locs, void* d_vals);
+/* shard_mode 2 only, between the two exchanges: the vote over every location
+ * loop from the gathered candidate records (L91-L93, Alg. 4), the
+ * hit list sorted ascending, and this rank's per-loop estimates of every hit
+ * (Alg. 5) into its slice of exchange buffer 2.  CUSFFT_INVALID_PARAM
+ * for other plans. */
+int cusfft_execute_mid(cusfft_plan_t plan);
 /* Plumbing of the caller-run exchange (no paper passage).
  * The exchange buffer: *d_buf points at world * (*bytes_per_rank) bytes of
  * device memory, rank r's slice at offset r * (*bytes_per_rank) (loop
  * sharding); for signal sharding *bytes_per_rank is the whole buffer. */
 int cusfft_exchange_buffer(cusfft_plan_t plan, void** d_buf, int64_t* bytes_per_rank);
+/* shard_mode 2: exchange buffer 1 (cusfft_exchange_buffer) holds the candidate
+ * records, world slices of ceil(L_loc / world) records; exchange buffer 2 the
+ * per-loop estimates, world slices of max_hits x (L / world) complex fp64
+ * (rank-major, hit-major).  Both are all-gathered (rank r's slice at offset
+ * r * bytes_per_rank).  CUSFFT_INVALID_PARAM for other plans. */
+int cusfft_exchange_buffer2(cusfft_plan_t plan, void** d_buf, int64_t* bytes_per_rank);
 /* 0: all-gather of the rank slices (loop sharding); 1: element-wise fp64 sum
- * all-reduce of the whole buffer (signal sharding); negative: error. */
+ * all-reduce of the whole buffer (signal sharding); 2: two all-gathers
+ * (shard_mode 2: buffer 1 after cusfft_execute_local, buffer 2 after
+ * cusfft_execute_mid); negative: error. */
 int32_t cusfft_exchange_kind(cusfft_plan_t plan);
 
 /* Paper: a and ai of Alg. 1 (L146-L153), the offset of Def. 1 (L81), the

@@ -33,7 +33,8 @@ EXPORTED = (
     "cusfft_params_default", "cusfft_default_B", "cusfft_plan", "cusfft_plan_dist", "cusfft_nccl_unique_id",
     "cusfft_destroy", "cusfft_set_stream", "cusfft_execute", "cusfft_execute_host", "cusfft_execute_batch",
     "cusfft_set_pipeline",
-    "cusfft_execute_local", "cusfft_execute_finish", "cusfft_exchange_buffer", "cusfft_exchange_kind",
+    "cusfft_execute_local", "cusfft_execute_mid", "cusfft_execute_finish", "cusfft_exchange_buffer",
+    "cusfft_exchange_buffer2", "cusfft_exchange_kind",
     "cusfft_get_info", "cusfft_get_debug", "cusfft_status", "cusfft_set_timing",
     "cusfft_get_stage_times", "cusfft_set_stage_limit", "cusfft_launches_per_execute", "cusfft_strerror",
     "cusfft_last_cuda_error", "cusfft_last_nccl_error", "cusfft_abi_version",
@@ -95,8 +96,10 @@ def load_library():
         "cusfft_execute_batch": (ctypes.c_int, [P, P, i64, i64, P, P]),
         "cusfft_set_pipeline": (ctypes.c_int, [P, i32]),
         "cusfft_execute_local": (ctypes.c_int, [P, P]),
+        "cusfft_execute_mid": (ctypes.c_int, [P]),
         "cusfft_execute_finish": (ctypes.c_int, [P, P, P]),
         "cusfft_exchange_buffer": (ctypes.c_int, [P, ctypes.POINTER(P), ctypes.POINTER(i64)]),
+        "cusfft_exchange_buffer2": (ctypes.c_int, [P, ctypes.POINTER(P), ctypes.POINTER(i64)]),
         "cusfft_exchange_kind": (i32, [P]),
         "cusfft_get_info": (ctypes.c_int, [P, P, P, P, P]),
         "cusfft_get_debug": (i64, [P, i32, P, i64]),
@@ -297,6 +300,11 @@ class Plan:
         self._use_current_stream()
         check(self._lib.cusfft_execute_local(self._h, ctypes.c_void_p(x.data_ptr())), "cusfft_execute_local")
 
+    def execute_mid(self):
+        """shard_mode 2, between the two exchanges: vote, sorted hit list, this rank's per-loop estimates."""
+        self._use_current_stream()
+        check(self._lib.cusfft_execute_mid(self._h), "cusfft_execute_mid")
+
     def execute_finish(self, locs, vals):
         self._use_current_stream()
         check(self._lib.cusfft_execute_finish(self._h, ctypes.c_void_p(locs.data_ptr()),
@@ -311,8 +319,17 @@ class Plan:
               "cusfft_exchange_buffer")
         return int(ptr.value), int(per.value)
 
+    def exchange_buffer2(self):
+        """shard_mode 2: (device pointer, bytes per rank) of the per-loop estimate all-gather buffer."""
+        ptr = ctypes.c_void_p()
+        per = ctypes.c_int64()
+        check(self._lib.cusfft_exchange_buffer2(self._h, ctypes.byref(ptr), ctypes.byref(per)),
+              "cusfft_exchange_buffer2")
+        return int(ptr.value), int(per.value)
+
     def exchange_kind(self) -> int:
-        """0: all-gather of rank slices (loop sharding); 1: fp64 sum all-reduce (signal sharding)."""
+        """0: all-gather of rank slices (loop sharding); 1: fp64 sum all-reduce (signal sharding);
+        2: two all-gathers (shard_mode 2: candidate records, then per-loop estimates)."""
         k = int(self._lib.cusfft_exchange_kind(self._h))
         if k < 0:
             check(k, "cusfft_exchange_kind")

@@ -19,7 +19,7 @@
 
 #include "../../include/cusfft.h"
 #include "plan_kernels.cuh"
-#include "tail.cuh"
+#include "exchange.cuh"
 
 using namespace cusfft;
 
@@ -185,6 +185,11 @@ struct cusfft_plan_s {
   std::vector<uint32_t> row0_h;              // same, host (+ total rows at [Lg])
   double2* d_staging = nullptr;              // [rows][B]
   int stage_grid = 1;
+  // gather 2 (ablation): the paper's remap + execute kernels on concurrent streams
+  bool remap = false;
+  double2* d_remap = nullptr;                // [nrm][B] one reordered chunk A' per stream
+  std::vector<cudaStream_t> rm_st;
+  std::vector<cudaEvent_t> rm_ev;            // [0] fork, [1 + i] join of stream i
   bool p2_ms = true;                         // phase 2 in the multi-slot form (k_fold_fft1_ms, R <= 16)
   int p2_spc = 2;                            // phase-2 slots per CTA (taps reused across them; 1 / 4 slower)
   int fork_at = 1;                           // estimation branch forks after phase 1 (0) or after the location phase 2 (1, measured ~0.5 us faster)
@@ -207,6 +212,13 @@ struct cusfft_plan_s {
   bool sel_cluster = false;       // k_select_cluster (256 <= B <= 65536, EXACT / THRESHOLD modes)
   int select1_smem = 0;
   // fused vote + estimate + output (k_tail) when its table fits shared memory
+  // shard_mode 2 (two all-gathers, exchange.cuh): candidate records, then per-loop estimates
+  bool mode2 = false;
+  int cmax = 0;                   // candidate records per rank slice (location loops of the busiest rank)
+  int64_t crec_bytes = 0;         // one candidate record: bitmap | count | J (the record's tail)
+  uint8_t* d_cand = nullptr;      // [world][cmax][crec_bytes]
+  double2* d_x2 = nullptr;        // [world][max_hits][Lg] per-loop estimates
+  int sort_smem = 0;              // k_hits_sort: npow2(max_hits) x 4 B
   int tail_esz = 0;               // bytes per vote-table element (1 / 2 / 4), 0: the k_vote / k_estimate / k_output chain
   int tail_smem = 0, tail_qoff = 0, tail_grid = 1;
   bool pk_direct = false;         // the cluster cutoff ORs its winners into k_tail's table (d_pk, zero block)
@@ -241,7 +253,7 @@ struct cusfft_plan_s {
     const void* b = nullptr;
     const void* c = nullptr;
     cudaGraphExec_t exec = nullptr;
-  } g_local, g_finish;
+  } g_local, g_mid, g_finish;
   // whole-transform graphs by (x, locs, vals): up to kGraphCache, least recently used replaced
   std::vector<GraphEntry> g_cache;
   std::vector<uint64_t> g_used;
@@ -313,12 +325,12 @@ void free_plan(cusfft_plan_t p) {
   }
   void* ptrs[] = {p->d_code, p->d_row0, p->d_staging, p->d_tw, p->d_ph_hi, p->d_ph_lo, p->d_slots, p->d_loc_sigma, p->d_u, p->d_v,
                   p->d_records, p->d_keys, p->d_zero, p->d_key_index, p->d_hits, p->d_hit_vals, p->d_hit_keys,
-                  p->d_per_loop, p->d_xbuf, p->d_locs_buf, p->d_vals_buf};
+                  p->d_per_loop, p->d_xbuf, p->d_locs_buf, p->d_vals_buf, p->d_cand, p->d_x2};
   for (void* q : ptrs)
     if (q) cudaFree(q);
   if (p->ev_made)
     for (auto& e : p->ev) cudaEventDestroy(e);
-  for (auto* g : {&p->g_local, &p->g_finish})
+  for (auto* g : {&p->g_local, &p->g_mid, &p->g_finish})
     if (g->exec) cudaGraphExecDestroy(g->exec);
   for (auto& g : p->g_cache)
     if (g.exec) cudaGraphExecDestroy(g.exec);
@@ -332,6 +344,9 @@ void free_plan(cusfft_plan_t p) {
   if (p->cap_stream2) cudaStreamDestroy(p->cap_stream2);
   if (p->ev_fork) cudaEventDestroy(p->ev_fork);
   if (p->ev_join) cudaEventDestroy(p->ev_join);
+  for (auto st : p->rm_st) cudaStreamDestroy(st);
+  for (auto e : p->rm_ev) cudaEventDestroy(e);
+  if (p->d_remap) cudaFree(p->d_remap);
   if (p->setaside) setaside_release(p->device);
   p->magic = 0;
   delete p;
@@ -343,7 +358,9 @@ int validate(int64_t n, int64_t k, int64_t B, int32_t L, const cusfft_params& q,
   if (L < 1 || L > kMaxLoops) return CUSFFT_INVALID_LOOPS;
   if (q.loc_loops > kMaxLoc) return CUSFFT_INVALID_LOOPS;
   if (world < 1 || rank < 0 || rank >= world) return CUSFFT_INVALID_LOOPS;
-  if (q.shard_mode != 0 && q.shard_mode != 1) return CUSFFT_INVALID_PARAM;
+  if (q.shard_mode < 0 || q.shard_mode > 2) return CUSFFT_INVALID_PARAM;
+  // shard_mode 2: the hit list is sorted in one CTA's shared memory, the median holds L values per thread
+  if (q.shard_mode == 2 && (q.max_hits > 32768 || L > kMedMaxL)) return CUSFFT_INVALID_PARAM;
   if (q.shard_mode == 1 && world > 1) {
     if (n % world) return CUSFFT_INVALID_PARAM;
   } else if (L % world) {
@@ -368,7 +385,8 @@ int validate(int64_t n, int64_t k, int64_t B, int32_t L, const cusfft_params& q,
   if (q.cutoff_mode == CUSFFT_CUTOFF_THRESHOLD && !(q.cutoff_threshold > 0.0)) return CUSFFT_INVALID_PARAM;
   if (q.tau_mode != 0 && q.tau_mode != 1) return CUSFFT_INVALID_PARAM;
   if (q.l2_persist != 0 && q.l2_persist != 1) return CUSFFT_INVALID_PARAM;
-  if (q.gather != 0 && q.gather != 1) return CUSFFT_INVALID_PARAM;
+  if (q.gather < 0 || q.gather > 2) return CUSFFT_INVALID_PARAM;
+  if (q.gather == 2 && q.shard_mode == 1) return CUSFFT_INVALID_PARAM;  // the remap ablation folds whole signals
   return CUSFFT_SUCCESS;
 }
 
@@ -678,7 +696,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   }
   P->logB1 = ilog2(P->B1);
   P->logB2 = ilog2(P->B2);
-  P->fused1 = P->B1 > 1 && P->B1 <= 256;
+  P->fused1 = P->B1 > 1 && P->B1 <= 256 && q.gather != 2;  // gather 2: the paper's remap + execute (unfused)
   P->kp2 = 1;
   while (P->kp2 < k) P->kp2 <<= 1;
   int smem_optin = 200 * 1024;
@@ -694,7 +712,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     const int64_t tab = ((int64_t)B * esz + 15) & ~int64_t(15);
     const int64_t need = tab + (kTailNT / 32) * kTailQ * 2;
     const char* et = std::getenv("CUSFFT_TAIL");  // CUSFFT_TAIL=0: the k_vote / k_estimate chain (tests, A/B)
-    if (need + 8 * 1024 <= smem_optin && !(et && et[0] == '0')) {  // + k_tail's static smem (hit queue)
+    // (shard_mode 2 votes with k_vote and estimates per rank: no fused tail)
+    if (need + 8 * 1024 <= smem_optin && !(et && et[0] == '0') && q.shard_mode != 2) {  // + k_tail's static smem (hit queue)
       P->tail_esz = esz;
       P->tail_qoff = (int)tab;
       P->tail_smem = (int)need;
@@ -852,8 +871,9 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       if ((rc = dalloc(&P->d_row0, (size_t)P->Lg))) return fail(rc);
       if ((rc = upload(P->d_row0, P->row0_h.data(), (size_t)P->Lg * sizeof(uint32_t)))) return fail(rc);
       if ((rc = dalloc(&P->d_staging, (size_t)(rows * B)))) return fail(rc);
-      // one resident wave of phase-1 CTAs (grid-stride loop), at most 4 per SM: with 4 gathers in
-      // flight per thread that is 4096 per SM, measured best
+      // one resident wave of phase-1 CTAs (grid-stride loop), at most 4 per SM: with one gather in
+      // flight per thread (schedule words prefetched) that is 1024 per SM, measured best
+      // (profiles/r02_stage_ab.md; dynamic chunking of the last quarter measured slower)
       int occ = 0;
       if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_stage_packed<kStageU>, 256, 0) != cudaSuccess || occ < 1) occ = 4;
       cudaGetLastError();
@@ -872,6 +892,38 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
         P->setaside = true;
       }
     }
+  }
+  if (q.gather == 2 && !P->staged) {  // the remap ablation: one chunk buffer and stream per concurrent loop
+    P->remap = true;
+    const int nrm = std::min(P->Lg, 32);  // GK110's 32 concurrent kernels (L351)
+    if ((rc = dalloc(&P->d_remap, (size_t)nrm * B))) return fail(rc);
+    P->rm_st.assign((size_t)nrm, nullptr);
+    P->rm_ev.assign((size_t)nrm + 1, nullptr);
+    for (auto& st : P->rm_st)
+      if (cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking) != cudaSuccess) {
+        g_last_cuda_error = (int)cudaGetLastError();
+        return fail(CUSFFT_CUDA);
+      }
+    for (auto& e : P->rm_ev)
+      if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess) {
+        g_last_cuda_error = (int)cudaGetLastError();
+        return fail(CUSFFT_CUDA);
+      }
+  }
+  if (q.shard_mode == 2) {  // two all-gathers: candidate records, then per-loop estimates (exchange.cuh)
+    P->mode2 = true;
+    P->cmax = (P->Lloc + world - 1) / world;
+    P->crec_bytes = P->lay.rec_bytes - P->lay.off_bitmap;
+    int np2 = 2;
+    while (np2 < P->max_hits) np2 <<= 1;
+    P->sort_smem = np2 * 4;
+    if (P->sort_smem > smem_optin) return fail(CUSFFT_INVALID_PARAM);
+    if (cudaFuncSetAttribute(k_hits_sort, cudaFuncAttributeMaxDynamicSharedMemorySize, P->sort_smem) != cudaSuccess) {
+      g_last_cuda_error = (int)cudaGetLastError();
+      return fail(CUSFFT_CUDA);
+    }
+    if ((rc = dalloc(&P->d_cand, (size_t)(world * P->cmax * P->crec_bytes)))) return fail(rc);
+    if ((rc = dalloc(&P->d_x2, (size_t)world * P->max_hits * P->Lg))) return fail(rc);
   }
   if (nccl_id) {  // the library-owned exchange (a world of 1 is allowed: a one-rank communicator)
     ncclUniqueId id;
@@ -957,6 +1009,37 @@ cudaError_t launch_direct_t(cusfft_plan_t P, const Filter& F, const double2* x, 
                   (const double2*)P->d_tw, (int)P->B, P->B2, F.w, F.R, (uint32_t)(P->n - 1), P->xlo, P->xspan, z);
 }
 
+// Steps 1+2 as the paper's asynchronous data layout transformation (gather 2,
+// PAPER.md:L345-L351, Fig. 4): per loop and chunk of B taps a remapping kernel
+// (A'[j] = x[index]) and an execution kernel (u += g A'); loop s on stream
+// s mod nrm, the streams forked from and joined back to st.
+int launch_remap(cusfft_plan_t P, const double2* x, int s0, int s1, cudaStream_t st, bool zero_block) {
+  const int B = (int)P->B;
+  const int nrm = (int)P->rm_st.size();
+  if (zero_block) CK(cudaMemsetAsync(P->d_zero, 0, (size_t)P->nzero * sizeof(int), st));
+  CK(cudaEventRecord(P->rm_ev[0], st));
+  for (int i = 0; i < nrm; ++i) CK(cudaStreamWaitEvent(P->rm_st[(size_t)i], P->rm_ev[0], 0));
+  const dim3 grid((unsigned)((B + 255) / 256)), blk(256);
+  for (int s = s0; s < s1; ++s) {
+    const int i = (s - s0) % nrm;
+    cudaStream_t rs = P->rm_st[(size_t)i];
+    double2* ap = P->d_remap + (size_t)i * B;
+    const Filter& F = P->filt[P->filt_of_local(s)];
+    const SlotParam& sp = P->slots_h[(size_t)P->lrank * P->Lg + s];
+    double2* u = P->d_u + (size_t)s * B;
+    for (int rr = 0; rr < F.R; ++rr) {
+      k_remap<<<grid, blk, 0, rs>>>(x, ap, sp.sigma, sp.tau, rr * B, B, F.w, (uint32_t)(P->n - 1));
+      k_remap_exec<<<grid, blk, 0, rs>>>(ap, (const double*)F.d_taps, u, rr * B, B, F.w);
+    }
+  }
+  CK(cudaGetLastError());
+  for (int i = 0; i < nrm; ++i) {
+    CK(cudaEventRecord(P->rm_ev[(size_t)i + 1], P->rm_st[(size_t)i]));
+    CK(cudaStreamWaitEvent(st, P->rm_ev[(size_t)i + 1], 0));
+  }
+  return CUSFFT_SUCCESS;
+}
+
 // Steps 1+2 (and the fused FFT pass 1) for local slots [s0, s1), all of one
 // filter: phase 2 of the staged fold, or the direct gather.
 int launch_fold_range(cusfft_plan_t P, const double2* x, int s0, int s1, cudaStream_t st, bool zero_block) {
@@ -981,6 +1064,8 @@ int launch_fold_range(cusfft_plan_t P, const double2* x, int s0, int s1, cudaStr
       case 128: e = launch_direct_t<128>(P, F, x, sp, u, v, s1 - s0, z, st); break;
       case 256: e = launch_direct_t<256>(P, F, x, sp, u, v, s1 - s0, z, st); break;
     }
+  } else if (P->remap) {
+    return launch_remap(P, x, s0, s1, st, zero_block);
   } else {
     dim3 grid((unsigned)((B + 255) / 256), (unsigned)(s1 - s0));
     e = launch_k(k_fold<16>, grid, dim3(256), 0, st, P->cur_prio, x, (const double*)F.d_taps, sp, u, (int)B, F.w,
@@ -1030,6 +1115,9 @@ SelArgs make_sel_args(cusfft_plan_t P) {
   sa.status = P->d_flags + 1;
   sa.pk = P->d_pk;
   sa.pk_esz = P->tail_esz;
+  if (P->mode2)  // this rank's location slots are its first local slots, in order
+    for (size_t i = 0; i < P->sel_slots_h.size(); ++i)
+      sa.cout[i] = P->d_cand + ((int64_t)P->rank * P->cmax + (int64_t)i) * P->crec_bytes;
   sa.threshold_mode = P->prm.cutoff_mode == CUSFFT_CUTOFF_THRESHOLD ? 1 : 0;
   {
     const double th = P->prm.cutoff_threshold;
@@ -1079,7 +1167,9 @@ int launch_select(cusfft_plan_t P, cudaStream_t st) {
 // slots = this rank's location slots [0, nloc_local) in order, shapes with
 // compiled instances (B = 8192, 16384, 32768).
 bool use_fft2_select(cusfft_plan_t P) {
-  if (!P->sel_cluster || P->xshard || P->prm.cutoff_mode != CUSFFT_CUTOFF_EXACT || P->B1 <= 1 || !P->fft2sel)
+  // (the location slots' FFT pass 1 must have run inside the fold: fused1)
+  if (!P->sel_cluster || P->xshard || P->prm.cutoff_mode != CUSFFT_CUTOFF_EXACT || P->B1 <= 1 || !P->fft2sel ||
+      !P->fused1)
     return false;
   const int key = P->B2 * 1000 + P->B1 / kSelCL;
   if (key != 64016 && key != 128016 && key != 128032) return false;
@@ -1149,6 +1239,13 @@ VoteArgs make_vote_args(cusfft_plan_t P) {
     va.bmp[q] = reinterpret_cast<const uint32_t*>(rec + P->lay.off_bitmap);
     va.Jp[q] = reinterpret_cast<const int*>(rec + P->lay.off_J);
     va.cntp[q] = reinterpret_cast<const int*>(rec + P->lay.off_cnt);
+    if (P->mode2) {  // the gathered candidate record: rank g = slot / Lg, its location slot i = slot mod Lg
+      const int64_t s = P->loc_slots_h[q];
+      const uint8_t* c = P->d_cand + ((s / P->Lg) * P->cmax + s % P->Lg) * P->crec_bytes;
+      va.bmp[q] = reinterpret_cast<const uint32_t*>(c);
+      va.Jp[q] = reinterpret_cast<const int*>(c + (P->lay.off_J - P->lay.off_bitmap));
+      va.cntp[q] = reinterpret_cast<const int*>(c + (P->lay.off_cnt - P->lay.off_bitmap));
+    }
     va.sig[q] = P->slots_h[P->loc_slots_h[q]].sigma;
     va.aa[q] = P->slots_h[P->loc_slots_h[q]].a;
   }
@@ -1241,6 +1338,40 @@ int launch_after_cutoff(cusfft_plan_t P, int64_t* locs, double2* vals, cudaStrea
   return CUSFFT_SUCCESS;
 }
 
+// shard_mode 2, after the candidate all-gather: every rank votes over all
+// location loops (k_vote), sorts the hit list (k_hits_sort) and estimates its
+// own loops for every hit into its slice of the estimate buffer (k_est_local).
+int launch_mid(cusfft_plan_t P, cudaStream_t st) {
+  if (P->stage_limit < 4) return CUSFFT_SUCCESS;
+  CK(launch_k(k_vote, dim3(P->vote_grid), dim3(256), P->vote_smem, st, P->cur_prio, make_vote_args(P)));
+  mark(P, 4);
+  if (P->stage_limit < 5) return CUSFFT_SUCCESS;
+  g_pdl = P->timing != 1;
+  CK(launch_k(k_hits_sort, dim3(1), dim3(kSortNT), (size_t)P->sort_smem, st, P->cur_prio, P->d_hits,
+              reinterpret_cast<const unsigned*>(P->d_flags), P->max_hits));
+  const int gx = std::max(1, std::min((P->max_hits * P->Lg + 255) / 256, P->sms * 4));
+  CK(launch_k(k_est_local, dim3(gx), dim3(256), 0, st, P->cur_prio, make_est_args(P), P->rank * P->Lg, P->Lg,
+              P->d_x2 + (size_t)P->rank * P->max_hits * P->Lg));
+  return CUSFFT_SUCCESS;
+}
+
+// shard_mode 2, after the estimate all-gather: medians (k_median) and the output.
+int launch_finish2(cusfft_plan_t P, int64_t* locs, double2* vals, cudaStream_t st) {
+  if (P->stage_limit < 5) return CUSFFT_SUCCESS;
+  const int gx = std::max(1, std::min((P->max_hits + 127) / 128, P->sms * 4));
+  CK(launch_k(k_median, dim3(gx), dim3(128), 0, st, P->cur_prio, make_est_args(P), (const double2*)P->d_x2,
+              P->world, P->Lg));
+  mark(P, 5);
+  if (P->stage_limit < 6) return CUSFFT_SUCCESS;
+  g_pdl = P->timing != 1;
+  CK(launch_k(k_output, dim3(1), dim3(1024), P->output_smem, st, P->cur_prio, (const int*)P->d_hits,
+              reinterpret_cast<const unsigned*>(P->d_flags), P->max_hits, (const double2*)P->d_hit_vals,
+              (const uint64_t*)P->d_hit_keys, P->d_ohist, (int)P->k, P->kp2, ilog2(P->n), locs, vals,
+              P->d_flags + 1));
+  mark(P, 6);
+  return CUSFFT_SUCCESS;
+}
+
 // Steps 1-4 of this rank's loops, one serial chain on P->stream.
 int launch_local(cusfft_plan_t P, const double2* x) {
   cudaStream_t st = P->stream;
@@ -1290,12 +1421,16 @@ int launch_finish(cusfft_plan_t P, int64_t* locs, double2* vals) {
 
 // The library-owned exchange (plans made with an ncclUniqueId): ONE collective
 // on the plan's stream, in place on the exchange buffer.
-int launch_exchange(cusfft_plan_t P, cudaStream_t st) {
+int launch_exchange(cusfft_plan_t P, cudaStream_t st, int which = 0) {
   if (!P->comm) return CUSFFT_SUCCESS;
   const NcclApi* api = nccl_api();
   const size_t per = (size_t)P->Lg * P->lay.rec_bytes;
   ncclResult_t r;
-  if (P->xshard)
+  if (P->mode2) {  // which 1: the candidate records; 2: the per-loop estimates (in place)
+    const size_t c = which == 1 ? (size_t)P->cmax * P->crec_bytes : (size_t)P->max_hits * P->Lg * sizeof(double2);
+    uint8_t* buf = which == 1 ? P->d_cand : reinterpret_cast<uint8_t*>(P->d_x2);
+    r = api->AllGather(buf + (size_t)P->rank * c, buf, c, ncclUint8, P->comm, st);
+  } else if (P->xshard)
     r = api->AllReduce(P->d_records, P->d_records, (size_t)P->L * P->lay.rec_bytes / 8, ncclFloat64, ncclSum, P->comm, st);
   else
     r = api->AllGather(P->d_records + (size_t)P->rank * per, P->d_records, per, ncclUint8, P->comm, st);
@@ -1304,6 +1439,17 @@ int launch_exchange(cusfft_plan_t P, cudaStream_t st) {
     return CUSFFT_NCCL;
   }
   return CUSFFT_SUCCESS;
+}
+
+// shard_mode 2 after Steps 1-4: candidate all-gather, vote + sort + local
+// estimates, estimate all-gather, medians + output (exchange.cuh).
+int launch_rest2(cusfft_plan_t P, int64_t* locs, double2* vals, cudaStream_t st) {
+  g_pdl = false;
+  if (P->comm) TRY(launch_exchange(P, st, 1));
+  TRY(launch_mid(P, st));
+  g_pdl = false;
+  if (P->comm) TRY(launch_exchange(P, st, 2));
+  return launch_finish2(P, locs, vals, st);
 }
 
 // The whole transform as two concurrent branches (graph capture, staged
@@ -1353,6 +1499,7 @@ int launch_branched(cusfft_plan_t P, const double2* x, int64_t* locs, double2* v
   CK(cudaStreamWaitEvent(a, P->ev_join, 0));
   g_pdl = false;
   if (lim < 4) return CUSFFT_SUCCESS;
+  if (P->mode2) return launch_rest2(P, locs, vals, a);
   if (P->comm) {
     TRY(launch_exchange(P, a));
     return launch_finish(P, locs, vals);
@@ -1448,6 +1595,7 @@ int execute_full(cusfft_plan_t plan, const void* d_x, int64_t* d_locs, void* d_v
       return launch_branched(plan, x, d_locs, v);
     }
     TRY(launch_local(plan, x));
+    if (plan->mode2) return launch_rest2(plan, d_locs, v, plan->stream);
     if (plan->comm) {
       g_pdl = false;
       TRY(launch_exchange(plan, plan->stream));
@@ -1569,12 +1717,27 @@ int cusfft_execute_local(cusfft_plan_t plan, const void* d_x) {
                      [&] { return launch_local(plan, reinterpret_cast<const double2*>(d_x)); });
 }
 
+int cusfft_execute_mid(cusfft_plan_t plan) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  if (!plan->mode2) return CUSFFT_INVALID_PARAM;
+  DeviceGuard g(plan->device);
+  return run_graphed(plan, plan->g_mid, nullptr, nullptr, nullptr, [&] {
+    g_pdl = false;
+    return launch_mid(plan, plan->stream);
+  });
+}
+
 int cusfft_execute_finish(cusfft_plan_t plan, int64_t* d_locs, void* d_vals) {
   if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
   if (!d_locs || !d_vals) return CUSFFT_NULL_PTR;
   DeviceGuard g(plan->device);
-  return run_graphed(plan, plan->g_finish, d_locs, d_vals, nullptr,
-                     [&] { return launch_finish(plan, d_locs, reinterpret_cast<double2*>(d_vals)); });
+  return run_graphed(plan, plan->g_finish, d_locs, d_vals, nullptr, [&] {
+    if (plan->mode2) {
+      g_pdl = false;
+      return launch_finish2(plan, d_locs, reinterpret_cast<double2*>(d_vals), plan->stream);
+    }
+    return launch_finish(plan, d_locs, reinterpret_cast<double2*>(d_vals));
+  });
 }
 
 int cusfft_execute(cusfft_plan_t plan, const void* d_x, int64_t* d_locs, void* d_vals) {
@@ -1687,14 +1850,23 @@ int cusfft_execute_host(cusfft_plan_t plan, const void* h_x, int64_t* h_locs, vo
 int cusfft_exchange_buffer(cusfft_plan_t plan, void** d_buf, int64_t* bytes_per_rank) {
   if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
   if (!d_buf || !bytes_per_rank) return CUSFFT_NULL_PTR;
-  *d_buf = plan->d_records;
-  *bytes_per_rank = (int64_t)plan->Lg * plan->lay.rec_bytes;
+  *d_buf = plan->mode2 ? plan->d_cand : plan->d_records;
+  *bytes_per_rank = plan->mode2 ? (int64_t)plan->cmax * plan->crec_bytes : (int64_t)plan->Lg * plan->lay.rec_bytes;
+  return CUSFFT_SUCCESS;
+}
+
+int cusfft_exchange_buffer2(cusfft_plan_t plan, void** d_buf, int64_t* bytes_per_rank) {
+  if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
+  if (!d_buf || !bytes_per_rank) return CUSFFT_NULL_PTR;
+  if (!plan->mode2) return CUSFFT_INVALID_PARAM;
+  *d_buf = plan->d_x2;
+  *bytes_per_rank = (int64_t)plan->max_hits * plan->Lg * (int64_t)sizeof(double2);
   return CUSFFT_SUCCESS;
 }
 
 int32_t cusfft_exchange_kind(cusfft_plan_t plan) {
   if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
-  return plan->xshard ? 1 : 0;
+  return plan->mode2 ? 2 : plan->xshard ? 1 : 0;
 }
 
 int cusfft_get_info(cusfft_plan_t plan, int64_t* info, int64_t* a, int64_t* sigma, int64_t* tau) {
@@ -1753,7 +1925,12 @@ int64_t cusfft_get_debug(cusfft_plan_t plan, int32_t what, void* dst, int64_t ca
       break;
     case CUSFFT_DEBUG_WINNERS:
       for (int r = 0; r < plan->Lloc; ++r) {
-        const uint8_t* rec = plan->d_records + (int64_t)slot_of(r) * plan->lay.rec_bytes;
+        const int64_t s = slot_of(r);
+        // shard_mode 2: the gathered candidate record (its offsets relative to the record's bitmap)
+        const uint8_t* rec = plan->mode2
+                                 ? plan->d_cand + ((s / plan->Lg) * plan->cmax + s % plan->Lg) * plan->crec_bytes -
+                                       plan->lay.off_bitmap
+                                 : plan->d_records + s * plan->lay.rec_bytes;
         int cnt = 0;
         CK(cudaMemcpy(&cnt, rec + plan->lay.off_cnt, 4, cudaMemcpyDeviceToHost));
         cnt = std::max(0, std::min(cnt, plan->Jcap));
@@ -1884,6 +2061,11 @@ int32_t cusfft_launches_per_execute(cusfft_plan_t plan) {
   int n = (plan->staged ? 1 : 0) + ranges /*fold per slot range*/ +
           ffts * (pass1 ? 2 : 1) /*fft*/ + (plan->sel_slots_h.empty() ? 0 : 1) +
           (plan->xshard && !plan->sel_slots_h.empty() ? 1 : 0) /*keys*/ + (plan->tail_esz ? 2 : 3);
+  if (plan->mode2) n += 1;  // k_vote + k_hits_sort + k_est_local + k_median + k_output (not k_vote + k_tail / k_estimate + k_output)
+  if (plan->remap) {  // a remap + an execution kernel per chunk of B taps instead of one fold per range
+    n -= ranges;
+    for (int s = 0; s < plan->Lg; ++s) n += 2 * plan->filt[plan->filt_of_local(s)].R;
+  }
   return n;
 }
 

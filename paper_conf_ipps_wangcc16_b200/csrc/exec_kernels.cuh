@@ -94,6 +94,38 @@ __global__ void __launch_bounds__(256) k_fold(const double2* __restrict__ x, con
 }
 
 // ---------------------------------------------------------------------------
+// The paper's asynchronous data layout transformation (PAPER.md:L345-L351,
+// §V.A, Fig. 4) as an ablation (params.gather = 2): the fold of one loop is
+// split into a remapping kernel, A'[j] = x[index(i0 + j)] for one chunk of B
+// taps (chunk size B, L349), and an execution kernel that folds the chunk from
+// the reordered array, u[j] += g[i0 + j] A'[j]; chunks of different loops run
+// on concurrent streams.  Same per-bucket addition order as k_fold (rounds
+// ascending, __dmul_rn / __dadd_rn), so u is bit-identical.
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_remap(const double2* __restrict__ x, double2* __restrict__ ap,
+                                               uint32_t sigma, uint32_t tau, int i0, int B, int w, uint32_t nmask) {
+  const int j = blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= B) return;
+  const int i = i0 + j;
+  ap[j] = i < w ? ld_gather(x + ((sigma * (uint32_t)i + tau) & nmask)) : make_double2(0.0, 0.0);
+}
+
+__global__ void __launch_bounds__(256) k_remap_exec(const double2* __restrict__ ap, const double* __restrict__ taps,
+                                                    double2* __restrict__ u, int i0, int B, int w) {
+  const int j = blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= B) return;
+  const int i = i0 + j;
+  double2 acc = i0 == 0 ? make_double2(0.0, 0.0) : u[j];
+  if (i < w) {
+    const double g = __ldg(taps + i);
+    const double2 a = ap[j];
+    acc.x = __dadd_rn(acc.x, __dmul_rn(g, a.x));
+    acc.y = __dadd_rn(acc.y, __dmul_rn(g, a.y));
+  }
+  u[j] = acc;
+}
+
+// ---------------------------------------------------------------------------
 // Staged gather, phase 1: the plan sorted every (slot, tap)
 // gather of this rank by address; the kernel walks them in that order, so
 // DRAM rows are opened once for all loops' samples that share them (the
@@ -153,46 +185,55 @@ __global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
   const uint32_t imask = (1u << A.ibits) - 1u;
   const uint32_t Bm = (1u << A.logB) - 1u, B2m = (1u << A.logB2) - 1u, Cm = (1u << A.logC) - 1u;
   const int T = gridDim.x * blockDim.x;
-  // The schedule words are software-pipelined one iteration ahead: the next
-  // iteration's U words are requested while this iteration's gathers are in
-  // flight, so no gather waits on a dependent schedule load (round 1 issued
-  // word c, waited for it, then gather c: U + 1 DRAM round trips per pass).
-  auto load_codes = [&](int q0, uint32_t* cd) {
-#pragma unroll
-    for (int c = 0; c < U; ++c) {
-      const int q = q0 + c * T;
-      cd[c] = 0u;
-      if (q < A.total)
-        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;"
-                     : "=r"(cd[c]) : "l"(A.code + q), "l"(pf));
-    }
+  // The schedule words are software-pipelined one pass ahead: the next pass's
+  // words are requested while this pass's gathers are in flight, so no gather
+  // waits on a dependent schedule load (round 1 issued word c, waited for it,
+  // then gather c: U + 1 DRAM round trips per pass).
+  auto ld_code = [&](int q) {
+    uint32_t c;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(c) : "l"(A.code + q), "l"(pf));
+    return c;
   };
-  uint32_t cd[U];
-  load_codes(blockIdx.x * blockDim.x + threadIdx.x, cd);
-  for (int q0 = blockIdx.x * blockDim.x + threadIdx.x; q0 < A.total; q0 += U * T) {
-    double2 v[U];
+  auto gather = [&](uint32_t code, double2& v) {
+    const uint32_t sl = code >> A.ibits, i = code & imask;
+    const double2* p = A.x + ((ssig[sl] * i + stau[sl]) & A.nmask);
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.L2::64B.v2.f64 {%0, %1}, [%2], %3;"
+                 : "=d"(v.x), "=d"(v.y) : "l"(p), "l"(pf));
+  };
+  auto stage = [&](uint32_t code, const double2& v) {
+    const uint32_t sl = code >> A.ibits, i = code & imask;
+    const uint32_t rr = i >> A.logB, j = i & Bm;
+    const uint32_t col = j & B2m, j1 = j >> A.logB2;
+    const uint32_t dst = ((srow[sl] + rr) << A.logB) + ((col >> A.logC) << 8) + ((col & Cm) << A.logB1) + j1;
+    asm volatile("st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %3;" ::"l"(A.staging + dst), "d"(v.x), "d"(v.y),
+                 "l"(pl));
+  };
+  const int send = A.total;
+  {
+    uint32_t cd[U];
+    const int q00 = blockIdx.x * blockDim.x + threadIdx.x;
 #pragma unroll
     for (int c = 0; c < U; ++c) {
-      if (q0 + c * T < A.total) {
-        const uint32_t sl = cd[c] >> A.ibits, i = cd[c] & imask;
-        const double2* p = A.x + ((ssig[sl] * i + stau[sl]) & A.nmask);
-        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.L2::64B.v2.f64 {%0, %1}, [%2], %3;"
-                     : "=d"(v[c].x), "=d"(v[c].y) : "l"(p), "l"(pf));
-      }
+      cd[c] = 0u;
+      if (q00 + c * T < send) cd[c] = ld_code(q00 + c * T);
     }
-    uint32_t nx[U];
-    load_codes(q0 + U * T, nx);
+    for (int q0 = q00; q0 < send; q0 += U * T) {
+      double2 v[U];
 #pragma unroll
-    for (int c = 0; c < U; ++c) {
-      if (q0 + c * T < A.total) {
-        const uint32_t sl = cd[c] >> A.ibits, i = cd[c] & imask;
-        const uint32_t rr = i >> A.logB, j = i & Bm;
-        const uint32_t col = j & B2m, j1 = j >> A.logB2;
-        const uint32_t dst = ((srow[sl] + rr) << A.logB) + ((col >> A.logC) << 8) + ((col & Cm) << A.logB1) + j1;
-        asm volatile("st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %3;" ::"l"(A.staging + dst), "d"(v[c].x),
-                     "d"(v[c].y), "l"(pl));
+      for (int c = 0; c < U; ++c)
+        if (q0 + c * T < send) gather(cd[c], v[c]);
+      uint32_t nx[U];
+#pragma unroll
+      for (int c = 0; c < U; ++c) {
+        const int q = q0 + U * T + c * T;
+        nx[c] = 0u;
+        if (q < send) nx[c] = ld_code(q);
       }
-      cd[c] = nx[c];
+#pragma unroll
+      for (int c = 0; c < U; ++c) {
+        if (q0 + c * T < send) stage(cd[c], v[c]);
+        cd[c] = nx[c];
+      }
     }
   }
   TRACE_END(6);
@@ -644,7 +685,24 @@ struct SelArgs {
   // per execution
   uint32_t* pk;
   int pk_esz;      // bytes per pk element (1 / 2 / 4: L_loc <= 8 / 16 / 32)
+  // optional (shard_mode 2): where selection i writes its candidate record
+  // (bitmap | count | J with the record's relative offsets) instead of its
+  // record, i.e. this rank's slice of the candidate all-gather buffer
+  uint8_t* cout[kMaxSel];
 };
+
+struct SelOut {
+  uint32_t* bitmap;
+  int* cnt;
+  int* J;
+};
+__device__ __forceinline__ SelOut sel_out(const SelArgs& A, int sel, uint8_t* rec) {
+  if (uint8_t* c = A.cout[sel])
+    return {reinterpret_cast<uint32_t*>(c), reinterpret_cast<int*>(c + (A.lay.off_cnt - A.lay.off_bitmap)),
+            reinterpret_cast<int*>(c + (A.lay.off_J - A.lay.off_bitmap))};
+  return {reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap), reinterpret_cast<int*>(rec + A.lay.off_cnt),
+          reinterpret_cast<int*>(rec + A.lay.off_J)};
+}
 
 struct GKeySrc {
   const uint64_t* keys;
@@ -820,8 +878,9 @@ __device__ __forceinline__ void select1_body(const SelArgs& A, int sel, uint8_t*
   __syncthreads();
   if (sel == 0) TRACE(13);
   // bitmap out + ascending winner list (thread t owns words [t wpt, (t+1) wpt))
-  uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap);
-  int* J = reinterpret_cast<int*>(rec + A.lay.off_J);
+  const SelOut so = sel_out(A, sel, rec);
+  uint32_t* bitmap = so.bitmap;
+  int* J = so.J;
   for (int w = tid; w < words; w += 1024) {
     bitmap[w] = sbits[w];
     if (write_pk && A.pk) pk_or_word(A, sel, sbits[w], (int64_t)w * 32);
@@ -840,7 +899,7 @@ __device__ __forceinline__ void select1_body(const SelArgs& A, int sel, uint8_t*
     }
   }
   if (tid == 0) {
-    *reinterpret_cast<int*>(rec + A.lay.off_cnt) = total;
+    *so.cnt = total;
     if (!A.threshold_mode && total != A.num) atomicOr(A.status + 1, 1);
   }
   if (sel == 0) TRACE(14);
@@ -889,8 +948,9 @@ template <int NT = kSelCNT>
 __device__ __forceinline__ void select_cluster_write(const SelArgs& A, uint8_t* rec, const uint32_t* sbits, int sel,
                                                      int r, int wpc, int wpt, int k0, int pos, int total) {
   const int tid = threadIdx.x;
-  uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap) + r * wpc;
-  int* J = reinterpret_cast<int*>(rec + A.lay.off_J);
+  const SelOut so = sel_out(A, sel, rec);
+  uint32_t* bitmap = so.bitmap + r * wpc;
+  int* J = so.J;
   for (int w = tid; w < wpc; w += NT) bitmap[w] = sbits[w];
   if (A.pk)  // k_tail's vote table
     for (int w = tid; w < wpc; w += NT) pk_or_word(A, sel, sbits[w], (int64_t)(r * wpc + w) * 32);
@@ -903,7 +963,7 @@ __device__ __forceinline__ void select_cluster_write(const SelArgs& A, uint8_t* 
     }
   }
   if (r == 0 && tid == 0) {
-    *reinterpret_cast<int*>(rec + A.lay.off_cnt) = total;
+    *so.cnt = total;
     if (!A.threshold_mode && total != A.num) atomicOr(A.status + 1, 1);
   }
 }
@@ -1691,8 +1751,9 @@ __global__ void __launch_bounds__(1024) k_select_sort(SelArgs A) {
   }
   for (int r = tid; r < A.num; r += 1024) atomicOr(&sbits[si[r] >> 5], 1u << (si[r] & 31));
   __syncthreads();
-  uint32_t* bitmap = reinterpret_cast<uint32_t*>(rec + A.lay.off_bitmap);
-  int* J = reinterpret_cast<int*>(rec + A.lay.off_J);
+  const SelOut so = sel_out(A, sel, rec);
+  uint32_t* bitmap = so.bitmap;
+  int* J = so.J;
   const int wpt = (words + 1023) >> 10;
   int cnt = 0;
   for (int w = tid * wpt; w < min(words, (tid + 1) * wpt); ++w) {
@@ -1710,7 +1771,7 @@ __global__ void __launch_bounds__(1024) k_select_sort(SelArgs A) {
     }
   }
   if (tid == 0) {
-    *reinterpret_cast<int*>(rec + A.lay.off_cnt) = total;
+    *so.cnt = total;
     if (total != A.num) atomicOr(A.status + 1, 1);
   }
 }

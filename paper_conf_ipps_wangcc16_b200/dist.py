@@ -12,6 +12,13 @@ the vote, the estimation and the output selection redundantly, so outputs are
 identical on all ranks and identical to the single-GPU plan (the loop draws
 depend only on (seed, r)).
 
+* loops, two collectives (``shard_mode=2``, the
+north_star's design) -- the same loop ownership; exchange #1 all-gathers
+only the location loops' candidate records (cutoff bitmap, count, winner
+list J); every rank votes (identical hit set) and estimates ITS loops for
+every hit; exchange #2 all-gathers those per-loop estimates; every rank takes
+the medians and selects the output.  Bit-identical to the single-GPU plan.
+
 * signal (``shard_mode=1``) -- rank g holds only the slice
 x[g n/G, (g+1) n/G) and folds the samples it owns for ALL L loops (Step 1-2
 restricted to its range; PAPER.md:L92 -- the fold is a sum over samples, and the
@@ -26,8 +33,11 @@ engine, so the gloo CPU tests drive this exact code with a test engine:
   engine.local(x)            Steps 1-4 for this rank's loops
   engine.exchange_tensor()   the exchange buffer (uint8 [world * per_rank] for
                              the all-gather; float64 [...] for the all-reduce)
-  engine.exchange_kind       0 = all-gather (loops), 1 = sum all-reduce (signal)
-  engine.finish()            Steps 4-6 + output, returns (locs, vals)
+  engine.exchange_kind       0 = all-gather (loops), 1 = sum all-reduce (signal),
+                             2 = two all-gathers (loops, shard_mode 2)
+  engine.mid()               kind 2 only: vote + this rank's per-loop estimates
+  engine.exchange_tensor2()  kind 2 only: the per-loop estimate buffer
+  engine.finish()            Steps 4-6 + output (kind 2: medians + output), returns (locs, vals)
 """
 from __future__ import annotations
 
@@ -81,6 +91,11 @@ class CudaEngine:
             self._buf = torch.as_tensor(_CudaBuffer(ptr, per, "<f8", 8), device=self.device)
         else:
             self._buf = torch.as_tensor(_CudaBuffer(ptr, per * world), device=self.device)
+        self._buf2 = None
+        if self.exchange_kind == 2:
+            ptr2, per2 = self.plan.exchange_buffer2()
+            self.per_rank2 = per2
+            self._buf2 = torch.as_tensor(_CudaBuffer(ptr2, per2 * world), device=self.device)
         self.locs = torch.empty(k, dtype=torch.int64, device=self.device)
         self.vals = torch.empty(k, dtype=torch.complex128, device=self.device)
 
@@ -91,6 +106,12 @@ class CudaEngine:
     def exchange_tensor(self):
         return self._buf
 
+    def mid(self):
+        self.plan.execute_mid()
+
+    def exchange_tensor2(self):
+        return self._buf2
+
     def finish(self):
         self.plan.execute_finish(self.locs, self.vals)
         return self.locs, self.vals
@@ -99,11 +120,18 @@ class CudaEngine:
         return self.plan.launches_per_execute()
 
 
+def _all_gather_inplace(buf, rank, world, group):
+    per = buf.numel() // world
+    # in place: input is this rank's slice of the output (NCCL in-place all-gather)
+    dist.all_gather_into_tensor(buf, buf[rank * per:(rank + 1) * per], group=group)
+
+
 class LoopShardedSfft:
-    """execute(x) = local steps, ONE collective (the engine's exchange kind:
-    all-gather for loop sharding, sum all-reduce for signal sharding), then
-    the remaining steps on every rank.  x is the whole signal or this rank's
-    slice, as the engine expects."""
+    """execute(x) = local steps, the engine's exchange (kind 0: one all-gather
+    of the per-loop records; 1: one sum all-reduce of the partial spectra;
+    2: all-gather of the candidate records, the vote and this rank's per-loop
+    estimates, all-gather of those), then the remaining steps on every rank.
+    x is the whole signal or this rank's slice, as the engine expects."""
 
     def __init__(self, engine, group=None):
         self.engine = engine
@@ -113,15 +141,20 @@ class LoopShardedSfft:
 
     def execute(self, x):
         self.engine.local(x)
+        kind = getattr(self.engine, "exchange_kind", 0)
+        if kind == 2:
+            if self.world > 1:
+                _all_gather_inplace(self.engine.exchange_tensor(), self.rank, self.world, self.group)
+            self.engine.mid()
+            if self.world > 1:
+                _all_gather_inplace(self.engine.exchange_tensor2(), self.rank, self.world, self.group)
+            return self.engine.finish()
         if self.world > 1:
             buf = self.engine.exchange_tensor()
-            if getattr(self.engine, "exchange_kind", 0) == 1:
+            if kind == 1:
                 dist.all_reduce(buf, op=dist.ReduceOp.SUM, group=self.group)
                 return self.engine.finish()
-            per = buf.numel() // self.world
-            mine = buf[self.rank * per:(self.rank + 1) * per]
-            # in place: input is this rank's slice of the output (NCCL in-place all-gather)
-            dist.all_gather_into_tensor(buf, mine, group=self.group)
+            _all_gather_inplace(buf, self.rank, self.world, self.group)
         return self.engine.finish()
 
 

@@ -3,11 +3,12 @@
 # each spec is lib[:VAR=val[,VAR=val]] (lib -> paper_conf_ipps_wangcc16_b200/libcusfft_<lib>.so)
 mkdir -p gpurun_out
 SPECS="$1"; shift
-timeout 600 python -m pytest tests/test_gpu_parity.py -q -x -p no:cacheprovider -k "C3_bench or paths_agree or shared_taps" > gpurun_out/pytest_ab.log 2>&1; echo pytest rc=$?; tail -2 gpurun_out/pytest_ab.log
+if [ -z "$NO_TESTS" ]; then timeout ${TEST_TIMEOUT:-600} python -m pytest ${TESTS:-tests/test_gpu_parity.py} -m gpu -q -x -p no:cacheprovider ${PYTEST_K:+-k "$PYTEST_K"} > gpurun_out/pytest_ab.log 2>&1; echo pytest rc=$?; tail -3 gpurun_out/pytest_ab.log; fi
 for rep in 1 2; do for spec in $SPECS; do
   l=${spec%%:*}; envs=""; [ "$spec" != "$l" ] && envs=$(echo ${spec#*:} | tr ',' ' ')
   tag=$(echo "$spec" | tr ':,=' '___')
-  env CUSFFT_LIB=libcusfft_$l.so $envs timeout 300 python bench.py --steps 30 --no-cpu-baseline --no-default-line "$@" > gpurun_out/ab_$tag.json 2> gpurun_out/ab_$tag.err
+  lib=libcusfft_$l.so; [ "$l" = default ] && lib=libcusfft.so
+  env CUSFFT_LIB=$lib $envs timeout 300 python bench.py --steps 30 --no-cpu-baseline --no-default-line "$@" > gpurun_out/ab_$tag.json 2> gpurun_out/ab_$tag.err
   python - "$tag" <<'PY'
 import json, sys
 d = json.load(open(f"gpurun_out/ab_{sys.argv[1]}.json"))

@@ -18,7 +18,7 @@ HEADER = os.path.join(ROOT, "include", "cusfft.h")
 def _header_functions():
     src = open(HEADER).read()
     src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
-    return sorted(set(re.findall(r"\b(cusfft_[A-Za-z_]+)\s*\(", src)))
+    return sorted(set(re.findall(r"\b(cusfft_[A-Za-z0-9_]+)\s*\(", src)))
 
 
 def test_header_and_binding_agree():
@@ -115,7 +115,8 @@ def test_plan_validation_before_device(kw, code):
 
 @pytest.mark.parametrize("world,L,shard,code", [
     (3, 16, 0, b.INVALID_LOOPS),   # loop sharding: world must divide L
-    (2, 16, 2, b.INVALID_PARAM),   # unknown shard mode
+    (2, 16, 3, b.INVALID_PARAM),   # unknown shard mode
+    (3, 16, 2, b.INVALID_LOOPS),   # two-exchange loop sharding: world must divide L
     (3, 16, 1, b.INVALID_PARAM),   # signal sharding: world must divide n
 ])
 def test_dist_plan_validation(world, L, shard, code):
@@ -124,6 +125,18 @@ def test_dist_plan_validation(world, L, shard, code):
     p.shard_mode = shard
     h = ctypes.c_void_p()
     assert lib.cusfft_plan_dist(ctypes.byref(h), 2 ** 14, 8, 64, L, ctypes.byref(p), 0, world, None) == code
+    assert not h.value
+
+
+def test_two_exchange_mode_limits():
+    """shard_mode 2 sorts the hit list in shared memory (max_hits <= 32768)
+    and takes medians of at most 64 loops per thread (include/cusfft.h)."""
+    lib = pkg.load_library()
+    p = pkg.default_params(2 ** 14, 8, 64)
+    p.shard_mode = 2
+    p.max_hits = 40000
+    h = ctypes.c_void_p()
+    assert lib.cusfft_plan_dist(ctypes.byref(h), 2 ** 14, 8, 64, 16, ctypes.byref(p), 0, 2, None) == b.INVALID_PARAM
     assert not h.value
 
 

@@ -18,6 +18,7 @@ import torch.distributed as dist
 import torch.multiprocessing as mp
 
 import oracle as O
+from paper_conf_ipps_wangcc16_b200._binding import DEBUG_HITS as DEBUG_HITS_ID, DEBUG_WINNERS as DEBUG_WINNERS_ID
 from paper_conf_ipps_wangcc16_b200.dist import LoopShardedSfft, loops_of_rank, signal_range, slot_of_loop
 from paper_conf_ipps_wangcc16_b200.workload import planted_signal
 
@@ -108,6 +109,108 @@ class OracleSignalEngine:
         G = O.filter_response(self.g, p.n, p.n // p.B)
         vals, _ = O.estimate(hits, uhat, self.sigma, self.tau, G, p.n, p.B)
         return O.select_output(hits, vals, p.k)
+
+
+class OracleTwoExchangeEngine:
+    """Test engine for exchange kind 2 (shard_mode 2): local() writes this
+    rank's location loops' winner lists J into its slice of buffer 1
+    (int64 [world][cmax][num]); mid() votes over every gathered list (the
+    hit set is identical on every rank; sorted), estimates this rank's loops
+    for every hit into its slice of buffer 2 (complex128 as fp64 pairs,
+    [world][HCAP][Lg]); finish() takes the medians over all loops and selects
+    the output.  The arithmetic is the oracle's."""
+
+    exchange_kind = 2
+    HCAP = 256
+
+    def __init__(self, x, p: O.SfftParams, rank: int, world: int):
+        self.x, self.p, self.rank, self.world = x, p, rank, world
+        self.a, self.sigma, self.tau = O.draw_permutations(p.seed, p.n, p.L, p.tau_mode)
+        self.g = O.filter_taps(p)
+        self.Lg = p.L // world
+        self.cmax = -(-p.loc_loops // world)
+        self.buf = torch.zeros(world * self.cmax * p.num_select, dtype=torch.int64)
+        self.buf2 = torch.zeros(world * self.HCAP * self.Lg * 2, dtype=torch.float64)
+        self.uhat = {}
+
+    def local(self, x):
+        p = self.p
+        for i, r in enumerate(loops_of_rank(self.rank, p.L, self.world)):
+            self.uhat[r] = O.bucket_fft(O.perm_filter(x, self.g, int(self.sigma[r]), int(self.tau[r]), p.B))
+            if r < p.loc_loops:  # location loops are a prefix of the rank's loops
+                c = (self.rank * self.cmax + i) * p.num_select
+                self.buf[c:c + p.num_select] = torch.from_numpy(O.cutoff(self.uhat[r], p.num_select))
+
+    def exchange_tensor(self):
+        return self.buf
+
+    def mid(self):
+        p = self.p
+        J = []
+        for r in range(p.loc_loops):
+            c = ((r % self.world) * self.cmax + r // self.world) * p.num_select
+            J.append(self.buf[c:c + p.num_select].numpy().copy())
+        self.hits = np.sort(O.location_recovery(J, self.a[:p.loc_loops], p.n, p.B, p.vote_threshold))
+        assert len(self.hits) <= self.HCAP
+        mine = loops_of_rank(self.rank, p.L, self.world)
+        G = O.filter_response(self.g, p.n, p.n // p.B)
+        _, per = O.estimate(self.hits, np.stack([self.uhat[r] for r in mine]), self.sigma[mine], self.tau[mine],
+                            G, p.n, p.B)
+        v = self.buf2.numpy().reshape(self.world, self.HCAP, self.Lg, 2)
+        v[self.rank, :len(self.hits), :, 0] = per.real
+        v[self.rank, :len(self.hits), :, 1] = per.imag
+
+    def exchange_tensor2(self):
+        return self.buf2
+
+    def finish(self):
+        p, H = self.p, len(self.hits)
+        v = self.buf2.numpy().reshape(self.world, self.HCAP, self.Lg, 2)[:, :H]
+        per = (v[..., 0] + 1j * v[..., 1]).transpose(1, 0, 2).reshape(H, p.L)  # loops in rank-major order
+        med = (p.L - 1) // 2
+        vals = np.sort(per.real, axis=1)[:, med] + 1j * np.sort(per.imag, axis=1)[:, med]
+        return O.select_output(self.hits, vals, p.k)
+
+
+def _two_worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        n, k = 2 ** 12, 6
+        x, S, X = planted_signal(n, k, seed=4)
+        p = O.make_params(n, k, L=8, loc_loops=5, vote_threshold=3, seed=9)
+        locs, vals = LoopShardedSfft(OracleTwoExchangeEngine(x, p, rank, world)).execute(x)
+        q.put((rank, locs.tolist(), vals.tolist()))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [1, 2, 4])
+def test_loop_sharded_two_exchanges_gloo(world):
+    """Exchange kind 2 (candidate records, then per-loop estimates): every
+    rank's output equals the single-process oracle exactly."""
+    n, k = 2 ** 12, 6
+    x, S, X = planted_signal(n, k, seed=4)
+    ref = O.sfft(x, O.make_params(n, k, L=8, loc_loops=5, vote_threshold=3, seed=9))
+    if world == 1:
+        p = O.make_params(n, k, L=8, loc_loops=5, vote_threshold=3, seed=9)
+        locs, vals = LoopShardedSfft(OracleTwoExchangeEngine(x, p, 0, 1)).execute(x)
+        assert np.array_equal(locs, ref.locs)
+        np.testing.assert_array_equal(vals, ref.vals)
+        return
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_two_worker, args=(r, world, port, q)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    out = [q.get(timeout=300) for _ in range(world)]
+    for pr in procs:
+        pr.join(timeout=60)
+        assert pr.exitcode == 0
+    for rank, locs, vals in out:
+        assert locs == ref.locs.tolist(), rank
+        np.testing.assert_array_equal(np.array(vals), ref.vals)
 
 
 def test_signal_range_partitions_x():
@@ -252,6 +355,54 @@ def test_dist_plans_emulated_allgather_match_single_gpu(world):
         assert e.plan.status() == 0
         assert torch.equal(locs, ref_l)
         assert torch.equal(vals, ref_v)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("world,n,k,L,Lloc", [(1, 2 ** 20, 100, 16, 8), (2, 2 ** 20, 100, 16, 8),
+                                              (4, 2 ** 22, 1000, 16, 8), (8, 2 ** 18, 50, 16, 5)])
+def test_two_exchange_plans_emulated_match_single_gpu(world, n, k, L, Lloc):
+    """shard_mode 2 ranks on one GPU (candidate all-gather and estimate
+    all-gather emulated by device copies) reproduce the single-GPU plan bit
+    for bit, at world 1 through the whole-transform call as well."""
+    from paper_conf_ipps_wangcc16_b200 import Plan
+    from paper_conf_ipps_wangcc16_b200.dist import CudaEngine
+    x, S, X = planted_signal(n, k, seed=8)
+    xd = torch.from_numpy(x).cuda()
+    kw = dict(seed=5, loc_loops=Lloc, vote_threshold=Lloc // 2 + 1, max_hits=8192)
+    ref = Plan(n, k, L=L, debug=1, **kw)
+    ref_l, ref_v = ref.execute(xd)
+    if world == 1:
+        one = Plan(n, k, L=L, shard_mode=2, debug=1, **kw)
+        assert one.exchange_kind() == 2
+        l1, v1 = one.execute(xd)
+        torch.cuda.synchronize()
+        assert one.status() == 0
+        assert torch.equal(l1, ref_l) and torch.equal(v1, ref_v)
+        h_ref = ref.debug(DEBUG_HITS_ID)
+        assert np.array_equal(np.sort(h_ref), one.debug(DEBUG_HITS_ID))  # sorted hit list
+        assert np.array_equal(ref.debug(DEBUG_WINNERS_ID), one.debug(DEBUG_WINNERS_ID))
+    engines = [CudaEngine(n, k, L=L, rank=r, world=world, shard_mode=2, **kw) for r in range(world)]
+    assert all(e.exchange_kind == 2 for e in engines)
+    for rep in range(2):  # the second execution replays the captured graphs
+        for e in engines:
+            e.local(xd)
+        torch.cuda.synchronize()
+        for name, per in (("exchange_tensor", engines[0].per_rank), ("exchange_tensor2", engines[0].per_rank2)):
+            if name == "exchange_tensor2":
+                for e in engines:
+                    e.mid()
+                torch.cuda.synchronize()
+            for dst in engines:
+                for r, src in enumerate(engines):
+                    if src is not dst:
+                        getattr(dst, name)()[r * per:(r + 1) * per].copy_(getattr(src, name)()[r * per:(r + 1) * per])
+            torch.cuda.synchronize()
+        for e in engines:
+            locs, vals = e.finish()
+            torch.cuda.synchronize()
+            assert e.plan.status() == 0
+            assert torch.equal(locs, ref_l)
+            assert torch.equal(vals, ref_v)
 
 
 @pytest.mark.gpu

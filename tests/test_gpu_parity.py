@@ -118,6 +118,8 @@ CASES = [
     (2 ** 16, 32, None, 16, dict(loc_loops=12, vote_threshold=7)),  # tail: 16-bit vote table (L_loc > 8)
     (2 ** 16, 32, None, 24, dict(loc_loops=20, vote_threshold=11)),  # tail: 32-bit table, warp-per-hit estimate (L > 16)
     (2 ** 21, 60, 32768, 8, dict(loc_loops=6, vote_threshold=4)),   # B > 16384, q0 enumeration (T <= L_loc/2)
+    (2 ** 18, 100, 4096, 16, dict(gather=2)),         # the paper's remap + execute
+    (2 ** 16, 20, None, 5, dict(loc_loops=5, vote_threshold=3, gather=2)),  # remap, odd L, one-pass FFT
 ]
 
 
@@ -314,11 +316,13 @@ def test_parity_snr_sweep(snr_db):
 @pytest.mark.parametrize("env,kw", [({"CUSFFT_NO_GRAPH": "1"}, {}), ({"CUSFFT_TAIL": "0"}, {}),
                                     ({"CUSFFT_FFT2SEL": "0"}, {}),
                                     ({}, dict(gather=1)), ({}, dict(l2_persist=0)),
-                                    ({"CUSFFT_TAIL": "0", "CUSFFT_NO_GRAPH": "1"}, dict(gather=1))])
+                                    ({"CUSFFT_TAIL": "0", "CUSFFT_NO_GRAPH": "1"}, dict(gather=1)),
+                                    ({}, dict(gather=2)), ({"CUSFFT_NO_GRAPH": "1"}, dict(gather=2))])
 def test_kernel_paths_agree(env, kw, monkeypatch):
     """Every alternative path (no CUDA graph, the k_vote / k_estimate /
-    k_output chain instead of the fused tail, the direct gather instead of
-    the staged one, no persisting-L2 set-aside) gives the default path's hits
+    k_output chain instead of the fused tail, the direct gather or the
+    paper's remap + execute kernels instead of the staged gather, no
+    persisting-L2 set-aside) gives the default path's hits
     and output exactly (same fold order, same selection rules)."""
     import torch
     from paper_conf_ipps_wangcc16_b200 import Plan
@@ -337,7 +341,7 @@ def test_kernel_paths_agree(env, kw, monkeypatch):
     torch.cuda.synchronize()
     assert alt.status() == 0
     assert alt.info()["tail"] == (0 if env.get("CUSFFT_TAIL") == "0" else 1)
-    assert alt.info()["staged"] == (0 if kw.get("gather") == 1 else 1)
+    assert alt.info()["staged"] == (0 if kw.get("gather") in (1, 2) else 1)
     assert np.array_equal(np.sort(alt.debug(DEBUG_HITS)), h0)
     assert torch.equal(l1, l0)
     assert torch.equal(v1, v0)
