@@ -167,9 +167,10 @@ int cusfft_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L,
  * sorts the hits ascending and estimates ITS loops for every hit (Alg. 5
  * L308-L325); exchange #2 all-gathers those per-loop estimates; every rank
  * takes the medians (L95, Alg. 5) and selects the output.  Bit-
- * identical to world = 1.  Needs max_hits <= 32768 (the hit list is sorted in
- * shared memory) and L <= 64; exchange #2 moves world x max_hits x L/world x 16
- * bytes, so set max_hits near the expected hit count.
+ * identical to world = 1.  Needs max_hits <= 32768 (the hits are put in
+ * ascending order by counting, quadratic in their number) and L <= 64;
+ * exchange #2 moves world x max_hits x L/world x 16 bytes, so set max_hits
+ * near the expected hit count.
  *
  * nccl_unique_id: NULL, or 128 bytes from cusfft_nccl_unique_id on one rank,
  * distributed to every rank by the caller (any channel).  With an id the plan

@@ -218,11 +218,12 @@ struct cusfft_plan_s {
   int64_t crec_bytes = 0;         // one candidate record: bitmap | count | J (the record's tail)
   uint8_t* d_cand = nullptr;      // [world][cmax][crec_bytes]
   double2* d_x2 = nullptr;        // [world][max_hits][Lg] per-loop estimates
-  int sort_smem = 0;              // k_hits_sort: npow2(max_hits) x 4 B
+  int* d_hits2 = nullptr;          // [max_hits] the hit list in ascending order (k_rank_est)
   int tail_esz = 0;               // bytes per vote-table element (1 / 2 / 4), 0: the k_vote / k_estimate / k_output chain
   int tail_smem = 0, tail_qoff = 0, tail_grid = 1;
   bool pk_direct = false;         // the cluster cutoff ORs its winners into k_tail's table (d_pk, zero block)
   uint32_t* d_pk = nullptr;
+  uint32_t* d_pkb = nullptr;      // otherwise (fused tail): the table built once by k_pk_build before k_tail
   int vote_smem = 0, vote_grid = 1, est_grid = 1, output_smem = 0;
   int* d_hits = nullptr;
   double2* d_hit_vals = nullptr;
@@ -325,7 +326,7 @@ void free_plan(cusfft_plan_t p) {
   }
   void* ptrs[] = {p->d_code, p->d_row0, p->d_staging, p->d_tw, p->d_ph_hi, p->d_ph_lo, p->d_slots, p->d_loc_sigma, p->d_u, p->d_v,
                   p->d_records, p->d_keys, p->d_zero, p->d_key_index, p->d_hits, p->d_hit_vals, p->d_hit_keys,
-                  p->d_per_loop, p->d_xbuf, p->d_locs_buf, p->d_vals_buf, p->d_cand, p->d_x2};
+                  p->d_per_loop, p->d_xbuf, p->d_locs_buf, p->d_vals_buf, p->d_cand, p->d_x2, p->d_hits2, p->d_pkb};
   for (void* q : ptrs)
     if (q) cudaFree(q);
   if (p->ev_made)
@@ -359,7 +360,7 @@ int validate(int64_t n, int64_t k, int64_t B, int32_t L, const cusfft_params& q,
   if (q.loc_loops > kMaxLoc) return CUSFFT_INVALID_LOOPS;
   if (world < 1 || rank < 0 || rank >= world) return CUSFFT_INVALID_LOOPS;
   if (q.shard_mode < 0 || q.shard_mode > 2) return CUSFFT_INVALID_PARAM;
-  // shard_mode 2: the hit list is sorted in one CTA's shared memory, the median holds L values per thread
+  // shard_mode 2: the hits are ranked by counting (quadratic in them), the median holds 2 values per lane
   if (q.shard_mode == 2 && (q.max_hits > 32768 || L > kMedMaxL)) return CUSFFT_INVALID_PARAM;
   if (q.shard_mode == 1 && world > 1) {
     if (n % world) return CUSFFT_INVALID_PARAM;
@@ -566,6 +567,13 @@ TailKernel tail_kernel(int esz, int L, int Lloc) {
   if (esz == 2) return seg ? k_tail<uint16_t, 16, 0> : k_tail<uint16_t, 32, 0>;
   return seg ? k_tail<uint32_t, 16, 0> : k_tail<uint32_t, 32, 0>;
 }
+// The vote-only instantiation (shard_mode 2: each rank estimates its own loops afterwards).
+TailKernel tail_vote_kernel(int esz, int Lloc) {
+  if (esz == 1 && Lloc == 8) return k_tail<uint8_t, 16, 8, false>;
+  if (esz == 1) return k_tail<uint8_t, 16, 0, false>;
+  if (esz == 2) return k_tail<uint16_t, 16, 0, false>;
+  return k_tail<uint32_t, 16, 0, false>;
+}
 
 int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, const cusfft_params* pin, int rank,
               int world, const void* nccl_id) {
@@ -712,8 +720,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     const int64_t tab = ((int64_t)B * esz + 15) & ~int64_t(15);
     const int64_t need = tab + (kTailNT / 32) * kTailQ * 2;
     const char* et = std::getenv("CUSFFT_TAIL");  // CUSFFT_TAIL=0: the k_vote / k_estimate chain (tests, A/B)
-    // (shard_mode 2 votes with k_vote and estimates per rank: no fused tail)
-    if (need + 8 * 1024 <= smem_optin && !(et && et[0] == '0') && q.shard_mode != 2) {  // + k_tail's static smem (hit queue)
+    // (shard_mode 2 runs it vote-only: each rank estimates its own loops afterwards)
+    if (need + 8 * 1024 <= smem_optin && !(et && et[0] == '0')) {  // + k_tail's static smem (hit queue)
       P->tail_esz = esz;
       P->tail_qoff = (int)tab;
       P->tail_smem = (int)need;
@@ -748,6 +756,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     P->d_hist = reinterpret_cast<uint32_t*>(P->d_zero + 8);
     P->d_ohist = P->d_hist + (size_t)nsel * 4096;
     if (P->pk_direct) P->d_pk = reinterpret_cast<uint32_t*>(P->d_zero + pk_off);
+    if (P->tail_esz && !P->pk_direct && (rc = dalloc(&P->d_pkb, (size_t)((B * P->tail_esz + 15) / 16) * 4)))
+      return fail(rc);
     if ((rc = dalloc(&P->d_key_index, (size_t)P->Lg))) return fail(rc);
     std::vector<int> kidx(P->Lg, -1);
     for (int i = 0; i < nsel; ++i) kidx[P->sel_slots_h[i] - lrank * P->Lg] = i;
@@ -780,6 +790,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   attr(set_dyn_smem(k_vote, smem_optin, smem_optin));
   attr(set_dyn_smem(k_output, smem_optin, smem_optin));
   if (P->tail_esz) attr(set_dyn_smem(tail_kernel(P->tail_esz, L, P->Lloc), P->tail_smem, smem_optin));
+  if (P->tail_esz && q.shard_mode == 2) attr(set_dyn_smem(tail_vote_kernel(P->tail_esz, P->Lloc), P->tail_smem, smem_optin));
   if (ae != cudaSuccess) {
     g_last_cuda_error = (int)ae;
     return fail(CUSFFT_CUDA);
@@ -914,16 +925,13 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     P->mode2 = true;
     P->cmax = (P->Lloc + world - 1) / world;
     P->crec_bytes = P->lay.rec_bytes - P->lay.off_bitmap;
-    int np2 = 2;
-    while (np2 < P->max_hits) np2 <<= 1;
-    P->sort_smem = np2 * 4;
-    if (P->sort_smem > smem_optin) return fail(CUSFFT_INVALID_PARAM);
-    if (cudaFuncSetAttribute(k_hits_sort, cudaFuncAttributeMaxDynamicSharedMemorySize, P->sort_smem) != cudaSuccess) {
+    if (set_dyn_smem(k_rank_est, P->max_hits * 4, smem_optin) != cudaSuccess) {  // k_rank_est stages the hit list
       g_last_cuda_error = (int)cudaGetLastError();
       return fail(CUSFFT_CUDA);
     }
     if ((rc = dalloc(&P->d_cand, (size_t)(world * P->cmax * P->crec_bytes)))) return fail(rc);
     if ((rc = dalloc(&P->d_x2, (size_t)world * P->max_hits * P->Lg))) return fail(rc);
+    if ((rc = dalloc(&P->d_hits2, (size_t)P->max_hits))) return fail(rc);
   }
   if (nccl_id) {  // the library-owned exchange (a world of 1 is allowed: a one-rank communicator)
     ncclUniqueId id;
@@ -1264,7 +1272,7 @@ VoteArgs make_vote_args(cusfft_plan_t P) {
   va.hits = P->d_hits;
   va.hit_count = reinterpret_cast<unsigned*>(P->d_flags);
   va.max_hits = P->max_hits;
-  va.pk = P->d_pk;
+  va.pk = P->d_pk ? P->d_pk : P->d_pkb;
   return va;
 }
 
@@ -1295,8 +1303,26 @@ EstArgs make_est_args(cusfft_plan_t P) {
   return ea;
 }
 
+// The vote table from the cutoff bitmaps (fused-tail plans whose cutoff does not OR into it).
+int launch_pk_build(cusfft_plan_t P, cudaStream_t st) {
+  if (!P->d_pkb) return CUSFFT_SUCCESS;
+  const VoteArgs va = make_vote_args(P);
+  const dim3 grid((unsigned)((P->B + 255) / 256));
+  cudaError_t e;
+  if (P->tail_esz == 1)
+    e = launch_k(k_pk_build<uint8_t>, grid, dim3(256), 0, st, P->cur_prio, va, reinterpret_cast<uint8_t*>(P->d_pkb));
+  else if (P->tail_esz == 2)
+    e = launch_k(k_pk_build<uint16_t>, grid, dim3(256), 0, st, P->cur_prio, va, reinterpret_cast<uint16_t*>(P->d_pkb));
+  else
+    e = launch_k(k_pk_build<uint32_t>, grid, dim3(256), 0, st, P->cur_prio, va, P->d_pkb);
+  CK(e);
+  g_pdl = P->timing != 1;
+  return CUSFFT_SUCCESS;
+}
+
 // Steps 5 + 6 in one kernel (tail.cuh).
 int launch_tail(cusfft_plan_t P, cudaStream_t st) {
+  TRY(launch_pk_build(P, st));
   TailArgs ta{};
   ta.v = make_vote_args(P);
   ta.e = make_est_args(P);
@@ -1339,18 +1365,27 @@ int launch_after_cutoff(cusfft_plan_t P, int64_t* locs, double2* vals, cudaStrea
 }
 
 // shard_mode 2, after the candidate all-gather: every rank votes over all
-// location loops (k_vote), sorts the hit list (k_hits_sort) and estimates its
-// own loops for every hit into its slice of the estimate buffer (k_est_local).
+// location loops (k_vote), ranks the hits into ascending order and estimates its
+// own loops for every hit into its slice of the estimate buffer (k_rank_est).
 int launch_mid(cusfft_plan_t P, cudaStream_t st) {
   if (P->stage_limit < 4) return CUSFFT_SUCCESS;
-  CK(launch_k(k_vote, dim3(P->vote_grid), dim3(256), P->vote_smem, st, P->cur_prio, make_vote_args(P)));
+  if (P->tail_esz) {  // the fused tail's vote, without its estimation
+    TRY(launch_pk_build(P, st));
+    TailArgs ta{};
+    ta.v = make_vote_args(P);
+    ta.e = make_est_args(P);
+    ta.q_off = P->tail_qoff;
+    CK(launch_k(tail_vote_kernel(P->tail_esz, P->Lloc), dim3((unsigned)P->tail_grid), dim3(kTailNT),
+                (size_t)P->tail_smem, st, P->cur_prio, ta));
+  } else {
+    CK(launch_k(k_vote, dim3(P->vote_grid), dim3(256), P->vote_smem, st, P->cur_prio, make_vote_args(P)));
+  }
   mark(P, 4);
   if (P->stage_limit < 5) return CUSFFT_SUCCESS;
   g_pdl = P->timing != 1;
-  CK(launch_k(k_hits_sort, dim3(1), dim3(kSortNT), (size_t)P->sort_smem, st, P->cur_prio, P->d_hits,
-              reinterpret_cast<const unsigned*>(P->d_flags), P->max_hits));
-  const int gx = std::max(1, std::min((P->max_hits * P->Lg + 255) / 256, P->sms * 4));
-  CK(launch_k(k_est_local, dim3(gx), dim3(256), 0, st, P->cur_prio, make_est_args(P), P->rank * P->Lg, P->Lg,
+  CK(launch_k(k_rank_est, dim3((unsigned)((P->max_hits + kRankC - 1) / kRankC)), dim3(kRankNT),
+              (size_t)P->max_hits * 4, st,
+              P->cur_prio, make_est_args(P), P->rank * P->Lg, P->Lg, P->d_hits2,
               P->d_x2 + (size_t)P->rank * P->max_hits * P->Lg));
   return CUSFFT_SUCCESS;
 }
@@ -1358,13 +1393,13 @@ int launch_mid(cusfft_plan_t P, cudaStream_t st) {
 // shard_mode 2, after the estimate all-gather: medians (k_median) and the output.
 int launch_finish2(cusfft_plan_t P, int64_t* locs, double2* vals, cudaStream_t st) {
   if (P->stage_limit < 5) return CUSFFT_SUCCESS;
-  const int gx = std::max(1, std::min((P->max_hits + 127) / 128, P->sms * 4));
-  CK(launch_k(k_median, dim3(gx), dim3(128), 0, st, P->cur_prio, make_est_args(P), (const double2*)P->d_x2,
+  const int gx = std::max(1, std::min((P->max_hits + 7) / 8, P->sms * 4));  // a warp per hit
+  CK(launch_k(k_median, dim3(gx), dim3(256), 0, st, P->cur_prio, make_est_args(P), (const double2*)P->d_x2,
               P->world, P->Lg));
   mark(P, 5);
   if (P->stage_limit < 6) return CUSFFT_SUCCESS;
   g_pdl = P->timing != 1;
-  CK(launch_k(k_output, dim3(1), dim3(1024), P->output_smem, st, P->cur_prio, (const int*)P->d_hits,
+  CK(launch_k(k_output, dim3(1), dim3(1024), P->output_smem, st, P->cur_prio, (const int*)P->d_hits2,
               reinterpret_cast<const unsigned*>(P->d_flags), P->max_hits, (const double2*)P->d_hit_vals,
               (const uint64_t*)P->d_hit_keys, P->d_ohist, (int)P->k, P->kp2, ilog2(P->n), locs, vals,
               P->d_flags + 1));
@@ -1939,8 +1974,8 @@ int64_t cusfft_get_debug(cusfft_plan_t plan, int32_t what, void* dst, int64_t ca
         for (int j = cnt; j < plan->Jcap; ++j) o[j] = -1;
       }
       break;
-    case CUSFFT_DEBUG_HITS:
-      CK(cudaMemcpy(out, plan->d_hits, need, cudaMemcpyDeviceToHost));
+    case CUSFFT_DEBUG_HITS:  // (shard_mode 2: the ascending list the medians are aligned with)
+      CK(cudaMemcpy(out, plan->mode2 ? plan->d_hits2 : plan->d_hits, need, cudaMemcpyDeviceToHost));
       break;
     case CUSFFT_DEBUG_HIT_VALS:
       CK(cudaMemcpy(out, plan->d_hit_vals, need, cudaMemcpyDeviceToHost));
@@ -2061,7 +2096,9 @@ int32_t cusfft_launches_per_execute(cusfft_plan_t plan) {
   int n = (plan->staged ? 1 : 0) + ranges /*fold per slot range*/ +
           ffts * (pass1 ? 2 : 1) /*fft*/ + (plan->sel_slots_h.empty() ? 0 : 1) +
           (plan->xshard && !plan->sel_slots_h.empty() ? 1 : 0) /*keys*/ + (plan->tail_esz ? 2 : 3);
-  if (plan->mode2) n += 1;  // k_vote + k_hits_sort + k_est_local + k_median + k_output (not k_vote + k_tail / k_estimate + k_output)
+  // shard_mode 2: vote (k_tail vote-only or k_vote) + k_rank_est + k_median + k_output
+  if (plan->mode2) n = n - (plan->tail_esz ? 2 : 3) + 4;
+  if (plan->d_pkb) n += 1;  // k_pk_build
   if (plan->remap) {  // a remap + an execution kernel per chunk of B taps instead of one fold per range
     n -= ranges;
     for (int s = 0; s < plan->Lg; ++s) n += 2 * plan->filt[plan->filt_of_local(s)].R;

@@ -7,10 +7,10 @@
 //           this rank's slice of the candidate buffer
 //   #1      all-gather of the candidate buffer (L_loc records)
 //   mid     every rank votes over all location loops (identical hit SET,
-//           PAPER.md:L91-L93, Alg. 4), sorts the hits ascending
-//           (the appends are unordered; the sort makes the hit list, and so
-//           the per-loop estimate slices, identical on every rank), and
-//           estimates ITS loops for every hit (Alg. 5)
+//           PAPER.md:L91-L93, Alg. 4; k_vote), ranks the hits
+//           (the appends are unordered; ascending order makes the hit list,
+//           and so the per-loop estimate slices, identical on every rank) and
+//           estimates ITS loops for every hit (Alg. 5; k_rank_est)
 //   #2      all-gather of the per-loop estimates [rank][hit][local loop]
 //   finish  median over all L loops per hit, re and im separately (L95,
 //           Alg. 5), then the output selection (k_output)
@@ -22,85 +22,75 @@
 
 namespace cusfft {
 
-// Ascending sort of the hit list in place (one CTA of 1024 threads, bitonic
-// over the next power of two >= H in shared memory; smem: npow2(max_hits) x 4
-// bytes).  Hits are distinct frequencies, so the order is unique.
-constexpr int kSortNT = 1024;
-__global__ void __launch_bounds__(kSortNT) k_hits_sort(int* __restrict__ hits, const unsigned* __restrict__ hit_count,
-                                                       int max_hits) {
+// The hit list in ascending order plus this rank's per-loop estimates, in one
+// kernel: a CTA takes a chunk of kRankC hits of the (unordered) list from the
+// vote; its warps count, over the whole list staged in shared memory
+// (max_hits x 4 bytes), the hits smaller than each of them (hits are distinct frequencies, so the ranks are a
+// permutation and the order is unique), the chunk's hits go to
+// hits_sorted[rank], and the CTA estimates them for this rank's slots s =
+// slot0 .. slot0 + Lg - 1 (the records this rank computed) into x2[rank][i].
+constexpr int kRankNT = 256, kRankC = 32;
+__global__ void __launch_bounds__(kRankNT) k_rank_est(EstArgs E, int slot0, int Lg, int* __restrict__ hits_sorted,
+                                                      double2* __restrict__ x2) {
   pdl_wait();
-  extern __shared__ __align__(16) int shv[];
-  const int H = min((int)*hit_count, max_hits);
-  int N = 2;
-  while (N < H) N <<= 1;
-  for (int i = threadIdx.x; i < N; i += kSortNT) shv[i] = i < H ? __ldcg(hits + i) : 0x7fffffff;
-  __syncthreads();
-  for (int size = 2; size <= N; size <<= 1) {
-    for (int stride = size >> 1; stride > 0; stride >>= 1) {
-      for (int t = threadIdx.x; t < (N >> 1); t += kSortNT) {
-        const int i = 2 * t - (t & (stride - 1));
-        const int j = i + stride;
-        const bool up = (i & size) == 0;
-        const int a = shv[i], b = shv[j];
-        if ((a > b) == up) {
-          shv[i] = b;
-          shv[j] = a;
-        }
-      }
-      __syncthreads();
-    }
-  }
-  for (int i = threadIdx.x; i < H; i += kSortNT) hits[i] = shv[i];
-}
-
-// This rank's per-loop estimates v_s(f) for every hit f (slots slot0 ..
-// slot0 + Lg - 1 of the records, which this rank computed): x2[h][i] for
-// local slot i.  Thread per (hit, local slot).
-__global__ void __launch_bounds__(256) k_est_local(EstArgs E, int slot0, int Lg, double2* __restrict__ x2) {
-  pdl_wait();
+  extern __shared__ __align__(16) int shl[];  // the whole hit list (max_hits entries)
+  __shared__ int srank[kRankC];
+  __shared__ uint32_t sf[kRankC];
   const int H = min((int)*E.hit_count, E.max_hits);
-  const int total = H * Lg;
-  for (int idx = blockIdx.x * blockDim.x + threadIdx.x; idx < total; idx += gridDim.x * blockDim.x) {
-    const int h = idx / Lg, i = idx - h * Lg;
+  const int h0 = blockIdx.x * kRankC;
+  if (h0 >= H) return;
+  const int tid = threadIdx.x, lane = tid & 31, wid = tid >> 5;
+  for (int i = tid; i < H; i += kRankNT) shl[i] = __ldcg(E.hits + i);  // independent loads: one L2 round trip
+  if (tid < kRankC) srank[tid] = 0;
+  __syncthreads();
+  // warp w counts, for every hit of the chunk (lane = chunk position), the
+  // smaller hits among list entries j = w, w + 8, ... (broadcast reads)
+  const int f = h0 + lane < H ? shl[h0 + lane] : 0;
+  int r = 0;
+#pragma unroll 8
+  for (int j = wid; j < H; j += kRankNT / 32) r += shl[j] < f;
+  atomicAdd(&srank[lane], r);
+  if (tid < kRankC) sf[tid] = (uint32_t)(h0 + tid < H ? shl[h0 + tid] : 0);
+  __syncthreads();
+  const int nh = min(kRankC, H - h0);
+  if (tid < nh) hits_sorted[srank[tid]] = (int)sf[tid];
+  for (int w = tid; w < nh * Lg; w += kRankNT) {
+    const int t = w / Lg, i = w - t * Lg;
     const SlotParam sp = E.slots[slot0 + i];
-    x2[idx] = loop_estimate(E, sp, slot0 + i, (uint32_t)__ldcg(E.hits + h));
+    x2[(int64_t)srank[t] * Lg + i] = loop_estimate(E, sp, slot0 + i, sf[t]);
   }
 }
 
 // Median of the L = G x Lg per-loop estimates of hit h (x2: [G][max_hits][Lg]
-// after the all-gather; rank g's local slot i is slot g Lg + i), element of
-// rank floor((L-1)/2) of the real and of the imaginary parts, ties by slot
-// (as the fused tail).  Writes the hit value, its key |val|^2 and the output
+// after the all-gather; rank g's local slot i is slot g Lg + i): one warp per
+// hit, lane l holding slots l and l + 32, the element of rank floor((L-1)/2)
+// of the real and of the imaginary parts, ties by slot (warp_rank_select, as
+// the fused tail).  Writes the hit value, its key |val|^2 and the output
 // histogram; debug plans also the per-loop values in slot order.
-constexpr int kMedMaxL = 64;
-__global__ void __launch_bounds__(128) k_median(EstArgs E, const double2* __restrict__ x2, int G, int Lg) {
+constexpr int kMedMaxL = 64;  // two values per lane
+__global__ void __launch_bounds__(256) k_median(EstArgs E, const double2* __restrict__ x2, int G, int Lg) {
   pdl_wait();
   const int H = min((int)*E.hit_count, E.max_hits);
   const int L = G * Lg;
   const int med = (L - 1) >> 1;
-  for (int h = blockIdx.x * blockDim.x + threadIdx.x; h < H; h += gridDim.x * blockDim.x) {
-    double re[kMedMaxL], im[kMedMaxL];
-    for (int g = 0; g < G; ++g)
-      for (int i = 0; i < Lg; ++i) {
-        const double2 v = __ldcg(x2 + ((int64_t)g * E.max_hits + h) * Lg + i);
-        re[g * Lg + i] = v.x;
-        im[g * Lg + i] = v.y;
-        if (E.per_loop) E.per_loop[(int64_t)h * L + g * Lg + i] = v;
-      }
-    double vr = 0.0, vi = 0.0;
-    for (int s = 0; s < L; ++s) {
-      int rr = 0, ri = 0;
-      for (int j = 0; j < L; ++j) {
-        rr += (re[j] < re[s]) || (re[j] == re[s] && j < s);
-        ri += (im[j] < im[s]) || (im[j] == im[s] && j < s);
-      }
-      if (rr == med) vr = re[s];
-      if (ri == med) vi = im[s];
+  const int lane = threadIdx.x & 31;
+  const int nw = (gridDim.x * blockDim.x) >> 5;
+  for (int h = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; h < H; h += nw) {  // warp-uniform
+    double2 v0 = make_double2(0.0, 0.0), v1 = make_double2(0.0, 0.0);
+    if (lane < L) v0 = __ldcg(x2 + ((int64_t)(lane / Lg) * E.max_hits + h) * Lg + lane % Lg);
+    if (lane + 32 < L) v1 = __ldcg(x2 + ((int64_t)((lane + 32) / Lg) * E.max_hits + h) * Lg + (lane + 32) % Lg);
+    if (E.per_loop) {
+      if (lane < L) E.per_loop[(int64_t)h * L + lane] = v0;
+      if (lane + 32 < L) E.per_loop[(int64_t)h * L + lane + 32] = v1;
     }
-    const uint64_t key = (uint64_t)__double_as_longlong(__dadd_rn(__dmul_rn(vr, vr), __dmul_rn(vi, vi)));
-    E.hit_vals[h] = make_double2(vr, vi);
-    E.hit_keys[h] = key;
-    atomicAdd(E.out_hist + ((uint32_t)(key >> 51) & 0xFFFu), 1u);
+    const double vr = warp_rank_select(v0.x, v1.x, L, med);
+    const double vi = warp_rank_select(v0.y, v1.y, L, med);
+    if (lane == 0) {
+      const uint64_t key = (uint64_t)__double_as_longlong(__dadd_rn(__dmul_rn(vr, vr), __dmul_rn(vi, vi)));
+      E.hit_vals[h] = make_double2(vr, vi);
+      E.hit_keys[h] = key;
+      atomicAdd(E.out_hist + ((uint32_t)(key >> 51) & 0xFFFu), 1u);
+    }
   }
 }
 

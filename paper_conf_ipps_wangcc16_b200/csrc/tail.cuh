@@ -338,7 +338,7 @@ __device__ __forceinline__ void tail_store(const EstArgs& E, unsigned hs, bool v
 // positions and estimated by this warp at once.
 constexpr int kTailHQ = 1024;  // CTA hit-queue capacity
 
-template <int LP>
+template <int LP, bool EST>
 __device__ __forceinline__ void tail_emit(const TailArgs& A, bool hit, uint32_t f, uint32_t* hq, int* nq,
                                           const SlotParam& sp0, const SlotParam& sp1) {
   const int lane = threadIdx.x & 31;
@@ -359,6 +359,7 @@ __device__ __forceinline__ void tail_emit(const TailArgs& A, bool hit, uint32_t 
   base = __shfl_sync(kFull, base, leader);
   const unsigned myslot = base + rank;
   if (hit && (int)myslot < A.v.max_hits) A.v.hits[myslot] = (int)f;
+  if (!EST) return;
   constexpr int G = 32 / LP;
   unsigned rem = hb;
   while (rem) {  // warp-uniform
@@ -395,9 +396,25 @@ __device__ __forceinline__ uint32_t tab_at(uint32_t base, uint32_t i) {
   return v;
 }
 
+// The vote table in global memory, built once from the location loops'
+// cutoff bitmaps (plans whose cutoff cannot OR its winners into it directly:
+// multi-GPU plans after the exchange); every k_tail CTA then bulk-copies it
+// instead of transposing the bitmaps itself.  Thread per bucket.
+template <typename ET>
+__global__ void __launch_bounds__(256) k_pk_build(VoteArgs V, ET* __restrict__ pk) {
+  pdl_wait();
+  const int b = blockIdx.x * blockDim.x + threadIdx.x;
+  if (b >= V.B) return;
+  uint32_t v = 0u;
+  for (int q = 0; q < V.Lloc; ++q) v |= ((__ldcg(V.bmp[q] + (b >> 5)) >> (b & 31)) & 1u) << q;
+  pk[b] = (ET)v;
+}
+
 // ET: vote table element; LP: estimation lanes per hit (16 or 32).
 // LL: L_loc at compile time (8, the default plans) or 0 (any L_loc <= 8 sizeof(ET)).
-template <typename ET, int LP, int LL>
+// EST = false: the vote only (shard_mode 2, exchange.cuh: each rank estimates
+// its own loops afterwards); the hits are written to the hit list unordered.
+template <typename ET, int LP, int LL, bool EST = true>
 __global__ void __launch_bounds__(kTailNT, 4) k_tail(TailArgs A) {
   pdl_wait();
   KTRACE(9);
@@ -554,7 +571,7 @@ __global__ void __launch_bounds__(kTailNT, 4) k_tail(TailArgs A) {
             hit = __popc(bits) >= V.T && (bits & ((1u << e) - 1u)) == 0u;
           }
         }
-        tail_emit<LP>(A, hit, f, s_hq, &s_nq, sp0, sp1);
+        tail_emit<LP, EST>(A, hit, f, s_hq, &s_nq, sp0, sp1);
       }
       __syncwarp();
     }
@@ -575,6 +592,13 @@ __global__ void __launch_bounds__(kTailNT, 4) k_tail(TailArgs A) {
 #endif
   const int nq = s_nq;
   if (tid == 0 && nq > 0) s_base = atomicAdd(V.hit_count, (unsigned)nq);
+  if (!EST) {
+    __syncthreads();
+    const unsigned base = s_base;
+    for (int i = tid; i < nq; i += kTailNT)
+      if ((int)(base + i) < V.max_hits) V.hits[base + i] = (int)s_hq[i];
+    return;
+  }
   constexpr int G = 32 / LP;
   constexpr int PASS = (kTailNT / 32) * G;  // hits per CTA pass
   const int h1 = wid * G + lane / LP;

@@ -4,7 +4,7 @@ conditions as bench.py's timed loop: L2 flushed (and, with --cold, the
 persisting lines reset) before every execution, the plan's CUDA graph
 launched on the current stream.  Writes a JSON summary (and optionally the
 Chrome trace) so bench.py's event-timed kernel numbers can be checked
-against it.  Usage: kernel_trace.py OUT.json [--config C3] [--reps 20] [--cold] [--chrome OUT.trace.json]
+against it.  Usage: kernel_trace.py OUT.json [--config C3] [--reps 20] [--cold] [--chrome OUT.trace.json] [--plan-kw JSON]
 """
 import argparse
 import json
@@ -26,6 +26,7 @@ ap.add_argument("--config", default="C3")
 ap.add_argument("--reps", type=int, default=20)
 ap.add_argument("--cold", action="store_true")
 ap.add_argument("--chrome", default="")
+ap.add_argument("--plan-kw", default="{}", help="extra plan parameters as JSON, e.g. '{\"shard_mode\": 2}'")
 args = ap.parse_args()
 
 n, k, L = bench.CONFIGS[args.config][:3]
@@ -33,7 +34,7 @@ B = default_B(n, k)
 x_np, S, X = bench.make_signal(n, k, 1)
 dev = torch.device("cuda", 0)
 x = torch.from_numpy(x_np).to(dev)
-plan = Plan(n, k, B=B, L=L, seed=3, device=0, **bench.plan_params(args.config))
+plan = Plan(n, k, B=B, L=L, seed=3, device=0, **{**bench.plan_params(args.config), **json.loads(args.plan_kw)})
 locs = torch.empty(k, dtype=torch.int64, device=dev)
 vals = torch.empty(k, dtype=torch.complex128, device=dev)
 flush = bench.L2Flush(dev)
@@ -68,7 +69,7 @@ for s0, e0, nm in starts:
         cur[1] = max(cur[1], e0)
 if cur:
     spans.append(cur[1] - cur[0])
-out = {"config": args.config, "reps": args.reps, "cold": args.cold,
+out = {"config": args.config, "plan_kw": json.loads(args.plan_kw), "reps": args.reps, "cold": args.cold,
        "how": "torch.profiler (CUPTI kernel activity), L2 flushed before every execution"
               + (" + cudaCtxResetPersistingL2Cache" if args.cold else ""),
        "kernels_us": {k_: {"launches": len(v), "mean": statistics.mean(v), "median": statistics.median(v),

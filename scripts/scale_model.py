@@ -1,11 +1,15 @@
 """Per-rank time model of loop-sharded C3 on G = 1, 2, 4, 8 GPUs, with the
-per-rank compute MEASURED on one B200.
+per-rank compute MEASURED on one B200, for both loop-sharded
+designs: one all-gather of the per-loop records (shard_mode 0) and two
+all-gathers, candidates then per-loop estimates (shard_mode 2).
 
 For each G the script builds rank 0's plan of a G-rank loop-sharded run
 (cusfft_plan_dist without a communicator), and times on the bench's terms
 (L2 flushed before every step, CUDA events, graphs):
   local  = cusfft_execute_local  (Steps 1-4 of this rank's L/G loops, one serial chain)
   finish = (local + cusfft_execute_finish) - local (vote + estimation + output over all L loops)
+  mode 2: mid = (local + cusfft_execute_mid) - local (vote, hit sort, this rank's estimates),
+          finish = (local + mid + finish) - (local + mid) (medians + output)
 The exchange buffer is filled with the records of a world = 1 plan of the same
 draws (the all-gather's result), so finish does the real work.  The
 all-gather itself cannot be timed on one GPU: it is modelled as
@@ -96,6 +100,60 @@ for G in (1, 2, 4, 8):
     out["ranks"][G] = {"local_us": local_us, "finish_us": finish_us, "allgather_bytes": ag_bytes,
                        "allgather_model_us": ag_us, "model_total_us": local_us + ag_us + finish_us,
                        "finish_equals_single_gpu_output": same}
+    p.close()
+# ---- shard_mode 2: the same, with the two exchange buffers filled from a world = 1 mode-2 plan
+from paper_conf_ipps_wangcc16_b200.dist import _CudaBuffer  # noqa: E402
+from paper_conf_ipps_wangcc16_b200 import DEBUG_PER_LOOP, DEBUG_NUM_HITS  # noqa: E402
+import numpy as np  # noqa: E402
+MH = 8192
+ref2 = Plan(n, k, B=B, L=L, seed=3, device=0, shard_mode=2, max_hits=MH, debug=1, **prm)
+l0, v0 = torch.empty_like(locs), torch.empty_like(vals)
+full2_us = timed(lambda: ref2.execute(x, l0, v0))
+ref2.execute(x, l0, v0)
+torch.cuda.synchronize()
+assert torch.equal(l0, locs) and torch.equal(v0, vals)
+c_ptr, c_per = ref2.exchange_buffer()
+Lloc = ref2.info()["loc_loops"]
+crec = c_per // Lloc
+ref_cand = torch.as_tensor(_CudaBuffer(c_ptr, c_per), device=dev).clone()
+H = int(ref2.debug(DEBUG_NUM_HITS)[0])
+per_loop = torch.from_numpy(np.ascontiguousarray(ref2.debug(DEBUG_PER_LOOP).reshape(H, L))).to(dev)
+out["mode2"] = {"single_gpu_us": full2_us, "hits": H, "max_hits": MH, "ranks": {}}
+for G in (1, 2, 4, 8):
+    p = Plan(n, k, B=B, L=L, seed=3, device=0, rank=0, world=G, shard_mode=2, max_hits=MH, **prm)
+    ptr, per = p.exchange_buffer()
+    ptr2, per2 = p.exchange_buffer2()
+    cand = torch.as_tensor(_CudaBuffer(ptr, per * G), device=dev)
+    x2 = torch.as_tensor(_CudaBuffer(ptr2, per2 * G, "<c16", 16), device=dev).view(G, MH, L // G)
+    cmax = per // crec
+    for r in range(Lloc):  # loop r: rank r % G, its location slot r // G
+        d = ((r % G) * cmax + r // G) * crec
+        cand[d:d + crec].copy_(ref_cand[r * crec:(r + 1) * crec])
+    for g in range(G):  # per-loop estimates of the sorted hits: rank g's local slot i = loop i G + g
+        x2[g, :H, :] = per_loop[:, g::G]
+    torch.cuda.synchronize()
+    l2 = torch.empty_like(locs)
+    v2 = torch.empty_like(vals)
+    local_us = timed(lambda: p.execute_local(x))
+
+    def lm():
+        p.execute_local(x)
+        p.execute_mid()
+
+    def lmf():
+        lm()
+        p.execute_finish(l2, v2)
+    lm_us = timed(lm)
+    lmf_us = timed(lmf)
+    lmf()
+    torch.cuda.synchronize()
+    same = torch.equal(l2, locs) and torch.equal(v2, vals)
+    b1, b2 = per * G, per2 * G
+    ag1 = 0.0 if G == 1 else ALPHA_US + (G - 1) / G * b1 / (BW_GBS * 1e3)
+    ag2 = 0.0 if G == 1 else ALPHA_US + (G - 1) / G * b2 / (BW_GBS * 1e3)
+    out["mode2"]["ranks"][G] = {"local_us": local_us, "mid_us": lm_us - local_us, "finish_us": lmf_us - lm_us,
+                                "allgather1_bytes": b1, "allgather2_bytes": b2, "allgather_model_us": ag1 + ag2,
+                                "model_total_us": lmf_us + ag1 + ag2, "finish_equals_single_gpu_output": same}
     p.close()
 print(json.dumps(out, indent=1))
 with open(sys.argv[1], "w") as f:
