@@ -281,6 +281,8 @@ def run_gpu(args):
     n, k, L, desc = CONFIGS[args.config]
     B = args.B or default_B(n, k)
     prm = plan_params(args.config, B)
+    if args.l2_persist is not None:
+        prm["l2_persist"] = args.l2_persist
     x_np, S, X = make_signal(n, k, args.signal_seed)
     x_pin = torch.from_numpy(x_np).pin_memory()
     x = x_pin.to(dev)
@@ -537,7 +539,9 @@ def run_gpu(args):
         "timed_region_ms_incl_flush": region_ms,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic,
-                     "kernel": "k_stage_packed (fold phase 1: address-ordered permute gather of x)",
+                     "kernel": ("k_stage_packed (fold phase 1: address-ordered permute gather of x)" if "warm" in gather
+                                else f"the whole fold stage ({int(info['staged'])} stage groups: phase 1 + phase 2 each)"
+                                if info["staged"] else "the whole fold stage (direct gather k_fold_fft1)"),
                      "algorithmic_bytes_per_launch": gather_bytes, "kernel_ms": rk_ms,
                      "algorithmic_bytes_note": f"L*w*32 B: {lw_local} gathers x one 32-B sector (SURVEY 8(d)); "
                                                f"{int(info['sectors'])} distinct sectors = {int(info['sectors']) * 32} B",
@@ -698,6 +702,8 @@ def main():
                     help="also time the cutoff variants (Alg. 3 sort, Alg. 6 threshold), the direct gather, no L2 set-aside")
     ap.add_argument("--k", type=int, default=0, help="C5k: sparsity k (the k sweep)")
     ap.add_argument("--bcst", type=float, default=1.0, help="B = floor_pow2(bcst sqrt(n k / log2 n)) (k sweep: 2 for k >= 2000)")
+    ap.add_argument("--l2-persist", type=int, default=None, choices=[0, 1],
+                    help="plan parameter l2_persist (default: the library default)")
     ap.add_argument("--snr", type=float, default=None, help="additive noise SNR in dB (C4 sweep); default noiseless")
     args = ap.parse_args()
     if args.warmup < 3:

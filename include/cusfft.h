@@ -273,8 +273,10 @@ int32_t cusfft_exchange_kind(cusfft_plan_t plan);
  * Plan facts (host arrays, caller-owned):
  *   info[0..15] = n, k, B, L, w (taps of the estimation filter), n/B, num_select, loc_loops,
  *                 vote_threshold, max_hits, distinct 32-B sectors of x this rank's gathers
- *                 touch (the fold's DRAM floor), staged (1: address-sorted two-phase gather,
- *                 DESIGN.md §6.2), w of the location filter, number of filters (1 or 2),
+ *                 touch (the fold's DRAM floor), staged (0: direct gather; g >= 1: the
+ *                 address-sorted two-phase gather, in g stage groups of
+ *                 consecutive slots, each staged and folded in turn when the staging of
+ *                 all slots would not fit L2), w of the location filter, number of filters (1 or 2),
  *                 fused tail (1: vote + estimation in one kernel), owns an NCCL
  *                 communicator (1)
  *   a, sigma, tau : int64 [L], in loop order r = 0..L-1 (NULL to skip).  sigma is

@@ -182,7 +182,12 @@ struct cusfft_plan_s {
   int64_t stage_total = 0;                   // gathers of this rank (sum of the local slots' w)
   uint32_t* d_code = nullptr;                // [stage_total] (local slot << ibits | i) in address order
   uint32_t* d_row0 = nullptr;                // [Lg] first staging row of each local slot
-  std::vector<uint32_t> row0_h;              // same, host (+ total rows at [Lg])
+  std::vector<uint32_t> row0_h;              // same, host (+ total rows at [Lg]); relative to the slot's group
+  // Stage groups (plans whose staging of all slots would not fit L2, e.g. C4): consecutive local
+  // slots [grp_s[g], grp_s[g + 1]) whose gathers are sorted, staged and folded together, one
+  // group after the other through one staging buffer; one group = the whole-plan staging.
+  std::vector<int> grp_s;
+  std::vector<int64_t> grp_off;              // first schedule word of each group (+ total at the end)
   double2* d_staging = nullptr;              // [rows][B]
   int stage_grid = 1;
   // gather 2 (ablation): the paper's remap + execute kernels on concurrent streams
@@ -837,51 +842,84 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     for (uint64_t b : bits) cnt += __builtin_popcountll(b);
     P->sectors = cnt;
   }
-  // ---- staged gather: every (local slot, tap) gather sorted by address at plan time
+  // ---- staged gather: every (local slot, tap) gather sorted by address at plan time, in
+  // groups of consecutive slots whose staging fits L2 (one group when all of it does)
   {
-    P->row0_h.assign((size_t)P->Lg + 1, 0u);
-    int64_t rows = 0, total = 0;
     int rmax = 0;
+    int64_t total = 0, rows_all = 0;
     for (int sl = 0; sl < P->Lg; ++sl) {
-      const Filter& F = P->filt[P->filt_of_local(sl)];
-      P->row0_h[sl] = (uint32_t)rows;
-      rows += F.R;
-      total += F.w;
-      rmax = std::max(rmax, F.R);
+      rmax = std::max(rmax, P->filt[P->filt_of_local(sl)].R);
+      total += P->filt[P->filt_of_local(sl)].w;
+      rows_all += P->filt[P->filt_of_local(sl)].R;
     }
-    P->row0_h[P->Lg] = (uint32_t)rows;
     P->stage_total = total;
+    const int64_t cap_rows = ((int64_t)64 << 20) / (B * 16);  // staging of one group <= 64 MB
+    int gs = rows_all <= cap_rows ? P->Lg : (int)std::max<int64_t>(1, cap_rows / std::max(1, rmax));
+    bool forced = false;
+    if (const char* e = std::getenv("CUSFFT_STAGE_GROUP")) {  // tests / A/B: force the group size
+      gs = std::max(1, std::atoi(e));
+      forced = true;
+    }
+    // several groups never straddle the location / estimation boundary (one filter and one
+    // branch each)
+    P->grp_s.clear();
+    for (int a = 0; a < P->Lg;) {
+      const int lim = (gs >= P->Lg) ? P->Lg : a < P->nloc_local ? P->nloc_local : P->Lg;
+      P->grp_s.push_back(a);
+      a = std::min(lim, a + gs);
+    }
+    P->grp_s.push_back(P->Lg);
+    const int ng = (int)P->grp_s.size() - 1;
+    P->row0_h.assign((size_t)P->Lg + 1, 0u);
+    int64_t rows_max = 0;
+    int gmax = 1;
+    for (int g = 0; g < ng; ++g) {
+      int64_t rows = 0;
+      for (int sl = P->grp_s[g]; sl < P->grp_s[g + 1]; ++sl) {
+        P->row0_h[sl] = (uint32_t)rows;
+        rows += P->filt[P->filt_of_local(sl)].R;
+      }
+      rows_max = std::max(rows_max, rows);
+      gmax = std::max(gmax, P->grp_s[g + 1] - P->grp_s[g]);
+    }
+    P->row0_h[P->Lg] = (uint32_t)rows_max;
     int ib = 1;
     while ((int64_t(1) << ib) < P->wmax) ++ib;
     int sb = 0;
-    while ((1 << sb) < P->Lg) ++sb;
+    while ((1 << sb) < gmax) ++sb;
     P->stage_ibits = ib;
-    const int64_t staging_bytes = rows * B * 16;
+    const int64_t staging_bytes = rows_max * B * 16;
     // the staging buffer must be (mostly) L2-resident between the two phases, phase 2
     // streams a CTA's R rows (4 KB each) into shared memory, and the schedule word must
-    // hold (slot, tap); signal-sharded plans gather only their slice (direct path)
-    P->staged = P->fused1 && !P->xshard && q.gather == 0 && staging_bytes <= (int64_t)64 << 20 && rmax <= 48 &&
+    // hold (slot in group, tap); signal-sharded plans gather only their slice (direct path)
+    P->staged = P->fused1 && !P->xshard && q.gather == 0 && (forced || staging_bytes <= (int64_t)64 << 20) && rmax <= 48 &&
                 ib + sb <= 32 && total < (int64_t)1 << 31;
     if (P->staged) {
       const uint32_t nm = (uint32_t)(n - 1);
-      std::vector<uint64_t> ev;
-      ev.reserve((size_t)total);
-      for (int sl = 0; sl < P->Lg; ++sl) {
-        const SlotParam& sp = P->slots_h[(size_t)lrank * P->Lg + sl];
-        const int w = P->filt[P->filt_of_local(sl)].w;
-        for (int i = 0; i < w; ++i) {
-          const uint32_t pos = (sp.sigma * (uint32_t)i + sp.tau) & nm;
-          ev.push_back(((uint64_t)pos << 32) | ((uint64_t)sl << ib) | (uint64_t)i);
-        }
-      }
-      std::sort(ev.begin(), ev.end());
       std::vector<uint32_t> code((size_t)total);
-      for (int64_t j = 0; j < total; ++j) code[(size_t)j] = (uint32_t)(ev[(size_t)j] & 0xFFFFFFFFull);
+      P->grp_off.assign((size_t)ng + 1, 0);
+      std::vector<uint64_t> ev;
+      for (int g = 0; g < ng; ++g) {
+        ev.clear();
+        for (int sl = P->grp_s[g]; sl < P->grp_s[g + 1]; ++sl) {
+          const SlotParam& sp = P->slots_h[(size_t)lrank * P->Lg + sl];
+          const int w = P->filt[P->filt_of_local(sl)].w;
+          const uint64_t sg = (uint64_t)(sl - P->grp_s[g]) << ib;
+          for (int i = 0; i < w; ++i) {
+            const uint32_t pos = (sp.sigma * (uint32_t)i + sp.tau) & nm;
+            ev.push_back(((uint64_t)pos << 32) | sg | (uint64_t)i);
+          }
+        }
+        std::sort(ev.begin(), ev.end());
+        const int64_t o = P->grp_off[g];
+        for (size_t j = 0; j < ev.size(); ++j) code[(size_t)o + j] = (uint32_t)(ev[j] & 0xFFFFFFFFull);
+        P->grp_off[g + 1] = o + (int64_t)ev.size();
+      }
       if ((rc = dalloc(&P->d_code, code.size()))) return fail(rc);
       if ((rc = upload(P->d_code, code.data(), code.size() * sizeof(uint32_t)))) return fail(rc);
       if ((rc = dalloc(&P->d_row0, (size_t)P->Lg))) return fail(rc);
       if ((rc = upload(P->d_row0, P->row0_h.data(), (size_t)P->Lg * sizeof(uint32_t)))) return fail(rc);
-      if ((rc = dalloc(&P->d_staging, (size_t)(rows * B)))) return fail(rc);
+      if ((rc = dalloc(&P->d_staging, (size_t)(rows_max * B)))) return fail(rc);
       // one resident wave of phase-1 CTAs (grid-stride loop), at most 4 per SM: with one gather in
       // flight per thread (schedule words prefetched) that is 1024 per SM, measured best
       // (profiles/r02_stage_ab.md; dynamic chunking of the last quarter measured slower)
@@ -891,10 +929,12 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       const int per = 256 * kStageU;
       int cps = std::min(occ, 4);
       if (const char* e = std::getenv("CUSFFT_STAGE_CPS")) cps = std::max(1, std::min(occ, std::atoi(e)));  // A/B (measurement)
-      P->stage_grid = (int)std::max<int64_t>(1, std::min<int64_t>((total + per - 1) / per, (int64_t)P->sms * cps));
+      int64_t gtot = 0;
+      for (int g = 0; g < ng; ++g) gtot = std::max(gtot, P->grp_off[g + 1] - P->grp_off[g]);
+      P->stage_grid = (int)std::max<int64_t>(1, std::min<int64_t>((gtot + per - 1) / per, (int64_t)P->sms * cps));
       // Persisting-L2 set-aside for the staging buffer: the staging stores carry evict_last
-      // (= persisting) and the x loads evict_first; without the set-aside C3 took 100 us
-      // instead of 87.  Device-wide and optional (params.l2_persist).
+      // (= persisting) and the x loads evict_first; C3 is 3 us slower without it
+      // (profiles/r02_stage_ab.md).  Device-wide and optional (params.l2_persist).
       int maxp = 0;
       cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev);
       const size_t win = std::min<size_t>((size_t)staging_bytes, (size_t)maxp);
@@ -965,10 +1005,13 @@ inline void mark(cusfft_plan_t P, int i) {
 // ---------------------------------------------------------------------------
 // Staged fold, phase 1: every gather of this rank in address order, each
 // sample stored at its phase-2 position.  Zeroes the per-execution block.
-int launch_stage1(cusfft_plan_t P, const double2* x, cudaStream_t st) {
-  StagePackArgs a{x, P->d_code, P->d_staging, P->d_slots + (size_t)P->lrank * P->Lg, P->d_row0,
-                  (int)P->stage_total, P->Lg, P->stage_ibits, ilog2(P->B), P->logB2, P->logB1,
-                  ilog2(256 / P->B1), (uint32_t)(P->n - 1), ZeroArgs{P->d_zero, P->nzero}};
+int launch_stage1(cusfft_plan_t P, const double2* x, cudaStream_t st, int g = 0) {
+  const int s0 = P->grp_s[(size_t)g], s1 = P->grp_s[(size_t)g + 1];
+  const int64_t o = P->grp_off[(size_t)g];
+  const ZeroArgs z = g == 0 ? ZeroArgs{P->d_zero, P->nzero} : ZeroArgs{nullptr, 0};
+  StagePackArgs a{x, P->d_code + o, P->d_staging, P->d_slots + (size_t)P->lrank * P->Lg + s0, P->d_row0 + s0,
+                  (int)(P->grp_off[(size_t)g + 1] - o), s1 - s0, P->stage_ibits, ilog2(P->B), P->logB2, P->logB1,
+                  ilog2(256 / P->B1), (uint32_t)(P->n - 1), z};
   CK(launch_k(k_stage_packed<kStageU>, dim3(P->stage_grid), dim3(256), 0, st, P->cur_prio, a));
   return CUSFFT_SUCCESS;
 }
@@ -1413,7 +1456,13 @@ int launch_local(cusfft_plan_t P, const double2* x) {
   mark(P, 0);
   g_pdl = false;  // the first kernel follows arbitrary caller work
   const int nl = P->nloc_local;
-  if (P->staged) {
+  if (P->staged && P->grp_s.size() > 2) {  // stage groups, one after the other through one staging buffer
+    for (size_t g = 0; g + 1 < P->grp_s.size(); ++g) {
+      TRY(launch_stage1(P, x, st, (int)g));
+      g_pdl = P->timing != 1;
+      TRY(launch_fold_range(P, x, P->grp_s[g], P->grp_s[g + 1], st, false));
+    }
+  } else if (P->staged) {
     TRY(launch_stage1(P, x, st));
     mark(P, 7);
     g_pdl = P->timing != 1;
@@ -1543,7 +1592,7 @@ int launch_branched(cusfft_plan_t P, const double2* x, int64_t* locs, double2* v
 }
 
 inline bool use_branches(cusfft_plan_t P) {
-  return P->timing != 1 && P->staged && P->nloc_local > 0 &&
+  return P->timing != 1 && P->staged && P->grp_s.size() == 2 && P->nloc_local > 0 &&
          P->nloc_local < P->Lg && !P->xshard;
 }
 
@@ -1908,7 +1957,7 @@ int cusfft_get_info(cusfft_plan_t plan, int64_t* info, int64_t* a, int64_t* sigm
   if (!valid_plan(plan)) return CUSFFT_INVALID_PLAN;
   if (info) {
     int64_t v[16] = {plan->n, plan->k, plan->B, plan->L, plan->filt[plan->nfilt - 1].w, plan->nb, plan->num,
-                     plan->Lloc, plan->T, plan->max_hits, plan->sectors, plan->staged ? 1 : 0,
+                     plan->Lloc, plan->T, plan->max_hits, plan->sectors, plan->staged ? (int64_t)plan->grp_s.size() - 1 : 0,
                      plan->filt[0].w, plan->nfilt, plan->tail_esz ? 1 : 0, plan->comm ? 1 : 0};
     std::memcpy(info, v, sizeof(v));
   }
@@ -2038,7 +2087,7 @@ int cusfft_get_stage_times(cusfft_plan_t plan, float* ms, int32_t cap) {
   }
   if (cap >= 7) {
     float t = -1.f;
-    if (!plan->staged || cudaEventElapsedTime(&t, plan->ev[0], plan->ev[7]) != cudaSuccess) {
+    if (!plan->staged || plan->grp_s.size() > 2 || cudaEventElapsedTime(&t, plan->ev[0], plan->ev[7]) != cudaSuccess) {
       t = -1.f;
       cudaGetLastError();
     }
@@ -2093,7 +2142,8 @@ int32_t cusfft_launches_per_execute(cusfft_plan_t plan) {
   const bool branched = use_branches(plan);
   const bool f2s = use_fft2_select(plan);  // location pass 2 inside the cutoff kernel
   const int ffts = f2s ? (ne > 0 ? 1 : 0) : (branched ? ranges : 1);
-  int n = (plan->staged ? 1 : 0) + ranges /*fold per slot range*/ +
+  const int ngrp = plan->staged ? (int)plan->grp_s.size() - 1 : 0;
+  int n = (ngrp > 1 ? 2 * ngrp - ranges : ngrp) + ranges /*phase 1 per group, fold per slot range (or group)*/ +
           ffts * (pass1 ? 2 : 1) /*fft*/ + (plan->sel_slots_h.empty() ? 0 : 1) +
           (plan->xshard && !plan->sel_slots_h.empty() ? 1 : 0) /*keys*/ + (plan->tail_esz ? 2 : 3);
   // shard_mode 2: vote (k_tail vote-only or k_vote) + k_rank_est + k_median + k_output

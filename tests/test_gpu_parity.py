@@ -130,6 +130,18 @@ def test_parity_shared_taps(n, k, B, L, extra):
     check_all(plan, ref, locs, vals, fold_bit_exact=True)
 
 
+@pytest.mark.parametrize("gs", [1, 3, 8])
+def test_parity_stage_groups_shared_taps(gs, monkeypatch):
+    """Stage groups (the staged gather of C4-sized plans, forced here at n =
+    2^18): every group's fold stays bit-exact with the oracle's Alg. 1 order."""
+    monkeypatch.setenv("CUSFFT_STAGE_GROUP", str(gs))
+    n, k, B, L = 2 ** 18, 100, 4096, 16
+    x, S, X = planted_signal(n, k, seed=77)
+    plan, ref, locs, vals = run_pair(x, n, k, B, L, shared_taps=True, seed=11)
+    assert plan.info()["staged"] == {1: 16, 3: 6, 8: 2}[gs]
+    check_all(plan, ref, locs, vals, fold_bit_exact=True)
+
+
 @pytest.mark.parametrize("n,k,B,L,extra", CASES[:6])
 def test_parity_own_filter(n, k, B, L, extra):
     """The plan builds its own filter on the GPU; the oracle builds its own."""
@@ -292,11 +304,12 @@ def test_stage_timing_and_launch_count():
 
 def test_C4_full_size_parity():
     """BASELINE.json configs[3] size: n = 2^27, k = 1000 (B = 65536, two-pass
-    FFT with B1 = B2 = 256, direct gather: the staging would not fit L2)."""
+    FFT with B1 = B2 = 256; the staging of all 16 loops (218 MB) would not fit
+    L2, so the staged gather runs in 4 stage groups of 4 loops)."""
     n, k = 2 ** 27, 1000
     x, S, X = planted_signal(n, k, seed=2)
     plan, ref, locs, vals = run_pair(x, n, k, None, 16, shared_taps=False, seed=4)
-    assert plan.info()["staged"] == 0
+    assert plan.info()["staged"] == 4
     check_all(plan, ref, locs, vals, fold_bit_exact=False)
     assert set(locs.tolist()) == set(S.tolist())
     assert O.l1_error(locs, vals, S, X, k) <= 1e-6
@@ -317,12 +330,13 @@ def test_parity_snr_sweep(snr_db):
                                     ({"CUSFFT_FFT2SEL": "0"}, {}),
                                     ({}, dict(gather=1)), ({}, dict(l2_persist=0)),
                                     ({"CUSFFT_TAIL": "0", "CUSFFT_NO_GRAPH": "1"}, dict(gather=1)),
-                                    ({}, dict(gather=2)), ({"CUSFFT_NO_GRAPH": "1"}, dict(gather=2))])
+                                    ({}, dict(gather=2)), ({"CUSFFT_NO_GRAPH": "1"}, dict(gather=2)),
+                                    ({"CUSFFT_STAGE_GROUP": "4"}, {}), ({"CUSFFT_STAGE_GROUP": "3"}, {})])
 def test_kernel_paths_agree(env, kw, monkeypatch):
     """Every alternative path (no CUDA graph, the k_vote / k_estimate /
     k_output chain instead of the fused tail, the direct gather or the
-    paper's remap + execute kernels instead of the staged gather, no
-    persisting-L2 set-aside) gives the default path's hits
+    paper's remap + execute kernels instead of the staged gather, the staged
+    gather in stage groups of 4 / 3 slots, no persisting-L2 set-aside) gives the default path's hits
     and output exactly (same fold order, same selection rules)."""
     import torch
     from paper_conf_ipps_wangcc16_b200 import Plan
@@ -341,7 +355,8 @@ def test_kernel_paths_agree(env, kw, monkeypatch):
     torch.cuda.synchronize()
     assert alt.status() == 0
     assert alt.info()["tail"] == (0 if env.get("CUSFFT_TAIL") == "0" else 1)
-    assert alt.info()["staged"] == (0 if kw.get("gather") in (1, 2) else 1)
+    groups = {"4": 4, "3": 6}.get(env.get("CUSFFT_STAGE_GROUP"), 1)  # groups never straddle slot 8
+    assert alt.info()["staged"] == (0 if kw.get("gather") in (1, 2) else groups)
     assert np.array_equal(np.sort(alt.debug(DEBUG_HITS)), h0)
     assert torch.equal(l1, l0)
     assert torch.equal(v1, v0)
