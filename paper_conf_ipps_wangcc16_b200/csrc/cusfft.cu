@@ -188,6 +188,7 @@ struct cusfft_plan_s {
   // group after the other through one staging buffer; one group = the whole-plan staging.
   std::vector<int> grp_s;
   std::vector<int64_t> grp_off;              // first schedule word of each group (+ total at the end)
+  bool grp_abs = false;                      // groups keep their own staging rows (all of it fits L2)
   double2* d_staging = nullptr;              // [rows][B]
   int stage_grid = 1;
   // gather 2 (ablation): the paper's remap + execute kernels on concurrent streams
@@ -870,17 +871,23 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     }
     P->grp_s.push_back(P->Lg);
     const int ng = (int)P->grp_s.size() - 1;
+    // rows: relative to the group (one shared buffer, groups staged one after the other) unless
+    // the staging of all loops fits, when every group keeps its own rows (groups may overlap)
+    P->grp_abs = rows_all <= cap_rows;
     P->row0_h.assign((size_t)P->Lg + 1, 0u);
     int64_t rows_max = 0;
     int gmax = 1;
-    for (int g = 0; g < ng; ++g) {
+    {
       int64_t rows = 0;
-      for (int sl = P->grp_s[g]; sl < P->grp_s[g + 1]; ++sl) {
-        P->row0_h[sl] = (uint32_t)rows;
-        rows += P->filt[P->filt_of_local(sl)].R;
+      for (int g = 0; g < ng; ++g) {
+        if (!P->grp_abs) rows = 0;
+        for (int sl = P->grp_s[g]; sl < P->grp_s[g + 1]; ++sl) {
+          P->row0_h[sl] = (uint32_t)rows;
+          rows += P->filt[P->filt_of_local(sl)].R;
+        }
+        rows_max = std::max(rows_max, rows);
+        gmax = std::max(gmax, P->grp_s[g + 1] - P->grp_s[g]);
       }
-      rows_max = std::max(rows_max, rows);
-      gmax = std::max(gmax, P->grp_s[g + 1] - P->grp_s[g]);
     }
     P->row0_h[P->Lg] = (uint32_t)rows_max;
     int ib = 1;
@@ -1549,11 +1556,18 @@ int launch_branched(cusfft_plan_t P, const double2* x, int64_t* locs, double2* v
   cudaStream_t a = P->stream, b = P->cap_stream2;
   const int nl = P->nloc_local;
   const int lim = P->stage_limit;
+  // two stage groups (location / estimation loops, each with its own staging rows): the
+  // estimation loops' phase 1 runs on the second branch, after the location loops' one
+  const bool split = P->grp_s.size() == 3;
   auto fork = [&]() -> int {
     CK(cudaEventRecord(P->ev_fork, a));
     CK(cudaStreamWaitEvent(b, P->ev_fork, 0));
     P->cur_prio = P->prio_lo;
     g_pdl = false;
+    if (split) {
+      TRY(launch_stage1(P, x, b, 1));
+      g_pdl = true;
+    }
     TRY(launch_fold_range(P, x, nl, P->Lg, b, false));
     g_pdl = true;
     if (lim >= 2) TRY(launch_bfft(P, nl, P->Lg, b));
@@ -1566,19 +1580,19 @@ int launch_branched(cusfft_plan_t P, const double2* x, int64_t* locs, double2* v
   g_pdl = false;
   mark(P, 0);
   TRY(launch_stage1(P, x, a));
-  mark(P, 7);
-  if (P->fork_at == 0) TRY(fork());
+  if (!split) mark(P, 7);
+  if (P->fork_at == 0 || split) TRY(fork());
   g_pdl = true;
   TRY(launch_fold_range(P, x, 0, nl, a, false));
-  if (P->fork_at == 1) TRY(fork());
+  if (P->fork_at == 1 && !split) TRY(fork());
   const bool f2s = use_fft2_select(P);  // location slots: FFT pass 2 inside the cutoff kernel (stage 3)
   if (lim >= 2 && !f2s) TRY(launch_bfft(P, 0, nl, a));
-  if (P->fork_at == 2) TRY(fork());
+  if (P->fork_at == 2 && !split) TRY(fork());
   if (f2s && lim >= 3)
     TRY(launch_fft2_select(P, a));
   else if (lim >= 3 && !P->xshard)
     TRY(launch_select(P, a));
-  if (P->fork_at == 3) TRY(fork());
+  if (P->fork_at == 3 && !split) TRY(fork());
   P->cur_prio = 0;
   CK(cudaStreamWaitEvent(a, P->ev_join, 0));
   g_pdl = false;
@@ -1592,7 +1606,8 @@ int launch_branched(cusfft_plan_t P, const double2* x, int64_t* locs, double2* v
 }
 
 inline bool use_branches(cusfft_plan_t P) {
-  return P->timing != 1 && P->staged && P->grp_s.size() == 2 && P->nloc_local > 0 &&
+  const bool split = P->grp_abs && P->grp_s.size() == 3 && P->grp_s[1] == P->nloc_local;  // phase 1 per branch
+  return P->timing != 1 && P->staged && (P->grp_s.size() == 2 || split) && P->nloc_local > 0 &&
          P->nloc_local < P->Lg && !P->xshard;
 }
 

@@ -331,12 +331,14 @@ def test_parity_snr_sweep(snr_db):
                                     ({}, dict(gather=1)), ({}, dict(l2_persist=0)),
                                     ({"CUSFFT_TAIL": "0", "CUSFFT_NO_GRAPH": "1"}, dict(gather=1)),
                                     ({}, dict(gather=2)), ({"CUSFFT_NO_GRAPH": "1"}, dict(gather=2)),
-                                    ({"CUSFFT_STAGE_GROUP": "4"}, {}), ({"CUSFFT_STAGE_GROUP": "3"}, {})])
+                                    ({"CUSFFT_STAGE_GROUP": "4"}, {}), ({"CUSFFT_STAGE_GROUP": "3"}, {}),
+                                    ({"CUSFFT_STAGE_GROUP": "8"}, {})])
 def test_kernel_paths_agree(env, kw, monkeypatch):
     """Every alternative path (no CUDA graph, the k_vote / k_estimate /
     k_output chain instead of the fused tail, the direct gather or the
     paper's remap + execute kernels instead of the staged gather, the staged
-    gather in stage groups of 4 / 3 slots, no persisting-L2 set-aside) gives the default path's hits
+    gather in stage groups of 4 / 3 slots or split over the two graph branches,
+    no persisting-L2 set-aside) gives the default path's hits
     and output exactly (same fold order, same selection rules)."""
     import torch
     from paper_conf_ipps_wangcc16_b200 import Plan
@@ -355,7 +357,8 @@ def test_kernel_paths_agree(env, kw, monkeypatch):
     torch.cuda.synchronize()
     assert alt.status() == 0
     assert alt.info()["tail"] == (0 if env.get("CUSFFT_TAIL") == "0" else 1)
-    groups = {"4": 4, "3": 6}.get(env.get("CUSFFT_STAGE_GROUP"), 1)  # groups never straddle slot 8
+    # groups never straddle slot 8; 8-loop groups = phase 1 split over the two graph branches
+    groups = {"4": 4, "3": 6, "8": 2}.get(env.get("CUSFFT_STAGE_GROUP"), 1)
     assert alt.info()["staged"] == (0 if kw.get("gather") in (1, 2) else groups)
     assert np.array_equal(np.sort(alt.debug(DEBUG_HITS)), h0)
     assert torch.equal(l1, l0)
