@@ -160,6 +160,7 @@ struct StagePackArgs {
   int total, nslots, ibits, logB, logB2, logB1, logC;
   uint32_t nmask;
   ZeroArgs zero;
+  int rows;  // staging rows this launch writes into (from row 0)
 };
 
 // U: gathers in flight per thread per pass (1 at 4 CTAs of 256 per SM; U = 2, 4, 8 and 2-3 CTAs
@@ -180,6 +181,18 @@ __global__ void __launch_bounds__(256) k_stage_packed(StagePackArgs A) {
     srow[i] = A.row0[i];
   }
   zero_part(A.zero);
+  // The staging lines are requested into L2 (evict_last) before the scattered
+  // stores land on them: when they are not resident (the cold state: after
+  // cudaCtxResetPersistingL2Cache or other work evicted them) every 16-B store
+  // would otherwise miss on its own (phase 1 cold: 46 -> 31 µs; warm they hit,
+  // +0.25 µs per transform; profiles/r02_stage_ab.md).  Fire-and-forget: the
+  // gathers do not wait on them.
+  {
+    const int64_t lines = (int64_t)A.rows << A.logB >> 3;  // 128-B lines (8 samples each)
+    const char* base = reinterpret_cast<const char*>(A.staging);
+    for (int64_t l = blockIdx.x * blockDim.x + threadIdx.x; l < lines; l += gridDim.x * blockDim.x)
+      asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(base + (l << 7)));
+  }
   __syncthreads();
   const uint64_t pf = l2_policy_first(), pl = l2_policy_last();
   const uint32_t imask = (1u << A.ibits) - 1u;
