@@ -1018,7 +1018,10 @@ int launch_stage1(cusfft_plan_t P, const double2* x, cudaStream_t st, int g = 0)
   const ZeroArgs z = g == 0 ? ZeroArgs{P->d_zero, P->nzero} : ZeroArgs{nullptr, 0};
   StagePackArgs a{x, P->d_code + o, P->d_staging, P->d_slots + (size_t)P->lrank * P->Lg + s0, P->d_row0 + s0,
                   (int)(P->grp_off[(size_t)g + 1] - o), s1 - s0, P->stage_ibits, ilog2(P->B), P->logB2, P->logB1,
-                  ilog2(256 / P->B1), (uint32_t)(P->n - 1), z, (int)P->row0_h[(size_t)P->Lg]};
+                  ilog2(256 / P->B1), (uint32_t)(P->n - 1), z,
+                  // staging rows to prefetch into L2: the whole buffer, by the first group (later
+                  // groups of a shared buffer find the lines the previous group used)
+                  g == 0 ? (int)P->row0_h[(size_t)P->Lg] : 0};
   CK(launch_k(k_stage_packed<kStageU>, dim3(P->stage_grid), dim3(256), 0, st, P->cur_prio, a));
   return CUSFFT_SUCCESS;
 }
