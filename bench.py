@@ -693,7 +693,8 @@ def main():
                          "(SURVEY N1, all-reduce) or loop sharding with two all-gathers (candidates, then "
                          "per-loop estimates: SURVEY 8(e) steps 1-5)")
     ap.add_argument("--B", type=int, default=0, help="bucket count (default: the paper's formula, DESIGN.md Z3)")
-    ap.add_argument("--pipeline", type=int, default=2, help="C5 batch: clone plans in flight per GPU")
+    ap.add_argument("--pipeline", type=int, default=3,
+                    help="C5 batch: clone plans in flight per GPU (3 measured best: 38.3 / 36.9 / 38.0 us per transform at 2 / 3 / 4)")
     ap.add_argument("--cpu-budget-s", type=float, default=15.0)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-cupti", action="store_true")
