@@ -795,8 +795,10 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   attr(set_dyn_smem(k_fft2_select<128, 32>, fft2sel_smem_bytes<128, 32>(), smem_optin));
   attr(set_dyn_smem(k_vote, smem_optin, smem_optin));
   attr(set_dyn_smem(k_output, smem_optin, smem_optin));
-  if (P->tail_esz) attr(set_dyn_smem(tail_kernel(P->tail_esz, L, P->Lloc), P->tail_smem, smem_optin));
-  if (P->tail_esz && q.shard_mode == 2) attr(set_dyn_smem(tail_vote_kernel(P->tail_esz, P->Lloc), P->tail_smem, smem_optin));
+  // (the per-function limits are raised to the device maximum, never lowered to this plan's
+  // need: plans of other shapes share the kernels)
+  if (P->tail_esz) attr(set_dyn_smem(tail_kernel(P->tail_esz, L, P->Lloc), smem_optin, smem_optin));
+  if (P->tail_esz && q.shard_mode == 2) attr(set_dyn_smem(tail_vote_kernel(P->tail_esz, P->Lloc), smem_optin, smem_optin));
   if (ae != cudaSuccess) {
     g_last_cuda_error = (int)ae;
     return fail(CUSFFT_CUDA);
@@ -972,7 +974,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     P->mode2 = true;
     P->cmax = (P->Lloc + world - 1) / world;
     P->crec_bytes = P->lay.rec_bytes - P->lay.off_bitmap;
-    if (set_dyn_smem(k_rank_est, P->max_hits * 4, smem_optin) != cudaSuccess) {  // k_rank_est stages the hit list
+    if (set_dyn_smem(k_rank_est, smem_optin, smem_optin) != cudaSuccess) {  // k_rank_est stages the hit list
       g_last_cuda_error = (int)cudaGetLastError();
       return fail(CUSFFT_CUDA);
     }

@@ -583,3 +583,34 @@ def test_l2_persist_opt_out():
     assert plan.info()["staged"]
     assert rt.cudaDeviceGetLimit(lim)[1] == before
     plan.close()
+
+
+@pytest.mark.gpu
+def test_plans_of_different_shapes_coexist():
+    """Kernels are shared by every plan of the process: creating a plan of a
+    small shape must not lower a per-function launch limit (dynamic shared
+    memory) another live plan needs — e.g. the fused tail's vote table at B =
+    32768 after a B = 512 plan, or the two-collective ranking's hit list."""
+    n1, k1 = 2 ** 21, 60
+    x1, S1, _ = planted_signal(n1, k1, seed=31)
+    n2, k2 = 2 ** 16, 20
+    x2, S2, _ = planted_signal(n2, k2, seed=32)
+    xd1, xd2 = torch.from_numpy(x1).to(DEV), torch.from_numpy(x2).to(DEV)
+    with Plan(n1, k1, B=32768, L=16, seed=3) as alone:  # before any other shape exists
+        l0, v0 = alone.execute(xd1)
+        torch.cuda.synchronize()
+    big = Plan(n1, k1, B=32768, L=16, seed=3)
+    big2 = Plan(n1, k1, B=32768, L=16, seed=3, shard_mode=2, max_hits=32768)
+    small = Plan(n2, k2, L=16, seed=4)
+    small2 = Plan(n2, k2, L=16, seed=4, shard_mode=2, max_hits=1024)
+    ls, vs = small.execute(xd2)
+    lb, vb = big.execute(xd1)
+    lb2, vb2 = big2.execute(xd1)
+    ls2, vs2 = small2.execute(xd2)
+    torch.cuda.synchronize()
+    for p in (big, big2, small, small2):
+        assert p.status() == 0
+    assert torch.equal(lb, lb2) and torch.equal(vb, vb2)
+    assert torch.equal(ls, ls2) and torch.equal(vs, vs2)
+    assert torch.equal(lb, l0) and torch.equal(vb, v0)
+    assert sorted(ls.tolist()) == sorted(S2.tolist())
