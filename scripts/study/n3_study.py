@@ -27,7 +27,7 @@ import numpy as np
 import oracle as O
 from paper_conf_ipps_wangcc16_b200.workload import planted_signal
 
-n, k, L_loc, L_est, T = 2 ** 24, 1000, 8, 8, 5
+n, k, L_loc, L_est, T = 2 ** 24, 1000, 8, int(os.environ.get("N3_LEST", "8")), 5  # N3_LEST: estimation-only loops
 B = int(os.environ.get("N3_B", "16384"))  # N3_B=8192: half the formula's buckets (Bcst = 1/2)
 nb = n // B
 
@@ -78,6 +78,14 @@ SETTINGS5 = {
     "all_d1e-7_lam0.75": (1e-7, 0.75, 1e-7, 1, 0.75),
     "all_d1e-7_lam0.5": (1e-7, 0.5, 1e-7, 1, 0.5),
 }
+# sixth round (N3_SET=6, with N3_LEST=4 / 6): fewer estimation-only loops (L = 12 / 14) at the
+# C3 bench filter
+SETTINGS6 = {
+    "all_d1e-7_lam0.75": (1e-7, 0.75, 1e-7, 1, 0.75),
+    "all_d1e-7_lam0.5": (1e-7, 0.5, 1e-7, 1, 0.5),
+}
+if os.environ.get("N3_SET") == "6":
+    SETTINGS = SETTINGS6
 if os.environ.get("N3_SET") == "5":
     SETTINGS = SETTINGS5
 if os.environ.get("N3_SET") == "4":
@@ -115,7 +123,7 @@ def run_setting(x, S, X, seed, name):
     med = (per_loop.shape[1] - 1) // 2
     vals = np.sort(per_loop.real, axis=1)[:, med] + 1j * np.sort(per_loop.imag, axis=1)[:, med]
     locs, out = O.select_output(hits, vals, k)
-    return {"setting": name, "B": B, "seed": seed, "delta_loc": d_loc, "lambda_loc_B": lam_loc, "delta_est": d_est,
+    return {"setting": name, "B": B, "L": L_loc + L_est, "seed": seed, "delta_loc": d_loc, "lambda_loc_B": lam_loc, "delta_est": d_est,
             "lambda_est_B": lam_est, "num": int(numf * k), "w_loc": len(g_loc), "w_est": len(g_est),
             "sum_w": L_loc * len(g_loc) + L_est * len(g_est),
             "exact": bool(set(locs.tolist()) == set(S.tolist())),
