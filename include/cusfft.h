@@ -120,8 +120,9 @@ typedef struct {
   double loc_lobefrac;     /* lambda of the location loops' filter; 0 (default): lobefrac        */
   int32_t l2_persist;      /* 1 (default): staged plans raise the device's persisting-L2 set-aside
                               while they live (see above); 0: never touch the device limit       */
-  int32_t gather;          /* 0 (default): address-sorted staged gather when its staging buffer fits
-                              L2, else direct; 1: always the direct gather;
+  int32_t gather;          /* 0 (default): address-sorted staged gather, in stage
+                              groups of consecutive loops when the staging of all loops would not
+                              fit L2, direct when one loop's would not; 1: always the direct gather;
                               2: the paper's remap + execute kernels on concurrent streams
                               (an ablation; not with shard_mode 1)           */
 } cusfft_params;
