@@ -535,18 +535,20 @@ def test_parity_separate_filters(n, k, extra):
 
 
 @pytest.mark.gpu
-def test_library_owned_nccl_exchange_world1():
+@pytest.mark.parametrize("shard_mode", [0, 2])
+def test_library_owned_nccl_exchange_world1(shard_mode):
     """cusfft_plan_dist with an ncclUniqueId: the plan owns a communicator and
-    cusfft_execute runs the whole transform with the collective inside the
-    plan's CUDA graph (a one-rank communicator on the single test GPU); the
-    output equals the plain plan's bit for bit."""
+    cusfft_execute runs the whole transform with the collective(s) inside the
+    plan's CUDA graph (a one-rank communicator on the single test GPU; shard
+    mode 2: both all-gathers); the output equals the plain plan's bit for bit."""
     from paper_conf_ipps_wangcc16_b200 import nccl_unique_id
     n, k = 2 ** 22, 1000
     x, S, X = planted_signal(n, k, seed=27)
     xd = torch.from_numpy(x).to(DEV)
     plain = Plan(n, k, L=16, seed=6)
     l0, v0 = plain.execute(xd)
-    owned = Plan(n, k, L=16, seed=6, rank=0, world=1, nccl_id=nccl_unique_id())
+    extra = dict(shard_mode=2, max_hits=8192) if shard_mode == 2 else {}
+    owned = Plan(n, k, L=16, seed=6, rank=0, world=1, nccl_id=nccl_unique_id(), **extra)
     assert owned.info()["owns_comm"] == 1
     for _ in range(2):  # capture, then replay
         l1, v1 = owned.execute(xd)
