@@ -1,3 +1,4 @@
+# sanitizers are closed on this pool (round 2): this script documents how the r02_sanitize logs were made
 # compute-sanitizer memcheck / racecheck / synccheck of the default path (direct launches, no graph)
 mkdir -p gpurun_out/sanitize
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1 || exit 1
