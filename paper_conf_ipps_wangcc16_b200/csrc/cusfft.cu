@@ -1037,22 +1037,34 @@ cudaError_t launch_p2_t(cusfft_plan_t P, const Filter& F, const double2* staging
     cudaFuncSetAttribute(k_fold_fft1_tma<B1T, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
     attr_set = true;
   }
-  if (P->p2_ms && F.R <= 16) {  // multi-slot form (k_fold_fft1_ms): 8 slots per CTA, 4 (R <= 8) or 2 in flight
-    constexpr int NSM = 8;
+  if (P->p2_ms && F.R <= 16) {  // multi-slot form (k_fold_fft1_ms)
+    // R <= 8: 8 slots per CTA, 4 in flight.  8 < R <= 16: 8 slots per CTA with 2 in flight
+    // (one CTA per SM), or 4 slots per CTA with 1 in flight (two CTAs per SM) for ranges of at
+    // most 4 slots or B <= 16384 (C4: 333 -> 325 us, C5 k = 1000: 62.1 -> 57.5 us; B = 32768
+    // ranges of 8 slots, C5 k = 4096, are faster with 8: profiles/r02_stage_ab.md)
     static thread_local bool ms_attr = false;
     if (!ms_attr) {
-      cudaFuncSetAttribute(k_fold_fft1_ms<B1T, NSM, 4, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           fold_ms_smem_bytes<B1T, NSM, 4, 8>());
-      cudaFuncSetAttribute(k_fold_fft1_ms<B1T, NSM, 2, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           fold_ms_smem_bytes<B1T, NSM, 2, 16>());
+      cudaFuncSetAttribute(k_fold_fft1_ms<B1T, 8, 4, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           fold_ms_smem_bytes<B1T, 8, 4, 8>());
+      cudaFuncSetAttribute(k_fold_fft1_ms<B1T, 8, 2, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           fold_ms_smem_bytes<B1T, 8, 2, 16>());
+      cudaFuncSetAttribute(k_fold_fft1_ms<B1T, 4, 1, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           fold_ms_smem_bytes<B1T, 4, 1, 16>());
       ms_attr = true;
     }
-    dim3 grid((unsigned)(P->B / 256), (unsigned)((nslots + NSM - 1) / NSM));
-    const bool r8 = F.R <= 8;
-    return launch_k(r8 ? k_fold_fft1_ms<B1T, NSM, 4, 8> : k_fold_fft1_ms<B1T, NSM, 2, 16>, grid, dim3(256),
-                    (size_t)(r8 ? fold_ms_smem_bytes<B1T, NSM, 4, 8>() : fold_ms_smem_bytes<B1T, NSM, 2, 16>()),
-                    st, P->cur_prio, staging, (const double*)F.d_taps_perm, P->prm.debug ? u : nullptr, v,
-                    (const double2*)P->d_tw, (int)P->B, P->B2, F.w, F.R, nslots, z);
+    auto kern = k_fold_fft1_ms<B1T, 8, 4, 8>;
+    int nsm = 8, smem = fold_ms_smem_bytes<B1T, 8, 4, 8>();
+    if (F.R > 8 && (nslots <= 4 || P->B <= 16384)) {
+      kern = k_fold_fft1_ms<B1T, 4, 1, 16>;
+      nsm = 4;
+      smem = fold_ms_smem_bytes<B1T, 4, 1, 16>();
+    } else if (F.R > 8) {
+      kern = k_fold_fft1_ms<B1T, 8, 2, 16>;
+      smem = fold_ms_smem_bytes<B1T, 8, 2, 16>();
+    }
+    dim3 grid((unsigned)(P->B / 256), (unsigned)((nslots + nsm - 1) / nsm));
+    return launch_k(kern, grid, dim3(256), (size_t)smem, st, P->cur_prio, staging, (const double*)F.d_taps_perm,
+                    P->prm.debug ? u : nullptr, v, (const double2*)P->d_tw, (int)P->B, P->B2, F.w, F.R, nslots, z);
   }
   // spc slots per CTA (their taps loaded once), double-buffered rows while two fit in shared memory
   const int spc = (2 * F.R * 4096 <= 160 * 1024) ? std::min(P->p2_spc, nslots) : 1;
