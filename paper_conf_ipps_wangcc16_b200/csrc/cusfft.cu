@@ -505,10 +505,12 @@ cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem,
   return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
 }
 
-// Batched M-point FFT passes: 512 elements per CTA for M <= 512 (measured best
-// at C3 against 256 and 1024), one sequence per CTA above.
+// Batched M-point FFT passes: 512 elements per CTA for M < 512 except M = 256
+// (measured best at C3 against 256 and 1024), one sequence per CTA above.
+// (M = 256, C4's row FFTs: 1024 elements per CTA, 17.8 vs 21.5 µs at 512 and 21.4 at 2048;
+// profiles/r02_stage_ab.md)
 template <int M>
-constexpr int fft_E() { return M < 512 ? 512 : M; }
+constexpr int fft_E() { return M == 256 ? 1024 : M < 512 ? 512 : M; }
 
 template <int M>
 cudaError_t launch_fft_t(const FftPassArgs& a, cudaStream_t st, int prio) {
