@@ -939,9 +939,13 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       cudaGetLastError();
       const int per = 256 * kStageU;
       int cps = std::min(occ, 4);
-      if (const char* e = std::getenv("CUSFFT_STAGE_CPS")) cps = std::max(1, std::min(occ, std::atoi(e)));  // A/B (measurement)
       int64_t gtot = 0;
       for (int g = 0; g < ng; ++g) gtot = std::max(gtot, P->grp_off[g + 1] - P->grp_off[g]);
+      // sparse sweeps (fewer than 3 gathers per KB of x, e.g. C4's 4-loop groups: 1.5) are faster
+      // with half the requests in flight (2 CTAs per SM: C4 304.5 -> 295.3 us); denser ones (C3: 7,
+      // C5 k = 1000: 25, k = 4096: 50 per KB) with 4 (profiles/r02_stage_ab.md)
+      if ((double)gtot * 1024.0 / ((double)n * 16.0) < 3.0) cps = std::min(cps, 2);
+      if (const char* e = std::getenv("CUSFFT_STAGE_CPS")) cps = std::max(1, std::min(occ, std::atoi(e)));  // A/B (measurement)
       P->stage_grid = (int)std::max<int64_t>(1, std::min<int64_t>((gtot + per - 1) / per, (int64_t)P->sms * cps));
       // Persisting-L2 set-aside for the staging buffer: the staging stores carry evict_last
       // (= persisting) and the x loads evict_first; C3 is 3 us slower without it
