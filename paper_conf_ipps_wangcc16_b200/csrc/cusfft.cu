@@ -703,7 +703,10 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
   P->lay.off_cnt = align256(P->lay.off_bitmap + ((B + 31) / 32) * 4);
   P->lay.off_J = P->lay.off_cnt + 16;
   P->lay.rec_bytes = align256(P->lay.off_J + (int64_t)P->Jcap * 4);
-  if (B <= 2048) {
+  // one FFT pass (and the direct fold) only below 2048 buckets: B = 2048 = 64 x 32 takes the
+  // staged fold with pass 1 inside it (C2: 47.2 -> 37.5 us, C5 k = 50: 49 -> 39 us; its one
+  // 2048-point FFT per loop ran on 16 CTAs)
+  if (B < 2048) {
     P->B1 = 1; P->B2 = (int)B;
   } else {
     const int lb = ilog2(B);

@@ -298,8 +298,9 @@ def test_stage_timing_and_launch_count():
     t = plan.stage_times()
     assert all(v >= 0 for nm, v in t.items() if nm != "gather") and t["fold"] > 0
     assert (t["gather"] > 0) == bool(plan.info()["staged"])
-    # C2 (B = 2048: one FFT pass, direct fold): fold x 2 slot ranges, FFT, cutoff, vote + estimation, output
-    assert plan.info()["tail"] == 1 and plan.launches_per_execute() == 6
+    # C2 (B = 2048 = 64 x 32: staged fold with FFT pass 1 inside): phase 1, phase 2 x 2 slot ranges,
+    # FFT pass 2, cutoff, vote + estimation, output (timing mode: no graph branches)
+    assert plan.info()["tail"] == 1 and plan.launches_per_execute() == 7
 
 
 def test_C4_full_size_parity():
