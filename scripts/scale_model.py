@@ -1,4 +1,4 @@
-"""Per-rank time model of loop-sharded C3 on G = 1, 2, 4, 8 GPUs, with the
+"""Per-rank time model of loop-sharded C3 (or C4: SCALE_CONFIG=C4) on G = 1, 2, 4, 8 GPUs, with the
 per-rank compute MEASURED on one B200, for both loop-sharded
 designs: one all-gather of the per-loop records (shard_mode 0) and two
 all-gathers, candidates then per-loop estimates (shard_mode 2).
@@ -32,9 +32,10 @@ from paper_conf_ipps_wangcc16_b200.dist import slot_of_loop  # noqa: E402
 ALPHA_US = 10.0   # assumed NCCL all-gather latency inside one NVSwitch domain (small messages)
 BW_GBS = 700.0    # assumed achieved all-gather bus bandwidth per GPU (NVLink 5, 900 GB/s per direction)
 
-n, k, L = bench.CONFIGS["C3"][:3]
+CFG = os.environ.get("SCALE_CONFIG", "C3")
+n, k, L = bench.CONFIGS[CFG][:3]
 B = default_B(n, k)
-prm = bench.plan_params("C3", B)
+prm = bench.plan_params(CFG, B)
 x_np, S, X = bench.make_signal(n, k, 1)
 dev = torch.device("cuda", 0)
 x = torch.from_numpy(x_np).to(dev)
@@ -69,7 +70,7 @@ ref_ptr, ref_per = ref.exchange_buffer()
 rec_bytes = ref_per // L
 ref_buf = torch.as_tensor(__import__("paper_conf_ipps_wangcc16_b200.dist", fromlist=["_CudaBuffer"])._CudaBuffer(
     ref_ptr, ref_per), device=dev)
-out = {"config": "C3", "filter": bench.filter_desc("C3"), "single_gpu_us": full_us,
+out = {"config": CFG, "filter": bench.filter_desc(CFG), "single_gpu_us": full_us,
        "allgather_model": {"alpha_us": ALPHA_US, "bw_gbs": BW_GBS,
                            "note": "assumed, not measured (one GPU in this environment)"},
        "ranks": {}}
