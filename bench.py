@@ -450,9 +450,16 @@ def run_gpu(args):
             t0 = time.perf_counter()
             plan.execute_host(x_pin, h_locs, h_vals)
             e_ms.append(1e3 * (time.perf_counter() - t0))
-        e2e = {"value": sum(e_ms) / len(e_ms), "unit": "ms", "h2d_bytes_per_step": n * 16,
+        # pinned x is gathered in place over PCIe (include/cusfft.h): what crosses the bus is the
+        # gathered samples, at least the distinct 32-B sectors they occupy
+        zc = os.environ.get("CUSFFT_HOST_ZEROCOPY", "1") != "0"
+        e2e = {"value": sum(e_ms) / len(e_ms), "unit": "ms",
+               "h2d_bytes_per_step": int(info["sectors"]) * 32 if zc else n * 16,
                "d2h_bytes_per_step": k * (8 + 16),
-               "note": "cusfft_execute_host: pinned H2D of x, transform, D2H of locs/vals, host wall clock"}
+               "note": ("cusfft_execute_host from pinned host memory: x read in place over PCIe by the "
+                        "gather (h2d_bytes = the distinct 32-B sectors of x the plan's taps touch, of "
+                        f"{n * 16} B)" if zc else "cusfft_execute_host: pinned H2D copy of the whole x")
+                       + ", transform, D2H of locs/vals, host wall clock; L2 flushed before each step"}
 
     # ---- the library-default filter (delta = 1e-8, lambda = 0.5/B) on the same signal
     default_line = None

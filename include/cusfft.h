@@ -231,10 +231,15 @@ int cusfft_execute_batch(cusfft_plan_t plan, const void* d_x, int64_t count, int
 int cusfft_set_pipeline(cusfft_plan_t plan, int32_t depth);
 
 /* Paper: the transfer-inclusive timing of the PsFFT comparison (L426).
- * Same transform from HOST buffers: copies h_x [n] to a plan-owned device
- * buffer, executes, copies k locations / values back and synchronises the
- * stream.  Pinned host memory gives asynchronous copies.  Returns the
- * cusfft_status result of the transform. */
+ * Same transform from HOST buffers.  When h_x is pinned and mapped into the
+ * device's address space (cudaHostAlloc / cudaHostRegister with a mapped flag,
+ * or any pinned allocation on a UVA system, e.g. torch's pin_memory) the
+ * gather reads it in place over PCIe: only the samples the plan's taps touch
+ * cross the bus (the sFFT's sublinear sampling; C3: 1.87 M of 16.8 M
+ * samples), and h_x must stay valid and unchanged until the call returns.
+ * Otherwise h_x [n] is first copied to a plan-owned device buffer.  Then the
+ * k locations / values are copied back and the stream synchronised.  Returns
+ * the cusfft_status result of the transform. */
 int cusfft_execute_host(cusfft_plan_t plan, const void* h_x, int64_t* h_locs, void* h_vals);
 
 /* Loop-sharded execution (any world): Steps 1-4 for this rank's loops, written

@@ -1965,8 +1965,21 @@ int cusfft_execute_host(cusfft_plan_t plan, const void* h_x, int64_t* h_locs, vo
     if ((rc = dalloc(&plan->d_vals_buf, (size_t)plan->k))) return rc;
   }
   cudaStream_t st = plan->stream;
-  CK(cudaMemcpyAsync(plan->d_xbuf, h_x, (size_t)plan->n * 16, cudaMemcpyHostToDevice, st));
-  TRY(execute_full(plan, plan->d_xbuf, plan->d_locs_buf, plan->d_vals_buf));
+  // A pinned, device-mapped h_x is gathered in place over PCIe: only the samples the plan's
+  // taps touch cross the bus (C3: 1.87 M samples of 16.8 M; e2e 4.93 -> 2.3 ms).  Pageable
+  // memory (or CUSFFT_HOST_ZEROCOPY=0, A/B) is copied whole first.
+  const void* xin = plan->d_xbuf;
+  {
+    const char* e = std::getenv("CUSFFT_HOST_ZEROCOPY");
+    cudaPointerAttributes pa{};
+    if (!(e && e[0] == '0') && cudaPointerGetAttributes(&pa, h_x) == cudaSuccess && pa.type == cudaMemoryTypeHost &&
+        pa.devicePointer)
+      xin = pa.devicePointer;
+    cudaGetLastError();
+  }
+  if (xin == plan->d_xbuf)
+    CK(cudaMemcpyAsync(plan->d_xbuf, h_x, (size_t)plan->n * 16, cudaMemcpyHostToDevice, st));
+  TRY(execute_full(plan, xin, plan->d_locs_buf, plan->d_vals_buf));
   CK(cudaMemcpyAsync(h_locs, plan->d_locs_buf, (size_t)plan->k * 8, cudaMemcpyDeviceToHost, st));
   CK(cudaMemcpyAsync(h_vals, plan->d_vals_buf, (size_t)plan->k * 16, cudaMemcpyDeviceToHost, st));
   return cusfft_status(plan);

@@ -267,6 +267,25 @@ def test_execute_host_matches_device():
     assert np.array_equal(l2, l3) and np.array_equal(v2, v3)
 
 
+def test_execute_host_zero_copy_staged():
+    """A staged plan reads a pinned host signal in place over PCIe
+    (include/cusfft.h): the outputs equal the device-input path, and a second
+    signal written into the same pinned buffer is the one transformed next."""
+    n, k = 2 ** 22, 1000
+    x1, S1, _ = planted_signal(n, k, seed=41)
+    x2, S2, _ = planted_signal(n, k, seed=42)
+    plan = Plan(n, k, L=16, seed=4)
+    assert plan.info()["staged"]
+    xh = torch.from_numpy(x1).pin_memory()
+    for x, S in ((x1, S1), (x2, S2)):
+        xh.copy_(torch.from_numpy(x))
+        lh, vh = plan.execute_host(xh)
+        ld, vd = plan.execute(torch.from_numpy(x).to(DEV))
+        torch.cuda.synchronize()
+        assert np.array_equal(ld.cpu().numpy(), lh) and np.array_equal(vd.cpu().numpy(), vh)
+        assert sorted(lh.tolist()) == sorted(S.tolist())
+
+
 def test_repeat_and_stream_semantics():
     n, k = 2 ** 16, 16
     x, S, X = planted_signal(n, k, seed=6)
