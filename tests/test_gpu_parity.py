@@ -554,6 +554,45 @@ def test_parity_separate_filters(n, k, extra):
     assert set(locs.tolist()) == set(S.tolist())
 
 
+@pytest.mark.parametrize("env,kw", [({"CUSFFT_STAGE_GROUP": "3"}, {}), ({}, dict(shard_mode=2, max_hits=8192)),
+                                    ({"CUSFFT_STAGE_GROUP": "4"}, dict(shard_mode=2, max_hits=8192))])
+def test_separate_filters_with_groups_and_two_exchanges(env, kw, monkeypatch):
+    """Combinations: separate location / estimation filters (N3) with stage
+    groups (each group one filter) and / or the two-collective finish (world
+    1): the output equals the plain separate-filter plan's bit for bit."""
+    n, k = 2 ** 22, 1000
+    x, S, X = planted_signal(n, k, seed=9)
+    xd = torch.from_numpy(x).to(DEV)
+    filt = dict(loc_tolerance=1e-6, loc_lobefrac=1.0 / 8192, tolerance=1e-7, lobefrac=0.75 / 8192)
+    base = Plan(n, k, L=16, seed=8, **filt)
+    l0, v0 = base.execute(xd)
+    for key, val in env.items():
+        monkeypatch.setenv(key, val)
+    alt = Plan(n, k, L=16, seed=8, **filt, **kw)
+    l1, v1 = alt.execute(xd)
+    torch.cuda.synchronize()
+    assert alt.status() == 0 and alt.info()["filters"] == 2
+    if env:
+        assert alt.info()["staged"] > 1
+    assert torch.equal(l0, l1) and torch.equal(v0, v1)
+    assert sorted(l1.tolist()) == sorted(S.tolist())
+
+
+def test_execute_host_zero_copy_stage_groups(monkeypatch):
+    """The in-place PCIe gather of a pinned host signal through stage groups
+    (several phase-1 launches read the host buffer)."""
+    monkeypatch.setenv("CUSFFT_STAGE_GROUP", "4")
+    n, k = 2 ** 22, 1000
+    x, S, X = planted_signal(n, k, seed=43)
+    plan = Plan(n, k, L=16, seed=4)
+    assert plan.info()["staged"] == 4
+    lh, vh = plan.execute_host(torch.from_numpy(x).pin_memory())
+    ld, vd = plan.execute(torch.from_numpy(x).to(DEV))
+    torch.cuda.synchronize()
+    assert np.array_equal(ld.cpu().numpy(), lh) and np.array_equal(vd.cpu().numpy(), vh)
+    assert sorted(lh.tolist()) == sorted(S.tolist())
+
+
 @pytest.mark.gpu
 @pytest.mark.parametrize("shard_mode", [0, 2])
 def test_library_owned_nccl_exchange_world1(shard_mode):
