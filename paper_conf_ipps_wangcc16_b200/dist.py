@@ -120,10 +120,30 @@ class CudaEngine:
         return self.plan.launches_per_execute()
 
 
+def _host_staged(buf, group) -> bool:
+    """gloo exchanges host tensors: a device buffer goes through host memory
+    (multi-process tests on one GPU; NCCL exchanges device memory directly)."""
+    return buf.is_cuda and dist.get_backend(group) == "gloo"
+
+
 def _all_gather_inplace(buf, rank, world, group):
     per = buf.numel() // world
+    if _host_staged(buf, group):
+        h = buf.cpu()
+        dist.all_gather_into_tensor(h, h[rank * per:(rank + 1) * per].clone(), group=group)
+        buf.copy_(h)
+        return
     # in place: input is this rank's slice of the output (NCCL in-place all-gather)
     dist.all_gather_into_tensor(buf, buf[rank * per:(rank + 1) * per], group=group)
+
+
+def _all_reduce_sum(buf, group):
+    if _host_staged(buf, group):
+        h = buf.cpu()
+        dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
+        buf.copy_(h)
+        return
+    dist.all_reduce(buf, op=dist.ReduceOp.SUM, group=group)
 
 
 class LoopShardedSfft:
@@ -152,7 +172,7 @@ class LoopShardedSfft:
         if self.world > 1:
             buf = self.engine.exchange_tensor()
             if kind == 1:
-                dist.all_reduce(buf, op=dist.ReduceOp.SUM, group=self.group)
+                _all_reduce_sum(buf, self.group)
                 return self.engine.finish()
             _all_gather_inplace(buf, self.rank, self.world, self.group)
         return self.engine.finish()

@@ -514,3 +514,64 @@ def test_batch_sharded_gloo():
         for _, _, _, gl, gv in out:  # every rank holds every result after the (optional) gather
             assert gl[b] == ref.locs.tolist()
             np.testing.assert_array_equal(np.array(gv[b]), ref.vals)
+
+
+# ---------------------------------------------------------------------------
+# The CUDA engine through a real collective: world-size processes on the one
+# test GPU, each with its own cusfft_plan_dist plan, exchanging over gloo
+# (host-staged: no kernel waits on another process).  Every rank's output must
+# equal the single-GPU plan's bit for bit (loop sharding, both kinds) or to
+# fp64 rounding of the reordered sum (signal sharding).
+# ---------------------------------------------------------------------------
+def _cuda_worker(rank, world, port, q, mode):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_ipps_wangcc16_b200.dist import CudaEngine
+        n, k, L = 2 ** 20, 100, 16
+        x, S, X = planted_signal(n, k, seed=8)
+        xd = torch.from_numpy(x).cuda()
+        kw = dict(max_hits=4096) if mode == 2 else {}
+        eng = CudaEngine(n, k, L=L, rank=rank, world=world, seed=5, shard_mode=mode, **kw)
+        if mode == 1:
+            lo, hi = signal_range(rank, n, world)
+            xd = xd[lo:hi].clone()
+        outs = []
+        for _ in range(2):  # capture, then replay
+            locs, vals = LoopShardedSfft(eng).execute(xd)
+            torch.cuda.synchronize()
+            outs.append((locs.cpu().tolist(), torch.view_as_real(vals).cpu().numpy().tolist(), eng.plan.status()))
+        q.put((rank, outs))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("mode,world", [(0, 2), (2, 2), (1, 2), (0, 4), (2, 4)])
+def test_cuda_engine_real_collective_gloo(mode, world):
+    from paper_conf_ipps_wangcc16_b200 import Plan
+    n, k, L = 2 ** 20, 100, 16
+    x, S, X = planted_signal(n, k, seed=8)
+    ref_l, ref_v = Plan(n, k, L=L, seed=5).execute(torch.from_numpy(x).cuda())
+    torch.cuda.synchronize()
+    ref_l, ref_v = ref_l.cpu().numpy(), ref_v.cpu().numpy()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_cuda_worker, args=(r, world, port, q, mode)) for r in range(world)]
+    for pr in procs:
+        pr.start()
+    out = [q.get(timeout=600) for _ in range(world)]
+    for pr in procs:
+        pr.join(timeout=120)
+        assert pr.exitcode == 0
+    for rank, runs in out:
+        for locs, vals, status in runs:
+            assert status == 0
+            v = np.array(vals)[:, 0] + 1j * np.array(vals)[:, 1]
+            assert locs == ref_l.tolist(), (rank, mode)
+            if mode == 1:  # the all-reduce sums partial spectra in another order
+                np.testing.assert_allclose(v, ref_v, rtol=1e-9, atol=1e-12 * np.abs(ref_v).max())
+            else:
+                np.testing.assert_array_equal(v, ref_v)
