@@ -906,11 +906,15 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     // the staging buffer must be (mostly) L2-resident between the two phases, phase 2
     // streams a CTA's R rows (4 KB each) into shared memory, and the schedule word must
     // hold (slot in group, tap); signal-sharded plans gather only their slice (direct path)
-    P->staged = P->fused1 && !P->xshard && q.gather == 0 && (forced || staging_bytes <= (int64_t)64 << 20) && rmax <= 48 &&
+    // (signal-sharded plans stage only their own samples: the other entries stay the zeros the
+    // staging buffer gets at plan time, so their groups must keep their own rows)
+    P->staged = P->fused1 && (!P->xshard || P->grp_abs || ng == 1) && q.gather == 0 &&
+                (forced || staging_bytes <= (int64_t)64 << 20) && rmax <= 48 &&
                 ib + sb <= 32 && total < (int64_t)1 << 31;
     if (P->staged) {
       const uint32_t nm = (uint32_t)(n - 1);
-      std::vector<uint32_t> code((size_t)total);
+      std::vector<uint32_t> code;
+      code.reserve((size_t)total);
       P->grp_off.assign((size_t)ng + 1, 0);
       std::vector<uint64_t> ev;
       for (int g = 0; g < ng; ++g) {
@@ -921,12 +925,13 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
           const uint64_t sg = (uint64_t)(sl - P->grp_s[g]) << ib;
           for (int i = 0; i < w; ++i) {
             const uint32_t pos = (sp.sigma * (uint32_t)i + sp.tau) & nm;
+            if (pos - P->xlo >= P->xspan) continue;  // signal-sharded: another rank's sample
             ev.push_back(((uint64_t)pos << 32) | sg | (uint64_t)i);
           }
         }
         std::sort(ev.begin(), ev.end());
         const int64_t o = P->grp_off[g];
-        for (size_t j = 0; j < ev.size(); ++j) code[(size_t)o + j] = (uint32_t)(ev[j] & 0xFFFFFFFFull);
+        for (size_t j = 0; j < ev.size(); ++j) code.push_back((uint32_t)(ev[j] & 0xFFFFFFFFull));
         P->grp_off[g + 1] = o + (int64_t)ev.size();
       }
       if ((rc = dalloc(&P->d_code, code.size()))) return fail(rc);
@@ -934,6 +939,10 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       if ((rc = dalloc(&P->d_row0, (size_t)P->Lg))) return fail(rc);
       if ((rc = upload(P->d_row0, P->row0_h.data(), (size_t)P->Lg * sizeof(uint32_t)))) return fail(rc);
       if ((rc = dalloc(&P->d_staging, (size_t)(rows_max * B)))) return fail(rc);
+      if (P->xshard && cudaMemset(P->d_staging, 0, (size_t)(rows_max * B) * sizeof(double2)) != cudaSuccess) {
+        g_last_cuda_error = (int)cudaGetLastError();  // (entries of other ranks' samples stay 0)
+        return fail(CUSFFT_CUDA);
+      }
       // one resident wave of phase-1 CTAs (grid-stride loop), at most 4 per SM: with one gather in
       // flight per thread (schedule words prefetched) that is 1024 per SM, measured best
       // (profiles/r02_stage_ab.md; dynamic chunking of the last quarter measured slower)
@@ -947,7 +956,7 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
       // sparse sweeps (fewer than 3 gathers per KB of x, e.g. C4's 4-loop groups: 1.5) are faster
       // with half the requests in flight (2 CTAs per SM: C4 304.5 -> 295.3 us); denser ones (C3: 7,
       // C5 k = 1000: 25, k = 4096: 50 per KB) with 4 (profiles/r02_stage_ab.md)
-      if ((double)gtot * 1024.0 / ((double)n * 16.0) < 3.0) cps = std::min(cps, 2);
+      if ((double)gtot * 1024.0 / ((double)P->xspan * 16.0) < 3.0) cps = std::min(cps, 2);
       if (const char* e = std::getenv("CUSFFT_STAGE_CPS")) cps = std::max(1, std::min(occ, std::atoi(e)));  // A/B (measurement)
       P->stage_grid = (int)std::max<int64_t>(1, std::min<int64_t>((gtot + per - 1) / per, (int64_t)P->sms * cps));
       // Persisting-L2 set-aside for the staging buffer: the staging stores carry evict_last
@@ -1027,7 +1036,8 @@ int launch_stage1(cusfft_plan_t P, const double2* x, cudaStream_t st, int g = 0)
   const int s0 = P->grp_s[(size_t)g], s1 = P->grp_s[(size_t)g + 1];
   const int64_t o = P->grp_off[(size_t)g];
   const ZeroArgs z = g == 0 ? ZeroArgs{P->d_zero, P->nzero} : ZeroArgs{nullptr, 0};
-  StagePackArgs a{x, P->d_code + o, P->d_staging, P->d_slots + (size_t)P->lrank * P->Lg + s0, P->d_row0 + s0,
+  // (signal-sharded: x holds samples [xlo, xlo + xspan); the kernel indexes by the absolute position)
+  StagePackArgs a{x - P->xlo, P->d_code + o, P->d_staging, P->d_slots + (size_t)P->lrank * P->Lg + s0, P->d_row0 + s0,
                   (int)(P->grp_off[(size_t)g + 1] - o), s1 - s0, P->stage_ibits, ilog2(P->B), P->logB2, P->logB1,
                   ilog2(256 / P->B1), (uint32_t)(P->n - 1), z,
                   // staging rows to prefetch into L2: the whole buffer, by the first group (later

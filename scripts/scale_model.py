@@ -1,7 +1,8 @@
 """Per-rank time model of loop-sharded C3 (or C4: SCALE_CONFIG=C4) on G = 1, 2, 4, 8 GPUs, with the
 per-rank compute MEASURED on one B200, for both loop-sharded
 designs: one all-gather of the per-loop records (shard_mode 0) and two
-all-gathers, candidates then per-loop estimates (shard_mode 2).
+all-gathers, candidates then per-loop estimates (shard_mode 2), and signal sharding
+(shard_mode 1: rank 0 folds only x[0, n/G), one all-reduce of the spectra, modelled as a ring).
 
 For each G the script builds rank 0's plan of a G-rank loop-sharded run
 (cusfft_plan_dist without a communicator), and times on the bench's terms
@@ -155,6 +156,34 @@ for G in (1, 2, 4, 8):
     out["mode2"]["ranks"][G] = {"local_us": local_us, "mid_us": lm_us - local_us, "finish_us": lmf_us - lm_us,
                                 "allgather1_bytes": b1, "allgather2_bytes": b2, "allgather_model_us": ag1 + ag2,
                                 "model_total_us": lmf_us + ag1 + ag2, "finish_equals_single_gpu_output": same}
+    p.close()
+# ---- signal sharding (shard_mode 1): rank 0 holds x[0, n/G); its exchange buffer then gets the
+# summed spectra of the world = 1 plan (the all-reduce's result), so finish does the real work
+ref_ptr1, ref_per1 = ref.exchange_buffer()
+ref_rec = torch.as_tensor(_CudaBuffer(ref_ptr1, ref_per1), device=dev).clone()
+out["signal"] = {"ranks": {}}
+for G in (2, 4, 8):
+    p = Plan(n, k, B=B, L=L, seed=3, device=0, rank=0, world=G, shard_mode=1, **prm)
+    ptr, per = p.exchange_buffer()
+    buf = torch.as_tensor(_CudaBuffer(ptr, per), device=dev)
+    xs = x[: n // G].clone()
+    local_us = timed(lambda: p.execute_local(xs))
+    l2 = torch.empty_like(locs)
+    v2 = torch.empty_like(vals)
+
+    def both():
+        p.execute_local(xs)
+        buf.copy_(ref_rec)
+        p.execute_finish(l2, v2)
+    copy_us = timed(lambda: buf.copy_(ref_rec))
+    finish_us = timed(both) - local_us - copy_us
+    both()
+    torch.cuda.synchronize()
+    same = torch.equal(l2, locs)
+    ar_us = ALPHA_US + 2 * (G - 1) / G * per / (BW_GBS * 1e3)
+    out["signal"]["ranks"][G] = {"local_us": local_us, "finish_us": finish_us, "allreduce_bytes": per,
+                                 "allreduce_model_us": ar_us, "model_total_us": local_us + ar_us + finish_us,
+                                 "staged": int(p.info()["staged"]), "finish_locs_equal_single_gpu": same}
     p.close()
 print(json.dumps(out, indent=1))
 with open(sys.argv[1], "w") as f:

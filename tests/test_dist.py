@@ -420,6 +420,8 @@ def test_signal_sharded_plans_emulated_allreduce(world, n, k, L):
     ref_l, ref_v = ref.execute(xd)
     engines = [CudaEngine(n, k, L=L, rank=r, world=world, seed=3, shard_mode=1) for r in range(world)]
     assert all(e.exchange_kind == 1 for e in engines)
+    if n == 2 ** 20:  # B = 2048: each rank stages (only) its own samples
+        assert all(e.plan.info()["staged"] == 1 for e in engines)
     for r, e in enumerate(engines):
         lo, hi = signal_range(r, n, world)
         e.local(xd[lo:hi].clone())  # the rank holds only its slice
