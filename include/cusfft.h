@@ -47,7 +47,7 @@ typedef enum {
   CUSFFT_INVALID_B = -2,      /* B not a power of two, B < 2, or B >= n               */
   CUSFFT_INVALID_K = -3,      /* k < 1, k > 8192, num_select < k or num_select > B    */
   CUSFFT_INVALID_LOOPS = -4,  /* L < 1, L > 64, L_loc > 32, T > L_loc, L_loc > L, or world !| L */
-  CUSFFT_INVALID_PARAM = -5,  /* filter/tolerance/lobefrac/box/taps out of range      */
+  CUSFFT_INVALID_PARAM = -5,  /* filter/tolerance/lobefrac/box/taps out of range (incl. a filter longer than n) */
   CUSFFT_NULL_PTR = -6,       /* a required pointer argument is NULL                  */
   CUSFFT_ALLOC = -7,          /* device allocation failed                             */
   CUSFFT_CUDA = -8,           /* a CUDA runtime call failed (cusfft_last_cuda_error)  */

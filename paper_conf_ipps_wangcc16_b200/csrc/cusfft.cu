@@ -660,7 +660,8 @@ int make_plan(cusfft_plan_t* out, int64_t n, int64_t k, int64_t B, int32_t L, co
     P->nfilt = (!q.taps && P->Lloc < L && (tl != q.tolerance || ll != q.lobefrac)) ? 2 : 1;
     for (int f = 0; f < P->nfilt; ++f) {
       const int64_t w64 = q.taps ? q.num_taps : filter_len(q.filter, P->filt[f].tolerance, P->filt[f].lobefrac);
-      if (w64 < 1 || w64 > (int64_t(1) << 30)) return fail(CUSFFT_INVALID_PARAM);
+      // (a filter longer than the signal would wrap around it: not the paper's flat window, L85)
+      if (w64 < 1 || w64 > (int64_t(1) << 30) || w64 > n) return fail(CUSFFT_INVALID_PARAM);
       P->filt[f].w = (int)w64;
       P->filt[f].R = (int)((w64 + B - 1) / B);
       P->wmax = std::max(P->wmax, (int)w64);

@@ -675,3 +675,42 @@ def test_plans_of_different_shapes_coexist():
     assert torch.equal(ls, ls2) and torch.equal(vs, vs2)
     assert torch.equal(lb, l0) and torch.equal(vb, v0)
     assert sorted(ls.tolist()) == sorted(S2.tolist())
+
+
+def _random_config(i):
+    """A seeded random small configuration (n, k, B, L, extra) covering the
+    parameter space the fixed CASES sample: B single- and two-pass, L_loc, T
+    with and without pair enumeration, both filters, tau modes, noise."""
+    rng = np.random.default_rng(1000 + i)
+    m = int(rng.integers(12, 19))
+    n = 2 ** m
+    k = int(rng.integers(1, 48))
+    L = int(rng.integers(5, 21))
+    Lloc = int(rng.integers(3, min(L, 12) + 1))
+    T = int(rng.integers(Lloc // 2 + 1, Lloc + 1)) if rng.random() < 0.7 else int(rng.integers(2, Lloc // 2 + 2))
+    T = max(1, min(T, Lloc))
+    B = None if rng.random() < 0.5 else 2 ** int(rng.integers(max(5, m - 10), min(m - 5, 14) + 1))
+    if B is not None and B <= 2 * k:
+        B = None
+    extra = dict(loc_loops=Lloc, vote_threshold=T, filter=int(rng.random() < 0.25), tau_mode=int(rng.random() < 0.85))
+    snr = None if rng.random() < 0.7 else float(rng.choice([10.0, 20.0, 40.0]))
+    return n, k, B, L, extra, snr
+
+
+@pytest.mark.parametrize("i", range(48))
+def test_parity_random_configs(i):
+    """Property sweep: 48 seeded random configurations, the GPU against the
+    oracle with shared taps (fold bit-exact, cutoff winners / hits / output
+    locations exact, values to 1e-9)."""
+    n, k, B, L, extra, snr = _random_config(i)
+    x, S, X = planted_signal(n, k, seed=77 + i, snr_db=snr)
+    plan, ref, locs, vals = run_pair(x, n, k, B, L, shared_taps=True, seed=100 + i, **extra)
+    check_all(plan, ref, locs, vals, fold_bit_exact=True)
+
+
+def test_filter_longer_than_signal_rejected():
+    """A filter of more taps than samples (n = 8192, B = 1024: w ~ 12,400 at
+    the default delta / lambda) would wrap around x: CUSFFT_INVALID_PARAM."""
+    with pytest.raises(b.CusfftError) as ei:
+        Plan(2 ** 13, 4, B=1024, L=8, seed=1)
+    assert ei.value.code == b.INVALID_PARAM
