@@ -6,6 +6,8 @@ taps (same per-bucket addition order, no FMA); floating-point values within
 1e-9 relative (north_star).  Near-ties in the cutoff (relative gap < 1e-12
 between the num-th and (num+1)-th |u^|^2) are reported, not failed.
 """
+import os
+
 import numpy as np
 import pytest
 
@@ -714,3 +716,37 @@ def test_filter_longer_than_signal_rejected():
     with pytest.raises(b.CusfftError) as ei:
         Plan(2 ** 13, 4, B=1024, L=8, seed=1)
     assert ei.value.code == b.INVALID_PARAM
+
+
+@pytest.mark.parametrize("i", range(16))
+def test_parity_random_staged_configs(i):
+    """Property sweep of the staged path (n = 2^20 ... 2^22, B >= 2048: address-
+    sorted phase 1, the fused FFT-pass-2 + cutoff cluster kernel where it
+    applies), randomly with the two-collective finish at world 1 and forced
+    stage groups; the GPU against the oracle with shared taps."""
+    rng = np.random.default_rng(5000 + i)
+    n = 2 ** int(rng.integers(20, 23))
+    k = int(rng.integers(20, 600))
+    L = int(rng.integers(8, 17))
+    Lloc = int(rng.integers(4, min(L, 10) + 1))
+    T = int(rng.integers(Lloc // 2 + 1, Lloc + 1))
+    B = int(O.default_B(n, k)) * int(rng.choice([1, 2]))
+    extra = dict(loc_loops=Lloc, vote_threshold=T)
+    if rng.random() < 0.3:
+        extra.update(shard_mode=2, max_hits=16384)
+    x, S, X = planted_signal(n, k, seed=300 + i)
+    env = {}
+    if rng.random() < 0.3:
+        env["CUSFFT_STAGE_GROUP"] = str(int(rng.integers(2, 5)))
+    old = {key: os.environ.get(key) for key in env}
+    os.environ.update(env)
+    try:
+        plan, ref, locs, vals = run_pair(x, n, k, max(B, 2048), L, shared_taps=True, seed=400 + i, **extra)
+    finally:
+        for key, v in old.items():
+            if v is None:
+                os.environ.pop(key, None)
+            else:
+                os.environ[key] = v
+    assert plan.info()["staged"] >= 1
+    check_all(plan, ref, locs, vals, fold_bit_exact=True)
