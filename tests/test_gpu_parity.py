@@ -679,6 +679,38 @@ def test_plans_of_different_shapes_coexist():
     assert sorted(ls.tolist()) == sorted(S2.tolist())
 
 
+def test_concurrent_plans_on_separate_streams():
+    """Distinct plans are independent (include/cusfft.h, Conventions): two
+    staged plans (each holding a
+    persisting-L2 window and its own branch streams) and a small plan enqueued
+    on three streams, interleaved several times without host synchronisation,
+    give the outputs of the same plans run one at a time."""
+    cases = [(2 ** 22, 1000, 51), (2 ** 22, 300, 52), (2 ** 16, 20, 53)]
+    plans, xs, ref = [], [], []
+    for n, k, seed in cases:
+        x, S, _ = planted_signal(n, k, seed=seed)
+        p = Plan(n, k, L=16, seed=seed)
+        xd = torch.from_numpy(x).to(DEV)
+        l0, v0 = p.execute(xd)
+        torch.cuda.synchronize()
+        assert sorted(l0.tolist()) == sorted(S.tolist())
+        plans.append(p)
+        xs.append(xd)
+        ref.append((l0.clone(), v0.clone()))
+    assert plans[0].info()["staged"] and plans[1].info()["staged"]
+    streams = [torch.cuda.Stream() for _ in plans]
+    outs = []
+    for rep in range(4):
+        for p, xd, s in zip(plans, xs, streams):
+            with torch.cuda.stream(s):
+                outs.append(p.execute(xd))
+    torch.cuda.synchronize()
+    for j, (l, v) in enumerate(outs):
+        i = j % len(plans)
+        assert plans[i].status() == 0
+        assert torch.equal(l, ref[i][0]) and torch.equal(v, ref[i][1]), (j, i)
+
+
 def _random_config(i):
     """A seeded random small configuration (n, k, B, L, extra) covering the
     parameter space the fixed CASES sample: B single- and two-pass, L_loc, T
